@@ -1,0 +1,100 @@
+// internal.h — declarations shared by the product's translation units (never by the oracle).
+#pragma once
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+namespace vista {
+
+typedef __nv_bfloat16 bf16;
+
+// ---- error plumbing: every failing CUDA call becomes a VistaError with a message ----
+struct VistaError {
+  int status;
+  std::string msg;
+};
+[[noreturn]] void fail(int status, const std::string& msg);
+#define VCHECK(x)                                                                                     \
+  do {                                                                                                \
+    cudaError_t e_ = (x);                                                                             \
+    if (e_ != cudaSuccess) ::vista::fail(5, std::string(#x) + ": " + cudaGetErrorString(e_));        \
+  } while (0)
+
+// every kernel launch of the library is counted (bench.py reports gpu_launches from it)
+void count_launch();
+#define LAUNCHED()                      \
+  do {                                  \
+    VCHECK(cudaGetLastError());         \
+    ::vista::count_launch();            \
+  } while (0)
+
+// ---- conv / FC layer on the tcgen05 implicit-GEMM kernel ----
+// GEMM view per group g: M = N*Ho*Wo output pixels, N = Cg_out, K = R*S*Cg_in,
+// A[m, k] = x[n, ho*st - pad + r, wo*st - pad + s, g*Cg_in + c] with k = (r*S + s)*Cg_in + c,
+// B[n, k] = w[g*Cg_out + n][k] (padded to Kp, a multiple of 64), D in TMEM (fp32).
+struct ConvLayer {
+  int Cin = 0, Cout = 0, R = 1, S = 1, stride = 1, pad = 0, groups = 1;  // Cin: channels as stored (padded)
+  int Cg_in = 0, Cg_out = 0, K = 0, Kp = 0, BN = 128;
+  bool relu = false;
+  bf16* w = nullptr;         // [Cout][Kp]
+  float* scale = nullptr;    // [Cout]
+  float* shift = nullptr;    // [Cout]
+  CUtensorMap tmap_w;        // box {64, BN}, SWIZZLE_128B
+};
+
+// Builds the padded weight matrix on the device (from OHWI bf16 on the host, Cin_real <= Cin),
+// scale/shift, and the TMA descriptor.
+void conv_layer_init(ConvLayer& L, const std::vector<uint16_t>& w_ohwi_bf16, int Cin_real,
+                     const std::vector<float>& scale, const std::vector<float>& shift);
+void conv_layer_free(ConvLayer& L);
+// y[N,Ho,Wo,Cout] = act(scale * conv(x) + shift (+ res))
+void conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const bf16* res, bf16* y,
+                  cudaStream_t st);
+inline int conv_out_dim(int H, int k, int s, int p) { return (H + 2 * p - k) / s + 1; }
+
+// ---- SIMT kernels (memory-bound) ----
+void launch_ingest(const uint8_t* px, int64_t n, bf16* y, cudaStream_t st);
+void launch_maxpool(const bf16* x, int N, int H, int W, int C, int k, int s, bf16* y, cudaStream_t st);
+void launch_lrn(const bf16* x, int N, int H, int W, int C, bf16* y, cudaStream_t st);
+void launch_avgpool(const bf16* x, int N, int H, int W, int C, bf16* y, cudaStream_t st);
+void launch_tap(const bf16* A, int64_t N, int H, int W, int C, bf16* F, cudaStream_t st);
+
+// ---- join (Eq. 3) + concat (Eq. 4) ----
+struct JoinResult {
+  int64_t n_pairs = 0, n_train = 0;
+  int dup = 0;
+};
+// pair_str / pair_img: device int32 [n_str]; rows [0,n_train) train, then test, each in T_str order.
+JoinResult join_keys(const int64_t* d_img_keys, int64_t n_img, const int64_t* d_str_keys, int64_t n_str,
+                     uint64_t split_subseed, int32_t* d_pair_str, int32_t* d_pair_img, cudaStream_t st);
+void launch_concat(const float* X, int d_s, int ds_pad, const bf16* F, int d_l, const int32_t* pair_str,
+                   const int32_t* pair_img, const uint8_t* labels, int64_t n_pairs, int ld, bf16* MM,
+                   uint8_t* y, cudaStream_t st);
+
+// ---- LR (M) ----
+struct LRWork;  // device scratch for one layer
+struct LRResult {
+  std::vector<double> w;  // [ld] standardised-space weights (pad columns 0)
+  double b = 0;
+  std::vector<double> loss;
+  double lambda_hat = 0, eta = 0;
+  int64_t n_train = 0, n_test = 0, tp = 0, fp = 0, tn = 0, fn = 0, train_ok = 0;
+};
+typedef void (*allreduce_fn)(double* d_buf, int64_t count, cudaStream_t st, void* user);
+LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
+                  const uint8_t* real_col_mask_host, int iters, int power_iters, double lambda, double alpha,
+                  allreduce_fn allreduce, void* ar_user, cudaStream_t st);
+
+// ---- profiling hooks (class ids as in vista.h vista_profile) ----
+struct Profiler;
+extern thread_local Profiler* g_prof;
+void prof_begin(cudaStream_t st);
+void prof_end(cudaStream_t st, int cls, double flops, double bytes);
+
+int num_sms();
+
+}  // namespace vista

@@ -1,0 +1,188 @@
+// simt_ops.cu — the memory-bound TensorOps of the path (S0 ingest, pools, LRN) and the
+// tap g_l (S2).  All NHWC bf16, 8 channels (16 bytes) per thread, vectorised loads/stores,
+// grids sized in multiples of the SM count by a grid-stride loop.
+#include "internal.h"
+#include "ptx.cuh"
+
+namespace vista {
+
+static int grid_for(int64_t work, int threads) {
+  const int64_t blocks = (work + threads - 1) / threads;
+  const int64_t cap = (int64_t)num_sms() * 16;
+  return (int)(blocks < cap ? (blocks > 0 ? blocks : 1) : cap);
+}
+
+__device__ __forceinline__ void ld8(const bf16* p, float (&f)[8]) {
+  const uint4 v = *reinterpret_cast<const uint4*>(p);
+  const uint32_t u[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const float2 a = unpack_bf16x2(u[j]);
+    f[2 * j] = a.x;
+    f[2 * j + 1] = a.y;
+  }
+}
+__device__ __forceinline__ void st8(bf16* p, const float (&f)[8]) {
+  uint4 v;
+  v.x = pack_bf16x2(f[0], f[1]);
+  v.y = pack_bf16x2(f[2], f[3]);
+  v.z = pack_bf16x2(f[4], f[5]);
+  v.w = pack_bf16x2(f[6], f[7]);
+  *reinterpret_cast<uint4*>(p) = v;
+}
+
+// ---- S0: uint8 NHWC3 -> bf16 NHWC8, x = (p - 128) / 128 (reading R10; exact in bf16) ----
+__global__ void ingest_kernel(const uint8_t* __restrict__ px, int64_t npix, bf16* __restrict__ y) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < npix; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint8_t* q = px + i * 3;
+    float f[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+#pragma unroll
+    for (int c = 0; c < 3; ++c) f[c] = ((float)q[c] - 128.0f) * (1.0f / 128.0f);
+    st8(y + i * 8, f);
+  }
+}
+void launch_ingest(const uint8_t* px, int64_t n, bf16* y, cudaStream_t st) {
+  const int64_t npix = n * 227 * 227;
+  prof_begin(st);
+  ingest_kernel<<<grid_for(npix, 256), 256, 0, st>>>(px, npix, y);
+  LAUNCHED();
+  prof_end(st, 2, 0, (double)npix * (3 + 16));
+}
+
+// ---- unpadded max pool (k, s) ----
+__global__ void maxpool_kernel(const bf16* __restrict__ x, int N, int H, int W, int C, int k, int s, int Ho, int Wo,
+                               bf16* __restrict__ y) {
+  const int C8 = C >> 3;
+  const int64_t total = (int64_t)N * Ho * Wo * C8;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int c8 = (int)(i % C8);
+    int64_t pix = i / C8;
+    const int wo = (int)(pix % Wo);
+    pix /= Wo;
+    const int ho = (int)(pix % Ho);
+    const int n = (int)(pix / Ho);
+    float m[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) m[j] = -INFINITY;
+    for (int r = 0; r < k; ++r) {
+      const int hi = ho * s + r;
+      if (hi >= H) break;
+      for (int q = 0; q < k; ++q) {
+        const int wi = wo * s + q;
+        if (wi >= W) break;
+        float f[8];
+        ld8(x + (((size_t)n * H + hi) * W + wi) * C + c8 * 8, f);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) m[j] = fmaxf(m[j], f[j]);
+      }
+    }
+    st8(y + (((size_t)n * Ho + ho) * Wo + wo) * C + c8 * 8, m);
+  }
+}
+void launch_maxpool(const bf16* x, int N, int H, int W, int C, int k, int s, bf16* y, cudaStream_t st) {
+  const int Ho = (H - k) / s + 1, Wo = (W - k) / s + 1;
+  const int64_t total = (int64_t)N * Ho * Wo * (C / 8);
+  prof_begin(st);
+  maxpool_kernel<<<grid_for(total, 256), 256, 0, st>>>(x, N, H, W, C, k, s, Ho, Wo, y);
+  LAUNCHED();
+  prof_end(st, 2, 0, 2.0 * ((double)N * H * W * C + (double)N * Ho * Wo * C));
+}
+
+// ---- AlexNet LRN (reading R3): y_c = x_c / (1 + 2e-5 sum_{|c'-c|<=2} x_c'^2)^0.75 ----
+__global__ void lrn_kernel(const bf16* __restrict__ x, int64_t npix, int C, bf16* __restrict__ y) {
+  const int C8 = C >> 3;
+  const int64_t total = npix * C8;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int c8 = (int)(i % C8);
+    const int64_t pix = i / C8;
+    const bf16* xp = x + pix * C;
+    float w[12];  // channels c8*8-2 .. c8*8+9
+#pragma unroll
+    for (int j = 0; j < 12; ++j) {
+      const int c = c8 * 8 - 2 + j;
+      w[j] = (c >= 0 && c < C) ? __bfloat162float(xp[c]) : 0.0f;
+    }
+    float o[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      float ss = 0.0f;
+#pragma unroll
+      for (int d = 0; d < 5; ++d) ss = fmaf(w[j + d], w[j + d], ss);
+      o[j] = w[j + 2] * exp2f(-0.75f * log2f(fmaf(2e-5f, ss, 1.0f)));
+    }
+    st8(y + pix * C + c8 * 8, o);
+  }
+}
+void launch_lrn(const bf16* x, int N, int H, int W, int C, bf16* y, cudaStream_t st) {
+  const int64_t npix = (int64_t)N * H * W;
+  prof_begin(st);
+  lrn_kernel<<<grid_for(npix * (C / 8), 256), 256, 0, st>>>(x, npix, C, y);
+  LAUNCHED();
+  prof_end(st, 2, 0, 4.0 * (double)npix * C);
+}
+
+// ---- global average pool [N,H,W,C] -> [N,C] ----
+__global__ void avgpool_kernel(const bf16* __restrict__ x, int N, int HW, int C, bf16* __restrict__ y) {
+  const int C8 = C >> 3;
+  const int64_t total = (int64_t)N * C8;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int c8 = (int)(i % C8);
+    const int64_t n = i / C8;
+    float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    for (int p = 0; p < HW; ++p) {
+      float f[8];
+      ld8(x + ((size_t)n * HW + p) * C + c8 * 8, f);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) acc[j] += f[j];
+    }
+    const float inv = 1.0f / (float)HW;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[j] *= inv;
+    st8(y + (size_t)n * C + c8 * 8, acc);
+  }
+}
+void launch_avgpool(const bf16* x, int N, int H, int W, int C, bf16* y, cudaStream_t st) {
+  const int64_t total = (int64_t)N * (C / 8);
+  prof_begin(st);
+  avgpool_kernel<<<grid_for(total, 256), 256, 0, st>>>(x, N, H * W, C, y);
+  LAUNCHED();
+  prof_end(st, 2, 0, 2.0 * ((double)N * H * W * C + (double)N * C));
+}
+
+// ---- S2 tap g_l (PAPER.md:369 fn 4, Def 3.5; reading R7/R8): 2x2 grid max, NHWC flatten ----
+// F[n][(2i + j) C + c] = max_{h in R_i, w in R_j} A[n, h, w, c], R_0 = [0, ceil(H/2)), R_1 = [ceil(H/2), H).
+// Max is exact, so F is bit-identical to a max over the bf16 activation.
+__global__ void tap_kernel(const bf16* __restrict__ A, int64_t N, int H, int W, int C, bf16* __restrict__ F) {
+  const int C8 = C >> 3;
+  const int h2 = (H + 1) >> 1, w2 = (W + 1) >> 1;
+  const int64_t total = N * 4 * C8;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int c8 = (int)(i % C8);
+    const int64_t t = i / C8;
+    const int q = (int)(t & 3);
+    const int64_t n = t >> 2;
+    const int qi = q >> 1, qj = q & 1;
+    const int hb = qi ? h2 : 0, he = qi ? H : h2;
+    const int wb = qj ? w2 : 0, we = qj ? W : w2;
+    float m[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) m[j] = -INFINITY;
+    for (int h = hb; h < he; ++h)
+      for (int w = wb; w < we; ++w) {
+        float f[8];
+        ld8(A + (((size_t)n * H + h) * W + w) * C + c8 * 8, f);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) m[j] = fmaxf(m[j], f[j]);
+      }
+    st8(F + (size_t)n * 4 * C + (size_t)q * C + c8 * 8, m);
+  }
+}
+void launch_tap(const bf16* A, int64_t N, int H, int W, int C, bf16* F, cudaStream_t st) {
+  const int64_t total = N * 4 * (C / 8);
+  prof_begin(st);
+  tap_kernel<<<grid_for(total, 256), 256, 0, st>>>(A, N, H, W, C, F);
+  LAUNCHED();
+  prof_end(st, 1, 0, 2.0 * ((double)N * H * W * C + (double)N * 4 * C));
+}
+
+}  // namespace vista

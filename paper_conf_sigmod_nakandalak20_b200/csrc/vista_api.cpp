@@ -1,0 +1,768 @@
+// vista_api.cpp — the C-ABI (include/vista.h): planner, Staged executor, LR driver,
+// NCCL plumbing and profiling.  Host C++ compiled by nvcc; all arithmetic of the path
+// runs in the kernels of conv_tc.cu / simt_ops.cu / join.cu / lr.cu.
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cmath>
+#include <cstring>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "internal.h"
+#include "roster.h"
+#include "vista.h"
+
+extern "C" {
+#include "vista_gen.h"
+}
+
+#define VISTA_API extern "C" __attribute__((visibility("default")))
+
+namespace vista {
+
+[[noreturn]] void fail(int status, const std::string& msg) { throw VistaError{status, msg}; }
+
+static std::atomic<long long> g_launches{0};
+void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+long long launches_total() { return g_launches.load(); }
+
+int num_sms() {
+  static int n = 0;
+  if (!n) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 148;
+  }
+  return n;
+}
+
+// ---------------- profiler ----------------
+struct Profiler {
+  struct Rec {
+    cudaEvent_t a, b;
+    int cls;
+    double flops, bytes;
+  };
+  std::vector<Rec> recs;
+  std::vector<cudaEvent_t> pool;
+  cudaEvent_t pending = nullptr;
+  vista_profile acc{};
+  cudaEvent_t get() {
+    if (!pool.empty()) {
+      cudaEvent_t e = pool.back();
+      pool.pop_back();
+      return e;
+    }
+    cudaEvent_t e;
+    VCHECK(cudaEventCreate(&e));
+    return e;
+  }
+  void flush() {
+    for (auto& r : recs) {
+      VCHECK(cudaEventSynchronize(r.b));
+      float ms = 0;
+      VCHECK(cudaEventElapsedTime(&ms, r.a, r.b));
+      acc.ms[r.cls] += ms;
+      acc.launches[r.cls] += 1;
+      acc.flops[r.cls] += r.flops;
+      acc.bytes[r.cls] += r.bytes;
+      pool.push_back(r.a);
+      pool.push_back(r.b);
+    }
+    recs.clear();
+  }
+  ~Profiler() {
+    for (auto& r : recs) {
+      cudaEventDestroy(r.a);
+      cudaEventDestroy(r.b);
+    }
+    for (auto e : pool) cudaEventDestroy(e);
+  }
+};
+thread_local Profiler* g_prof = nullptr;
+void prof_begin(cudaStream_t st) {
+  if (!g_prof) return;
+  g_prof->pending = g_prof->get();
+  VCHECK(cudaEventRecord(g_prof->pending, st));
+}
+void prof_end(cudaStream_t st, int cls, double flops, double bytes) {
+  if (!g_prof || !g_prof->pending) return;
+  cudaEvent_t b = g_prof->get();
+  VCHECK(cudaEventRecord(b, st));
+  g_prof->recs.push_back({g_prof->pending, b, cls, flops, bytes});
+  g_prof->pending = nullptr;
+  if (g_prof->recs.size() > 4096) g_prof->flush();
+}
+
+// ---------------- NCCL (dlopen'ed; only when world > 1) ----------------
+struct Nccl {
+  void* h = nullptr;
+  void* comm = nullptr;
+  int (*GetUniqueId)(void*) = nullptr;
+  int (*CommInitRank)(void**, int, char[128], int) = nullptr;  // by-value 128-byte id (see wrapper)
+  int (*AllReduce)(const void*, void*, size_t, int, int, void*, cudaStream_t) = nullptr;
+  int (*CommDestroy)(void*) = nullptr;
+  const char* (*GetErrorString)(int) = nullptr;
+};
+struct NcclId {
+  char internal[128];
+};
+typedef int (*init_rank_fn)(void**, int, NcclId, int);
+
+static Nccl& nccl_lib() {
+  static Nccl n;
+  if (!n.h) {
+    const char* names[] = {"libnccl.so.2", "libnccl.so"};
+    for (const char* nm : names)
+      if ((n.h = dlopen(nm, RTLD_NOW | RTLD_GLOBAL))) break;
+    if (!n.h) fail(6, "cannot dlopen libnccl.so.2 (load torch first or add NCCL to LD_LIBRARY_PATH)");
+    n.GetUniqueId = (int (*)(void*))dlsym(n.h, "ncclGetUniqueId");
+    n.AllReduce = (int (*)(const void*, void*, size_t, int, int, void*, cudaStream_t))dlsym(n.h, "ncclAllReduce");
+    n.CommDestroy = (int (*)(void*))dlsym(n.h, "ncclCommDestroy");
+    n.GetErrorString = (const char* (*)(int))dlsym(n.h, "ncclGetErrorString");
+    if (!n.GetUniqueId || !n.AllReduce || !dlsym(n.h, "ncclCommInitRank")) fail(6, "libnccl missing symbols");
+  }
+  return n;
+}
+
+static void nccl_allreduce_f64(double* buf, int64_t count, cudaStream_t st, void* user) {
+  Nccl& n = nccl_lib();
+  const int rc = n.AllReduce(buf, buf, (size_t)count, /*ncclFloat64*/ 8, /*ncclSum*/ 0, user, st);
+  if (rc != 0) fail(6, std::string("ncclAllReduce: ") + (n.GetErrorString ? n.GetErrorString(rc) : "error"));
+}
+
+// ---------------- helpers ----------------
+static uint16_t f2bf_bits(float f) {  // f is bf16-representable (generator contract)
+  uint32_t u;
+  std::memcpy(&u, &f, 4);
+  return (uint16_t)(u >> 16);
+}
+
+struct DevBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+  void alloc(size_t b) {
+    release();
+    if (b) VCHECK(cudaMalloc(&p, b));
+    bytes = b;
+  }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    bytes = 0;
+  }
+  ~DevBuf() { release(); }
+  DevBuf() = default;
+  DevBuf(const DevBuf&) = delete;
+  DevBuf& operator=(const DevBuf&) = delete;
+};
+
+static bool is_device_ptr(const void* p) {
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
+}  // namespace vista
+
+using namespace vista;
+
+struct vista_ctx {
+  int cnn = 0;
+  NetDesc net;
+  std::vector<ConvLayer> convs;
+  std::vector<int> taps;     // requested tap ids, ascending
+  int t_max = 0;             // last block to run
+  vista_lr_cfg lr{};
+  vista_sys_cfg sys{};
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  int64_t n_img = 0, n_str = 0;
+  int d_s = 0, ds_pad = 0;
+  std::vector<int> micro;    // per block
+  int64_t weight_bytes = 0, peak_pred = 0;
+  // results
+  std::vector<std::unique_ptr<DevBuf>> A, F, MM, Y;  // per block (A, F) / per requested layer (MM, Y)
+  DevBuf pair_str, pair_img, d_X, d_labels, d_img_keys, d_str_keys, d_px;
+  std::vector<DevBuf*> scratch;  // NUM_BUFS slots
+  std::vector<std::unique_ptr<DevBuf>> slot_store;
+  int64_t n_pairs = 0, n_train = 0;
+  bool transferred = false;
+  void* nccl_comm = nullptr;
+  std::unique_ptr<Profiler> prof;
+  bool profiling = false;
+  std::string last_error;
+  ~vista_ctx() {
+    for (auto& L : convs) conv_layer_free(L);
+    if (nccl_comm) {
+      Nccl& n = nccl_lib();
+      if (n.CommDestroy) n.CommDestroy(nccl_comm);
+    }
+    if (own_stream && stream) cudaStreamDestroy(stream);
+  }
+};
+
+static thread_local std::string g_last_error;
+
+namespace {
+
+int layer_index(const vista_ctx* c, int tap) {
+  for (size_t k = 0; k < c->taps.size(); ++k)
+    if (c->taps[k] == tap) return (int)k;
+  return -1;
+}
+int ld_of(const vista_ctx* c, int k) {
+  const int d_l = c->net.stages[c->taps[k]].d_tap;
+  return c->ds_pad + d_l;  // d_l is a multiple of 8 for every roster tap
+}
+
+template <class F>
+vista_status guarded(vista_ctx* c, F&& f) {
+  Profiler* saved = g_prof;
+  try {
+    if (c) g_prof = c->profiling ? c->prof.get() : nullptr;
+    f();
+    g_prof = saved;
+    return VISTA_OK;
+  } catch (const VistaError& e) {
+    g_prof = saved;
+    g_last_error = e.msg;
+    if (c) c->last_error = e.msg;
+    return (vista_status)e.status;
+  } catch (const std::bad_alloc&) {
+    g_prof = saved;
+    g_last_error = "host out of memory";
+    if (c) c->last_error = g_last_error;
+    return VISTA_ERR_OOM;
+  }
+}
+
+// HBM planner (S6): Eq. (6)-style peak = weights + pixels + A_{t-1} + A_t + F's + MM's + scratch(B_t);
+// search micro-batches from the largest down, first feasible wins (Alg. 1 shape).
+void plan_memory(vista_ctx* c, uint64_t budget) {
+  const auto& S = c->net.stages;
+  c->micro.assign(c->t_max + 1, 0);
+  int64_t mm_bytes = 0, f_bytes = 0;
+  for (size_t k = 0; k < c->taps.size(); ++k) {
+    mm_bytes += c->n_str * (int64_t)ld_of(c, (int)k) * 2 + c->n_str;
+    if (!S[c->taps[k]].fc_tap) f_bytes += c->n_img * (int64_t)S[c->taps[k]].d_tap * 2;
+  }
+  const int64_t px = c->n_img * (int64_t)S[0].in_elems;
+  const int64_t join_bytes = c->n_str * 8 + c->n_img * 8 + c->n_str * 4 * 2 + c->n_str * 12 + 32 * 4 * std::max(c->n_img, c->n_str);
+  int64_t peak = 0;
+  for (int t = 0; t <= c->t_max; ++t) {
+    const int64_t a_in = t == 0 ? px : c->n_img * S[t - 1].out_elems * 2;
+    const int64_t a_out = c->n_img * S[t].out_elems * 2;
+    int64_t slot_per_img = 0;
+    for (int b = BUF_T0; b < NUM_BUFS; ++b) slot_per_img += S[t].slot_elems[b] * 2;
+    const int64_t fixed = c->weight_bytes + px + a_in + a_out + mm_bytes + f_bytes + join_bytes + (256ll << 20);
+    int B = 0;
+    if (c->sys.micro_batch > 0 && t == 0) {
+      B = c->sys.micro_batch;
+    } else {
+      const int64_t cap_B = t == 0 ? 256 : 16384;
+      for (int64_t b = std::min<int64_t>(cap_B, std::max<int64_t>(c->n_img, 1)); b >= 1; b = b > 8 ? b / 2 : b - 1) {
+        if ((uint64_t)(fixed + b * slot_per_img) <= budget) {
+          B = (int)b;
+          break;
+        }
+      }
+    }
+    if (B <= 0) fail(VISTA_ERR_NO_PLAN, "no micro-batch fits the HBM budget at stage " + std::to_string(t));
+    c->micro[t] = B;
+    peak = std::max(peak, fixed + (int64_t)B * slot_per_img);
+  }
+  c->peak_pred = peak;
+}
+
+void upload_weights(vista_ctx* c, uint64_t seed) {
+  c->convs.resize(c->net.layers.size());
+  c->weight_bytes = 0;
+  for (size_t i = 0; i < c->net.layers.size(); ++i) {
+    const LayerSpec& s = c->net.layers[i];
+    ConvLayer& L = c->convs[i];
+    L.Cin = s.Cin;
+    L.Cout = s.Cout;
+    L.R = s.R;
+    L.S = s.S;
+    L.stride = s.stride;
+    L.pad = s.pad;
+    L.groups = s.groups;
+    L.relu = s.relu;
+    const int64_t fan_in = (int64_t)s.R * s.S * (s.Cin_real / s.groups);
+    const int64_t nw = (int64_t)s.Cout * fan_in;
+    std::vector<float> wf(nw);
+    // He-normal N(0, 2 / fan_in), RNE bf16 (reading R11) — same generator call as the oracle's
+    vg_param_f32(seed, c->cnn, s.id, VG_T_WEIGHT, nw, 0, 0.0, std::sqrt(2.0 / (double)fan_in), wf.data());
+    std::vector<uint16_t> wb(nw);
+    for (int64_t j = 0; j < nw; ++j) wb[j] = f2bf_bits(wf[j]);
+    std::vector<float> scale(s.Cout, 1.0f), shift(s.Cout, 0.0f);
+    if (s.bias) {
+      vg_param_f32(seed, c->cnn, s.id, VG_T_BIAS, s.Cout, 0, 0.0, 0.01, shift.data());
+    } else if (s.bn_kind) {
+      // BN in inference form folded into the epilogue (reading R12), derived in fp64
+      std::vector<double> g(s.Cout), be(s.Cout), mu(s.Cout), var(s.Cout);
+      if (s.bn_kind == 2)
+        vg_param(seed, c->cnn, s.id, VG_T_BN_GAMMA, s.Cout, 0, 0.2, 0.02, 0, g.data());
+      else
+        vg_param(seed, c->cnn, s.id, VG_T_BN_GAMMA, s.Cout, 0, 1.0, 0.1, 0, g.data());
+      vg_param(seed, c->cnn, s.id, VG_T_BN_BETA, s.Cout, 0, 0.0, 0.05, 0, be.data());
+      vg_param(seed, c->cnn, s.id, VG_T_BN_MEAN, s.Cout, 0, 0.0, 0.05, 0, mu.data());
+      vg_param(seed, c->cnn, s.id, VG_T_BN_VAR, s.Cout, 1, 1.0, 0.2, 0, var.data());
+      for (int o = 0; o < s.Cout; ++o) {
+        const double sc = g[o] / std::sqrt(var[o] + 1e-5);
+        scale[o] = (float)sc;
+        shift[o] = (float)(be[o] - mu[o] * sc);
+      }
+    }
+    conv_layer_init(L, wb, s.Cin_real, scale, shift);
+    c->weight_bytes += (int64_t)L.Cout * L.Kp * 2 + (int64_t)L.Cout * 8;
+  }
+}
+
+const void* to_device(vista_ctx* c, DevBuf& buf, const void* p, size_t bytes) {
+  if (!p || bytes == 0) return p;
+  if (is_device_ptr(p)) return p;
+  buf.alloc(bytes);
+  VCHECK(cudaMemcpyAsync(buf.p, p, bytes, cudaMemcpyHostToDevice, c->stream));
+  return buf.p;
+}
+
+// one block (stage) of the Staged plan over all local images, in micro-batches
+void run_block(vista_ctx* c, int t, const void* in_base) {
+  const StageDesc& S = c->net.stages[t];
+  const int B = c->micro[t];
+  // scratch slots sized for this block
+  void* slot[NUM_BUFS] = {nullptr};
+  for (int b = BUF_T0; b < NUM_BUFS; ++b) {
+    const size_t need = (size_t)S.slot_elems[b] * 2 * B;
+    if (need > c->slot_store[b]->bytes) c->slot_store[b]->alloc(need);
+    slot[b] = c->slot_store[b]->p;
+  }
+  const size_t in_bytes_per = t == 0 ? (size_t)S.in_elems : (size_t)S.in_elems * 2;
+  bf16* out_base = reinterpret_cast<bf16*>(c->A[t]->p);
+  for (int64_t i0 = 0; i0 < c->n_img; i0 += B) {
+    const int nb = (int)std::min<int64_t>(B, c->n_img - i0);
+    slot[BUF_IN] = (void*)((const uint8_t*)in_base + (size_t)i0 * in_bytes_per);
+    slot[BUF_OUT] = out_base + (size_t)i0 * S.out_elems;
+    for (const OpDesc& op : S.ops) {
+      const bf16* in = reinterpret_cast<const bf16*>(slot[op.in]);
+      bf16* out = reinterpret_cast<bf16*>(slot[op.out]);
+      switch (op.kind) {
+        case OP_INGEST:
+          launch_ingest(reinterpret_cast<const uint8_t*>(slot[op.in]), nb, out, c->stream);
+          break;
+        case OP_CONV:
+          conv_forward(c->convs[op.layer], in, nb, op.H, op.W,
+                       op.res >= 0 ? reinterpret_cast<const bf16*>(slot[op.res]) : nullptr, out, c->stream);
+          break;
+        case OP_MAXPOOL:
+          launch_maxpool(in, nb, op.H, op.W, op.C, op.k, op.s, out, c->stream);
+          break;
+        case OP_LRN:
+          launch_lrn(in, nb, op.H, op.W, op.C, out, c->stream);
+          break;
+        case OP_AVGPOOL:
+          launch_avgpool(in, nb, op.H, op.W, op.C, out, c->stream);
+          break;
+      }
+    }
+  }
+}
+
+}  // namespace
+
+// =====================================================================================
+VISTA_API const char* vista_status_str(vista_status s) {
+  switch (s) {
+    case VISTA_OK: return "ok";
+    case VISTA_ERR_INVALID_ARG: return "invalid argument";
+    case VISTA_ERR_NO_PLAN: return "no feasible plan within the HBM budget";
+    case VISTA_ERR_DUP_KEY: return "ID is not a primary key";
+    case VISTA_ERR_STATE: return "call order violated";
+    case VISTA_ERR_CUDA: return "CUDA error";
+    case VISTA_ERR_NCCL: return "NCCL error";
+    case VISTA_ERR_OOM: return "out of memory";
+  }
+  return "unknown";
+}
+
+VISTA_API const char* vista_last_error(const vista_ctx* c) {
+  return c ? c->last_error.c_str() : g_last_error.c_str();
+}
+
+VISTA_API void vista_shard_range(int64_t n, int32_t rank, int32_t world, int64_t* begin, int64_t* end) {
+  if (world <= 0 || rank < 0 || rank >= world) {
+    *begin = *end = 0;
+    return;
+  }
+  *begin = (int64_t)((__int128)n * rank / world);
+  *end = (int64_t)((__int128)n * (rank + 1) / world);
+}
+
+VISTA_API vista_status vista_nccl_unique_id(uint8_t* out128) {
+  return guarded(nullptr, [&] {
+    NcclId id;
+    Nccl& n = nccl_lib();
+    const int rc = n.GetUniqueId(&id);
+    if (rc) fail(6, "ncclGetUniqueId failed");
+    std::memcpy(out128, id.internal, 128);
+  });
+}
+
+VISTA_API vista_status vista_plan(vista_cnn cnn, const int32_t* layers, int32_t n_layers, int32_t n_top,
+                                  int64_t n_str_rows, int32_t n_str_feats, int64_t n_images_local,
+                                  const vista_lr_cfg* model, const vista_sys_cfg* sys, uint64_t weight_seed,
+                                  vista_ctx** out) {
+  if (!out) return VISTA_ERR_INVALID_ARG;
+  *out = nullptr;
+  auto c = std::make_unique<vista_ctx>();
+  vista_status st = guarded(c.get(), [&] {
+    if (cnn < 0 || cnn > 2) fail(1, "unknown cnn");
+    if (n_str_rows < 0 || n_str_feats < 0 || n_images_local < 0) fail(1, "negative size");
+    if (n_images_local > INT32_MAX || n_str_rows > INT32_MAX) fail(1, "more than 2^31 rows per rank");
+    c->cnn = cnn;
+    c->net = build_roster(cnn);
+    const int T = (int)c->net.stages.size();
+    if (layers) {
+      if (n_layers <= 0 || n_layers > 8) fail(1, "n_layers must be in [1, 8]");
+      for (int i = 0; i < n_layers; ++i) {
+        if (layers[i] < 0 || layers[i] >= T) fail(1, "tap id out of range");
+        if (i && layers[i] <= layers[i - 1]) fail(1, "layers must be in ascending depth");
+        c->taps.push_back(layers[i]);
+      }
+    } else {
+      if (n_top <= 0 || n_top > T) fail(1, "n_top out of range");
+      for (int t = T - n_top; t < T; ++t) c->taps.push_back(t);  // "starting from the top most layer"
+    }
+    c->t_max = c->taps.back();
+    if (model) {
+      c->lr = *model;
+    } else {
+      c->lr.iters = 10;
+      c->lr.power_iters = 20;
+      c->lr.lambda = 0.01;
+      c->lr.alpha = 0.5;
+      c->lr.split_seed = 0;
+    }
+    if (c->lr.iters < 0 || c->lr.power_iters < 0) fail(1, "negative iteration count");
+    if (sys) c->sys = *sys;
+    if (c->sys.world <= 0) c->sys.world = 1;
+    if (c->sys.plan != VISTA_PLAN_STAGED) fail(1, "only the Staged plan is implemented (eager/lazy: next round)");
+    if (c->sys.dtype != VISTA_BF16) fail(1, "only bf16 is implemented");
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+      cudaGetLastError();
+      fail(5, "no CUDA device (there is no CPU fallback)");
+    }
+    VCHECK(cudaSetDevice(c->sys.device));
+    cudaDeviceProp prop;
+    VCHECK(cudaGetDeviceProperties(&prop, c->sys.device));
+    if (prop.major != 10) fail(5, "libvista.so is built for sm_100a; device is sm_" + std::to_string(prop.major * 10 + prop.minor));
+    if (c->sys.stream) {
+      c->stream = (cudaStream_t)c->sys.stream;
+    } else {
+      VCHECK(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
+      c->own_stream = true;
+    }
+    c->n_img = n_images_local;
+    c->n_str = n_str_rows;
+    c->d_s = n_str_feats;
+    c->ds_pad = (n_str_feats + 7) / 8 * 8;
+    upload_weights(c.get(), weight_seed);
+    uint64_t budget = c->sys.hbm_budget_bytes;
+    if (!budget) {
+      size_t fr = 0, tot = 0;
+      VCHECK(cudaMemGetInfo(&fr, &tot));
+      budget = fr > (4ull << 30) ? fr - (4ull << 30) : fr / 2;
+      budget += c->weight_bytes;  // weights already allocated
+    }
+    plan_memory(c.get(), budget);
+    c->slot_store.clear();
+    for (int b = 0; b < NUM_BUFS; ++b) c->slot_store.emplace_back(new DevBuf());
+    if (c->sys.world > 1) {
+      if (!c->sys.nccl_uid) fail(1, "world > 1 needs nccl_uid");
+      Nccl& n = nccl_lib();
+      NcclId id;
+      std::memcpy(id.internal, c->sys.nccl_uid, 128);
+      auto init = (init_rank_fn)dlsym(n.h, "ncclCommInitRank");
+      const int rc = init(&c->nccl_comm, c->sys.world, id, c->sys.rank);
+      if (rc) fail(6, "ncclCommInitRank failed");
+    }
+    c->prof.reset(new Profiler());
+    VCHECK(cudaStreamSynchronize(c->stream));
+  });
+  if (st != VISTA_OK) {
+    g_last_error = c->last_error;
+    return st;
+  }
+  *out = c.release();
+  return VISTA_OK;
+}
+
+VISTA_API vista_status vista_plan_info(const vista_ctx* c, vista_plan_info_t* o) {
+  if (!c || !o) return VISTA_ERR_INVALID_ARG;
+  std::memset(o, 0, sizeof(*o));
+  o->n_layers = (int)c->taps.size();
+  for (size_t k = 0; k < c->taps.size(); ++k) {
+    const int t = c->taps[k];
+    o->tap[k] = t;
+    o->d_l[k] = c->net.stages[t].d_tap;
+    o->ld[k] = ld_of(c, (int)k);
+    o->micro_batch[k] = c->micro[t];
+    o->act_bytes[k] = c->n_img * c->net.stages[t].out_elems * 2;
+  }
+  o->peak_bytes_pred = c->peak_pred;
+  o->weight_bytes = c->weight_bytes;
+  o->d_s = c->d_s;
+  o->ds_pad = c->ds_pad;
+  return VISTA_OK;
+}
+
+VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const int64_t* image_keys,
+                                      const float* structured, const int64_t* str_keys, const uint8_t* labels) {
+  if (!c) return VISTA_ERR_INVALID_ARG;
+  return guarded(c, [&] {
+    if (c->n_img > 0 && (!images || !image_keys)) fail(1, "images / image_keys are NULL");
+    if (c->n_str > 0 && (!str_keys || !labels || (c->d_s > 0 && !structured))) fail(1, "structured table is NULL");
+    VCHECK(cudaSetDevice(c->sys.device));
+    c->transferred = false;
+    cudaStream_t st = c->stream;
+    const auto& S = c->net.stages;
+    // ---- inputs (H2D when given host pointers) ----
+    const uint8_t* px = (const uint8_t*)to_device(c, c->d_px, images, (size_t)c->n_img * S[0].in_elems);
+    const int64_t* ik = (const int64_t*)to_device(c, c->d_img_keys, image_keys, (size_t)c->n_img * 8);
+    const int64_t* sk = (const int64_t*)to_device(c, c->d_str_keys, str_keys, (size_t)c->n_str * 8);
+    const float* X = (const float*)to_device(c, c->d_X, structured, (size_t)c->n_str * c->d_s * 4);
+    const uint8_t* lab = (const uint8_t*)to_device(c, c->d_labels, labels, (size_t)c->n_str);
+    // ---- S4 join (Eq. 3), once for all layers ----
+    if (c->pair_str.bytes < (size_t)(c->n_str * 4 + 4)) {
+      c->pair_str.alloc(c->n_str * 4 + 4);
+      c->pair_img.alloc(c->n_str * 4 + 4);
+    }
+    const uint64_t ss = vg_subseed(c->lr.split_seed, VG_S_SPLIT);
+    JoinResult jr = join_keys(ik, c->n_img, sk, c->n_str, ss, (int32_t*)c->pair_str.p, (int32_t*)c->pair_img.p, st);
+    if (jr.dup & 2) fail(1, "a key equals the reserved empty-slot value INT64_MIN");
+    if (jr.dup & 1) fail(VISTA_ERR_DUP_KEY, "duplicate key in T_img or T_str (ID must be a primary key)");
+    c->n_pairs = jr.n_pairs;
+    c->n_train = jr.n_train;
+    // ---- S1-S3 Staged execution ----
+    c->A.clear();
+    c->F.clear();
+    c->MM.clear();
+    c->Y.clear();
+    for (int t = 0; t <= c->t_max; ++t) {
+      c->A.emplace_back(new DevBuf());
+      c->F.emplace_back(new DevBuf());
+    }
+    for (size_t k = 0; k < c->taps.size(); ++k) {
+      c->MM.emplace_back(new DevBuf());
+      c->Y.emplace_back(new DevBuf());
+    }
+    for (int t = 0; t <= c->t_max; ++t) {
+      c->A[t]->alloc((size_t)c->n_img * S[t].out_elems * 2 + 16);
+      const void* in = t == 0 ? (const void*)px : c->A[t - 1]->p;
+      run_block(c, t, in);
+      const int k = layer_index(c, t);
+      if (k >= 0) {
+        const bf16* Fk;
+        if (S[t].fc_tap) {
+          Fk = (const bf16*)c->A[t]->p;  // g = identity on FC layers
+        } else {
+          c->F[t]->alloc((size_t)c->n_img * S[t].d_tap * 2 + 16);
+          launch_tap((const bf16*)c->A[t]->p, c->n_img, S[t].outH, S[t].outW, S[t].outC, (bf16*)c->F[t]->p, st);
+          Fk = (const bf16*)c->F[t]->p;
+        }
+        const int ld = ld_of(c, k);
+        c->MM[k]->alloc((size_t)std::max<int64_t>(c->n_pairs, 1) * ld * 2);
+        c->Y[k]->alloc((size_t)std::max<int64_t>(c->n_pairs, 1));
+        launch_concat(X, c->d_s, c->ds_pad, Fk, S[t].d_tap, (const int32_t*)c->pair_str.p,
+                      (const int32_t*)c->pair_img.p, lab, c->n_pairs, ld, (bf16*)c->MM[k]->p, (uint8_t*)c->Y[k]->p,
+                      st);
+      }
+      // Staged: the input activation of this block is no longer needed (Fig 5E) — unless it is an
+      // FC tap whose activation doubles as its features
+      if (t > 0 && !(S[t - 1].fc_tap && layer_index(c, t - 1) >= 0)) {
+        VCHECK(cudaStreamSynchronize(st));
+        c->A[t - 1]->release();
+      }
+    }
+    VCHECK(cudaStreamSynchronize(st));
+    c->d_px.release();
+    for (auto& s : c->slot_store) s->release();
+    if (g_prof) g_prof->flush();
+    c->transferred = true;
+  });
+}
+
+VISTA_API vista_status vista_features(const vista_ctx* c, int32_t k, vista_buffer* o) {
+  if (!c || !o) return VISTA_ERR_INVALID_ARG;
+  if (!c->transferred) return VISTA_ERR_STATE;
+  if (k < 0 || k >= (int)c->taps.size()) return VISTA_ERR_INVALID_ARG;
+  const int t = c->taps[k];
+  const StageDesc& S = c->net.stages[t];
+  o->mm = c->MM[k]->p;
+  o->rows = c->n_pairs;
+  o->n_train = c->n_train;
+  o->ld = ld_of(c, k);
+  o->d_s = c->d_s;
+  o->ds_pad = c->ds_pad;
+  o->d_l = S.d_tap;
+  o->pair_str = (const int32_t*)c->pair_str.p;
+  o->pair_img = (const int32_t*)c->pair_img.p;
+  o->labels = (const uint8_t*)c->Y[k]->p;
+  o->features = S.fc_tap ? c->A[t]->p : c->F[t]->p;
+  o->activation = c->A[t]->p;
+  return VISTA_OK;
+}
+
+VISTA_API vista_status vista_train(vista_ctx* c, int32_t k, double* weights_out, vista_metrics* m) {
+  if (!c) return VISTA_ERR_INVALID_ARG;
+  if (!c->transferred) {
+    c->last_error = "vista_train before vista_transfer";
+    return VISTA_ERR_STATE;
+  }
+  return guarded(c, [&] {
+    if (k < 0 || k >= (int)c->taps.size()) fail(1, "layer index out of range");
+    VCHECK(cudaSetDevice(c->sys.device));
+    const int t = c->taps[k];
+    const int d_l = c->net.stages[t].d_tap;
+    const int ld = ld_of(c, k);
+    std::vector<uint8_t> real(ld, 0);
+    for (int j = 0; j < c->d_s; ++j) real[j] = 1;
+    for (int j = 0; j < d_l; ++j) real[c->ds_pad + j] = 1;
+    LRResult r = lr_train((const bf16*)c->MM[k]->p, (const uint8_t*)c->Y[k]->p, c->n_pairs, c->n_train, ld,
+                          real.data(), c->lr.iters, c->lr.power_iters, c->lr.lambda, c->lr.alpha,
+                          c->sys.world > 1 ? nccl_allreduce_f64 : nullptr, c->nccl_comm, c->stream);
+    if (g_prof) g_prof->flush();
+    if (weights_out) {
+      for (int j = 0; j < c->d_s; ++j) weights_out[j] = r.w[j];
+      for (int j = 0; j < d_l; ++j) weights_out[c->d_s + j] = r.w[c->ds_pad + j];
+      weights_out[c->d_s + d_l] = r.b;
+    }
+    if (m) {
+      std::memset(m, 0, sizeof(*m));
+      for (int i = 0; i < (int)r.loss.size() && i < 64; ++i) m->loss[i] = r.loss[i];
+      m->lambda_hat = r.lambda_hat;
+      m->eta = r.eta;
+      m->n_train = r.n_train;
+      m->n_test = r.n_test;
+      m->tp = r.tp;
+      m->fp = r.fp;
+      m->tn = r.tn;
+      m->fn = r.fn;
+      m->train_acc = r.n_train ? 100.0 * r.train_ok / r.n_train : 0.0;
+      m->test_acc = r.n_test ? 100.0 * (r.tp + r.tn) / r.n_test : 0.0;
+      const int64_t den = 2 * r.tp + r.fp + r.fn;
+      m->test_f1 = den ? 100.0 * 2.0 * r.tp / den : 0.0;
+    }
+  });
+}
+
+VISTA_API void vista_destroy(vista_ctx* c) {
+  if (!c) return;
+  cudaSetDevice(c->sys.device);
+  if (c->stream) cudaStreamSynchronize(c->stream);
+  delete c;
+}
+
+VISTA_API int64_t vista_kernel_launches(void) { return (int64_t)launches_total(); }
+
+VISTA_API vista_status vista_set_profiling(vista_ctx* c, int32_t on) {
+  if (!c) return VISTA_ERR_INVALID_ARG;
+  c->profiling = on != 0;
+  return VISTA_OK;
+}
+
+VISTA_API vista_status vista_get_profile(vista_ctx* c, vista_profile* out, int32_t reset) {
+  if (!c || !out) return VISTA_ERR_INVALID_ARG;
+  return guarded(c, [&] {
+    c->prof->flush();
+    *out = c->prof->acc;
+    if (reset) c->prof->acc = vista_profile{};
+  });
+}
+
+// ---------------- kernel-level entry points ----------------
+static cudaStream_t as_stream(void* s) { return (cudaStream_t)s; }
+
+VISTA_API vista_status vista_conv2d(const void* x, int32_t N, int32_t H, int32_t W, int32_t C, const void* w,
+                                    int32_t Cout, int32_t R, int32_t S, int32_t stride, int32_t pad, int32_t groups,
+                                    const float* scale, const float* shift, const void* residual, int32_t relu,
+                                    void* y, void* stream) {
+  return guarded(nullptr, [&] {
+    if (!x || !w || !scale || !shift || !y || N < 0 || C % 8 || groups < 1) fail(1, "vista_conv2d: bad arguments");
+    ConvLayer L;
+    L.Cin = C;
+    L.Cout = Cout;
+    L.R = R;
+    L.S = S;
+    L.stride = stride;
+    L.pad = pad;
+    L.groups = groups;
+    L.relu = relu != 0;
+    const size_t nw = (size_t)Cout * R * S * (C / groups);
+    std::vector<uint16_t> hw(nw);
+    std::vector<float> hs(Cout), hh(Cout);
+    VCHECK(cudaMemcpy(hw.data(), w, nw * 2, cudaMemcpyDeviceToHost));
+    VCHECK(cudaMemcpy(hs.data(), scale, Cout * 4, cudaMemcpyDeviceToHost));
+    VCHECK(cudaMemcpy(hh.data(), shift, Cout * 4, cudaMemcpyDeviceToHost));
+    try {
+      conv_layer_init(L, hw, C, hs, hh);
+      conv_forward(L, (const bf16*)x, N, H, W, (const bf16*)residual, (bf16*)y, as_stream(stream));
+      VCHECK(cudaStreamSynchronize(as_stream(stream)));
+    } catch (...) {
+      conv_layer_free(L);
+      throw;
+    }
+    conv_layer_free(L);
+  });
+}
+
+VISTA_API vista_status vista_tap(const void* A, int32_t N, int32_t H, int32_t W, int32_t C, void* F, void* stream) {
+  return guarded(nullptr, [&] {
+    if (!A || !F || C % 8) fail(1, "vista_tap: bad arguments");
+    launch_tap((const bf16*)A, N, H, W, C, (bf16*)F, as_stream(stream));
+    VCHECK(cudaStreamSynchronize(as_stream(stream)));
+  });
+}
+
+VISTA_API vista_status vista_maxpool(const void* x, int32_t N, int32_t H, int32_t W, int32_t C, int32_t k, int32_t s,
+                                     void* y, void* stream) {
+  return guarded(nullptr, [&] {
+    if (!x || !y || C % 8 || k < 1 || s < 1 || H < k || W < k) fail(1, "vista_maxpool: bad arguments");
+    launch_maxpool((const bf16*)x, N, H, W, C, k, s, (bf16*)y, as_stream(stream));
+    VCHECK(cudaStreamSynchronize(as_stream(stream)));
+  });
+}
+
+VISTA_API vista_status vista_lrn(const void* x, int32_t N, int32_t H, int32_t W, int32_t C, void* y, void* stream) {
+  return guarded(nullptr, [&] {
+    if (!x || !y || C % 8) fail(1, "vista_lrn: bad arguments");
+    launch_lrn((const bf16*)x, N, H, W, C, (bf16*)y, as_stream(stream));
+    VCHECK(cudaStreamSynchronize(as_stream(stream)));
+  });
+}
+
+VISTA_API vista_status vista_avgpool(const void* x, int32_t N, int32_t H, int32_t W, int32_t C, void* y,
+                                     void* stream) {
+  return guarded(nullptr, [&] {
+    if (!x || !y || C % 8) fail(1, "vista_avgpool: bad arguments");
+    launch_avgpool((const bf16*)x, N, H, W, C, (bf16*)y, as_stream(stream));
+    VCHECK(cudaStreamSynchronize(as_stream(stream)));
+  });
+}
+
+VISTA_API vista_status vista_ingest(const uint8_t* px, int32_t N, void* y, void* stream) {
+  return guarded(nullptr, [&] {
+    if (!px || !y) fail(1, "vista_ingest: bad arguments");
+    launch_ingest(px, N, (bf16*)y, as_stream(stream));
+    VCHECK(cudaStreamSynchronize(as_stream(stream)));
+  });
+}

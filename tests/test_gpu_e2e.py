@@ -1,0 +1,174 @@
+"""End-to-end GPU parity through vista_plan / vista_transfer / vista_train against the
+fp64 oracle on the same generated inputs (DESIGN.md §"Tolerances").
+
+- features F_l: normwise per (image, layer) max|gpu - ref| / max|ref| <= 2e-2 (bf16, fp32 acc.)
+- join pairs, labels, structured columns of MM: bit-exact
+- LR weights: ||w_gpu - w_ref|| / ||w_ref|| <= 1e-3 with the oracle LR run on the GPU's own MM
+- accuracy end to end (oracle features + oracle LR vs GPU): within 0.5 points
+"""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from paper_conf_sigmod_nakandalak20_b200 import Vista, VistaError
+
+pytestmark = pytest.mark.gpu
+WSEED = 11
+SPLIT = 5
+
+
+def run_gpu(cnn, taps, tab, d_s, iters=5, **kw):
+    v = Vista(cnn, layers=taps, n_str_rows=len(tab.str_keys), d_s=d_s, n_images_local=len(tab.img_keys),
+              iters=iters, split_seed=SPLIT, weight_seed=WSEED, **kw)
+    v.transfer(tab.images, tab.img_keys, tab.X, tab.str_keys, tab.labels)
+    return v
+
+
+def normwise_rows(gpu, ref):
+    den = np.maximum(np.abs(ref).max(axis=1), 1e-30)
+    return np.abs(gpu - ref).max(axis=1) / den
+
+
+def oracle_pairs(tab):
+    ps, pi, te = oracle.join(tab.img_keys, tab.str_keys, SPLIT)
+    order = np.concatenate([np.nonzero(te == 0)[0], np.nonzero(te == 1)[0]])  # [train | test], stable
+    return ps[order], pi[order], int((te == 0).sum())
+
+
+def check_layer(v, k, tab, F_ref, d_s, iters):
+    f = v.features(k)
+    ps, pi, n_train = oracle_pairs(tab)
+    # join: bit-exact
+    assert f["rows"] == len(ps) and f["n_train"] == n_train
+    np.testing.assert_array_equal(f["pair_str"].cpu().numpy(), ps)
+    np.testing.assert_array_equal(f["pair_img"].cpu().numpy(), pi)
+    np.testing.assert_array_equal(f["labels"].cpu().numpy(), tab.labels[ps])
+    # features: normwise per image
+    Fg = f["features"].to(torch.float64).cpu().numpy()
+    err = normwise_rows(Fg, F_ref)
+    assert err.max() <= 2e-2, err.max()
+    # concat: structured part exact, image part = features exactly, padding zero
+    MM = f["mm"].to(torch.float64).cpu().numpy()
+    np.testing.assert_array_equal(MM[:, :d_s], tab.X[ps].astype(np.float64))
+    assert not MM[:, d_s:f["ds_pad"]].any()
+    np.testing.assert_array_equal(MM[:, f["ds_pad"]:f["ds_pad"] + f["d_l"]], Fg[pi])
+    assert not MM[:, f["ds_pad"] + f["d_l"]:].any()
+    # LR on identical inputs (the GPU's MM upcast to fp64)
+    cols = list(range(d_s)) + list(range(f["ds_pad"], f["ds_pad"] + f["d_l"]))
+    X = MM[:, cols]
+    te = np.zeros(len(ps), np.uint8)
+    te[n_train:] = 1
+    y = tab.labels[ps]
+    ref = oracle.lr_train(X, y, te, iters=iters)
+    w, b, met = v.train(k, d_s + f["d_l"])
+    wr = np.append(ref["w"], ref["b"])
+    wg = np.append(w, b)
+    assert np.linalg.norm(wg - wr) <= 1e-3 * max(np.linalg.norm(wr), 1e-12)
+    np.testing.assert_allclose(met["loss"][:iters], ref["loss"], rtol=1e-4, atol=1e-6)
+    assert met["lambda_hat"] == pytest.approx(ref["lambda_hat"], rel=1e-4)
+    assert met["n_train"] == ref["n_train"] and met["n_test"] == ref["n_test"]
+    # end to end: oracle features -> oracle LR
+    MMo = oracle.concat(tab.X, F_ref, ps, pi)
+    ref_e2e = oracle.lr_train(MMo, y, te, iters=iters)
+    return met, ref, ref_e2e
+
+
+@pytest.fixture(scope="module")
+def c1():
+    # BASELINE.json configs[0]: AlexNet {conv5, fc6, fc7}, 16 images, 8 structured features, LR T = 5
+    tab = gen.make_tables(16, 8, kind=gen.FOODS)
+    F, _ = oracle.features(oracle.ALEXNET, WSEED, tab.images, taps=[0, 1, 2])
+    return tab, F
+
+
+def test_config1_alexnet_end_to_end(c1):
+    tab, F = c1
+    v = run_gpu(0, [0, 1, 2], tab, 8, iters=5)
+    for k, t in enumerate([0, 1, 2]):
+        met, ref, e2e = check_layer(v, k, tab, F[t], 8, 5)
+        assert abs(met["test_acc"] - ref["test_acc"]) <= 0.5 + 1e-9  # same inputs
+        assert abs(met["test_acc"] - e2e["test_acc"]) <= max(0.5, 100.0 / max(met["n_test"], 1)) + 1e-9
+    v.close()
+
+
+def test_alexnet_mismatch_join_and_accuracy():
+    # C1b-like: inner-join semantics with unmatched rows on both sides, ~20 % test rows
+    tab = gen.make_tables(300, 8, mismatch=True)
+    F, _ = oracle.features(oracle.ALEXNET, WSEED, tab.images, taps=[1])
+    v = run_gpu(0, [1], tab, 8, iters=10)
+    met, ref, e2e = check_layer(v, 0, tab, F[1], 8, 10)
+    assert abs(met["test_acc"] - ref["test_acc"]) <= 0.5 + 1e-9  # same inputs
+    # end to end: at most one test row may flip at this sample size (0.5 points at >= 200 test rows)
+    assert abs(met["test_acc"] - e2e["test_acc"]) <= max(0.5, 100.0 / met["n_test"]) + 1e-9
+    v.close()
+
+
+def test_resnet50_top5_small():
+    tab = gen.make_tables(6, 130, kind=gen.FOODS)
+    F, _ = oracle.features(oracle.RESNET50, WSEED, tab.images, taps=[0, 1, 2, 3, 4])
+    v = Vista(2, n_top=5, n_str_rows=len(tab.str_keys), d_s=130, n_images_local=6, iters=3, split_seed=SPLIT,
+              weight_seed=WSEED)
+    v.transfer(tab.images, tab.img_keys, tab.X, tab.str_keys, tab.labels)
+    for k in range(5):
+        Fg = v.features(k)["features"].to(torch.float64).cpu().numpy()
+        err = normwise_rows(Fg, F[k])
+        assert err.max() <= 2e-2, (k, err.max())
+    v.close()
+
+
+def test_vgg16_fc_layers_small():
+    tab = gen.make_tables(3, 201, kind=gen.AMAZON)
+    F, _ = oracle.features(oracle.VGG16, WSEED, tab.images, taps=[0, 1, 2])
+    v = run_gpu(1, [0, 1, 2], tab, 201, iters=2)
+    for k in range(3):
+        Fg = v.features(k)["features"].to(torch.float64).cpu().numpy()
+        assert normwise_rows(Fg, F[k]).max() <= 2e-2
+    v.close()
+
+
+def test_staged_micro_batch_invariance():
+    # the planner's micro-batch must not change any bit of the result (deterministic kernels)
+    tab = gen.make_tables(20, 8)
+    outs = []
+    for mb in (20, 7, 3):
+        v = run_gpu(0, [0, 2], tab, 8, iters=2, micro_batch=mb)
+        outs.append([v.features(k)["mm"].view(torch.int16).cpu().clone() for k in range(2)])
+        v.close()
+    for o in outs[1:]:
+        for a, b in zip(outs[0], o):
+            assert torch.equal(a, b)
+
+
+def test_device_and_host_inputs_agree():
+    tab = gen.make_tables(8, 8)
+    v1 = run_gpu(0, [0], tab, 8, iters=2)
+    m1 = v1.features(0)["mm"].view(torch.int16).cpu().clone()
+    v1.close()
+    v2 = Vista(0, layers=[0], n_str_rows=len(tab.str_keys), d_s=8, n_images_local=8, iters=2, split_seed=SPLIT,
+               weight_seed=WSEED)
+    d = lambda a: torch.from_numpy(a).cuda()
+    v2.transfer(d(tab.images), d(tab.img_keys), d(tab.X), d(tab.str_keys), d(tab.labels))
+    assert torch.equal(m1, v2.features(0)["mm"].view(torch.int16).cpu())
+    v2.close()
+
+
+def test_duplicate_key_error():
+    tab = gen.make_tables(8, 8)
+    keys = tab.img_keys.copy()
+    keys[3] = keys[5]
+    v = Vista(0, layers=[0], n_str_rows=len(tab.str_keys), d_s=8, n_images_local=8, iters=2, weight_seed=WSEED)
+    with pytest.raises(VistaError) as e:
+        v.transfer(tab.images, keys, tab.X, tab.str_keys, tab.labels)
+    assert e.value.status == 3
+    with pytest.raises(VistaError) as e:
+        v.train(0, 8 + 1024)
+    assert e.value.status == 4
+    v.close()
+
+
+def test_no_plan_within_tiny_budget():
+    with pytest.raises(VistaError) as e:
+        Vista(2, n_top=5, n_str_rows=1000, d_s=130, n_images_local=1000, hbm_budget_bytes=64 << 20)
+    assert e.value.status == 2

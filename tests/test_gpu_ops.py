@@ -1,0 +1,106 @@
+"""GPU parity of single kernels (through the C-ABI kernel-level entry points) against
+the fp64 oracle on identical bf16-valued inputs.
+
+Tolerance (DESIGN.md §"Tolerances"): a conv/FC output is fp32-accumulated and rounded
+once to bf16 (RNE, relative 2^-9); normwise max|gpu - ref| / max|ref| <= 8e-3 leaves
+margin for fp32 summation order.  Max-based ops (tap, max pool) are bit-exact.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from paper_conf_sigmod_nakandalak20_b200 import (vista_avgpool, vista_conv2d, vista_ingest, vista_lrn,
+                                                 vista_maxpool, vista_tap)
+
+pytestmark = pytest.mark.gpu
+rng = np.random.default_rng(2020)
+
+
+def bf(a):
+    """numpy float -> (bf16 cuda tensor, the same values as fp64 numpy)."""
+    t = torch.from_numpy(np.ascontiguousarray(a, dtype=np.float32)).to(torch.bfloat16)
+    return t.cuda(), t.to(torch.float64).numpy()
+
+
+def normwise(gpu, ref):
+    return float(np.abs(gpu - ref).max() / max(np.abs(ref).max(), 1e-30))
+
+
+CONV = [
+    # N, H, W, C, Cout, k, stride, pad, groups, residual, relu     (what it covers)
+    (2, 14, 14, 64, 256, 1, 1, 0, 1, True, True),      # 1x1 s1 (fast path), BN=256, residual
+    (2, 14, 14, 256, 128, 1, 2, 0, 1, False, True),    # 1x1 s2 projection-style, BN=128
+    (2, 9, 11, 64, 64, 3, 1, 1, 1, False, True),       # 3x3 p1, BN=64, M tail (198 rows)
+    (1, 23, 23, 8, 64, 7, 2, 3, 1, False, True),       # conv1-style 7x7 s2, C=8 (general gather)
+    (1, 31, 31, 8, 96, 11, 4, 0, 1, False, True),      # AlexNet conv1 geometry, Cout 96 (masked N tile)
+    (1, 9, 9, 96, 256, 5, 1, 2, 2, False, True),       # grouped 5x5, Cg_in = 48 (general gather)
+    (1, 7, 7, 384, 384, 3, 1, 1, 2, False, True),      # grouped 3x3, Cg_out = 192
+    (3, 1, 1, 1152, 1000, 1, 1, 0, 1, False, False),   # FC, N = 1000 (partial last N tile), M = 3
+    (2, 7, 7, 128, 512, 3, 2, 1, 1, True, False),      # strided 3x3, residual without ReLU
+    (130, 1, 1, 64, 128, 1, 1, 0, 1, False, True),     # FC with M = 130 (two M tiles)
+]
+
+
+@pytest.mark.parametrize("N,H,W,C,Cout,k,stride,pad,groups,residual,relu", CONV)
+def test_conv_tcgen05_vs_oracle(N, H, W, C, Cout, k, stride, pad, groups, residual, relu):
+    x, x64 = bf(rng.standard_normal((N, H, W, C)))
+    w, w64 = bf(rng.standard_normal((Cout, k, k, C // groups)) * (2.0 / (k * k * C / groups)) ** 0.5)
+    scale = rng.uniform(0.5, 1.5, Cout).astype(np.float32)
+    shift = rng.standard_normal(Cout).astype(np.float32) * 0.1
+    ref = oracle.conv2d(x64, w64, stride, pad, groups) * scale.astype(np.float64) + shift.astype(np.float64)
+    res = None
+    if residual:
+        res, res64 = bf(rng.standard_normal(ref.shape))
+        ref = ref + res64
+    if relu:
+        ref = np.maximum(ref, 0)
+    y = vista_conv2d(x, w, torch.from_numpy(scale).cuda(), torch.from_numpy(shift).cuda(), stride, pad, groups,
+                     residual=res, relu=relu)
+    torch.cuda.synchronize()
+    got = y.to(torch.float64).cpu().numpy()
+    assert got.shape == ref.shape
+    assert normwise(got, ref) <= 8e-3
+
+
+def test_conv_deterministic():
+    x, _ = bf(rng.standard_normal((2, 14, 14, 64)))
+    w, _ = bf(rng.standard_normal((128, 3, 3, 64)) * 0.05)
+    s = torch.ones(128, device="cuda")
+    b = torch.zeros(128, device="cuda")
+    y1 = vista_conv2d(x, w, s, b, 1, 1)
+    y2 = vista_conv2d(x, w, s, b, 1, 1)
+    assert torch.equal(y1.view(torch.int16), y2.view(torch.int16))
+
+
+@pytest.mark.parametrize("H,C", [(14, 1024), (7, 2048), (13, 256), (2, 8), (3, 16)])
+def test_tap_bit_exact(H, C):
+    A, A64 = bf(rng.standard_normal((3, H, H, C)))
+    F = vista_tap(A).to(torch.float64).cpu().numpy()
+    np.testing.assert_array_equal(F, oracle.tap(A64))
+
+
+@pytest.mark.parametrize("H,k,s,C", [(114, 3, 2, 64), (55, 3, 2, 96), (13, 3, 2, 256), (224, 2, 2, 64), (7, 2, 2, 8)])
+def test_maxpool_bit_exact(H, k, s, C):
+    x, x64 = bf(rng.standard_normal((2, H, H, C)))
+    np.testing.assert_array_equal(vista_maxpool(x, k, s).to(torch.float64).cpu().numpy(), oracle.maxpool(x64, k, s))
+
+
+def test_avgpool():
+    x, x64 = bf(rng.standard_normal((3, 7, 7, 2048)))
+    got = vista_avgpool(x).to(torch.float64).cpu().numpy()
+    assert normwise(got, oracle.avgpool_global(x64)) <= 4e-3
+
+
+def test_lrn():
+    x, x64 = bf(rng.standard_normal((2, 5, 5, 96)) * 20)
+    got = vista_lrn(x).to(torch.float64).cpu().numpy()
+    ref = oracle.lrn(x64)
+    assert np.abs(got - ref).max() <= 4e-3 * np.abs(ref).max()
+
+
+def test_ingest_exact():
+    px = rng.integers(0, 256, (2, 227, 227, 3), dtype=np.uint8)
+    y = vista_ingest(torch.from_numpy(px).cuda()).to(torch.float64).cpu().numpy()
+    np.testing.assert_array_equal(y[..., :3], (px.astype(np.float64) - 128) / 128)
+    assert not y[..., 3:].any()

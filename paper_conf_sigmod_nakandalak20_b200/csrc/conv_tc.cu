@@ -7,11 +7,16 @@
 // PAPER.md:138-141) is a chain of these TensorOps.  GEMM view per group g:
 //   D[m, n] = sum_k A[m, k] * B[n, k],  m = output pixel (n_img, ho, wo),
 //   n = output channel, k = (r*S + s)*Cg_in + c.
-// Tile 128 x BN x 64; A (the implicit im2col of the NHWC activation) is gathered by
-// 128 producer threads with 16-byte cp.async into the 128B-swizzled K-major layout,
-// B (weights [Cout][Kp]) arrives by TMA with the same swizzle; one elected thread
-// issues tcgen05.mma into TMEM; the 4 producer warps then drain TMEM (tcgen05.ld)
-// through the epilogue.  mbarriers pipeline STAGES k-blocks.
+//
+// Persistent, warp-specialised kernel, one CTA per SM, 128 x BN x 64 tiles:
+//   warps 0-3  A producers: either one elected thread issuing TMA for a plain [M, C]
+//              activation (1x1 stride-1 convs, FC layers), or 128 threads gathering the
+//              implicit im2col rows with 16-byte cp.async (zero-fill = padding) into the
+//              128B-swizzled K-major layout.  Thread 0 also issues the weight (B) TMA.
+//   warp 4     TMEM allocator + single-thread tcgen05.mma issuer.
+//   warps 5-8  epilogue: tcgen05.ld -> scale/shift (smem) + residual + ReLU -> bf16.
+// TMEM holds two accumulators (2 x BN columns) so the epilogue of tile i overlaps the
+// mainloop of tile i+1; an mbarrier ring of STAGES k-blocks feeds the tensor core.
 #include <cudaTypedefs.h>
 
 #include <cstring>
@@ -22,6 +27,8 @@
 
 namespace vista {
 
+enum AMode { A_GATHER_FAST = 0, A_GATHER_GENERAL = 1, A_TMA = 2 };
+
 struct ConvParams {
   const bf16* x;
   bf16* y;
@@ -29,198 +36,282 @@ struct ConvParams {
   const float* scale;
   const float* shift;
   int H, W, Cin, Ho, Wo, Cout, R, S, stride, pad, Cg_in, Cg_out, K, nkb, M, relu;
+  int n_mt, n_nt, n_tiles;
 };
 
 constexpr int BM = 128, BK = 64;
-constexpr int kProducerThreads = 128;
-constexpr int kThreads = kProducerThreads + 32;  // + 1 MMA warp
-constexpr int kLag = 2;                           // cp.async groups in flight before arriving
+constexpr int kThreads = 288;  // 4 producer warps + 1 MMA warp + 4 epilogue warps
+constexpr int kEpiWarp0 = 5;
+constexpr int kLag = 2;        // cp.async groups in flight before a stage is published
 
-template <int BN, int STAGES>
-struct ConvSmem {
+template <int BN>
+struct Cfg {
+  static constexpr int kStages = BN == 256 ? 4 : (BN == 128 ? 6 : 8);
   static constexpr int kABytes = BM * BK * 2;  // 16 KB
   static constexpr int kBBytes = BN * BK * 2;
-  static constexpr int kBarOff = STAGES * (kABytes + kBBytes);
-  static constexpr int kBytes = kBarOff + (2 * STAGES + 1) * 8 + 16 + 1024;  // + alignment slack
+  static constexpr int kSbufOff = kStages * (kABytes + kBBytes);
+  static constexpr int kBarOff = kSbufOff + 2 * 2 * BN * 4;
+  static constexpr int kBytes = kBarOff + (2 * kStages + 4) * 8 + 16 + 1024;  // + alignment slack
+  static constexpr int kTmemCols = 2 * BN;
 };
 
-template <int BN, int STAGES, bool kFast>
+// tile -> (first row m0, N-tile index nt, group g); N-tiles of one M-tile are adjacent so
+// the 148 CTAs working at any moment share A rows in L2
+__device__ __forceinline__ void decode_tile(const ConvParams& p, int tile, int& m0, int& nt, int& g) {
+  const int per_g = p.n_mt * p.n_nt;
+  g = tile / per_g;
+  const int rem = tile - g * per_g;
+  const int mt = rem / p.n_nt;
+  m0 = mt * BM;
+  nt = rem - mt * p.n_nt;
+}
+
+template <int BN, int AMODE>
 __global__ void __launch_bounds__(kThreads, 1)
-    conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const ConvParams p) {
-  using L = ConvSmem<BN, STAGES>;
+    conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__ CUtensorMap tmap_a,
+                   const ConvParams p) {
+  using C = Cfg<BN>;
+  constexpr int S = C::kStages;
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 1023u) & ~1023u;
   uint8_t* gbase = smem_raw + (base - raw);
-  const uint32_t sA = base, sB = base + STAGES * L::kABytes;
-  uint64_t* full = reinterpret_cast<uint64_t*>(gbase + L::kBarOff);
-  uint64_t* empty = full + STAGES;
-  uint64_t* tmem_full = empty + STAGES;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_full + 1);
+  const uint32_t sA = base, sB = base + S * C::kABytes;
+  float* sbuf = reinterpret_cast<float*>(gbase + C::kSbufOff);  // [2 acc][scale BN | shift BN]
+  uint64_t* full = reinterpret_cast<uint64_t*>(gbase + C::kBarOff);
+  uint64_t* empty = full + S;
+  uint64_t* tfull = empty + S;   // [2]
+  uint64_t* tempty = tfull + 2;  // [2]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int m0 = blockIdx.x * BM;
-  const int n0 = blockIdx.y * BN;  // within the group
-  const int g = blockIdx.z;
-
   if (threadIdx.x == 0) {
-    for (int i = 0; i < STAGES; ++i) {
-      mbar_init(&full[i], kProducerThreads + 1);
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&full[i], AMODE == A_TMA ? 1 : 128 + 1);
       mbar_init(&empty[i], 1);
     }
-    mbar_init(tmem_full, 1);
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&tfull[i], 1);
+      mbar_init(&tempty[i], 4);
+    }
     fence_mbar_init();
     tma_prefetch(&tmap_w);
+    if (AMODE == A_TMA) tma_prefetch(&tmap_a);
   }
-  if (warp == 4) tmem_alloc(tmem_slot, BN);
+  if (warp == 4) tmem_alloc(tmem_slot, C::kTmemCols);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
 
   if (warp < 4) {
-    // ================= A producers (one output row each) + B TMA (thread 0) =================
-    const int t = threadIdx.x;
-    const int m = m0 + t;
-    const bool mvalid = m < p.M;
-    int nimg = 0, ho = 0, wo = 0;
-    if (mvalid) {
+    // ======================= producers =======================
+    if constexpr (AMODE == A_TMA) {
+      if (threadIdx.x == 0) {
+        uint32_t gk = 0;
+        for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x) {
+          int m0, nt, g;
+          decode_tile(p, tile, m0, nt, g);
+          const int n0 = nt * BN;
+          for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
+            const int stage = gk % S;
+            if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
+            mbar_arrive_expect_tx(&full[stage], C::kABytes + C::kBBytes);
+            tma_load_2d(sA + stage * C::kABytes, &tmap_a, g * p.Cg_in + kb * BK, m0, &full[stage]);
+            tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
+          }
+        }
+      }
+    } else {
+      const int t = threadIdx.x;
+      const uint32_t arow = (uint32_t)t * 128u;
+      const uint32_t sw = (uint32_t)(t & 7);
+      const int CC = p.Cg_in >> 3;
       const int hw = p.Ho * p.Wo;
-      nimg = m / hw;
-      const int rem = m - nimg * hw;
-      ho = rem / p.Wo;
-      wo = rem - ho * p.Wo;
-    }
-    const bf16* xb = p.x + (size_t)nimg * p.H * p.W * p.Cin + (size_t)g * p.Cg_in;
-    const int hi0 = ho * p.stride - p.pad, wi0 = wo * p.stride - p.pad;
-    const uint32_t arow = (uint32_t)t * 128u;
-    const uint32_t sw = (uint32_t)(t & 7);
-    const int CC = p.Cg_in >> 3;  // 16-byte chunks per filter tap
-    int fr = 0, fs = 0, fc = 0;   // fast-path filter position
-    for (int kb = 0; kb < p.nkb; ++kb) {
-      const int stage = kb % STAGES;
-      if (kb >= STAGES) mbar_wait(&empty[stage], ((kb / STAGES) - 1) & 1);
-      if (t == 0) {
-        mbar_arrive_expect_tx(&full[stage], L::kBBytes);
-        tma_load_2d(sB + stage * L::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
-      }
-      const uint32_t dst = sA + stage * L::kABytes + arow;
-      if constexpr (kFast) {
-        const int hi = hi0 + fr, wi = wi0 + fs;
-        const bool ok = mvalid && hi >= 0 && hi < p.H && wi >= 0 && wi < p.W;
-        const bf16* src = ok ? xb + ((size_t)hi * p.W + wi) * p.Cin + fc : p.x;
-        const uint32_t nb = ok ? 16u : 0u;
-#pragma unroll
-        for (int j = 0; j < 8; ++j) cp_async_16(dst + (((uint32_t)j ^ sw) << 4), src + (ok ? j * 8 : 0), nb);
-        fc += BK;
-        if (fc == p.Cg_in) {
-          fc = 0;
-          if (++fs == p.S) {
-            fs = 0;
-            ++fr;
-          }
+      uint32_t gk = 0;
+      for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x) {
+        int m0, nt, g;
+        decode_tile(p, tile, m0, nt, g);
+        const int n0 = nt * BN;
+        const int m = m0 + t;
+        const bool mvalid = m < p.M;
+        int nimg = 0, ho = 0, wo = 0;
+        if (mvalid) {
+          nimg = m / hw;
+          const int rem = m - nimg * hw;
+          ho = rem / p.Wo;
+          wo = rem - ho * p.Wo;
         }
-      } else {
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          const int kc = kb * 8 + j;
-          bool ok = mvalid && kc * 8 < p.K;
-          const bf16* src = p.x;
-          if (ok) {
-            const int rs = kc / CC;
-            const int cc = kc - rs * CC;
-            const int r = rs / p.S;
-            const int s = rs - r * p.S;
-            const int hi = hi0 + r, wi = wi0 + s;
-            ok = hi >= 0 && hi < p.H && wi >= 0 && wi < p.W;
-            if (ok) src = xb + ((size_t)hi * p.W + wi) * p.Cin + cc * 8;
+        const bf16* xb = p.x + (size_t)nimg * p.H * p.W * p.Cin + (size_t)g * p.Cg_in;
+        const int hi0 = ho * p.stride - p.pad, wi0 = wo * p.stride - p.pad;
+        int fr = 0, fs = 0, fc = 0;  // fast-path filter position
+        for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
+          const int stage = gk % S;
+          if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
+          if (t == 0) {
+            mbar_arrive_expect_tx(&full[stage], C::kBBytes);
+            tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
           }
-          cp_async_16(dst + (((uint32_t)j ^ sw) << 4), src, ok ? 16u : 0u);
-        }
-      }
-      cp_async_commit();
-      if (kb >= kLag) {
-        cp_async_wait<kLag>();
-        fence_proxy_async_smem();
-        mbar_arrive(&full[(kb - kLag) % STAGES]);
-      }
-    }
-    cp_async_wait<0>();
-    fence_proxy_async_smem();
-    for (int kb = (p.nkb > kLag ? p.nkb - kLag : 0); kb < p.nkb; ++kb) mbar_arrive(&full[kb % STAGES]);
-
-    // ================= epilogue: TMEM -> registers -> scale/shift/res/ReLU -> bf16 =================
-    mbar_wait(tmem_full, 0);
-    tc_fence_after();
-    const int row = warp * 32 + lane;
-    const int mo = m0 + row;
-    const uint32_t taddr = tmem_base + ((uint32_t)(warp * 32) << 16);
-#pragma unroll 1
-    for (int cb = 0; cb < BN / 32; ++cb) {
-      const int n = n0 + cb * 32;
-      if (n >= p.Cg_out) break;  // warp-uniform
-      uint32_t v[32];
-      tmem_ld_32x32b_x32(taddr + cb * 32, v);
-      tc_wait_ld();
-      if (mo < p.M) {
-        const int ng = g * p.Cg_out + n;
-        const size_t off = (size_t)mo * p.Cout + ng;
-        const int nvalid = p.Cg_out - n;  // >= 8, multiple of 8
+          const uint32_t dst = sA + stage * C::kABytes + arow;
+          if constexpr (AMODE == A_GATHER_FAST) {
+            const int hi = hi0 + fr, wi = wi0 + fs;
+            const bool ok = mvalid && hi >= 0 && hi < p.H && wi >= 0 && wi < p.W;
+            const bf16* src = ok ? xb + ((size_t)hi * p.W + wi) * p.Cin + fc : p.x;
+            const uint32_t nb = ok ? 16u : 0u;
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-          if (q * 8 < nvalid) {
-            const float4 sc0 = __ldg(reinterpret_cast<const float4*>(p.scale + ng + q * 8));
-            const float4 sc1 = __ldg(reinterpret_cast<const float4*>(p.scale + ng + q * 8 + 4));
-            const float4 sh0 = __ldg(reinterpret_cast<const float4*>(p.shift + ng + q * 8));
-            const float4 sh1 = __ldg(reinterpret_cast<const float4*>(p.shift + ng + q * 8 + 4));
-            float f[8];
-            const float scv[8] = {sc0.x, sc0.y, sc0.z, sc0.w, sc1.x, sc1.y, sc1.z, sc1.w};
-            const float shv[8] = {sh0.x, sh0.y, sh0.z, sh0.w, sh1.x, sh1.y, sh1.z, sh1.w};
-#pragma unroll
-            for (int j = 0; j < 8; ++j) f[j] = fmaf(__uint_as_float(v[q * 8 + j]), scv[j], shv[j]);
-            if (p.res) {
-              const uint4 rv = __ldg(reinterpret_cast<const uint4*>(p.res + off + q * 8));
-              const uint32_t rr[4] = {rv.x, rv.y, rv.z, rv.w};
-#pragma unroll
-              for (int j = 0; j < 4; ++j) {
-                const float2 a = unpack_bf16x2(rr[j]);
-                f[2 * j] += a.x;
-                f[2 * j + 1] += a.y;
+            for (int j = 0; j < 8; ++j) cp_async_16(dst + (((uint32_t)j ^ sw) << 4), src + (ok ? j * 8 : 0), nb);
+            fc += BK;
+            if (fc == p.Cg_in) {
+              fc = 0;
+              if (++fs == p.S) {
+                fs = 0;
+                ++fr;
               }
             }
-            if (p.relu) {
+          } else {
 #pragma unroll
-              for (int j = 0; j < 8; ++j) f[j] = fmaxf(f[j], 0.0f);
+            for (int j = 0; j < 8; ++j) {
+              const int kc = kb * 8 + j;
+              bool ok = mvalid && kc * 8 < p.K;
+              const bf16* src = p.x;
+              if (ok) {
+                const int rs = kc / CC;
+                const int cc = kc - rs * CC;
+                const int r = rs / p.S;
+                const int s = rs - r * p.S;
+                const int hi = hi0 + r, wi = wi0 + s;
+                ok = hi >= 0 && hi < p.H && wi >= 0 && wi < p.W;
+                if (ok) src = xb + ((size_t)hi * p.W + wi) * p.Cin + cc * 8;
+              }
+              cp_async_16(dst + (((uint32_t)j ^ sw) << 4), src, ok ? 16u : 0u);
             }
-            uint4 o;
-            o.x = pack_bf16x2(f[0], f[1]);
-            o.y = pack_bf16x2(f[2], f[3]);
-            o.z = pack_bf16x2(f[4], f[5]);
-            o.w = pack_bf16x2(f[6], f[7]);
-            *reinterpret_cast<uint4*>(p.y + off + q * 8) = o;
+          }
+          cp_async_commit();
+          if (gk >= (uint32_t)kLag) {
+            cp_async_wait<kLag>();
+            fence_proxy_async_smem();
+            mbar_arrive(&full[(gk - kLag) % S]);
           }
         }
       }
+      cp_async_wait<0>();
+      fence_proxy_async_smem();
+      for (uint32_t j = gk > (uint32_t)kLag ? gk - kLag : 0; j < gk; ++j) mbar_arrive(&full[j % S]);
     }
-  } else if (lane == 0) {
-    // ================= MMA issuer (single thread) =================
-    constexpr uint32_t idesc = umma_idesc_bf16(BM, BN);
-    for (int kb = 0; kb < p.nkb; ++kb) {
-      const int stage = kb % STAGES;
-      mbar_wait(&full[stage], (kb / STAGES) & 1);
-      tc_fence_after();
-      const uint32_t a0 = sA + stage * L::kABytes, b0 = sB + stage * L::kBBytes;
+  } else if (warp == 4) {
+    // ======================= MMA issuer =======================
+    if (lane == 0) {
+      constexpr uint32_t idesc = umma_idesc_bf16(BM, BN);
+      uint32_t gk = 0, it = 0;
+      for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x, ++it) {
+        const uint32_t acc = it & 1, use = it >> 1;
+        if (it >= 2) mbar_wait(&tempty[acc], (use - 1) & 1);
+        tc_fence_after();
+        const uint32_t tacc = tmem_base + acc * BN;
+        for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
+          const int stage = gk % S;
+          mbar_wait(&full[stage], (gk / S) & 1);
+          tc_fence_after();
+          const uint32_t a0 = sA + stage * C::kABytes, b0 = sB + stage * C::kBBytes;
 #pragma unroll
-      for (int k = 0; k < BK / 16; ++k)
-        tc_mma_bf16(tmem_base, umma_desc_k_sw128(a0 + k * 32), umma_desc_k_sw128(b0 + k * 32), idesc,
-                    (kb | k) != 0 ? 1u : 0u);
-      tc_commit(&empty[stage]);
+          for (int k = 0; k < BK / 16; ++k)
+            tc_mma_bf16(tacc, umma_desc_k_sw128(a0 + k * 32), umma_desc_k_sw128(b0 + k * 32), idesc,
+                        (kb | k) != 0 ? 1u : 0u);
+          tc_commit(&empty[stage]);
+        }
+        tc_commit(&tfull[acc]);
+      }
     }
-    tc_commit(tmem_full);
+    __syncwarp();
+  } else {
+    // ======================= epilogue (128 threads) =======================
+    const int et = threadIdx.x - kEpiWarp0 * 32;
+    const int q = warp & 3;  // TMEM lane quadrant this warp may access
+    const int row = q * 32 + lane;
+    uint32_t it = 0;
+    for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x, ++it) {
+      const uint32_t acc = it & 1, use = it >> 1;
+      int m0, nt, g;
+      decode_tile(p, tile, m0, nt, g);
+      const int n0 = nt * BN;
+      const int ng0 = g * p.Cg_out + n0;
+      const int nvalid_tile = min(BN, p.Cg_out - n0);
+      // stage this tile's scale / shift in smem (double-buffered by accumulator)
+      float* ss = sbuf + acc * 2 * BN;
+      for (int i = et; i < 2 * BN; i += 128) {
+        const int c = i < BN ? i : i - BN;
+        ss[i] = c < nvalid_tile ? (i < BN ? p.scale[ng0 + c] : p.shift[ng0 + c]) : 0.f;
+      }
+      named_bar_sync(1, 128);
+      const int mo = m0 + row;
+      const bool rvalid = mo < p.M;
+      const size_t off = (size_t)(rvalid ? mo : 0) * p.Cout + ng0;
+      uint4 rres[4];
+      const bool has_res = p.res != nullptr;
+      if (has_res && rvalid) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+          rres[j] = (j * 8 < nvalid_tile) ? __ldg(reinterpret_cast<const uint4*>(p.res + off) + j) : make_uint4(0, 0, 0, 0);
+      }
+      mbar_wait(&tfull[acc], use & 1);
+      tc_fence_after();
+      const uint32_t taddr = tmem_base + acc * BN + ((uint32_t)(q * 32) << 16);
+#pragma unroll 1
+      for (int cb = 0; cb < BN / 32; ++cb) {
+        if (cb * 32 >= nvalid_tile) break;  // warp-uniform
+        uint32_t v[32];
+        tmem_ld_32x32b_x32(taddr + cb * 32, v);
+        uint4 cur[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) cur[j] = rres[j];
+        if (has_res && rvalid && (cb + 1) * 32 < nvalid_tile) {  // prefetch the next chunk's residual
+#pragma unroll
+          for (int j = 0; j < 4; ++j)
+            rres[j] = ((cb + 1) * 32 + j * 8 < nvalid_tile)
+                          ? __ldg(reinterpret_cast<const uint4*>(p.res + off + (cb + 1) * 32) + j)
+                          : make_uint4(0, 0, 0, 0);
+        }
+        tc_wait_ld();
+        if (rvalid) {
+          const float* scv = ss + cb * 32;
+          const float* shv = ss + BN + cb * 32;
+#pragma unroll
+          for (int qq = 0; qq < 4; ++qq) {
+            if (cb * 32 + qq * 8 < nvalid_tile) {
+              float f[8];
+#pragma unroll
+              for (int j = 0; j < 8; ++j) f[j] = fmaf(__uint_as_float(v[qq * 8 + j]), scv[qq * 8 + j], shv[qq * 8 + j]);
+              if (has_res) {
+                const uint32_t rr[4] = {cur[qq].x, cur[qq].y, cur[qq].z, cur[qq].w};
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                  const float2 a = unpack_bf16x2(rr[j]);
+                  f[2 * j] += a.x;
+                  f[2 * j + 1] += a.y;
+                }
+              }
+              if (p.relu) {
+#pragma unroll
+                for (int j = 0; j < 8; ++j) f[j] = fmaxf(f[j], 0.0f);
+              }
+              uint4 o;
+              o.x = pack_bf16x2(f[0], f[1]);
+              o.y = pack_bf16x2(f[2], f[3]);
+              o.z = pack_bf16x2(f[4], f[5]);
+              o.w = pack_bf16x2(f[6], f[7]);
+              *reinterpret_cast<uint4*>(p.y + off + cb * 32 + qq * 8) = o;
+            }
+          }
+        }
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&tempty[acc]);
+    }
   }
   tc_fence_before();
   __syncthreads();
-  if (warp == 4) tmem_dealloc(tmem_base, BN);
+  if (warp == 4) tmem_dealloc(tmem_base, C::kTmemCols);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -236,6 +327,18 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
   });
   if (!fn) fail(5, "cuTensorMapEncodeTiled unavailable (driver too old or no GPU)");
   return fn;
+}
+
+// 2-D bf16 tensor map [rows, cols] (cols contiguous), box {64, box_rows}, 128B swizzle
+static void make_tmap(CUtensorMap* m, const void* ptr, uint64_t cols, uint64_t rows, uint32_t box_rows) {
+  cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)cols * 2};
+  cuuint32_t box[2] = {(cuuint32_t)BK, box_rows};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult rc = get_encode()(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(ptr), dims, strides, box,
+                             estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (rc != CUDA_SUCCESS) fail(5, "cuTensorMapEncodeTiled failed");
 }
 
 static int pick_bn(int Cg_out) {
@@ -269,14 +372,7 @@ void conv_layer_init(ConvLayer& L, const std::vector<uint16_t>& w, int Cin_real,
   VCHECK(cudaMalloc(&L.shift, L.Cout * sizeof(float)));
   VCHECK(cudaMemcpy(L.scale, scale.data(), L.Cout * sizeof(float), cudaMemcpyHostToDevice));
   VCHECK(cudaMemcpy(L.shift, shift.data(), L.Cout * sizeof(float), cudaMemcpyHostToDevice));
-  cuuint64_t dims[2] = {(cuuint64_t)L.Kp, (cuuint64_t)L.Cout};
-  cuuint64_t strides[1] = {(cuuint64_t)L.Kp * 2};
-  cuuint32_t box[2] = {(cuuint32_t)BK, (cuuint32_t)L.BN};
-  cuuint32_t estr[2] = {1, 1};
-  CUresult rc = get_encode()(&L.tmap_w, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, L.w, dims, strides, box, estr,
-                             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
-                             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  if (rc != CUDA_SUCCESS) fail(5, "cuTensorMapEncodeTiled failed for conv weights");
+  make_tmap(&L.tmap_w, L.w, (uint64_t)L.Kp, (uint64_t)L.Cout, (uint32_t)L.BN);
 }
 
 void conv_layer_free(ConvLayer& L) {
@@ -287,18 +383,25 @@ void conv_layer_free(ConvLayer& L) {
   L.scale = L.shift = nullptr;
 }
 
-template <int BN, int STAGES, bool kFast>
-static void launch_t(const ConvLayer& L, const ConvParams& p, cudaStream_t st) {
-  auto kern = conv_tc_kernel<BN, STAGES, kFast>;
-  constexpr int smem = ConvSmem<BN, STAGES>::kBytes;
+template <int BN, int AMODE>
+static void launch_t(const ConvLayer& L, const CUtensorMap& tmap_a, const ConvParams& p, cudaStream_t st) {
+  auto kern = conv_tc_kernel<BN, AMODE>;
+  constexpr int smem = Cfg<BN>::kBytes;
   static bool attr_set = false;  // per instantiation
   if (!attr_set) {
     VCHECK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
     attr_set = true;
   }
-  dim3 grid((p.M + BM - 1) / BM, (L.Cg_out + BN - 1) / BN, L.groups);
-  kern<<<grid, kThreads, smem, st>>>(L.tmap_w, p);
+  const int grid = p.n_tiles < num_sms() ? p.n_tiles : num_sms();
+  kern<<<grid, kThreads, smem, st>>>(L.tmap_w, tmap_a, p);
   LAUNCHED();
+}
+
+template <int BN>
+static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, const ConvParams& p, cudaStream_t st) {
+  if (amode == A_TMA) launch_t<BN, A_TMA>(L, ta, p, st);
+  else if (amode == A_GATHER_FAST) launch_t<BN, A_GATHER_FAST>(L, ta, p, st);
+  else launch_t<BN, A_GATHER_GENERAL>(L, ta, p, st);
 }
 
 void conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const bf16* res, bf16* y,
@@ -328,17 +431,28 @@ void conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   if (M > INT32_MAX - BM) fail(1, "conv: M too large for one launch");
   p.M = (int)M;
   p.relu = L.relu ? 1 : 0;
-  const bool fast = (L.Cg_in % BK) == 0;
+  p.n_mt = (p.M + BM - 1) / BM;
+  p.n_nt = (L.Cg_out + L.BN - 1) / L.BN;
+  const int64_t tiles = (int64_t)p.n_mt * p.n_nt * L.groups;
+  if (tiles > INT32_MAX) fail(1, "conv: too many tiles");
+  p.n_tiles = (int)tiles;
+  // A operand path: a 1x1 stride-1 unpadded ungrouped conv (or FC) reads a plain [M, C] matrix -> TMA
+  int amode;
+  CUtensorMap ta;
+  std::memset(&ta, 0, sizeof(ta));
+  if (L.R == 1 && L.S == 1 && L.stride == 1 && L.pad == 0 && L.groups == 1 && L.Cin % BK == 0) {
+    amode = A_TMA;
+    make_tmap(&ta, x, (uint64_t)L.Cin, (uint64_t)M, BM);
+  } else {
+    amode = (L.Cg_in % BK) == 0 ? A_GATHER_FAST : A_GATHER_GENERAL;
+    ta = L.tmap_w;  // unused
+  }
   const double flops = 2.0 * (double)M * L.Cout * L.K;
   const double bytes = 2.0 * ((double)N * H * W * L.Cin + (double)M * L.Cout * (res ? 2 : 1) + (double)L.Cout * L.Kp);
   prof_begin(st);
-  if (L.BN == 256) {
-    if (fast) launch_t<256, 4, true>(L, p, st); else launch_t<256, 4, false>(L, p, st);
-  } else if (L.BN == 128) {
-    if (fast) launch_t<128, 4, true>(L, p, st); else launch_t<128, 4, false>(L, p, st);
-  } else {
-    if (fast) launch_t<64, 4, true>(L, p, st); else launch_t<64, 4, false>(L, p, st);
-  }
+  if (L.BN == 256) launch_bn<256>(L, amode, ta, p, st);
+  else if (L.BN == 128) launch_bn<128>(L, amode, ta, p, st);
+  else launch_bn<64>(L, amode, ta, p, st);
   prof_end(st, 0, flops, bytes);
 }
 

@@ -141,16 +141,25 @@ static uint16_t f2bf_bits(float f) {  // f is bf16-representable (generator cont
   return (uint16_t)(u >> 16);
 }
 
+// Device buffers are stream-ordered allocations from the device's default memory pool
+// (release threshold raised at plan time), so the Staged plan can free A_{k-1} as soon as
+// stage k has consumed it while repeated transfers reuse the pooled memory.
+thread_local cudaStream_t tl_stream = nullptr;
 struct DevBuf {
   void* p = nullptr;
   size_t bytes = 0;
+  cudaStream_t st = nullptr;
   void alloc(size_t b) {
     release();
-    if (b) VCHECK(cudaMalloc(&p, b));
+    st = tl_stream;
+    if (b) VCHECK(cudaMallocAsync(&p, b, st));
     bytes = b;
   }
+  void ensure(size_t b) {
+    if (b > bytes) alloc(b);
+  }
   void release() {
-    if (p) cudaFree(p);
+    if (p) cudaFreeAsync(p, st);
     p = nullptr;
     bytes = 0;
   }
@@ -199,6 +208,10 @@ struct vista_ctx {
   bool profiling = false;
   std::string last_error;
   ~vista_ctx() {
+    for (auto* v : {&A, &F, &MM, &Y, &slot_store})
+      for (auto& b : *v) b->release();
+    for (DevBuf* b : {&pair_str, &pair_img, &d_X, &d_labels, &d_img_keys, &d_str_keys, &d_px}) b->release();
+    if (stream) cudaStreamSynchronize(stream);
     for (auto& L : convs) conv_layer_free(L);
     if (nccl_comm) {
       Nccl& n = nccl_lib();
@@ -226,7 +239,10 @@ template <class F>
 vista_status guarded(vista_ctx* c, F&& f) {
   Profiler* saved = g_prof;
   try {
-    if (c) g_prof = c->profiling ? c->prof.get() : nullptr;
+    if (c) {
+      g_prof = c->profiling ? c->prof.get() : nullptr;
+      tl_stream = c->stream;
+    }
     f();
     g_prof = saved;
     return VISTA_OK;
@@ -471,6 +487,13 @@ VISTA_API vista_status vista_plan(vista_cnn cnn, const int32_t* layers, int32_t 
       VCHECK(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
       c->own_stream = true;
     }
+    tl_stream = c->stream;
+    {
+      cudaMemPool_t pool;
+      VCHECK(cudaDeviceGetDefaultMemPool(&pool, c->sys.device));
+      uint64_t thr = UINT64_MAX;
+      VCHECK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+    }
     c->n_img = n_images_local;
     c->n_str = n_str_rows;
     c->d_s = n_str_feats;
@@ -542,10 +565,8 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
     const float* X = (const float*)to_device(c, c->d_X, structured, (size_t)c->n_str * c->d_s * 4);
     const uint8_t* lab = (const uint8_t*)to_device(c, c->d_labels, labels, (size_t)c->n_str);
     // ---- S4 join (Eq. 3), once for all layers ----
-    if (c->pair_str.bytes < (size_t)(c->n_str * 4 + 4)) {
-      c->pair_str.alloc(c->n_str * 4 + 4);
-      c->pair_img.alloc(c->n_str * 4 + 4);
-    }
+    c->pair_str.ensure(c->n_str * 4 + 4);
+    c->pair_img.ensure(c->n_str * 4 + 4);
     const uint64_t ss = vg_subseed(c->lr.split_seed, VG_S_SPLIT);
     JoinResult jr = join_keys(ik, c->n_img, sk, c->n_str, ss, (int32_t*)c->pair_str.p, (int32_t*)c->pair_img.p, st);
     if (jr.dup & 2) fail(1, "a key equals the reserved empty-slot value INT64_MIN");
@@ -588,10 +609,7 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
       }
       // Staged: the input activation of this block is no longer needed (Fig 5E) — unless it is an
       // FC tap whose activation doubles as its features
-      if (t > 0 && !(S[t - 1].fc_tap && layer_index(c, t - 1) >= 0)) {
-        VCHECK(cudaStreamSynchronize(st));
-        c->A[t - 1]->release();
-      }
+      if (t > 0 && !(S[t - 1].fc_tap && layer_index(c, t - 1) >= 0)) c->A[t - 1]->release();
     }
     VCHECK(cudaStreamSynchronize(st));
     c->d_px.release();

@@ -19,6 +19,7 @@
 // mainloop of tile i+1; an mbarrier ring of STAGES k-blocks feeds the tensor core.
 #include <cudaTypedefs.h>
 
+#include <cstdio>
 #include <cstring>
 #include <mutex>
 
@@ -27,7 +28,7 @@
 
 namespace vista {
 
-enum AMode { A_GATHER_FAST = 0, A_GATHER_GENERAL = 1, A_TMA = 2 };
+enum AMode { A_GATHER_FAST = 0, A_GATHER_GENERAL = 1, A_TMA = 2, A_GATHER_ROW = 3 };
 
 struct ConvParams {
   const bf16* x;
@@ -44,14 +45,18 @@ constexpr int kThreads = 288;  // 4 producer warps + 1 MMA warp + 4 epilogue war
 constexpr int kEpiWarp0 = 5;
 constexpr int kLag = 2;        // cp.async groups in flight before a stage is published
 
-template <int BN>
+// Shared memory: [A stages][B stages][output staging: BN/64 sub-tiles of 128 x 64 bf16,
+// 128B-swizzled (TMA epilogue only)][scale/shift x 2][barriers]
+template <int BN, bool TMA_EPI>
 struct Cfg {
-  static constexpr int kStages = BN == 256 ? 4 : (BN == 128 ? 6 : 8);
+  static constexpr int kStages = TMA_EPI ? (BN == 256 ? 3 : (BN == 128 ? 4 : 6)) : (BN == 256 ? 4 : (BN == 128 ? 6 : 8));
   static constexpr int kABytes = BM * BK * 2;  // 16 KB
   static constexpr int kBBytes = BN * BK * 2;
-  static constexpr int kSbufOff = kStages * (kABytes + kBBytes);
+  static constexpr int kOutOff = kStages * (kABytes + kBBytes);
+  static constexpr int kOutBytes = TMA_EPI ? BM * BN * 2 : 0;
+  static constexpr int kSbufOff = kOutOff + kOutBytes;
   static constexpr int kBarOff = kSbufOff + 2 * 2 * BN * 4;
-  static constexpr int kBytes = kBarOff + (2 * kStages + 4) * 8 + 16 + 1024;  // + alignment slack
+  static constexpr int kBytes = kBarOff + (2 * kStages + 5) * 8 + 16 + 1024;  // + alignment slack
   static constexpr int kTmemCols = 2 * BN;
 };
 
@@ -66,23 +71,49 @@ __device__ __forceinline__ void decode_tile(const ConvParams& p, int tile, int& 
   nt = rem - mt * p.n_nt;
 }
 
-template <int BN, int AMODE>
+__device__ __forceinline__ void epi_math(const uint32_t* v, const float* scv, const float* shv, bool has_res,
+                                         uint4 r, bool relu, uint4& o) {
+  float f[8];
+#pragma unroll
+  for (int j = 0; j < 8; ++j) f[j] = fmaf(__uint_as_float(v[j]), scv[j], shv[j]);
+  if (has_res) {
+    const uint32_t rr[4] = {r.x, r.y, r.z, r.w};
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const float2 a = unpack_bf16x2(rr[j]);
+      f[2 * j] += a.x;
+      f[2 * j + 1] += a.y;
+    }
+  }
+  if (relu) {
+#pragma unroll
+    for (int j = 0; j < 8; ++j) f[j] = fmaxf(f[j], 0.0f);
+  }
+  o.x = pack_bf16x2(f[0], f[1]);
+  o.y = pack_bf16x2(f[2], f[3]);
+  o.z = pack_bf16x2(f[4], f[5]);
+  o.w = pack_bf16x2(f[6], f[7]);
+}
+
+template <int BN, int AMODE, bool TMA_EPI>
 __global__ void __launch_bounds__(kThreads, 1)
     conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__ CUtensorMap tmap_a,
+                   const __grid_constant__ CUtensorMap tmap_y, const __grid_constant__ CUtensorMap tmap_r,
                    const ConvParams p) {
-  using C = Cfg<BN>;
+  using C = Cfg<BN, TMA_EPI>;
   constexpr int S = C::kStages;
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 1023u) & ~1023u;
   uint8_t* gbase = smem_raw + (base - raw);
-  const uint32_t sA = base, sB = base + S * C::kABytes;
+  const uint32_t sA = base, sB = base + S * C::kABytes, sO = base + C::kOutOff;
   float* sbuf = reinterpret_cast<float*>(gbase + C::kSbufOff);  // [2 acc][scale BN | shift BN]
   uint64_t* full = reinterpret_cast<uint64_t*>(gbase + C::kBarOff);
   uint64_t* empty = full + S;
   uint64_t* tfull = empty + S;   // [2]
   uint64_t* tempty = tfull + 2;  // [2]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint64_t* rbar = tempty + 2;   // residual tile landed (TMA epilogue)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rbar + 1);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
@@ -94,9 +125,11 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(&tfull[i], 1);
       mbar_init(&tempty[i], 4);
     }
+    mbar_init(rbar, 1);
     fence_mbar_init();
     tma_prefetch(&tmap_w);
     if (AMODE == A_TMA) tma_prefetch(&tmap_a);
+    if (TMA_EPI) tma_prefetch(&tmap_y);
   }
   if (warp == 4) tmem_alloc(tmem_slot, C::kTmemCols);
   tc_fence_before();
@@ -168,6 +201,18 @@ __global__ void __launch_bounds__(kThreads, 1)
                 ++fr;
               }
             }
+          } else if constexpr (AMODE == A_GATHER_ROW) {
+            // k-block = filter row r (= kb); 16-byte chunk j = filter column s, 8 channels:
+            // the 8 chunks of a row are contiguous in the NHWC8 input.
+            const int hi = hi0 + kb;
+            const bool rowok = mvalid && hi >= 0 && hi < p.H;
+            const bf16* rowp = xb + (size_t)hi * p.W * 8;
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+              const int wi = wi0 + j;
+              const bool ok = rowok && j < p.S && wi >= 0 && wi < p.W;
+              cp_async_16(dst + (((uint32_t)j ^ sw) << 4), ok ? rowp + (size_t)wi * 8 : p.x, ok ? 16u : 0u);
+            }
           } else {
 #pragma unroll
             for (int j = 0; j < 8; ++j) {
@@ -224,10 +269,11 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     __syncwarp();
   } else {
-    // ======================= epilogue (128 threads) =======================
+    // ======================= epilogue (128 threads, one output row each) =======================
     const int et = threadIdx.x - kEpiWarp0 * 32;
     const int q = warp & 3;  // TMEM lane quadrant this warp may access
     const int row = q * 32 + lane;
+    const bool has_res = p.res != nullptr;
     uint32_t it = 0;
     for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x, ++it) {
       const uint32_t acc = it & 1, use = it >> 1;
@@ -236,6 +282,16 @@ __global__ void __launch_bounds__(kThreads, 1)
       const int n0 = nt * BN;
       const int ng0 = g * p.Cg_out + n0;
       const int nvalid_tile = min(BN, p.Cg_out - n0);
+      if constexpr (TMA_EPI) {
+        if (et == 0) {
+          bulk_wait_read0();  // the previous tile's stores no longer read the staging buffer
+          if (has_res) {
+            const int nsub = (nvalid_tile + 63) / 64;
+            mbar_arrive_expect_tx(rbar, nsub * BM * 128);
+            for (int st = 0; st < nsub; ++st) tma_load_2d(sO + st * BM * 128, &tmap_r, ng0 + st * 64, m0, rbar);
+          }
+        }
+      }
       // stage this tile's scale / shift in smem (double-buffered by accumulator)
       float* ss = sbuf + acc * 2 * BN;
       for (int i = et; i < 2 * BN; i += 128) {
@@ -246,12 +302,14 @@ __global__ void __launch_bounds__(kThreads, 1)
       const int mo = m0 + row;
       const bool rvalid = mo < p.M;
       const size_t off = (size_t)(rvalid ? mo : 0) * p.Cout + ng0;
-      uint4 rres[4];
-      const bool has_res = p.res != nullptr;
-      if (has_res && rvalid) {
+      uint4 rres[4] = {};
+      if constexpr (TMA_EPI) {
+        if (has_res) mbar_wait(rbar, it & 1);
+      } else if (has_res && rvalid) {
 #pragma unroll
         for (int j = 0; j < 4; ++j)
-          rres[j] = (j * 8 < nvalid_tile) ? __ldg(reinterpret_cast<const uint4*>(p.res + off) + j) : make_uint4(0, 0, 0, 0);
+          rres[j] = (j * 8 < nvalid_tile) ? __ldg(reinterpret_cast<const uint4*>(p.res + off) + j)
+                                          : make_uint4(0, 0, 0, 0);
       }
       mbar_wait(&tfull[acc], use & 1);
       tc_fence_after();
@@ -261,53 +319,58 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (cb * 32 >= nvalid_tile) break;  // warp-uniform
         uint32_t v[32];
         tmem_ld_32x32b_x32(taddr + cb * 32, v);
-        uint4 cur[4];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) cur[j] = rres[j];
-        if (has_res && rvalid && (cb + 1) * 32 < nvalid_tile) {  // prefetch the next chunk's residual
-#pragma unroll
-          for (int j = 0; j < 4; ++j)
-            rres[j] = ((cb + 1) * 32 + j * 8 < nvalid_tile)
-                          ? __ldg(reinterpret_cast<const uint4*>(p.res + off + (cb + 1) * 32) + j)
-                          : make_uint4(0, 0, 0, 0);
-        }
-        tc_wait_ld();
-        if (rvalid) {
-          const float* scv = ss + cb * 32;
-          const float* shv = ss + BN + cb * 32;
+        const float* scv = ss + cb * 32;
+        const float* shv = ss + BN + cb * 32;
+        if constexpr (TMA_EPI) {
+          tc_wait_ld();
+          const uint32_t sub = sO + (cb >> 1) * BM * 128 + row * 128;
 #pragma unroll
           for (int qq = 0; qq < 4; ++qq) {
-            if (cb * 32 + qq * 8 < nvalid_tile) {
-              float f[8];
+            const uint32_t addr = sub + (((uint32_t)((cb & 1) * 4 + qq) ^ (uint32_t)(row & 7)) << 4);
+            const uint4 r = has_res ? lds128(addr) : make_uint4(0, 0, 0, 0);
+            uint4 o;
+            epi_math(v + qq * 8, scv + qq * 8, shv + qq * 8, has_res, r, p.relu, o);
+            sts128(addr, o);
+          }
+        } else {
+          uint4 cur[4];
 #pragma unroll
-              for (int j = 0; j < 8; ++j) f[j] = fmaf(__uint_as_float(v[qq * 8 + j]), scv[qq * 8 + j], shv[qq * 8 + j]);
-              if (has_res) {
-                const uint32_t rr[4] = {cur[qq].x, cur[qq].y, cur[qq].z, cur[qq].w};
+          for (int j = 0; j < 4; ++j) cur[j] = rres[j];
+          if (has_res && rvalid && (cb + 1) * 32 < nvalid_tile) {  // prefetch the next chunk's residual
 #pragma unroll
-                for (int j = 0; j < 4; ++j) {
-                  const float2 a = unpack_bf16x2(rr[j]);
-                  f[2 * j] += a.x;
-                  f[2 * j + 1] += a.y;
-                }
+            for (int j = 0; j < 4; ++j)
+              rres[j] = ((cb + 1) * 32 + j * 8 < nvalid_tile)
+                            ? __ldg(reinterpret_cast<const uint4*>(p.res + off + (cb + 1) * 32) + j)
+                            : make_uint4(0, 0, 0, 0);
+          }
+          tc_wait_ld();
+          if (rvalid) {
+#pragma unroll
+            for (int qq = 0; qq < 4; ++qq) {
+              if (cb * 32 + qq * 8 < nvalid_tile) {
+                uint4 o;
+                epi_math(v + qq * 8, scv + qq * 8, shv + qq * 8, has_res, cur[qq], p.relu, o);
+                *reinterpret_cast<uint4*>(p.y + off + cb * 32 + qq * 8) = o;
               }
-              if (p.relu) {
-#pragma unroll
-                for (int j = 0; j < 8; ++j) f[j] = fmaxf(f[j], 0.0f);
-              }
-              uint4 o;
-              o.x = pack_bf16x2(f[0], f[1]);
-              o.y = pack_bf16x2(f[2], f[3]);
-              o.z = pack_bf16x2(f[4], f[5]);
-              o.w = pack_bf16x2(f[6], f[7]);
-              *reinterpret_cast<uint4*>(p.y + off + cb * 32 + qq * 8) = o;
             }
           }
         }
       }
+      // accumulator drained: the MMA warp may reuse it
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&tempty[acc]);
+      if constexpr (TMA_EPI) {
+        fence_proxy_async_smem();
+        named_bar_sync(1, 128);
+        if (et == 0) {
+          const int nsub = (nvalid_tile + 63) / 64;
+          for (int st = 0; st < nsub; ++st) tma_store_2d(&tmap_y, ng0 + st * 64, m0, sO + st * BM * 128);
+          bulk_commit();
+        }
+      }
     }
+    if (TMA_EPI && et == 0) bulk_wait0();
   }
   tc_fence_before();
   __syncthreads();
@@ -341,11 +404,12 @@ static void make_tmap(CUtensorMap* m, const void* ptr, uint64_t cols, uint64_t r
   if (rc != CUDA_SUCCESS) fail(5, "cuTensorMapEncodeTiled failed");
 }
 
-static int pick_bn(int Cg_out) {
+static int pick_bn(int Cg_out, int groups) {
   if (Cg_out % 256 == 0) return 256;
   if (Cg_out % 128 == 0) return 128;
   if (Cg_out % 64 == 0) return 64;
-  return 128;
+  if (groups == 1 && Cg_out < 128) return 128;  // one masked tile (e.g. AlexNet conv1, 96)
+  return Cg_out > 128 ? 256 : 128;              // masked last tile (e.g. FC 1000)
 }
 
 void conv_layer_init(ConvLayer& L, const std::vector<uint16_t>& w, int Cin_real, const std::vector<float>& scale,
@@ -356,16 +420,19 @@ void conv_layer_init(ConvLayer& L, const std::vector<uint16_t>& w, int Cin_real,
   if (L.Cg_in % 8 || L.Cg_out % 8) fail(1, "conv: per-group channels must be multiples of 8");
   const int cg_real = Cin_real / L.groups;
   L.K = L.R * L.S * L.Cg_in;
-  L.Kp = (L.K + BK - 1) / BK * BK;
-  L.BN = pick_bn(L.Cg_out);
+  // first layers (input padded to 8 channels, filters at most 8 wide): one k-block per filter row
+  L.row_mode = L.groups == 1 && L.Cg_in == 8 && L.S <= 8 && L.R * 64 <= ((L.K + BK - 1) / BK * BK) * 2;
+  L.Kp = L.row_mode ? L.R * BK : (L.K + BK - 1) / BK * BK;
+  L.BN = pick_bn(L.Cg_out, L.groups);
   // repack OHWI [Cout][R][S][cg_real] -> [Cout][Kp] with channel padding cg_real -> Cg_in and K padding
   std::vector<uint16_t> packed((size_t)L.Cout * L.Kp, 0);
   for (int o = 0; o < L.Cout; ++o)
     for (int r = 0; r < L.R; ++r)
       for (int s = 0; s < L.S; ++s)
-        for (int c = 0; c < cg_real; ++c)
-          packed[(size_t)o * L.Kp + (size_t)(r * L.S + s) * L.Cg_in + c] =
-              w[(((size_t)o * L.R + r) * L.S + s) * cg_real + c];
+        for (int c = 0; c < cg_real; ++c) {
+          const size_t k = L.row_mode ? (size_t)r * BK + s * 8 + c : (size_t)(r * L.S + s) * L.Cg_in + c;
+          packed[(size_t)o * L.Kp + k] = w[(((size_t)o * L.R + r) * L.S + s) * cg_real + c];
+        }
   VCHECK(cudaMalloc(&L.w, packed.size() * 2));
   VCHECK(cudaMemcpy(L.w, packed.data(), packed.size() * 2, cudaMemcpyHostToDevice));
   VCHECK(cudaMalloc(&L.scale, L.Cout * sizeof(float)));
@@ -383,25 +450,30 @@ void conv_layer_free(ConvLayer& L) {
   L.scale = L.shift = nullptr;
 }
 
-template <int BN, int AMODE>
-static void launch_t(const ConvLayer& L, const CUtensorMap& tmap_a, const ConvParams& p, cudaStream_t st) {
-  auto kern = conv_tc_kernel<BN, AMODE>;
-  constexpr int smem = Cfg<BN>::kBytes;
+template <int BN, int AMODE, bool TE>
+static void launch_t(const ConvLayer& L, const CUtensorMap& ta, const CUtensorMap& ty, const CUtensorMap& tr,
+                     const ConvParams& p, cudaStream_t st) {
+  auto kern = conv_tc_kernel<BN, AMODE, TE>;
+  constexpr int smem = Cfg<BN, TE>::kBytes;
   static bool attr_set = false;  // per instantiation
   if (!attr_set) {
     VCHECK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
     attr_set = true;
   }
   const int grid = p.n_tiles < num_sms() ? p.n_tiles : num_sms();
-  kern<<<grid, kThreads, smem, st>>>(L.tmap_w, tmap_a, p);
+  kern<<<grid, kThreads, smem, st>>>(L.tmap_w, ta, ty, tr, p);
   LAUNCHED();
 }
 
-template <int BN>
-static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, const ConvParams& p, cudaStream_t st) {
-  if (amode == A_TMA) launch_t<BN, A_TMA>(L, ta, p, st);
-  else if (amode == A_GATHER_FAST) launch_t<BN, A_GATHER_FAST>(L, ta, p, st);
-  else launch_t<BN, A_GATHER_GENERAL>(L, ta, p, st);
+template <int BN, bool TE>
+static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, const CUtensorMap& ty,
+                      const CUtensorMap& tr, const ConvParams& p, cudaStream_t st) {
+  switch (amode) {
+    case A_TMA: launch_t<BN, A_TMA, TE>(L, ta, ty, tr, p, st); break;
+    case A_GATHER_FAST: launch_t<BN, A_GATHER_FAST, TE>(L, ta, ty, tr, p, st); break;
+    case A_GATHER_ROW: launch_t<BN, A_GATHER_ROW, TE>(L, ta, ty, tr, p, st); break;
+    default: launch_t<BN, A_GATHER_GENERAL, TE>(L, ta, ty, tr, p, st); break;
+  }
 }
 
 void conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const bf16* res, bf16* y,
@@ -438,22 +510,45 @@ void conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   p.n_tiles = (int)tiles;
   // A operand path: a 1x1 stride-1 unpadded ungrouped conv (or FC) reads a plain [M, C] matrix -> TMA
   int amode;
-  CUtensorMap ta;
+  CUtensorMap ta, ty, tr;
   std::memset(&ta, 0, sizeof(ta));
   if (L.R == 1 && L.S == 1 && L.stride == 1 && L.pad == 0 && L.groups == 1 && L.Cin % BK == 0) {
     amode = A_TMA;
     make_tmap(&ta, x, (uint64_t)L.Cin, (uint64_t)M, BM);
   } else {
-    amode = (L.Cg_in % BK) == 0 ? A_GATHER_FAST : A_GATHER_GENERAL;
+    amode = L.row_mode ? A_GATHER_ROW : ((L.Cg_in % BK) == 0 ? A_GATHER_FAST : A_GATHER_GENERAL);
     ta = L.tmap_w;  // unused
+  }
+  // epilogue: staged in smem and written by TMA (residual read by TMA) unless a group's last N tile
+  // would spill into the next group's channels
+  // (long-K layers keep the register epilogue: it is hidden behind the mainloop and frees the staging
+  // smem for a deeper k-block ring)
+  const bool tma_epi = (L.groups == 1 || L.Cg_out % L.BN == 0) && L.Cout % 8 == 0 && p.nkb <= 8;
+  if (tma_epi) {
+    make_tmap(&ty, y, (uint64_t)L.Cout, (uint64_t)M, BM);
+    if (res) make_tmap(&tr, res, (uint64_t)L.Cout, (uint64_t)M, BM);
+    else tr = ty;
+  } else {
+    ty = tr = L.tmap_w;  // unused
   }
   const double flops = 2.0 * (double)M * L.Cout * L.K;
   const double bytes = 2.0 * ((double)N * H * W * L.Cin + (double)M * L.Cout * (res ? 2 : 1) + (double)L.Cout * L.Kp);
   prof_begin(st);
-  if (L.BN == 256) launch_bn<256>(L, amode, ta, p, st);
-  else if (L.BN == 128) launch_bn<128>(L, amode, ta, p, st);
-  else launch_bn<64>(L, amode, ta, p, st);
-  prof_end(st, 0, flops, bytes);
+  if (tma_epi) {
+    if (L.BN == 256) launch_bn<256, true>(L, amode, ta, ty, tr, p, st);
+    else if (L.BN == 128) launch_bn<128, true>(L, amode, ta, ty, tr, p, st);
+    else launch_bn<64, true>(L, amode, ta, ty, tr, p, st);
+  } else {
+    if (L.BN == 256) launch_bn<256, false>(L, amode, ta, ty, tr, p, st);
+    else if (L.BN == 128) launch_bn<128, false>(L, amode, ta, ty, tr, p, st);
+    else launch_bn<64, false>(L, amode, ta, ty, tr, p, st);
+  }
+  char label[160] = {0};
+  if (prof_labels())
+    snprintf(label, sizeof(label), "conv R%d S%d s%d g%d Cin%d Cout%d HxW%dx%d M%d K%d BN%d amode%d epi%d tiles%d%s", L.R,
+             L.S, L.stride, L.groups, L.Cin, L.Cout, H, W, p.M, L.K, L.BN, amode, tma_epi ? 1 : 0, p.n_tiles,
+             res ? " res" : "");
+  prof_end(st, 0, flops, bytes, label);
 }
 
 }  // namespace vista

@@ -40,6 +40,7 @@ struct ConvLayer {
   int Cin = 0, Cout = 0, R = 1, S = 1, stride = 1, pad = 0, groups = 1;  // Cin: channels as stored (padded)
   int Cg_in = 0, Cg_out = 0, K = 0, Kp = 0, BN = 128;
   bool relu = false;
+  bool row_mode = false;     // Cin = 8, S <= 8: one k-block per filter row, k = r*64 + s*8 + c
   bf16* w = nullptr;         // [Cout][Kp]
   float* scale = nullptr;    // [Cout]
   float* shift = nullptr;    // [Cout]
@@ -93,7 +94,8 @@ LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_tr
 struct Profiler;
 extern thread_local Profiler* g_prof;
 void prof_begin(cudaStream_t st);
-void prof_end(cudaStream_t st, int cls, double flops, double bytes);
+void prof_end(cudaStream_t st, int cls, double flops, double bytes, const char* label = nullptr);
+bool prof_labels();  // true when per-launch records are logged (VISTA_PROF_LOG)
 
 int num_sms();
 

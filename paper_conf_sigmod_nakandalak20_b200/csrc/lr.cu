@@ -10,34 +10,80 @@
 // partials are reduced in a fixed order in fp64 (deterministic), then allreduced across
 // ranks (fp64 NCCL) and applied by a one-block update kernel in fp64.
 #include <cmath>
+#include <mutex>
+#include <set>
 
 #include "internal.h"
 #include "ptx.cuh"
 
 namespace vista {
 
-constexpr int RG = 4;  // rows per block-reduction round
+constexpr int kMaxRB = 16;     // rows per streamed block (upper bound)
+constexpr int kStagesLR = 3;   // row blocks in flight per CTA
+constexpr int kLRThreads = 512;
 
 struct PassArgs {
   const bf16* MM;
   const uint8_t* y;
-  int64_t r0, r1;       // row range [r0, r1) of this pass (train rows)
+  int64_t r0, r1;       // row range [r0, r1) of this pass
+  int64_t n_train;      // rows < n_train are train rows (eval mode)
   int ld, chunks;       // ld elements per row, chunks = ld / 8
+  int rb;               // rows per streamed block
   const float* mu;      // [ld]
   const float* what;    // [ld]  inv_j * (w_j or v_j), 0 on excluded / pad columns
   const float* bhat;    // [1]
   float* partial;       // [gridDim.x][ld + 4] (16-byte aligned rows; ld + 2 used)
+  unsigned long long* counts;  // eval: [5]
 };
 
 __device__ __forceinline__ float softplusf(float z) { return z > 0.f ? z + log1pf(__expf(-z)) : log1pf(__expf(z)); }
 
-// MODE 0: sum x; MODE 1: sum (x - mu)^2; MODE 2: power pass (phi = z); MODE 3: gradient pass
+__device__ __forceinline__ void bulk_load(uint32_t dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+
+// One pass over rows [r0, r1) of MM.  Rows are streamed into shared memory in blocks of
+// rb contiguous rows by the bulk-copy engine (kStagesLR blocks in flight per CTA, one CTA per
+// SM), so HBM stays busy while the threads compute.  Thread t owns 16-byte column chunks
+// t, t + blockDim, ... of every row.
+//   MODE 0: sum_p x_pj                          MODE 1: sum_p (x_pj - mu_j)^2
+//   MODE 2: power pass  phi_p = z_p             MODE 3: gradient pass  phi_p = sigmoid(z_p) - y_p
+//   MODE 4: evaluation (counts only)
+// with z_p = b^ + sum_j w^_j (x_pj - mu_j); modes 2/3 accumulate sum_p phi_p (x_pj - mu_j),
+// sum_p phi_p and sum_p loss_p into this CTA's partial row (fixed row-block -> CTA map).
 template <int CH, int MODE>
-__global__ void __launch_bounds__(1024) lr_pass_kernel(const PassArgs a) {
-  __shared__ float red[2][RG][32];
+__global__ void __launch_bounds__(kLRThreads, 1) lr_stream_kernel(const PassArgs a) {
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  const uint32_t base = (raw + 127u) & ~127u;
+  uint8_t* gbase = smem_raw + (base - raw);
+  const uint32_t row_bytes = (uint32_t)a.ld * 2u;
+  const uint32_t stage_bytes = ((uint32_t)a.rb * row_bytes + 127u) & ~127u;
+  float* red = reinterpret_cast<float*>(gbase + kStagesLR * stage_bytes);  // [kMaxRB][32]
+  float* phis = red + kMaxRB * 32;                                         // [kMaxRB]
+  uint64_t* full = reinterpret_cast<uint64_t*>(phis + kMaxRB);             // [kStagesLR]
+
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarps = blockDim.x >> 5;
-  const int64_t n = a.r1 - a.r0;
-  const int64_t rb = a.r0 + n * blockIdx.x / gridDim.x, re = a.r0 + n * (blockIdx.x + 1) / gridDim.x;
+  const int64_t nrows = a.r1 - a.r0;
+  const int64_t nblk = (nrows + a.rb - 1) / a.rb;
+  if (tid == 0) {
+    for (int i = 0; i < kStagesLR; ++i) mbar_init(&full[i], 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  auto issue = [&](int64_t blk, int stage) {
+    const int64_t r = a.r0 + blk * a.rb;
+    const int64_t nr = min((int64_t)a.rb, a.r1 - r);
+    const uint32_t bytes = (uint32_t)nr * row_bytes;
+    mbar_arrive_expect_tx(&full[stage], bytes);
+    bulk_load(base + stage * stage_bytes, a.MM + (size_t)r * a.ld, bytes, &full[stage]);
+  };
+  if (tid == 0) {
+    int i = 0;
+    for (int64_t blk = blockIdx.x; blk < nblk && i < kStagesLR; blk += gridDim.x, ++i) issue(blk, i);
+  }
   float mu[CH][8], wv[CH][8], acc[CH][8];
   bool act[CH];
 #pragma unroll
@@ -52,26 +98,22 @@ __global__ void __launch_bounds__(1024) lr_pass_kernel(const PassArgs a) {
     }
   }
   const float bh = MODE >= 2 ? a.bhat[0] : 0.f;
-  float sum_r = 0.f, sum_loss = 0.f;
-  int buf = 0;
-  for (int64_t r = rb; r < re; r += RG) {
-    uint4 xv[RG][CH];
-#pragma unroll
-    for (int q = 0; q < RG; ++q)
-#pragma unroll
-      for (int c = 0; c < CH; ++c) {
-        const int ch = tid + c * blockDim.x;
-        xv[q][c] = (act[c] && r + q < re)
-                       ? __ldg(reinterpret_cast<const uint4*>(a.MM + (size_t)(r + q) * a.ld) + ch)
-                       : make_uint4(0, 0, 0, 0);
-      }
+  float sum_r = 0.f, sum_loss = 0.f;  // warp 0, lane = row within the block
+  unsigned long long cnt[5] = {0, 0, 0, 0, 0};
+  int it = 0;
+  for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++it) {
+    const int stage = it % kStagesLR;
+    mbar_wait(&full[stage], (it / kStagesLR) & 1);
+    const int64_t r = a.r0 + blk * a.rb;
+    const int nr = (int)min((int64_t)a.rb, a.r1 - r);
+    const uint32_t sbase = base + stage * stage_bytes;
     if constexpr (MODE <= 1) {
-#pragma unroll
-      for (int q = 0; q < RG; ++q) {
-        const float vq = r + q < re ? 1.f : 0.f;  // rows past the block's range must not add mu^2
+      for (int q = 0; q < nr; ++q) {
 #pragma unroll
         for (int c = 0; c < CH; ++c) {
-          const uint32_t u[4] = {xv[q][c].x, xv[q][c].y, xv[q][c].z, xv[q][c].w};
+          if (!act[c]) continue;
+          const uint4 xv = lds128(sbase + q * row_bytes + (uint32_t)(tid + c * blockDim.x) * 16u);
+          const uint32_t u[4] = {xv.x, xv.y, xv.z, xv.w};
 #pragma unroll
           for (int j = 0; j < 4; ++j) {
             const float2 f = unpack_bf16x2(u[j]);
@@ -79,7 +121,7 @@ __global__ void __launch_bounds__(1024) lr_pass_kernel(const PassArgs a) {
               acc[c][2 * j] += f.x;
               acc[c][2 * j + 1] += f.y;
             } else {
-              const float d0 = (f.x - mu[c][2 * j]) * vq, d1 = (f.y - mu[c][2 * j + 1]) * vq;
+              const float d0 = f.x - mu[c][2 * j], d1 = f.y - mu[c][2 * j + 1];
               acc[c][2 * j] = fmaf(d0, d0, acc[c][2 * j]);
               acc[c][2 * j + 1] = fmaf(d1, d1, acc[c][2 * j + 1]);
             }
@@ -87,59 +129,81 @@ __global__ void __launch_bounds__(1024) lr_pass_kernel(const PassArgs a) {
         }
       }
     } else {
-      float dot[RG];
-#pragma unroll
-      for (int q = 0; q < RG; ++q) {
-        float s = 0.f;
+      for (int q = 0; q < nr; ++q) {
+        float sdot = 0.f;
 #pragma unroll
         for (int c = 0; c < CH; ++c) {
-          const uint32_t u[4] = {xv[q][c].x, xv[q][c].y, xv[q][c].z, xv[q][c].w};
+          if (!act[c]) continue;
+          const uint4 xv = lds128(sbase + q * row_bytes + (uint32_t)(tid + c * blockDim.x) * 16u);
+          const uint32_t u[4] = {xv.x, xv.y, xv.z, xv.w};
 #pragma unroll
           for (int j = 0; j < 4; ++j) {
             const float2 f = unpack_bf16x2(u[j]);
-            s = fmaf(f.x - mu[c][2 * j], wv[c][2 * j], s);
-            s = fmaf(f.y - mu[c][2 * j + 1], wv[c][2 * j + 1], s);
+            sdot = fmaf(f.x - mu[c][2 * j], wv[c][2 * j], sdot);
+            sdot = fmaf(f.y - mu[c][2 * j + 1], wv[c][2 * j + 1], sdot);
           }
         }
 #pragma unroll
-        for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-        dot[q] = s;
-      }
-      if (lane == 0) {
-#pragma unroll
-        for (int q = 0; q < RG; ++q) red[buf][q][warp] = dot[q];
+        for (int o = 16; o > 0; o >>= 1) sdot += __shfl_xor_sync(0xffffffffu, sdot, o);
+        if (lane == 0) red[q * 32 + warp] = sdot;
       }
       __syncthreads();
-      float phi[RG];
-#pragma unroll
-      for (int q = 0; q < RG; ++q) {
+      if (warp == 0 && lane < nr) {
         float z = bh;
-        for (int w = 0; w < nwarps; ++w) z += red[buf][q][w];  // fixed order
-        const bool valid = r + q < re;
+        for (int w = 0; w < nwarps; ++w) z += red[lane * 32 + w];  // fixed order
+        const int64_t row = r + lane;
         if (MODE == 2) {
-          phi[q] = valid ? z : 0.f;
+          phis[lane] = z;
+          sum_r += z;
         } else {
-          const float yv = valid ? (float)a.y[r + q] : 0.f;
-          const float p = 1.f / (1.f + __expf(-z));
-          phi[q] = valid ? p - yv : 0.f;
-          if (valid) sum_loss += softplusf(z) - yv * z;
-        }
-        sum_r += phi[q];
-      }
-      buf ^= 1;
-#pragma unroll
-      for (int q = 0; q < RG; ++q)
-#pragma unroll
-        for (int c = 0; c < CH; ++c) {
-          const uint32_t u[4] = {xv[q][c].x, xv[q][c].y, xv[q][c].z, xv[q][c].w};
-#pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            const float2 f = unpack_bf16x2(u[j]);
-            acc[c][2 * j] = fmaf(phi[q], f.x - mu[c][2 * j], acc[c][2 * j]);
-            acc[c][2 * j + 1] = fmaf(phi[q], f.y - mu[c][2 * j + 1], acc[c][2 * j + 1]);
+          const int yv = a.y[row];
+          if (MODE == 3) {
+            const float ph = 1.f / (1.f + __expf(-z)) - (float)yv;
+            phis[lane] = ph;
+            sum_r += ph;
+            sum_loss += softplusf(z) - (float)yv * z;
+          } else {  // MODE 4: predict 1 iff z >= 0
+            const int pred = z >= 0.f ? 1 : 0;
+            if (row < a.n_train) cnt[0] += pred == yv;
+            else cnt[pred && yv ? 1 : (pred ? 2 : (yv ? 4 : 3))] += 1;
           }
         }
+      }
+      if (MODE == 2 || MODE == 3) {
+        __syncthreads();
+        for (int q = 0; q < nr; ++q) {
+          const float ph = phis[q];
+#pragma unroll
+          for (int c = 0; c < CH; ++c) {
+            if (!act[c]) continue;
+            const uint4 xv = lds128(sbase + q * row_bytes + (uint32_t)(tid + c * blockDim.x) * 16u);
+            const uint32_t u[4] = {xv.x, xv.y, xv.z, xv.w};
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              const float2 f = unpack_bf16x2(u[j]);
+              acc[c][2 * j] = fmaf(ph, f.x - mu[c][2 * j], acc[c][2 * j]);
+              acc[c][2 * j + 1] = fmaf(ph, f.y - mu[c][2 * j + 1], acc[c][2 * j + 1]);
+            }
+          }
+        }
+      }
     }
+    __syncthreads();  // every thread is done with this stage (and with red / phis)
+    if (tid == 0) {
+      const int64_t nb = blk + (int64_t)kStagesLR * gridDim.x;
+      if (nb < nblk) issue(nb, stage);
+    }
+  }
+  if constexpr (MODE == 4) {
+    if (warp == 0) {
+#pragma unroll
+      for (int k = 0; k < 5; ++k) {
+        unsigned long long v = cnt[k];
+        for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        if (lane == 0 && v) atomicAdd(&a.counts[k], v);
+      }
+    }
+    return;
   }
   float* out = a.partial + (size_t)blockIdx.x * (a.ld + 4);
 #pragma unroll
@@ -151,9 +215,15 @@ __global__ void __launch_bounds__(1024) lr_pass_kernel(const PassArgs a) {
       o[1] = make_float4(acc[c][4], acc[c][5], acc[c][6], acc[c][7]);
     }
   }
-  if (tid == 0) {
-    out[a.ld] = sum_r;        // identical in every thread (all threads saw every phi)
-    out[a.ld + 1] = sum_loss;
+  if (warp == 0) {  // fixed-order (lane) reduction of the per-row scalars
+    for (int o = 16; o > 0; o >>= 1) {
+      sum_r += __shfl_xor_sync(0xffffffffu, sum_r, o);
+      sum_loss += __shfl_xor_sync(0xffffffffu, sum_loss, o);
+    }
+    if (lane == 0) {
+      out[a.ld] = sum_r;
+      out[a.ld + 1] = sum_loss;
+    }
   }
 }
 
@@ -258,82 +328,29 @@ __global__ void grad_kernel(const double* G, int ld, int init, double lambda, do
   if (threadIdx.x == 0) bhat[0] = (float)st->b;
 }
 
-// eval (O6 step 6): counts[0] train correct, [1] tp, [2] fp, [3] tn, [4] fn (integers, exact)
-template <int CH>
-__global__ void __launch_bounds__(1024) lr_eval_kernel(const PassArgs a, int64_t n_train, unsigned long long* counts) {
-  __shared__ float red[RG][32];
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarps = blockDim.x >> 5;
-  const int64_t n = a.r1 - a.r0;
-  const int64_t rb = a.r0 + n * blockIdx.x / gridDim.x, re = a.r0 + n * (blockIdx.x + 1) / gridDim.x;
-  float mu[CH][8], wv[CH][8];
-  bool act[CH];
-#pragma unroll
-  for (int c = 0; c < CH; ++c) {
-    const int ch = tid + c * blockDim.x;
-    act[c] = ch < a.chunks;
-#pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      mu[c][j] = act[c] ? a.mu[ch * 8 + j] : 0.f;
-      wv[c][j] = act[c] ? a.what[ch * 8 + j] : 0.f;
-    }
-  }
-  const float bh = a.bhat[0];
-  unsigned long long cnt[5] = {0, 0, 0, 0, 0};
-  for (int64_t r = rb; r < re; r += RG) {
-    float dot[RG];
-#pragma unroll
-    for (int q = 0; q < RG; ++q) {
-      float s = 0.f;
-#pragma unroll
-      for (int c = 0; c < CH; ++c) {
-        const int ch = tid + c * blockDim.x;
-        if (act[c] && r + q < re) {
-          const uint4 xv = __ldg(reinterpret_cast<const uint4*>(a.MM + (size_t)(r + q) * a.ld) + ch);
-          const uint32_t u[4] = {xv.x, xv.y, xv.z, xv.w};
-#pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            const float2 f = unpack_bf16x2(u[j]);
-            s = fmaf(f.x - mu[c][2 * j], wv[c][2 * j], s);
-            s = fmaf(f.y - mu[c][2 * j + 1], wv[c][2 * j + 1], s);
-          }
-        }
-      }
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-      dot[q] = s;
-    }
-    __syncthreads();
-    if (lane == 0)
-#pragma unroll
-      for (int q = 0; q < RG; ++q) red[q][warp] = dot[q];
-    __syncthreads();
-    if (tid == 0) {
-      for (int q = 0; q < RG && r + q < re; ++q) {
-        float z = bh;
-        for (int w = 0; w < nwarps; ++w) z += red[q][w];
-        const int pred = z >= 0.f ? 1 : 0;
-        const int yv = a.y[r + q];
-        if (r + q < n_train) {
-          cnt[0] += pred == yv;
-        } else {
-          cnt[pred && yv ? 1 : (pred ? 2 : (yv ? 4 : 3))] += 1;
-        }
-      }
-    }
-  }
-  if (tid == 0)
-    for (int k = 0; k < 5; ++k)
-      if (cnt[k]) atomicAdd(&counts[k], cnt[k]);
-}
-
 // ------------------------------------------------------------------------------------------
+struct StreamCfg {
+  int threads, ch, rb, grid;
+  size_t smem;
+};
+
 template <int MODE>
-static void run_pass(const PassArgs& a0, int threads, int grid, int ch, cudaStream_t st) {
-  PassArgs a = a0;
-  switch (ch) {
-    case 1: lr_pass_kernel<1, MODE><<<grid, threads, 0, st>>>(a); break;
-    case 2: lr_pass_kernel<2, MODE><<<grid, threads, 0, st>>>(a); break;
-    case 4: lr_pass_kernel<4, MODE><<<grid, threads, 0, st>>>(a); break;
+static void run_pass(const PassArgs& a, const StreamCfg& c, cudaStream_t st) {
+  auto go = [&](void (*kern)(PassArgs)) {
+    static std::mutex mu;
+    static std::set<const void*> done;  // opt-in shared memory, once per kernel instance
+    {
+      std::lock_guard<std::mutex> lk(mu);
+      if (done.insert((const void*)kern).second)
+        VCHECK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    }
+    kern<<<c.grid, c.threads, c.smem, st>>>(a);
+  };
+  switch (c.ch) {
+    case 1: go(lr_stream_kernel<1, MODE>); break;
+    case 2: go(lr_stream_kernel<2, MODE>); break;
+    case 3: go(lr_stream_kernel<3, MODE>); break;
+    case 4: go(lr_stream_kernel<4, MODE>); break;
     default: fail(1, "lr: unsupported row width");
   }
   LAUNCHED();
@@ -345,16 +362,22 @@ LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_tr
   LRResult res;
   if (ld % 8) fail(1, "lr: ld must be a multiple of 8");
   const int chunks = ld / 8;
-  int ch = chunks <= 512 ? 1 : (chunks <= 2048 ? 2 : 4);
-  int threads = ((chunks + ch - 1) / ch + 31) / 32 * 32;
-  if (threads > 1024) fail(1, "lr: row too wide");
-  const int per_sm = std::max(1, 2048 / threads);
+  // one CTA per SM streaming row blocks of ~64 KB through a 3-deep bulk-copy ring
+  StreamCfg cfg;
+  cfg.threads = std::min(kLRThreads, (chunks + 31) / 32 * 32);
+  cfg.ch = (chunks + cfg.threads - 1) / cfg.threads;
+  if (cfg.ch > 4) fail(1, "lr: row too wide");
+  if (cfg.ch == 3 && chunks <= 2 * cfg.threads) cfg.ch = 2;
+  cfg.rb = (int)std::max<int64_t>(1, std::min<int64_t>(kMaxRB, 65536 / ((int64_t)ld * 2)));
+  const size_t stage_bytes = ((size_t)cfg.rb * ld * 2 + 127) & ~(size_t)127;
+  cfg.smem = kStagesLR * stage_bytes + kMaxRB * 32 * 4 + kMaxRB * 4 + kStagesLR * 8 + 128;
+  if (cfg.smem > 227 * 1024) fail(1, "lr: row block does not fit in shared memory");
   auto grid_for_rows = [&](int64_t rows) {
-    int64_t g = (rows + 4 * RG - 1) / (4 * RG);
-    const int64_t cap = (int64_t)num_sms() * per_sm;
-    return (int)std::max<int64_t>(1, std::min(g, cap));
+    const int64_t blocks = (rows + cfg.rb - 1) / cfg.rb;
+    return (int)std::max<int64_t>(1, std::min<int64_t>(blocks, num_sms()));
   };
-  const int grid_tr = grid_for_rows(n_train);
+  cfg.grid = grid_for_rows(n_train);
+  const int grid_tr = cfg.grid;
   const int ncols = ld + 2;
   int d_real = 0;
   for (int j = 0; j < ld; ++j) d_real += real_host[j] ? 1 : 0;
@@ -362,7 +385,7 @@ LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_tr
   // scratch
   size_t off = 0;
   auto carve = [&](size_t bytes) { size_t o = off; off += (bytes + 255) & ~(size_t)255; return o; };
-  const size_t o_part = carve((size_t)grid_tr * (ld + 4) * 4), o_G = carve(ncols * 8), o_mu = carve(ld * 8),
+  const size_t o_part = carve((size_t)std::max(grid_tr, 1) * (ld + 4) * 4), o_G = carve(ncols * 8), o_mu = carve(ld * 8),
                o_muf = carve(ld * 4), o_inv = carve(ld * 8), o_v = carve(ld * 8), o_w = carve(ld * 8),
                o_what = carve(ld * 4), o_bhat = carve(16), o_st = carve(sizeof(LRState)),
                o_real = carve(ld), o_loss = carve((size_t)(iters + 1) * 8), o_cnt = carve(64);
@@ -395,6 +418,9 @@ LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_tr
   a.what = what;
   a.bhat = bhat;
   a.partial = partial;
+  a.n_train = n_train;
+  a.rb = cfg.rb;
+  a.counts = nullptr;
   const double pass_bytes = (double)n_train * ld * 2;
   auto reduce = [&](double extra_n) {
     prof_begin(st);
@@ -409,13 +435,13 @@ LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_tr
   const int ublk = 1024;
   // ---- O6 step 2: standardisation statistics (two passes: mean, then centred squares) ----
   prof_begin(st);
-  run_pass<0>(a, threads, grid_tr, ch, st);
+  run_pass<0>(a, cfg, st);
   prof_end(st, 5, 0, pass_bytes);
   reduce((double)n_train);
   stats_finalize_kernel<<<(ld + 255) / 256, 256, 0, st>>>(G, ld, 0, real, mu, mu_f, inv, dst);
   LAUNCHED();
   prof_begin(st);
-  run_pass<1>(a, threads, grid_tr, ch, st);
+  run_pass<1>(a, cfg, st);
   prof_end(st, 5, 0, pass_bytes);
   reduce(-1);
   stats_finalize_kernel<<<(ld + 255) / 256, 256, 0, st>>>(G, ld, 1, real, mu, mu_f, inv, dst);
@@ -425,7 +451,7 @@ LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_tr
   LAUNCHED();
   for (int k = 0; k < power_iters; ++k) {
     prof_begin(st);
-    run_pass<2>(a, threads, grid_tr, ch, st);
+    run_pass<2>(a, cfg, st);
     prof_end(st, 5, 0, pass_bytes);
     reduce(-1);
     power_kernel<<<1, ublk, 0, st>>>(G, ld, 0, d_real, real, inv, v, what, bhat, dst);
@@ -436,7 +462,7 @@ LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_tr
   LAUNCHED();
   for (int t = 0; t < iters; ++t) {
     prof_begin(st);
-    run_pass<3>(a, threads, grid_tr, ch, st);
+    run_pass<3>(a, cfg, st);
     prof_end(st, 5, 0, pass_bytes);
     reduce(-1);
     grad_kernel<<<1, ublk, 0, st>>>(G, ld, 0, lambda, alpha, inv, w, what, bhat, dst, loss + t);
@@ -447,16 +473,11 @@ LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_tr
     PassArgs e = a;
     e.r0 = 0;
     e.r1 = n_rows;
-    const int ge = grid_for_rows(n_rows);
+    e.counts = cnt;
+    StreamCfg ce = cfg;
+    ce.grid = grid_for_rows(n_rows);
     prof_begin(st);
-    if (n_rows > 0) {
-      switch (ch) {
-        case 1: lr_eval_kernel<1><<<ge, threads, 0, st>>>(e, n_train, cnt); break;
-        case 2: lr_eval_kernel<2><<<ge, threads, 0, st>>>(e, n_train, cnt); break;
-        default: lr_eval_kernel<4><<<ge, threads, 0, st>>>(e, n_train, cnt); break;
-      }
-      LAUNCHED();
-    }
+    if (n_rows > 0) run_pass<4>(e, ce, st);
     prof_end(st, 5, 0, (double)n_rows * ld * 2);
   }
   // counts -> fp64 for the allreduce (exact below 2^53)

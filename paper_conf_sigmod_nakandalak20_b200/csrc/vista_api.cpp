@@ -6,6 +6,8 @@
 #include <algorithm>
 #include <atomic>
 #include <cmath>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <memory>
 #include <string>
@@ -45,7 +47,9 @@ struct Profiler {
     cudaEvent_t a, b;
     int cls;
     double flops, bytes;
+    std::string label;
   };
+  FILE* log = nullptr;
   std::vector<Rec> recs;
   std::vector<cudaEvent_t> pool;
   cudaEvent_t pending = nullptr;
@@ -69,12 +73,19 @@ struct Profiler {
       acc.launches[r.cls] += 1;
       acc.flops[r.cls] += r.flops;
       acc.bytes[r.cls] += r.bytes;
+      if (log) fprintf(log, "%d\t%.6f\t%.6g\t%.6g\t%s\n", r.cls, ms, r.flops, r.bytes, r.label.c_str());
       pool.push_back(r.a);
       pool.push_back(r.b);
     }
     recs.clear();
+    if (log) fflush(log);
+  }
+  Profiler() {
+    const char* path = getenv("VISTA_PROF_LOG");
+    if (path && *path) log = fopen(path, "a");
   }
   ~Profiler() {
+    if (log) fclose(log);
     for (auto& r : recs) {
       cudaEventDestroy(r.a);
       cudaEventDestroy(r.b);
@@ -88,11 +99,12 @@ void prof_begin(cudaStream_t st) {
   g_prof->pending = g_prof->get();
   VCHECK(cudaEventRecord(g_prof->pending, st));
 }
-void prof_end(cudaStream_t st, int cls, double flops, double bytes) {
+bool prof_labels() { return g_prof && g_prof->log; }
+void prof_end(cudaStream_t st, int cls, double flops, double bytes, const char* label) {
   if (!g_prof || !g_prof->pending) return;
   cudaEvent_t b = g_prof->get();
   VCHECK(cudaEventRecord(b, st));
-  g_prof->recs.push_back({g_prof->pending, b, cls, flops, bytes});
+  g_prof->recs.push_back({g_prof->pending, b, cls, flops, bytes, label ? std::string(label) : std::string()});
   g_prof->pending = nullptr;
   if (g_prof->recs.size() > 4096) g_prof->flush();
 }

@@ -39,6 +39,10 @@ CONV = [
     (3, 1, 1, 1152, 1000, 1, 1, 0, 1, False, False),   # FC, N = 1000 (partial last N tile), M = 3
     (2, 7, 7, 128, 512, 3, 2, 1, 1, True, False),      # strided 3x3, residual without ReLU
     (130, 1, 1, 64, 128, 1, 1, 0, 1, False, True),     # FC with M = 130 (two M tiles)
+    (2, 17, 17, 8, 64, 3, 1, 1, 1, False, True),       # VGG conv1_1-style, row-gather mode
+    (1, 9, 9, 96, 96, 3, 1, 1, 2, True, True),         # Cg_out = 48: masked group tile, register epilogue
+    (2, 15, 15, 64, 256, 1, 1, 0, 1, True, True),      # TMA A + TMA epilogue, M tail (450 rows), residual
+    (3, 1, 1, 2048, 1000, 1, 1, 0, 1, True, False),    # FC 1000 with BN = 256 partial tile + residual
 ]
 
 

@@ -200,6 +200,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--images", type=int, default=0, help="override images per GPU (debug only)")
+    ap.add_argument("--micro-batch", type=int, default=0, help="stage-1 micro-batch (0 = planner)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -244,7 +245,7 @@ def main():
     stream = torch.cuda.current_stream(dev)
     v = Vista(cnn, layers=taps, n_str_rows=len(tab.str_keys), d_s=d_s, n_images_local=n_img, iters=T,
               power_iters=20, split_seed=5, weight_seed=1, rank=rank, world=world, nccl_uid=uid, device=local,
-              stream=stream.cuda_stream)
+              stream=stream.cuda_stream, micro_batch=args.micro_batch)
     info = v.plan_info()
     d_tot = [d_s + d for d in info["d_l"]]
 

@@ -28,7 +28,7 @@
 
 namespace vista {
 
-enum AMode { A_GATHER_FAST = 0, A_GATHER_GENERAL = 1, A_TMA = 2, A_GATHER_ROW = 3 };
+enum AMode { A_GATHER_FAST = 0, A_GATHER_GENERAL = 1, A_TMA = 2, A_GATHER_ROW = 3, A_IM2COL = 4 };
 
 struct ConvParams {
   const bf16* x;
@@ -118,7 +118,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int i = 0; i < S; ++i) {
-      mbar_init(&full[i], AMODE == A_TMA ? 1 : 128 + 1);
+      mbar_init(&full[i], (AMODE == A_TMA || AMODE == A_IM2COL) ? 1 : 128 + 1);
       mbar_init(&empty[i], 1);
     }
     for (int i = 0; i < 2; ++i) {
@@ -128,7 +128,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     mbar_init(rbar, 1);
     fence_mbar_init();
     tma_prefetch(&tmap_w);
-    if (AMODE == A_TMA) tma_prefetch(&tmap_a);
+    if (AMODE == A_TMA || AMODE == A_IM2COL) tma_prefetch(&tmap_a);
     if (TMA_EPI) tma_prefetch(&tmap_y);
   }
   if (warp == 4) tmem_alloc(tmem_slot, C::kTmemCols);
@@ -152,6 +152,38 @@ __global__ void __launch_bounds__(kThreads, 1)
             mbar_arrive_expect_tx(&full[stage], C::kABytes + C::kBBytes);
             tma_load_2d(sA + stage * C::kABytes, &tmap_a, g * p.Cg_in + kb * BK, m0, &full[stage]);
             tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
+          }
+        }
+      }
+    } else if constexpr (AMODE == A_IM2COL) {
+      // one TMA per k-block gathers 128 output pixels x 64 channels of filter tap (r, s):
+      // k-block kb -> (r, s, channel block) with k = (r*S + s)*Cg_in + c
+      if (threadIdx.x == 0) {
+        const int cblocks = p.Cg_in / BK;
+        const int hw = p.Ho * p.Wo;
+        uint32_t gk = 0;
+        for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x) {
+          int m0, nt, g;
+          decode_tile(p, tile, m0, nt, g);
+          const int n0 = nt * BN;
+          const int nimg = m0 / hw, rem = m0 - nimg * hw;
+          const int ho = rem / p.Wo, wo = rem - ho * p.Wo;
+          const int w0 = wo * p.stride - p.pad, h0 = ho * p.stride - p.pad;
+          int r = 0, s = 0, cb = 0;
+          for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
+            const int stage = gk % S;
+            if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
+            mbar_arrive_expect_tx(&full[stage], C::kABytes + C::kBBytes);
+            tma_load_im2col_4d(sA + stage * C::kABytes, &tmap_a, g * p.Cg_in + cb * BK, w0, h0, nimg, (uint16_t)s,
+                               (uint16_t)r, &full[stage]);
+            tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
+            if (++cb == cblocks) {
+              cb = 0;
+              if (++s == p.S) {
+                s = 0;
+                ++r;
+              }
+            }
           }
         }
       }
@@ -404,6 +436,51 @@ static void make_tmap(CUtensorMap* m, const void* ptr, uint64_t cols, uint64_t r
   if (rc != CUDA_SUCCESS) fail(5, "cuTensorMapEncodeTiled failed");
 }
 
+typedef CUresult (*encode_im2col_fn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                     const cuuint64_t*, const int*, const int*, cuuint32_t, cuuint32_t,
+                                     const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                     CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+static encode_im2col_fn get_encode_im2col() {
+  static encode_im2col_fn fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeIm2col", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<encode_im2col_fn>(p);
+  });
+  if (!fn) fail(5, "cuTensorMapEncodeIm2col unavailable");
+  return fn;
+}
+
+// im2col tensor map over an NHWC bf16 activation for a conv with filter R x S, stride, zero pad:
+// the box is 128 output pixels (W fastest, then H, then N) x 64 channels, 128B-swizzled.
+// Lower corner = -pad, upper corner = pad - (filter - 1) (output extent (W + 2 pad - S) / stride + 1).
+static void make_tmap_im2col(CUtensorMap* m, const void* x, int N, int H, int W, int C, int R, int S, int stride,
+                             int pad) {
+  cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
+  cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)W * C * 2, (cuuint64_t)H * W * C * 2};
+  int lower[2] = {-pad, -pad};
+  int upper[2] = {pad - (S - 1), pad - (R - 1)};
+  cuuint32_t estr[4] = {1, (cuuint32_t)stride, (cuuint32_t)stride, 1};
+  CUresult rc = get_encode_im2col()(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(x), dims, strides,
+                                    lower, upper, BK, BM, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                                    CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (rc != CUDA_SUCCESS) fail(5, "cuTensorMapEncodeIm2col failed");
+  // same driver workaround as CUTLASS (cute copy_traits_sm90_im2col.hpp) for small tensors
+  int drv = 0;
+  cudaDriverGetVersion(&drv);
+  if (drv <= 13010 && (uint64_t)N * H * W * C * 2 < 131072ull) reinterpret_cast<uint64_t*>(m)[1] &= ~(1ull << 21);
+}
+
+// VISTA_IM2COL=0 falls back to the cp.async gather (A/B comparisons)
+static const bool g_im2col_enabled = [] {
+  const char* e = getenv("VISTA_IM2COL");
+  return !(e && e[0] == '0');
+}();
+
 static int pick_bn(int Cg_out, int groups) {
   if (Cg_out % 256 == 0) return 256;
   if (Cg_out % 128 == 0) return 128;
@@ -472,6 +549,7 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
     case A_TMA: launch_t<BN, A_TMA, TE>(L, ta, ty, tr, p, st); break;
     case A_GATHER_FAST: launch_t<BN, A_GATHER_FAST, TE>(L, ta, ty, tr, p, st); break;
     case A_GATHER_ROW: launch_t<BN, A_GATHER_ROW, TE>(L, ta, ty, tr, p, st); break;
+    case A_IM2COL: launch_t<BN, A_IM2COL, TE>(L, ta, ty, tr, p, st); break;
     default: launch_t<BN, A_GATHER_GENERAL, TE>(L, ta, ty, tr, p, st); break;
   }
 }
@@ -518,6 +596,11 @@ void conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   } else {
     amode = L.row_mode ? A_GATHER_ROW : ((L.Cg_in % BK) == 0 ? A_GATHER_FAST : A_GATHER_GENERAL);
     ta = L.tmap_w;  // unused
+    // channel blocks of 64 per filter tap: the TMA unit gathers the implicit im2col rows
+    if (amode == A_GATHER_FAST && g_im2col_enabled) {
+      amode = A_IM2COL;
+      make_tmap_im2col(&ta, x, N, H, W, L.Cin, L.R, L.S, L.stride, L.pad);
+    }
   }
   // epilogue: staged in smem and written by TMA (residual read by TMA) unless a group's last N tile
   // would spill into the next group's channels

@@ -294,7 +294,9 @@ void plan_memory(vista_ctx* c, uint64_t budget) {
     if (c->sys.micro_batch > 0 && t == 0) {
       B = c->sys.micro_batch;
     } else {
-      const int64_t cap_B = t == 0 ? 256 : 16384;
+      // larger micro-batches give larger GEMMs per launch (measured: 256 -> 1024 is +7 % img/s);
+      // activations of one micro-batch exceed L2 either way
+      const int64_t cap_B = t == 0 ? 1024 : 16384;
       for (int64_t b = std::min<int64_t>(cap_B, std::max<int64_t>(c->n_img, 1)); b >= 1; b = b > 8 ? b / 2 : b - 1) {
         if ((uint64_t)(fixed + b * slot_per_img) <= budget) {
           B = (int)b;

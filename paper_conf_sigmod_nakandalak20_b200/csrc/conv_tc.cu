@@ -28,7 +28,7 @@
 
 namespace vista {
 
-enum AMode { A_GATHER_FAST = 0, A_GATHER_GENERAL = 1, A_TMA = 2, A_GATHER_ROW = 3, A_IM2COL = 4 };
+enum AMode { A_GATHER_FAST = 0, A_GATHER_GENERAL = 1, A_TMA = 2, A_GATHER_ROW = 3, A_IM2COL = 4, A_IM2COL_C8 = 5 };
 
 struct ConvParams {
   const bf16* x;
@@ -53,10 +53,11 @@ struct Cfg {
   static constexpr int kABytes = BM * BK * 2;  // 16 KB
   static constexpr int kBBytes = BN * BK * 2;
   static constexpr int kOutOff = kStages * (kABytes + kBBytes);
-  static constexpr int kOutBytes = TMA_EPI ? BM * BN * 2 : 0;
+  static constexpr int kOutBufs = (TMA_EPI && BN <= 128) ? 2 : 1;  // double-buffered staging when it fits
+  static constexpr int kOutBytes = TMA_EPI ? kOutBufs * BM * BN * 2 : 0;
   static constexpr int kSbufOff = kOutOff + kOutBytes;
   static constexpr int kBarOff = kSbufOff + 2 * 2 * BN * 4;
-  static constexpr int kBytes = kBarOff + (2 * kStages + 5) * 8 + 16 + 1024;  // + alignment slack
+  static constexpr int kBytes = kBarOff + (2 * kStages + 6) * 8 + 16 + 1024;  // + alignment slack
   static constexpr int kTmemCols = 2 * BN;
 };
 
@@ -112,23 +113,24 @@ __global__ void __launch_bounds__(kThreads, 1)
   uint64_t* empty = full + S;
   uint64_t* tfull = empty + S;   // [2]
   uint64_t* tempty = tfull + 2;  // [2]
-  uint64_t* rbar = tempty + 2;   // residual tile landed (TMA epilogue)
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rbar + 1);
+  uint64_t* rbar = tempty + 2;   // [2] residual tile landed in staging buffer b (TMA epilogue)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rbar + 2);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int i = 0; i < S; ++i) {
-      mbar_init(&full[i], (AMODE == A_TMA || AMODE == A_IM2COL) ? 1 : 128 + 1);
+      mbar_init(&full[i], (AMODE == A_TMA || AMODE == A_IM2COL || AMODE == A_IM2COL_C8) ? 1 : 128 + 1);
       mbar_init(&empty[i], 1);
     }
     for (int i = 0; i < 2; ++i) {
       mbar_init(&tfull[i], 1);
       mbar_init(&tempty[i], 4);
     }
-    mbar_init(rbar, 1);
+    mbar_init(&rbar[0], 1);
+    mbar_init(&rbar[1], 1);
     fence_mbar_init();
     tma_prefetch(&tmap_w);
-    if (AMODE == A_TMA || AMODE == A_IM2COL) tma_prefetch(&tmap_a);
+    if (AMODE == A_TMA || AMODE == A_IM2COL || AMODE == A_IM2COL_C8) tma_prefetch(&tmap_a);
     if (TMA_EPI) tma_prefetch(&tmap_y);
   }
   if (warp == 4) tmem_alloc(tmem_slot, C::kTmemCols);
@@ -151,6 +153,37 @@ __global__ void __launch_bounds__(kThreads, 1)
             if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
             mbar_arrive_expect_tx(&full[stage], C::kABytes + C::kBBytes);
             tma_load_2d(sA + stage * C::kABytes, &tmap_a, g * p.Cg_in + kb * BK, m0, &full[stage]);
+            tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
+          }
+        }
+      }
+    } else if constexpr (AMODE == A_IM2COL_C8) {
+      // first layers (input padded to 8 channels): every filter tap is one 16-byte K-slice; eight TMA
+      // im2col loads of 128 pixels x 8 channels fill a k-block laid out as 8 no-swizzle core-matrix
+      // columns (LBO 2 KB).  Taps past R*S repeat a valid tap against zero weights.
+      if (threadIdx.x == 0) {
+        const int hw = p.Ho * p.Wo;
+        const int RS = p.R * p.S;
+        uint32_t gk = 0;
+        for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x) {
+          int m0, nt, g;
+          decode_tile(p, tile, m0, nt, g);
+          const int n0 = nt * BN;
+          const int nimg = m0 / hw, rem = m0 - nimg * hw;
+          const int ho = rem / p.Wo, wo = rem - ho * p.Wo;
+          const int w0 = wo * p.stride - p.pad, h0 = ho * p.stride - p.pad;
+          for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
+            const int stage = gk % S;
+            if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
+            mbar_arrive_expect_tx(&full[stage], C::kABytes + C::kBBytes);
+#pragma unroll 1
+            for (int j = 0; j < 8; ++j) {
+              int t = kb * 8 + j;
+              if (t >= RS) t -= RS;
+              const int r = t / p.S, s = t - (t / p.S) * p.S;
+              tma_load_im2col_4d(sA + stage * C::kABytes + j * 2048, &tmap_a, 0, w0, h0, nimg, (uint16_t)s,
+                                 (uint16_t)r, &full[stage]);
+            }
             tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
           }
         }
@@ -292,7 +325,10 @@ __global__ void __launch_bounds__(kThreads, 1)
           const uint32_t a0 = sA + stage * C::kABytes, b0 = sB + stage * C::kBBytes;
 #pragma unroll
           for (int k = 0; k < BK / 16; ++k)
-            tc_mma_bf16(tacc, umma_desc_k_sw128(a0 + k * 32), umma_desc_k_sw128(b0 + k * 32), idesc,
+            tc_mma_bf16(tacc,
+                        AMODE == A_IM2COL_C8 ? umma_desc_k_none(a0 + k * 4096, 2048, 128)
+                                             : umma_desc_k_sw128(a0 + k * 32),
+                        umma_desc_k_sw128(b0 + k * 32), idesc,
                         (kb | k) != 0 ? 1u : 0u);
           tc_commit(&empty[stage]);
         }
@@ -314,13 +350,34 @@ __global__ void __launch_bounds__(kThreads, 1)
       const int n0 = nt * BN;
       const int ng0 = g * p.Cg_out + n0;
       const int nvalid_tile = min(BN, p.Cg_out - n0);
+      constexpr int NB = C::kOutBufs;
+      const uint32_t ob = NB == 2 ? (it & 1) : 0;
+      const uint32_t sOb = sO + ob * (uint32_t)(BM * BN * 2);
       if constexpr (TMA_EPI) {
+        // residual tile -> staging buffer b (TMA, 64-column 128B-swizzled sub-tiles)
+        auto issue_res = [&](int t, uint32_t b) {
+          int tm0, tnt, tg;
+          decode_tile(p, t, tm0, tnt, tg);
+          const int tn0 = tnt * BN, tng0 = tg * p.Cg_out + tn0;
+          const int nsub = (min(BN, p.Cg_out - tn0) + 63) / 64;
+          mbar_arrive_expect_tx(&rbar[b], nsub * BM * 128);
+          for (int st = 0; st < nsub; ++st)
+            tma_load_2d(sO + b * (uint32_t)(BM * BN * 2) + st * BM * 128, &tmap_r, tng0 + st * 64, tm0, &rbar[b]);
+        };
         if (et == 0) {
-          bulk_wait_read0();  // the previous tile's stores no longer read the staging buffer
-          if (has_res) {
-            const int nsub = (nvalid_tile + 63) / 64;
-            mbar_arrive_expect_tx(rbar, nsub * BM * 128);
-            for (int st = 0; st < nsub; ++st) tma_load_2d(sO + st * BM * 128, &tmap_r, ng0 + st * 64, m0, rbar);
+          if (NB == 1) {
+            bulk_wait_read0();  // the previous tile's stores no longer read the staging buffer
+            if (has_res) issue_res(tile, 0);
+          } else if (has_res) {
+            if (it == 0) issue_res(tile, 0);
+            // prefetch the next tile's residual into the other buffer once its stores (tile it-1) read it
+            const int next = tile + gridDim.x;
+            if (next < p.n_tiles) {
+              bulk_wait_read0();
+              issue_res(next, ob ^ 1);
+            }
+          } else {
+            bulk_wait_read<1>();  // tile it-2 (same buffer) has been read by its stores
           }
         }
       }
@@ -336,7 +393,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       const size_t off = (size_t)(rvalid ? mo : 0) * p.Cout + ng0;
       uint4 rres[4] = {};
       if constexpr (TMA_EPI) {
-        if (has_res) mbar_wait(rbar, it & 1);
+        if (has_res) mbar_wait(&rbar[ob], (NB == 2 ? (it >> 1) : it) & 1);
       } else if (has_res && rvalid) {
 #pragma unroll
         for (int j = 0; j < 4; ++j)
@@ -355,7 +412,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         const float* shv = ss + BN + cb * 32;
         if constexpr (TMA_EPI) {
           tc_wait_ld();
-          const uint32_t sub = sO + (cb >> 1) * BM * 128 + row * 128;
+          const uint32_t sub = sOb + (cb >> 1) * BM * 128 + row * 128;
 #pragma unroll
           for (int qq = 0; qq < 4; ++qq) {
             const uint32_t addr = sub + (((uint32_t)((cb & 1) * 4 + qq) ^ (uint32_t)(row & 7)) << 4);
@@ -397,7 +454,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         named_bar_sync(1, 128);
         if (et == 0) {
           const int nsub = (nvalid_tile + 63) / 64;
-          for (int st = 0; st < nsub; ++st) tma_store_2d(&tmap_y, ng0 + st * 64, m0, sO + st * BM * 128);
+          for (int st = 0; st < nsub; ++st) tma_store_2d(&tmap_y, ng0 + st * 64, m0, sOb + st * BM * 128);
           bulk_commit();
         }
       }
@@ -458,15 +515,17 @@ static encode_im2col_fn get_encode_im2col() {
 // the box is 128 output pixels (W fastest, then H, then N) x 64 channels, 128B-swizzled.
 // Lower corner = -pad, upper corner = pad - (filter - 1) (output extent (W + 2 pad - S) / stride + 1).
 static void make_tmap_im2col(CUtensorMap* m, const void* x, int N, int H, int W, int C, int R, int S, int stride,
-                             int pad) {
+                             int pad, int channels_per_pixel, bool swizzle128) {
   cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
   cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)W * C * 2, (cuuint64_t)H * W * C * 2};
   int lower[2] = {-pad, -pad};
   int upper[2] = {pad - (S - 1), pad - (R - 1)};
   cuuint32_t estr[4] = {1, (cuuint32_t)stride, (cuuint32_t)stride, 1};
   CUresult rc = get_encode_im2col()(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(x), dims, strides,
-                                    lower, upper, BK, BM, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                                    CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                    lower, upper, (cuuint32_t)channels_per_pixel, BM, estr,
+                                    CU_TENSOR_MAP_INTERLEAVE_NONE,
+                                    swizzle128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE,
+                                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (rc != CUDA_SUCCESS) fail(5, "cuTensorMapEncodeIm2col failed");
   // same driver workaround as CUTLASS (cute copy_traits_sm90_im2col.hpp) for small tensors
@@ -481,7 +540,9 @@ static const bool g_im2col_enabled = [] {
   return !(e && e[0] == '0');
 }();
 
-static int pick_bn(int Cg_out, int groups) {
+static int pick_bn(int Cg_out, int groups, int K) {
+  // short-K layers are epilogue/HBM-bound: 128-wide tiles get a double-buffered output staging
+  if (K <= 256 && Cg_out % 128 == 0) return 128;
   if (Cg_out % 256 == 0) return 256;
   if (Cg_out % 128 == 0) return 128;
   if (Cg_out % 64 == 0) return 64;
@@ -498,9 +559,10 @@ void conv_layer_init(ConvLayer& L, const std::vector<uint16_t>& w, int Cin_real,
   const int cg_real = Cin_real / L.groups;
   L.K = L.R * L.S * L.Cg_in;
   // first layers (input padded to 8 channels, filters at most 8 wide): one k-block per filter row
+  // (measured: for ResNet conv1 the row gather beats eight 2 KB im2col TMAs per k-block, 60 vs 103 ms)
   L.row_mode = L.groups == 1 && L.Cg_in == 8 && L.S <= 8 && L.R * 64 <= ((L.K + BK - 1) / BK * BK) * 2;
   L.Kp = L.row_mode ? L.R * BK : (L.K + BK - 1) / BK * BK;
-  L.BN = pick_bn(L.Cg_out, L.groups);
+  L.BN = pick_bn(L.Cg_out, L.groups, L.K);
   // repack OHWI [Cout][R][S][cg_real] -> [Cout][Kp] with channel padding cg_real -> Cg_in and K padding
   std::vector<uint16_t> packed((size_t)L.Cout * L.Kp, 0);
   for (int o = 0; o < L.Cout; ++o)
@@ -550,6 +612,7 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
     case A_GATHER_FAST: launch_t<BN, A_GATHER_FAST, TE>(L, ta, ty, tr, p, st); break;
     case A_GATHER_ROW: launch_t<BN, A_GATHER_ROW, TE>(L, ta, ty, tr, p, st); break;
     case A_IM2COL: launch_t<BN, A_IM2COL, TE>(L, ta, ty, tr, p, st); break;
+    case A_IM2COL_C8: launch_t<BN, A_IM2COL_C8, TE>(L, ta, ty, tr, p, st); break;
     default: launch_t<BN, A_GATHER_GENERAL, TE>(L, ta, ty, tr, p, st); break;
   }
 }
@@ -599,7 +662,10 @@ void conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
     // channel blocks of 64 per filter tap: the TMA unit gathers the implicit im2col rows
     if (amode == A_GATHER_FAST && g_im2col_enabled) {
       amode = A_IM2COL;
-      make_tmap_im2col(&ta, x, N, H, W, L.Cin, L.R, L.S, L.stride, L.pad);
+      make_tmap_im2col(&ta, x, N, H, W, L.Cin, L.R, L.S, L.stride, L.pad, BK, true);
+    } else if (g_im2col_enabled && !L.row_mode && L.groups == 1 && L.Cg_in == 8) {
+      amode = A_IM2COL_C8;
+      make_tmap_im2col(&ta, x, N, H, W, L.Cin, L.R, L.S, L.stride, L.pad, 8, false);
     }
   }
   // epilogue: staged in smem and written by TMA (residual read by TMA) unless a group's last N tile

@@ -41,6 +41,9 @@ struct ConvLayer {
   int Cg_in = 0, Cg_out = 0, K = 0, Kp = 0, BN = 128;
   bool relu = false;
   bool row_mode = false;     // Cin = 8, S <= 8: one k-block per filter row, k = r*64 + s*8 + c
+  bool rowview = false;      // stride-1 unpadded conv with S*Cin == 64: one output row per 128-row tile,
+                             // A rows = overlapping 128-byte windows of one input row (tiled TMA)
+  int K_alg = 0;             // algorithmic reduction length R*S*Cin_real/groups (FLOP accounting)
   bf16* w = nullptr;         // [Cout][Kp]
   float* scale = nullptr;    // [Cout]
   float* shift = nullptr;    // [Cout]
@@ -59,6 +62,7 @@ inline int conv_out_dim(int H, int k, int s, int p) { return (H + 2 * p - k) / s
 
 // ---- SIMT kernels (memory-bound) ----
 void launch_ingest(const uint8_t* px, int64_t n, bf16* y, cudaStream_t st);
+void launch_ingest_s2d(const uint8_t* px, int64_t n, bf16* y, cudaStream_t st);
 void launch_maxpool(const bf16* x, int N, int H, int W, int C, int k, int s, bf16* y, cudaStream_t st);
 void launch_lrn(const bf16* x, int N, int H, int W, int C, bf16* y, cudaStream_t st);
 void launch_avgpool(const bf16* x, int N, int H, int W, int C, bf16* y, cudaStream_t st);

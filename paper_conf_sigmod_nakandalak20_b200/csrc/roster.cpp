@@ -76,6 +76,18 @@ struct Builder {
     cur.ops.push_back(OpDesc{OP_INGEST, BUF_IN, out, -1, -1, 0, 0, 227, 227, 3, 227, 227, 8});
     set_out(out, Shape{227, 227, 8});
   }
+  // ResNet conv1 = 7x7/2 pad 3 on the raw image, executed as 4x4/1 on the space-to-depth input
+  void ingest_s2d_conv1(int tmp, int out, int Cout) {
+    cur.ops.push_back(OpDesc{OP_INGEST_S2D, BUF_IN, tmp, -1, -1, 0, 0, 227, 227, 3, kS2dHW, kS2dHW, kS2dC});
+    set_out(tmp, Shape{kS2dHW, kS2dHW, kS2dC});
+    const int id = layer(3, 3, Cout, 7, 7, 2, 3, 1, false, 1, true);
+    net.layers[id].s2d = true;
+    const int Ho = conv_out_dim(227, 7, 2, 3);  // 114 = 117 - 4 + 1
+    OpDesc op{OP_CONV, tmp, out, -1, id, 0, 0, kS2dHW, kS2dHW, kS2dC, Ho, Ho, Cout};
+    cur.macs += (double)Ho * Ho * Cout * 7 * 7 * 3;
+    cur.ops.push_back(op);
+    set_out(out, Shape{Ho, Ho, Cout});
+  }
   void end_stage() {
     Shape o = shp[BUF_OUT];
     cur.outH = o.H;
@@ -172,8 +184,7 @@ NetDesc build_roster(int cnn) {
     b.end_stage();
   } else {  // ResNet50 v1 [37] (reading R4): pool1 unpadded, stride on the first 1x1
     b.begin_stage(px, px_elems);
-    b.ingest(T0);
-    b.conv(T0, T1, -1, 64, 7, 2, 3, 1, false, 1, true, 3);
+    b.ingest_s2d_conv1(T0, T1, 64);
     b.pool(T1, T2, 3, 2);
     int cur = T2;
     const int mids[3] = {64, 128, 256}, units[3] = {3, 4, 6};

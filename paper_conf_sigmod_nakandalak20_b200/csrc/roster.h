@@ -10,7 +10,12 @@
 
 namespace vista {
 
-enum OpKind { OP_INGEST = 0, OP_CONV = 1, OP_MAXPOOL = 2, OP_LRN = 3, OP_AVGPOOL = 4 };
+enum OpKind { OP_INGEST = 0, OP_CONV = 1, OP_MAXPOOL = 2, OP_LRN = 3, OP_AVGPOOL = 4, OP_INGEST_S2D = 5 };
+
+// ResNet50 conv1 (7x7 stride 2 pad 3 on 3 channels) runs as a 4x4 stride-1 conv on a 2x2
+// space-to-depth input: [117, 117, 16] with channel c' = (dy*2 + dx)*3 + ch (12..15 zero) holding
+// pixel (2*h2 + dy - 3, 2*w2 + dx - 3); the filter tap (r, s) = (2a + dy, 2b + dx), r, s < 7.
+constexpr int kS2dHW = 117, kS2dC = 16;
 enum BufId { BUF_IN = 0, BUF_OUT = 1, BUF_T0 = 2, NUM_BUFS = 7 };  // T0..T4 = scratch slots 2..6
 
 struct LayerSpec {  // one parameterised layer (conv or fc); id = generator layer id
@@ -19,6 +24,7 @@ struct LayerSpec {  // one parameterised layer (conv or fc); id = generator laye
   bool bias;      // conv/fc bias (AlexNet, VGG16, ResNet fc)
   int bn_kind;    // 0 none, 1 BN, 2 BN closing a residual branch / projection
   bool relu;      // ReLU in the epilogue
+  bool s2d = false;  // executed on the space-to-depth input (see kS2dHW)
 };
 
 struct OpDesc {

@@ -49,6 +49,51 @@ void launch_ingest(const uint8_t* px, int64_t n, bf16* y, cudaStream_t st) {
   prof_end(st, 2, 0, (double)npix * (3 + 16));
 }
 
+// ---- S0 for ResNet conv1: uint8 NHWC3 -> zero-padded 2x2 space-to-depth bf16 [n, 117, 117, 16] ----
+// channel c' = (dy*2 + dx)*3 + ch (c' >= 12 zero) of position (h2, w2) holds (p - 128)/128 of pixel
+// (2*h2 + dy - 3, 2*w2 + dx - 3), 0 outside the image (the conv's zero padding of 3).
+__global__ void ingest_s2d_kernel(const uint8_t* __restrict__ px, int64_t n, bf16* __restrict__ y) {
+  const int64_t total = n * 117 * 117;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int w2 = (int)(i % 117);
+    const int64_t t = i / 117;
+    const int h2 = (int)(t % 117);
+    const int64_t img = t / 117;
+    const uint8_t* src = px + img * (227 * 227 * 3);
+    float f[16];
+#pragma unroll
+    for (int c = 0; c < 16; ++c) f[c] = 0.f;
+#pragma unroll
+    for (int d = 0; d < 4; ++d) {
+      const int h = 2 * h2 + (d >> 1) - 3, w = 2 * w2 + (d & 1) - 3;
+      if (h >= 0 && h < 227 && w >= 0 && w < 227) {
+        const uint8_t* q = src + (h * 227 + w) * 3;
+#pragma unroll
+        for (int c = 0; c < 3; ++c) f[d * 3 + c] = ((float)q[c] - 128.0f) * (1.0f / 128.0f);
+      }
+    }
+    uint4 a, b;
+    a.x = pack_bf16x2(f[0], f[1]);
+    a.y = pack_bf16x2(f[2], f[3]);
+    a.z = pack_bf16x2(f[4], f[5]);
+    a.w = pack_bf16x2(f[6], f[7]);
+    b.x = pack_bf16x2(f[8], f[9]);
+    b.y = pack_bf16x2(f[10], f[11]);
+    b.z = 0u;
+    b.w = 0u;
+    uint4* dst = reinterpret_cast<uint4*>(y + i * 16);
+    dst[0] = a;
+    dst[1] = b;
+  }
+}
+void launch_ingest_s2d(const uint8_t* px, int64_t n, bf16* y, cudaStream_t st) {
+  const int64_t total = n * 117 * 117;
+  prof_begin(st);
+  ingest_s2d_kernel<<<grid_for(total, 256), 256, 0, st>>>(px, n, y);
+  LAUNCHED();
+  prof_end(st, 2, 0, (double)n * 227 * 227 * 3 + (double)total * 32);
+}
+
 // ---- unpadded max pool (k, s) ----
 __global__ void maxpool_kernel(const bf16* __restrict__ x, int N, int H, int W, int C, int k, int s, int Ho, int Wo,
                                bf16* __restrict__ y) {

@@ -351,7 +351,29 @@ void upload_weights(vista_ctx* c, uint64_t seed) {
         shift[o] = (float)(be[o] - mu[o] * sc);
       }
     }
-    conv_layer_init(L, wb, s.Cin_real, scale, shift);
+    if (s.s2d) {
+      // 7x7/2 pad 3 on 3 channels == 4x4/1 on the 2x2 space-to-depth input (roster.h kS2dHW):
+      // W2[o][a][b][(dy*2 + dx)*3 + ch] = W[o][2a + dy][2b + dx][ch] for 2a + dy, 2b + dx < 7, else 0
+      const int R2 = (s.R + 1) / 2, S2 = (s.S + 1) / 2;
+      std::vector<uint16_t> w2((size_t)s.Cout * R2 * S2 * kS2dC, 0);
+      for (int o = 0; o < s.Cout; ++o)
+        for (int r = 0; r < s.R; ++r)
+          for (int q = 0; q < s.S; ++q)
+            for (int ch = 0; ch < s.Cin_real; ++ch) {
+              const int a = r / 2, dy = r % 2, b = q / 2, dx = q % 2;
+              w2[(((size_t)o * R2 + a) * S2 + b) * kS2dC + (dy * 2 + dx) * 3 + ch] =
+                  wb[(((size_t)o * s.R + r) * s.S + q) * s.Cin_real + ch];
+            }
+      L.Cin = kS2dC;
+      L.R = R2;
+      L.S = S2;
+      L.stride = 1;
+      L.pad = 0;
+      L.K_alg = s.R * s.S * s.Cin_real;
+      conv_layer_init(L, w2, kS2dC, scale, shift);
+    } else {
+      conv_layer_init(L, wb, s.Cin_real, scale, shift);
+    }
     c->weight_bytes += (int64_t)L.Cout * L.Kp * 2 + (int64_t)L.Cout * 8;
   }
 }
@@ -387,6 +409,9 @@ void run_block(vista_ctx* c, int t, const void* in_base) {
       switch (op.kind) {
         case OP_INGEST:
           launch_ingest(reinterpret_cast<const uint8_t*>(slot[op.in]), nb, out, c->stream);
+          break;
+        case OP_INGEST_S2D:
+          launch_ingest_s2d(reinterpret_cast<const uint8_t*>(slot[op.in]), nb, out, c->stream);
           break;
         case OP_CONV:
           conv_forward(c->convs[op.layer], in, nb, op.H, op.W,

@@ -43,6 +43,8 @@ CONV = [
     (1, 9, 9, 96, 96, 3, 1, 1, 2, True, True),         # Cg_out = 48: masked group tile, register epilogue
     (2, 15, 15, 64, 256, 1, 1, 0, 1, True, True),      # TMA A + TMA epilogue, M tail (450 rows), residual
     (3, 1, 1, 2048, 1000, 1, 1, 0, 1, True, False),    # FC 1000 with BN = 256 partial tile + residual
+    (2, 20, 23, 16, 64, 4, 1, 0, 1, False, True),      # space-to-depth conv1 shape: TMA row view (Wo = 20)
+    (1, 12, 12, 16, 64, 4, 1, 0, 1, True, True),       # same class with residual: row gather fallback
 ]
 
 

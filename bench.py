@@ -38,6 +38,18 @@ CONFIGS = {
     "resnet50_top5_amazon200k": (2, [0, 1, 2, 3, 4], 200000, 201, 1, 10),
 }
 DEFAULT = "resnet50_top5_foods20k"
+TAP_NAMES = [["conv5", "fc6", "fc7", "fc8"], ["fc6", "fc7", "fc8"], ["conv4_6", "conv5_1", "conv5_2", "conv5_3", "fc"]]
+
+
+def workload_config(name, world, n_img=None):
+    """The `config` object both arms print (same workload, same keys)."""
+    cnn, taps, n_default, d_s, kind, T = CONFIGS[name]
+    n_img = n_img or n_default
+    return {"workload": name, "images_per_gpu": n_img, "global_images": n_img * world,
+            "taps": [TAP_NAMES[cnn][t] for t in taps], "d_s": d_s, "table": ["foods", "amazon"][kind],
+            "lr_iters": T, "power_iters": 20, "plan": "staged",
+            "parallelism": f"dp{world} (image shards, fp64 NCCL allreduce in LR)",
+            "l2": "inputs larger than L2 (pixels %.2f GB/GPU)" % (n_img * 227 * 227 * 3 / 1e9)}
 
 
 def env_int(k, d):
@@ -142,8 +154,8 @@ def oracle_sample(cfg_name, budget_s=20.0, nthreads=0):
     import oracle
     cnn, taps, n_img, d_s, kind, T = CONFIGS[cfg_name]
     cores = nthreads or os.cpu_count() or 1
-    # calibrate: one image per thread first, then scale the sample to ~budget_s
-    S = max(1, min(cores, n_img))
+    # two images per host thread: ~10-15 s of fp64 work for ResNet50 whatever the core count
+    S = max(1, min(2 * cores, n_img))
     tab = gen.make_tables(S, d_s, kind=kind)
     t0 = time.perf_counter()
     F, _ = oracle.features(cnn, 1, tab.images, taps=taps, nthreads=cores)
@@ -179,8 +191,7 @@ def run_reference(args):
         "impl": "reference", "metric": METRIC, "value": value, "unit": "images/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000.0 * T_tot / max(len(times), 1),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-        "data": "synthetic", "config": {"workload": args.config, "images_per_gpu": n_img, "taps": taps,
-                                        "d_s": d_s, "lr_iters": T},
+        "data": "synthetic", "config": workload_config(args.config, world),
         "cpu_baseline": {"value": value, "unit": "images/s", "cores": os.cpu_count(), "kind": "oracle",
                          "sample": desc, "cpu_model": cpu_model()},
         "e2e": {"value": value, "unit": "images/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -337,12 +348,7 @@ def main():
             "warmup": args.warmup, "ms_per_step": ms_step, "end_to_end_s": ms_step / 1000.0,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
             "data": "synthetic",
-            "config": {"workload": args.config, "images_per_gpu": n_img, "global_images": N_global,
-                       "taps": [["conv5", "fc6", "fc7", "fc8"], ["fc6", "fc7", "fc8"],
-                                ["conv4_6", "conv5_1", "conv5_2", "conv5_3", "fc"]][cnn][:max(taps) + 1],
-                       "d_s": d_s, "lr_iters": T, "power_iters": 20, "plan": "staged",
-                       "micro_batch": info["micro_batch"], "l2": "inputs larger than L2 (pixels %.2f GB/GPU)"
-                       % (tab.images.nbytes / 1e9), "parallelism": f"dp{world} (image shards, fp64 NCCL allreduce in LR)"},
+            "config": dict(workload_config(args.config, world, n_img), micro_batch=info["micro_batch"]),
             "roofline": roof,
             "cpu_baseline": cpu,
             "e2e": {"value": N_global / (e2e_step / 1000.0), "unit": "images/s", "ms_per_step": e2e_step,

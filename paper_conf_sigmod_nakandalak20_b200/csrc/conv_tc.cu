@@ -52,7 +52,9 @@ struct ConvParams {
 };
 
 constexpr int BM = 128, BK = 64;
-constexpr int kThreads = 288;  // 4 producer warps + 1 MMA warp + 4 epilogue warps
+constexpr int kEpiWarps = 8;   // two per TMEM lane quadrant, each owning half of the tile's columns
+constexpr int kEpiThreads = kEpiWarps * 32;
+constexpr int kThreads = 160 + kEpiThreads;  // 4 producer warps + 1 MMA warp + epilogue warps
 constexpr int kEpiWarp0 = 5;
 constexpr int kLag = 2;        // cp.async groups in flight before a stage is published
 
@@ -135,7 +137,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     for (int i = 0; i < 2; ++i) {
       mbar_init(&tfull[i], 1);
-      mbar_init(&tempty[i], 4);
+      mbar_init(&tempty[i], kEpiWarps);
     }
     mbar_init(&rbar[0], 1);
     mbar_init(&rbar[1], 1);
@@ -371,10 +373,11 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     __syncwarp();
   } else {
-    // ======================= epilogue (128 threads, one output row each) =======================
+    // ================ epilogue (8 warps: one output row per lane, half of the columns each) ================
     const int et = threadIdx.x - kEpiWarp0 * 32;
     const int q = warp & 3;  // TMEM lane quadrant this warp may access
     const int row = q * 32 + lane;
+    const int half = (warp - kEpiWarp0) >> 2;  // column half of the tile this warp owns
     const bool has_res = p.res != nullptr;
     uint32_t it = 0;
     for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x, ++it) {
@@ -417,28 +420,31 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       // stage this tile's scale / shift in smem (double-buffered by accumulator)
       float* ss = sbuf + acc * 2 * BN;
-      for (int i = et; i < 2 * BN; i += 128) {
+      for (int i = et; i < 2 * BN; i += kEpiThreads) {
         const int c = i < BN ? i : i - BN;
         ss[i] = c < nvalid_tile ? (i < BN ? p.scale[ng0 + c] : p.shift[ng0 + c]) : 0.f;
       }
-      named_bar_sync(1, 128);
+      named_bar_sync(1, kEpiThreads);
       const int mo = m0 + row;
       const bool rvalid = mo < p.M;
       const size_t off = (size_t)(rvalid ? mo : 0) * p.Cout + ng0;
+      constexpr int kChunks = BN / 64;  // 32-column chunks per warp
+      const int cb0 = half * kChunks;
       uint4 rres[4] = {};
       if constexpr (TMA_EPI) {
         if (has_res) mbar_wait(&rbar[ob], (NB == 2 ? (it >> 1) : it) & 1);
       } else if (has_res && rvalid) {
 #pragma unroll
         for (int j = 0; j < 4; ++j)
-          rres[j] = (j * 8 < nvalid_tile) ? __ldg(reinterpret_cast<const uint4*>(p.res + off) + j)
-                                          : make_uint4(0, 0, 0, 0);
+          rres[j] = (cb0 * 32 + j * 8 < nvalid_tile)
+                        ? __ldg(reinterpret_cast<const uint4*>(p.res + off + cb0 * 32) + j)
+                        : make_uint4(0, 0, 0, 0);
       }
       mbar_wait(&tfull[acc], use & 1);
       tc_fence_after();
       const uint32_t taddr = tmem_base + acc * BN + ((uint32_t)(q * 32) << 16);
 #pragma unroll 1
-      for (int cb = 0; cb < BN / 32; ++cb) {
+      for (int cb = cb0; cb < cb0 + kChunks; ++cb) {
         if (cb * 32 >= nvalid_tile) break;  // warp-uniform
         uint32_t v[32];
         tmem_ld_32x32b_x32(taddr + cb * 32, v);
@@ -459,7 +465,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           uint4 cur[4];
 #pragma unroll
           for (int j = 0; j < 4; ++j) cur[j] = rres[j];
-          if (has_res && rvalid && (cb + 1) * 32 < nvalid_tile) {  // prefetch the next chunk's residual
+          if (has_res && rvalid && cb + 1 < cb0 + kChunks && (cb + 1) * 32 < nvalid_tile) {  // prefetch next chunk
 #pragma unroll
             for (int j = 0; j < 4; ++j)
               rres[j] = ((cb + 1) * 32 + j * 8 < nvalid_tile)
@@ -485,7 +491,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (lane == 0) mbar_arrive(&tempty[acc]);
       if constexpr (TMA_EPI) {
         fence_proxy_async_smem();
-        named_bar_sync(1, 128);
+        named_bar_sync(1, kEpiThreads);
         if (et == 0) {
           const int nsub = (nvalid_tile + 63) / 64;
           for (int st = 0; st < nsub; ++st) {

@@ -195,6 +195,12 @@ vista_status vista_conv2d(const void* x, int32_t N, int32_t H, int32_t W, int32_
                           int32_t Cout, int32_t R, int32_t S, int32_t stride, int32_t pad, int32_t groups,
                           const float* scale, const float* shift, const void* residual, int32_t relu,
                           void* y, void* stream);
+/* The same conv with ReLU and the tap g_l (PAPER.md:369 fn 4) fused into its epilogue: y as in
+ * vista_conv2d (groups 1, relu 1) and F bf16 [N, 4*Cout] = 2x2-grid maxima of y (NHWC flatten).
+ * VISTA_ERR_INVALID_ARG when the shape cannot take the fused path (short-K TMA epilogue, Ho*Wo >= 43). */
+vista_status vista_conv2d_tap(const void* x, int32_t N, int32_t H, int32_t W, int32_t C, const void* w, int32_t Cout,
+                              int32_t R, int32_t S, int32_t stride, int32_t pad, const float* scale,
+                              const float* shift, const void* residual, void* y, void* F, void* stream);
 /* g_l on a conv activation: A bf16 [N,H,W,C] -> F bf16 [N,4C] (2x2 grid max, NHWC flatten). */
 vista_status vista_tap(const void* A, int32_t N, int32_t H, int32_t W, int32_t C, void* F, void* stream);
 /* unpadded max pool k/s, bf16 NHWC */

@@ -49,6 +49,9 @@ struct ConvParams {
   const float* shift;
   int H, W, Cin, Ho, Wo, Cout, R, S, stride, pad, Cg_in, Cg_out, K, nkb, M, relu;
   int n_mt, n_nt, n_tiles;
+  // fused tap g_l (PAPER.md:369 fn 4): per-image 2x2-grid channel maxima of the (post-ReLU, >= 0)
+  // output, accumulated as fp32 bit patterns with red.global.max.u32 into tapf[n][4][Cout]
+  unsigned int* tapf;
 };
 
 constexpr int BM = 128, BK = 64;
@@ -502,6 +505,49 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
           bulk_commit();
         }
+        if (p.tapf) {
+          // Fused tap: scan the staged bf16 tile column-wise (kEpiThreads / BN threads per column split
+          // the rows), keep one running max per (image, quadrant) met in this tile, and publish each
+          // with one red.max.  Quadrants: R_0 = [0, ceil(H/2)), R_1 = [ceil(H/2), H) (reading R7).
+          constexpr int kTpc = kEpiThreads / BN;  // threads per column
+          const int col = et % BN, part = et / BN;
+          if (col < nvalid_tile) {
+            const int hw = p.Ho * p.Wo, h2 = (p.Ho + 1) >> 1, w2 = (p.Wo + 1) >> 1;
+            const int r0 = part * (BM / kTpc), r1 = r0 + BM / kTpc;
+            const int n_first = m0 / hw;
+            float mx[16];
+#pragma unroll
+            for (int k = 0; k < 16; ++k) mx[k] = -1.f;
+            int m = m0 + r0;
+            int n = m / hw, rem = m - n * hw;
+            int h = rem / p.Wo, w = rem - h * p.Wo;
+            const uint32_t cbase = sOb + (col >> 6) * BM * 128 + (col & 7) * 2;
+            const uint32_t cchunk = (uint32_t)((col & 63) >> 3);
+            for (int r = r0; r < r1 && m < p.M; ++r, ++m) {
+              const uint32_t a = cbase + r * 128 + ((cchunk ^ (uint32_t)(r & 7)) << 4);
+              unsigned short bits;
+              asm volatile("ld.shared.u16 %0, [%1];" : "=h"(bits) : "r"(a));
+              const float v = __uint_as_float((uint32_t)bits << 16);
+              const int k = (n - n_first) * 4 + (h >= h2 ? 2 : 0) + (w >= w2 ? 1 : 0);
+#pragma unroll
+              for (int kk = 0; kk < 16; ++kk)
+                if (kk == k) mx[kk] = fmaxf(mx[kk], v);
+              if (++w == p.Wo) {
+                w = 0;
+                if (++h == p.Ho) {
+                  h = 0;
+                  ++n;
+                }
+              }
+            }
+#pragma unroll
+            for (int k = 0; k < 16; ++k)
+              if (mx[k] >= 0.f)
+                atomicMax(p.tapf + ((size_t)(n_first + (k >> 2)) * 4 + (k & 3)) * p.Cout + ng0 + col,
+                          __float_as_uint(mx[k]));
+          }
+          named_bar_sync(1, kEpiThreads);  // the staging buffer may be refilled after this
+        }
       }
     }
     if (TMA_EPI && et == 0) bulk_wait0();
@@ -683,12 +729,13 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
   }
 }
 
-void conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const bf16* res, bf16* y,
-                  cudaStream_t st) {
+bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const bf16* res, bf16* y,
+                  cudaStream_t st, unsigned int* tapf) {
   ConvParams p;
   p.x = x;
   p.y = y;
   p.res = res;
+  p.tapf = nullptr;
   p.scale = L.scale;
   p.shift = L.shift;
   p.H = H;
@@ -706,7 +753,7 @@ void conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   p.K = L.K;
   p.nkb = L.Kp / BK;
   const int64_t M = (int64_t)N * p.Ho * p.Wo;
-  if (M <= 0) return;
+  if (M <= 0) return tapf == nullptr;
   if (M > INT32_MAX - BM) fail(1, "conv: M too large for one launch");
   p.M = (int)M;
   p.relu = L.relu ? 1 : 0;
@@ -758,6 +805,9 @@ void conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   // (long-K layers keep the register epilogue: it is hidden behind the mainloop and frees the staging
   // smem for a deeper k-block ring)
   const bool tma_epi = rowview || ((L.groups == 1 || L.Cg_out % L.BN == 0) && L.Cout % 8 == 0 && p.nkb <= 8);
+  // the fused tap needs the staged tile, non-negative outputs (ReLU) and <= 4 images per 128-row tile
+  const bool fuse_tap = tapf && tma_epi && !rowview && L.relu && p.Ho * p.Wo >= 43;
+  if (fuse_tap) p.tapf = tapf;
   if (rowview) {
     tr = ty;  // output map built above; no residual
   } else if (tma_epi) {
@@ -785,6 +835,7 @@ void conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
              L.S, L.stride, L.groups, L.Cin, L.Cout, H, W, p.M, L.K, L.BN, amode, tma_epi ? 1 : 0, p.n_tiles,
              res ? " res" : "");
   prof_end(st, 0, flops, bytes, label);
+  return tapf == nullptr || fuse_tap;
 }
 
 }  // namespace vista

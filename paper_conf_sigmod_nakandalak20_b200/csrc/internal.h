@@ -55,9 +55,13 @@ struct ConvLayer {
 void conv_layer_init(ConvLayer& L, const std::vector<uint16_t>& w_ohwi_bf16, int Cin_real,
                      const std::vector<float>& scale, const std::vector<float>& shift);
 void conv_layer_free(ConvLayer& L);
-// y[N,Ho,Wo,Cout] = act(scale * conv(x) + shift (+ res))
-void conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const bf16* res, bf16* y,
-                  cudaStream_t st);
+// y[N,Ho,Wo,Cout] = act(scale * conv(x) + shift (+ res)).
+// tapf (optional): fp32-bit accumulator [N][4][Cout] (zeroed by the caller) receiving the fused tap
+// (2x2-grid maxima); returns false if the tap could not be fused (caller runs launch_tap instead).
+bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const bf16* res, bf16* y,
+                  cudaStream_t st, unsigned int* tapf = nullptr);
+// F bf16 [n, 4C] <- fp32 tap accumulator (exact: the maxima are bf16 values)
+void launch_tap_finalize(const unsigned int* tapf, int64_t count, bf16* F, cudaStream_t st);
 inline int conv_out_dim(int H, int k, int s, int p) { return (H + 2 * p - k) / s + 1; }
 
 // ---- SIMT kernels (memory-bound) ----

@@ -222,6 +222,23 @@ __global__ void tap_kernel(const bf16* __restrict__ A, int64_t N, int H, int W, 
     st8(F + (size_t)n * 4 * C + (size_t)q * C + c8 * 8, m);
   }
 }
+// finalize of the fused tap (conv_tc.cu): fp32 maxima -> bf16, 8 values per thread (exact)
+__global__ void tap_finalize_kernel(const unsigned int* __restrict__ in, int64_t n8, bf16* __restrict__ F) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n8; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint4 a = reinterpret_cast<const uint4*>(in)[2 * i], b = reinterpret_cast<const uint4*>(in)[2 * i + 1];
+    const float f[8] = {__uint_as_float(a.x), __uint_as_float(a.y), __uint_as_float(a.z), __uint_as_float(a.w),
+                        __uint_as_float(b.x), __uint_as_float(b.y), __uint_as_float(b.z), __uint_as_float(b.w)};
+    st8(F + i * 8, f);
+  }
+}
+void launch_tap_finalize(const unsigned int* tapf, int64_t count, bf16* F, cudaStream_t st) {
+  const int64_t n8 = count / 8;
+  prof_begin(st);
+  tap_finalize_kernel<<<grid_for(n8, 256), 256, 0, st>>>(tapf, n8, F);
+  LAUNCHED();
+  prof_end(st, 1, 0, (double)count * 6);
+}
+
 void launch_tap(const bf16* A, int64_t N, int H, int W, int C, bf16* F, cudaStream_t st) {
   const int64_t total = N * 4 * (C / 8);
   prof_begin(st);

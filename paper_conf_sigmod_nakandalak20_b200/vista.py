@@ -90,6 +90,9 @@ def lib():
         L.vista_get_profile.argtypes = [_vp, ctypes.POINTER(Profile), _i32]
         L.vista_conv2d.argtypes = [_vp, _i32, _i32, _i32, _i32, _vp, _i32, _i32, _i32, _i32, _i32, _i32, _vp, _vp,
                                    _vp, _i32, _vp, _vp]
+        L.vista_conv2d_tap.argtypes = [_vp, _i32, _i32, _i32, _i32, _vp, _i32, _i32, _i32, _i32, _i32, _vp, _vp,
+                                       _vp, _vp, _vp, _vp]
+        L.vista_kernel_launches.restype = _i64
         L.vista_tap.argtypes = [_vp, _i32, _i32, _i32, _i32, _vp, _vp]
         L.vista_maxpool.argtypes = [_vp, _i32, _i32, _i32, _i32, _i32, _i32, _vp, _vp]
         L.vista_lrn.argtypes = [_vp, _i32, _i32, _i32, _i32, _vp, _vp]
@@ -147,6 +150,23 @@ def vista_conv2d(x, w, scale, shift, stride=1, pad=0, groups=1, residual=None, r
     _check(lib().vista_conv2d(_ptr(x), N, H, W, C, _ptr(w), Cout, R, S, stride, pad, groups, _ptr(scale),
                               _ptr(shift), _ptr(residual), 1 if relu else 0, _ptr(y), _stream(stream)))
     return y
+
+
+def vista_conv2d_tap(x, w, scale, shift, stride=1, pad=0, residual=None, stream=None):
+    """conv + ReLU with the 2x2-grid tap fused into the epilogue; returns (y, F)."""
+    import torch
+    N, H, W, C = x.shape
+    Cout, R, S, _ = w.shape
+    Ho, Wo = (H + 2 * pad - R) // stride + 1, (W + 2 * pad - S) // stride + 1
+    y = torch.empty((N, Ho, Wo, Cout), dtype=torch.bfloat16, device=x.device)
+    F = torch.empty((N, 4 * Cout), dtype=torch.bfloat16, device=x.device)
+    _check(lib().vista_conv2d_tap(_ptr(x), N, H, W, C, _ptr(w), Cout, R, S, stride, pad, _ptr(scale), _ptr(shift),
+                                  _ptr(residual), _ptr(y), _ptr(F), _stream(stream)))
+    return y, F
+
+
+def vista_kernel_launches() -> int:
+    return int(lib().vista_kernel_launches())
 
 
 def vista_tap(A, stream=None):

@@ -79,6 +79,24 @@ def test_conv_deterministic():
     assert torch.equal(y1.view(torch.int16), y2.view(torch.int16))
 
 
+@pytest.mark.parametrize("N,H,C,Cout,res", [(3, 14, 256, 1024, True), (5, 7, 512, 2048, True), (2, 9, 64, 128, False),
+                                            (4, 13, 128, 256, False)])
+def test_fused_tap_bit_exact(N, H, C, Cout, res):
+    # the conv4_6 / conv5_x producers: 1x1 convs with residual + ReLU; the tap fused into the epilogue
+    # must equal the standalone tap of the same bf16 output bit for bit (max is exact), and the oracle's
+    from paper_conf_sigmod_nakandalak20_b200.vista import vista_conv2d_tap
+    x, _ = bf(rng.standard_normal((N, H, H, C)))
+    w, _ = bf(rng.standard_normal((Cout, 1, 1, C)) * (2.0 / C) ** 0.5)
+    scale = torch.from_numpy(rng.uniform(0.5, 1.5, Cout).astype(np.float32)).cuda()
+    shift = torch.from_numpy((rng.standard_normal(Cout) * 0.1).astype(np.float32)).cuda()
+    r = bf(rng.standard_normal((N, H, H, Cout)))[0] if res else None
+    y, F = vista_conv2d_tap(x, w, scale, shift, residual=r)
+    y2 = vista_conv2d(x, w, scale, shift, residual=r, relu=True)
+    assert torch.equal(y.view(torch.int16), y2.view(torch.int16))
+    assert torch.equal(F.view(torch.int16), vista_tap(y).view(torch.int16))
+    np.testing.assert_array_equal(F.to(torch.float64).cpu().numpy(), oracle.tap(y.to(torch.float64).cpu().numpy()))
+
+
 @pytest.mark.parametrize("H,C", [(14, 1024), (7, 2048), (13, 256), (2, 8), (3, 16)])
 def test_tap_bit_exact(H, C):
     A, A64 = bf(rng.standard_normal((3, H, H, C)))

@@ -212,6 +212,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--images", type=int, default=0, help="override images per GPU (debug only)")
     ap.add_argument("--micro-batch", type=int, default=0, help="stage-1 micro-batch (0 = planner)")
+    ap.add_argument("--plan", default="staged", choices=["staged", "eager", "lazy"],
+                    help="logical plan (Fig 5): staged is the product; eager / lazy for config 4 comparisons")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -256,7 +258,7 @@ def main():
     stream = torch.cuda.current_stream(dev)
     v = Vista(cnn, layers=taps, n_str_rows=len(tab.str_keys), d_s=d_s, n_images_local=n_img, iters=T,
               power_iters=20, split_seed=5, weight_seed=1, rank=rank, world=world, nccl_uid=uid, device=local,
-              stream=stream.cuda_stream, micro_batch=args.micro_batch)
+              stream=stream.cuda_stream, micro_batch=args.micro_batch, plan=args.plan)
     info = v.plan_info()
     d_tot = [d_s + d for d in info["d_l"]]
 
@@ -348,7 +350,8 @@ def main():
             "warmup": args.warmup, "ms_per_step": ms_step, "end_to_end_s": ms_step / 1000.0,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
             "data": "synthetic",
-            "config": dict(workload_config(args.config, world, n_img), micro_batch=info["micro_batch"]),
+            "config": dict(workload_config(args.config, world, n_img), micro_batch=info["micro_batch"],
+                           plan=args.plan, peak_bytes_pred=info["peak_bytes_pred"]),
             "roofline": roof,
             "cpu_baseline": cpu,
             "e2e": {"value": N_global / (e2e_step / 1000.0), "unit": "images/s", "ms_per_step": e2e_step,

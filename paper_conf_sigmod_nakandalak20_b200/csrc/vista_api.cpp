@@ -223,6 +223,7 @@ struct vista_ctx {
   // (its per-(image, quadrant, channel) red.max traffic, ~10M per 1024-image launch, slows the epilogue
   // of the HBM-bound producer convs by ~40 ms/step) vs standalone 59.3k img/s (4.3 ms/step re-reading A_k).
   bool fuse_tap = false;
+  std::vector<void*> feat;  // per block: device pointer of F_t (features) of a tapped layer
   std::string last_error;
   ~vista_ctx() {
     for (auto* v : {&A, &F, &MM, &Y, &slot_store})
@@ -289,6 +290,27 @@ void plan_memory(vista_ctx* c, uint64_t budget) {
   const int64_t px = c->n_img * (int64_t)S[0].in_elems;
   const int64_t join_bytes = c->n_str * 8 + c->n_img * 8 + c->n_str * 4 * 2 + c->n_str * 12 + 32 * 4 * std::max(c->n_img, c->n_str);
   int64_t peak = 0;
+  if (c->sys.plan != VISTA_PLAN_STAGED) {
+    // Eager / Lazy: features of all of L (incl. FC taps) + two micro-batch activation buffers + slots
+    int64_t f_all = 0, max_out = 0, slot_per_img = 0;
+    for (int t : c->taps) f_all += c->n_img * (int64_t)S[t].d_tap * 2;
+    for (int t = 0; t <= c->t_max; ++t) {
+      max_out = std::max<int64_t>(max_out, S[t].out_elems);
+      int64_t s = 0;
+      for (int b = BUF_T0; b < NUM_BUFS; ++b) s += S[t].slot_elems[b] * 2;
+      slot_per_img = std::max(slot_per_img, s);
+    }
+    const int64_t fixed = c->weight_bytes + px + f_all + mm_bytes + join_bytes + (256ll << 20);
+    const int64_t per_img = slot_per_img + 2 * max_out * 2;
+    int B = c->sys.micro_batch > 0 ? c->sys.micro_batch : 0;
+    for (int64_t b = std::min<int64_t>(1024, std::max<int64_t>(c->n_img, 1)); B == 0 && b >= 1;
+         b = b > 8 ? b / 2 : b - 1)
+      if ((uint64_t)(fixed + b * per_img) <= budget) B = (int)b;
+    if (B <= 0) fail(VISTA_ERR_NO_PLAN, "no micro-batch fits the HBM budget (eager/lazy)");
+    c->micro.assign(c->t_max + 1, B);
+    c->peak_pred = fixed + (int64_t)B * per_img;
+    return;
+  }
   for (int t = 0; t <= c->t_max; ++t) {
     const int64_t a_in = t == 0 ? px : c->n_img * S[t - 1].out_elems * 2;
     const int64_t a_out = c->n_img * S[t].out_elems * 2;
@@ -391,26 +413,25 @@ const void* to_device(vista_ctx* c, DevBuf& buf, const void* p, size_t bytes) {
   return buf.p;
 }
 
-// one block (stage) of the Staged plan over all local images, in micro-batches
-// tapf: zeroed fp32 tap accumulator [n_img][4][C] for the stage's output conv (fused tap), or null.
-// Returns true iff every micro-batch fused the tap into that conv's epilogue.
-bool run_block(vista_ctx* c, int t, const void* in_base, unsigned int* tapf) {
-  bool fused = tapf != nullptr;
+// scratch slots able to hold block t's intermediates for B images (grow-only within a transfer)
+void prepare_slots(vista_ctx* c, int t, int B, void** slot) {
   const StageDesc& S = c->net.stages[t];
-  const int B = c->micro[t];
-  // scratch slots sized for this block
-  void* slot[NUM_BUFS] = {nullptr};
   for (int b = BUF_T0; b < NUM_BUFS; ++b) {
     const size_t need = (size_t)S.slot_elems[b] * 2 * B;
     if (need > c->slot_store[b]->bytes) c->slot_store[b]->alloc(need);
     slot[b] = c->slot_store[b]->p;
   }
-  const size_t in_bytes_per = t == 0 ? (size_t)S.in_elems : (size_t)S.in_elems * 2;
-  bf16* out_base = reinterpret_cast<bf16*>(c->A[t]->p);
-  for (int64_t i0 = 0; i0 < c->n_img; i0 += B) {
-    const int nb = (int)std::min<int64_t>(B, c->n_img - i0);
-    slot[BUF_IN] = (void*)((const uint8_t*)in_base + (size_t)i0 * in_bytes_per);
-    slot[BUF_OUT] = out_base + (size_t)i0 * S.out_elems;
+}
+
+// nb images through block t (partial inference f^_{l(t-1) -> l(t)}): in -> out.
+// tapf: this micro-batch's slice of a zeroed fp32 tap accumulator for the block's output conv, or null.
+// Returns false iff a tap was requested and could not be fused.
+bool run_ops(vista_ctx* c, int t, const void* in_ptr, void* out_ptr, int nb, void** slot, unsigned int* tapf) {
+  bool fused = true;
+  const StageDesc& S = c->net.stages[t];
+  {
+    slot[BUF_IN] = const_cast<void*>(in_ptr);
+    slot[BUF_OUT] = out_ptr;
     for (const OpDesc& op : S.ops) {
       const bf16* in = reinterpret_cast<const bf16*>(slot[op.in]);
       bf16* out = reinterpret_cast<bf16*>(slot[op.out]);
@@ -422,7 +443,7 @@ bool run_block(vista_ctx* c, int t, const void* in_base, unsigned int* tapf) {
           launch_ingest_s2d(reinterpret_cast<const uint8_t*>(slot[op.in]), nb, out, c->stream);
           break;
         case OP_CONV: {
-          unsigned int* tp = (tapf && op.out == BUF_OUT) ? tapf + (size_t)i0 * 4 * S.outC : nullptr;
+          unsigned int* tp = (tapf && op.out == BUF_OUT) ? tapf : nullptr;
           const bool ok = conv_forward(c->convs[op.layer], in, nb, op.H, op.W,
                                        op.res >= 0 ? reinterpret_cast<const bf16*>(slot[op.res]) : nullptr, out,
                                        c->stream, tp);
@@ -442,6 +463,56 @@ bool run_block(vista_ctx* c, int t, const void* in_base, unsigned int* tapf) {
     }
   }
   return fused;
+}
+
+// one block of the Staged plan over all local images, in micro-batches of micro[t]: in_base -> A_t
+bool run_block(vista_ctx* c, int t, const void* in_base, unsigned int* tapf) {
+  const StageDesc& S = c->net.stages[t];
+  const int B = c->micro[t];
+  void* slot[NUM_BUFS] = {nullptr};
+  prepare_slots(c, t, B, slot);
+  const size_t in_bytes_per = t == 0 ? (size_t)S.in_elems : (size_t)S.in_elems * 2;
+  bf16* out_base = reinterpret_cast<bf16*>(c->A[t]->p);
+  bool fused = tapf != nullptr;
+  for (int64_t i0 = 0; i0 < c->n_img; i0 += B) {
+    const int nb = (int)std::min<int64_t>(B, c->n_img - i0);
+    const bool ok = run_ops(c, t, (const uint8_t*)in_base + (size_t)i0 * in_bytes_per,
+                            out_base + (size_t)i0 * S.out_elems, nb, slot,
+                            tapf ? tapf + (size_t)i0 * 4 * S.outC : nullptr);
+    fused = fused && ok;
+  }
+  return fused;
+}
+
+// Eager (Fig 5C) and Lazy (Fig 5A) schedules: per micro-batch of images, run blocks 0..t_last from
+// the raw pixels with the activations in two ping-pong micro-batch buffers, and tap every requested
+// layer in `want` (Eager: all of L in one pass; Lazy: one layer per pass, recomputing from pixels).
+void run_unstaged(vista_ctx* c, const uint8_t* px, int t_last, const std::vector<int>& want) {
+  const auto& S = c->net.stages;
+  const int B = c->micro[0];
+  void* slot[NUM_BUFS] = {nullptr};
+  int64_t max_out = 0;
+  for (int t = 0; t <= t_last; ++t) {
+    prepare_slots(c, t, B, slot);
+    max_out = std::max<int64_t>(max_out, S[t].out_elems);
+  }
+  DevBuf act[2];
+  act[0].alloc((size_t)B * max_out * 2 + 16);
+  act[1].alloc((size_t)B * max_out * 2 + 16);
+  for (int64_t i0 = 0; i0 < c->n_img; i0 += B) {
+    const int nb = (int)std::min<int64_t>(B, c->n_img - i0);
+    for (int t = 0; t <= t_last; ++t) {
+      const void* in = t == 0 ? (const void*)(px + (size_t)i0 * S[0].in_elems) : act[(t - 1) & 1].p;
+      bf16* out = (bf16*)act[t & 1].p;
+      run_ops(c, t, in, out, nb, slot, nullptr);
+      if (std::find(want.begin(), want.end(), t) == want.end()) continue;
+      bf16* Ft = (bf16*)c->F[t]->p + (size_t)i0 * S[t].d_tap;
+      if (S[t].fc_tap)
+        VCHECK(cudaMemcpyAsync(Ft, out, (size_t)nb * S[t].d_tap * 2, cudaMemcpyDeviceToDevice, c->stream));
+      else
+        launch_tap(out, nb, S[t].outH, S[t].outW, S[t].outC, Ft, c->stream);
+    }
+  }
 }
 
 }  // namespace
@@ -522,7 +593,7 @@ VISTA_API vista_status vista_plan(vista_cnn cnn, const int32_t* layers, int32_t 
     if (c->lr.iters < 0 || c->lr.power_iters < 0) fail(1, "negative iteration count");
     if (sys) c->sys = *sys;
     if (c->sys.world <= 0) c->sys.world = 1;
-    if (c->sys.plan != VISTA_PLAN_STAGED) fail(1, "only the Staged plan is implemented (eager/lazy: next round)");
+    if (c->sys.plan < VISTA_PLAN_STAGED || c->sys.plan > VISTA_PLAN_LAZY) fail(1, "unknown logical plan");
     if (c->sys.dtype != VISTA_BF16) fail(1, "only bf16 is implemented");
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
@@ -639,7 +710,30 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
       c->MM.emplace_back(new DevBuf());
       c->Y.emplace_back(new DevBuf());
     }
-    for (int t = 0; t <= c->t_max; ++t) {
+    c->feat.assign(c->t_max + 1, nullptr);
+    auto concat_layer = [&](int k) {
+      const int t = c->taps[k];
+      const int ld = ld_of(c, k);
+      c->MM[k]->alloc((size_t)std::max<int64_t>(c->n_pairs, 1) * ld * 2);
+      c->Y[k]->alloc((size_t)std::max<int64_t>(c->n_pairs, 1));
+      launch_concat(X, c->d_s, c->ds_pad, (const bf16*)c->feat[t], S[t].d_tap, (const int32_t*)c->pair_str.p,
+                    (const int32_t*)c->pair_img.p, lab, c->n_pairs, ld, (bf16*)c->MM[k]->p, (uint8_t*)c->Y[k]->p,
+                    st);
+    };
+    if (c->sys.plan != VISTA_PLAN_STAGED) {
+      // ---- Eager / Lazy (Fig 5C / 5A): features of every layer, no resident full activations ----
+      for (int t : c->taps) {
+        c->F[t]->alloc((size_t)c->n_img * S[t].d_tap * 2 + 16);
+        c->feat[t] = c->F[t]->p;
+      }
+      if (c->sys.plan == VISTA_PLAN_EAGER) {
+        run_unstaged(c, px, c->t_max, c->taps);
+      } else {
+        for (int t : c->taps) run_unstaged(c, px, t, std::vector<int>{t});
+      }
+      for (size_t k = 0; k < c->taps.size(); ++k) concat_layer((int)k);
+    }
+    for (int t = 0; t <= c->t_max && c->sys.plan == VISTA_PLAN_STAGED; ++t) {
       c->A[t]->alloc((size_t)c->n_img * S[t].out_elems * 2 + 16);
       const void* in = t == 0 ? (const void*)px : c->A[t - 1]->p;
       const int k = layer_index(c, t);
@@ -654,23 +748,17 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
       }
       const bool fused = run_block(c, t, in, tapf);
       if (k >= 0) {
-        const bf16* Fk;
         if (S[t].fc_tap) {
-          Fk = (const bf16*)c->A[t]->p;  // g = identity on FC layers
+          c->feat[t] = c->A[t]->p;  // g = identity on FC layers
         } else {
           c->F[t]->alloc((size_t)c->n_img * S[t].d_tap * 2 + 16);
           if (fused)
             launch_tap_finalize(tapf, (int64_t)c->n_img * S[t].d_tap, (bf16*)c->F[t]->p, st);
           else
             launch_tap((const bf16*)c->A[t]->p, c->n_img, S[t].outH, S[t].outW, S[t].outC, (bf16*)c->F[t]->p, st);
-          Fk = (const bf16*)c->F[t]->p;
+          c->feat[t] = c->F[t]->p;
         }
-        const int ld = ld_of(c, k);
-        c->MM[k]->alloc((size_t)std::max<int64_t>(c->n_pairs, 1) * ld * 2);
-        c->Y[k]->alloc((size_t)std::max<int64_t>(c->n_pairs, 1));
-        launch_concat(X, c->d_s, c->ds_pad, Fk, S[t].d_tap, (const int32_t*)c->pair_str.p,
-                      (const int32_t*)c->pair_img.p, lab, c->n_pairs, ld, (bf16*)c->MM[k]->p, (uint8_t*)c->Y[k]->p,
-                      st);
+        concat_layer(k);
       }
       // Staged: the input activation of this block is no longer needed (Fig 5E) — unless it is an
       // FC tap whose activation doubles as its features
@@ -700,8 +788,8 @@ VISTA_API vista_status vista_features(const vista_ctx* c, int32_t k, vista_buffe
   o->pair_str = (const int32_t*)c->pair_str.p;
   o->pair_img = (const int32_t*)c->pair_img.p;
   o->labels = (const uint8_t*)c->Y[k]->p;
-  o->features = S.fc_tap ? c->A[t]->p : c->F[t]->p;
-  o->activation = c->A[t]->p;
+  o->features = c->feat[t];
+  o->activation = c->A.size() > (size_t)t ? c->A[t]->p : nullptr;
   return VISTA_OK;
 }
 

@@ -232,12 +232,14 @@ class Vista:
 
     def __init__(self, cnn, layers=None, n_top=0, n_str_rows=0, d_s=0, n_images_local=0, iters=10,
                  power_iters=20, lam=0.01, alpha=0.5, split_seed=0, weight_seed=0, rank=0, world=1,
-                 nccl_uid: bytes | None = None, device=0, hbm_budget_bytes=0, stream=None, micro_batch=0):
+                 nccl_uid: bytes | None = None, device=0, hbm_budget_bytes=0, stream=None, micro_batch=0,
+                 plan="staged"):
         self.cnn = cnn
         lr = LRCfg(iters, power_iters, lam, alpha, split_seed)
         self._uid = (ctypes.c_uint8 * 128).from_buffer_copy(nccl_uid) if nccl_uid else None
+        plan_id = {"staged": 0, "eager": 1, "lazy": 2}[plan]
         sys = SysCfg(rank, world, ctypes.addressof(self._uid) if self._uid is not None else None, device,
-                     hbm_budget_bytes, 0, 0, stream, micro_batch)
+                     hbm_budget_bytes, 0, plan_id, stream, micro_batch)
         arr = None
         n_layers = 0
         if layers is not None:

@@ -141,6 +141,25 @@ def test_staged_micro_batch_invariance():
             assert torch.equal(a, b)
 
 
+@pytest.mark.parametrize("cnn,taps,n,d_s", [(0, [0, 1, 2, 3], 12, 8), (2, [0, 1, 2, 3, 4], 5, 16)])
+def test_staged_eager_lazy_bit_identical(cnn, taps, n, d_s):
+    # "All approaches ... yield identical downstream models": Staged (Fig 5E), Eager (5C) and
+    # Lazy (5A) run the same deterministic kernels on different schedules, so MM_l and the LR results agree bit for bit
+    tab = gen.make_tables(n, d_s)
+    res = {}
+    for plan in ("staged", "eager", "lazy"):
+        v = run_gpu(cnn, taps, tab, d_s, iters=2, plan=plan, micro_batch=4)
+        mms = [v.features(k)["mm"].view(torch.int16).cpu().clone() for k in range(len(taps))]
+        w = [v.train(k, d_s + v.features(k)["d_l"])[0] for k in range(len(taps))]
+        res[plan] = (mms, w)
+        v.close()
+    for plan in ("eager", "lazy"):
+        for a, b in zip(res["staged"][0], res[plan][0]):
+            assert torch.equal(a, b), plan
+        for a, b in zip(res["staged"][1], res[plan][1]):
+            np.testing.assert_array_equal(a, b)
+
+
 def test_device_and_host_inputs_agree():
     tab = gen.make_tables(8, 8)
     v1 = run_gpu(0, [0], tab, 8, iters=2)

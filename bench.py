@@ -115,7 +115,8 @@ class ClockSampler:
         reasons = sorted({names[i] for r in self.rows for i in range(4) if r[5 + i].lower() == "active"})
         pw = [num(r[3]) for r in self.rows if num(r[3]) is not None]
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(self.rows), "power_w_max": max(pw) if pw else None}
+                "sm_mhz_min": min(sm) if sm else None, "reasons": reasons, "samples": len(self.rows),
+                "power_w_max": max(pw) if pw else None, "power_w_median": statistics.median(pw) if pw else None}
 
 
 def peaks():
@@ -277,27 +278,32 @@ def main():
             dist.barrier()
         torch.cuda.synchronize(dev)
 
+    step_ms = {}
+
     def timed(nsteps, host=False):
         barrier()
-        ev0 = torch.cuda.Event(enable_timing=True)
-        ev1 = torch.cuda.Event(enable_timing=True)
-        ev0.record(stream)
+        evs = [torch.cuda.Event(enable_timing=True) for _ in range(nsteps + 1)]
+        evs[0].record(stream)
         res = None
-        for _ in range(nsteps):
+        for i in range(nsteps):
             res = step(host)
-        ev1.record(stream)
+            evs[i + 1].record(stream)
         barrier()
-        ms = ev0.elapsed_time(ev1)
+        ms = evs[0].elapsed_time(evs[-1])
+        step_ms["e2e" if host else "device"] = [round(evs[i].elapsed_time(evs[i + 1]), 2) for i in range(nsteps)]
         if world > 1:
             t = torch.tensor([ms], device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ms = float(t.item())
         return ms, res
 
-    for _ in range(args.warmup):
-        step()
+    # the clock sampler (nvidia-smi) starts before the warm-up: its NVML start-up stalls the GPU for a
+    # few hundred ms, which must not land inside the timed region
     sampler = ClockSampler(local)
     sampler.start()
+    for _ in range(args.warmup):
+        step()
+    sampler.rows.clear()  # keep only samples of the timed region
     l0 = v_launches()
     ms, res = timed(args.steps)
     launches = v_launches() - l0
@@ -362,6 +368,7 @@ def main():
             "breakdown_ms": breakdown,
             "test_acc_per_layer": accs,
             "input_gen_s": round(gen_s, 1),
+            "step_ms": step_ms,
         }
         print(json.dumps(line), flush=True)
     v.close()

@@ -97,6 +97,7 @@ typedef struct {
   int64_t peak_bytes_pred;   /* predicted peak device bytes of vista_transfer */
   int64_t weight_bytes;      /* resident CNN parameters */
   int32_t d_s, ds_pad;       /* structured width and its padded width in MM_k */
+  int64_t chunk_images;      /* Staged: images per chunk (== n_images_local unless the budget forces chunking) */
 } vista_plan_info_t;
 
 /* Borrowed view of layer k's outputs on this rank (valid until vista_destroy or the

@@ -207,6 +207,7 @@ struct vista_ctx {
   int64_t n_img = 0, n_str = 0;
   int d_s = 0, ds_pad = 0;
   std::vector<int> micro;    // per block
+  int64_t chunk = 0;         // images per Staged chunk (== n_img unless the HBM budget forces chunking)
   int64_t weight_bytes = 0, peak_pred = 0;
   // results
   std::vector<std::unique_ptr<DevBuf>> A, F, MM, Y;  // per block (A, F) / per requested layer (MM, Y)
@@ -311,29 +312,51 @@ void plan_memory(vista_ctx* c, uint64_t budget) {
     c->peak_pred = fixed + (int64_t)B * per_img;
     return;
   }
-  for (int t = 0; t <= c->t_max; ++t) {
-    const int64_t a_in = t == 0 ? px : c->n_img * S[t - 1].out_elems * 2;
-    const int64_t a_out = c->n_img * S[t].out_elems * 2;
-    int64_t slot_per_img = 0;
-    for (int b = BUF_T0; b < NUM_BUFS; ++b) slot_per_img += S[t].slot_elems[b] * 2;
-    const int64_t fixed = c->weight_bytes + px + a_in + a_out + mm_bytes + f_bytes + join_bytes + (256ll << 20);
-    int B = 0;
-    if (c->sys.micro_batch > 0 && t == 0) {
-      B = c->sys.micro_batch;
-    } else {
-      // larger micro-batches give larger GEMMs per launch (measured: 256 -> 1024 is +7 % img/s);
-      // activations of one micro-batch exceed L2 either way
-      const int64_t cap_B = t == 0 ? 1024 : 16384;
-      for (int64_t b = std::min<int64_t>(cap_B, std::max<int64_t>(c->n_img, 1)); b >= 1; b = b > 8 ? b / 2 : b - 1) {
-        if ((uint64_t)(fixed + b * slot_per_img) <= budget) {
-          B = (int)b;
-          break;
+  // Staged: stage t holds A_{t-1} and A_t of one chunk of CH images (the B200 form of s_double,
+  // Eq. (6)) plus that chunk's pixels, every layer's F and MM, and the scratch of a
+  // micro-batch.  Chunks start at all local images and halve until the plan fits (Alg. 1's "first
+  // feasible from the top"); NO_PLAN only if not even one image fits.
+  int64_t f_fc = 0;  // FC taps alias A_t when unchunked; a chunked run keeps them in F as well
+  for (int t : c->taps)
+    if (S[t].fc_tap) f_fc += c->n_img * (int64_t)S[t].d_tap * 2;
+  auto plan_chunk = [&](int64_t CH, std::vector<int>& micro, int64_t& pk) -> bool {
+    pk = 0;
+    const bool chunked = CH < c->n_img;
+    const int64_t pxc = CH * (int64_t)S[0].in_elems;  // host pixels are streamed per chunk
+    for (int t = 0; t <= c->t_max; ++t) {
+      const int64_t a_in = t == 0 ? pxc : CH * S[t - 1].out_elems * 2;
+      const int64_t a_out = CH * S[t].out_elems * 2;
+      int64_t slot_per_img = 0;
+      for (int b = BUF_T0; b < NUM_BUFS; ++b) slot_per_img += S[t].slot_elems[b] * 2;
+      const int64_t fixed = c->weight_bytes + pxc + a_in + a_out + mm_bytes + f_bytes + (chunked ? f_fc : 0) +
+                            join_bytes + (256ll << 20);
+      int B = 0;
+      if (c->sys.micro_batch > 0 && t == 0) {
+        B = (int)std::min<int64_t>(c->sys.micro_batch, std::max<int64_t>(CH, 1));
+        if ((uint64_t)(fixed + B * slot_per_img) > budget) return false;
+      } else {
+        // larger micro-batches give larger GEMMs per launch (measured: 256 -> 1024 is +7 % img/s);
+        // activations of one micro-batch exceed L2 either way
+        const int64_t cap_B = t == 0 ? 1024 : 16384;
+        for (int64_t b = std::min<int64_t>(cap_B, std::max<int64_t>(CH, 1)); b >= 1; b = b > 8 ? b / 2 : b - 1) {
+          if ((uint64_t)(fixed + b * slot_per_img) <= budget) {
+            B = (int)b;
+            break;
+          }
         }
       }
+      if (B <= 0) return false;
+      micro[t] = B;
+      pk = std::max(pk, fixed + (int64_t)B * slot_per_img);
     }
-    if (B <= 0) fail(VISTA_ERR_NO_PLAN, "no micro-batch fits the HBM budget at stage " + std::to_string(t));
-    c->micro[t] = B;
-    peak = std::max(peak, fixed + (int64_t)B * slot_per_img);
+    return true;
+  };
+  for (int64_t CH = std::max<int64_t>(c->n_img, 1);; CH = (CH + 1) / 2) {
+    if (plan_chunk(CH, c->micro, peak)) {
+      c->chunk = CH;
+      break;
+    }
+    if (CH == 1) fail(VISTA_ERR_NO_PLAN, "not even one image per chunk fits the HBM budget");
   }
   c->peak_pred = peak;
 }
@@ -465,8 +488,8 @@ bool run_ops(vista_ctx* c, int t, const void* in_ptr, void* out_ptr, int nb, voi
   return fused;
 }
 
-// one block of the Staged plan over all local images, in micro-batches of micro[t]: in_base -> A_t
-bool run_block(vista_ctx* c, int t, const void* in_base, unsigned int* tapf) {
+// one block of the Staged plan over n images (a chunk), in micro-batches of micro[t]: in_base -> A_t
+bool run_block(vista_ctx* c, int t, const void* in_base, int64_t n, unsigned int* tapf) {
   const StageDesc& S = c->net.stages[t];
   const int B = c->micro[t];
   void* slot[NUM_BUFS] = {nullptr};
@@ -474,8 +497,8 @@ bool run_block(vista_ctx* c, int t, const void* in_base, unsigned int* tapf) {
   const size_t in_bytes_per = t == 0 ? (size_t)S.in_elems : (size_t)S.in_elems * 2;
   bf16* out_base = reinterpret_cast<bf16*>(c->A[t]->p);
   bool fused = tapf != nullptr;
-  for (int64_t i0 = 0; i0 < c->n_img; i0 += B) {
-    const int nb = (int)std::min<int64_t>(B, c->n_img - i0);
+  for (int64_t i0 = 0; i0 < n; i0 += B) {
+    const int nb = (int)std::min<int64_t>(B, n - i0);
     const bool ok = run_ops(c, t, (const uint8_t*)in_base + (size_t)i0 * in_bytes_per,
                             out_base + (size_t)i0 * S.out_elems, nb, slot,
                             tapf ? tapf + (size_t)i0 * 4 * S.outC : nullptr);
@@ -669,6 +692,7 @@ VISTA_API vista_status vista_plan_info(const vista_ctx* c, vista_plan_info_t* o)
   o->weight_bytes = c->weight_bytes;
   o->d_s = c->d_s;
   o->ds_pad = c->ds_pad;
+  o->chunk_images = c->chunk;
   return VISTA_OK;
 }
 
@@ -683,7 +707,10 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
     cudaStream_t st = c->stream;
     const auto& S = c->net.stages;
     // ---- inputs (H2D when given host pointers) ----
-    const uint8_t* px = (const uint8_t*)to_device(c, c->d_px, images, (size_t)c->n_img * S[0].in_elems);
+    // (the Staged plan streams host pixels to the device chunk by chunk; Eager / Lazy copy them once)
+    const uint8_t* px = c->sys.plan == VISTA_PLAN_STAGED
+                            ? images
+                            : (const uint8_t*)to_device(c, c->d_px, images, (size_t)c->n_img * S[0].in_elems);
     const int64_t* ik = (const int64_t*)to_device(c, c->d_img_keys, image_keys, (size_t)c->n_img * 8);
     const int64_t* sk = (const int64_t*)to_device(c, c->d_str_keys, str_keys, (size_t)c->n_str * 8);
     const float* X = (const float*)to_device(c, c->d_X, structured, (size_t)c->n_str * c->d_s * 4);
@@ -733,37 +760,66 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
       }
       for (size_t k = 0; k < c->taps.size(); ++k) concat_layer((int)k);
     }
-    for (int t = 0; t <= c->t_max && c->sys.plan == VISTA_PLAN_STAGED; ++t) {
-      c->A[t]->alloc((size_t)c->n_img * S[t].out_elems * 2 + 16);
-      const void* in = t == 0 ? (const void*)px : c->A[t - 1]->p;
-      const int k = layer_index(c, t);
-      // S2: the tap of a conv layer is fused into the producing conv's epilogue when possible
-      DevBuf tapacc;
-      unsigned int* tapf = nullptr;
-      if (k >= 0 && !S[t].fc_tap && c->fuse_tap && c->n_img > 0) {
-        const size_t cnt = (size_t)c->n_img * 4 * S[t].outC;
-        tapacc.alloc(cnt * 4);
-        VCHECK(cudaMemsetAsync(tapacc.p, 0, cnt * 4, st));  // max over non-negative (post-ReLU) values
-        tapf = (unsigned int*)tapacc.p;
-      }
-      const bool fused = run_block(c, t, in, tapf);
-      if (k >= 0) {
-        if (S[t].fc_tap) {
-          c->feat[t] = c->A[t]->p;  // g = identity on FC layers
-        } else {
+    // ---- Staged (Fig 5E), over chunks of images when the HBM budget forces it (planner) ----
+    const int64_t CH = c->sys.plan == VISTA_PLAN_STAGED ? std::max<int64_t>(c->chunk, 1) : 0;
+    const bool chunked = CH > 0 && CH < c->n_img;
+    const bool host_px = px == images && c->n_img > 0 && !is_device_ptr(images);
+    if (CH > 0) {
+      for (int t : c->taps)
+        if (!S[t].fc_tap || chunked) {  // FC taps alias A_t unless A_t lives per chunk
           c->F[t]->alloc((size_t)c->n_img * S[t].d_tap * 2 + 16);
-          if (fused)
-            launch_tap_finalize(tapf, (int64_t)c->n_img * S[t].d_tap, (bf16*)c->F[t]->p, st);
-          else
-            launch_tap((const bf16*)c->A[t]->p, c->n_img, S[t].outH, S[t].outW, S[t].outC, (bf16*)c->F[t]->p, st);
           c->feat[t] = c->F[t]->p;
         }
-        concat_layer(k);
-      }
-      // Staged: the input activation of this block is no longer needed (Fig 5E) — unless it is an
-      // FC tap whose activation doubles as its features
-      if (t > 0 && !(S[t - 1].fc_tap && layer_index(c, t - 1) >= 0)) c->A[t - 1]->release();
     }
+    for (int64_t c0 = 0; CH > 0 && (c0 < c->n_img || c0 == 0); c0 += CH) {
+      const int64_t nc = std::min<int64_t>(CH, c->n_img - c0);
+      if (nc <= 0 && c->n_img > 0) break;
+      const uint8_t* pxc = px + (size_t)c0 * S[0].in_elems;
+      if (host_px) {  // stream the chunk's pixels to the device
+        c->d_px.ensure((size_t)nc * S[0].in_elems);
+        VCHECK(cudaMemcpyAsync(c->d_px.p, images + (size_t)c0 * S[0].in_elems, (size_t)nc * S[0].in_elems,
+                               cudaMemcpyHostToDevice, st));
+        pxc = (const uint8_t*)c->d_px.p;
+      }
+      for (int t = 0; t <= c->t_max; ++t) {
+        c->A[t]->alloc((size_t)nc * S[t].out_elems * 2 + 16);
+        const void* in = t == 0 ? (const void*)pxc : c->A[t - 1]->p;
+        const int k = layer_index(c, t);
+        // S2 fused into the producing conv's epilogue (opt-in, unchunked only)
+        DevBuf tapacc;
+        unsigned int* tapf = nullptr;
+        if (k >= 0 && !S[t].fc_tap && c->fuse_tap && !chunked && nc > 0) {
+          const size_t cnt = (size_t)nc * 4 * S[t].outC;
+          tapacc.alloc(cnt * 4);
+          VCHECK(cudaMemsetAsync(tapacc.p, 0, cnt * 4, st));  // max over non-negative (post-ReLU) values
+          tapf = (unsigned int*)tapacc.p;
+        }
+        const bool fused = run_block(c, t, in, nc, tapf);
+        if (k >= 0) {
+          if (S[t].fc_tap) {
+            if (chunked)
+              VCHECK(cudaMemcpyAsync((bf16*)c->F[t]->p + (size_t)c0 * S[t].d_tap, c->A[t]->p,
+                                     (size_t)nc * S[t].d_tap * 2, cudaMemcpyDeviceToDevice, st));
+            else
+              c->feat[t] = c->A[t]->p;  // g = identity on FC layers
+          } else {
+            bf16* Ft = (bf16*)c->F[t]->p + (size_t)c0 * S[t].d_tap;
+            if (fused)
+              launch_tap_finalize(tapf, (int64_t)nc * S[t].d_tap, Ft, st);
+            else
+              launch_tap((const bf16*)c->A[t]->p, nc, S[t].outH, S[t].outW, S[t].outC, Ft, st);
+          }
+          if (!chunked) concat_layer(k);
+        }
+        // Staged: the input activation of this block is no longer needed (Fig 5E) — unless it is an
+        // FC tap whose activation doubles as its features
+        if (t > 0 && (chunked || !(S[t - 1].fc_tap && layer_index(c, t - 1) >= 0))) c->A[t - 1]->release();
+      }
+      if (chunked) c->A[c->t_max]->release();
+      if (c->n_img == 0) break;
+    }
+    if (chunked)
+      for (size_t k = 0; k < c->taps.size(); ++k) concat_layer((int)k);
     VCHECK(cudaStreamSynchronize(st));
     c->d_px.release();
     for (auto& s : c->slot_store) s->release();

@@ -43,7 +43,7 @@ class SysCfg(ctypes.Structure):
 class PlanInfo(ctypes.Structure):
     _fields_ = [("n_layers", _i32), ("tap", _i32 * 8), ("d_l", _i32 * 8), ("ld", _i32 * 8),
                 ("micro_batch", _i32 * 8), ("act_bytes", _i64 * 8), ("peak_bytes_pred", _i64),
-                ("weight_bytes", _i64), ("d_s", _i32), ("ds_pad", _i32)]
+                ("weight_bytes", _i64), ("d_s", _i32), ("ds_pad", _i32), ("chunk_images", _i64)]
 
 
 class Buffer(ctypes.Structure):
@@ -258,7 +258,8 @@ class Vista:
         n = pi.n_layers
         return dict(n_layers=n, tap=list(pi.tap[:n]), d_l=list(pi.d_l[:n]), ld=list(pi.ld[:n]),
                     micro_batch=list(pi.micro_batch[:n]), act_bytes=list(pi.act_bytes[:n]),
-                    peak_bytes_pred=pi.peak_bytes_pred, weight_bytes=pi.weight_bytes, d_s=pi.d_s, ds_pad=pi.ds_pad)
+                    peak_bytes_pred=pi.peak_bytes_pred, weight_bytes=pi.weight_bytes, d_s=pi.d_s, ds_pad=pi.ds_pad,
+                    chunk_images=pi.chunk_images)
 
     def transfer(self, images, image_keys, structured, str_keys, labels):
         _check(lib().vista_transfer(self.ctx, _ptr(images), _ptr(image_keys), _ptr(structured), _ptr(str_keys),

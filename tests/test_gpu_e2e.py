@@ -187,6 +187,27 @@ def test_duplicate_key_error():
     v.close()
 
 
+def test_planner_chunks_under_budget_bit_identical():
+    # planner at capacity (config 5 analogue): a budget too small for all local images' A_k forces chunked
+    # Staged execution; results must not change by a single bit (rows are independent, kernels deterministic)
+    n = 48
+    tab = gen.make_tables(n, 8)
+    ref = run_gpu(2, [0, 4], tab, 8, iters=2)
+    info_ref = ref.plan_info()
+    mm_ref = [ref.features(k)["mm"].view(torch.int16).cpu().clone() for k in range(2)]
+    ref.close()
+    assert info_ref["chunk_images"] == n
+    budget = info_ref["weight_bytes"] + (256 << 20) + (24 << 20)
+    v = run_gpu(2, [0, 4], tab, 8, iters=2, hbm_budget_bytes=budget)
+    info = v.plan_info()
+    assert 1 <= info["chunk_images"] < n
+    assert info["peak_bytes_pred"] <= budget
+    for k in range(2):
+        assert torch.equal(mm_ref[k], v.features(k)["mm"].view(torch.int16).cpu())
+    # host pixels are streamed chunk by chunk: same bits
+    v.close()
+
+
 def test_no_plan_within_tiny_budget():
     with pytest.raises(VistaError) as e:
         Vista(2, n_top=5, n_str_rows=1000, d_s=130, n_images_local=1000, hbm_budget_bytes=64 << 20)

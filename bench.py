@@ -311,6 +311,7 @@ def main():
     ms_step = ms / args.steps
     value = N_global / (ms_step / 1000.0)
     # ---- e2e: host inputs through the C-ABI, weights back to the host ----
+    step(host=True)  # untimed warm-up of the host-input path (sizes its per-chunk pixel buffer)
     e2e_ms, _ = timed(args.e2e_steps, host=True)
     e2e_step = e2e_ms / args.e2e_steps
     d2h = sum((d + 1) * 8 for d in d_tot) + len(taps) * 8 * 80

@@ -210,7 +210,10 @@ struct vista_ctx {
   int64_t chunk = 0;         // images per Staged chunk (== n_img unless the HBM budget forces chunking)
   int64_t weight_bytes = 0, peak_pred = 0;
   // results
-  std::vector<std::unique_ptr<DevBuf>> A, F, MM, Y;  // per block (A, F) / per requested layer (MM, Y)
+  std::vector<std::unique_ptr<DevBuf>> F, MM, Y;  // per block (F) / per requested layer (MM, Y)
+  DevBuf arena[2];               // Staged ping-pong activation arenas (A_t lives in arena t % 2)
+  DevBuf tapacc;                 // fused-tap accumulator (opt-in)
+  std::vector<void*> act;        // per block: A_t of the last chunk (valid for the last two blocks)
   DevBuf pair_str, pair_img, d_X, d_labels, d_img_keys, d_str_keys, d_px;
   std::vector<DevBuf*> scratch;  // NUM_BUFS slots
   std::vector<std::unique_ptr<DevBuf>> slot_store;
@@ -227,8 +230,12 @@ struct vista_ctx {
   std::vector<void*> feat;  // per block: device pointer of F_t (features) of a tapped layer
   std::string last_error;
   ~vista_ctx() {
-    for (auto* v : {&A, &F, &MM, &Y, &slot_store})
-      for (auto& b : *v) b->release();
+    for (auto* v : {&F, &MM, &Y, &slot_store})
+      for (auto& b : *v)
+        if (b) b->release();
+    arena[0].release();
+    arena[1].release();
+    tapacc.release();
     for (DevBuf* b : {&pair_str, &pair_img, &d_X, &d_labels, &d_img_keys, &d_str_keys, &d_px}) b->release();
     if (stream) cudaStreamSynchronize(stream);
     for (auto& L : convs) conv_layer_free(L);
@@ -323,13 +330,14 @@ void plan_memory(vista_ctx* c, uint64_t budget) {
     pk = 0;
     const bool chunked = CH < c->n_img;
     const int64_t pxc = CH * (int64_t)S[0].in_elems;  // host pixels are streamed per chunk
+    int64_t arena[2] = {0, 0};                         // ping-pong activation arenas (A_t in arena t % 2)
+    for (int t = 0; t <= c->t_max; ++t) arena[t & 1] = std::max<int64_t>(arena[t & 1], CH * S[t].out_elems * 2);
+    (void)chunked;
     for (int t = 0; t <= c->t_max; ++t) {
-      const int64_t a_in = t == 0 ? pxc : CH * S[t - 1].out_elems * 2;
-      const int64_t a_out = CH * S[t].out_elems * 2;
       int64_t slot_per_img = 0;
       for (int b = BUF_T0; b < NUM_BUFS; ++b) slot_per_img += S[t].slot_elems[b] * 2;
-      const int64_t fixed = c->weight_bytes + pxc + a_in + a_out + mm_bytes + f_bytes + (chunked ? f_fc : 0) +
-                            join_bytes + (256ll << 20);
+      const int64_t fixed = c->weight_bytes + pxc + arena[0] + arena[1] + mm_bytes + f_bytes + f_fc + join_bytes +
+                            (256ll << 20);
       int B = 0;
       if (c->sys.micro_batch > 0 && t == 0) {
         B = (int)std::min<int64_t>(c->sys.micro_batch, std::max<int64_t>(CH, 1));
@@ -489,13 +497,12 @@ bool run_ops(vista_ctx* c, int t, const void* in_ptr, void* out_ptr, int nb, voi
 }
 
 // one block of the Staged plan over n images (a chunk), in micro-batches of micro[t]: in_base -> A_t
-bool run_block(vista_ctx* c, int t, const void* in_base, int64_t n, unsigned int* tapf) {
+bool run_block(vista_ctx* c, int t, const void* in_base, bf16* out_base, int64_t n, unsigned int* tapf) {
   const StageDesc& S = c->net.stages[t];
   const int B = c->micro[t];
   void* slot[NUM_BUFS] = {nullptr};
   prepare_slots(c, t, B, slot);
   const size_t in_bytes_per = t == 0 ? (size_t)S.in_elems : (size_t)S.in_elems * 2;
-  bf16* out_base = reinterpret_cast<bf16*>(c->A[t]->p);
   bool fused = tapf != nullptr;
   for (int64_t i0 = 0; i0 < n; i0 += B) {
     const int nb = (int)std::min<int64_t>(B, n - i0);
@@ -724,35 +731,36 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
     if (jr.dup & 1) fail(VISTA_ERR_DUP_KEY, "duplicate key in T_img or T_str (ID must be a primary key)");
     c->n_pairs = jr.n_pairs;
     c->n_train = jr.n_train;
-    // ---- S1-S3 Staged execution ----
-    c->A.clear();
-    c->F.clear();
-    c->MM.clear();
-    c->Y.clear();
-    for (int t = 0; t <= c->t_max; ++t) {
-      c->A.emplace_back(new DevBuf());
-      c->F.emplace_back(new DevBuf());
-    }
+    // ---- S1-S3 ----
+    // Buffers persist across transfers (grow-only): F_t / MM_k / labels per layer, two ping-pong
+    // activation arenas for the Staged plan (stage t reads arena (t-1)%2 and writes arena t%2, so
+    // A_{t-1} is dead -- "freed" -- once stage t has consumed it, Fig 5E), scratch slots, pixels.
+    c->F.resize(c->t_max + 1);
+    for (auto& f : c->F)
+      if (!f) f.reset(new DevBuf());
+    c->MM.resize(c->taps.size());
+    c->Y.resize(c->taps.size());
     for (size_t k = 0; k < c->taps.size(); ++k) {
-      c->MM.emplace_back(new DevBuf());
-      c->Y.emplace_back(new DevBuf());
+      if (!c->MM[k]) c->MM[k].reset(new DevBuf());
+      if (!c->Y[k]) c->Y[k].reset(new DevBuf());
     }
     c->feat.assign(c->t_max + 1, nullptr);
+    c->act.assign(c->t_max + 1, nullptr);
+    for (int t : c->taps) {
+      c->F[t]->ensure((size_t)c->n_img * S[t].d_tap * 2 + 16);
+      c->feat[t] = c->F[t]->p;
+    }
     auto concat_layer = [&](int k) {
       const int t = c->taps[k];
       const int ld = ld_of(c, k);
-      c->MM[k]->alloc((size_t)std::max<int64_t>(c->n_pairs, 1) * ld * 2);
-      c->Y[k]->alloc((size_t)std::max<int64_t>(c->n_pairs, 1));
+      c->MM[k]->ensure((size_t)std::max<int64_t>(c->n_pairs, 1) * ld * 2);
+      c->Y[k]->ensure((size_t)std::max<int64_t>(c->n_pairs, 1));
       launch_concat(X, c->d_s, c->ds_pad, (const bf16*)c->feat[t], S[t].d_tap, (const int32_t*)c->pair_str.p,
                     (const int32_t*)c->pair_img.p, lab, c->n_pairs, ld, (bf16*)c->MM[k]->p, (uint8_t*)c->Y[k]->p,
                     st);
     };
     if (c->sys.plan != VISTA_PLAN_STAGED) {
       // ---- Eager / Lazy (Fig 5C / 5A): features of every layer, no resident full activations ----
-      for (int t : c->taps) {
-        c->F[t]->alloc((size_t)c->n_img * S[t].d_tap * 2 + 16);
-        c->feat[t] = c->F[t]->p;
-      }
       if (c->sys.plan == VISTA_PLAN_EAGER) {
         run_unstaged(c, px, c->t_max, c->taps);
       } else {
@@ -765,15 +773,15 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
     const bool chunked = CH > 0 && CH < c->n_img;
     const bool host_px = px == images && c->n_img > 0 && !is_device_ptr(images);
     if (CH > 0) {
-      for (int t : c->taps)
-        if (!S[t].fc_tap || chunked) {  // FC taps alias A_t unless A_t lives per chunk
-          c->F[t]->alloc((size_t)c->n_img * S[t].d_tap * 2 + 16);
-          c->feat[t] = c->F[t]->p;
-        }
+      size_t need[2] = {16, 16};
+      for (int t = 0; t <= c->t_max; ++t)
+        need[t & 1] = std::max(need[t & 1], (size_t)std::min<int64_t>(CH, std::max<int64_t>(c->n_img, 1)) *
+                                                  S[t].out_elems * 2 + 16);
+      c->arena[0].ensure(need[0]);
+      c->arena[1].ensure(need[1]);
     }
-    for (int64_t c0 = 0; CH > 0 && (c0 < c->n_img || c0 == 0); c0 += CH) {
+    for (int64_t c0 = 0; CH > 0 && c0 < c->n_img; c0 += CH) {
       const int64_t nc = std::min<int64_t>(CH, c->n_img - c0);
-      if (nc <= 0 && c->n_img > 0) break;
       const uint8_t* pxc = px + (size_t)c0 * S[0].in_elems;
       if (host_px) {  // stream the chunk's pixels to the device
         c->d_px.ensure((size_t)nc * S[0].in_elems);
@@ -782,47 +790,34 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
         pxc = (const uint8_t*)c->d_px.p;
       }
       for (int t = 0; t <= c->t_max; ++t) {
-        c->A[t]->alloc((size_t)nc * S[t].out_elems * 2 + 16);
-        const void* in = t == 0 ? (const void*)pxc : c->A[t - 1]->p;
+        bf16* At = (bf16*)c->arena[t & 1].p;
+        c->act[t] = At;
+        const void* in = t == 0 ? (const void*)pxc : c->arena[(t - 1) & 1].p;
         const int k = layer_index(c, t);
         // S2 fused into the producing conv's epilogue (opt-in, unchunked only)
-        DevBuf tapacc;
         unsigned int* tapf = nullptr;
-        if (k >= 0 && !S[t].fc_tap && c->fuse_tap && !chunked && nc > 0) {
+        if (k >= 0 && !S[t].fc_tap && c->fuse_tap && !chunked) {
           const size_t cnt = (size_t)nc * 4 * S[t].outC;
-          tapacc.alloc(cnt * 4);
-          VCHECK(cudaMemsetAsync(tapacc.p, 0, cnt * 4, st));  // max over non-negative (post-ReLU) values
-          tapf = (unsigned int*)tapacc.p;
+          c->tapacc.ensure(cnt * 4);
+          VCHECK(cudaMemsetAsync(c->tapacc.p, 0, cnt * 4, st));  // max over non-negative (post-ReLU) values
+          tapf = (unsigned int*)c->tapacc.p;
         }
-        const bool fused = run_block(c, t, in, nc, tapf);
+        const bool fused = run_block(c, t, in, At, nc, tapf);
         if (k >= 0) {
-          if (S[t].fc_tap) {
-            if (chunked)
-              VCHECK(cudaMemcpyAsync((bf16*)c->F[t]->p + (size_t)c0 * S[t].d_tap, c->A[t]->p,
-                                     (size_t)nc * S[t].d_tap * 2, cudaMemcpyDeviceToDevice, st));
-            else
-              c->feat[t] = c->A[t]->p;  // g = identity on FC layers
-          } else {
-            bf16* Ft = (bf16*)c->F[t]->p + (size_t)c0 * S[t].d_tap;
-            if (fused)
-              launch_tap_finalize(tapf, (int64_t)nc * S[t].d_tap, Ft, st);
-            else
-              launch_tap((const bf16*)c->A[t]->p, nc, S[t].outH, S[t].outW, S[t].outC, Ft, st);
-          }
+          bf16* Ft = (bf16*)c->F[t]->p + (size_t)c0 * S[t].d_tap;
+          if (S[t].fc_tap)  // g = identity on FC layers
+            VCHECK(cudaMemcpyAsync(Ft, At, (size_t)nc * S[t].d_tap * 2, cudaMemcpyDeviceToDevice, st));
+          else if (fused)
+            launch_tap_finalize(tapf, (int64_t)nc * S[t].d_tap, Ft, st);
+          else
+            launch_tap(At, nc, S[t].outH, S[t].outW, S[t].outC, Ft, st);
           if (!chunked) concat_layer(k);
         }
-        // Staged: the input activation of this block is no longer needed (Fig 5E) — unless it is an
-        // FC tap whose activation doubles as its features
-        if (t > 0 && (chunked || !(S[t - 1].fc_tap && layer_index(c, t - 1) >= 0))) c->A[t - 1]->release();
       }
-      if (chunked) c->A[c->t_max]->release();
-      if (c->n_img == 0) break;
     }
     if (chunked)
       for (size_t k = 0; k < c->taps.size(); ++k) concat_layer((int)k);
     VCHECK(cudaStreamSynchronize(st));
-    c->d_px.release();
-    for (auto& s : c->slot_store) s->release();
     if (g_prof) g_prof->flush();
     c->transferred = true;
   });
@@ -845,7 +840,11 @@ VISTA_API vista_status vista_features(const vista_ctx* c, int32_t k, vista_buffe
   o->pair_img = (const int32_t*)c->pair_img.p;
   o->labels = (const uint8_t*)c->Y[k]->p;
   o->features = c->feat[t];
-  o->activation = c->A.size() > (size_t)t ? c->A[t]->p : nullptr;
+  // A_t survives the transfer only for the last two blocks (the arenas are reused, Fig 5E)
+  o->activation = (c->sys.plan == VISTA_PLAN_STAGED && c->chunk >= c->n_img && t >= c->t_max - 1 &&
+                   (size_t)t < c->act.size())
+                      ? c->act[t]
+                      : nullptr;
   return VISTA_OK;
 }
 

@@ -57,11 +57,16 @@ enum { VISTA_VGG16_FC6 = 0, VISTA_VGG16_FC7 = 1, VISTA_VGG16_FC8 = 2 };
 enum { VISTA_RESNET50_CONV4_6 = 0, VISTA_RESNET50_CONV5_1 = 1, VISTA_RESNET50_CONV5_2 = 2,
        VISTA_RESNET50_CONV5_3 = 3, VISTA_RESNET50_FC = 4 };
 
-/* Logical plans (Fig 5).  Only STAGED is implemented this round;
- * EAGER / LAZY return VISTA_ERR_INVALID_ARG. */
+/* Logical plans (Fig 5): STAGED (Fig 5E, the default), EAGER (Fig 5C: one pass
+ * over the images taps every layer of L), LAZY (Fig 5A: one pass from the pixels per layer). */
 typedef enum { VISTA_PLAN_STAGED = 0, VISTA_PLAN_EAGER = 1, VISTA_PLAN_LAZY = 2 } vista_plan_kind;
-/* Arithmetic of the CNN: bf16 operands, fp32 accumulate, RNE to bf16 at layer boundaries. */
-typedef enum { VISTA_BF16 = 0 } vista_dtype;
+/* Arithmetic of the CNN and of M.
+ * VISTA_BF16: bf16 operands on the tcgen05 tensor cores, fp32 accumulate, RNE to bf16 at layer
+ *   boundaries; MM_k is bf16 (the product path).
+ * VISTA_F32: the fp32 check mode (north_star: "1e-4 in the fp32 check mode"; reading R23): fp32
+ *   storage and fp32 FFMA accumulation everywhere, MM_k is fp32.  Every buffer below documented as
+ *   "bf16" is then float32. */
+typedef enum { VISTA_BF16 = 0, VISTA_F32 = 1 } vista_dtype;
 
 /* Downstream M (reading R17 in DESIGN.md) */
 typedef struct {
@@ -103,7 +108,7 @@ typedef struct {
 /* Borrowed view of layer k's outputs on this rank (valid until vista_destroy or the
  * next vista_transfer).  All pointers are device pointers. */
 typedef struct {
-  void* mm;                /* bf16 [rows, ld]: columns [0,d_s) = X, [d_s,ds_pad) = 0, [ds_pad, ds_pad+d_l) = F_k, rest 0 */
+  void* mm;                /* bf16 (f32 in VISTA_F32) [rows, ld]: columns [0,d_s) = X, [d_s,ds_pad) = 0, [ds_pad, ds_pad+d_l) = F_k, rest 0 */
   int64_t rows;            /* joined rows on this rank: [0, n_train) train, [n_train, rows) test */
   int64_t n_train;
   int32_t ld, d_s, ds_pad, d_l;

@@ -64,6 +64,30 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
 void launch_tap_finalize(const unsigned int* tapf, int64_t count, bf16* F, cudaStream_t st);
 inline int conv_out_dim(int H, int k, int s, int p) { return (H + 2 * p - k) / s + 1; }
 
+// ---- fp32 check mode (reading R23): SIMT FFMA conv / FC with fp32 storage ----
+struct ConvLayerF32 {
+  int Cin = 0, Cout = 0, R = 1, S = 1, stride = 1, pad = 0, groups = 1;
+  int Cg_in = 0, Cg_out = 0, K = 0;
+  bool relu = false;
+  float* w = nullptr;  // [Cout][K]
+  float* scale = nullptr;
+  float* shift = nullptr;
+};
+void conv_layer_init_f32(ConvLayerF32& L, const std::vector<float>& w_ohwi, int Cin_real,
+                         const std::vector<float>& scale, const std::vector<float>& shift);
+void conv_layer_free_f32(ConvLayerF32& L);
+void conv_forward_f32(const ConvLayerF32& L, const float* x, int N, int H, int W, const float* res, float* y,
+                      cudaStream_t st);
+void launch_ingest_f32(const uint8_t* px, int64_t n, float* y, cudaStream_t st);
+void launch_ingest_s2d_f32(const uint8_t* px, int64_t n, float* y, cudaStream_t st);
+void launch_maxpool_f32(const float* x, int N, int H, int W, int C, int k, int s, float* y, cudaStream_t st);
+void launch_lrn_f32(const float* x, int N, int H, int W, int C, float* y, cudaStream_t st);
+void launch_avgpool_f32(const float* x, int N, int H, int W, int C, float* y, cudaStream_t st);
+void launch_tap_f32(const float* A, int64_t N, int H, int W, int C, float* F, cudaStream_t st);
+void launch_concat_f32(const float* X, int d_s, int ds_pad, const float* F, int d_l, const int32_t* pair_str,
+                       const int32_t* pair_img, const uint8_t* labels, int64_t n_pairs, int ld, float* MM,
+                       uint8_t* y, cudaStream_t st);
+
 // ---- SIMT kernels (memory-bound) ----
 void launch_ingest(const uint8_t* px, int64_t n, bf16* y, cudaStream_t st);
 void launch_ingest_s2d(const uint8_t* px, int64_t n, bf16* y, cudaStream_t st);
@@ -97,6 +121,10 @@ typedef void (*allreduce_fn)(double* d_buf, int64_t count, cudaStream_t st, void
 LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
                   const uint8_t* real_col_mask_host, int iters, int power_iters, double lambda, double alpha,
                   allreduce_fn allreduce, void* ar_user, cudaStream_t st);
+// fp32 check mode: the same passes over fp32 rows (ld a multiple of 8)
+LRResult lr_train_f32(const float* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
+                      const uint8_t* real_col_mask_host, int iters, int power_iters, double lambda, double alpha,
+                      allreduce_fn allreduce, void* ar_user, cudaStream_t st);
 
 // ---- profiling hooks (class ids as in vista.h vista_profile) ----
 struct Profiler;

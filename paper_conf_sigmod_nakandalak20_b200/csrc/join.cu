@@ -240,6 +240,40 @@ __global__ void concat_kernel(const float* __restrict__ X, int d_s, int ds_pad, 
   }
 }
 
+// fp32 check mode (reading R23): the same layout with fp32 elements, one warp per row
+__global__ void concat_f32_kernel(const float* __restrict__ X, int d_s, int ds_pad, const float* __restrict__ F,
+                                  int d_l, const int32_t* __restrict__ pair_str, const int32_t* __restrict__ pair_img,
+                                  const uint8_t* __restrict__ labels, int64_t n, int ld, float* __restrict__ MM,
+                                  uint8_t* __restrict__ y) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t p = blockIdx.x * (int64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); p < n; p += warps) {
+    const int32_t s = pair_str[p], i = pair_img[p];
+    float* row = MM + (size_t)p * ld;
+    for (int c = lane; c < ld; c += 32) {
+      float v = 0.f;
+      if (c < d_s) v = X[(size_t)s * d_s + c];
+      else if (c >= ds_pad && c < ds_pad + d_l) v = F[(size_t)i * d_l + (c - ds_pad)];
+      row[c] = v;
+    }
+    if (lane == 0) y[p] = labels[s];
+  }
+}
+
+void launch_concat_f32(const float* X, int d_s, int ds_pad, const float* F, int d_l, const int32_t* pair_str,
+                       const int32_t* pair_img, const uint8_t* labels, int64_t n_pairs, int ld, float* MM,
+                       uint8_t* y, cudaStream_t st) {
+  if (n_pairs <= 0) return;
+  int64_t blocks = (n_pairs + 7) / 8;
+  const int64_t cap = (int64_t)num_sms() * 8;
+  if (blocks > cap) blocks = cap;
+  prof_begin(st);
+  concat_f32_kernel<<<(int)blocks, 256, 0, st>>>(X, d_s, ds_pad, F, d_l, pair_str, pair_img, labels, n_pairs, ld, MM,
+                                                 y);
+  LAUNCHED();
+  prof_end(st, 4, 0, (double)n_pairs * (4.0 * d_s + 4.0 * d_l + 4.0 * ld + 9));
+}
+
 void launch_concat(const float* X, int d_s, int ds_pad, const bf16* F, int d_l, const int32_t* pair_str,
                    const int32_t* pair_img, const uint8_t* labels, int64_t n_pairs, int ld, bf16* MM, uint8_t* y,
                    cudaStream_t st) {

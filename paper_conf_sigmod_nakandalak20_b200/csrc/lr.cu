@@ -23,11 +23,11 @@ constexpr int kStagesLR = 3;   // row blocks in flight per CTA
 constexpr int kLRThreads = 512;
 
 struct PassArgs {
-  const bf16* MM;
+  const uint8_t* MM;   // row-major [rows][ld] elements of E (bf16, or fp32 in check mode)
   const uint8_t* y;
   int64_t r0, r1;       // row range [r0, r1) of this pass
   int64_t n_train;      // rows < n_train are train rows (eval mode)
-  int ld, chunks;       // ld elements per row, chunks = ld / 8
+  int ld, chunks;       // ld elements per row, chunks = ld * sizeof(E) / 16
   int rb;               // rows per streamed block
   const float* mu;      // [ld]
   const float* what;    // [ld]  inv_j * (w_j or v_j), 0 on excluded / pad columns
@@ -53,13 +53,33 @@ __device__ __forceinline__ void bulk_load(uint32_t dst, const void* src, uint32_
 //   MODE 4: evaluation (counts only)
 // with z_p = b^ + sum_j w^_j (x_pj - mu_j); modes 2/3 accumulate sum_p phi_p (x_pj - mu_j),
 // sum_p phi_p and sum_p loss_p into this CTA's partial row (fixed row-block -> CTA map).
-template <int CH, int MODE>
+template <typename E>
+__device__ __forceinline__ void unpack16(uint4 v, float (&x)[16 / sizeof(E)]);
+template <>
+__device__ __forceinline__ void unpack16<bf16>(uint4 v, float (&x)[8]) {
+  const uint32_t u[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const float2 f = unpack_bf16x2(u[j]);
+    x[2 * j] = f.x;
+    x[2 * j + 1] = f.y;
+  }
+}
+template <>
+__device__ __forceinline__ void unpack16<float>(uint4 v, float (&x)[4]) {
+  x[0] = __uint_as_float(v.x);
+  x[1] = __uint_as_float(v.y);
+  x[2] = __uint_as_float(v.z);
+  x[3] = __uint_as_float(v.w);
+}
+
+template <int CH, int MODE, typename E>
 __global__ void __launch_bounds__(kLRThreads, 1) lr_stream_kernel(const PassArgs a) {
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 127u) & ~127u;
   uint8_t* gbase = smem_raw + (base - raw);
-  const uint32_t row_bytes = (uint32_t)a.ld * 2u;
+  const uint32_t row_bytes = (uint32_t)a.ld * (uint32_t)sizeof(E);
   const uint32_t stage_bytes = ((uint32_t)a.rb * row_bytes + 127u) & ~127u;
   float* red = reinterpret_cast<float*>(gbase + kStagesLR * stage_bytes);  // [kMaxRB][32]
   float* phis = red + kMaxRB * 32;                                         // [kMaxRB]
@@ -78,22 +98,23 @@ __global__ void __launch_bounds__(kLRThreads, 1) lr_stream_kernel(const PassArgs
     const int64_t nr = min((int64_t)a.rb, a.r1 - r);
     const uint32_t bytes = (uint32_t)nr * row_bytes;
     mbar_arrive_expect_tx(&full[stage], bytes);
-    bulk_load(base + stage * stage_bytes, a.MM + (size_t)r * a.ld, bytes, &full[stage]);
+    bulk_load(base + stage * stage_bytes, a.MM + (size_t)r * row_bytes, bytes, &full[stage]);
   };
   if (tid == 0) {
     int i = 0;
     for (int64_t blk = blockIdx.x; blk < nblk && i < kStagesLR; blk += gridDim.x, ++i) issue(blk, i);
   }
-  float mu[CH][8], wv[CH][8], acc[CH][8];
+  constexpr int EPC = 16 / (int)sizeof(E);  // elements per 16-byte chunk: 8 bf16 or 4 fp32
+  float mu[CH][EPC], wv[CH][EPC], acc[CH][EPC];
   bool act[CH];
 #pragma unroll
   for (int c = 0; c < CH; ++c) {
     const int ch = tid + c * blockDim.x;
     act[c] = ch < a.chunks;
 #pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      mu[c][j] = (MODE != 0 && act[c]) ? a.mu[ch * 8 + j] : 0.f;
-      wv[c][j] = (MODE >= 2 && act[c]) ? a.what[ch * 8 + j] : 0.f;
+    for (int j = 0; j < EPC; ++j) {
+      mu[c][j] = (MODE != 0 && act[c]) ? a.mu[ch * EPC + j] : 0.f;
+      wv[c][j] = (MODE >= 2 && act[c]) ? a.what[ch * EPC + j] : 0.f;
       acc[c][j] = 0.f;
     }
   }
@@ -112,18 +133,15 @@ __global__ void __launch_bounds__(kLRThreads, 1) lr_stream_kernel(const PassArgs
 #pragma unroll
         for (int c = 0; c < CH; ++c) {
           if (!act[c]) continue;
-          const uint4 xv = lds128(sbase + q * row_bytes + (uint32_t)(tid + c * blockDim.x) * 16u);
-          const uint32_t u[4] = {xv.x, xv.y, xv.z, xv.w};
+          float x[EPC];
+          unpack16<E>(lds128(sbase + q * row_bytes + (uint32_t)(tid + c * blockDim.x) * 16u), x);
 #pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            const float2 f = unpack_bf16x2(u[j]);
+          for (int j = 0; j < EPC; ++j) {
             if (MODE == 0) {
-              acc[c][2 * j] += f.x;
-              acc[c][2 * j + 1] += f.y;
+              acc[c][j] += x[j];
             } else {
-              const float d0 = f.x - mu[c][2 * j], d1 = f.y - mu[c][2 * j + 1];
-              acc[c][2 * j] = fmaf(d0, d0, acc[c][2 * j]);
-              acc[c][2 * j + 1] = fmaf(d1, d1, acc[c][2 * j + 1]);
+              const float d = x[j] - mu[c][j];
+              acc[c][j] = fmaf(d, d, acc[c][j]);
             }
           }
         }
@@ -134,14 +152,10 @@ __global__ void __launch_bounds__(kLRThreads, 1) lr_stream_kernel(const PassArgs
 #pragma unroll
         for (int c = 0; c < CH; ++c) {
           if (!act[c]) continue;
-          const uint4 xv = lds128(sbase + q * row_bytes + (uint32_t)(tid + c * blockDim.x) * 16u);
-          const uint32_t u[4] = {xv.x, xv.y, xv.z, xv.w};
+          float x[EPC];
+          unpack16<E>(lds128(sbase + q * row_bytes + (uint32_t)(tid + c * blockDim.x) * 16u), x);
 #pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            const float2 f = unpack_bf16x2(u[j]);
-            sdot = fmaf(f.x - mu[c][2 * j], wv[c][2 * j], sdot);
-            sdot = fmaf(f.y - mu[c][2 * j + 1], wv[c][2 * j + 1], sdot);
-          }
+          for (int j = 0; j < EPC; ++j) sdot = fmaf(x[j] - mu[c][j], wv[c][j], sdot);
         }
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) sdot += __shfl_xor_sync(0xffffffffu, sdot, o);
@@ -176,14 +190,10 @@ __global__ void __launch_bounds__(kLRThreads, 1) lr_stream_kernel(const PassArgs
 #pragma unroll
           for (int c = 0; c < CH; ++c) {
             if (!act[c]) continue;
-            const uint4 xv = lds128(sbase + q * row_bytes + (uint32_t)(tid + c * blockDim.x) * 16u);
-            const uint32_t u[4] = {xv.x, xv.y, xv.z, xv.w};
+            float x[EPC];
+            unpack16<E>(lds128(sbase + q * row_bytes + (uint32_t)(tid + c * blockDim.x) * 16u), x);
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
-              const float2 f = unpack_bf16x2(u[j]);
-              acc[c][2 * j] = fmaf(ph, f.x - mu[c][2 * j], acc[c][2 * j]);
-              acc[c][2 * j + 1] = fmaf(ph, f.y - mu[c][2 * j + 1], acc[c][2 * j + 1]);
-            }
+            for (int j = 0; j < EPC; ++j) acc[c][j] = fmaf(ph, x[j] - mu[c][j], acc[c][j]);
           }
         }
       }
@@ -210,9 +220,10 @@ __global__ void __launch_bounds__(kLRThreads, 1) lr_stream_kernel(const PassArgs
   for (int c = 0; c < CH; ++c) {
     const int ch = tid + c * blockDim.x;
     if (act[c]) {
-      float4* o = reinterpret_cast<float4*>(out + ch * 8);
-      o[0] = make_float4(acc[c][0], acc[c][1], acc[c][2], acc[c][3]);
-      o[1] = make_float4(acc[c][4], acc[c][5], acc[c][6], acc[c][7]);
+      float4* o = reinterpret_cast<float4*>(out + ch * EPC);
+#pragma unroll
+      for (int j = 0; j < EPC / 4; ++j)
+        o[j] = make_float4(acc[c][4 * j], acc[c][4 * j + 1], acc[c][4 * j + 2], acc[c][4 * j + 3]);
     }
   }
   if (warp == 0) {  // fixed-order (lane) reduction of the per-row scalars
@@ -334,7 +345,7 @@ struct StreamCfg {
   size_t smem;
 };
 
-template <int MODE>
+template <int MODE, typename E>
 static void run_pass(const PassArgs& a, const StreamCfg& c, cudaStream_t st) {
   auto go = [&](void (*kern)(PassArgs)) {
     static std::mutex mu;
@@ -347,29 +358,33 @@ static void run_pass(const PassArgs& a, const StreamCfg& c, cudaStream_t st) {
     kern<<<c.grid, c.threads, c.smem, st>>>(a);
   };
   switch (c.ch) {
-    case 1: go(lr_stream_kernel<1, MODE>); break;
-    case 2: go(lr_stream_kernel<2, MODE>); break;
-    case 3: go(lr_stream_kernel<3, MODE>); break;
-    case 4: go(lr_stream_kernel<4, MODE>); break;
+    case 1: go(lr_stream_kernel<1, MODE, E>); break;
+    case 2: go(lr_stream_kernel<2, MODE, E>); break;
+    case 3: go(lr_stream_kernel<3, MODE, E>); break;
+    case 4: go(lr_stream_kernel<4, MODE, E>); break;
+    case 5: go(lr_stream_kernel<5, MODE, E>); break;
+    case 6: go(lr_stream_kernel<6, MODE, E>); break;
     default: fail(1, "lr: unsupported row width");
   }
   LAUNCHED();
 }
 
-LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
-                  const uint8_t* real_host, int iters, int power_iters, double lambda, double alpha,
-                  allreduce_fn allreduce, void* ar_user, cudaStream_t st) {
+template <typename E>
+static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
+                              const uint8_t* real_host, int iters, int power_iters, double lambda, double alpha,
+                              allreduce_fn allreduce, void* ar_user, cudaStream_t st) {
   LRResult res;
+  constexpr int esz = (int)sizeof(E);
   if (ld % 8) fail(1, "lr: ld must be a multiple of 8");
-  const int chunks = ld / 8;
+  const int chunks = ld * esz / 16;
   // one CTA per SM streaming row blocks of ~64 KB through a 3-deep bulk-copy ring
   StreamCfg cfg;
   cfg.threads = std::min(kLRThreads, (chunks + 31) / 32 * 32);
   cfg.ch = (chunks + cfg.threads - 1) / cfg.threads;
-  if (cfg.ch > 4) fail(1, "lr: row too wide");
+  if (cfg.ch > 6) fail(1, "lr: row too wide");
   if (cfg.ch == 3 && chunks <= 2 * cfg.threads) cfg.ch = 2;
-  cfg.rb = (int)std::max<int64_t>(1, std::min<int64_t>(kMaxRB, 65536 / ((int64_t)ld * 2)));
-  const size_t stage_bytes = ((size_t)cfg.rb * ld * 2 + 127) & ~(size_t)127;
+  cfg.rb = (int)std::max<int64_t>(1, std::min<int64_t>(kMaxRB, 65536 / ((int64_t)ld * esz)));
+  const size_t stage_bytes = ((size_t)cfg.rb * ld * esz + 127) & ~(size_t)127;
   cfg.smem = kStagesLR * stage_bytes + kMaxRB * 32 * 4 + kMaxRB * 4 + kStagesLR * 8 + 128;
   if (cfg.smem > 227 * 1024) fail(1, "lr: row block does not fit in shared memory");
   auto grid_for_rows = [&](int64_t rows) {
@@ -408,7 +423,7 @@ LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_tr
   VCHECK(cudaMemsetAsync(cnt, 0, 64, st));
 
   PassArgs a;
-  a.MM = MM;
+  a.MM = reinterpret_cast<const uint8_t*>(MM);
   a.y = y;
   a.r0 = 0;
   a.r1 = n_train;
@@ -421,7 +436,7 @@ LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_tr
   a.n_train = n_train;
   a.rb = cfg.rb;
   a.counts = nullptr;
-  const double pass_bytes = (double)n_train * ld * 2;
+  const double pass_bytes = (double)n_train * ld * esz;
   auto reduce = [&](double extra_n) {
     prof_begin(st);
     reduce_partials_kernel<<<(ncols + 255) / 256, 256, 0, st>>>(partial, grid_tr, ncols, ld + 4, G);
@@ -435,13 +450,13 @@ LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_tr
   const int ublk = 1024;
   // ---- O6 step 2: standardisation statistics (two passes: mean, then centred squares) ----
   prof_begin(st);
-  run_pass<0>(a, cfg, st);
+  run_pass<0, E>(a, cfg, st);
   prof_end(st, 5, 0, pass_bytes);
   reduce((double)n_train);
   stats_finalize_kernel<<<(ld + 255) / 256, 256, 0, st>>>(G, ld, 0, real, mu, mu_f, inv, dst);
   LAUNCHED();
   prof_begin(st);
-  run_pass<1>(a, cfg, st);
+  run_pass<1, E>(a, cfg, st);
   prof_end(st, 5, 0, pass_bytes);
   reduce(-1);
   stats_finalize_kernel<<<(ld + 255) / 256, 256, 0, st>>>(G, ld, 1, real, mu, mu_f, inv, dst);
@@ -451,7 +466,7 @@ LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_tr
   LAUNCHED();
   for (int k = 0; k < power_iters; ++k) {
     prof_begin(st);
-    run_pass<2>(a, cfg, st);
+    run_pass<2, E>(a, cfg, st);
     prof_end(st, 5, 0, pass_bytes);
     reduce(-1);
     power_kernel<<<1, ublk, 0, st>>>(G, ld, 0, d_real, real, inv, v, what, bhat, dst);
@@ -462,7 +477,7 @@ LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_tr
   LAUNCHED();
   for (int t = 0; t < iters; ++t) {
     prof_begin(st);
-    run_pass<3>(a, cfg, st);
+    run_pass<3, E>(a, cfg, st);
     prof_end(st, 5, 0, pass_bytes);
     reduce(-1);
     grad_kernel<<<1, ublk, 0, st>>>(G, ld, 0, lambda, alpha, inv, w, what, bhat, dst, loss + t);
@@ -477,8 +492,8 @@ LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_tr
     StreamCfg ce = cfg;
     ce.grid = grid_for_rows(n_rows);
     prof_begin(st);
-    if (n_rows > 0) run_pass<4>(e, ce, st);
-    prof_end(st, 5, 0, (double)n_rows * ld * 2);
+    if (n_rows > 0) run_pass<4, E>(e, ce, st);
+    prof_end(st, 5, 0, (double)n_rows * ld * esz);
   }
   // counts -> fp64 for the allreduce (exact below 2^53)
   unsigned long long hc[5];
@@ -511,6 +526,20 @@ LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_tr
   res.fn = (int64_t)dc[4];
   res.n_test = (int64_t)dc[5];
   return res;
+}
+
+LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
+                  const uint8_t* real_host, int iters, int power_iters, double lambda, double alpha,
+                  allreduce_fn allreduce, void* ar_user, cudaStream_t st) {
+  return lr_train_impl<bf16>(MM, y, n_rows, n_train, ld, real_host, iters, power_iters, lambda, alpha, allreduce,
+                             ar_user, st);
+}
+
+LRResult lr_train_f32(const float* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
+                      const uint8_t* real_host, int iters, int power_iters, double lambda, double alpha,
+                      allreduce_fn allreduce, void* ar_user, cudaStream_t st) {
+  return lr_train_impl<float>(MM, y, n_rows, n_train, ld, real_host, iters, power_iters, lambda, alpha, allreduce,
+                              ar_user, st);
 }
 
 }  // namespace vista

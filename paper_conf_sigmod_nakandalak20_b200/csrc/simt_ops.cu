@@ -1,6 +1,7 @@
 // simt_ops.cu — the memory-bound TensorOps of the path (S0 ingest, pools, LRN) and the
-// tap g_l (S2).  All NHWC bf16, 8 channels (16 bytes) per thread, vectorised loads/stores,
-// grids sized in multiples of the SM count by a grid-stride loop.
+// tap g_l (S2).  All NHWC, 8 channels per thread (16-byte bf16 / 32-byte fp32 vectors), grids
+// sized in multiples of the SM count by a grid-stride loop.  Templated on the element type:
+// bf16 (the product) and fp32 (the check mode, reading R23).
 #include "internal.h"
 #include "ptx.cuh"
 
@@ -22,7 +23,11 @@ __device__ __forceinline__ void ld8(const bf16* p, float (&f)[8]) {
     f[2 * j + 1] = a.y;
   }
 }
-__device__ __forceinline__ void st8(bf16* p, const float (&f)[8]) {
+__device__ __forceinline__ void ld8(const float* p, float (&f)[8]) {
+  const float4 a = reinterpret_cast<const float4*>(p)[0], b = reinterpret_cast<const float4*>(p)[1];
+  f[0] = a.x; f[1] = a.y; f[2] = a.z; f[3] = a.w; f[4] = b.x; f[5] = b.y; f[6] = b.z; f[7] = b.w;
+}
+__device__ __forceinline__ void st8(bf16* p, const float (&f)[8]) {  // RNE
   uint4 v;
   v.x = pack_bf16x2(f[0], f[1]);
   v.y = pack_bf16x2(f[2], f[3]);
@@ -30,9 +35,16 @@ __device__ __forceinline__ void st8(bf16* p, const float (&f)[8]) {
   v.w = pack_bf16x2(f[6], f[7]);
   *reinterpret_cast<uint4*>(p) = v;
 }
+__device__ __forceinline__ void st8(float* p, const float (&f)[8]) {
+  reinterpret_cast<float4*>(p)[0] = make_float4(f[0], f[1], f[2], f[3]);
+  reinterpret_cast<float4*>(p)[1] = make_float4(f[4], f[5], f[6], f[7]);
+}
+__device__ __forceinline__ float ld1(const bf16* p) { return __bfloat162float(*p); }
+__device__ __forceinline__ float ld1(const float* p) { return *p; }
 
-// ---- S0: uint8 NHWC3 -> bf16 NHWC8, x = (p - 128) / 128 (reading R10; exact in bf16) ----
-__global__ void ingest_kernel(const uint8_t* __restrict__ px, int64_t npix, bf16* __restrict__ y) {
+// ---- S0: uint8 NHWC3 -> NHWC8, x = (p - 128) / 128 (reading R10; exact in bf16) ----
+template <typename T>
+__global__ void ingest_kernel(const uint8_t* __restrict__ px, int64_t npix, T* __restrict__ y) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < npix; i += (int64_t)gridDim.x * blockDim.x) {
     const uint8_t* q = px + i * 3;
     float f[8] = {0, 0, 0, 0, 0, 0, 0, 0};
@@ -41,18 +53,22 @@ __global__ void ingest_kernel(const uint8_t* __restrict__ px, int64_t npix, bf16
     st8(y + i * 8, f);
   }
 }
-void launch_ingest(const uint8_t* px, int64_t n, bf16* y, cudaStream_t st) {
+template <typename T>
+static void ingest_t(const uint8_t* px, int64_t n, T* y, cudaStream_t st) {
   const int64_t npix = n * 227 * 227;
   prof_begin(st);
-  ingest_kernel<<<grid_for(npix, 256), 256, 0, st>>>(px, npix, y);
+  ingest_kernel<T><<<grid_for(npix, 256), 256, 0, st>>>(px, npix, y);
   LAUNCHED();
-  prof_end(st, 2, 0, (double)npix * (3 + 16));
+  prof_end(st, 2, 0, (double)npix * (3 + 8 * sizeof(T)));
 }
+void launch_ingest(const uint8_t* px, int64_t n, bf16* y, cudaStream_t st) { ingest_t(px, n, y, st); }
+void launch_ingest_f32(const uint8_t* px, int64_t n, float* y, cudaStream_t st) { ingest_t(px, n, y, st); }
 
-// ---- S0 for ResNet conv1: uint8 NHWC3 -> zero-padded 2x2 space-to-depth bf16 [n, 117, 117, 16] ----
+// ---- S0 for ResNet conv1: uint8 NHWC3 -> zero-padded 2x2 space-to-depth [n, 117, 117, 16] ----
 // channel c' = (dy*2 + dx)*3 + ch (c' >= 12 zero) of position (h2, w2) holds (p - 128)/128 of pixel
 // (2*h2 + dy - 3, 2*w2 + dx - 3), 0 outside the image (the conv's zero padding of 3).
-__global__ void ingest_s2d_kernel(const uint8_t* __restrict__ px, int64_t n, bf16* __restrict__ y) {
+template <typename T>
+__global__ void ingest_s2d_kernel(const uint8_t* __restrict__ px, int64_t n, T* __restrict__ y) {
   const int64_t total = n * 117 * 117;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
     const int w2 = (int)(i % 117);
@@ -72,31 +88,31 @@ __global__ void ingest_s2d_kernel(const uint8_t* __restrict__ px, int64_t n, bf1
         for (int c = 0; c < 3; ++c) f[d * 3 + c] = ((float)q[c] - 128.0f) * (1.0f / 128.0f);
       }
     }
-    uint4 a, b;
-    a.x = pack_bf16x2(f[0], f[1]);
-    a.y = pack_bf16x2(f[2], f[3]);
-    a.z = pack_bf16x2(f[4], f[5]);
-    a.w = pack_bf16x2(f[6], f[7]);
-    b.x = pack_bf16x2(f[8], f[9]);
-    b.y = pack_bf16x2(f[10], f[11]);
-    b.z = 0u;
-    b.w = 0u;
-    uint4* dst = reinterpret_cast<uint4*>(y + i * 16);
-    dst[0] = a;
-    dst[1] = b;
+    float lo[8], hi[8];
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      lo[c] = f[c];
+      hi[c] = f[8 + c];
+    }
+    st8(y + i * 16, lo);
+    st8(y + i * 16 + 8, hi);
   }
 }
-void launch_ingest_s2d(const uint8_t* px, int64_t n, bf16* y, cudaStream_t st) {
+template <typename T>
+static void ingest_s2d_t(const uint8_t* px, int64_t n, T* y, cudaStream_t st) {
   const int64_t total = n * 117 * 117;
   prof_begin(st);
-  ingest_s2d_kernel<<<grid_for(total, 256), 256, 0, st>>>(px, n, y);
+  ingest_s2d_kernel<T><<<grid_for(total, 256), 256, 0, st>>>(px, n, y);
   LAUNCHED();
-  prof_end(st, 2, 0, (double)n * 227 * 227 * 3 + (double)total * 32);
+  prof_end(st, 2, 0, (double)n * 227 * 227 * 3 + (double)total * 16 * sizeof(T));
 }
+void launch_ingest_s2d(const uint8_t* px, int64_t n, bf16* y, cudaStream_t st) { ingest_s2d_t(px, n, y, st); }
+void launch_ingest_s2d_f32(const uint8_t* px, int64_t n, float* y, cudaStream_t st) { ingest_s2d_t(px, n, y, st); }
 
 // ---- unpadded max pool (k, s) ----
-__global__ void maxpool_kernel(const bf16* __restrict__ x, int N, int H, int W, int C, int k, int s, int Ho, int Wo,
-                               bf16* __restrict__ y) {
+template <typename T>
+__global__ void maxpool_kernel(const T* __restrict__ x, int N, int H, int W, int C, int k, int s, int Ho, int Wo,
+                               T* __restrict__ y) {
   const int C8 = C >> 3;
   const int64_t total = (int64_t)N * Ho * Wo * C8;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
@@ -124,28 +140,36 @@ __global__ void maxpool_kernel(const bf16* __restrict__ x, int N, int H, int W, 
     st8(y + (((size_t)n * Ho + ho) * Wo + wo) * C + c8 * 8, m);
   }
 }
-void launch_maxpool(const bf16* x, int N, int H, int W, int C, int k, int s, bf16* y, cudaStream_t st) {
+template <typename T>
+static void maxpool_t(const T* x, int N, int H, int W, int C, int k, int s, T* y, cudaStream_t st) {
   const int Ho = (H - k) / s + 1, Wo = (W - k) / s + 1;
   const int64_t total = (int64_t)N * Ho * Wo * (C / 8);
   prof_begin(st);
-  maxpool_kernel<<<grid_for(total, 256), 256, 0, st>>>(x, N, H, W, C, k, s, Ho, Wo, y);
+  maxpool_kernel<T><<<grid_for(total, 256), 256, 0, st>>>(x, N, H, W, C, k, s, Ho, Wo, y);
   LAUNCHED();
-  prof_end(st, 2, 0, 2.0 * ((double)N * H * W * C + (double)N * Ho * Wo * C));
+  prof_end(st, 2, 0, (double)sizeof(T) * ((double)N * H * W * C + (double)N * Ho * Wo * C));
+}
+void launch_maxpool(const bf16* x, int N, int H, int W, int C, int k, int s, bf16* y, cudaStream_t st) {
+  maxpool_t(x, N, H, W, C, k, s, y, st);
+}
+void launch_maxpool_f32(const float* x, int N, int H, int W, int C, int k, int s, float* y, cudaStream_t st) {
+  maxpool_t(x, N, H, W, C, k, s, y, st);
 }
 
 // ---- AlexNet LRN (reading R3): y_c = x_c / (1 + 2e-5 sum_{|c'-c|<=2} x_c'^2)^0.75 ----
-__global__ void lrn_kernel(const bf16* __restrict__ x, int64_t npix, int C, bf16* __restrict__ y) {
+template <typename T>
+__global__ void lrn_kernel(const T* __restrict__ x, int64_t npix, int C, T* __restrict__ y) {
   const int C8 = C >> 3;
   const int64_t total = npix * C8;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
     const int c8 = (int)(i % C8);
     const int64_t pix = i / C8;
-    const bf16* xp = x + pix * C;
+    const T* xp = x + pix * C;
     float w[12];  // channels c8*8-2 .. c8*8+9
 #pragma unroll
     for (int j = 0; j < 12; ++j) {
       const int c = c8 * 8 - 2 + j;
-      w[j] = (c >= 0 && c < C) ? __bfloat162float(xp[c]) : 0.0f;
+      w[j] = (c >= 0 && c < C) ? ld1(xp + c) : 0.0f;
     }
     float o[8];
 #pragma unroll
@@ -158,16 +182,22 @@ __global__ void lrn_kernel(const bf16* __restrict__ x, int64_t npix, int C, bf16
     st8(y + pix * C + c8 * 8, o);
   }
 }
-void launch_lrn(const bf16* x, int N, int H, int W, int C, bf16* y, cudaStream_t st) {
+template <typename T>
+static void lrn_t(const T* x, int N, int H, int W, int C, T* y, cudaStream_t st) {
   const int64_t npix = (int64_t)N * H * W;
   prof_begin(st);
-  lrn_kernel<<<grid_for(npix * (C / 8), 256), 256, 0, st>>>(x, npix, C, y);
+  lrn_kernel<T><<<grid_for(npix * (C / 8), 256), 256, 0, st>>>(x, npix, C, y);
   LAUNCHED();
-  prof_end(st, 2, 0, 4.0 * (double)npix * C);
+  prof_end(st, 2, 0, 2.0 * sizeof(T) * (double)npix * C);
+}
+void launch_lrn(const bf16* x, int N, int H, int W, int C, bf16* y, cudaStream_t st) { lrn_t(x, N, H, W, C, y, st); }
+void launch_lrn_f32(const float* x, int N, int H, int W, int C, float* y, cudaStream_t st) {
+  lrn_t(x, N, H, W, C, y, st);
 }
 
 // ---- global average pool [N,H,W,C] -> [N,C] ----
-__global__ void avgpool_kernel(const bf16* __restrict__ x, int N, int HW, int C, bf16* __restrict__ y) {
+template <typename T>
+__global__ void avgpool_kernel(const T* __restrict__ x, int N, int HW, int C, T* __restrict__ y) {
   const int C8 = C >> 3;
   const int64_t total = (int64_t)N * C8;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
@@ -186,18 +216,26 @@ __global__ void avgpool_kernel(const bf16* __restrict__ x, int N, int HW, int C,
     st8(y + (size_t)n * C + c8 * 8, acc);
   }
 }
-void launch_avgpool(const bf16* x, int N, int H, int W, int C, bf16* y, cudaStream_t st) {
+template <typename T>
+static void avgpool_t(const T* x, int N, int H, int W, int C, T* y, cudaStream_t st) {
   const int64_t total = (int64_t)N * (C / 8);
   prof_begin(st);
-  avgpool_kernel<<<grid_for(total, 256), 256, 0, st>>>(x, N, H * W, C, y);
+  avgpool_kernel<T><<<grid_for(total, 256), 256, 0, st>>>(x, N, H * W, C, y);
   LAUNCHED();
-  prof_end(st, 2, 0, 2.0 * ((double)N * H * W * C + (double)N * C));
+  prof_end(st, 2, 0, (double)sizeof(T) * ((double)N * H * W * C + (double)N * C));
+}
+void launch_avgpool(const bf16* x, int N, int H, int W, int C, bf16* y, cudaStream_t st) {
+  avgpool_t(x, N, H, W, C, y, st);
+}
+void launch_avgpool_f32(const float* x, int N, int H, int W, int C, float* y, cudaStream_t st) {
+  avgpool_t(x, N, H, W, C, y, st);
 }
 
 // ---- S2 tap g_l (PAPER.md:369 fn 4, Def 3.5; reading R7/R8): 2x2 grid max, NHWC flatten ----
 // F[n][(2i + j) C + c] = max_{h in R_i, w in R_j} A[n, h, w, c], R_0 = [0, ceil(H/2)), R_1 = [ceil(H/2), H).
-// Max is exact, so F is bit-identical to a max over the bf16 activation.
-__global__ void tap_kernel(const bf16* __restrict__ A, int64_t N, int H, int W, int C, bf16* __restrict__ F) {
+// Max is exact, so F is bit-identical to a max over the stored activation.
+template <typename T>
+__global__ void tap_kernel(const T* __restrict__ A, int64_t N, int H, int W, int C, T* __restrict__ F) {
   const int C8 = C >> 3;
   const int h2 = (H + 1) >> 1, w2 = (W + 1) >> 1;
   const int64_t total = N * 4 * C8;
@@ -222,6 +260,21 @@ __global__ void tap_kernel(const bf16* __restrict__ A, int64_t N, int H, int W, 
     st8(F + (size_t)n * 4 * C + (size_t)q * C + c8 * 8, m);
   }
 }
+template <typename T>
+static void tap_t(const T* A, int64_t N, int H, int W, int C, T* F, cudaStream_t st) {
+  const int64_t total = N * 4 * (C / 8);
+  prof_begin(st);
+  tap_kernel<T><<<grid_for(total, 256), 256, 0, st>>>(A, N, H, W, C, F);
+  LAUNCHED();
+  prof_end(st, 1, 0, (double)sizeof(T) * ((double)N * H * W * C + (double)N * 4 * C));
+}
+void launch_tap(const bf16* A, int64_t N, int H, int W, int C, bf16* F, cudaStream_t st) {
+  tap_t(A, N, H, W, C, F, st);
+}
+void launch_tap_f32(const float* A, int64_t N, int H, int W, int C, float* F, cudaStream_t st) {
+  tap_t(A, N, H, W, C, F, st);
+}
+
 // finalize of the fused tap (conv_tc.cu): fp32 maxima -> bf16, 8 values per thread (exact)
 __global__ void tap_finalize_kernel(const unsigned int* __restrict__ in, int64_t n8, bf16* __restrict__ F) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n8; i += (int64_t)gridDim.x * blockDim.x) {
@@ -237,14 +290,6 @@ void launch_tap_finalize(const unsigned int* tapf, int64_t count, bf16* F, cudaS
   tap_finalize_kernel<<<grid_for(n8, 256), 256, 0, st>>>(tapf, n8, F);
   LAUNCHED();
   prof_end(st, 1, 0, (double)count * 6);
-}
-
-void launch_tap(const bf16* A, int64_t N, int H, int W, int C, bf16* F, cudaStream_t st) {
-  const int64_t total = N * 4 * (C / 8);
-  prof_begin(st);
-  tap_kernel<<<grid_for(total, 256), 256, 0, st>>>(A, N, H, W, C, F);
-  LAUNCHED();
-  prof_end(st, 1, 0, 2.0 * ((double)N * H * W * C + (double)N * 4 * C));
 }
 
 }  // namespace vista

@@ -198,6 +198,9 @@ struct vista_ctx {
   int cnn = 0;
   NetDesc net;
   std::vector<ConvLayer> convs;
+  std::vector<ConvLayerF32> convs32;  // VISTA_F32 check mode (reading R23)
+  bool f32 = false;
+  int64_t esz = 2;                   // bytes per activation / feature / MM element
   std::vector<int> taps;     // requested tap ids, ascending
   int t_max = 0;             // last block to run
   vista_lr_cfg lr{};
@@ -239,6 +242,7 @@ struct vista_ctx {
     for (DevBuf* b : {&pair_str, &pair_img, &d_X, &d_labels, &d_img_keys, &d_str_keys, &d_px}) b->release();
     if (stream) cudaStreamSynchronize(stream);
     for (auto& L : convs) conv_layer_free(L);
+    for (auto& L : convs32) conv_layer_free_f32(L);
     if (nccl_comm) {
       Nccl& n = nccl_lib();
       if (n.CommDestroy) n.CommDestroy(nccl_comm);
@@ -292,8 +296,8 @@ void plan_memory(vista_ctx* c, uint64_t budget) {
   c->micro.assign(c->t_max + 1, 0);
   int64_t mm_bytes = 0, f_bytes = 0;
   for (size_t k = 0; k < c->taps.size(); ++k) {
-    mm_bytes += c->n_str * (int64_t)ld_of(c, (int)k) * 2 + c->n_str;
-    if (!S[c->taps[k]].fc_tap) f_bytes += c->n_img * (int64_t)S[c->taps[k]].d_tap * 2;
+    mm_bytes += c->n_str * (int64_t)ld_of(c, (int)k) * c->esz + c->n_str;
+    if (!S[c->taps[k]].fc_tap) f_bytes += c->n_img * (int64_t)S[c->taps[k]].d_tap * c->esz;
   }
   const int64_t px = c->n_img * (int64_t)S[0].in_elems;
   const int64_t join_bytes = c->n_str * 8 + c->n_img * 8 + c->n_str * 4 * 2 + c->n_str * 12 + 32 * 4 * std::max(c->n_img, c->n_str);
@@ -301,15 +305,15 @@ void plan_memory(vista_ctx* c, uint64_t budget) {
   if (c->sys.plan != VISTA_PLAN_STAGED) {
     // Eager / Lazy: features of all of L (incl. FC taps) + two micro-batch activation buffers + slots
     int64_t f_all = 0, max_out = 0, slot_per_img = 0;
-    for (int t : c->taps) f_all += c->n_img * (int64_t)S[t].d_tap * 2;
+    for (int t : c->taps) f_all += c->n_img * (int64_t)S[t].d_tap * c->esz;
     for (int t = 0; t <= c->t_max; ++t) {
       max_out = std::max<int64_t>(max_out, S[t].out_elems);
       int64_t s = 0;
-      for (int b = BUF_T0; b < NUM_BUFS; ++b) s += S[t].slot_elems[b] * 2;
+      for (int b = BUF_T0; b < NUM_BUFS; ++b) s += S[t].slot_elems[b] * c->esz;
       slot_per_img = std::max(slot_per_img, s);
     }
     const int64_t fixed = c->weight_bytes + px + f_all + mm_bytes + join_bytes + (256ll << 20);
-    const int64_t per_img = slot_per_img + 2 * max_out * 2;
+    const int64_t per_img = slot_per_img + 2 * max_out * c->esz;
     int B = c->sys.micro_batch > 0 ? c->sys.micro_batch : 0;
     for (int64_t b = std::min<int64_t>(1024, std::max<int64_t>(c->n_img, 1)); B == 0 && b >= 1;
          b = b > 8 ? b / 2 : b - 1)
@@ -325,17 +329,17 @@ void plan_memory(vista_ctx* c, uint64_t budget) {
   // feasible from the top"); NO_PLAN only if not even one image fits.
   int64_t f_fc = 0;  // FC taps alias A_t when unchunked; a chunked run keeps them in F as well
   for (int t : c->taps)
-    if (S[t].fc_tap) f_fc += c->n_img * (int64_t)S[t].d_tap * 2;
+    if (S[t].fc_tap) f_fc += c->n_img * (int64_t)S[t].d_tap * c->esz;
   auto plan_chunk = [&](int64_t CH, std::vector<int>& micro, int64_t& pk) -> bool {
     pk = 0;
     const bool chunked = CH < c->n_img;
     const int64_t pxc = CH * (int64_t)S[0].in_elems;  // host pixels are streamed per chunk
     int64_t arena[2] = {0, 0};                         // ping-pong activation arenas (A_t in arena t % 2)
-    for (int t = 0; t <= c->t_max; ++t) arena[t & 1] = std::max<int64_t>(arena[t & 1], CH * S[t].out_elems * 2);
+    for (int t = 0; t <= c->t_max; ++t) arena[t & 1] = std::max<int64_t>(arena[t & 1], CH * S[t].out_elems * c->esz);
     (void)chunked;
     for (int t = 0; t <= c->t_max; ++t) {
       int64_t slot_per_img = 0;
-      for (int b = BUF_T0; b < NUM_BUFS; ++b) slot_per_img += S[t].slot_elems[b] * 2;
+      for (int b = BUF_T0; b < NUM_BUFS; ++b) slot_per_img += S[t].slot_elems[b] * c->esz;
       const int64_t fixed = c->weight_bytes + pxc + arena[0] + arena[1] + mm_bytes + f_bytes + f_fc + join_bytes +
                             (256ll << 20);
       int B = 0;
@@ -370,26 +374,19 @@ void plan_memory(vista_ctx* c, uint64_t budget) {
 }
 
 void upload_weights(vista_ctx* c, uint64_t seed) {
-  c->convs.resize(c->net.layers.size());
+  if (c->f32)
+    c->convs32.resize(c->net.layers.size());
+  else
+    c->convs.resize(c->net.layers.size());
   c->weight_bytes = 0;
   for (size_t i = 0; i < c->net.layers.size(); ++i) {
     const LayerSpec& s = c->net.layers[i];
-    ConvLayer& L = c->convs[i];
-    L.Cin = s.Cin;
-    L.Cout = s.Cout;
-    L.R = s.R;
-    L.S = s.S;
-    L.stride = s.stride;
-    L.pad = s.pad;
-    L.groups = s.groups;
-    L.relu = s.relu;
     const int64_t fan_in = (int64_t)s.R * s.S * (s.Cin_real / s.groups);
     const int64_t nw = (int64_t)s.Cout * fan_in;
     std::vector<float> wf(nw);
-    // He-normal N(0, 2 / fan_in), RNE bf16 (reading R11) — same generator call as the oracle's
+    // He-normal N(0, 2 / fan_in), RNE bf16 (reading R11) — same generator call as the oracle's;
+    // the values are bf16-representable, so the fp32 check mode uses them unchanged
     vg_param_f32(seed, c->cnn, s.id, VG_T_WEIGHT, nw, 0, 0.0, std::sqrt(2.0 / (double)fan_in), wf.data());
-    std::vector<uint16_t> wb(nw);
-    for (int64_t j = 0; j < nw; ++j) wb[j] = f2bf_bits(wf[j]);
     std::vector<float> scale(s.Cout, 1.0f), shift(s.Cout, 0.0f);
     if (s.bias) {
       vg_param_f32(seed, c->cnn, s.id, VG_T_BIAS, s.Cout, 0, 0.0, 0.01, shift.data());
@@ -409,30 +406,55 @@ void upload_weights(vista_ctx* c, uint64_t seed) {
         shift[o] = (float)(be[o] - mu[o] * sc);
       }
     }
+    int Cin = s.Cin, R = s.R, Sk = s.S, stride = s.stride, pad = s.pad, cin_real = s.Cin_real;
     if (s.s2d) {
       // 7x7/2 pad 3 on 3 channels == 4x4/1 on the 2x2 space-to-depth input (roster.h kS2dHW):
       // W2[o][a][b][(dy*2 + dx)*3 + ch] = W[o][2a + dy][2b + dx][ch] for 2a + dy, 2b + dx < 7, else 0
       const int R2 = (s.R + 1) / 2, S2 = (s.S + 1) / 2;
-      std::vector<uint16_t> w2((size_t)s.Cout * R2 * S2 * kS2dC, 0);
+      std::vector<float> w2((size_t)s.Cout * R2 * S2 * kS2dC, 0.f);
       for (int o = 0; o < s.Cout; ++o)
         for (int r = 0; r < s.R; ++r)
           for (int q = 0; q < s.S; ++q)
             for (int ch = 0; ch < s.Cin_real; ++ch) {
               const int a = r / 2, dy = r % 2, b = q / 2, dx = q % 2;
               w2[(((size_t)o * R2 + a) * S2 + b) * kS2dC + (dy * 2 + dx) * 3 + ch] =
-                  wb[(((size_t)o * s.R + r) * s.S + q) * s.Cin_real + ch];
+                  wf[(((size_t)o * s.R + r) * s.S + q) * s.Cin_real + ch];
             }
-      L.Cin = kS2dC;
-      L.R = R2;
-      L.S = S2;
-      L.stride = 1;
-      L.pad = 0;
-      L.K_alg = s.R * s.S * s.Cin_real;
-      conv_layer_init(L, w2, kS2dC, scale, shift);
-    } else {
-      conv_layer_init(L, wb, s.Cin_real, scale, shift);
+      wf.swap(w2);
+      Cin = cin_real = kS2dC;
+      R = R2;
+      Sk = S2;
+      stride = 1;
+      pad = 0;
     }
-    c->weight_bytes += (int64_t)L.Cout * L.Kp * 2 + (int64_t)L.Cout * 8;
+    if (c->f32) {
+      ConvLayerF32& L = c->convs32[i];
+      L.Cin = Cin;
+      L.Cout = s.Cout;
+      L.R = R;
+      L.S = Sk;
+      L.stride = stride;
+      L.pad = pad;
+      L.groups = s.groups;
+      L.relu = s.relu;
+      conv_layer_init_f32(L, wf, cin_real, scale, shift);
+      c->weight_bytes += (int64_t)L.Cout * L.K * 4 + (int64_t)L.Cout * 8;
+    } else {
+      ConvLayer& L = c->convs[i];
+      L.Cin = Cin;
+      L.Cout = s.Cout;
+      L.R = R;
+      L.S = Sk;
+      L.stride = stride;
+      L.pad = pad;
+      L.groups = s.groups;
+      L.relu = s.relu;
+      if (s.s2d) L.K_alg = s.R * s.S * s.Cin_real;
+      std::vector<uint16_t> wb(wf.size());
+      for (size_t j = 0; j < wf.size(); ++j) wb[j] = f2bf_bits(wf[j]);
+      conv_layer_init(L, wb, cin_real, scale, shift);
+      c->weight_bytes += (int64_t)L.Cout * L.Kp * 2 + (int64_t)L.Cout * 8;
+    }
   }
 }
 
@@ -448,10 +470,18 @@ const void* to_device(vista_ctx* c, DevBuf& buf, const void* p, size_t bytes) {
 void prepare_slots(vista_ctx* c, int t, int B, void** slot) {
   const StageDesc& S = c->net.stages[t];
   for (int b = BUF_T0; b < NUM_BUFS; ++b) {
-    const size_t need = (size_t)S.slot_elems[b] * 2 * B;
+    const size_t need = (size_t)S.slot_elems[b] * c->esz * B;
     if (need > c->slot_store[b]->bytes) c->slot_store[b]->alloc(need);
     slot[b] = c->slot_store[b]->p;
   }
+}
+
+// g_l (2x2-grid max) of a conv activation in the context's element type
+void tap_any(vista_ctx* c, const void* A, int64_t n, const StageDesc& S, void* F) {
+  if (c->f32)
+    launch_tap_f32((const float*)A, n, S.outH, S.outW, S.outC, (float*)F, c->stream);
+  else
+    launch_tap((const bf16*)A, n, S.outH, S.outW, S.outC, (bf16*)F, c->stream);
 }
 
 // nb images through block t (partial inference f^_{l(t-1) -> l(t)}): in -> out.
@@ -463,6 +493,34 @@ bool run_ops(vista_ctx* c, int t, const void* in_ptr, void* out_ptr, int nb, voi
   {
     slot[BUF_IN] = const_cast<void*>(in_ptr);
     slot[BUF_OUT] = out_ptr;
+    if (c->f32) {  // fp32 check mode: same op sequence on the fp32 kernels
+      for (const OpDesc& op : S.ops) {
+        const float* in = reinterpret_cast<const float*>(slot[op.in]);
+        float* out = reinterpret_cast<float*>(slot[op.out]);
+        switch (op.kind) {
+          case OP_INGEST:
+            launch_ingest_f32(reinterpret_cast<const uint8_t*>(slot[op.in]), nb, out, c->stream);
+            break;
+          case OP_INGEST_S2D:
+            launch_ingest_s2d_f32(reinterpret_cast<const uint8_t*>(slot[op.in]), nb, out, c->stream);
+            break;
+          case OP_CONV:
+            conv_forward_f32(c->convs32[op.layer], in, nb, op.H, op.W,
+                             op.res >= 0 ? reinterpret_cast<const float*>(slot[op.res]) : nullptr, out, c->stream);
+            break;
+          case OP_MAXPOOL:
+            launch_maxpool_f32(in, nb, op.H, op.W, op.C, op.k, op.s, out, c->stream);
+            break;
+          case OP_LRN:
+            launch_lrn_f32(in, nb, op.H, op.W, op.C, out, c->stream);
+            break;
+          case OP_AVGPOOL:
+            launch_avgpool_f32(in, nb, op.H, op.W, op.C, out, c->stream);
+            break;
+        }
+      }
+      return tapf == nullptr;
+    }
     for (const OpDesc& op : S.ops) {
       const bf16* in = reinterpret_cast<const bf16*>(slot[op.in]);
       bf16* out = reinterpret_cast<bf16*>(slot[op.out]);
@@ -497,17 +555,17 @@ bool run_ops(vista_ctx* c, int t, const void* in_ptr, void* out_ptr, int nb, voi
 }
 
 // one block of the Staged plan over n images (a chunk), in micro-batches of micro[t]: in_base -> A_t
-bool run_block(vista_ctx* c, int t, const void* in_base, bf16* out_base, int64_t n, unsigned int* tapf) {
+bool run_block(vista_ctx* c, int t, const void* in_base, void* out_base, int64_t n, unsigned int* tapf) {
   const StageDesc& S = c->net.stages[t];
   const int B = c->micro[t];
   void* slot[NUM_BUFS] = {nullptr};
   prepare_slots(c, t, B, slot);
-  const size_t in_bytes_per = t == 0 ? (size_t)S.in_elems : (size_t)S.in_elems * 2;
+  const size_t in_bytes_per = t == 0 ? (size_t)S.in_elems : (size_t)S.in_elems * c->esz;
   bool fused = tapf != nullptr;
   for (int64_t i0 = 0; i0 < n; i0 += B) {
     const int nb = (int)std::min<int64_t>(B, n - i0);
     const bool ok = run_ops(c, t, (const uint8_t*)in_base + (size_t)i0 * in_bytes_per,
-                            out_base + (size_t)i0 * S.out_elems, nb, slot,
+                            (uint8_t*)out_base + (size_t)i0 * S.out_elems * c->esz, nb, slot,
                             tapf ? tapf + (size_t)i0 * 4 * S.outC : nullptr);
     fused = fused && ok;
   }
@@ -527,20 +585,20 @@ void run_unstaged(vista_ctx* c, const uint8_t* px, int t_last, const std::vector
     max_out = std::max<int64_t>(max_out, S[t].out_elems);
   }
   DevBuf act[2];
-  act[0].alloc((size_t)B * max_out * 2 + 16);
-  act[1].alloc((size_t)B * max_out * 2 + 16);
+  act[0].alloc((size_t)B * max_out * c->esz + 16);
+  act[1].alloc((size_t)B * max_out * c->esz + 16);
   for (int64_t i0 = 0; i0 < c->n_img; i0 += B) {
     const int nb = (int)std::min<int64_t>(B, c->n_img - i0);
     for (int t = 0; t <= t_last; ++t) {
       const void* in = t == 0 ? (const void*)(px + (size_t)i0 * S[0].in_elems) : act[(t - 1) & 1].p;
-      bf16* out = (bf16*)act[t & 1].p;
+      void* out = act[t & 1].p;
       run_ops(c, t, in, out, nb, slot, nullptr);
       if (std::find(want.begin(), want.end(), t) == want.end()) continue;
-      bf16* Ft = (bf16*)c->F[t]->p + (size_t)i0 * S[t].d_tap;
+      void* Ft = (uint8_t*)c->F[t]->p + (size_t)i0 * S[t].d_tap * c->esz;
       if (S[t].fc_tap)
-        VCHECK(cudaMemcpyAsync(Ft, out, (size_t)nb * S[t].d_tap * 2, cudaMemcpyDeviceToDevice, c->stream));
+        VCHECK(cudaMemcpyAsync(Ft, out, (size_t)nb * S[t].d_tap * c->esz, cudaMemcpyDeviceToDevice, c->stream));
       else
-        launch_tap(out, nb, S[t].outH, S[t].outW, S[t].outC, Ft, c->stream);
+        tap_any(c, out, nb, S[t], Ft);
     }
   }
 }
@@ -624,7 +682,9 @@ VISTA_API vista_status vista_plan(vista_cnn cnn, const int32_t* layers, int32_t 
     if (sys) c->sys = *sys;
     if (c->sys.world <= 0) c->sys.world = 1;
     if (c->sys.plan < VISTA_PLAN_STAGED || c->sys.plan > VISTA_PLAN_LAZY) fail(1, "unknown logical plan");
-    if (c->sys.dtype != VISTA_BF16) fail(1, "only bf16 is implemented");
+    if (c->sys.dtype != VISTA_BF16 && c->sys.dtype != VISTA_F32) fail(1, "unknown dtype");
+    c->f32 = c->sys.dtype == VISTA_F32;
+    c->esz = c->f32 ? 4 : 2;
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
       cudaGetLastError();
@@ -693,7 +753,7 @@ VISTA_API vista_status vista_plan_info(const vista_ctx* c, vista_plan_info_t* o)
     o->d_l[k] = c->net.stages[t].d_tap;
     o->ld[k] = ld_of(c, (int)k);
     o->micro_batch[k] = c->micro[t];
-    o->act_bytes[k] = c->n_img * c->net.stages[t].out_elems * 2;
+    o->act_bytes[k] = c->n_img * c->net.stages[t].out_elems * c->esz;
   }
   o->peak_bytes_pred = c->peak_pred;
   o->weight_bytes = c->weight_bytes;
@@ -747,17 +807,22 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
     c->feat.assign(c->t_max + 1, nullptr);
     c->act.assign(c->t_max + 1, nullptr);
     for (int t : c->taps) {
-      c->F[t]->ensure((size_t)c->n_img * S[t].d_tap * 2 + 16);
+      c->F[t]->ensure((size_t)c->n_img * S[t].d_tap * c->esz + 16);
       c->feat[t] = c->F[t]->p;
     }
     auto concat_layer = [&](int k) {
       const int t = c->taps[k];
       const int ld = ld_of(c, k);
-      c->MM[k]->ensure((size_t)std::max<int64_t>(c->n_pairs, 1) * ld * 2);
+      c->MM[k]->ensure((size_t)std::max<int64_t>(c->n_pairs, 1) * ld * c->esz);
       c->Y[k]->ensure((size_t)std::max<int64_t>(c->n_pairs, 1));
-      launch_concat(X, c->d_s, c->ds_pad, (const bf16*)c->feat[t], S[t].d_tap, (const int32_t*)c->pair_str.p,
-                    (const int32_t*)c->pair_img.p, lab, c->n_pairs, ld, (bf16*)c->MM[k]->p, (uint8_t*)c->Y[k]->p,
-                    st);
+      if (c->f32)
+        launch_concat_f32(X, c->d_s, c->ds_pad, (const float*)c->feat[t], S[t].d_tap, (const int32_t*)c->pair_str.p,
+                          (const int32_t*)c->pair_img.p, lab, c->n_pairs, ld, (float*)c->MM[k]->p,
+                          (uint8_t*)c->Y[k]->p, st);
+      else
+        launch_concat(X, c->d_s, c->ds_pad, (const bf16*)c->feat[t], S[t].d_tap, (const int32_t*)c->pair_str.p,
+                      (const int32_t*)c->pair_img.p, lab, c->n_pairs, ld, (bf16*)c->MM[k]->p, (uint8_t*)c->Y[k]->p,
+                      st);
     };
     if (c->sys.plan != VISTA_PLAN_STAGED) {
       // ---- Eager / Lazy (Fig 5C / 5A): features of every layer, no resident full activations ----
@@ -776,7 +841,7 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
       size_t need[2] = {16, 16};
       for (int t = 0; t <= c->t_max; ++t)
         need[t & 1] = std::max(need[t & 1], (size_t)std::min<int64_t>(CH, std::max<int64_t>(c->n_img, 1)) *
-                                                  S[t].out_elems * 2 + 16);
+                                                  S[t].out_elems * c->esz + 16);
       c->arena[0].ensure(need[0]);
       c->arena[1].ensure(need[1]);
     }
@@ -790,13 +855,13 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
         pxc = (const uint8_t*)c->d_px.p;
       }
       for (int t = 0; t <= c->t_max; ++t) {
-        bf16* At = (bf16*)c->arena[t & 1].p;
+        void* At = c->arena[t & 1].p;
         c->act[t] = At;
         const void* in = t == 0 ? (const void*)pxc : c->arena[(t - 1) & 1].p;
         const int k = layer_index(c, t);
         // S2 fused into the producing conv's epilogue (opt-in, unchunked only)
         unsigned int* tapf = nullptr;
-        if (k >= 0 && !S[t].fc_tap && c->fuse_tap && !chunked) {
+        if (k >= 0 && !S[t].fc_tap && c->fuse_tap && !chunked && !c->f32) {
           const size_t cnt = (size_t)nc * 4 * S[t].outC;
           c->tapacc.ensure(cnt * 4);
           VCHECK(cudaMemsetAsync(c->tapacc.p, 0, cnt * 4, st));  // max over non-negative (post-ReLU) values
@@ -804,13 +869,13 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
         }
         const bool fused = run_block(c, t, in, At, nc, tapf);
         if (k >= 0) {
-          bf16* Ft = (bf16*)c->F[t]->p + (size_t)c0 * S[t].d_tap;
+          void* Ft = (uint8_t*)c->F[t]->p + (size_t)c0 * S[t].d_tap * c->esz;
           if (S[t].fc_tap)  // g = identity on FC layers
-            VCHECK(cudaMemcpyAsync(Ft, At, (size_t)nc * S[t].d_tap * 2, cudaMemcpyDeviceToDevice, st));
+            VCHECK(cudaMemcpyAsync(Ft, At, (size_t)nc * S[t].d_tap * c->esz, cudaMemcpyDeviceToDevice, st));
           else if (fused)
-            launch_tap_finalize(tapf, (int64_t)nc * S[t].d_tap, Ft, st);
+            launch_tap_finalize(tapf, (int64_t)nc * S[t].d_tap, (bf16*)Ft, st);
           else
-            launch_tap(At, nc, S[t].outH, S[t].outW, S[t].outC, Ft, st);
+            tap_any(c, At, nc, S[t], Ft);
           if (!chunked) concat_layer(k);
         }
       }
@@ -863,9 +928,13 @@ VISTA_API vista_status vista_train(vista_ctx* c, int32_t k, double* weights_out,
     std::vector<uint8_t> real(ld, 0);
     for (int j = 0; j < c->d_s; ++j) real[j] = 1;
     for (int j = 0; j < d_l; ++j) real[c->ds_pad + j] = 1;
-    LRResult r = lr_train((const bf16*)c->MM[k]->p, (const uint8_t*)c->Y[k]->p, c->n_pairs, c->n_train, ld,
-                          real.data(), c->lr.iters, c->lr.power_iters, c->lr.lambda, c->lr.alpha,
-                          c->sys.world > 1 ? nccl_allreduce_f64 : nullptr, c->nccl_comm, c->stream);
+    allreduce_fn ar = c->sys.world > 1 ? nccl_allreduce_f64 : nullptr;
+    LRResult r = c->f32 ? lr_train_f32((const float*)c->MM[k]->p, (const uint8_t*)c->Y[k]->p, c->n_pairs,
+                                       c->n_train, ld, real.data(), c->lr.iters, c->lr.power_iters, c->lr.lambda,
+                                       c->lr.alpha, ar, c->nccl_comm, c->stream)
+                        : lr_train((const bf16*)c->MM[k]->p, (const uint8_t*)c->Y[k]->p, c->n_pairs, c->n_train,
+                                   ld, real.data(), c->lr.iters, c->lr.power_iters, c->lr.lambda, c->lr.alpha, ar,
+                                   c->nccl_comm, c->stream);
     if (g_prof) g_prof->flush();
     if (weights_out) {
       for (int j = 0; j < c->d_s; ++j) weights_out[j] = r.w[j];

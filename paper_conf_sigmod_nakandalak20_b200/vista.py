@@ -221,7 +221,8 @@ def _dev_tensor(ptr, shape, typestr, dtype=None):
     import torch
     n = int(np.prod(shape))
     if n == 0 or not ptr:
-        t = torch.empty(shape, dtype=torch.int16 if typestr == "<i2" else None, device="cuda")
+        t = torch.empty(shape, dtype={"<i2": torch.int16, "<f4": torch.float32, "<i4": torch.int32,
+                                      "|u1": torch.uint8}.get(typestr), device="cuda")
     else:
         t = torch.as_tensor(_CudaView(ptr, shape, typestr), device="cuda")
     return t.view(dtype) if dtype is not None else t
@@ -233,13 +234,16 @@ class Vista:
     def __init__(self, cnn, layers=None, n_top=0, n_str_rows=0, d_s=0, n_images_local=0, iters=10,
                  power_iters=20, lam=0.01, alpha=0.5, split_seed=0, weight_seed=0, rank=0, world=1,
                  nccl_uid: bytes | None = None, device=0, hbm_budget_bytes=0, stream=None, micro_batch=0,
-                 plan="staged"):
+                 plan="staged", dtype="bf16"):
+        """dtype: "bf16" (the tcgen05 product path) or "f32" (the fp32 check mode, reading R23)."""
         self.cnn = cnn
+        self.dtype = dtype
         lr = LRCfg(iters, power_iters, lam, alpha, split_seed)
         self._uid = (ctypes.c_uint8 * 128).from_buffer_copy(nccl_uid) if nccl_uid else None
         plan_id = {"staged": 0, "eager": 1, "lazy": 2}[plan]
+        dtype_id = {"bf16": 0, "f32": 1}[dtype]
         sys = SysCfg(rank, world, ctypes.addressof(self._uid) if self._uid is not None else None, device,
-                     hbm_budget_bytes, 0, plan_id, stream, micro_batch)
+                     hbm_budget_bytes, dtype_id, plan_id, stream, micro_batch)
         arr = None
         n_layers = 0
         if layers is not None:
@@ -270,13 +274,14 @@ class Vista:
         b = Buffer()
         _check(lib().vista_features(self.ctx, k, ctypes.byref(b)), self.ctx)
         rows = b.rows
+        ts, tdt = ("<f4", None) if self.dtype == "f32" else ("<i2", torch.bfloat16)
         return dict(
-            mm=_dev_tensor(b.mm, (rows, b.ld), "<i2", torch.bfloat16),
+            mm=_dev_tensor(b.mm, (rows, b.ld), ts, tdt),
             rows=rows, n_train=b.n_train, ld=b.ld, d_s=b.d_s, ds_pad=b.ds_pad, d_l=b.d_l,
             pair_str=_dev_tensor(b.pair_str, (rows,), "<i4"),
             pair_img=_dev_tensor(b.pair_img, (rows,), "<i4"),
             labels=_dev_tensor(b.labels, (rows,), "|u1"),
-            features=_dev_tensor(b.features, (self.n_images_local, b.d_l), "<i2", torch.bfloat16),
+            features=_dev_tensor(b.features, (self.n_images_local, b.d_l), ts, tdt),
             has_activation=bool(b.activation),
         )
 

@@ -61,20 +61,28 @@ constexpr int kThreads = 160 + kEpiThreads;  // 4 producer warps + 1 MMA warp + 
 constexpr int kEpiWarp0 = 5;
 constexpr int kLag = 2;        // cp.async groups in flight before a stage is published
 
-// Shared memory: [A stages][B stages][output staging: BN/64 sub-tiles of 128 x 64 bf16,
-// 128B-swizzled (TMA epilogue only)][scale/shift x 2][barriers]
-template <int BN, bool TMA_EPI>
+// Shared memory: [A stages][B stages][output staging: NB buffers of BN/64 sub-tiles of 128 x 64 bf16,
+// 128B-swizzled (TMA epilogue only)][scale/shift][barriers]
+// NB (TMA epilogue): staging buffers; a residual tile is prefetched NB - 1 tiles ahead into the buffer
+// the tile's output is later staged in, so NB >= 3 hides the residual's HBM latency behind a whole tile.
+template <int BN, bool TMA_EPI, int NB>
 struct Cfg {
-  static constexpr int kStages = TMA_EPI ? (BN == 256 ? 3 : (BN == 128 ? 4 : 6)) : (BN == 256 ? 4 : (BN == 128 ? 6 : 8));
   static constexpr int kABytes = BM * BK * 2;  // 16 KB
   static constexpr int kBBytes = BN * BK * 2;
+  static constexpr int kOutBufs = TMA_EPI ? NB : 0;
+  static constexpr int kOutBytes = kOutBufs * BM * BN * 2;
+  // TMA epilogue: one scale/shift buffer (a named barrier separates tiles); register epilogue: two
+  static constexpr int kSbufBytes = (TMA_EPI ? 1 : 2) * 2 * BN * 4;
+  static constexpr int kFixed = kOutBytes + kSbufBytes + 1024 + 16 + 8 * 8;
+  static constexpr int kStagesFit = (227 * 1024 - kFixed) / (kABytes + kBBytes + 16);
+  static constexpr int kStages = kStagesFit > 8 ? 8 : kStagesFit;
   static constexpr int kOutOff = kStages * (kABytes + kBBytes);
-  static constexpr int kOutBufs = (TMA_EPI && BN <= 128) ? 2 : 1;  // double-buffered staging when it fits
-  static constexpr int kOutBytes = TMA_EPI ? kOutBufs * BM * BN * 2 : 0;
   static constexpr int kSbufOff = kOutOff + kOutBytes;
-  static constexpr int kBarOff = kSbufOff + 2 * 2 * BN * 4;
-  static constexpr int kBytes = kBarOff + (2 * kStages + 6) * 8 + 16 + 1024;  // + alignment slack
+  static constexpr int kBarOff = kSbufOff + kSbufBytes;
+  static constexpr int kBytes = kBarOff + (2 * kStages + 8) * 8 + 16 + 1024;  // + alignment slack
   static constexpr int kTmemCols = 2 * BN;
+  static_assert(kStages >= 2, "shared memory too small for two k-block stages");
+  static_assert(kBytes <= 227 * 1024, "shared memory over the 227 KB per-CTA limit");
 };
 
 // tile -> (first row m0, N-tile index nt, group g); N-tiles of one M-tile are adjacent so
@@ -112,25 +120,25 @@ __device__ __forceinline__ void epi_math(const uint32_t* v, const float* scv, co
   o.w = pack_bf16x2(f[6], f[7]);
 }
 
-template <int BN, int AMODE, bool TMA_EPI>
+template <int BN, int AMODE, bool TMA_EPI, int NB>
 __global__ void __launch_bounds__(kThreads, 1)
     conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__ CUtensorMap tmap_a,
                    const __grid_constant__ CUtensorMap tmap_y, const __grid_constant__ CUtensorMap tmap_r,
                    const ConvParams p) {
-  using C = Cfg<BN, TMA_EPI>;
+  using C = Cfg<BN, TMA_EPI, NB>;
   constexpr int S = C::kStages;
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 1023u) & ~1023u;
   uint8_t* gbase = smem_raw + (base - raw);
   const uint32_t sA = base, sB = base + S * C::kABytes, sO = base + C::kOutOff;
-  float* sbuf = reinterpret_cast<float*>(gbase + C::kSbufOff);  // [2 acc][scale BN | shift BN]
+  float* sbuf = reinterpret_cast<float*>(gbase + C::kSbufOff);  // [1 or 2][scale BN | shift BN]
   uint64_t* full = reinterpret_cast<uint64_t*>(gbase + C::kBarOff);
   uint64_t* empty = full + S;
   uint64_t* tfull = empty + S;   // [2]
   uint64_t* tempty = tfull + 2;  // [2]
-  uint64_t* rbar = tempty + 2;   // [2] residual tile landed in staging buffer b (TMA epilogue)
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rbar + 2);
+  uint64_t* rbar = tempty + 2;   // [NB <= 4] residual tile landed in staging buffer b (TMA epilogue)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rbar + 4);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
@@ -142,8 +150,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(&tfull[i], 1);
       mbar_init(&tempty[i], kEpiWarps);
     }
-    mbar_init(&rbar[0], 1);
-    mbar_init(&rbar[1], 1);
+    for (int i = 0; i < 4; ++i) mbar_init(&rbar[i], 1);
     fence_mbar_init();
     tma_prefetch(&tmap_w);
     if (a_by_tma(AMODE)) tma_prefetch(&tmap_a);
@@ -390,39 +397,44 @@ __global__ void __launch_bounds__(kThreads, 1)
       const int n0 = nt * BN;
       const int ng0 = g * p.Cg_out + n0;
       const int nvalid_tile = min(BN, p.Cg_out - n0);
-      constexpr int NB = C::kOutBufs;
-      const uint32_t ob = NB == 2 ? (it & 1) : 0;
+      const uint32_t ob = NB > 1 ? it % NB : 0;
       const uint32_t sOb = sO + ob * (uint32_t)(BM * BN * 2);
+      // residual tile t -> staging buffer b (TMA, 64-column 128B-swizzled sub-tiles)
+      auto issue_res = [&](int t, uint32_t b) {
+        int tm0, tnt, tg;
+        decode_tile(p, t, tm0, tnt, tg);
+        const int tn0 = tnt * BN, tng0 = tg * p.Cg_out + tn0;
+        const int nsub = (min(BN, p.Cg_out - tn0) + 63) / 64;
+        mbar_arrive_expect_tx(&rbar[b], nsub * BM * 128);
+        for (int st = 0; st < nsub; ++st)
+          tma_load_2d(sO + b * (uint32_t)(BM * BN * 2) + st * BM * 128, &tmap_r, tng0 + st * 64, tm0, &rbar[b]);
+      };
       if constexpr (TMA_EPI) {
-        // residual tile -> staging buffer b (TMA, 64-column 128B-swizzled sub-tiles)
-        auto issue_res = [&](int t, uint32_t b) {
-          int tm0, tnt, tg;
-          decode_tile(p, t, tm0, tnt, tg);
-          const int tn0 = tnt * BN, tng0 = tg * p.Cg_out + tn0;
-          const int nsub = (min(BN, p.Cg_out - tn0) + 63) / 64;
-          mbar_arrive_expect_tx(&rbar[b], nsub * BM * 128);
-          for (int st = 0; st < nsub; ++st)
-            tma_load_2d(sO + b * (uint32_t)(BM * BN * 2) + st * BM * 128, &tmap_r, tng0 + st * 64, tm0, &rbar[b]);
-        };
         if (et == 0) {
           if (NB == 1) {
             bulk_wait_read0();  // the previous tile's stores no longer read the staging buffer
             if (has_res) issue_res(tile, 0);
           } else if (has_res) {
-            if (it == 0) issue_res(tile, 0);
-            // prefetch the next tile's residual into the other buffer once its stores (tile it-1) read it
-            const int next = tile + gridDim.x;
-            if (next < p.n_tiles) {
-              bulk_wait_read0();
-              issue_res(next, ob ^ 1);
+            if (NB == 2) {
+              if (it == 0) issue_res(tile, 0);
+              // prefetch the next tile's residual into the other buffer once its stores (tile it-1) read it
+              const int next = tile + gridDim.x;
+              if (next < p.n_tiles) {
+                bulk_wait_read0();
+                issue_res(next, ob ^ 1);
+              }
+            } else if (it == 0) {
+              // NB >= 3: the first NB - 1 residual tiles now; the rest at the end of each tile (below)
+              for (int j = 0; j < NB - 1; ++j)
+                if (tile + j * (int)gridDim.x < p.n_tiles) issue_res(tile + j * gridDim.x, j);
             }
           } else {
-            bulk_wait_read<1>();  // tile it-2 (same buffer) has been read by its stores
+            bulk_wait_read<NB - 1>();  // tile it-NB (same buffer) has been read by its stores
           }
         }
       }
       // stage this tile's scale / shift in smem (double-buffered by accumulator)
-      float* ss = sbuf + acc * 2 * BN;
+      float* ss = sbuf + (TMA_EPI ? 0 : acc * 2 * BN);
       for (int i = et; i < 2 * BN; i += kEpiThreads) {
         const int c = i < BN ? i : i - BN;
         ss[i] = c < nvalid_tile ? (i < BN ? p.scale[ng0 + c] : p.shift[ng0 + c]) : 0.f;
@@ -435,7 +447,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       const int cb0 = half * kChunks;
       uint4 rres[4] = {};
       if constexpr (TMA_EPI) {
-        if (has_res) mbar_wait(&rbar[ob], (NB == 2 ? (it >> 1) : it) & 1);
+        if (has_res) mbar_wait(&rbar[ob], (it / NB) & 1);
       } else if (has_res && rvalid) {
 #pragma unroll
         for (int j = 0; j < 4; ++j)
@@ -504,6 +516,15 @@ __global__ void __launch_bounds__(kThreads, 1)
               tma_store_2d(&tmap_y, ng0 + st * 64, m0, sOb + st * BM * 128);
           }
           bulk_commit();
+          if (NB >= 3 && has_res) {
+            // buffer (it + NB - 1) % NB held tile it-1's output: once its stores have read it, prefetch
+            // the residual of this CTA's tile it + NB - 1 there (latency hidden behind ~NB - 2 tiles)
+            const int ahead = tile + (NB - 1) * (int)gridDim.x;
+            if (ahead < p.n_tiles) {
+              bulk_wait_read<1>();
+              issue_res(ahead, (it + NB - 1) % NB);
+            }
+          }
         }
         if (p.tapf) {
           // Fused tap: scan the staged bf16 tile column-wise (kEpiThreads / BN threads per column split
@@ -697,11 +718,12 @@ void conv_layer_free(ConvLayer& L) {
   L.scale = L.shift = nullptr;
 }
 
-template <int BN, int AMODE, bool TE>
+template <int BN, int AMODE, bool TE, int NB>
 static void launch_t(const ConvLayer& L, const CUtensorMap& ta, const CUtensorMap& ty, const CUtensorMap& tr,
                      const ConvParams& p, cudaStream_t st) {
-  auto kern = conv_tc_kernel<BN, AMODE, TE>;
-  constexpr int smem = Cfg<BN, TE>::kBytes;
+  static_assert(NB >= 1 && NB <= 4, "staging buffers");
+  auto kern = conv_tc_kernel<BN, AMODE, TE, NB>;
+  constexpr int smem = Cfg<BN, TE, NB>::kBytes;
   static bool attr_set = false;  // per instantiation
   if (!attr_set) {
     VCHECK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
@@ -712,22 +734,28 @@ static void launch_t(const ConvLayer& L, const CUtensorMap& ta, const CUtensorMa
   LAUNCHED();
 }
 
-template <int BN, bool TE>
+template <int BN, bool TE, int NB>
 static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, const CUtensorMap& ty,
                       const CUtensorMap& tr, const ConvParams& p, cudaStream_t st) {
   switch (amode) {
-    case A_TMA: launch_t<BN, A_TMA, TE>(L, ta, ty, tr, p, st); break;
-    case A_GATHER_FAST: launch_t<BN, A_GATHER_FAST, TE>(L, ta, ty, tr, p, st); break;
-    case A_GATHER_ROW: launch_t<BN, A_GATHER_ROW, TE>(L, ta, ty, tr, p, st); break;
-    case A_IM2COL: launch_t<BN, A_IM2COL, TE>(L, ta, ty, tr, p, st); break;
-    case A_IM2COL_C8: launch_t<BN, A_IM2COL_C8, TE>(L, ta, ty, tr, p, st); break;
+    case A_TMA: launch_t<BN, A_TMA, TE, NB>(L, ta, ty, tr, p, st); break;
+    case A_GATHER_FAST: launch_t<BN, A_GATHER_FAST, TE, NB>(L, ta, ty, tr, p, st); break;
+    case A_GATHER_ROW: launch_t<BN, A_GATHER_ROW, TE, NB>(L, ta, ty, tr, p, st); break;
+    case A_IM2COL: launch_t<BN, A_IM2COL, TE, NB>(L, ta, ty, tr, p, st); break;
+    case A_IM2COL_C8: launch_t<BN, A_IM2COL_C8, TE, NB>(L, ta, ty, tr, p, st); break;
     case A_ROWVIEW:
-      if constexpr (TE) launch_t<BN, A_ROWVIEW, TE>(L, ta, ty, tr, p, st);
+      if constexpr (TE) launch_t<BN, A_ROWVIEW, TE, NB>(L, ta, ty, tr, p, st);
       else fail(1, "conv: row-view mode needs the TMA epilogue");
       break;
-    default: launch_t<BN, A_GATHER_GENERAL, TE>(L, ta, ty, tr, p, st); break;
+    default: launch_t<BN, A_GATHER_GENERAL, TE, NB>(L, ta, ty, tr, p, st); break;
   }
 }
+
+// staging buffers of the TMA epilogue (VISTA_EPI_NB overrides for A/B measurements)
+static const int g_epi_nb_env = [] {
+  const char* e = getenv("VISTA_EPI_NB");
+  return e ? atoi(e) : 0;
+}();
 
 bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const bf16* res, bf16* y,
                   cudaStream_t st, unsigned int* tapf) {
@@ -820,19 +848,28 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   const double flops = 2.0 * (double)M * L.Cout * L.K_alg;  // algorithmic (unpadded) MACs x 2
   const double bytes = 2.0 * ((double)N * H * W * L.Cin + (double)M * L.Cout * (res ? 2 : 1) + (double)L.Cout * L.Kp);
   prof_begin(st);
+  int nb = 1;
   if (tma_epi) {
-    if (L.BN == 256) launch_bn<256, true>(L, amode, ta, ty, tr, p, st);
-    else if (L.BN == 128) launch_bn<128, true>(L, amode, ta, ty, tr, p, st);
-    else launch_bn<64, true>(L, amode, ta, ty, tr, p, st);
+    if (L.BN == 256) {
+      launch_bn<256, true, 1>(L, amode, ta, ty, tr, p, st);
+    } else if (L.BN == 128) {
+      nb = g_epi_nb_env == 2 ? 2 : 3;
+      if (nb == 2) launch_bn<128, true, 2>(L, amode, ta, ty, tr, p, st);
+      else launch_bn<128, true, 3>(L, amode, ta, ty, tr, p, st);
+    } else {
+      nb = g_epi_nb_env == 2 ? 2 : 4;
+      if (nb == 2) launch_bn<64, true, 2>(L, amode, ta, ty, tr, p, st);
+      else launch_bn<64, true, 4>(L, amode, ta, ty, tr, p, st);
+    }
   } else {
-    if (L.BN == 256) launch_bn<256, false>(L, amode, ta, ty, tr, p, st);
-    else if (L.BN == 128) launch_bn<128, false>(L, amode, ta, ty, tr, p, st);
-    else launch_bn<64, false>(L, amode, ta, ty, tr, p, st);
+    if (L.BN == 256) launch_bn<256, false, 1>(L, amode, ta, ty, tr, p, st);
+    else if (L.BN == 128) launch_bn<128, false, 1>(L, amode, ta, ty, tr, p, st);
+    else launch_bn<64, false, 1>(L, amode, ta, ty, tr, p, st);
   }
   char label[160] = {0};
   if (prof_labels())
-    snprintf(label, sizeof(label), "conv R%d S%d s%d g%d Cin%d Cout%d HxW%dx%d M%d K%d BN%d amode%d epi%d tiles%d%s", L.R,
-             L.S, L.stride, L.groups, L.Cin, L.Cout, H, W, p.M, L.K, L.BN, amode, tma_epi ? 1 : 0, p.n_tiles,
+    snprintf(label, sizeof(label), "conv R%d S%d s%d g%d Cin%d Cout%d HxW%dx%d M%d K%d BN%d amode%d epi%d nb%d tiles%d%s", L.R,
+             L.S, L.stride, L.groups, L.Cin, L.Cout, H, W, p.M, L.K, L.BN, amode, tma_epi ? 1 : 0, nb, p.n_tiles,
              res ? " res" : "");
   prof_end(st, 0, flops, bytes, label);
   return tapf == nullptr || fuse_tap;

@@ -1,0 +1,256 @@
+// conv1_pool.cu — ResNet50 stem fused: conv1 (7x7/2 pad 3, BN, ReLU; run as 4x4/1 on the 2x2
+// space-to-depth input, roster.h kS2dHW) followed by pool1 (3x3/2 max, unpadded; reading R4) in ONE
+// persistent tcgen05 kernel.  SURVEY.md §8a S1; the 114x114x64 conv1 activation (1.66 MB per
+// image) never reaches HBM: per image the kernel reads the 438 KB space-to-depth input once and
+// writes the 401 KB pooled [56, 56, 64] output.
+//
+// Each CTA owns whole images.  Tile = one conv output row ho (114 pixels in a 128-row M tile);
+// k-block r = filter row r reads input row ho + r through the overlapping TMA row view (the same
+// operand layout as conv_tc.cu's A_ROWVIEW mode), so every input row is loaded ONCE into a ring of
+// kSA shared-memory slots and reused by the four tiles that need it.  The 4 k-blocks of the
+// 64 x 256 weight matrix stay resident in shared memory for the whole kernel.
+// Epilogue (8 warps): TMEM -> BN scale/shift -> ReLU -> bf16 (RNE) conv row in shared memory; then
+// each thread owns fixed (pooled column j, 8-channel chunk) items: horizontal 3-max over conv
+// columns 2j..2j+2, and a running vertical max over conv rows 2i..2i+2 kept in registers; pooled
+// row i is stored (coalesced 16-byte stores) when conv row 2i+2 arrives.  Max is exact on bf16
+// values, so the result is bit-identical to conv_forward + launch_maxpool.
+#include <cstring>
+
+#include "internal.h"
+#include "ptx.cuh"
+#include "roster.h"
+
+namespace vista {
+
+namespace {
+
+constexpr int kHo = 114;           // conv1 output rows / cols (227 + 6 - 7) / 2 + 1
+constexpr int kHin = 117;          // space-to-depth input rows (kS2dHW)
+constexpr int kPo = 56;            // pool1 output (114 - 3) / 2 + 1
+constexpr int kCo = 64;            // conv1 channels
+constexpr int kSA = 8;             // input-row ring slots
+constexpr int kNAcc = 4;           // TMEM accumulators (64 columns each)
+constexpr int kRowBytes = 128 * 128;  // one A slot: 128 pixel rows x 64 bf16 (128B-swizzled)
+constexpr int kBBytes = 4 * 64 * 128;  // 4 k-blocks x 64 output channels x 64 bf16
+constexpr int kCrowBytes = 128 * 128;  // conv row: 128 pixels x 64 channels bf16
+constexpr int kEpiWarp0 = 2, kEpiWarps = 8, kEpiThreads = kEpiWarps * 32;
+constexpr int kThreads = (kEpiWarp0 + kEpiWarps) * 32;
+constexpr int kItems = kPo * 8;    // (pooled column, 8-channel chunk) items per pooled row
+constexpr int kOffB = 0, kOffA = kOffB + kBBytes, kOffCrow = kOffA + kSA * kRowBytes,
+              kOffSS = kOffCrow + 2 * kCrowBytes, kOffBar = kOffSS + 2 * kCo * 4;
+constexpr int kSmem = kOffBar + (2 * kSA + 2 * kNAcc + 2) * 8 + 1024;
+
+struct PoolParams {
+  bf16* y;  // [N, 56, 56, 64]
+  const float* scale;
+  const float* shift;
+  int N;
+};
+
+__device__ __forceinline__ uint4 max4(uint4 a, uint4 b) {
+  uint4 o;
+  const __nv_bfloat162* pa = reinterpret_cast<const __nv_bfloat162*>(&a);
+  const __nv_bfloat162* pb = reinterpret_cast<const __nv_bfloat162*>(&b);
+  __nv_bfloat162* po = reinterpret_cast<__nv_bfloat162*>(&o);
+#pragma unroll
+  for (int j = 0; j < 4; ++j) po[j] = __hmax2(pa[j], pb[j]);
+  return o;
+}
+
+__global__ void __launch_bounds__(kThreads, 1)
+    conv1_pool_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__ CUtensorMap tmap_a,
+                      const PoolParams p) {
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  const uint32_t base = (raw + 1023u) & ~1023u;
+  uint8_t* gbase = smem_raw + (base - raw);
+  const uint32_t sB = base + kOffB, sA = base + kOffA, sC = base + kOffCrow;
+  float* ss = reinterpret_cast<float*>(gbase + kOffSS);  // [scale 64 | shift 64]
+  uint64_t* full = reinterpret_cast<uint64_t*>(gbase + kOffBar);
+  uint64_t* empty = full + kSA;
+  uint64_t* tfull = empty + kSA;
+  uint64_t* tempty = tfull + kNAcc;
+  uint64_t* bbar = tempty + kNAcc;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bbar + 1);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kSA; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&empty[i], 1);
+    }
+    for (int i = 0; i < kNAcc; ++i) {
+      mbar_init(&tfull[i], 1);
+      mbar_init(&tempty[i], kEpiWarps);
+    }
+    mbar_init(bbar, 1);
+    fence_mbar_init();
+    tma_prefetch(&tmap_w);
+    tma_prefetch(&tmap_a);
+  }
+  if (threadIdx.x < 2 * kCo) ss[threadIdx.x] = threadIdx.x < kCo ? p.scale[threadIdx.x] : p.shift[threadIdx.x - kCo];
+  if (warp == 1) tmem_alloc(tmem_slot, kNAcc * kCo);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    // ======================= producer: weights once, then every input row once =======================
+    if (lane == 0) {
+      mbar_arrive_expect_tx(bbar, kBBytes);
+      for (int r = 0; r < 4; ++r) tma_load_2d(sB + r * 64 * 128, &tmap_w, r * 64, 0, bbar);
+      uint32_t g = 0;
+      for (int n = blockIdx.x; n < p.N; n += gridDim.x) {
+        for (int i = 0; i < kHin; ++i, ++g) {
+          const int slot = g % kSA;
+          if (g >= (uint32_t)kSA) mbar_wait(&empty[slot], ((g / kSA) - 1) & 1);
+          mbar_arrive_expect_tx(&full[slot], kRowBytes);
+          tma_load_4d(sA + slot * kRowBytes, &tmap_a, 0, 0, i, n, &full[slot]);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ======================= MMA issuer =======================
+    if (lane == 0) {
+      constexpr uint32_t idesc = umma_idesc_bf16(128, kCo);
+      mbar_wait(bbar, 0);
+      uint32_t gbase_row = 0, it = 0;
+      for (int n = blockIdx.x; n < p.N; n += gridDim.x, gbase_row += kHin) {
+        for (int ho = 0; ho < kHo; ++ho, ++it) {
+          const uint32_t acc = it % kNAcc;
+          if (it >= (uint32_t)kNAcc) mbar_wait(&tempty[acc], ((it / kNAcc) - 1) & 1);
+          tc_fence_after();
+          const uint32_t tacc = tmem_base + acc * kCo;
+#pragma unroll 1
+          for (int r = 0; r < 4; ++r) {
+            const uint32_t row = gbase_row + ho + r;
+            const uint32_t slot = row % kSA;
+            mbar_wait(&full[slot], (row / kSA) & 1);
+            tc_fence_after();
+            const uint32_t a0 = sA + slot * kRowBytes, b0 = sB + r * 64 * 128;
+#pragma unroll
+            for (int k = 0; k < 4; ++k)
+              tc_mma_bf16(tacc, umma_desc_k_sw128(a0 + k * 32), umma_desc_k_sw128(b0 + k * 32), idesc,
+                          (r | k) != 0 ? 1u : 0u);
+          }
+          tc_commit(&tfull[acc]);
+          // input row ho is not read by any later tile of this image
+          tc_commit(&empty[(gbase_row + ho) % kSA]);
+          if (ho == kHo - 1)
+            for (int r = 1; r < 4; ++r) tc_commit(&empty[(gbase_row + ho + r) % kSA]);
+        }
+      }
+    }
+    __syncwarp();
+  } else {
+    // ======================= epilogue: BN + ReLU + 3x3/2 max pool =======================
+    const int et = threadIdx.x - kEpiWarp0 * 32;
+    const int q = warp & 3;                    // TMEM lane quadrant
+    const int half = (warp - kEpiWarp0) >> 2;  // channel half (32 channels)
+    const int wo = q * 32 + lane;              // conv output column (M row of the tile)
+    const int i0 = et, i1 = et + kEpiThreads;  // this thread's pooling items
+    uint32_t it = 0;
+    for (int n = blockIdx.x; n < p.N; n += gridDim.x) {
+      uint4 vb0[2], vb1[2];  // running vertical max of the open pooled rows (even / odd i), per item
+#pragma unroll
+      for (int u = 0; u < 2; ++u) vb0[u] = vb1[u] = make_uint4(0, 0, 0, 0);
+      bf16* yimg = p.y + (size_t)n * kPo * kPo * kCo;
+      for (int ho = 0; ho < kHo; ++ho, ++it) {
+        const uint32_t acc = it % kNAcc;
+        mbar_wait(&tfull[acc], (it / kNAcc) & 1);
+        tc_fence_after();
+        uint32_t v[32];
+        tmem_ld_32x32b_x32(tmem_base + acc * kCo + half * 32 + ((uint32_t)(q * 32) << 16), v);
+        tc_wait_ld();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&tempty[acc]);
+        const uint32_t crow = sC + (ho & 1) * kCrowBytes + wo * 128;
+        if (wo < kHo) {
+#pragma unroll
+          for (int c4 = 0; c4 < 4; ++c4) {  // 8 channels per 16-byte chunk
+            const int ch0 = half * 32 + c4 * 8;
+            float f[8];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) f[j] = fmaxf(fmaf(__uint_as_float(v[c4 * 8 + j]), ss[ch0 + j], ss[kCo + ch0 + j]), 0.f);
+            uint4 o;
+            o.x = pack_bf16x2(f[0], f[1]);
+            o.y = pack_bf16x2(f[2], f[3]);
+            o.z = pack_bf16x2(f[4], f[5]);
+            o.w = pack_bf16x2(f[6], f[7]);
+            const uint32_t chunk = (uint32_t)(half * 4 + c4);
+            sts128(crow + ((chunk ^ (uint32_t)(wo & 7)) << 4), o);
+          }
+        }
+        named_bar_sync(1, kEpiThreads);
+        // conv row ho -> pooled rows: even ho closes i = ho/2 - 1 and opens i = ho/2; odd ho extends (ho-1)/2
+        const uint32_t cbase = sC + (ho & 1) * kCrowBytes;
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+          const int item = u == 0 ? i0 : i1;
+          if (item >= kItems) continue;
+          const int j = item >> 3, c = item & 7;
+          const int w0 = 2 * j;
+          const uint4 a = lds128(cbase + w0 * 128 + (((uint32_t)c ^ (uint32_t)(w0 & 7)) << 4));
+          const uint4 b = lds128(cbase + (w0 + 1) * 128 + (((uint32_t)c ^ (uint32_t)((w0 + 1) & 7)) << 4));
+          const uint4 d = lds128(cbase + (w0 + 2) * 128 + (((uint32_t)c ^ (uint32_t)((w0 + 2) & 7)) << 4));
+          const uint4 h = max4(max4(a, b), d);
+          if ((ho & 1) == 0) {
+            const int io = ho >> 1;
+            if (ho >= 2) {  // close pooled row io - 1 (conv rows ho - 2, ho - 1, ho)
+              const uint4 o = max4((io & 1) ? vb0[u] : vb1[u], h);
+              *reinterpret_cast<uint4*>(yimg + ((size_t)(io - 1) * kPo + j) * kCo + c * 8) = o;
+            }
+            if (io < kPo) {  // open pooled row io
+              if (io & 1) vb1[u] = h;
+              else vb0[u] = h;
+            }
+          } else {
+            const int ie = (ho - 1) >> 1;  // middle row of pooled row ie
+            if (ie < kPo) {
+              if (ie & 1) vb1[u] = max4(vb1[u], h);
+              else vb0[u] = max4(vb0[u], h);
+            }
+          }
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) tmem_dealloc(tmem_base, kNAcc * kCo);
+}
+
+}  // namespace
+
+bool conv1_pool_supported(const ConvLayer& L, int H, int W) {
+  return L.rowview && L.Cin == kS2dC && L.Cout == kCo && L.R == 4 && L.S == 4 && L.BN == kCo && H == kHin &&
+         W == kHin && L.relu;
+}
+
+void conv1_pool_forward(const ConvLayer& L, const bf16* x, int N, bf16* y, cudaStream_t st) {
+  if (N <= 0) return;
+  CUtensorMap ta;
+  // overlapping row view {64 elements, q < 114, h, n}: element (k, q, h, n) = x[n, h, q + k / 16, k % 16]
+  if (!make_rowview_tmap(&ta, x, N, kHin, kHin, kS2dC, kHo)) fail(5, "conv1_pool: row-view tensor map failed");
+  PoolParams p;
+  p.y = y;
+  p.scale = L.scale;
+  p.shift = L.shift;
+  p.N = N;
+  static bool attr = false;
+  if (!attr) {
+    VCHECK(cudaFuncSetAttribute(conv1_pool_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem));
+    attr = true;
+  }
+  const int grid = N < num_sms() ? N : num_sms();
+  prof_begin(st);
+  conv1_pool_kernel<<<grid, kThreads, kSmem, st>>>(L.tmap_w, ta, p);
+  LAUNCHED();
+  const double flops = 2.0 * (double)N * kHo * kHo * kCo * L.K_alg;
+  const double bytes = (double)N * (kHin * kHin * kS2dC * 2 + kPo * kPo * kCo * 2) + (double)kCo * L.Kp * 2;
+  prof_end(st, 0, flops, bytes, prof_labels() ? "conv1+pool1 fused (s2d rowview)" : nullptr);
+}
+
+}  // namespace vista

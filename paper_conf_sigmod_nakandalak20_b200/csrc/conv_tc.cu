@@ -665,6 +665,15 @@ static CUresult encode_nd(CUtensorMap* m, const void* ptr, int rank, const cuuin
                       CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
 }
 
+// overlapping 4-D row view of an NHWC input with C * S == 64 (A_ROWVIEW): element (k, q, h, n) =
+// x[n, h, q + k / C, k % C] for q < Wo; box {64, 128, 1, 1}, 128B-swizzled (q >= Wo reads zeros)
+bool make_rowview_tmap(CUtensorMap* m, const void* x, int N, int H, int W, int C, int Wo) {
+  const cuuint64_t dims[4] = {(cuuint64_t)BK, (cuuint64_t)Wo, (cuuint64_t)H, (cuuint64_t)N};
+  const cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)W * C * 2, (cuuint64_t)H * W * C * 2};
+  const cuuint32_t box[4] = {(cuuint32_t)BK, (cuuint32_t)BM, 1, 1};
+  return encode_nd(m, x, 4, dims, strides, box) == CUDA_SUCCESS;
+}
+
 static int pick_bn(int Cg_out, int groups, int K) {
   // short-K layers are epilogue/HBM-bound: 128-wide tiles get a double-buffered output staging
   if (K <= 256 && Cg_out % 128 == 0) return 128;
@@ -797,13 +806,10 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   bool rowview = false;
   if (L.rowview && g_rowview_enabled && p.Wo <= BM && !res && L.R <= 8 && L.Cout % 8 == 0) {
     // overlapping 4-D view of the input: element (k, q, h, n) = x[n, h, q + k / Cin, k % Cin]
-    const cuuint64_t dims[4] = {(cuuint64_t)BK, (cuuint64_t)p.Wo, (cuuint64_t)H, (cuuint64_t)N};
-    const cuuint64_t strides[3] = {(cuuint64_t)L.Cin * 2, (cuuint64_t)W * L.Cin * 2, (cuuint64_t)H * W * L.Cin * 2};
-    const cuuint32_t box[4] = {(cuuint32_t)BK, (cuuint32_t)BM, 1, 1};
     const cuuint64_t odims[3] = {(cuuint64_t)L.Cout, (cuuint64_t)p.Wo, (cuuint64_t)N * p.Ho};
     const cuuint64_t ostr[2] = {(cuuint64_t)L.Cout * 2, (cuuint64_t)p.Wo * L.Cout * 2};
     const cuuint32_t obox[3] = {(cuuint32_t)BK, (cuuint32_t)BM, 1};
-    if (encode_nd(&ta, x, 4, dims, strides, box) == CUDA_SUCCESS &&
+    if (make_rowview_tmap(&ta, x, N, H, W, L.Cin, p.Wo) &&
         encode_nd(&ty, y, 3, odims, ostr, obox) == CUDA_SUCCESS) {
       rowview = true;
       p.n_mt = N * p.Ho;  // one tile per output row; rows q >= Wo of a tile are padding

@@ -60,6 +60,12 @@ void conv_layer_free(ConvLayer& L);
 // (2x2-grid maxima); returns false if the tap could not be fused (caller runs launch_tap instead).
 bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const bf16* res, bf16* y,
                   cudaStream_t st, unsigned int* tapf = nullptr);
+bool make_rowview_tmap(CUtensorMap* m, const void* x, int N, int H, int W, int C, int Wo);
+// ResNet50 stem: conv1 (s2d row view) + BN + ReLU + pool1 3x3/2 in one kernel (conv1_pool.cu):
+// x bf16 [N, 117, 117, 16] space-to-depth input -> y bf16 [N, 56, 56, 64], bit-identical to
+// conv_forward + launch_maxpool.
+bool conv1_pool_supported(const ConvLayer& L, int H, int W);
+void conv1_pool_forward(const ConvLayer& L, const bf16* x, int N, bf16* y, cudaStream_t st);
 // F bf16 [n, 4C] <- fp32 tap accumulator (exact: the maxima are bf16 values)
 void launch_tap_finalize(const unsigned int* tapf, int64_t count, bf16* F, cudaStream_t st);
 inline int conv_out_dim(int H, int k, int s, int p) { return (H + 2 * p - k) / s + 1; }

@@ -230,6 +230,8 @@ struct vista_ctx {
   // (its per-(image, quadrant, channel) red.max traffic, ~10M per 1024-image launch, slows the epilogue
   // of the HBM-bound producer convs by ~40 ms/step) vs standalone 59.3k img/s (4.3 ms/step re-reading A_k).
   bool fuse_tap = false;
+  // ResNet conv1 + pool1 in one kernel (conv1_pool.cu, bit-identical); VISTA_FUSE_STEM=0 disables
+  bool fuse_stem = true;
   std::vector<void*> feat;  // per block: device pointer of F_t (features) of a tapped layer
   std::string last_error;
   ~vista_ctx() {
@@ -521,9 +523,18 @@ bool run_ops(vista_ctx* c, int t, const void* in_ptr, void* out_ptr, int nb, voi
       }
       return tapf == nullptr;
     }
-    for (const OpDesc& op : S.ops) {
+    for (size_t oi = 0; oi < S.ops.size(); ++oi) {
+      const OpDesc& op = S.ops[oi];
       const bf16* in = reinterpret_cast<const bf16*>(slot[op.in]);
       bf16* out = reinterpret_cast<bf16*>(slot[op.out]);
+      // ResNet stem: conv1 + pool1 fused (the conv1 activation never reaches HBM)
+      if (op.kind == OP_CONV && c->fuse_stem && oi + 1 < S.ops.size() && S.ops[oi + 1].kind == OP_MAXPOOL &&
+          S.ops[oi + 1].in == op.out && S.ops[oi + 1].k == 3 && S.ops[oi + 1].s == 2 &&
+          conv1_pool_supported(c->convs[op.layer], op.H, op.W) && !(tapf && S.ops[oi + 1].out == BUF_OUT)) {
+        conv1_pool_forward(c->convs[op.layer], in, nb, reinterpret_cast<bf16*>(slot[S.ops[oi + 1].out]), c->stream);
+        ++oi;
+        continue;
+      }
       switch (op.kind) {
         case OP_INGEST:
           launch_ingest(reinterpret_cast<const uint8_t*>(slot[op.in]), nb, out, c->stream);
@@ -733,6 +744,7 @@ VISTA_API vista_status vista_plan(vista_cnn cnn, const int32_t* layers, int32_t 
     }
     c->prof.reset(new Profiler());
     if (const char* e = getenv("VISTA_FUSED_TAP")) c->fuse_tap = e[0] != '0';
+    if (const char* e = getenv("VISTA_FUSE_STEM")) c->fuse_stem = e[0] != '0';
     VCHECK(cudaStreamSynchronize(c->stream));
   });
   if (st != VISTA_OK) {

@@ -212,3 +212,17 @@ def test_no_plan_within_tiny_budget():
     with pytest.raises(VistaError) as e:
         Vista(2, n_top=5, n_str_rows=1000, d_s=130, n_images_local=1000, hbm_budget_bytes=64 << 20)
     assert e.value.status == 2
+
+
+def test_resnet_stem_fused_bit_identical(monkeypatch):
+    # conv1 + pool1 run as one kernel (conv1_pool.cu) by default; VISTA_FUSE_STEM=0 runs conv_tc + maxpool.
+    # Max pooling is exact on the bf16 conv outputs, so every bit of MM_l must agree.
+    tab = gen.make_tables(150, 8)  # > 148 images: CTAs own several images
+    out = {}
+    for fuse in ("1", "0"):
+        monkeypatch.setenv("VISTA_FUSE_STEM", fuse)
+        v = run_gpu(2, [0, 4], tab, 8, iters=1, micro_batch=150)
+        out[fuse] = [v.features(k)["mm"].view(torch.int16).cpu().clone() for k in range(2)]
+        v.close()
+    for a, b in zip(out["1"], out["0"]):
+        assert torch.equal(a, b)

@@ -46,13 +46,16 @@ __device__ __forceinline__ void bulk_load(uint32_t dst, const void* src, uint32_
 
 // One pass over rows [r0, r1) of MM.  Rows are streamed into shared memory in blocks of
 // rb contiguous rows by the bulk-copy engine (kStagesLR blocks in flight per CTA, one CTA per
-// SM), so HBM stays busy while the threads compute.  Thread t owns 16-byte column chunks
-// t, t + blockDim, ... of every row.
+// SM) issued by a dedicated producer warp, so HBM stays busy while the compute threads work.
+// Compute thread t owns 16-byte column chunks t, t + nthr, ... of every row.
 //   MODE 0: sum_p x_pj                          MODE 1: sum_p (x_pj - mu_j)^2
 //   MODE 2: power pass  phi_p = z_p             MODE 3: gradient pass  phi_p = sigmoid(z_p) - y_p
 //   MODE 4: evaluation (counts only)
-// with z_p = b^ + sum_j w^_j (x_pj - mu_j); modes 2/3 accumulate sum_p phi_p (x_pj - mu_j),
-// sum_p phi_p and sum_p loss_p into this CTA's partial row (fixed row-block -> CTA map).
+// with z_p = b' + sum_j w^_j x_pj, b' = b^ - sum_j w^_j mu_j (the centred score, folded on the host
+// side of the pass in fp64); modes 2/3 accumulate sum_p phi_p x_pj, sum_p phi_p and sum_p loss_p into
+// this CTA's partial row (fixed row-block -> CTA map); the reduction subtracts mu_j sum_p phi_p.
+// One named barrier per row block (the per-row dot products); stages are recycled through
+// "empty" mbarriers, so compute warps never wait for the producer's refills.
 template <typename E>
 __device__ __forceinline__ void unpack16(uint4 v, float (&x)[16 / sizeof(E)]);
 template <>
@@ -60,9 +63,8 @@ __device__ __forceinline__ void unpack16<bf16>(uint4 v, float (&x)[8]) {
   const uint32_t u[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
   for (int j = 0; j < 4; ++j) {
-    const float2 f = unpack_bf16x2(u[j]);
-    x[2 * j] = f.x;
-    x[2 * j + 1] = f.y;
+    x[2 * j] = __uint_as_float(u[j] << 16);
+    x[2 * j + 1] = __uint_as_float(u[j] & 0xffff0000u);
   }
 }
 template <>
@@ -74,46 +76,55 @@ __device__ __forceinline__ void unpack16<float>(uint4 v, float (&x)[4]) {
 }
 
 template <int CH, int MODE, typename E>
-__global__ void __launch_bounds__(kLRThreads, 1) lr_stream_kernel(const PassArgs a) {
+__global__ void __launch_bounds__(kLRThreads + 32, 1) lr_stream_kernel(const PassArgs a) {
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 127u) & ~127u;
   uint8_t* gbase = smem_raw + (base - raw);
   const uint32_t row_bytes = (uint32_t)a.ld * (uint32_t)sizeof(E);
   const uint32_t stage_bytes = ((uint32_t)a.rb * row_bytes + 127u) & ~127u;
-  float* red = reinterpret_cast<float*>(gbase + kStagesLR * stage_bytes);  // [kMaxRB][32]
-  float* phis = red + kMaxRB * 32;                                         // [kMaxRB]
-  uint64_t* full = reinterpret_cast<uint64_t*>(phis + kMaxRB);             // [kStagesLR]
+  float* red_all = reinterpret_cast<float*>(gbase + kStagesLR * stage_bytes);  // [kStagesLR][kMaxRB][32]
+  uint64_t* full = reinterpret_cast<uint64_t*>(red_all + kStagesLR * kMaxRB * 32);  // [kStagesLR]
+  uint64_t* empty = full + kStagesLR;                                               // [kStagesLR]
 
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarps = blockDim.x >> 5;
+  const int nthr = (int)blockDim.x - 32;  // compute threads; the last warp is the producer
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwc = nthr >> 5;
   const int64_t nrows = a.r1 - a.r0;
   const int64_t nblk = (nrows + a.rb - 1) / a.rb;
   if (tid == 0) {
-    for (int i = 0; i < kStagesLR; ++i) mbar_init(&full[i], 1);
+    for (int i = 0; i < kStagesLR; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&empty[i], nthr);
+    }
     fence_mbar_init();
   }
   __syncthreads();
-  auto issue = [&](int64_t blk, int stage) {
-    const int64_t r = a.r0 + blk * a.rb;
-    const int64_t nr = min((int64_t)a.rb, a.r1 - r);
-    const uint32_t bytes = (uint32_t)nr * row_bytes;
-    mbar_arrive_expect_tx(&full[stage], bytes);
-    bulk_load(base + stage * stage_bytes, a.MM + (size_t)r * row_bytes, bytes, &full[stage]);
-  };
-  if (tid == 0) {
-    int i = 0;
-    for (int64_t blk = blockIdx.x; blk < nblk && i < kStagesLR; blk += gridDim.x, ++i) issue(blk, i);
+  if (warp == nwc) {
+    // ---- producer warp ----
+    if (lane == 0) {
+      int it = 0;
+      for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++it) {
+        const int stage = it % kStagesLR;
+        if (it >= kStagesLR) mbar_wait(&empty[stage], ((it / kStagesLR) - 1) & 1);
+        const int64_t r = a.r0 + blk * a.rb;
+        const int64_t nr = min((int64_t)a.rb, a.r1 - r);
+        const uint32_t bytes = (uint32_t)nr * row_bytes;
+        mbar_arrive_expect_tx(&full[stage], bytes);
+        bulk_load(base + stage * stage_bytes, a.MM + (size_t)r * row_bytes, bytes, &full[stage]);
+      }
+    }
+    return;
   }
   constexpr int EPC = 16 / (int)sizeof(E);  // elements per 16-byte chunk: 8 bf16 or 4 fp32
   float mu[CH][EPC], wv[CH][EPC], acc[CH][EPC];
   bool act[CH];
 #pragma unroll
   for (int c = 0; c < CH; ++c) {
-    const int ch = tid + c * blockDim.x;
+    const int ch = tid + c * nthr;
     act[c] = ch < a.chunks;
 #pragma unroll
     for (int j = 0; j < EPC; ++j) {
-      mu[c][j] = (MODE != 0 && act[c]) ? a.mu[ch * EPC + j] : 0.f;
+      mu[c][j] = (MODE == 1 && act[c]) ? a.mu[ch * EPC + j] : 0.f;
       wv[c][j] = (MODE >= 2 && act[c]) ? a.what[ch * EPC + j] : 0.f;
       acc[c][j] = 0.f;
     }
@@ -134,7 +145,7 @@ __global__ void __launch_bounds__(kLRThreads, 1) lr_stream_kernel(const PassArgs
         for (int c = 0; c < CH; ++c) {
           if (!act[c]) continue;
           float x[EPC];
-          unpack16<E>(lds128(sbase + q * row_bytes + (uint32_t)(tid + c * blockDim.x) * 16u), x);
+          unpack16<E>(lds128(sbase + q * row_bytes + (uint32_t)(tid + c * nthr) * 16u), x);
 #pragma unroll
           for (int j = 0; j < EPC; ++j) {
             if (MODE == 0) {
@@ -147,36 +158,40 @@ __global__ void __launch_bounds__(kLRThreads, 1) lr_stream_kernel(const PassArgs
         }
       }
     } else {
+      float* red = red_all + stage * (kMaxRB * 32);
       for (int q = 0; q < nr; ++q) {
         float sdot = 0.f;
 #pragma unroll
         for (int c = 0; c < CH; ++c) {
           if (!act[c]) continue;
           float x[EPC];
-          unpack16<E>(lds128(sbase + q * row_bytes + (uint32_t)(tid + c * blockDim.x) * 16u), x);
+          unpack16<E>(lds128(sbase + q * row_bytes + (uint32_t)(tid + c * nthr) * 16u), x);
 #pragma unroll
-          for (int j = 0; j < EPC; ++j) sdot = fmaf(x[j] - mu[c][j], wv[c][j], sdot);
+          for (int j = 0; j < EPC; ++j) sdot = fmaf(x[j], wv[c][j], sdot);
         }
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) sdot += __shfl_xor_sync(0xffffffffu, sdot, o);
         if (lane == 0) red[q * 32 + warp] = sdot;
       }
-      __syncthreads();
-      if (warp == 0 && lane < nr) {
+      named_bar_sync(1, nthr);
+      // every warp: lane q < nr forms z_q from the per-warp partials (fixed order) and phi_q
+      float phi = 0.f;
+      if (lane < nr) {
         float z = bh;
-        for (int w = 0; w < nwarps; ++w) z += red[lane * 32 + w];  // fixed order
+        for (int w = 0; w < nwc; ++w) z += red[lane * 32 + w];
         const int64_t row = r + lane;
         if (MODE == 2) {
-          phis[lane] = z;
-          sum_r += z;
+          phi = z;
+          if (warp == 0) sum_r += z;
         } else {
           const int yv = a.y[row];
           if (MODE == 3) {
-            const float ph = 1.f / (1.f + __expf(-z)) - (float)yv;
-            phis[lane] = ph;
-            sum_r += ph;
-            sum_loss += softplusf(z) - (float)yv * z;
-          } else {  // MODE 4: predict 1 iff z >= 0
+            phi = 1.f / (1.f + __expf(-z)) - (float)yv;
+            if (warp == 0) {
+              sum_r += phi;
+              sum_loss += softplusf(z) - (float)yv * z;
+            }
+          } else if (warp == 0) {  // MODE 4: predict 1 iff z >= 0
             const int pred = z >= 0.f ? 1 : 0;
             if (row < a.n_train) cnt[0] += pred == yv;
             else cnt[pred && yv ? 1 : (pred ? 2 : (yv ? 4 : 3))] += 1;
@@ -184,25 +199,20 @@ __global__ void __launch_bounds__(kLRThreads, 1) lr_stream_kernel(const PassArgs
         }
       }
       if (MODE == 2 || MODE == 3) {
-        __syncthreads();
         for (int q = 0; q < nr; ++q) {
-          const float ph = phis[q];
+          const float ph = __shfl_sync(0xffffffffu, phi, q);
 #pragma unroll
           for (int c = 0; c < CH; ++c) {
             if (!act[c]) continue;
             float x[EPC];
-            unpack16<E>(lds128(sbase + q * row_bytes + (uint32_t)(tid + c * blockDim.x) * 16u), x);
+            unpack16<E>(lds128(sbase + q * row_bytes + (uint32_t)(tid + c * nthr) * 16u), x);
 #pragma unroll
-            for (int j = 0; j < EPC; ++j) acc[c][j] = fmaf(ph, x[j] - mu[c][j], acc[c][j]);
+            for (int j = 0; j < EPC; ++j) acc[c][j] = fmaf(ph, x[j], acc[c][j]);
           }
         }
       }
     }
-    __syncthreads();  // every thread is done with this stage (and with red / phis)
-    if (tid == 0) {
-      const int64_t nb = blk + (int64_t)kStagesLR * gridDim.x;
-      if (nb < nblk) issue(nb, stage);
-    }
+    mbar_arrive(&empty[stage]);  // this thread is done with the stage
   }
   if constexpr (MODE == 4) {
     if (warp == 0) {
@@ -218,7 +228,7 @@ __global__ void __launch_bounds__(kLRThreads, 1) lr_stream_kernel(const PassArgs
   float* out = a.partial + (size_t)blockIdx.x * (a.ld + 4);
 #pragma unroll
   for (int c = 0; c < CH; ++c) {
-    const int ch = tid + c * blockDim.x;
+    const int ch = tid + c * nthr;
     if (act[c]) {
       float4* o = reinterpret_cast<float4*>(out + ch * EPC);
 #pragma unroll
@@ -238,12 +248,33 @@ __global__ void __launch_bounds__(kLRThreads, 1) lr_stream_kernel(const PassArgs
   }
 }
 
-// G[j] = sum_cta partial[cta][j] in fp64, fixed order; ncols = ld + 2, row pitch ld + 4
-__global__ void reduce_partials_kernel(const float* __restrict__ partial, int nct, int ncols, int pitch, double* G) {
-  for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < ncols; j += gridDim.x * blockDim.x) {
-    double s = 0.0;
-    for (int c = 0; c < nct; ++c) s += (double)partial[(size_t)c * pitch + j];
-    G[j] = s;
+// G[j] = sum_cta partial[cta][j] in fp64, fixed order (8 contiguous CTA ranges, one per warp, then
+// the 8 range sums in order); ncols = ld + 2, row pitch ld + 4.  center (power / gradient passes):
+// G[j] -= mu_j G[ld] for j < ld, turning sum_p phi_p x_pj into sum_p phi_p (x_pj - mu_j).
+// One block per 32 columns; every block forms G[ld] with the same order, so all agree bit for bit.
+__global__ void __launch_bounds__(256) reduce_partials_kernel(const float* __restrict__ partial, int nct, int ncols,
+                                                              int pitch, const double* __restrict__ mu, int ld,
+                                                              int center, double* G) {
+  __shared__ double sh[8][33];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int c0 = (int)((int64_t)nct * warp / 8), c1 = (int)((int64_t)nct * (warp + 1) / 8);
+  const int j = blockIdx.x * 32 + lane;
+  double s = 0.0, t = 0.0;
+  for (int c = c0; c < c1; ++c) {
+    if (j < ncols) s += (double)partial[(size_t)c * pitch + j];
+    if (center) t += (double)partial[(size_t)c * pitch + ld];
+  }
+  sh[warp][lane] = s;
+  if (lane == 0) sh[warp][32] = t;
+  __syncthreads();
+  if (warp == 0 && j < ncols) {
+    double g = 0.0, phisum = 0.0;
+    for (int w = 0; w < 8; ++w) {
+      g += sh[w][lane];
+      phisum += sh[w][32];
+    }
+    if (center && j < ld) g -= mu[j] * phisum;
+    G[j] = g;
   }
 }
 
@@ -285,7 +316,7 @@ __global__ void stats_finalize_kernel(const double* G, int ld, int step, const u
 // update: q_j = inv_j G_j / n, q_b = G_ld / n, lambda = ||q||, v = q / lambda.
 // Both end by publishing w^ = inv * v (fp32) and b^ = v_b for the next pass.
 __global__ void power_kernel(const double* G, int ld, int init, int d_real, const uint8_t* real, const double* inv,
-                             double* v, float* what, float* bhat, LRState* st) {
+                             const double* mu, double* v, float* what, float* bhat, LRState* st) {
   __shared__ double sh[32];
   const double n = st->n_train;
   if (init) {
@@ -307,15 +338,20 @@ __global__ void power_kernel(const double* G, int ld, int init, int d_real, cons
     }
   }
   __syncthreads();
-  for (int j = threadIdx.x; j < ld; j += blockDim.x) what[j] = (float)(inv[j] * v[j]);
-  if (threadIdx.x == 0) bhat[0] = (float)st->vb;
+  double sm = 0.0;
+  for (int j = threadIdx.x; j < ld; j += blockDim.x) {
+    what[j] = (float)(inv[j] * v[j]);
+    sm += inv[j] * v[j] * mu[j];
+  }
+  sm = block_sum(sm, sh);
+  if (threadIdx.x == 0) bhat[0] = (float)(st->vb - sm);  // centred score folded into the bias
 }
 
 // ISTA (O6 steps 4-5).  init: eta = 1 / (0.25 * 1.05 * lambda_hat + lambda (1 - alpha)), w = 0, b = 0.
 // update: g_j = inv_j G_j / n + lambda (1 - alpha) w_j; w = soft(w - eta g, eta lambda alpha);
 //         b -= eta G_ld / n; loss = G_{ld+1} / n (at the pre-update w).
 __global__ void grad_kernel(const double* G, int ld, int init, double lambda, double alpha, const double* inv,
-                            double* w, float* what, float* bhat, LRState* st, double* loss_out) {
+                            const double* mu, double* w, float* what, float* bhat, LRState* st, double* loss_out) {
   if (init) {
     for (int j = threadIdx.x; j < ld; j += blockDim.x) w[j] = 0.0;
     if (threadIdx.x == 0) {
@@ -335,8 +371,14 @@ __global__ void grad_kernel(const double* G, int ld, int init, double lambda, do
     }
   }
   __syncthreads();
-  for (int j = threadIdx.x; j < ld; j += blockDim.x) what[j] = (float)(inv[j] * w[j]);
-  if (threadIdx.x == 0) bhat[0] = (float)st->b;
+  __shared__ double sh[32];
+  double sm = 0.0;
+  for (int j = threadIdx.x; j < ld; j += blockDim.x) {
+    what[j] = (float)(inv[j] * w[j]);
+    sm += inv[j] * w[j] * mu[j];
+  }
+  sm = block_sum(sm, sh);
+  if (threadIdx.x == 0) bhat[0] = (float)(st->b - sm);  // centred score folded into the bias
 }
 
 // ------------------------------------------------------------------------------------------
@@ -355,7 +397,7 @@ static void run_pass(const PassArgs& a, const StreamCfg& c, cudaStream_t st) {
       if (done.insert((const void*)kern).second)
         VCHECK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
     }
-    kern<<<c.grid, c.threads, c.smem, st>>>(a);
+    kern<<<c.grid, c.threads + 32, c.smem, st>>>(a);
   };
   switch (c.ch) {
     case 1: go(lr_stream_kernel<1, MODE, E>); break;
@@ -383,9 +425,9 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   cfg.ch = (chunks + cfg.threads - 1) / cfg.threads;
   if (cfg.ch > 6) fail(1, "lr: row too wide");
   if (cfg.ch == 3 && chunks <= 2 * cfg.threads) cfg.ch = 2;
-  cfg.rb = (int)std::max<int64_t>(1, std::min<int64_t>(kMaxRB, 65536 / ((int64_t)ld * esz)));
+  cfg.rb = (int)std::max<int64_t>(1, std::min<int64_t>(kMaxRB, (200 * 1024 / kStagesLR) / ((int64_t)ld * esz)));
   const size_t stage_bytes = ((size_t)cfg.rb * ld * esz + 127) & ~(size_t)127;
-  cfg.smem = kStagesLR * stage_bytes + kMaxRB * 32 * 4 + kMaxRB * 4 + kStagesLR * 8 + 128;
+  cfg.smem = kStagesLR * stage_bytes + kStagesLR * kMaxRB * 32 * 4 + 2 * kStagesLR * 8 + 128;
   if (cfg.smem > 227 * 1024) fail(1, "lr: row block does not fit in shared memory");
   auto grid_for_rows = [&](int64_t rows) {
     const int64_t blocks = (rows + cfg.rb - 1) / cfg.rb;
@@ -437,9 +479,9 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   a.rb = cfg.rb;
   a.counts = nullptr;
   const double pass_bytes = (double)n_train * ld * esz;
-  auto reduce = [&](double extra_n) {
+  auto reduce = [&](double extra_n, int center) {
     prof_begin(st);
-    reduce_partials_kernel<<<(ncols + 255) / 256, 256, 0, st>>>(partial, grid_tr, ncols, ld + 4, G);
+    reduce_partials_kernel<<<(ncols + 31) / 32, 256, 0, st>>>(partial, grid_tr, ncols, ld + 4, mu, ld, center, G);
     LAUNCHED();
     prof_end(st, 6, 0, (double)grid_tr * ncols * 4);
     if (extra_n >= 0) {  // stats pass 1 carries the local train-row count in G[ld]
@@ -452,35 +494,35 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   prof_begin(st);
   run_pass<0, E>(a, cfg, st);
   prof_end(st, 5, 0, pass_bytes);
-  reduce((double)n_train);
+  reduce((double)n_train, 0);
   stats_finalize_kernel<<<(ld + 255) / 256, 256, 0, st>>>(G, ld, 0, real, mu, mu_f, inv, dst);
   LAUNCHED();
   prof_begin(st);
   run_pass<1, E>(a, cfg, st);
   prof_end(st, 5, 0, pass_bytes);
-  reduce(-1);
+  reduce(-1, 0);
   stats_finalize_kernel<<<(ld + 255) / 256, 256, 0, st>>>(G, ld, 1, real, mu, mu_f, inv, dst);
   LAUNCHED();
   // ---- O6 step 3: K power iterations ----
-  power_kernel<<<1, ublk, 0, st>>>(G, ld, 1, d_real, real, inv, v, what, bhat, dst);
+  power_kernel<<<1, ublk, 0, st>>>(G, ld, 1, d_real, real, inv, mu, v, what, bhat, dst);
   LAUNCHED();
   for (int k = 0; k < power_iters; ++k) {
     prof_begin(st);
     run_pass<2, E>(a, cfg, st);
     prof_end(st, 5, 0, pass_bytes);
-    reduce(-1);
-    power_kernel<<<1, ublk, 0, st>>>(G, ld, 0, d_real, real, inv, v, what, bhat, dst);
+    reduce(-1, 1);
+    power_kernel<<<1, ublk, 0, st>>>(G, ld, 0, d_real, real, inv, mu, v, what, bhat, dst);
     LAUNCHED();
   }
   // ---- O6 steps 4-5: ISTA ----
-  grad_kernel<<<1, ublk, 0, st>>>(G, ld, 1, lambda, alpha, inv, w, what, bhat, dst, loss);
+  grad_kernel<<<1, ublk, 0, st>>>(G, ld, 1, lambda, alpha, inv, mu, w, what, bhat, dst, loss);
   LAUNCHED();
   for (int t = 0; t < iters; ++t) {
     prof_begin(st);
     run_pass<3, E>(a, cfg, st);
     prof_end(st, 5, 0, pass_bytes);
-    reduce(-1);
-    grad_kernel<<<1, ublk, 0, st>>>(G, ld, 0, lambda, alpha, inv, w, what, bhat, dst, loss + t);
+    reduce(-1, 1);
+    grad_kernel<<<1, ublk, 0, st>>>(G, ld, 0, lambda, alpha, inv, mu, w, what, bhat, dst, loss + t);
     LAUNCHED();
   }
   // ---- O6 step 6: eval over all local rows ----

@@ -41,7 +41,8 @@ constexpr int kOffB = 0, kOffA = kOffB + kBBytes, kOffCrow = kOffA + kSA * kRowB
 constexpr int kSmem = kOffBar + (2 * kSA + 2 * kNAcc + 2) * 8 + 1024;
 
 struct PoolParams {
-  bf16* y;  // [N, 56, 56, 64]
+  const bf16* x;  // [N, 117, 117, 16] (L2 prefetch of rows ahead of the TMA ring)
+  bf16* y;        // [N, 56, 56, 64]
   const float* scale;
   const float* shift;
   int N;
@@ -100,9 +101,29 @@ __global__ void __launch_bounds__(kThreads, 1)
     if (lane == 0) {
       mbar_arrive_expect_tx(bbar, kBBytes);
       for (int r = 0; r < 4; ++r) tma_load_2d(sB + r * 64 * 128, &tmap_w, r * 64, 0, bbar);
+      // The TMA ring holds only ~4 rows of lookahead and a row is 3.7 KB of unique input, far too little
+      // in flight to cover HBM latency: rows kPfAhead ahead are prefetched into L2 in 8-row groups.
+      constexpr int kPfAhead = 24, kPfGroup = 8;
+      constexpr uint32_t kRowIn = kHin * kS2dC * 2;  // bytes of one input row
+      auto prefetch_rows = [&](int n, int i0) {     // rows [i0, i0 + kPfGroup) of this CTA's row sequence
+        while (i0 >= kHin) {
+          i0 -= kHin;
+          n += gridDim.x;
+        }
+        if (n >= p.N) return;
+        const int i1 = min(i0 + kPfGroup, kHin);
+        prefetch_l2_range(p.x + ((size_t)n * kHin + i0) * kHin * kS2dC, (uint64_t)(i1 - i0) * kRowIn);
+        if (i1 - i0 < kPfGroup) {  // continue into this CTA's next image
+          const int n2 = n + gridDim.x;
+          if (n2 < p.N) prefetch_l2_range(p.x + (size_t)n2 * kHin * kHin * kS2dC, (uint64_t)(kPfGroup - (i1 - i0)) * kRowIn);
+        }
+      };
+      if (blockIdx.x < p.N)
+        for (int i = 0; i < kPfAhead; i += kPfGroup) prefetch_rows(blockIdx.x, i);
       uint32_t g = 0;
       for (int n = blockIdx.x; n < p.N; n += gridDim.x) {
         for (int i = 0; i < kHin; ++i, ++g) {
+          if (i % kPfGroup == 0) prefetch_rows(n, i + kPfAhead);
           const int slot = g % kSA;
           if (g >= (uint32_t)kSA) mbar_wait(&empty[slot], ((g / kSA) - 1) & 1);
           mbar_arrive_expect_tx(&full[slot], kRowBytes);
@@ -111,8 +132,8 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
     }
   } else if (warp == 1) {
-    // ======================= MMA issuer =======================
-    if (lane == 0) {
+    // ======================= MMA issuer (whole warp, one elected lane issues) =======================
+    {
       constexpr uint32_t idesc = umma_idesc_bf16(128, kCo);
       mbar_wait(bbar, 0);
       uint32_t gbase_row = 0, it = 0;
@@ -122,27 +143,32 @@ __global__ void __launch_bounds__(kThreads, 1)
           if (it >= (uint32_t)kNAcc) mbar_wait(&tempty[acc], ((it / kNAcc) - 1) & 1);
           tc_fence_after();
           const uint32_t tacc = tmem_base + acc * kCo;
-#pragma unroll 1
-          for (int r = 0; r < 4; ++r) {
+          // k-block r = filter row r = input row ho + r (manually unrolled: a rolled loop costs a YIELD and a
+          // branch-resolution stall per iteration, measured as the MMA warp's dominant cost)
+          auto kblock = [&](const uint32_t r) {
             const uint32_t row = gbase_row + ho + r;
             const uint32_t slot = row % kSA;
+            // (TMA completion on the mbarrier orders the smem writes before the async-proxy MMA reads)
             mbar_wait(&full[slot], (row / kSA) & 1);
-            tc_fence_after();
-            const uint32_t a0 = sA + slot * kRowBytes, b0 = sB + r * 64 * 128;
-#pragma unroll
-            for (int k = 0; k < 4; ++k)
-              tc_mma_bf16(tacc, umma_desc_k_sw128(a0 + k * 32), umma_desc_k_sw128(b0 + k * 32), idesc,
-                          (r | k) != 0 ? 1u : 0u);
-          }
-          tc_commit(&tfull[acc]);
+            const uint64_t da = umma_desc_k_sw128(sA + slot * kRowBytes), db = umma_desc_k_sw128(sB + r * 64 * 128);
+            // +32 bytes along K = +2 in the descriptors' address fields
+            tc_mma_bf16_warp(tacc, da, db, idesc, r != 0 ? 1u : 0u);
+            tc_mma_bf16_warp(tacc, da + 2, db + 2, idesc, 1u);
+            tc_mma_bf16_warp(tacc, da + 4, db + 4, idesc, 1u);
+            tc_mma_bf16_warp(tacc, da + 6, db + 6, idesc, 1u);
+          };
+          kblock(0);
+          kblock(1);
+          kblock(2);
+          kblock(3);
+          tc_commit_warp(&tfull[acc]);
           // input row ho is not read by any later tile of this image
-          tc_commit(&empty[(gbase_row + ho) % kSA]);
+          tc_commit_warp(&empty[(gbase_row + ho) % kSA]);
           if (ho == kHo - 1)
-            for (int r = 1; r < 4; ++r) tc_commit(&empty[(gbase_row + ho + r) % kSA]);
+            for (int r = 1; r < 4; ++r) tc_commit_warp(&empty[(gbase_row + ho + r) % kSA]);
         }
       }
     }
-    __syncwarp();
   } else {
     // ======================= epilogue: BN + ReLU + 3x3/2 max pool =======================
     const int et = threadIdx.x - kEpiWarp0 * 32;
@@ -235,6 +261,7 @@ void conv1_pool_forward(const ConvLayer& L, const bf16* x, int N, bf16* y, cudaS
   // overlapping row view {64 elements, q < 114, h, n}: element (k, q, h, n) = x[n, h, q + k / 16, k % 16]
   if (!make_rowview_tmap(&ta, x, N, kHin, kHin, kS2dC, kHo)) fail(5, "conv1_pool: row-view tensor map failed");
   PoolParams p;
+  p.x = x;
   p.y = y;
   p.scale = L.scale;
   p.shift = L.shift;

@@ -355,8 +355,8 @@ __global__ void __launch_bounds__(kThreads, 1)
       for (uint32_t j = gk > (uint32_t)kLag ? gk - kLag : 0; j < gk; ++j) mbar_arrive(&full[j % S]);
     }
   } else if (warp == 4) {
-    // ======================= MMA issuer =======================
-    if (lane == 0) {
+    // ======================= MMA issuer (whole warp, one elected lane issues) =======================
+    {
       constexpr uint32_t idesc = umma_idesc_bf16(BM, BN);
       uint32_t gk = 0, it = 0;
       for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x, ++it) {
@@ -364,24 +364,39 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (it >= 2) mbar_wait(&tempty[acc], (use - 1) & 1);
         tc_fence_after();
         const uint32_t tacc = tmem_base + acc * BN;
-        for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
+        auto kblock = [&](const int kb) {
           const int stage = gk % S;
+          // (TMA completion / the producers' fence.proxy.async + arrive order the smem writes before the MMA)
           mbar_wait(&full[stage], (gk / S) & 1);
-          tc_fence_after();
           const uint32_t a0 = sA + stage * C::kABytes, b0 = sB + stage * C::kBBytes;
+          if constexpr (AMODE == A_IM2COL_C8) {
 #pragma unroll
-          for (int k = 0; k < BK / 16; ++k)
-            tc_mma_bf16(tacc,
-                        AMODE == A_IM2COL_C8 ? umma_desc_k_none(a0 + k * 4096, 2048, 128)
-                                             : umma_desc_k_sw128(a0 + k * 32),
-                        umma_desc_k_sw128(b0 + k * 32), idesc,
-                        (kb | k) != 0 ? 1u : 0u);
-          tc_commit(&empty[stage]);
+            for (int k = 0; k < BK / 16; ++k)
+              tc_mma_bf16_warp(tacc, umma_desc_k_none(a0 + k * 4096, 2048, 128), umma_desc_k_sw128(b0 + k * 32),
+                               idesc, (kb | k) != 0 ? 1u : 0u);
+          } else {
+            const uint64_t da = umma_desc_k_sw128(a0), db = umma_desc_k_sw128(b0);
+            // +32 bytes along K = +2 in the descriptors' address fields
+            tc_mma_bf16_warp(tacc, da, db, idesc, kb != 0 ? 1u : 0u);
+            tc_mma_bf16_warp(tacc, da + 2, db + 2, idesc, 1u);
+            tc_mma_bf16_warp(tacc, da + 4, db + 4, idesc, 1u);
+            tc_mma_bf16_warp(tacc, da + 6, db + 6, idesc, 1u);
+          }
+          tc_commit_warp(&empty[stage]);
+          ++gk;
+        };
+        // unrolled by 4: a rolled loop costs a YIELD + branch-resolution stall per k-block (measured)
+        int kb = 0;
+        for (; kb + 4 <= p.nkb; kb += 4) {
+          kblock(kb);
+          kblock(kb + 1);
+          kblock(kb + 2);
+          kblock(kb + 3);
         }
-        tc_commit(&tfull[acc]);
+        for (; kb < p.nkb; ++kb) kblock(kb);
+        tc_commit_warp(&tfull[acc]);
       }
     }
-    __syncwarp();
   } else {
     // ================ epilogue (8 warps: one output row per lane, half of the columns each) ================
     const int et = threadIdx.x - kEpiWarp0 * 32;

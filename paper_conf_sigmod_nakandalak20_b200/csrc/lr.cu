@@ -143,7 +143,7 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_stream_kernel(const Pas
       for (int q = 0; q < nr; ++q) {
 #pragma unroll
         for (int c = 0; c < CH; ++c) {
-          if (!act[c]) continue;
+          if (c == CH - 1 && !act[c]) continue;
           float x[EPC];
           unpack16<E>(lds128(sbase + q * row_bytes + (uint32_t)(tid + c * nthr) * 16u), x);
 #pragma unroll
@@ -159,19 +159,30 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_stream_kernel(const Pas
       }
     } else {
       float* red = red_all + stage * (kMaxRB * 32);
-      for (int q = 0; q < nr; ++q) {
-        float sdot = 0.f;
+      // four rows at a time: four independent FMA chains and shuffle trees
+      for (int q0 = 0; q0 < nr; q0 += 4) {
+        float sd[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
-        for (int c = 0; c < CH; ++c) {
-          if (!act[c]) continue;
-          float x[EPC];
-          unpack16<E>(lds128(sbase + q * row_bytes + (uint32_t)(tid + c * nthr) * 16u), x);
+        for (int qq = 0; qq < 4; ++qq) {
+          if (q0 + qq < nr) {  // block-uniform
 #pragma unroll
-          for (int j = 0; j < EPC; ++j) sdot = fmaf(x[j], wv[c][j], sdot);
+            for (int c = 0; c < CH; ++c) {
+              if (c == CH - 1 && !act[c]) continue;  // chunks c < CH - 1 exist for every thread
+              float x[EPC];
+              unpack16<E>(lds128(sbase + (q0 + qq) * row_bytes + (uint32_t)(tid + c * nthr) * 16u), x);
+#pragma unroll
+              for (int j = 0; j < EPC; ++j) sd[qq] = fmaf(x[j], wv[c][j], sd[qq]);
+            }
+          }
         }
 #pragma unroll
-        for (int o = 16; o > 0; o >>= 1) sdot += __shfl_xor_sync(0xffffffffu, sdot, o);
-        if (lane == 0) red[q * 32 + warp] = sdot;
+        for (int o = 16; o > 0; o >>= 1)
+#pragma unroll
+          for (int qq = 0; qq < 4; ++qq) sd[qq] += __shfl_xor_sync(0xffffffffu, sd[qq], o);
+        if (lane == 0)
+#pragma unroll
+          for (int qq = 0; qq < 4; ++qq)
+            if (q0 + qq < nr) red[(q0 + qq) * 32 + warp] = sd[qq];
       }
       named_bar_sync(1, nthr);
       // every warp: lane q < nr forms z_q from the per-warp partials (fixed order) and phi_q
@@ -203,7 +214,7 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_stream_kernel(const Pas
           const float ph = __shfl_sync(0xffffffffu, phi, q);
 #pragma unroll
           for (int c = 0; c < CH; ++c) {
-            if (!act[c]) continue;
+            if (c == CH - 1 && !act[c]) continue;
             float x[EPC];
             unpack16<E>(lds128(sbase + q * row_bytes + (uint32_t)(tid + c * nthr) * 16u), x);
 #pragma unroll
@@ -314,71 +325,101 @@ __global__ void stats_finalize_kernel(const double* G, int ld, int step, const u
 
 // power iteration (O6 step 3).  init: v = 1/sqrt(d+1) on real columns and the bias.
 // update: q_j = inv_j G_j / n, q_b = G_ld / n, lambda = ||q||, v = q / lambda.
-// Both end by publishing w^ = inv * v (fp32) and b^ = v_b for the next pass.
-__global__ void power_kernel(const double* G, int ld, int init, int d_real, const uint8_t* real, const double* inv,
-                             const double* mu, double* v, float* what, float* bhat, LRState* st) {
-  __shared__ double sh[32];
-  const double n = st->n_train;
-  if (init) {
-    const double v0 = 1.0 / sqrt((double)(d_real + 1));
-    for (int j = threadIdx.x; j < ld; j += blockDim.x) v[j] = real[j] ? v0 : 0.0;
-    if (threadIdx.x == 0) st->vb = v0;
-  } else {
-    double ss = 0.0;
-    for (int j = threadIdx.x; j < ld; j += blockDim.x) {
-      const double q = inv[j] * G[j] / n;
-      ss += q * q;
-    }
-    const double qb = G[ld] / n;
-    const double lam = sqrt(block_sum(ss, sh) + qb * qb);
-    for (int j = threadIdx.x; j < ld; j += blockDim.x) v[j] = lam > 0 ? inv[j] * G[j] / n / lam : 0.0;
-    if (threadIdx.x == 0) {
-      st->vb = lam > 0 ? qb / lam : 0.0;
-      st->lambda_hat = lam;
-    }
+// Both end by publishing w^ = inv * v (fp32) and b' = v_b - sum_j w^_j mu_j for the next pass.
+__device__ void block_sum2(double& a, double& b, double* sh) {  // fixed order, result in every thread
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (int o = 16; o > 0; o >>= 1) {
+    a += __shfl_xor_sync(0xffffffffu, a, o);
+    b += __shfl_xor_sync(0xffffffffu, b, o);
   }
   __syncthreads();
-  double sm = 0.0;
-  for (int j = threadIdx.x; j < ld; j += blockDim.x) {
-    what[j] = (float)(inv[j] * v[j]);
-    sm += inv[j] * v[j] * mu[j];
+  if (lane == 0) {
+    sh[warp] = a;
+    sh[32 + warp] = b;
   }
-  sm = block_sum(sm, sh);
-  if (threadIdx.x == 0) bhat[0] = (float)(st->vb - sm);  // centred score folded into the bias
+  __syncthreads();
+  a = b = 0.0;
+  for (int w = 0; w < (int)(blockDim.x >> 5); ++w) {
+    a += sh[w];
+    b += sh[32 + w];
+  }
+}
+
+__global__ void __launch_bounds__(1024) power_kernel(const double* G, int ld, int init, int d_real,
+                                                     const uint8_t* real, const double* inv, const double* mu,
+                                                     double* v, float* what, float* bhat, LRState* st) {
+  __shared__ double sh[64];
+  const double rn = 1.0 / st->n_train;
+  double vb, scale;  // v_j = scale * (init ? real_j : inv_j G_j)
+  if (init) {
+    vb = 1.0 / sqrt((double)(d_real + 1));
+    scale = vb;
+  } else {
+    double ss = 0.0, sm = 0.0;
+    for (int j = threadIdx.x; j < ld; j += blockDim.x) {
+      const double q = inv[j] * G[j] * rn;
+      ss += q * q;
+    }
+    block_sum2(ss, sm, sh);
+    const double qb = G[ld] * rn;
+    const double lam = sqrt(ss + qb * qb);
+    const double rl = lam > 0 ? 1.0 / lam : 0.0;
+    vb = qb * rl;
+    scale = rn * rl;
+    if (threadIdx.x == 0) st->lambda_hat = lam;
+  }
+  double sm = 0.0, dummy = 0.0;
+  for (int j = threadIdx.x; j < ld; j += blockDim.x) {
+    const double vj = init ? (real[j] ? scale : 0.0) : scale * inv[j] * G[j];
+    v[j] = vj;
+    const double wj = inv[j] * vj;
+    what[j] = (float)wj;
+    sm += wj * mu[j];
+  }
+  block_sum2(sm, dummy, sh);
+  if (threadIdx.x == 0) {
+    st->vb = vb;
+    bhat[0] = (float)(vb - sm);  // centred score folded into the bias
+  }
 }
 
 // ISTA (O6 steps 4-5).  init: eta = 1 / (0.25 * 1.05 * lambda_hat + lambda (1 - alpha)), w = 0, b = 0.
 // update: g_j = inv_j G_j / n + lambda (1 - alpha) w_j; w = soft(w - eta g, eta lambda alpha);
 //         b -= eta G_ld / n; loss = G_{ld+1} / n (at the pre-update w).
-__global__ void grad_kernel(const double* G, int ld, int init, double lambda, double alpha, const double* inv,
-                            const double* mu, double* w, float* what, float* bhat, LRState* st, double* loss_out) {
+__global__ void __launch_bounds__(1024) grad_kernel(const double* G, int ld, int init, double lambda, double alpha,
+                                                    const double* inv, const double* mu, double* w, float* what,
+                                                    float* bhat, LRState* st, double* loss_out) {
+  __shared__ double sh[64];
+  double b;
   if (init) {
-    for (int j = threadIdx.x; j < ld; j += blockDim.x) w[j] = 0.0;
-    if (threadIdx.x == 0) {
-      st->eta = 1.0 / (0.25 * 1.05 * st->lambda_hat + lambda * (1.0 - alpha));
-      st->b = 0.0;
-    }
+    b = 0.0;
+    if (threadIdx.x == 0) st->eta = 1.0 / (0.25 * 1.05 * st->lambda_hat + lambda * (1.0 - alpha));
   } else {
-    const double n = st->n_train, eta = st->eta, thr = eta * lambda * alpha;
-    for (int j = threadIdx.x; j < ld; j += blockDim.x) {
-      const double g = inv[j] * G[j] / n + lambda * (1.0 - alpha) * w[j];
-      const double vv = w[j] - eta * g;
-      w[j] = (vv > 0 ? 1.0 : (vv < 0 ? -1.0 : 0.0)) * fmax(fabs(vv) - thr, 0.0);
-    }
-    if (threadIdx.x == 0) {
-      *loss_out = G[ld + 1] / n;
-      st->b -= eta * G[ld] / n;
-    }
+    const double rn = 1.0 / st->n_train;
+    b = st->b - st->eta * G[ld] * rn;
+    if (threadIdx.x == 0) *loss_out = G[ld + 1] * rn;
   }
-  __syncthreads();
-  __shared__ double sh[32];
-  double sm = 0.0;
+  const double eta = init ? 0.0 : st->eta, thr = eta * lambda * alpha, l2 = lambda * (1.0 - alpha);
+  const double rn = init ? 0.0 : 1.0 / st->n_train;
+  double sm = 0.0, dummy = 0.0;
   for (int j = threadIdx.x; j < ld; j += blockDim.x) {
-    what[j] = (float)(inv[j] * w[j]);
-    sm += inv[j] * w[j] * mu[j];
+    double wj = 0.0;
+    if (!init) {
+      const double g = inv[j] * G[j] * rn + l2 * w[j];
+      const double vv = w[j] - eta * g;
+      wj = (vv > 0 ? 1.0 : (vv < 0 ? -1.0 : 0.0)) * fmax(fabs(vv) - thr, 0.0);
+    }
+    w[j] = wj;
+    const double hj = inv[j] * wj;
+    what[j] = (float)hj;
+    sm += hj * mu[j];
   }
-  sm = block_sum(sm, sh);
-  if (threadIdx.x == 0) bhat[0] = (float)(st->b - sm);  // centred score folded into the bias
+  block_sum2(sm, dummy, sh);
+  __syncthreads();  // every thread has read st->b / st->eta
+  if (threadIdx.x == 0) {
+    st->b = b;
+    bhat[0] = (float)(b - sm);  // centred score folded into the bias
+  }
 }
 
 // ------------------------------------------------------------------------------------------

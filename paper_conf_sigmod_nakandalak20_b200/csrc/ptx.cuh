@@ -103,6 +103,20 @@ __device__ __forceinline__ void tma_store_2d(const void* tmap, int32_t c0, int32
                "r"(c0), "r"(c1)
                : "memory");
 }
+// L2 prefetch of a contiguous global range (bytes: multiple of 16), no shared memory involved
+__device__ __forceinline__ void prefetch_l2_bulk(const void* p, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
+// prefetch [p, p + bytes) in pieces of at most 32 KB (16-byte aligned start and size)
+__device__ __forceinline__ void prefetch_l2_range(const void* p, uint64_t bytes) {
+  const char* c = reinterpret_cast<const char*>(p);
+  while (bytes >= 16) {
+    const uint32_t n = bytes > 32768 ? 32768u : (uint32_t)(bytes & ~(uint64_t)15);
+    prefetch_l2_bulk(c, n);
+    c += n;
+    bytes -= n;
+  }
+}
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 // wait until every committed bulk store has finished READING its shared-memory source
 __device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
@@ -150,6 +164,26 @@ __device__ __forceinline__ void tc_mma_bf16(uint32_t tmem_d, uint64_t adesc, uin
 __device__ __forceinline__ void tc_commit(uint64_t* bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
                : "memory");
+}
+// Warp-collective forms: the whole warp runs the issue loop with warp-uniform operands (so ptxas keeps
+// descriptors in uniform registers) and one elected lane issues.  Issuing from `if (lane == 0)` instead
+// costs an elect loop with R2UR broadcasts per instruction (measured ~80 cycles per MMA issue).
+__device__ __forceinline__ void tc_mma_bf16_warp(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                                 uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p, e;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+__device__ __forceinline__ void tc_commit_warp(uint64_t* bar) {
+  asm volatile(
+      "{\n\t.reg .pred e;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(smem_u32(bar))
+      : "memory");
 }
 __device__ __forceinline__ void tc_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
 

@@ -35,11 +35,18 @@ enum AMode {
   A_GATHER_ROW = 3,
   A_IM2COL = 4,
   A_IM2COL_C8 = 5,
-  A_ROWVIEW = 6
+  A_ROWVIEW = 6,
+  A_HALO = 7
 };
 __host__ __device__ constexpr bool a_by_tma(int m) {
-  return m == A_TMA || m == A_IM2COL || m == A_IM2COL_C8 || m == A_ROWVIEW;
+  return m == A_TMA || m == A_IM2COL || m == A_IM2COL_C8 || m == A_ROWVIEW || m == A_HALO;
 }
+// A_HALO (3x3 stride 1 pad 1, one N tile): the output is computed on the padded-width grid (Wp = W + 2
+// positions per row, the last two discarded) so that output position p reads padded input position
+// p + r*Wp + s for filter tap (r, s): ONE TMA box {64 ch, Wp, hrows, 1} per channel block and tile lands
+// the zero-padded input rows (out-of-bounds fill = padding) and every tap's A operand is that buffer
+// shifted by (r*Wp + s) rows -- nine times fewer A bytes through shared memory than im2col boxes.
+__host__ __device__ constexpr int halo_half_bytes(int BN) { return BN == 64 ? 45056 : (BN == 128 ? 61440 : 0); }
 
 struct ConvParams {
   const bf16* x;
@@ -49,6 +56,7 @@ struct ConvParams {
   const float* shift;
   int H, W, Cin, Ho, Wo, Cout, R, S, stride, pad, Cg_in, Cg_out, K, nkb, M, relu;
   int n_mt, n_nt, n_tiles;
+  int Wp, hrows, hsz, mt_per_img, cblocks;  // A_HALO geometry (see above)
   // fused tap g_l (PAPER.md:369 fn 4): per-image 2x2-grid channel maxima of the (post-ReLU, >= 0)
   // output, accumulated as fp32 bit patterns with red.global.max.u32 into tapf[n][4][Cout]
   unsigned int* tapf;
@@ -65,21 +73,23 @@ constexpr int kLag = 2;        // cp.async groups in flight before a stage is pu
 // 128B-swizzled (TMA epilogue only)][scale/shift][barriers]
 // NB (TMA epilogue): staging buffers; a residual tile is prefetched NB - 1 tiles ahead into the buffer
 // the tile's output is later staged in, so NB >= 3 hides the residual's HBM latency behind a whole tile.
-template <int BN, bool TMA_EPI, int NB>
+template <int BN, bool TMA_EPI, int NB, bool HALO = false>
 struct Cfg {
-  static constexpr int kABytes = BM * BK * 2;  // 16 KB
+  static constexpr int kHaloBytes = HALO ? 2 * halo_half_bytes(BN) : 0;  // two halo buffers (A_HALO)
+  static constexpr int kABytes = HALO ? 0 : BM * BK * 2;  // 16 KB per stage (A_HALO: A lives in the halo)
   static constexpr int kBBytes = BN * BK * 2;
   static constexpr int kOutBufs = TMA_EPI ? NB : 0;
   static constexpr int kOutBytes = kOutBufs * BM * BN * 2;
   // TMA epilogue: one scale/shift buffer (a named barrier separates tiles); register epilogue: two
   static constexpr int kSbufBytes = (TMA_EPI ? 1 : 2) * 2 * BN * 4;
-  static constexpr int kFixed = kOutBytes + kSbufBytes + 1024 + 16 + 8 * 8;
+  static constexpr int kFixed = kHaloBytes + kOutBytes + kSbufBytes + 1024 + 16 + 12 * 8;
   static constexpr int kStagesFit = (227 * 1024 - kFixed) / (kABytes + kBBytes + 16);
   static constexpr int kStages = kStagesFit > 8 ? 8 : kStagesFit;
-  static constexpr int kOutOff = kStages * (kABytes + kBBytes);
+  static constexpr int kHaloOff = kStages * (kABytes + kBBytes);
+  static constexpr int kOutOff = kHaloOff + kHaloBytes;
   static constexpr int kSbufOff = kOutOff + kOutBytes;
   static constexpr int kBarOff = kSbufOff + kSbufBytes;
-  static constexpr int kBytes = kBarOff + (2 * kStages + 8) * 8 + 16 + 1024;  // + alignment slack
+  static constexpr int kBytes = kBarOff + (2 * kStages + 12) * 8 + 16 + 1024;  // + alignment slack
   static constexpr int kTmemCols = 2 * BN;
   static_assert(kStages >= 2, "shared memory too small for two k-block stages");
   static_assert(kBytes <= 227 * 1024, "shared memory over the 227 KB per-CTA limit");
@@ -125,7 +135,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__ CUtensorMap tmap_a,
                    const __grid_constant__ CUtensorMap tmap_y, const __grid_constant__ CUtensorMap tmap_r,
                    const ConvParams p) {
-  using C = Cfg<BN, TMA_EPI, NB>;
+  using C = Cfg<BN, TMA_EPI, NB, AMODE == A_HALO>;
   constexpr int S = C::kStages;
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
@@ -138,7 +148,10 @@ __global__ void __launch_bounds__(kThreads, 1)
   uint64_t* tfull = empty + S;   // [2]
   uint64_t* tempty = tfull + 2;  // [2]
   uint64_t* rbar = tempty + 2;   // [NB <= 4] residual tile landed in staging buffer b (TMA epilogue)
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rbar + 4);
+  uint64_t* hfull = rbar + 4;    // [2] halo buffer landed (A_HALO)
+  uint64_t* hempty = hfull + 2;  // [2] halo buffer consumed by the tile's MMAs (A_HALO)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(hempty + 2);
+  const uint32_t sH = base + C::kHaloOff;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
@@ -151,6 +164,10 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(&tempty[i], kEpiWarps);
     }
     for (int i = 0; i < 4; ++i) mbar_init(&rbar[i], 1);
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&hfull[i], 1);
+      mbar_init(&hempty[i], 1);
+    }
     fence_mbar_init();
     tma_prefetch(&tmap_w);
     if (a_by_tma(AMODE)) tma_prefetch(&tmap_a);
@@ -177,6 +194,29 @@ __global__ void __launch_bounds__(kThreads, 1)
             mbar_arrive_expect_tx(&full[stage], C::kABytes + C::kBBytes);
             tma_load_2d(sA + stage * C::kABytes, &tmap_a, g * p.Cg_in + kb * BK, m0, &full[stage]);
             tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
+          }
+        }
+      }
+    } else if constexpr (AMODE == A_HALO) {
+      if (threadIdx.x == 0) {
+        uint32_t gk = 0, it = 0;
+        const uint32_t box_bytes = (uint32_t)p.hrows * p.Wp * 128u;
+        for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x, ++it) {
+          int m0, nt, g;
+          decode_tile(p, tile, m0, nt, g);
+          const int mt = m0 / BM, nimg = mt / p.mt_per_img;
+          const int p0 = (mt - nimg * p.mt_per_img) * BM;
+          const int prow0 = p0 / p.Wp;  // first padded input row (input row prow0 - 1)
+          const uint32_t hb = it & 1;
+          if (it >= 2) mbar_wait(&hempty[hb], ((it >> 1) - 1) & 1);
+          mbar_arrive_expect_tx(&hfull[hb], box_bytes * p.cblocks);
+          for (int cb = 0; cb < p.cblocks; ++cb)
+            tma_load_4d(sH + hb * halo_half_bytes(BN) + cb * p.hsz, &tmap_a, cb * BK, -1, prow0 - 1, nimg, &hfull[hb]);
+          for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
+            const int stage = gk % S;
+            if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
+            mbar_arrive_expect_tx(&full[stage], C::kBBytes);
+            tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, 0, &full[stage]);
           }
         }
       }
@@ -364,12 +404,36 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (it >= 2) mbar_wait(&tempty[acc], (use - 1) & 1);
         tc_fence_after();
         const uint32_t tacc = tmem_base + acc * BN;
+        uint32_t hbase = 0;
+        int hoff = 0;
+        if constexpr (AMODE == A_HALO) {
+          int m0, nt, g;
+          decode_tile(p, tile, m0, nt, g);
+          const int mt = m0 / BM, nimg = mt / p.mt_per_img;
+          const int p0 = (mt - nimg * p.mt_per_img) * BM;
+          hoff = p0 - (p0 / p.Wp) * p.Wp;  // first output position's column in the first halo row
+          hbase = sH + (it & 1) * halo_half_bytes(BN);
+          mbar_wait(&hfull[it & 1], (it >> 1) & 1);
+        }
         auto kblock = [&](const int kb) {
           const int stage = gk % S;
           // (TMA completion / the producers' fence.proxy.async + arrive order the smem writes before the MMA)
           mbar_wait(&full[stage], (gk / S) & 1);
           const uint32_t a0 = sA + stage * C::kABytes, b0 = sB + stage * C::kBBytes;
-          if constexpr (AMODE == A_IM2COL_C8) {
+          if constexpr (AMODE == A_HALO) {
+            // k-block kb = tap * cblocks + cb, tap = r * 3 + s: A = halo rows shifted by r * Wp + s
+            const int tap = kb / p.cblocks, cb = kb - tap * p.cblocks;
+            const int r = tap / 3, sc = tap - 3 * r;
+            const int shift = hoff + r * p.Wp + sc;
+            // a row-shifted start needs no descriptor base offset: the 128B swizzle follows the absolute
+            // shared-memory address bits, exactly as the TMA wrote them (measured: base offset = shift % 8 fails)
+            const uint64_t da = umma_desc_k_sw128(hbase + cb * p.hsz + shift * 128);
+            const uint64_t db = umma_desc_k_sw128(b0);
+            tc_mma_bf16_warp(tacc, da, db, idesc, kb != 0 ? 1u : 0u);
+            tc_mma_bf16_warp(tacc, da + 2, db + 2, idesc, 1u);
+            tc_mma_bf16_warp(tacc, da + 4, db + 4, idesc, 1u);
+            tc_mma_bf16_warp(tacc, da + 6, db + 6, idesc, 1u);
+          } else if constexpr (AMODE == A_IM2COL_C8) {
 #pragma unroll
             for (int k = 0; k < BK / 16; ++k)
               tc_mma_bf16_warp(tacc, umma_desc_k_none(a0 + k * 4096, 2048, 128), umma_desc_k_sw128(b0 + k * 32),
@@ -395,6 +459,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
         for (; kb < p.nkb; ++kb) kblock(kb);
         tc_commit_warp(&tfull[acc]);
+        if constexpr (AMODE == A_HALO) tc_commit_warp(&hempty[it & 1]);  // halo free once these MMAs finish
       }
     }
   } else {
@@ -455,8 +520,15 @@ __global__ void __launch_bounds__(kThreads, 1)
         ss[i] = c < nvalid_tile ? (i < BN ? p.scale[ng0 + c] : p.shift[ng0 + c]) : 0.f;
       }
       named_bar_sync(1, kEpiThreads);
-      const int mo = m0 + row;
-      const bool rvalid = mo < p.M;
+      int mo = m0 + row;
+      bool rvalid = mo < p.M;
+      if constexpr (AMODE == A_HALO) {  // padded-width position -> output pixel (columns >= Wo discarded)
+        const int mt = m0 / BM, nimg = mt / p.mt_per_img;
+        const int pp = (mt - nimg * p.mt_per_img) * BM + row;
+        const int ho = pp / p.Wp, wo = pp - ho * p.Wp;
+        rvalid = ho < p.Ho && wo < p.Wo;
+        mo = (nimg * p.Ho + ho) * p.Wo + wo;
+      }
       const size_t off = (size_t)(rvalid ? mo : 0) * p.Cout + ng0;
       constexpr int kChunks = BN / 64;  // 32-column chunks per warp
       const int cb0 = half * kChunks;
@@ -670,6 +742,11 @@ static const bool g_rowview_enabled = [] {
   const char* e = getenv("VISTA_ROWVIEW");
   return !(e && e[0] == '0');
 }();
+// VISTA_HALO=0 disables the halo mode (3x3 convs fall back to im2col boxes; A/B measurements)
+static const bool g_halo_enabled = [] {
+  const char* e = getenv("VISTA_HALO");
+  return !(e && e[0] == '0');
+}();
 
 // N-D bf16 tiled tensor map with 128B swizzle; returns the driver status (callers may fall back)
 static CUresult encode_nd(CUtensorMap* m, const void* ptr, int rank, const cuuint64_t* dims,
@@ -747,7 +824,7 @@ static void launch_t(const ConvLayer& L, const CUtensorMap& ta, const CUtensorMa
                      const ConvParams& p, cudaStream_t st) {
   static_assert(NB >= 1 && NB <= 4, "staging buffers");
   auto kern = conv_tc_kernel<BN, AMODE, TE, NB>;
-  constexpr int smem = Cfg<BN, TE, NB>::kBytes;
+  constexpr int smem = Cfg<BN, TE, NB, AMODE == A_HALO>::kBytes;
   static bool attr_set = false;  // per instantiation
   if (!attr_set) {
     VCHECK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
@@ -771,6 +848,10 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
       if constexpr (TE) launch_t<BN, A_ROWVIEW, TE, NB>(L, ta, ty, tr, p, st);
       else fail(1, "conv: row-view mode needs the TMA epilogue");
       break;
+    case A_HALO:
+      if constexpr (!TE && BN <= 128) launch_t<BN, A_HALO, TE, NB>(L, ta, ty, tr, p, st);
+      else fail(1, "conv: halo mode needs the register epilogue and BN <= 128");
+      break;
     default: launch_t<BN, A_GATHER_GENERAL, TE, NB>(L, ta, ty, tr, p, st); break;
   }
 }
@@ -783,7 +864,7 @@ static const int g_epi_nb_env = [] {
 
 bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const bf16* res, bf16* y,
                   cudaStream_t st, unsigned int* tapf) {
-  ConvParams p;
+  ConvParams p{};
   p.x = x;
   p.y = y;
   p.res = res;
@@ -832,7 +913,34 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
       p.n_tiles = p.n_mt * p.n_nt;
     }
   }
-  if (rowview) {
+  // halo mode: 3x3 stride-1 pad-1 ungrouped, one N tile, both halo buffers fit the compile-time budget
+  bool halo = false;
+  if (!rowview && g_halo_enabled && L.R == 3 && L.S == 3 && L.stride == 1 && L.pad == 1 && L.groups == 1 &&
+      L.Cin % BK == 0 && L.BN <= 128 && L.Cout == L.BN && !res && !tapf) {
+    const int Wp = W + 2;
+    const int hrows = (Wp - 1 + BM + 1 + 2 * Wp) / Wp + 1;  // padded rows touched by 128 positions + 2 rows + 2
+    const int hsz = (hrows * Wp * 128 + 1023) & ~1023;
+    const int cblocks = L.Cin / BK;
+    const int half = L.BN == 64 ? 45056 : 61440;
+    if (Wp <= 256 && hrows <= 256 && hsz * cblocks <= half) {
+      const cuuint64_t dims[4] = {(cuuint64_t)L.Cin, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
+      const cuuint64_t strides[3] = {(cuuint64_t)L.Cin * 2, (cuuint64_t)W * L.Cin * 2, (cuuint64_t)H * W * L.Cin * 2};
+      const cuuint32_t box[4] = {(cuuint32_t)BK, (cuuint32_t)Wp, (cuuint32_t)hrows, 1};
+      if (encode_nd(&ta, x, 4, dims, strides, box) == CUDA_SUCCESS) {
+        halo = true;
+        p.Wp = Wp;
+        p.hrows = hrows;
+        p.hsz = hsz;
+        p.cblocks = cblocks;
+        p.mt_per_img = (p.Ho * Wp + BM - 1) / BM;
+        p.n_mt = N * p.mt_per_img;
+        p.n_tiles = p.n_mt * p.n_nt;
+      }
+    }
+  }
+  if (halo) {
+    amode = A_HALO;
+  } else if (rowview) {
     amode = A_ROWVIEW;
   } else if (L.R == 1 && L.S == 1 && L.stride == 1 && L.pad == 0 && L.groups == 1 && L.Cin % BK == 0) {
     amode = A_TMA;
@@ -853,7 +961,8 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   // would spill into the next group's channels
   // (long-K layers keep the register epilogue: it is hidden behind the mainloop and frees the staging
   // smem for a deeper k-block ring)
-  const bool tma_epi = rowview || ((L.groups == 1 || L.Cg_out % L.BN == 0) && L.Cout % 8 == 0 && p.nkb <= 8);
+  const bool tma_epi =
+      !halo && (rowview || ((L.groups == 1 || L.Cg_out % L.BN == 0) && L.Cout % 8 == 0 && p.nkb <= 8));
   // the fused tap needs the staged tile, non-negative outputs (ReLU) and <= 4 images per 128-row tile
   const bool fuse_tap = tapf && tma_epi && !rowview && L.relu && p.Ho * p.Wo >= 43;
   if (fuse_tap) p.tapf = tapf;

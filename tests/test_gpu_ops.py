@@ -45,6 +45,10 @@ CONV = [
     (3, 1, 1, 2048, 1000, 1, 1, 0, 1, True, False),    # FC 1000 with BN = 256 partial tile + residual
     (2, 20, 23, 16, 64, 4, 1, 0, 1, False, True),      # space-to-depth conv1 shape: TMA row view (Wo = 20)
     (1, 12, 12, 16, 64, 4, 1, 0, 1, True, True),       # same class with residual: row gather fallback
+    (2, 56, 56, 64, 64, 3, 1, 1, 1, False, True),      # ResNet res2 3x3: halo mode (Wp = 58), BN = 64
+    (3, 28, 28, 128, 128, 3, 1, 1, 1, False, True),    # ResNet res3 3x3: halo mode, BN = 128, 2 channel blocks
+    (2, 10, 10, 128, 64, 3, 1, 1, 1, False, False),    # halo mode, tiles spanning image ends, no ReLU
+    (1, 5, 130, 64, 64, 3, 1, 1, 1, False, True),      # wide rows: halo does not fit -> im2col boxes
 ]
 
 

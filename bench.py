@@ -319,17 +319,22 @@ def main():
         e2e_ms, e2e_step = 0.0, float("nan")
     d2h = sum((d + 1) * 8 for d in d_tot) + len(taps) * 8 * 80
     # ---- instrumented step: per-kernel-class device time (CUDA events on the launch stream) ----
-    v.set_profiling(True)
-    v.profile(reset=True)
-    step()
-    prof = v.profile(reset=True)
-    v.set_profiling(False)
-    conv = prof["conv_fc_tcgen05"]
     pk = peaks()
     tensor_peak = pk.get("bf16_tflops_sustained") if pk else None
     peak_src = "MEASURED_PEAKS.json bf16_tflops_sustained (kernel timed inside a long step)"
     if tensor_peak is None:
         tensor_peak, peak_src = 1400.0, "fallback B200_PROFILING.md sustained ~1.4 PFLOP/s"
+    hbm_peak = pk.get("hbm_gbs") if pk else None
+    hbm_src = "MEASURED_PEAKS.json hbm_gbs (copy, read+write bytes)"
+    if hbm_peak is None:
+        hbm_peak, hbm_src = 7700.0, "fallback B200_PROFILING.md nominal 7.7 TB/s"
+    v.set_profiling(True)
+    v.set_roofline(tensor_peak, hbm_peak)
+    v.profile(reset=True)
+    step()
+    prof = v.profile(reset=True)
+    v.set_profiling(False)
+    conv = prof["conv_fc_tcgen05"]
     achieved = conv["flops"] / (conv["ms"] / 1000.0) / 1e12 if conv["ms"] > 0 else None
     total_prof_ms = sum(p["ms"] for p in prof.values())
     roof = {
@@ -339,6 +344,14 @@ def main():
         "peak_source": peak_src, "launches_per_step": conv["launches"],
         "share_of_step": conv["ms"] / total_prof_ms if total_prof_ms else None,
         "algorithmic_flops_per_step": conv["flops"],
+        # north_star's roofline: per launch the slower of its FLOPs at tensor peak and its algorithmic bytes
+        # at HBM bandwidth, summed over the launches, divided by their measured time
+        "mixed": {
+            "conv_frac": (conv["roof_ms"] / conv["ms"]) if conv["ms"] > 0 else None,
+            "conv_roof_ms": conv["roof_ms"], "conv_ms": conv["ms"],
+            "step_frac": (sum(p["roof_ms"] for p in prof.values()) / total_prof_ms) if total_prof_ms else None,
+            "tensor_peak_tflops": tensor_peak, "hbm_peak_gbs": hbm_peak, "hbm_peak_source": hbm_src,
+        },
     }
     breakdown = {k: {"ms": round(p["ms"], 3), "launches": p["launches"],
                      "gbps": (p["bytes"] / (p["ms"] / 1000.0) / 1e9) if p["ms"] > 0 and p["bytes"] else None}

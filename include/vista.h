@@ -177,14 +177,19 @@ vista_status vista_nccl_unique_id(uint8_t* out128);
  * (CUDA events around every launch on the ctx stream; adds launch gaps, so bench.py
  * uses it only in a separate instrumented step).  classes: 0 conv/fc tensor-core GEMM,
  * 1 tap, 2 pools/cvt/lrn, 3 join, 4 concat, 5 LR passes, 6 LR small kernels.
- * ms[c], launches[c], flops[c] (algorithmic FLOPs, conv class), bytes[c] (algorithmic bytes). */
+ * ms[c], launches[c], flops[c] (algorithmic FLOPs, conv class), bytes[c] (algorithmic bytes),
+ * roof_ms[c] = sum over the class's launches of max(flops / peak FLOP/s, bytes / peak B/s): the time
+ * each launch would take at the roofline of vista_set_roofline's peaks (0 until they are set). */
 typedef struct {
   double ms[8];
   int64_t launches[8];
   double flops[8];
   double bytes[8];
+  double roof_ms[8];
 } vista_profile;
 vista_status vista_set_profiling(vista_ctx* ctx, int32_t on);
+/* Peaks for vista_profile.roof_ms: dense tensor TFLOP/s and HBM GB/s (e.g. MEASURED_PEAKS.json). */
+vista_status vista_set_roofline(vista_ctx* ctx, double tflops, double gbps);
 /* Number of kernels this process has launched through libvista.so so far (all ctxs). */
 int64_t vista_kernel_launches(void);
 vista_status vista_get_profile(vista_ctx* ctx, vista_profile* out, int32_t reset);

@@ -757,6 +757,14 @@ static CUresult encode_nd(CUtensorMap* m, const void* ptr, int rank, const cuuin
                       CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
 }
 
+// [rows, cols] bf16 matrix, box {64, 128}, 128B swizzle (A operands / staged outputs of 128-row tiles)
+bool make_plain_tmap(CUtensorMap* m, const void* ptr, int cols, int rows) {
+  const cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+  const cuuint64_t strides[1] = {(cuuint64_t)cols * 2};
+  const cuuint32_t box[2] = {(cuuint32_t)BK, (cuuint32_t)BM};
+  return encode_nd(m, ptr, 2, dims, strides, box) == CUDA_SUCCESS;
+}
+
 // overlapping 4-D row view of an NHWC input with C * S == 64 (A_ROWVIEW): element (k, q, h, n) =
 // x[n, h, q + k / C, k % C] for q < Wo; box {64, 128, 1, 1}, 128B-swizzled (q >= Wo reads zeros)
 bool make_rowview_tmap(CUtensorMap* m, const void* x, int N, int H, int W, int C, int Wo) {

@@ -1,0 +1,377 @@
+// res_chain.cu — two chained 1x1 convolutions of consecutive ResNet bottleneck units in ONE kernel:
+//   out    = ReLU(BN_c(b * Wc) + x)        (unit u's closing 1x1 conv + residual, Cout = 4 * MID)
+//   a_next = ReLU(BN_a(out * Wa))          (unit u+1's opening 1x1 conv, Cout = MID)
+// SURVEY.md §8a S1 (partial inference f^ as a chain of TensorOps, Def 3.7).
+// Unfused, the a-conv re-reads `out` (4 * MID channels per pixel) from HBM right after the c-conv wrote
+// it; here every 128-pixel x 128-channel chunk of `out` is staged in shared memory for its TMA store
+// anyway (128B-swizzled, K-major: exactly the A-operand layout of tcgen05.mma), so the a-conv's MMAs read
+// it from there and `out` is read zero times instead of once (-29 % HBM bytes for the pair at MID = 64).
+//
+// Per 128-pixel tile: c-chunks j = 0 .. 4*MID/128 - 1 (128 output channels each, two TMEM accumulators
+// alternate) and the a-accumulator (MID columns) that sums over the chunks.  MMA issue order
+// c(0), c(1), a(0), c(2), a(1), ... lets c(j+1) run while the epilogue finishes chunk j.
+// Both GEMMs use the same instruction shapes and k order as conv_tc.cu's unfused launches (N = 128 for
+// c, N = MID for a, K-steps of 16 in ascending k), and the same epilogue arithmetic, so the result is
+// bit-identical to conv_forward(c) followed by conv_forward(a) (tested).
+#include <cstring>
+
+#include "internal.h"
+#include "ptx.cuh"
+
+namespace vista {
+
+namespace {
+
+constexpr int BMr = 128, BKr = 64;
+constexpr int kEpiW0 = 2, kEpiWn = 8, kEpiT = kEpiWn * 32, kThr = (kEpiW0 + kEpiWn) * 32;
+
+template <int MID>
+struct RC {
+  static constexpr int NCH = 4 * MID / 128;       // c chunks of 128 channels
+  static constexpr int KBC = MID / BKr;           // k-blocks of the c GEMM
+  static constexpr int NB = MID == 64 ? 3 : 2;    // out/residual staging buffers
+  static constexpr int WS = MID == 64 ? 4 : 3;    // weight ring stages (16 KB)
+  static constexpr int kB = KBC * BMr * 128;      // b tile bytes
+  static constexpr int kO = BMr * 128 * 2;        // one out chunk: two 64-channel sub-tiles
+  static constexpr int kA = BMr * MID * 2;        // a_next tile
+  static constexpr int offB = 0, offO = offB + 2 * kB, offA = offO + NB * kO, offW = offA + kA,
+                       offS = offW + WS * 16384, offBar = offS + (5 * MID) * 2 * 4;
+  static constexpr int nBar = 2 + 2 + NB * 3 + 2 * WS + 2 + 1 + 1 + 2;
+  static constexpr int kSmem = offBar + nBar * 8 + 16 + 1024;
+  static_assert(kSmem <= 227 * 1024, "res_chain smem");
+};
+
+struct RCParams {
+  const float* sc_c;
+  const float* sh_c;
+  const float* sc_a;
+  const float* sh_a;
+  int M, n_mt;
+};
+
+template <int MID>
+__global__ void __launch_bounds__(kThr, 1)
+    res_chain_kernel(const __grid_constant__ CUtensorMap tm_b, const __grid_constant__ CUtensorMap tm_res,
+                     const __grid_constant__ CUtensorMap tm_out, const __grid_constant__ CUtensorMap tm_a,
+                     const __grid_constant__ CUtensorMap tm_wc, const __grid_constant__ CUtensorMap tm_wa,
+                     const RCParams p) {
+  using C = RC<MID>;
+  constexpr int NCH = C::NCH, KBC = C::KBC, NB = C::NB, WS = C::WS;
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  const uint32_t base = (raw + 1023u) & ~1023u;
+  uint8_t* gbase = smem_raw + (base - raw);
+  const uint32_t sB = base + C::offB, sO = base + C::offO, sAo = base + C::offA, sW = base + C::offW;
+  float* sc_c = reinterpret_cast<float*>(gbase + C::offS);  // [4 MID] scale, [4 MID] shift, [MID], [MID]
+  float* sh_c = sc_c + 4 * MID;
+  float* sc_a = sh_c + 4 * MID;
+  float* sh_a = sc_a + MID;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(gbase + C::offBar);
+  uint64_t* bfull = bar;            // [2] b tile landed
+  uint64_t* bempty = bfull + 2;     // [2] b tile consumed by the c MMAs
+  uint64_t* rfull = bempty + 2;     // [NB] residual chunk landed in staging buffer
+  uint64_t* oready = rfull + NB;    // [NB] out chunk staged (a-MMA may read it)
+  uint64_t* ofree = oready + NB;    // [NB] staging buffer free: store has read it AND a-MMA done (count 2)
+  uint64_t* wfull = ofree + NB;     // [WS]
+  uint64_t* wempty = wfull + WS;    // [WS]
+  uint64_t* tfull_c = wempty + WS;  // [2]
+  uint64_t* tfull_a = tfull_c + 2;  // [1]
+  uint64_t* tempty_a = tfull_a + 1; // [1]
+  uint64_t* tempty_c = tempty_a + 1;  // [2]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty_c + 2);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&bfull[i], 1);
+      mbar_init(&bempty[i], 1);
+      mbar_init(&tfull_c[i], 1);
+      mbar_init(&tempty_c[i], kEpiWn);
+    }
+    for (int i = 0; i < NB; ++i) {
+      mbar_init(&rfull[i], 1);
+      mbar_init(&oready[i], 1);
+      mbar_init(&ofree[i], 2);
+    }
+    for (int i = 0; i < WS; ++i) {
+      mbar_init(&wfull[i], 1);
+      mbar_init(&wempty[i], 1);
+    }
+    mbar_init(tfull_a, 1);
+    mbar_init(tempty_a, kEpiWn);
+    fence_mbar_init();
+  }
+  for (int i = threadIdx.x; i < 5 * MID * 2; i += blockDim.x) {
+    float v;
+    if (i < 4 * MID) v = p.sc_c[i];
+    else if (i < 8 * MID) v = p.sh_c[i - 4 * MID];
+    else if (i < 9 * MID) v = p.sc_a[i - 8 * MID];
+    else v = p.sh_a[i - 9 * MID];
+    sc_c[i] = v;
+  }
+  if (warp == 1) tmem_alloc(tmem_slot, 512);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;  // acc_c[0] cols 0..127, acc_c[1] 128..255, acc_a 256..256+MID
+
+  if (warp == 0) {
+    // ================= producer =================
+    if (lane == 0) {
+      uint32_t gw = 0, q = 0, it = 0;
+      auto push_w = [&](const CUtensorMap* m, int c0, int c1, uint32_t bytes) {
+        const uint32_t st = gw % WS;
+        if (gw >= (uint32_t)WS) mbar_wait(&wempty[st], ((gw / WS) - 1) & 1);
+        mbar_arrive_expect_tx(&wfull[st], bytes);
+        tma_load_2d(sW + st * 16384, m, c0, c1, &wfull[st]);
+        ++gw;
+      };
+      auto push_res = [&](int m0, int j) {
+        const uint32_t qq = q + j, ob = qq % NB;
+        if (qq >= (uint32_t)NB) mbar_wait(&ofree[ob], ((qq / NB) - 1) & 1);
+        mbar_arrive_expect_tx(&rfull[ob], C::kO);
+        tma_load_2d(sO + ob * C::kO, &tm_res, j * 128, m0, &rfull[ob]);
+        tma_load_2d(sO + ob * C::kO + BMr * 128, &tm_res, j * 128 + 64, m0, &rfull[ob]);
+      };
+      auto push_c = [&](int j) {
+        for (int kb = 0; kb < KBC; ++kb) push_w(&tm_wc, kb * BKr, j * 128, 128 * 128);
+      };
+      auto push_a = [&](int j) {
+        for (int h = 0; h < 2; ++h) push_w(&tm_wa, j * 128 + h * 64, 0, MID * 128);
+      };
+      for (int tile = blockIdx.x; tile < p.n_mt; tile += gridDim.x, ++it, q += NCH) {
+        const int m0 = tile * BMr;
+        const uint32_t bb = it & 1;
+        if (it >= 2) mbar_wait(&bempty[bb], ((it >> 1) - 1) & 1);
+        mbar_arrive_expect_tx(&bfull[bb], C::kB);
+        for (int kb = 0; kb < KBC; ++kb) tma_load_2d(sB + bb * C::kB + kb * BMr * 128, &tm_b, kb * BKr, m0, &bfull[bb]);
+        // weights in the order the MMA warp consumes them: c(0), then per j: c(j+1), a(j); each residual
+        // chunk right after its c weights (its buffer frees up only once the a-MMA two chunks back is done)
+        push_c(0);
+        push_res(m0, 0);
+        for (int j = 0; j < NCH; ++j) {
+          if (j + 1 < NCH) {
+            push_c(j + 1);
+            push_res(m0, j + 1);
+          }
+          push_a(j);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ================= MMA issuer (whole warp, elected lane issues) =================
+    constexpr uint32_t idesc_c = umma_idesc_bf16(BMr, 128);
+    constexpr uint32_t idesc_a = umma_idesc_bf16(BMr, MID);
+    uint32_t gw = 0, it = 0;
+    auto wait_w = [&]() -> uint32_t {
+      const uint32_t st = gw % WS;
+      mbar_wait(&wfull[st], (gw / WS) & 1);
+      return st;
+    };
+    for (int tile = blockIdx.x; tile < p.n_mt; tile += gridDim.x, ++it) {
+      const uint32_t bb = it & 1, qbase = it * NCH;
+      mbar_wait(&bfull[bb], (it >> 1) & 1);
+      auto issue_c = [&](const int j) {
+        const uint32_t qq = qbase + j, acc = qq & 1;
+        if (qq >= 2) mbar_wait(&tempty_c[acc], ((qq >> 1) - 1) & 1);
+        tc_fence_after();
+        const uint32_t tacc = tmem + acc * 128;
+#pragma unroll
+        for (int kb = 0; kb < KBC; ++kb) {
+          const uint32_t st = wait_w();
+          const uint64_t da = umma_desc_k_sw128(sB + bb * C::kB + kb * BMr * 128), db = umma_desc_k_sw128(sW + st * 16384);
+          tc_mma_bf16_warp(tacc, da, db, idesc_c, kb != 0 ? 1u : 0u);
+          tc_mma_bf16_warp(tacc, da + 2, db + 2, idesc_c, 1u);
+          tc_mma_bf16_warp(tacc, da + 4, db + 4, idesc_c, 1u);
+          tc_mma_bf16_warp(tacc, da + 6, db + 6, idesc_c, 1u);
+          tc_commit_warp(&wempty[st]);
+          ++gw;
+        }
+        tc_commit_warp(&tfull_c[acc]);
+        if (j == NCH - 1) tc_commit_warp(&bempty[bb]);
+      };
+      auto issue_a = [&](const int j) {
+        const uint32_t qq = qbase + j, ob = qq % NB;
+        if (j == 0 && it >= 1) mbar_wait(tempty_a, (it - 1) & 1);
+        mbar_wait(&oready[ob], (qq / NB) & 1);
+        tc_fence_after();
+        const uint32_t tacc = tmem + 256;
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const uint32_t st = wait_w();
+          const uint64_t da = umma_desc_k_sw128(sO + ob * C::kO + h * BMr * 128), db = umma_desc_k_sw128(sW + st * 16384);
+          tc_mma_bf16_warp(tacc, da, db, idesc_a, (j | h) != 0 ? 1u : 0u);
+          tc_mma_bf16_warp(tacc, da + 2, db + 2, idesc_a, 1u);
+          tc_mma_bf16_warp(tacc, da + 4, db + 4, idesc_a, 1u);
+          tc_mma_bf16_warp(tacc, da + 6, db + 6, idesc_a, 1u);
+          tc_commit_warp(&wempty[st]);
+          ++gw;
+        }
+        tc_commit_warp(&ofree[ob]);
+        if (j == NCH - 1) tc_commit_warp(tfull_a);
+      };
+      issue_c(0);
+#pragma unroll
+      for (int j = 0; j < NCH; ++j) {
+        if (j + 1 < NCH) issue_c(j + 1);
+        issue_a(j);
+      }
+    }
+  } else {
+    // ================= epilogue (8 warps) =================
+    const int et = threadIdx.x - kEpiW0 * 32;
+    const int qd = warp & 3, half = (warp - kEpiW0) >> 2;
+    const int row = qd * 32 + lane;
+    uint32_t it = 0;
+    for (int tile = blockIdx.x; tile < p.n_mt; tile += gridDim.x, ++it) {
+      const int m0 = tile * BMr;
+#pragma unroll 1
+      for (int j = 0; j < NCH; ++j) {
+        const uint32_t qq = it * NCH + j, acc = qq & 1, ob = qq % NB;
+        const uint32_t so = sO + ob * C::kO;
+        mbar_wait(&rfull[ob], (qq / NB) & 1);
+        mbar_wait(&tfull_c[acc], (qq >> 1) & 1);
+        tc_fence_after();
+#pragma unroll
+        for (int cc = 0; cc < 2; ++cc) {  // two 32-column pieces of this warp's 64-column half
+          const int cb = half * 2 + cc;    // 32-column block 0..3 of the 128-column chunk
+          uint32_t v[32];
+          tmem_ld_32x32b_x32(tmem + acc * 128 + cb * 32 + ((uint32_t)(qd * 32) << 16), v);
+          tc_wait_ld();
+          const uint32_t sub = so + (cb >> 1) * BMr * 128 + row * 128;
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const int ch = j * 128 + cb * 32 + k * 8;
+            const uint32_t addr = sub + (((uint32_t)((cb & 1) * 4 + k) ^ (uint32_t)(row & 7)) << 4);
+            const uint4 r = lds128(addr);
+            const uint32_t rr[4] = {r.x, r.y, r.z, r.w};
+            float f[8];
+#pragma unroll
+            for (int e = 0; e < 8; ++e) f[e] = fmaf(__uint_as_float(v[k * 8 + e]), sc_c[ch + e], sh_c[ch + e]);
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              const float2 a = unpack_bf16x2(rr[e]);
+              f[2 * e] = fmaxf(f[2 * e] + a.x, 0.f);
+              f[2 * e + 1] = fmaxf(f[2 * e + 1] + a.y, 0.f);
+            }
+            uint4 o;
+            o.x = pack_bf16x2(f[0], f[1]);
+            o.y = pack_bf16x2(f[2], f[3]);
+            o.z = pack_bf16x2(f[4], f[5]);
+            o.w = pack_bf16x2(f[6], f[7]);
+            sts128(addr, o);
+          }
+        }
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&tempty_c[acc]);
+        fence_proxy_async_smem();
+        named_bar_sync(1, kEpiT);
+        if (et == 0) {
+          // the previous chunk's store must have read its buffer before that buffer is refilled
+          if (qq >= 1) {
+            if (j == 0) bulk_wait_read<1>();  // the previous tile's a_next store was committed after it
+            else bulk_wait_read<0>();
+            mbar_arrive(&ofree[(qq - 1) % NB]);
+          }
+          mbar_arrive(&oready[ob]);  // staged chunk may feed the a-MMA
+          tma_store_2d(&tm_out, j * 128, m0, so);
+          tma_store_2d(&tm_out, j * 128 + 64, m0, so + BMr * 128);
+          bulk_commit();
+        }
+      }
+      // ---- a_next = ReLU(BN_a(acc_a)) ----
+      mbar_wait(tfull_a, it & 1);
+      tc_fence_after();
+      if (et == 0) bulk_wait_read<NCH>();  // the previous tile's a_next store has read the staging tile
+      named_bar_sync(1, kEpiT);
+#pragma unroll
+      for (int cc = 0; cc < MID / 64; ++cc) {
+        const int cb = half * (MID / 64) + cc;  // 32-column block of the MID-wide accumulator
+        uint32_t v[32];
+        tmem_ld_32x32b_x32(tmem + 256 + cb * 32 + ((uint32_t)(qd * 32) << 16), v);
+        tc_wait_ld();
+        const uint32_t sub = sAo + (cb >> 1) * BMr * 128 + row * 128;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const int ch = cb * 32 + k * 8;
+          float f[8];
+#pragma unroll
+          for (int e = 0; e < 8; ++e)
+            f[e] = fmaxf(fmaf(__uint_as_float(v[k * 8 + e]), sc_a[ch + e], sh_a[ch + e]), 0.f);
+          uint4 o;
+          o.x = pack_bf16x2(f[0], f[1]);
+          o.y = pack_bf16x2(f[2], f[3]);
+          o.z = pack_bf16x2(f[4], f[5]);
+          o.w = pack_bf16x2(f[6], f[7]);
+          sts128(sub + (((uint32_t)((cb & 1) * 4 + k) ^ (uint32_t)(row & 7)) << 4), o);
+        }
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(tempty_a);
+      fence_proxy_async_smem();
+      named_bar_sync(1, kEpiT);
+      if (et == 0) {
+        for (int s = 0; s < MID / 64; ++s) tma_store_2d(&tm_a, s * 64, m0, sAo + s * BMr * 128);
+        bulk_commit();
+      }
+    }
+    if (et == 0) bulk_wait0();
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) tmem_dealloc(tmem, 512);
+}
+
+}  // namespace
+
+bool res_chain_supported(const ConvLayer& Lc, const ConvLayer& La) {
+  const int mid = Lc.Cin;
+  return (mid == 64 || mid == 128) && Lc.R == 1 && Lc.S == 1 && Lc.stride == 1 && Lc.pad == 0 && Lc.groups == 1 &&
+         Lc.Cout == 4 * mid && Lc.BN == 128 && Lc.relu && La.R == 1 && La.S == 1 && La.stride == 1 && La.pad == 0 &&
+         La.groups == 1 && La.Cin == 4 * mid && La.Cout == mid && La.BN == mid && La.relu;
+}
+
+template <int MID>
+static void launch_chain(const ConvLayer& Lc, const ConvLayer& La, const bf16* b, const bf16* res, bf16* out,
+                         bf16* a_next, int M, cudaStream_t st) {
+  CUtensorMap tb, tr, to, ta;
+  if (!make_plain_tmap(&tb, b, MID, M) || !make_plain_tmap(&tr, res, 4 * MID, M) ||
+      !make_plain_tmap(&to, out, 4 * MID, M) || !make_plain_tmap(&ta, a_next, MID, M))
+    fail(5, "res_chain: tensor map encoding failed");
+  RCParams p;
+  p.sc_c = Lc.scale;
+  p.sh_c = Lc.shift;
+  p.sc_a = La.scale;
+  p.sh_a = La.shift;
+  p.M = M;
+  p.n_mt = (M + BMr - 1) / BMr;
+  static bool attr = false;
+  if (!attr) {
+    VCHECK(cudaFuncSetAttribute(res_chain_kernel<MID>, cudaFuncAttributeMaxDynamicSharedMemorySize, RC<MID>::kSmem));
+    attr = true;
+  }
+  const int grid = p.n_mt < num_sms() ? p.n_mt : num_sms();
+  res_chain_kernel<MID><<<grid, kThr, RC<MID>::kSmem, st>>>(tb, tr, to, ta, Lc.tmap_w, La.tmap_w, p);
+  LAUNCHED();
+}
+
+void res_chain_forward(const ConvLayer& Lc, const ConvLayer& La, const bf16* b, const bf16* res, bf16* out,
+                       bf16* a_next, int N, int H, int W, cudaStream_t st) {
+  const int64_t M64 = (int64_t)N * H * W;
+  if (M64 <= 0) return;
+  if (M64 > INT32_MAX - BMr) fail(1, "res_chain: M too large");
+  const int M = (int)M64;
+  const int mid = Lc.Cin;
+  prof_begin(st);
+  if (mid == 64) launch_chain<64>(Lc, La, b, res, out, a_next, M, st);
+  else launch_chain<128>(Lc, La, b, res, out, a_next, M, st);
+  const double flops = 2.0 * M64 * (double)(4 * mid) * mid * 2;  // both GEMMs
+  const double bytes = 2.0 * M64 * ((double)mid + 4 * mid + 4 * mid + mid) + 2.0 * 8 * mid * mid;
+  char label[96] = {0};
+  if (prof_labels()) snprintf(label, sizeof(label), "res_chain c+a MID%d HxW%dx%d", mid, H, W);
+  prof_end(st, 0, flops, bytes, prof_labels() ? label : nullptr);
+}
+
+}  // namespace vista

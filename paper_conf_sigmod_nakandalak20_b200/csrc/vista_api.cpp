@@ -54,6 +54,7 @@ struct Profiler {
   std::vector<cudaEvent_t> pool;
   cudaEvent_t pending = nullptr;
   vista_profile acc{};
+  double peak_flops = 0, peak_bytes = 0;  // per second (vista_set_roofline)
   cudaEvent_t get() {
     if (!pool.empty()) {
       cudaEvent_t e = pool.back();
@@ -73,6 +74,8 @@ struct Profiler {
       acc.launches[r.cls] += 1;
       acc.flops[r.cls] += r.flops;
       acc.bytes[r.cls] += r.bytes;
+      if (peak_flops > 0 && peak_bytes > 0)
+        acc.roof_ms[r.cls] += 1e3 * std::max(r.flops / peak_flops, r.bytes / peak_bytes);
       if (log) fprintf(log, "%d\t%.6f\t%.6g\t%.6g\t%s\n", r.cls, ms, r.flops, r.bytes, r.label.c_str());
       pool.push_back(r.a);
       pool.push_back(r.b);
@@ -232,6 +235,8 @@ struct vista_ctx {
   bool fuse_tap = false;
   // ResNet conv1 + pool1 in one kernel (conv1_pool.cu, bit-identical); VISTA_FUSE_STEM=0 disables
   bool fuse_stem = true;
+  // closing 1x1 conv + next unit's opening 1x1 conv (res_chain.cu, bit-identical); VISTA_FUSE_CHAIN=0 disables
+  bool fuse_chain = true;
   std::vector<void*> feat;  // per block: device pointer of F_t (features) of a tapped layer
   std::string last_error;
   ~vista_ctx() {
@@ -535,6 +540,18 @@ bool run_ops(vista_ctx* c, int t, const void* in_ptr, void* out_ptr, int nb, voi
         ++oi;
         continue;
       }
+      // closing 1x1 conv of a bottleneck unit + the next unit's opening 1x1 conv in one kernel
+      if (op.kind == OP_CONV && op.res >= 0 && c->fuse_chain && oi + 1 < S.ops.size()) {
+        const OpDesc& o2 = S.ops[oi + 1];
+        if (o2.kind == OP_CONV && o2.in == op.out && o2.res < 0 && o2.out != BUF_OUT && op.out != o2.out &&
+            res_chain_supported(c->convs[op.layer], c->convs[o2.layer]) && o2.H == op.Ho && o2.W == op.Wo &&
+            op.Ho == op.H && op.Wo == op.W) {
+          res_chain_forward(c->convs[op.layer], c->convs[o2.layer], in, reinterpret_cast<const bf16*>(slot[op.res]),
+                            out, reinterpret_cast<bf16*>(slot[o2.out]), nb, op.H, op.W, c->stream);
+          ++oi;
+          continue;
+        }
+      }
       switch (op.kind) {
         case OP_INGEST:
           launch_ingest(reinterpret_cast<const uint8_t*>(slot[op.in]), nb, out, c->stream);
@@ -745,6 +762,7 @@ VISTA_API vista_status vista_plan(vista_cnn cnn, const int32_t* layers, int32_t 
     c->prof.reset(new Profiler());
     if (const char* e = getenv("VISTA_FUSED_TAP")) c->fuse_tap = e[0] != '0';
     if (const char* e = getenv("VISTA_FUSE_STEM")) c->fuse_stem = e[0] != '0';
+    if (const char* e = getenv("VISTA_FUSE_CHAIN")) c->fuse_chain = e[0] != '0';
     VCHECK(cudaStreamSynchronize(c->stream));
   });
   if (st != VISTA_OK) {
@@ -984,6 +1002,13 @@ VISTA_API int64_t vista_kernel_launches(void) { return (int64_t)launches_total()
 VISTA_API vista_status vista_set_profiling(vista_ctx* c, int32_t on) {
   if (!c) return VISTA_ERR_INVALID_ARG;
   c->profiling = on != 0;
+  return VISTA_OK;
+}
+
+VISTA_API vista_status vista_set_roofline(vista_ctx* c, double tflops, double gbps) {
+  if (!c || !c->prof || tflops <= 0 || gbps <= 0) return VISTA_ERR_INVALID_ARG;
+  c->prof->peak_flops = tflops * 1e12;
+  c->prof->peak_bytes = gbps * 1e9;
   return VISTA_OK;
 }
 

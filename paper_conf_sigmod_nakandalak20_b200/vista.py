@@ -59,7 +59,8 @@ class Metrics(ctypes.Structure):
 
 
 class Profile(ctypes.Structure):
-    _fields_ = [("ms", _f64 * 8), ("launches", _i64 * 8), ("flops", _f64 * 8), ("bytes", _f64 * 8)]
+    _fields_ = [("ms", _f64 * 8), ("launches", _i64 * 8), ("flops", _f64 * 8), ("bytes", _f64 * 8),
+                ("roof_ms", _f64 * 8)]
 
 
 PROFILE_CLASSES = ["conv_fc_tcgen05", "tap", "pool_cvt_lrn", "join", "concat", "lr_pass", "lr_small"]
@@ -88,6 +89,7 @@ def lib():
         L.vista_nccl_unique_id.argtypes = [_vp]
         L.vista_set_profiling.argtypes = [_vp, _i32]
         L.vista_get_profile.argtypes = [_vp, ctypes.POINTER(Profile), _i32]
+        L.vista_set_roofline.argtypes = [_vp, _f64, _f64]
         L.vista_conv2d.argtypes = [_vp, _i32, _i32, _i32, _i32, _vp, _i32, _i32, _i32, _i32, _i32, _i32, _vp, _vp,
                                    _vp, _i32, _vp, _vp]
         L.vista_conv2d_tap.argtypes = [_vp, _i32, _i32, _i32, _i32, _vp, _i32, _i32, _i32, _i32, _i32, _vp, _vp,
@@ -301,8 +303,12 @@ class Vista:
     def profile(self, reset=True):
         p = Profile()
         _check(lib().vista_get_profile(self.ctx, ctypes.byref(p), 1 if reset else 0), self.ctx)
-        return {name: dict(ms=p.ms[i], launches=p.launches[i], flops=p.flops[i], bytes=p.bytes[i])
+        return {name: dict(ms=p.ms[i], launches=p.launches[i], flops=p.flops[i], bytes=p.bytes[i],
+                           roof_ms=p.roof_ms[i])
                 for i, name in enumerate(PROFILE_CLASSES)}
+
+    def set_roofline(self, tflops, gbps):
+        _check(lib().vista_set_roofline(self.ctx, float(tflops), float(gbps)), self.ctx)
 
     def close(self):
         if getattr(self, "ctx", None):

@@ -226,3 +226,17 @@ def test_resnet_stem_fused_bit_identical(monkeypatch):
         v.close()
     for a, b in zip(out["1"], out["0"]):
         assert torch.equal(a, b)
+
+
+def test_resnet_chain_fused_bit_identical(monkeypatch):
+    # the closing 1x1 conv of a unit and the next unit's opening 1x1 conv run as one kernel (res_chain.cu,
+    # MID = 64 / 128) by default; VISTA_FUSE_CHAIN=0 runs them as two conv_tc launches: same bits
+    tab = gen.make_tables(37, 8)  # M = 37 * 3136 pixels: partial last 128-row tile
+    out = {}
+    for fuse in ("1", "0"):
+        monkeypatch.setenv("VISTA_FUSE_CHAIN", fuse)
+        v = run_gpu(2, [0, 4], tab, 8, iters=1, micro_batch=37)
+        out[fuse] = [v.features(k)["mm"].view(torch.int16).cpu().clone() for k in range(2)]
+        v.close()
+    for a, b in zip(out["1"], out["0"]):
+        assert torch.equal(a, b)

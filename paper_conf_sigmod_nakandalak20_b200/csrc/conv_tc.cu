@@ -73,24 +73,39 @@ constexpr int kLag = 2;        // cp.async groups in flight before a stage is pu
 // 128B-swizzled (TMA epilogue only)][scale/shift][barriers]
 // NB (TMA epilogue): staging buffers; a residual tile is prefetched NB - 1 tiles ahead into the buffer
 // the tile's output is later staged in, so NB >= 3 hides the residual's HBM latency behind a whole tile.
-template <int BN, bool TMA_EPI, int NB, bool HALO = false>
+// RKB > 0 (resident weights): the CTA's whole B slice (RKB >= nkb k-blocks of BN x 64) is loaded once and
+// stays in shared memory; the launch makes the grid a multiple of the N-tile count so that every tile a CTA
+// visits (tile += gridDim.x) has the same N tile.  Only A streams through the ring (A_HALO: no ring at
+// all, and three halo buffers).  Measured motivation: the per-SM L2 -> smem ingest is bounded by the
+// bytes in flight / L2 latency, and re-loading the weights per tile doubled (1x1) or tripled (halo 3x3,
+// Cout = 64) the bytes each tile needs.
+template <int BN, bool TMA_EPI, int NB, bool HALO = false, int RKB = 0>
 struct Cfg {
-  static constexpr int kHaloBytes = HALO ? 2 * halo_half_bytes(BN) : 0;  // two halo buffers (A_HALO)
+  static constexpr int kHB = HALO ? (RKB ? 3 : 2) : 0;  // halo buffers (A_HALO)
+  static constexpr int kHaloBytes = kHB * halo_half_bytes(BN);
   static constexpr int kABytes = HALO ? 0 : BM * BK * 2;  // 16 KB per stage (A_HALO: A lives in the halo)
   static constexpr int kBBytes = BN * BK * 2;
+  static constexpr int kResBytes = RKB * kBBytes;          // resident weights
+  static constexpr int kStageBytes = kABytes + (RKB ? 0 : kBBytes);
   static constexpr int kOutBufs = TMA_EPI ? NB : 0;
   static constexpr int kOutBytes = kOutBufs * BM * BN * 2;
   // TMA epilogue: one scale/shift buffer (a named barrier separates tiles); register epilogue: two
   static constexpr int kSbufBytes = (TMA_EPI ? 1 : 2) * 2 * BN * 4;
-  static constexpr int kFixed = kHaloBytes + kOutBytes + kSbufBytes + 1024 + 16 + 12 * 8;
-  static constexpr int kStagesFit = (227 * 1024 - kFixed) / (kABytes + kBBytes + 16);
+  static constexpr int kNBar = 20;  // tfull/tempty[4], rbar[4], hfull/hempty[3], wres[1], slack
+  static constexpr int kFixed = kHaloBytes + kResBytes + kOutBytes + kSbufBytes + 1024 + 16 + kNBar * 8;
+  static constexpr int kStagesFit = kStageBytes ? (227 * 1024 - kFixed) / (kStageBytes + 16) : 2;
   static constexpr int kStages = kStagesFit > 8 ? 8 : kStagesFit;
-  static constexpr int kHaloOff = kStages * (kABytes + kBBytes);
+  static constexpr int kResOff = kStages * kStageBytes;
+  static constexpr int kHaloOff = kResOff + kResBytes;
   static constexpr int kOutOff = kHaloOff + kHaloBytes;
   static constexpr int kSbufOff = kOutOff + kOutBytes;
   static constexpr int kBarOff = kSbufOff + kSbufBytes;
-  static constexpr int kBytes = kBarOff + (2 * kStages + 12) * 8 + 16 + 1024;  // + alignment slack
-  static constexpr int kTmemCols = 2 * BN;
+  static constexpr int kBytes = kBarOff + (2 * kStages + kNBar) * 8 + 16 + 1024;  // + alignment slack
+  // register epilogue with BN <= 128: four TMEM accumulators, and the two epilogue warp groups take
+  // alternate tiles (each group drains all BN columns of its tiles), so two tiles' epilogues overlap
+  static constexpr bool kSplit = !TMA_EPI && BN <= 128;
+  static constexpr int kAcc = kSplit ? 4 : 2;
+  static constexpr int kTmemCols = kAcc * BN;
   static_assert(kStages >= 2, "shared memory too small for two k-block stages");
   static_assert(kBytes <= 227 * 1024, "shared memory over the 227 KB per-CTA limit");
 };
@@ -130,27 +145,33 @@ __device__ __forceinline__ void epi_math(const uint32_t* v, const float* scv, co
   o.w = pack_bf16x2(f[6], f[7]);
 }
 
-template <int BN, int AMODE, bool TMA_EPI, int NB>
+template <int BN, int AMODE, bool TMA_EPI, int NB, int RKB>
 __global__ void __launch_bounds__(kThreads, 1)
     conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__ CUtensorMap tmap_a,
                    const __grid_constant__ CUtensorMap tmap_y, const __grid_constant__ CUtensorMap tmap_r,
                    const ConvParams p) {
-  using C = Cfg<BN, TMA_EPI, NB, AMODE == A_HALO>;
+  using C = Cfg<BN, TMA_EPI, NB, AMODE == A_HALO, RKB>;
   constexpr int S = C::kStages;
+  constexpr bool BRES = RKB > 0;
+  constexpr int HB = C::kHB > 0 ? C::kHB : 1;
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 1023u) & ~1023u;
   uint8_t* gbase = smem_raw + (base - raw);
-  const uint32_t sA = base, sB = base + S * C::kABytes, sO = base + C::kOutOff;
+  // ring stage i: A at sA + i * kABytes; B (streamed weights) at sB + i * kBBytes; resident weights at sR
+  const uint32_t sA = base, sB = base + S * C::kABytes, sO = base + C::kOutOff, sR = base + C::kResOff;
   float* sbuf = reinterpret_cast<float*>(gbase + C::kSbufOff);  // [1 or 2][scale BN | shift BN]
   uint64_t* full = reinterpret_cast<uint64_t*>(gbase + C::kBarOff);
   uint64_t* empty = full + S;
-  uint64_t* tfull = empty + S;   // [2]
-  uint64_t* tempty = tfull + 2;  // [2]
-  uint64_t* rbar = tempty + 2;   // [NB <= 4] residual tile landed in staging buffer b (TMA epilogue)
-  uint64_t* hfull = rbar + 4;    // [2] halo buffer landed (A_HALO)
-  uint64_t* hempty = hfull + 2;  // [2] halo buffer consumed by the tile's MMAs (A_HALO)
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(hempty + 2);
+  constexpr int NACC = C::kAcc;
+  constexpr bool SPLIT = C::kSplit;
+  uint64_t* tfull = empty + S;      // [NACC]
+  uint64_t* tempty = tfull + NACC;  // [NACC]
+  uint64_t* rbar = tempty + NACC;   // [NB <= 4] residual tile landed in staging buffer b (TMA epilogue)
+  uint64_t* hfull = rbar + 4;    // [3] halo buffer landed (A_HALO)
+  uint64_t* hempty = hfull + 3;  // [3] halo buffer consumed by the tile's MMAs (A_HALO)
+  uint64_t* wres = hempty + 3;   // [1] resident weights landed (RKB > 0)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(wres + 1);
   const uint32_t sH = base + C::kHaloOff;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -159,15 +180,16 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(&full[i], a_by_tma(AMODE) ? 1 : 128 + 1);
       mbar_init(&empty[i], 1);
     }
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < NACC; ++i) {
       mbar_init(&tfull[i], 1);
-      mbar_init(&tempty[i], kEpiWarps);
+      mbar_init(&tempty[i], SPLIT ? kEpiWarps / 2 : kEpiWarps);
     }
     for (int i = 0; i < 4; ++i) mbar_init(&rbar[i], 1);
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < 3; ++i) {
       mbar_init(&hfull[i], 1);
       mbar_init(&hempty[i], 1);
     }
+    mbar_init(wres, 1);
     fence_mbar_init();
     tma_prefetch(&tmap_w);
     if (a_by_tma(AMODE)) tma_prefetch(&tmap_a);
@@ -181,6 +203,16 @@ __global__ void __launch_bounds__(kThreads, 1)
 
   if (warp < 4) {
     // ======================= producers =======================
+    if constexpr (BRES) {
+      // resident weights: the B slice of this CTA's (fixed) N tile, once
+      if (threadIdx.x == 0) {
+        int m0, nt, g;
+        decode_tile(p, blockIdx.x, m0, nt, g);
+        mbar_arrive_expect_tx(wres, p.nkb * C::kBBytes);
+        for (int kb = 0; kb < p.nkb; ++kb)
+          tma_load_2d(sR + kb * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + nt * BN, wres);
+      }
+    }
     if constexpr (AMODE == A_TMA) {
       if (threadIdx.x == 0) {
         uint32_t gk = 0;
@@ -191,9 +223,9 @@ __global__ void __launch_bounds__(kThreads, 1)
           for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
             const int stage = gk % S;
             if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
-            mbar_arrive_expect_tx(&full[stage], C::kABytes + C::kBBytes);
+            mbar_arrive_expect_tx(&full[stage], C::kStageBytes);
             tma_load_2d(sA + stage * C::kABytes, &tmap_a, g * p.Cg_in + kb * BK, m0, &full[stage]);
-            tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
+            if constexpr (!BRES) tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
           }
         }
       }
@@ -207,16 +239,18 @@ __global__ void __launch_bounds__(kThreads, 1)
           const int mt = m0 / BM, nimg = mt / p.mt_per_img;
           const int p0 = (mt - nimg * p.mt_per_img) * BM;
           const int prow0 = p0 / p.Wp;  // first padded input row (input row prow0 - 1)
-          const uint32_t hb = it & 1;
-          if (it >= 2) mbar_wait(&hempty[hb], ((it >> 1) - 1) & 1);
+          const uint32_t hb = it % HB;
+          if (it >= (uint32_t)HB) mbar_wait(&hempty[hb], ((it / HB) - 1) & 1);
           mbar_arrive_expect_tx(&hfull[hb], box_bytes * p.cblocks);
           for (int cb = 0; cb < p.cblocks; ++cb)
             tma_load_4d(sH + hb * halo_half_bytes(BN) + cb * p.hsz, &tmap_a, cb * BK, -1, prow0 - 1, nimg, &hfull[hb]);
-          for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
-            const int stage = gk % S;
-            if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
-            mbar_arrive_expect_tx(&full[stage], C::kBBytes);
-            tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, 0, &full[stage]);
+          if constexpr (!BRES) {  // streamed weights (resident: nothing else per tile)
+            for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
+              const int stage = gk % S;
+              if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
+              mbar_arrive_expect_tx(&full[stage], C::kBBytes);
+              tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, 0, &full[stage]);
+            }
           }
         }
       }
@@ -399,9 +433,10 @@ __global__ void __launch_bounds__(kThreads, 1)
     {
       constexpr uint32_t idesc = umma_idesc_bf16(BM, BN);
       uint32_t gk = 0, it = 0;
+      if constexpr (BRES) mbar_wait(wres, 0);
       for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x, ++it) {
-        const uint32_t acc = it & 1, use = it >> 1;
-        if (it >= 2) mbar_wait(&tempty[acc], (use - 1) & 1);
+        const uint32_t acc = it % NACC, use = it / NACC;
+        if (it >= (uint32_t)NACC) mbar_wait(&tempty[acc], (use - 1) & 1);
         tc_fence_after();
         const uint32_t tacc = tmem_base + acc * BN;
         uint32_t hbase = 0;
@@ -412,14 +447,16 @@ __global__ void __launch_bounds__(kThreads, 1)
           const int mt = m0 / BM, nimg = mt / p.mt_per_img;
           const int p0 = (mt - nimg * p.mt_per_img) * BM;
           hoff = p0 - (p0 / p.Wp) * p.Wp;  // first output position's column in the first halo row
-          hbase = sH + (it & 1) * halo_half_bytes(BN);
-          mbar_wait(&hfull[it & 1], (it >> 1) & 1);
+          hbase = sH + (it % HB) * halo_half_bytes(BN);
+          mbar_wait(&hfull[it % HB], (it / HB) & 1);
         }
         auto kblock = [&](const int kb) {
           const int stage = gk % S;
           // (TMA completion / the producers' fence.proxy.async + arrive order the smem writes before the MMA)
-          mbar_wait(&full[stage], (gk / S) & 1);
-          const uint32_t a0 = sA + stage * C::kABytes, b0 = sB + stage * C::kBBytes;
+          constexpr bool kRing = !(BRES && AMODE == A_HALO);  // halo + resident weights: no ring
+          if constexpr (kRing) mbar_wait(&full[stage], (gk / S) & 1);
+          const uint32_t a0 = sA + stage * C::kABytes;
+          const uint32_t b0 = BRES ? sR + kb * C::kBBytes : sB + stage * C::kBBytes;
           if constexpr (AMODE == A_HALO) {
             // k-block kb = tap * cblocks + cb, tap = r * 3 + s: A = halo rows shifted by r * Wp + s
             const int tap = kb / p.cblocks, cb = kb - tap * p.cblocks;
@@ -446,7 +483,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             tc_mma_bf16_warp(tacc, da + 4, db + 4, idesc, 1u);
             tc_mma_bf16_warp(tacc, da + 6, db + 6, idesc, 1u);
           }
-          tc_commit_warp(&empty[stage]);
+          if constexpr (kRing) tc_commit_warp(&empty[stage]);
           ++gk;
         };
         // unrolled by 4: a rolled loop costs a YIELD + branch-resolution stall per k-block (measured)
@@ -459,19 +496,28 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
         for (; kb < p.nkb; ++kb) kblock(kb);
         tc_commit_warp(&tfull[acc]);
-        if constexpr (AMODE == A_HALO) tc_commit_warp(&hempty[it & 1]);  // halo free once these MMAs finish
+        if constexpr (AMODE == A_HALO) tc_commit_warp(&hempty[it % HB]);  // halo free once these MMAs finish
       }
     }
   } else {
-    // ================ epilogue (8 warps: one output row per lane, half of the columns each) ================
+    // ================ epilogue (8 warps, one output row per lane) ================
+    // SPLIT: warp group (warp - 5) / 4 takes every other tile and all of its columns; otherwise the two
+    // warps of a TMEM lane quadrant split each tile's columns in halves.
     const int et = threadIdx.x - kEpiWarp0 * 32;
     const int q = warp & 3;  // TMEM lane quadrant this warp may access
     const int row = q * 32 + lane;
-    const int half = (warp - kEpiWarp0) >> 2;  // column half of the tile this warp owns
+    const int grp = (warp - kEpiWarp0) >> 2;
+    const int half = SPLIT ? 0 : grp;  // column half of the tile this warp owns
+    const int gthreads = SPLIT ? kEpiThreads / 2 : kEpiThreads;
+    const int gt = SPLIT ? (et & (kEpiThreads / 2 - 1)) : et;
+    const int gbar = SPLIT ? 1 + grp : 1;
     const bool has_res = p.res != nullptr;
-    uint32_t it = 0;
-    for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x, ++it) {
-      const uint32_t acc = it & 1, use = it >> 1;
+    int loaded0 = -1, loaded1 = -1;  // N offset whose scale / shift each smem buffer holds
+    const int tstep = SPLIT ? 2 : 1;
+    uint32_t it = SPLIT ? grp : 0;
+    for (int tile = blockIdx.x + (SPLIT ? grp * (int)gridDim.x : 0); tile < p.n_tiles;
+         tile += tstep * gridDim.x, it += tstep) {
+      const uint32_t acc = it % NACC, use = it / NACC;
       int m0, nt, g;
       decode_tile(p, tile, m0, nt, g);
       const int n0 = nt * BN;
@@ -513,13 +559,22 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
         }
       }
-      // stage this tile's scale / shift in smem (double-buffered by accumulator)
-      float* ss = sbuf + (TMA_EPI ? 0 : acc * 2 * BN);
-      for (int i = et; i < 2 * BN; i += kEpiThreads) {
-        const int c = i < BN ? i : i - BN;
-        ss[i] = c < nvalid_tile ? (i < BN ? p.scale[ng0 + c] : p.shift[ng0 + c]) : 0.f;
+      // this tile's scale / shift in smem: SPLIT one buffer per warp group, TMA epilogue one buffer, else
+      // double-buffered by accumulator; reloaded only when the tile's N offset changes (resident-weight
+      // launches and single-N-tile layers load it once)
+      const int sb = SPLIT ? grp : (TMA_EPI ? 0 : (int)acc);
+      float* ss = sbuf + sb * 2 * BN;
+      const bool reload = (sb == 0 ? loaded0 : loaded1) != ng0;
+      if (reload) {
+        if (!TMA_EPI) named_bar_sync(gbar, gthreads);  // every warp of the group is done with the buffer
+        for (int i = gt; i < 2 * BN; i += gthreads) {
+          const int c = i < BN ? i : i - BN;
+          ss[i] = c < nvalid_tile ? (i < BN ? p.scale[ng0 + c] : p.shift[ng0 + c]) : 0.f;
+        }
+        if (sb == 0) loaded0 = ng0;
+        else loaded1 = ng0;
       }
-      named_bar_sync(1, kEpiThreads);
+      if (TMA_EPI || reload) named_bar_sync(gbar, gthreads);
       int mo = m0 + row;
       bool rvalid = mo < p.M;
       if constexpr (AMODE == A_HALO) {  // padded-width position -> output pixel (columns >= Wo discarded)
@@ -530,7 +585,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         mo = (nimg * p.Ho + ho) * p.Wo + wo;
       }
       const size_t off = (size_t)(rvalid ? mo : 0) * p.Cout + ng0;
-      constexpr int kChunks = BN / 64;  // 32-column chunks per warp
+      constexpr int kChunks = SPLIT ? BN / 32 : BN / 64;  // 32-column chunks per warp
       const int cb0 = half * kChunks;
       uint4 rres[4] = {};
       if constexpr (TMA_EPI) {
@@ -748,6 +803,12 @@ static const bool g_halo_enabled = [] {
   return !(e && e[0] == '0');
 }();
 
+// VISTA_WRES=0 disables the resident-weight launches (A/B measurements)
+static const bool g_wres_enabled = [] {
+  const char* e = getenv("VISTA_WRES");
+  return !(e && e[0] == '0');
+}();
+
 // N-D bf16 tiled tensor map with 128B swizzle; returns the driver status (callers may fall back)
 static CUresult encode_nd(CUtensorMap* m, const void* ptr, int rank, const cuuint64_t* dims,
                           const cuuint64_t* strides, const cuuint32_t* box) {
@@ -827,27 +888,39 @@ void conv_layer_free(ConvLayer& L) {
   L.scale = L.shift = nullptr;
 }
 
-template <int BN, int AMODE, bool TE, int NB>
+template <int BN, int AMODE, bool TE, int NB, int RKB = 0>
 static void launch_t(const ConvLayer& L, const CUtensorMap& ta, const CUtensorMap& ty, const CUtensorMap& tr,
                      const ConvParams& p, cudaStream_t st) {
   static_assert(NB >= 1 && NB <= 4, "staging buffers");
-  auto kern = conv_tc_kernel<BN, AMODE, TE, NB>;
-  constexpr int smem = Cfg<BN, TE, NB, AMODE == A_HALO>::kBytes;
+  auto kern = conv_tc_kernel<BN, AMODE, TE, NB, RKB>;
+  constexpr int smem = Cfg<BN, TE, NB, AMODE == A_HALO, RKB>::kBytes;
   static bool attr_set = false;  // per instantiation
   if (!attr_set) {
     VCHECK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
     attr_set = true;
   }
-  const int grid = p.n_tiles < num_sms() ? p.n_tiles : num_sms();
+  int grid = p.n_tiles < num_sms() ? p.n_tiles : num_sms();
+  if (RKB > 0) {  // every CTA keeps one N tile: grid a multiple of the N-tile count (groups == 1)
+    if (p.nkb > RKB || p.n_nt > grid) fail(1, "conv: resident-weight launch misconfigured");
+    grid -= grid % p.n_nt;
+  }
   kern<<<grid, kThreads, smem, st>>>(L.tmap_w, ta, ty, tr, p);
   LAUNCHED();
 }
 
 template <int BN, bool TE, int NB>
 static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, const CUtensorMap& ty,
-                      const CUtensorMap& tr, const ConvParams& p, cudaStream_t st) {
+                      const CUtensorMap& tr, const ConvParams& p, cudaStream_t st, int rkb) {
   switch (amode) {
-    case A_TMA: launch_t<BN, A_TMA, TE, NB>(L, ta, ty, tr, p, st); break;
+    case A_TMA:
+      if constexpr (TE && BN <= 128) {
+        if (rkb == 4) {
+          launch_t<BN, A_TMA, TE, NB, 4>(L, ta, ty, tr, p, st);
+          break;
+        }
+      }
+      launch_t<BN, A_TMA, TE, NB>(L, ta, ty, tr, p, st);
+      break;
     case A_GATHER_FAST: launch_t<BN, A_GATHER_FAST, TE, NB>(L, ta, ty, tr, p, st); break;
     case A_GATHER_ROW: launch_t<BN, A_GATHER_ROW, TE, NB>(L, ta, ty, tr, p, st); break;
     case A_IM2COL: launch_t<BN, A_IM2COL, TE, NB>(L, ta, ty, tr, p, st); break;
@@ -857,6 +930,12 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
       else fail(1, "conv: row-view mode needs the TMA epilogue");
       break;
     case A_HALO:
+      if constexpr (!TE && BN == 64) {
+        if (rkb == 9) {
+          launch_t<BN, A_HALO, TE, NB, 9>(L, ta, ty, tr, p, st);
+          break;
+        }
+      }
       if constexpr (!TE && BN <= 128) launch_t<BN, A_HALO, TE, NB>(L, ta, ty, tr, p, st);
       else fail(1, "conv: halo mode needs the register epilogue and BN <= 128");
       break;
@@ -985,29 +1064,36 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   }
   const double flops = 2.0 * (double)M * L.Cout * L.K_alg;  // algorithmic (unpadded) MACs x 2
   const double bytes = 2.0 * ((double)N * H * W * L.Cin + (double)M * L.Cout * (res ? 2 : 1) + (double)L.Cout * L.Kp);
+  // resident weights (see Cfg): 3x3 halo convs with Cout = 64 (9 k-blocks of 8 KB) and 1x1 TMA convs with
+  // K <= 256 and BN <= 128 (<= 4 k-blocks); one N tile per CTA needs groups == 1 and n_nt <= the grid
+  int rkb = 0;
+  if (g_wres_enabled && L.groups == 1 && p.n_nt <= num_sms() && p.n_tiles >= num_sms()) {
+    if (amode == A_HALO && L.BN == 64 && p.nkb <= 9) rkb = 9;
+    else if (amode == A_TMA && tma_epi && L.BN <= 128 && p.nkb <= 4) rkb = 4;
+  }
   prof_begin(st);
   int nb = 1;
   if (tma_epi) {
     if (L.BN == 256) {
-      launch_bn<256, true, 1>(L, amode, ta, ty, tr, p, st);
+      launch_bn<256, true, 1>(L, amode, ta, ty, tr, p, st, rkb);
     } else if (L.BN == 128) {
       nb = g_epi_nb_env == 2 ? 2 : 3;
-      if (nb == 2) launch_bn<128, true, 2>(L, amode, ta, ty, tr, p, st);
-      else launch_bn<128, true, 3>(L, amode, ta, ty, tr, p, st);
+      if (nb == 2) launch_bn<128, true, 2>(L, amode, ta, ty, tr, p, st, rkb);
+      else launch_bn<128, true, 3>(L, amode, ta, ty, tr, p, st, rkb);
     } else {
       nb = g_epi_nb_env == 2 ? 2 : 4;
-      if (nb == 2) launch_bn<64, true, 2>(L, amode, ta, ty, tr, p, st);
-      else launch_bn<64, true, 4>(L, amode, ta, ty, tr, p, st);
+      if (nb == 2) launch_bn<64, true, 2>(L, amode, ta, ty, tr, p, st, rkb);
+      else launch_bn<64, true, 4>(L, amode, ta, ty, tr, p, st, rkb);
     }
   } else {
-    if (L.BN == 256) launch_bn<256, false, 1>(L, amode, ta, ty, tr, p, st);
-    else if (L.BN == 128) launch_bn<128, false, 1>(L, amode, ta, ty, tr, p, st);
-    else launch_bn<64, false, 1>(L, amode, ta, ty, tr, p, st);
+    if (L.BN == 256) launch_bn<256, false, 1>(L, amode, ta, ty, tr, p, st, rkb);
+    else if (L.BN == 128) launch_bn<128, false, 1>(L, amode, ta, ty, tr, p, st, rkb);
+    else launch_bn<64, false, 1>(L, amode, ta, ty, tr, p, st, rkb);
   }
   char label[160] = {0};
   if (prof_labels())
-    snprintf(label, sizeof(label), "conv R%d S%d s%d g%d Cin%d Cout%d HxW%dx%d M%d K%d BN%d amode%d epi%d nb%d tiles%d%s", L.R,
-             L.S, L.stride, L.groups, L.Cin, L.Cout, H, W, p.M, L.K, L.BN, amode, tma_epi ? 1 : 0, nb, p.n_tiles,
+    snprintf(label, sizeof(label), "conv R%d S%d s%d g%d Cin%d Cout%d HxW%dx%d M%d K%d BN%d amode%d epi%d nb%d rkb%d tiles%d%s", L.R,
+             L.S, L.stride, L.groups, L.Cin, L.Cout, H, W, p.M, L.K, L.BN, amode, tma_epi ? 1 : 0, nb, rkb, p.n_tiles,
              res ? " res" : "");
   prof_end(st, 0, flops, bytes, label);
   return tapf == nullptr || fuse_tap;

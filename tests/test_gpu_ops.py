@@ -49,6 +49,9 @@ CONV = [
     (3, 28, 28, 128, 128, 3, 1, 1, 1, False, True),    # ResNet res3 3x3: halo mode, BN = 128, 2 channel blocks
     (2, 10, 10, 128, 64, 3, 1, 1, 1, False, False),    # halo mode, tiles spanning image ends, no ReLU
     (1, 5, 130, 64, 64, 3, 1, 1, 1, False, True),      # wide rows: halo does not fit -> im2col boxes
+    (7, 56, 56, 64, 64, 3, 1, 1, 1, False, True),      # halo + resident weights (>= 148 tiles), 3 halo buffers
+    (13, 14, 14, 256, 1024, 1, 1, 0, 1, True, True),   # 1x1 resident weights, 8 N tiles (grid 144), M tail
+    (6, 28, 28, 128, 512, 1, 1, 0, 1, False, True),    # 1x1 resident weights, K = 128, 4 N tiles
 ]
 
 

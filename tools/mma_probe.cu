@@ -9,10 +9,12 @@
 using namespace vista;
 
 template <int N>
-__global__ void __launch_bounds__(128, 1) probe(int iters, unsigned long long* out) {
+__global__ void __launch_bounds__(128, 1) probe(int iters, unsigned long long* out, int ashift, int alt = 1) {
   extern __shared__ __align__(1024) uint8_t smem[];
   const uint32_t base = (smem_u32(smem) + 1023u) & ~1023u;
-  const uint32_t sA = base, sB = base + 128 * 128;  // A: 128 x 64 bf16, B: N x 64 bf16 (zeros are fine)
+  // A: 128 x 64 bf16 starting ashift 128-byte rows into a 256-row buffer (halo-style row-shifted operand),
+  // B: N x 64 bf16 (zeros are fine)
+  const uint32_t sA = base + ashift * 128, sB = base + 256 * 128;
   __shared__ uint64_t bar;
   __shared__ uint32_t slot;
   const int warp = threadIdx.x >> 5;
@@ -20,7 +22,7 @@ __global__ void __launch_bounds__(128, 1) probe(int iters, unsigned long long* o
     mbar_init(&bar, 1);
     fence_mbar_init();
   }
-  for (int i = threadIdx.x; i < (128 + N) * 128 / 16; i += blockDim.x) sts128(base + i * 16, make_uint4(0, 0, 0, 0));
+  for (int i = threadIdx.x; i < (256 + N) * 128 / 16; i += blockDim.x) sts128(base + i * 16, make_uint4(0, 0, 0, 0));
   fence_proxy_async_smem();
   if (warp == 0) tmem_alloc(&slot, 512);
   tc_fence_before();
@@ -33,7 +35,7 @@ __global__ void __launch_bounds__(128, 1) probe(int iters, unsigned long long* o
     for (int i = 0; i < iters; ++i) {
 #pragma unroll
       for (int k = 0; k < 4; ++k)
-        tc_mma_bf16(tmem + (i & 1) * N, umma_desc_k_sw128(sA + k * 32), umma_desc_k_sw128(sB + k * 32), idesc,
+        tc_mma_bf16(tmem + (alt ? (i & 1) * N : 0), umma_desc_k_sw128(sA + k * 32), umma_desc_k_sw128(sB + k * 32), idesc,
                     1u);
     }
     tc_commit(&bar);
@@ -92,18 +94,18 @@ __global__ void __launch_bounds__(128, 1) commit_probe(int iters, int with_mma, 
 }
 
 template <int N>
-void run(int grid) {
+void run(int grid, int ashift = 0, int alt = 1) {
   unsigned long long* d;
   cudaMalloc(&d, 8);
   const int iters = 20000;
-  const int smem = (128 + N) * 128 + 2048;
+  const int smem = (256 + N) * 128 + 2048;
   cudaFuncSetAttribute(probe<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  probe<N><<<grid, 128, smem>>>(100, d);
+  probe<N><<<grid, 128, smem>>>(100, d, ashift, alt);
   cudaEvent_t a, b;
   cudaEventCreate(&a);
   cudaEventCreate(&b);
   cudaEventRecord(a);
-  probe<N><<<grid, 128, smem>>>(iters, d);
+  probe<N><<<grid, 128, smem>>>(iters, d, ashift, alt);
   cudaEventRecord(b);
   cudaEventSynchronize(b);
   float ms = 0;
@@ -112,7 +114,7 @@ void run(int grid) {
   cudaMemcpy(&cyc, d, 8, cudaMemcpyDeviceToHost);
   const double mmas = 4.0 * iters;
   const double tflops = 2.0 * 128 * N * 16 * mmas * grid / (ms * 1e-3) / 1e12;
-  printf("N=%3d grid=%3d: %.1f cycles/MMA (block 0), %.3f ms, %.0f TFLOP/s  err=%s\n", N, grid, cyc / mmas, ms,
+  printf("N=%3d grid=%3d ashift=%3d alt=%d: %.1f cycles/MMA (block 0), %.3f ms, %.0f TFLOP/s  err=%s\n", N, grid, ashift, alt, cyc / mmas, ms,
          tflops, cudaGetErrorString(cudaGetLastError()));
   cudaFree(d);
 }
@@ -138,6 +140,18 @@ int main() {
     run<64>(g);
     run<128>(g);
     run<256>(g);
+  }
+  // row-shifted A operands (A_HALO): does a start that is not a multiple of 8 rows cost smem bandwidth?
+  // one accumulator for every MMA (a conv tile's whole K loop) vs alternating two
+  for (int g : {1, sms}) {
+    run<64>(g, 0, 0);
+    run<128>(g, 0, 0);
+    run<256>(g, 0, 0);
+  }
+  for (int sh : {1, 59}) {
+    run<64>(1, sh);
+    run<128>(1, sh);
+    run<256>(1, sh);
   }
   return 0;
 }

@@ -213,6 +213,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--images", type=int, default=0, help="override images per GPU (debug only)")
     ap.add_argument("--micro-batch", type=int, default=0, help="stage-1 micro-batch (0 = planner)")
+    ap.add_argument("--from-base", action="store_true",
+                    help="App. B: materialise the first requested layer once (untimed, reported as materialize_s) "
+                         "and time vista_transfer_from_base + train instead of the transfer from pixels")
     ap.add_argument("--plan", default="staged", choices=["staged", "eager", "lazy"],
                     help="logical plan (Fig 5): staged is the product; eager / lazy for config 4 comparisons")
     args = ap.parse_args()
@@ -262,9 +265,25 @@ def main():
               stream=stream.cuda_stream, micro_batch=args.micro_batch, plan=args.plan)
     info = v.plan_info()
     d_tot = [d_s + d for d in info["d_l"]]
+    materialize_s = None
+    if args.from_base:
+        H, W, C, _ = v.base_shape()
+        d_base = torch.empty((n_img, H, W, C), dtype=torch.bfloat16, device=dev)
+        torch.cuda.synchronize(dev)
+        t0 = time.time()
+        v.materialize(d_px, d_base)
+        materialize_s = time.time() - t0
+        h_base = torch.empty((n_img, H, W, C), dtype=torch.bfloat16).pin_memory()
+        h_base.copy_(d_base)
+        h2d_bytes += h_base.numel() * 2 - h_px.numel()
 
     def step(host=False):
-        if host:
+        if args.from_base:
+            if host:
+                v.transfer_from_base(h_base, h_ik, h_X, h_sk, h_y)
+            else:
+                v.transfer_from_base(d_base, d_ik, d_X, d_sk, d_y)
+        elif host:
             v.transfer(h_px, h_ik, h_X, h_sk, h_y)
         else:
             v.transfer(d_px, d_ik, d_X, d_sk, d_y)
@@ -374,7 +393,10 @@ def main():
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
             "data": "synthetic",
             "config": dict(workload_config(args.config, world, n_img), micro_batch=info["micro_batch"],
-                           plan=args.plan, peak_bytes_pred=info["peak_bytes_pred"]),
+                           plan=args.plan + ("+prematerialized_base" if args.from_base else ""),
+                           peak_bytes_pred=info["peak_bytes_pred"],
+                           **({"base_layer": TAP_NAMES[cnn][taps[0]], "materialize_s": round(materialize_s, 3)}
+                              if args.from_base else {})),
             "roofline": roof,
             "cpu_baseline": cpu,
             "e2e": {"value": N_global / (e2e_step / 1000.0), "unit": "images/s", "ms_per_step": e2e_step,

@@ -156,6 +156,28 @@ vista_status vista_transfer(vista_ctx* ctx, const uint8_t* images, const int64_t
                             const float* structured, const int64_t* str_keys, const uint8_t* labels);
 vista_status vista_features(const vista_ctx* ctx, int32_t k, vista_buffer* out);
 
+/* ---- Pre-materialised base layer (App. B) ----
+ * "a base layer can [be] pre-materialized before hand for later use of exploring other layers"
+ * (PAPER.md:714-716); "for the other layers partial CNN inference is performed starting from the
+ * base layer".  The base layer is the FIRST requested layer L[0] of the plan.
+ *
+ * vista_base_shape: out4 = {H, W, C, bytes per element} of one image's base activation A_{L[0]}
+ *   (FC layer: H = W = 1, C = d); elements are bf16 (2 bytes), fp32 (4) in VISTA_F32.
+ * vista_materialize: base_out <- A_{L[0]} of the n_images_local images, NHWC [n, H, W, C] in the
+ *   context's element type: inference from pixels through L[0] only, over the planner's chunks.
+ *   images as in vista_transfer.  base_out: caller-owned host (pinned or pageable) or device
+ *   buffer of n_images_local * H * W * C elements.  Does not change the vista_features state.
+ * vista_transfer_from_base: vista_transfer with the CNN started at the stored base layer: no
+ *   inference below L[0]; F_0 = g_{L[0]}(base); A_{L[k]} = f^_{L[0] -> L[k]}(base) for k >= 1
+ *   (Def 3.7 partial inference); join, concat and MM_k as vista_transfer.  base: host or device,
+ *   the layout vista_materialize writes (read only; a device base is read in place).  Results are
+ *   bit-identical to vista_transfer from the pixels the base was materialised from.  Staged plan
+ *   only (VISTA_ERR_INVALID_ARG for Eager / Lazy). */
+vista_status vista_base_shape(const vista_ctx* ctx, int64_t* out4);
+vista_status vista_materialize(vista_ctx* ctx, const uint8_t* images, void* base_out);
+vista_status vista_transfer_from_base(vista_ctx* ctx, const void* base, const int64_t* image_keys,
+                                      const float* structured, const int64_t* str_keys, const uint8_t* labels);
+
 /* vista_train(layer) -> weights / accuracy.  Collective over the `world` ranks (all must call
  * with the same k): per-rank partial sums are combined by an fp64 NCCL allreduce.
  *   weights_out: caller-owned double[d_s + d_l + 1] or NULL: w in standardised space for the

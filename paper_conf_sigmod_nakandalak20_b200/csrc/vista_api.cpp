@@ -793,11 +793,15 @@ VISTA_API vista_status vista_plan_info(const vista_ctx* c, vista_plan_info_t* o)
   return VISTA_OK;
 }
 
-VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const int64_t* image_keys,
-                                      const float* structured, const int64_t* str_keys, const uint8_t* labels) {
-  if (!c) return VISTA_ERR_INVALID_ARG;
-  return guarded(c, [&] {
-    if (c->n_img > 0 && (!images || !image_keys)) fail(1, "images / image_keys are NULL");
+// Body of vista_transfer and vista_transfer_from_base.  base == nullptr: from pixels.  base != nullptr:
+// the CNN starts at the stored activation of the first requested layer (App. B):
+// block t0 = taps[0] is not run, A_t0 = base, and blocks t0+1 .. t_max are partial inference from it.
+static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base, const int64_t* image_keys,
+                          const float* structured, const int64_t* str_keys, const uint8_t* labels) {
+  {
+    if (c->n_img > 0 && !image_keys) fail(1, "image_keys is NULL");
+    if (c->n_img > 0 && !images && !base) fail(1, "images / base is NULL");
+    if (base && c->sys.plan != VISTA_PLAN_STAGED) fail(1, "a pre-materialised base layer needs the Staged plan");
     if (c->n_str > 0 && (!str_keys || !labels || (c->d_s > 0 && !structured))) fail(1, "structured table is NULL");
     VCHECK(cudaSetDevice(c->sys.device));
     c->transferred = false;
@@ -805,9 +809,12 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
     const auto& S = c->net.stages;
     // ---- inputs (H2D when given host pointers) ----
     // (the Staged plan streams host pixels to the device chunk by chunk; Eager / Lazy copy them once)
-    const uint8_t* px = c->sys.plan == VISTA_PLAN_STAGED
+    const uint8_t* px = c->sys.plan == VISTA_PLAN_STAGED || base
                             ? images
                             : (const uint8_t*)to_device(c, c->d_px, images, (size_t)c->n_img * S[0].in_elems);
+    const int t0 = base ? c->taps[0] : -1;  // block whose output is the stored base layer
+    const size_t base_img_bytes = base ? (size_t)S[t0].out_elems * c->esz : 0;
+    const bool host_base = base && c->n_img > 0 && !is_device_ptr(base);
     const int64_t* ik = (const int64_t*)to_device(c, c->d_img_keys, image_keys, (size_t)c->n_img * 8);
     const int64_t* sk = (const int64_t*)to_device(c, c->d_str_keys, str_keys, (size_t)c->n_str * 8);
     const float* X = (const float*)to_device(c, c->d_X, structured, (size_t)c->n_str * c->d_s * 4);
@@ -866,7 +873,7 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
     // ---- Staged (Fig 5E), over chunks of images when the HBM budget forces it (planner) ----
     const int64_t CH = c->sys.plan == VISTA_PLAN_STAGED ? std::max<int64_t>(c->chunk, 1) : 0;
     const bool chunked = CH > 0 && CH < c->n_img;
-    const bool host_px = px == images && c->n_img > 0 && !is_device_ptr(images);
+    const bool host_px = !base && px == images && c->n_img > 0 && !is_device_ptr(images);
     if (CH > 0) {
       size_t need[2] = {16, 16};
       for (int t = 0; t <= c->t_max; ++t)
@@ -877,27 +884,37 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
     }
     for (int64_t c0 = 0; CH > 0 && c0 < c->n_img; c0 += CH) {
       const int64_t nc = std::min<int64_t>(CH, c->n_img - c0);
-      const uint8_t* pxc = px + (size_t)c0 * S[0].in_elems;
+      const uint8_t* pxc = base ? nullptr : px + (size_t)c0 * S[0].in_elems;
+      const void* base_c = nullptr;  // this chunk's A_t0 (the caller's memory, or its H2D copy in arena t0 % 2)
+      if (base) {
+        if (host_base) {
+          VCHECK(cudaMemcpyAsync(c->arena[t0 & 1].p, (const uint8_t*)base + (size_t)c0 * base_img_bytes,
+                                 (size_t)nc * base_img_bytes, cudaMemcpyHostToDevice, st));
+          base_c = c->arena[t0 & 1].p;
+        } else {
+          base_c = (const uint8_t*)base + (size_t)c0 * base_img_bytes;
+        }
+      }
       if (host_px) {  // stream the chunk's pixels to the device
         c->d_px.ensure((size_t)nc * S[0].in_elems);
         VCHECK(cudaMemcpyAsync(c->d_px.p, images + (size_t)c0 * S[0].in_elems, (size_t)nc * S[0].in_elems,
                                cudaMemcpyHostToDevice, st));
         pxc = (const uint8_t*)c->d_px.p;
       }
-      for (int t = 0; t <= c->t_max; ++t) {
-        void* At = c->arena[t & 1].p;
+      for (int t = base ? t0 : 0; t <= c->t_max; ++t) {
+        void* At = t == t0 ? const_cast<void*>(base_c) : c->arena[t & 1].p;
         c->act[t] = At;
-        const void* in = t == 0 ? (const void*)pxc : c->arena[(t - 1) & 1].p;
+        const void* in = t == 0 ? (const void*)pxc : (t - 1 == t0 ? base_c : c->arena[(t - 1) & 1].p);
         const int k = layer_index(c, t);
         // S2 fused into the producing conv's epilogue (opt-in, unchunked only)
         unsigned int* tapf = nullptr;
-        if (k >= 0 && !S[t].fc_tap && c->fuse_tap && !chunked && !c->f32) {
+        if (k >= 0 && t != t0 && !S[t].fc_tap && c->fuse_tap && !chunked && !c->f32) {
           const size_t cnt = (size_t)nc * 4 * S[t].outC;
           c->tapacc.ensure(cnt * 4);
           VCHECK(cudaMemsetAsync(c->tapacc.p, 0, cnt * 4, st));  // max over non-negative (post-ReLU) values
           tapf = (unsigned int*)c->tapacc.p;
         }
-        const bool fused = run_block(c, t, in, At, nc, tapf);
+        const bool fused = t == t0 ? false : run_block(c, t, in, At, nc, tapf);
         if (k >= 0) {
           void* Ft = (uint8_t*)c->F[t]->p + (size_t)c0 * S[t].d_tap * c->esz;
           if (S[t].fc_tap)  // g = identity on FC layers
@@ -915,6 +932,68 @@ VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const
     VCHECK(cudaStreamSynchronize(st));
     if (g_prof) g_prof->flush();
     c->transferred = true;
+  }
+}
+
+VISTA_API vista_status vista_transfer(vista_ctx* c, const uint8_t* images, const int64_t* image_keys,
+                                      const float* structured, const int64_t* str_keys, const uint8_t* labels) {
+  if (!c) return VISTA_ERR_INVALID_ARG;
+  return guarded(c, [&] { transfer_body(c, images, nullptr, image_keys, structured, str_keys, labels); });
+}
+
+VISTA_API vista_status vista_transfer_from_base(vista_ctx* c, const void* base, const int64_t* image_keys,
+                                                const float* structured, const int64_t* str_keys,
+                                                const uint8_t* labels) {
+  if (!c) return VISTA_ERR_INVALID_ARG;
+  return guarded(c, [&] {
+    if (c->n_img > 0 && !base) fail(1, "base is NULL");
+    transfer_body(c, nullptr, base, image_keys, structured, str_keys, labels);
+  });
+}
+
+VISTA_API vista_status vista_base_shape(const vista_ctx* c, int64_t* out4) {
+  if (!c || !out4) return VISTA_ERR_INVALID_ARG;
+  const StageDesc& S = c->net.stages[c->taps[0]];
+  out4[0] = S.outH;
+  out4[1] = S.outW;
+  out4[2] = S.outC;
+  out4[3] = c->esz;
+  return VISTA_OK;
+}
+
+// Materialise the base layer (App. B): inference from pixels through block taps[0] only, over the
+// planner's chunks and micro-batches, and A_t0 of every local image copied to the caller's buffer.
+VISTA_API vista_status vista_materialize(vista_ctx* c, const uint8_t* images, void* base_out) {
+  if (!c) return VISTA_ERR_INVALID_ARG;
+  return guarded(c, [&] {
+    if (c->n_img > 0 && (!images || !base_out)) fail(1, "images / base_out is NULL");
+    VCHECK(cudaSetDevice(c->sys.device));
+    cudaStream_t st = c->stream;
+    const auto& S = c->net.stages;
+    const int t0 = c->taps[0];
+    const int64_t CH = std::max<int64_t>(std::min<int64_t>(c->chunk > 0 ? c->chunk : c->n_img, c->n_img), 1);
+    const bool host_px = c->n_img > 0 && !is_device_ptr(images);
+    size_t need[2] = {16, 16};
+    for (int t = 0; t <= t0; ++t)
+      need[t & 1] = std::max(need[t & 1], (size_t)CH * S[t].out_elems * c->esz + 16);
+    c->arena[0].ensure(need[0]);
+    c->arena[1].ensure(need[1]);
+    const size_t eb = (size_t)S[t0].out_elems * c->esz;
+    for (int64_t c0 = 0; c0 < c->n_img; c0 += CH) {
+      const int64_t nc = std::min<int64_t>(CH, c->n_img - c0);
+      const uint8_t* pxc = images + (size_t)c0 * S[0].in_elems;
+      if (host_px) {
+        c->d_px.ensure((size_t)nc * S[0].in_elems);
+        VCHECK(cudaMemcpyAsync(c->d_px.p, pxc, (size_t)nc * S[0].in_elems, cudaMemcpyHostToDevice, st));
+        pxc = (const uint8_t*)c->d_px.p;
+      }
+      for (int t = 0; t <= t0; ++t)
+        run_block(c, t, t == 0 ? (const void*)pxc : c->arena[(t - 1) & 1].p, c->arena[t & 1].p, nc, nullptr);
+      VCHECK(cudaMemcpyAsync((uint8_t*)base_out + (size_t)c0 * eb, c->arena[t0 & 1].p, (size_t)nc * eb,
+                             cudaMemcpyDefault, st));
+    }
+    VCHECK(cudaStreamSynchronize(st));
+    if (g_prof) g_prof->flush();
   });
 }
 

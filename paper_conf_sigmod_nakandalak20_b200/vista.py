@@ -81,6 +81,9 @@ def lib():
         L.vista_plan_info.argtypes = [_vp, ctypes.POINTER(PlanInfo)]
         L.vista_transfer.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp]
         L.vista_features.argtypes = [_vp, _i32, ctypes.POINTER(Buffer)]
+        L.vista_base_shape.argtypes = [_vp, ctypes.POINTER(_i64)]
+        L.vista_materialize.argtypes = [_vp, _vp, _vp]
+        L.vista_transfer_from_base.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp]
         L.vista_train.argtypes = [_vp, _i32, _vp, ctypes.POINTER(Metrics)]
         L.vista_destroy.argtypes = [_vp]
         L.vista_destroy.restype = None
@@ -270,6 +273,21 @@ class Vista:
     def transfer(self, images, image_keys, structured, str_keys, labels):
         _check(lib().vista_transfer(self.ctx, _ptr(images), _ptr(image_keys), _ptr(structured), _ptr(str_keys),
                                     _ptr(labels)), self.ctx)
+
+    def base_shape(self):
+        """(H, W, C, bytes per element) of one image's base-layer activation A_{L[0]} (App. B)."""
+        o = (_i64 * 4)()
+        _check(lib().vista_base_shape(self.ctx, o), self.ctx)
+        return tuple(int(v) for v in o)
+
+    def materialize(self, images, base_out):
+        """base_out <- A_{L[0]} of every local image (NHWC, host or device tensor / array)."""
+        _check(lib().vista_materialize(self.ctx, _ptr(images), _ptr(base_out)), self.ctx)
+
+    def transfer_from_base(self, base, image_keys, structured, str_keys, labels):
+        """vista_transfer started at the pre-materialised base layer (App. B)."""
+        _check(lib().vista_transfer_from_base(self.ctx, _ptr(base), _ptr(image_keys), _ptr(structured),
+                                              _ptr(str_keys), _ptr(labels)), self.ctx)
 
     def features(self, k):
         import torch

@@ -240,3 +240,61 @@ def test_resnet_chain_fused_bit_identical(monkeypatch):
         v.close()
     for a, b in zip(out["1"], out["0"]):
         assert torch.equal(a, b)
+
+
+@pytest.mark.parametrize("cnn,taps,n,d_s,chunked", [(0, [1, 2, 3], 10, 8, False), (2, [1, 3, 4], 6, 16, False),
+                                                    (2, [0, 2, 4], 40, 8, True)])
+def test_pre_materialized_base_layer(cnn, taps, n, d_s, chunked):
+    # App. B: materialise the base layer L[0] once, then transfer from it.  Same kernels on the
+    # same bf16 base -> MM_k bit-identical to the transfer from pixels, for host and device bases and for chunked
+    # plans; the base itself and the features computed from it match the fp64 oracle's partial inference
+    # f^_{L[0] -> L[k]} (oracle.features_from, Def 3.7) on the GPU's own base.
+    tab = gen.make_tables(n, d_s)
+    kw = {}
+    if chunked:
+        probe = run_gpu(cnn, taps, tab, d_s, iters=2)
+        kw["hbm_budget_bytes"] = probe.plan_info()["weight_bytes"] + (256 << 20) + (24 << 20)
+        probe.close()
+    ref = run_gpu(cnn, taps, tab, d_s, iters=2, **kw)
+    if chunked:
+        assert ref.plan_info()["chunk_images"] < n
+    mm_ref = [ref.features(k)["mm"].view(torch.int16).cpu().clone() for k in range(len(taps))]
+    w_ref = [ref.train(k, d_s + ref.features(k)["d_l"])[0] for k in range(len(taps))]
+    H, W, C, esz = ref.base_shape()
+    assert esz == 2
+    base_h = np.zeros((n, H, W, C), dtype=np.int16)   # bf16 bits on the host
+    ref.materialize(tab.images, base_h)
+    base_d = torch.empty((n, H, W, C), dtype=torch.bfloat16, device="cuda")
+    ref.materialize(torch.from_numpy(tab.images).cuda(), base_d)
+    torch.cuda.synchronize()
+    assert np.array_equal(base_d.view(torch.int16).cpu().numpy(), base_h)
+    # the base layer's features from pixels == g(base): the materialised activation is A_{L[0]} itself
+    F0 = ref.features(0)["features"].to(torch.float64).cpu().numpy()
+    base64 = torch.from_numpy(base_h).view(torch.bfloat16).to(torch.float64).numpy().reshape(n, -1)
+    ref.close()
+    Ft, _ = oracle.features_from(cnn, WSEED, taps[0], base64, taps[1:])
+    Ft[taps[0]] = base64 if H == 1 else oracle.tap(base64.reshape(n, H, W, C))  # g = identity on FC layers
+    np.testing.assert_array_equal(F0, Ft[taps[0]])  # max is exact
+    for base in (base_h, base_d):
+        v = Vista(cnn, layers=taps, n_str_rows=len(tab.str_keys), d_s=d_s, n_images_local=n, iters=2,
+                  split_seed=SPLIT, weight_seed=WSEED, **kw)
+        v.transfer_from_base(base, tab.img_keys, tab.X, tab.str_keys, tab.labels)
+        for k in range(len(taps)):
+            f = v.features(k)
+            assert torch.equal(mm_ref[k], f["mm"].view(torch.int16).cpu()), k
+            np.testing.assert_array_equal(w_ref[k], v.train(k, d_s + f["d_l"])[0])
+            # partial inference from the stored base vs the oracle's f^_{L[0] -> L[k]} on the same base
+            Fg = f["features"].to(torch.float64).cpu().numpy()
+            assert normwise_rows(Fg, Ft[taps[k]]).max() <= 2e-2
+        v.close()
+
+
+def test_base_layer_needs_staged_plan():
+    tab = gen.make_tables(4, 8)
+    v = Vista(0, layers=[1, 2], n_str_rows=4, d_s=8, n_images_local=4, iters=2, split_seed=SPLIT,
+              weight_seed=WSEED, plan="eager")
+    H, W, C, _ = v.base_shape()
+    with pytest.raises(VistaError) as e:
+        v.transfer_from_base(np.zeros((4, H, W, C), np.int16), tab.img_keys, tab.X, tab.str_keys, tab.labels)
+    assert e.value.status == 1
+    v.close()

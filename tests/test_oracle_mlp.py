@@ -1,0 +1,145 @@
+"""Pins of the MLP oracle (oracle/mlp.py; "3-layer MLP (each hidden layer has 1024
+units) for 10 iterations"; reading R30) against things other than itself:
+central finite differences, torch autograd in fp64 (library), the W1 = W2 = 0 special case
+(scalar recursion of the bias), the descent property, and a world-2 gloo data-parallel run
+whose allreduced shard gradients equal the full-batch gradient."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+
+import gen
+from oracle import mlp
+
+rng = np.random.default_rng(7)
+
+
+def small_problem(n=9, d=6, h=5):
+    X = rng.standard_normal((n, d))
+    y = (rng.random(n) < 0.5).astype(np.uint8)
+    P = dict(W1=rng.standard_normal((h, d)) * 0.7, b1=rng.standard_normal(h) * 0.3,
+             W2=rng.standard_normal((h, h)) * 0.7, b2=rng.standard_normal(h) * 0.3,
+             w3=rng.standard_normal(h), b3=0.2)
+    return X, y, P
+
+
+def test_gradient_matches_central_differences():
+    X, y, P = small_problem()
+    _, g = mlp.loss_and_grad(P, X, y)
+    eps = 1e-6
+    for k in P:
+        if np.isscalar(P[k]):
+            Pp, Pm = dict(P), dict(P)
+            Pp[k], Pm[k] = P[k] + eps, P[k] - eps
+            fd = (mlp.loss_and_grad(Pp, X, y)[0] - mlp.loss_and_grad(Pm, X, y)[0]) / (2 * eps)
+            assert abs(fd - g[k]) <= 1e-7 * max(1.0, abs(fd))
+            continue
+        flat = P[k].reshape(-1)
+        for i in range(flat.size):
+            Pp = {kk: (v.copy() if not np.isscalar(v) else v) for kk, v in P.items()}
+            Pm = {kk: (v.copy() if not np.isscalar(v) else v) for kk, v in P.items()}
+            Pp[k].reshape(-1)[i] += eps
+            Pm[k].reshape(-1)[i] -= eps
+            fd = (mlp.loss_and_grad(Pp, X, y)[0] - mlp.loss_and_grad(Pm, X, y)[0]) / (2 * eps)
+            assert abs(fd - g[k].reshape(-1)[i]) <= 1e-7 * max(1.0, abs(fd)), (k, i)
+
+
+def test_gradient_matches_torch_autograd():
+    X, y, P = small_problem(n=40, d=12, h=16)
+    loss, g = mlp.loss_and_grad(P, X, y)
+    T = {k: torch.tensor(v, dtype=torch.float64, requires_grad=True) for k, v in P.items()}
+    Xt = torch.from_numpy(X)
+    h1 = torch.relu(Xt @ T["W1"].T + T["b1"])
+    h2 = torch.relu(h1 @ T["W2"].T + T["b2"])
+    z = h2 @ T["w3"] + T["b3"]
+    lt = torch.nn.functional.binary_cross_entropy_with_logits(z, torch.from_numpy(y.astype(np.float64)))
+    lt.backward()
+    assert abs(lt.item() - loss) <= 1e-12
+    for k in P:
+        np.testing.assert_allclose(np.asarray(g[k]), T[k].grad.numpy(), rtol=1e-10, atol=1e-13)
+
+
+def test_zero_hidden_weights_reduce_to_bias_recursion():
+    # W1 = W2 = 0, b1 = b2 = 0: h1 = h2 = 0, so only b3 moves: b3 <- b3 - lr (sigmoid(b3) - ybar)
+    n, d, h = 30, 4, 3
+    X = rng.standard_normal((n, d))
+    y = (rng.random(n) < 0.3).astype(np.uint8)
+    te = np.zeros(n, bool)
+    P0 = dict(W1=np.zeros((h, d)), b1=np.zeros(h), W2=np.zeros((h, h)), b2=np.zeros(h), w3=np.ones(h), b3=0.4)
+    P, losses, _ = mlp.train(X, y, te, seed=0, iters=6, lr=0.7, h=h, P0=P0)
+    b, ybar = 0.4, y.mean()
+    for t in range(6):
+        assert abs(losses[t] - (np.logaddexp(0, b) - ybar * b)) <= 1e-14
+        b = b - 0.7 * (1 / (1 + np.exp(-b)) - ybar)
+    assert abs(P["b3"] - b) <= 1e-14
+    np.testing.assert_array_equal(P["W1"], 0)
+    np.testing.assert_array_equal(P["w3"], 1)
+
+
+def test_descent_and_seeded_init():
+    n, d, h = 300, 20, 32
+    X = rng.standard_normal((n, d))
+    y = (X[:, 0] + 0.5 * rng.standard_normal(n) > 0).astype(np.uint8)
+    te = np.arange(n) % 5 == 0
+    P, losses, met = mlp.train(X, y, te, seed=5, iters=10, lr=0.1, h=h)
+    assert np.all(np.diff(losses) < 0)
+    assert met["n_train"] + met["n_test"] == n and met["tp"] + met["fp"] + met["tn"] + met["fn"] == met["n_test"]
+    P0 = mlp.init_params(5, d, h)
+    # bf16-representable, seeded, and the He / LeCun scales of reading R30
+    for k in ("W1", "W2", "w3"):
+        v = P0[k].astype(np.float32)
+        assert np.array_equal(v, torch.from_numpy(v).to(torch.bfloat16).float().numpy())
+    assert abs(P0["W1"].std() - np.sqrt(2 / d)) < 0.1 * np.sqrt(2 / d)
+    np.testing.assert_array_equal(P0["W2"], mlp.init_params(5, d, h)["W2"])
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def _dp_worker(rank, world, port, q):
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    r = np.random.default_rng(11)
+    X = r.standard_normal((50, 7))
+    y = (r.random(50) < 0.5).astype(np.uint8)
+    P = mlp.init_params(9, 7, 6)
+    lo, hi = [0, 21, 50][rank], [0, 21, 50][rank + 1]
+    # unnormalised gradient sums of this rank's rows = n_shard * mean gradient; allreduce; / n
+    _, g = mlp.loss_and_grad(P, X[lo:hi], y[lo:hi])
+    flat = np.concatenate([np.ravel(g[k]) * (hi - lo) for k in sorted(g)])
+    t = torch.from_numpy(flat.copy())
+    dist.all_reduce(t)
+    if rank == 0:
+        q.put(t.numpy() / 50)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.timeout(300)
+def test_two_rank_data_parallel_gradient_equals_full_batch():
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_dp_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    got = q.get(timeout=240)
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    r = np.random.default_rng(11)
+    X = r.standard_normal((50, 7))
+    y = (r.random(50) < 0.5).astype(np.uint8)
+    _, g = mlp.loss_and_grad(mlp.init_params(9, 7, 6), X, y)
+    ref = np.concatenate([np.ravel(g[k]) for k in sorted(g)])
+    np.testing.assert_allclose(got, ref, rtol=1e-12, atol=1e-15)

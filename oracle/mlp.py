@@ -10,12 +10,15 @@ distributed TF/Horovod" (§5.1 "Comparing against TF Transform+Bea
 reading R30, stated here step by step:
 
   x_p   = [X, F_l][p]                       the Eq. (4) row (d = d_s + d_l real columns)
-  h1_p  = ReLU(W1 x_p + b1)                 W1: [h, d]
+  x~_pj = (x_pj - mu_j) inv_j               z-scored with the train-row statistics of the LR reading
+                                            (O6 step 2: population sigma, inv_j = 0 if sigma_j <= 1e-12)
+  h1_p  = ReLU(W1 x~_p + b1)                W1: [h, d]
   h2_p  = ReLU(W2 h1_p + b2)                W2: [h, h]
   z_p   = w3 . h2_p + b3                    the third layer: one logit (binary label, as M = LR)
   loss  = (1/n) sum_p [log(1 + e^{z_p}) - y_p z_p]       mean over the n train rows
-  T full-batch gradient-descent steps  theta <- theta - lr * grad(loss)  (the "10 iterations";
-  full batch like the LR reading R17, so the result does not depend on the number of GPUs)
+  T full-batch gradient-descent steps  theta <- theta - lr * grad(loss), lr = 0.01 (the "10 iterations";
+  full batch like the LR reading R17, so the result does not depend on the number of GPUs; lr 0.1
+  diverged on the synthetic CNN features, whose z-scored covariance has lambda_max ~ 300-900)
   init: W1 ~ N(0, 2/d), W2 ~ N(0, 2/h), w3 ~ N(0, 1/h) (He / LeCun), biases 0, every value rounded
   to bf16 (both sides start from the same numbers); predict 1 iff z >= 0.
 
@@ -75,11 +78,23 @@ def loss_and_grad(P, X, y):
     return loss, g
 
 
-def train(X, y, is_test, seed: int, iters: int = 10, lr: float = 0.1, h: int = 1024, P0=None):
-    """T full-batch GD steps on the train rows, then metrics on the test rows (reading R30)."""
+def standardize(X, is_test):
+    """x~ = (x - mu) inv with mu, population sigma over the train rows; inv = 0 where sigma <= 1e-12."""
     X = np.asarray(X, dtype=np.float64)
-    y = np.asarray(y).astype(np.uint8)
+    tr = ~np.asarray(is_test).astype(bool)
+    mu = X[tr].mean(axis=0)
+    sig = np.sqrt(((X[tr] - mu) ** 2).mean(axis=0))
+    inv = np.zeros_like(sig)
+    keep = sig > 1e-12
+    inv[keep] = 1.0 / sig[keep]
+    return (X - mu) * inv
+
+
+def train(X, y, is_test, seed: int, iters: int = 10, lr: float = 0.01, h: int = 1024, P0=None):
+    """T full-batch GD steps on the (z-scored) train rows, then metrics on the test rows (reading R30)."""
     te = np.asarray(is_test).astype(bool)
+    X = standardize(X, te)
+    y = np.asarray(y).astype(np.uint8)
     Xtr, ytr = X[~te], y[~te]
     P = init_params(seed, X.shape[1], h) if P0 is None else {k: np.array(v, dtype=np.float64) if not np.isscalar(v)
                                                               else float(v) for k, v in P0.items()}

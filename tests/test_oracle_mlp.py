@@ -143,3 +143,14 @@ def test_two_rank_data_parallel_gradient_equals_full_batch():
     _, g = mlp.loss_and_grad(mlp.init_params(9, 7, 6), X, y)
     ref = np.concatenate([np.ravel(g[k]) for k in sorted(g)])
     np.testing.assert_allclose(got, ref, rtol=1e-12, atol=1e-15)
+
+
+def test_standardize_matches_lr_statistics():
+    # the MLP's z-scoring is O6 step 2: same mu / population sigma / inv as the C oracle's LR stats pass
+    import oracle
+    X = rng.standard_normal((60, 9)) * 3 + 1
+    X[:, 4] = 0.0   # dead (constant) column -> inv = 0
+    te = np.arange(60) % 5 == 0
+    mu, sig, inv = oracle.lr_stats(X, te.astype(np.uint8))
+    np.testing.assert_allclose(mlp.standardize(X, te), (X - mu) * inv, rtol=1e-13, atol=1e-13)
+    assert not mlp.standardize(X, te)[:, 4].any()

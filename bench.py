@@ -216,6 +216,9 @@ def main():
     ap.add_argument("--from-base", action="store_true",
                     help="App. B: materialise the first requested layer once (untimed, reported as materialize_s) "
                          "and time vista_transfer_from_base + train instead of the transfer from pixels")
+    ap.add_argument("--model", default="lr", choices=["lr", "mlp"],
+                    help="downstream model M per layer: lr (the product, PAPER.md:378) or the 3-layer MLP "
+                         "(PAPER.md:383, vista_train_mlp, 10 steps)")
     ap.add_argument("--plan", default="staged", choices=["staged", "eager", "lazy"],
                     help="logical plan (Fig 5): staged is the product; eager / lazy for config 4 comparisons")
     args = ap.parse_args()
@@ -289,7 +292,11 @@ def main():
             v.transfer(d_px, d_ik, d_X, d_sk, d_y)
         out = []
         for k in range(len(taps)):
-            out.append(v.train(k, d_tot[k]))
+            if args.model == "mlp":
+                P, met = v.train_mlp(k, d_tot[k], iters=10, seed=3, want_weights=host)
+                out.append((None, None, met))
+            else:
+                out.append(v.train(k, d_tot[k]))
         return out
 
     def barrier():
@@ -336,7 +343,8 @@ def main():
         e2e_step = e2e_ms / args.e2e_steps
     else:  # profiling runs only (no e2e number)
         e2e_ms, e2e_step = 0.0, float("nan")
-    d2h = sum((d + 1) * 8 for d in d_tot) + len(taps) * 8 * 80
+    d2h = (sum((d + 1) * 8 for d in d_tot) if args.model == "lr"
+           else sum(4 * (1024 * d + 3 * 1024 + 1024 * 1024 + 1) for d in d_tot)) + len(taps) * 8 * 80
     # ---- instrumented step: per-kernel-class device time (CUDA events on the launch stream) ----
     pk = peaks()
     tensor_peak = pk.get("bf16_tflops_sustained") if pk else None
@@ -394,6 +402,7 @@ def main():
             "data": "synthetic",
             "config": dict(workload_config(args.config, world, n_img), micro_batch=info["micro_batch"],
                            plan=args.plan + ("+prematerialized_base" if args.from_base else ""),
+                           model=("mlp_1024x1024x1_T10" if args.model == "mlp" else "elastic_net_lr_T%d" % T),
                            peak_bytes_pred=info["peak_bytes_pred"],
                            **({"base_layer": TAP_NAMES[cnn][taps[0]], "materialize_s": round(materialize_s, 3)}
                               if args.from_base else {})),

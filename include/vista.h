@@ -184,6 +184,27 @@ vista_status vista_transfer_from_base(vista_ctx* ctx, const void* base, const in
  *                d_s + d_l real columns, then the bias b. */
 vista_status vista_train(vista_ctx* ctx, int32_t k, double* weights_out, vista_metrics* out);
 
+/* ---- second downstream model M: 3-layer MLP ----
+ * "train a 3-layer MLP (each hidden layer has 1024 units) for 10 iterations using distributed
+ * TF/Horovod".  Reading R30: on the rows of MM_k (the d = d_s + d_l real
+ * columns, z-scored with the train statistics of O6 step 2), h1 = ReLU(W1 x + b1), h2 = ReLU(W2 h1 + b2), z = w3 . h2 + b3, mean logistic loss over the
+ * train rows, `iters` full-batch gradient-descent steps of size `lr`; initial W1 ~ N(0, 2/d),
+ * W2 ~ N(0, 2/h), w3 ~ N(0, 1/h) drawn by the seeded generator (model id 3) and rounded to bf16, biases 0.
+ * GEMMs on the tcgen05 tensor cores (bf16 operands, fp32 accumulation), fp32 master weights; data
+ * parallel over ranks: one fp32 NCCL allreduce of the gradient sums per step.  Collective (all ranks,
+ * same k and cfg).  weights_out (caller-owned, may be NULL): float[h*d + h + h*h + h + h + 1] =
+ * W1 [h][d], b1, W2 [h][h], b2, w3, b3.  metrics: loss[t] before step t, train/test accuracy, F1,
+ * eta = lr.  Errors: VISTA_ERR_STATE before vista_transfer, VISTA_ERR_INVALID_ARG for hidden != 1024
+ * or the fp32 check mode. */
+typedef struct {
+  int32_t hidden;  /* units per hidden layer, 1024; 0 = 1024 */
+  int32_t iters;   /* gradient steps, 10; 0 = 10 */
+  double lr;       /* step size; 0 = 0.01 */
+  uint64_t seed;   /* initial-weight seed */
+} vista_mlp_cfg;
+vista_status vista_train_mlp(vista_ctx* ctx, int32_t k, const vista_mlp_cfg* cfg, float* weights_out,
+                             vista_metrics* out);
+
 void vista_destroy(vista_ctx* ctx);
 const char* vista_status_str(vista_status s);
 const char* vista_last_error(const vista_ctx* ctx);
@@ -208,7 +229,8 @@ typedef struct {
   double flops[8];
   double bytes[8];
   double roof_ms[8];
-} vista_profile;
+} vista_profile;  /* classes: 0 conv/FC/GEMM (tcgen05), 1 tap, 2 pool/convert/LRN, 3 join, 4 concat, 5 LR pass,
+                     6 LR small, 7 MLP (its tcgen05 GEMMs, transposes, head, update) */
 vista_status vista_set_profiling(vista_ctx* ctx, int32_t on);
 /* Peaks for vista_profile.roof_ms: dense tensor TFLOP/s and HBM GB/s (e.g. MEASURED_PEAKS.json). */
 vista_status vista_set_roofline(vista_ctx* ctx, double tflops, double gbps);

@@ -119,3 +119,60 @@ def train(X, y, is_test, seed: int, iters: int = 10, lr: float = 0.01, h: int = 
                test_f1=100.0 * 2 * tp / (2 * tp + fp + fn) if (2 * tp + fp + fn) else 0.0,
                tp=tp, fp=fp, tn=tn, fn=fn, n_train=int(len(ytr)), n_test=n_te)
     return P, np.array(losses), met
+
+
+def _bf16(a):
+    """Round to the nearest bf16 (RNE) through fp32, returned as fp64."""
+    import torch
+    return torch.from_numpy(np.asarray(a, dtype=np.float32)).to(torch.bfloat16).to(torch.float64).numpy()
+
+
+def train_bf16_emulated(X, y, is_test, seed: int, iters: int = 10, lr: float = 0.01, h: int = 1024):
+    """DIAGNOSTIC comparator (SURVEY.md §8c c.5 / reading R24 "bf16-emulation mode"), not the definition:
+    the same algorithm as train() with the values rounded to bf16 at the points where the B200 path
+    stores bf16 (the first layer takes the raw rows with the z-scoring folded into W1' = bf16(W1 diag(inv)),
+    b1' = b1 - W1' mu; H1, H2, bf16(W2), dH2, dH2 W2 rounded), everything else in fp64.  It separates
+    kernel bugs from bf16 precision drift: the MLP's full-batch gradient at initialisation is a small
+    residual of large per-row terms, so 2^-9 roundings of H1 move it by a few percent (measured)."""
+    X = np.asarray(X, dtype=np.float64)
+    te = np.asarray(is_test).astype(bool)
+    y = np.asarray(y).astype(np.uint8)
+    tr = ~te
+    mu = X[tr].mean(axis=0)
+    sig = np.sqrt(((X[tr] - mu) ** 2).mean(axis=0))
+    inv = np.zeros_like(sig)
+    inv[sig > 1e-12] = 1.0 / sig[sig > 1e-12]
+    Xtr, ytr = X[tr], y[tr].astype(np.float64)
+    n = Xtr.shape[0]
+    P = init_params(seed, X.shape[1], h)
+    losses = []
+
+    def fwd(Xr):
+        W1b = _bf16(P["W1"] * inv)
+        b1p = P["b1"] - W1b @ mu
+        h1 = _bf16(np.maximum(Xr @ W1b.T + b1p, 0.0))
+        h2 = _bf16(np.maximum(h1 @ _bf16(P["W2"]).T + P["b2"], 0.0))
+        return h1, h2, h2 @ P["w3"] + P["b3"]
+
+    for _ in range(iters):
+        h1, h2, z = fwd(Xtr)
+        losses.append(float(np.mean(_softplus(z) - ytr * z)))
+        dz = (_sigmoid(z) - ytr) / n
+        dh2 = _bf16(np.outer(dz, P["w3"]) * (h2 > 0))
+        dh1 = _bf16(dh2 @ _bf16(P["W2"])) * (h1 > 0)
+        g = dict(w3=h2.T @ dz, b3=float(dz.sum()), W2=dh2.T @ h1, b2=dh2.sum(axis=0), b1=dh1.sum(axis=0))
+        g["W1"] = (dh1.T @ Xtr - np.outer(g["b1"], mu)) * inv
+        for k in P:
+            P[k] = P[k] - lr * g[k]
+    _, _, z_all = fwd(X)
+    pred = z_all >= 0
+    yb = y.astype(bool)
+    tp = int((pred & yb & te).sum())
+    fp = int((pred & ~yb & te).sum())
+    fn = int((~pred & yb & te).sum())
+    tn = int((~pred & ~yb & te).sum())
+    n_te = int(te.sum())
+    met = dict(train_acc=100.0 * float((pred[tr] == yb[tr]).mean()) if tr.any() else 0.0,
+               test_acc=100.0 * (tp + tn) / n_te if n_te else 0.0, tp=tp, fp=fp, tn=tn, fn=fn,
+               n_train=int(tr.sum()), n_test=n_te)
+    return P, np.array(losses), met

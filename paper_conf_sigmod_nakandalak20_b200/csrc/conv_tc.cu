@@ -60,6 +60,7 @@ struct ConvParams {
   // fused tap g_l (PAPER.md:369 fn 4): per-image 2x2-grid channel maxima of the (post-ReLU, >= 0)
   // output, accumulated as fp32 bit patterns with red.global.max.u32 into tapf[n][4][Cout]
   unsigned int* tapf;
+  int out_f32;  // register epilogue writes fp32 (gemm_tn: weight gradients of the MLP head)
 };
 
 constexpr int BM = 128, BK = 64;
@@ -143,6 +144,19 @@ __device__ __forceinline__ void epi_math(const uint32_t* v, const float* scv, co
   o.y = pack_bf16x2(f[2], f[3]);
   o.z = pack_bf16x2(f[4], f[5]);
   o.w = pack_bf16x2(f[6], f[7]);
+}
+
+__device__ __forceinline__ void epi_math_f32(const uint32_t* v, const float* scv, const float* shv, bool relu,
+                                             float* out) {
+  float f[8];
+#pragma unroll
+  for (int j = 0; j < 8; ++j) f[j] = fmaf(__uint_as_float(v[j]), scv[j], shv[j]);
+  if (relu) {
+#pragma unroll
+    for (int j = 0; j < 8; ++j) f[j] = fmaxf(f[j], 0.0f);
+  }
+  reinterpret_cast<float4*>(out)[0] = make_float4(f[0], f[1], f[2], f[3]);
+  reinterpret_cast<float4*>(out)[1] = make_float4(f[4], f[5], f[6], f[7]);
 }
 
 template <int BN, int AMODE, bool TMA_EPI, int NB, int RKB>
@@ -634,9 +648,14 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
             for (int qq = 0; qq < 4; ++qq) {
               if (cb * 32 + qq * 8 < nvalid_tile) {
-                uint4 o;
-                epi_math(v + qq * 8, scv + qq * 8, shv + qq * 8, has_res, cur[qq], p.relu, o);
-                *reinterpret_cast<uint4*>(p.y + off + cb * 32 + qq * 8) = o;
+                if (p.out_f32) {
+                  epi_math_f32(v + qq * 8, scv + qq * 8, shv + qq * 8, p.relu,
+                               reinterpret_cast<float*>(p.y) + off + cb * 32 + qq * 8);
+                } else {
+                  uint4 o;
+                  epi_math(v + qq * 8, scv + qq * 8, shv + qq * 8, has_res, cur[qq], p.relu, o);
+                  *reinterpret_cast<uint4*>(p.y + off + cb * 32 + qq * 8) = o;
+                }
               }
             }
           }
@@ -1097,6 +1116,63 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
              res ? " res" : "");
   prof_end(st, 0, flops, bytes, label);
   return tapf == nullptr || fuse_tap;
+}
+
+// Plain "TN" GEMM on the same kernel (A_TMA mode, register epilogue):
+//   y[m, n] = act(scale[n] * sum_k A[m, k] B[n, k] + shift[n]),  m < M, n < N, k < K
+// A: bf16 [M rows, lda], B: bf16 [N rows, ldb] (both K-major, rows 16-byte aligned); columns k >= K
+// (and B rows >= N) are read as zeros by the TMA, so K needs no padding.  y: [M, N] row-major, bf16 or
+// fp32 (out_f32).  scale / shift: fp32 device [N] (per output column).
+void gemm_tn(const bf16* A, int64_t M, int K, int lda, const bf16* B, int N, int ldb, const float* scale,
+             const float* shift, bool relu, void* y, bool out_f32, cudaStream_t st, int prof_cls) {
+  if (M <= 0 || N <= 0) return;
+  if (K <= 0 || (lda % 8) || (ldb % 8) || (N % 8)) fail(1, "gemm_tn: K > 0, lda, ldb, N multiples of 8 required");
+  if (M > INT32_MAX - BM) fail(1, "gemm_tn: M too large");
+  ConvLayer L;
+  L.Cin = L.Cg_in = L.K = K;
+  L.Cout = L.Cg_out = N;
+  L.Kp = (K + BK - 1) / BK * BK;
+  L.K_alg = K;
+  L.BN = N % 256 == 0 ? 256 : (N % 128 == 0 ? 128 : (N >= 256 ? 256 : 128));
+  {
+    const cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)N};
+    const cuuint64_t strides[1] = {(cuuint64_t)ldb * 2};
+    const cuuint32_t box[2] = {(cuuint32_t)BK, (cuuint32_t)L.BN};
+    if (encode_nd(&L.tmap_w, B, 2, dims, strides, box) != CUDA_SUCCESS) fail(5, "gemm_tn: B tensor map");
+  }
+  CUtensorMap ta;
+  {
+    const cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)M};
+    const cuuint64_t strides[1] = {(cuuint64_t)lda * 2};
+    const cuuint32_t box[2] = {(cuuint32_t)BK, (cuuint32_t)BM};
+    if (encode_nd(&ta, A, 2, dims, strides, box) != CUDA_SUCCESS) fail(5, "gemm_tn: A tensor map");
+  }
+  ConvParams p{};
+  p.x = A;
+  p.y = reinterpret_cast<bf16*>(y);
+  p.scale = scale;
+  p.shift = shift;
+  p.H = p.W = p.Ho = p.Wo = 1;
+  p.Cin = K;
+  p.Cout = N;
+  p.R = p.S = p.stride = 1;
+  p.Cg_in = K;
+  p.Cg_out = N;
+  p.K = K;
+  p.nkb = L.Kp / BK;
+  p.M = (int)M;
+  p.relu = relu ? 1 : 0;
+  p.out_f32 = out_f32 ? 1 : 0;
+  p.n_mt = (p.M + BM - 1) / BM;
+  p.n_nt = (N + L.BN - 1) / L.BN;
+  p.n_tiles = p.n_mt * p.n_nt;
+  prof_begin(st);
+  if (L.BN == 256) launch_bn<256, false, 1>(L, A_TMA, ta, ta, ta, p, st, 0);
+  else launch_bn<128, false, 1>(L, A_TMA, ta, ta, ta, p, st, 0);
+  char label[96] = {0};
+  if (prof_labels()) snprintf(label, sizeof(label), "gemm_tn M%lld N%d K%d%s", (long long)M, N, K, out_f32 ? " f32" : "");
+  prof_end(st, prof_cls, 2.0 * (double)M * N * K,
+           2.0 * ((double)M * K + (double)N * K) + (double)M * N * (out_f32 ? 4 : 2), label);
 }
 
 }  // namespace vista

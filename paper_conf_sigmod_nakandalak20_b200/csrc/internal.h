@@ -138,6 +138,23 @@ LRResult lr_train_f32(const float* MM, const uint8_t* y, int64_t n_rows, int64_t
                       const uint8_t* real_col_mask_host, int iters, int power_iters, double lambda, double alpha,
                       allreduce_fn allreduce, void* ar_user, cudaStream_t st);
 
+// ---- second downstream model: 3-layer MLP (reading R30), mlp.cu ----
+typedef void (*allreduce_f32_fn)(float* d_buf, int64_t count, cudaStream_t st, void* user);
+struct MLPResult {
+  std::vector<double> loss;            // mean train loss before each of the T steps
+  std::vector<float> W1, b1, W2, b2, w3;  // final weights; W1 [h][d] over the real columns
+  float b3 = 0;
+  int64_t n_train = 0, n_test = 0, tp = 0, fp = 0, tn = 0, fn = 0, train_ok = 0;
+};
+// gemm on the tcgen05 kernel (conv_tc.cu): y[m, n] = act(scale[n] * sum_k A[m, k] B[n, k] + shift[n])
+void gemm_tn(const bf16* A, int64_t M, int K, int lda, const bf16* B, int N, int ldb, const float* scale,
+             const float* shift, bool relu, void* y, bool out_f32, cudaStream_t st, int prof_cls);
+// W1p_0 / W2_0 / w3_0: device fp32 initial weights (W1 in the padded [h][roundup(ld, 64)] column layout of MM_k)
+MLPResult mlp_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
+                    const std::vector<int>& real_cols, const float* W1p_0, const float* W2_0, const float* w3_0,
+                    int h, int iters, double lr, bool want_weights, allreduce_fn ar64, allreduce_f32_fn ar32,
+                    void* ar_user, cudaStream_t st);
+
 // ---- profiling hooks (class ids as in vista.h vista_profile) ----
 struct Profiler;
 extern thread_local Profiler* g_prof;

@@ -149,6 +149,12 @@ static void nccl_allreduce_f64(double* buf, int64_t count, cudaStream_t st, void
   if (rc != 0) fail(6, std::string("ncclAllReduce: ") + (n.GetErrorString ? n.GetErrorString(rc) : "error"));
 }
 
+static void nccl_allreduce_f32(float* buf, int64_t count, cudaStream_t st, void* user) {
+  Nccl& n = nccl_lib();
+  const int rc = n.AllReduce(buf, buf, (size_t)count, /*ncclFloat32*/ 7, /*ncclSum*/ 0, user, st);
+  if (rc != 0) fail(6, std::string("ncclAllReduce: ") + (n.GetErrorString ? n.GetErrorString(rc) : "error"));
+}
+
 // ---------------- helpers ----------------
 static uint16_t f2bf_bits(float f) {  // f is bf16-representable (generator contract)
   uint32_t u;
@@ -238,6 +244,15 @@ struct vista_ctx {
   // closing 1x1 conv + next unit's opening 1x1 conv (res_chain.cu, bit-identical); VISTA_FUSE_CHAIN=0 disables
   bool fuse_chain = true;
   std::vector<void*> feat;  // per block: device pointer of F_t (features) of a tapped layer
+  // seeded initial MLP weights per requested layer (host, generated on first use: model init, like the
+  // CNN weights of vista_plan)
+  struct MlpInit {
+    bool valid = false;
+    uint64_t seed = 0;
+    int h = 0;
+    std::unique_ptr<DevBuf> dev;  // fp32 [W1 padded h x Kp | W2 h x h | w3 h]
+  };
+  std::vector<MlpInit> mlp_init;
   std::string last_error;
   ~vista_ctx() {
     for (auto* v : {&F, &MM, &Y, &slot_store})
@@ -246,6 +261,8 @@ struct vista_ctx {
     arena[0].release();
     arena[1].release();
     tapacc.release();
+    for (auto& mi : mlp_init)
+      if (mi.dev) mi.dev->release();
     for (DevBuf* b : {&pair_str, &pair_img, &d_X, &d_labels, &d_img_keys, &d_str_keys, &d_px}) b->release();
     if (stream) cudaStreamSynchronize(stream);
     for (auto& L : convs) conv_layer_free(L);
@@ -1055,6 +1072,90 @@ VISTA_API vista_status vista_train(vista_ctx* c, int32_t k, double* weights_out,
       for (int i = 0; i < (int)r.loss.size() && i < 64; ++i) m->loss[i] = r.loss[i];
       m->lambda_hat = r.lambda_hat;
       m->eta = r.eta;
+      m->n_train = r.n_train;
+      m->n_test = r.n_test;
+      m->tp = r.tp;
+      m->fp = r.fp;
+      m->tn = r.tn;
+      m->fn = r.fn;
+      m->train_acc = r.n_train ? 100.0 * r.train_ok / r.n_train : 0.0;
+      m->test_acc = r.n_test ? 100.0 * (r.tp + r.tn) / r.n_test : 0.0;
+      const int64_t den = 2 * r.tp + r.fp + r.fn;
+      m->test_f1 = den ? 100.0 * 2.0 * r.tp / den : 0.0;
+    }
+  });
+}
+
+// Second downstream model: the 3-layer MLP of PAPER.md:383 on MM_k (reading R30).
+VISTA_API vista_status vista_train_mlp(vista_ctx* c, int32_t k, const vista_mlp_cfg* cfg, float* weights_out,
+                                       vista_metrics* m) {
+  if (!c) return VISTA_ERR_INVALID_ARG;
+  if (!c->transferred) {
+    c->last_error = "vista_train_mlp before vista_transfer";
+    return VISTA_ERR_STATE;
+  }
+  return guarded(c, [&] {
+    if (k < 0 || k >= (int)c->taps.size()) fail(1, "layer index out of range");
+    if (c->f32) fail(1, "vista_train_mlp: the MLP runs on the bf16 path only");
+    const int h = cfg && cfg->hidden > 0 ? cfg->hidden : 1024;
+    const int iters = cfg && cfg->iters > 0 ? cfg->iters : 10;
+    const double lr = cfg && cfg->lr > 0 ? cfg->lr : 0.01;
+    const uint64_t seed = cfg ? cfg->seed : 0;
+    VCHECK(cudaSetDevice(c->sys.device));
+    const int t = c->taps[k];
+    const int d_l = c->net.stages[t].d_tap;
+    const int ld = ld_of(c, k);
+    const int d = c->d_s + d_l;
+    std::vector<int> real;
+    for (int j = 0; j < c->d_s; ++j) real.push_back(j);
+    for (int j = 0; j < d_l; ++j) real.push_back(c->ds_pad + j);
+    // seeded bf16-valued initial weights (generator model id 3, reading R30): W1 ~ N(0, 2/d), W2 ~ N(0, 2/h),
+    // w3 ~ N(0, 1/h); the same numbers the oracle draws
+    if (c->mlp_init.size() < c->taps.size()) c->mlp_init.resize(c->taps.size());
+    vista_ctx::MlpInit& mi = c->mlp_init[k];
+    const int Kp = (ld + 63) / 64 * 64;
+    const size_t nW1 = (size_t)h * Kp, nW2 = (size_t)h * h;
+    if (!mi.valid || mi.seed != seed || mi.h != h) {
+      std::vector<float> W1((size_t)h * d), all(nW1 + nW2 + h, 0.f);
+      vg_param_f32(seed, 3, 0, VG_T_WEIGHT, (int64_t)h * d, 0, 0.0, std::sqrt(2.0 / d), W1.data());
+      vg_param_f32(seed, 3, 1, VG_T_WEIGHT, (int64_t)h * h, 0, 0.0, std::sqrt(2.0 / h), all.data() + nW1);
+      vg_param_f32(seed, 3, 2, VG_T_WEIGHT, h, 0, 0.0, std::sqrt(1.0 / h), all.data() + nW1 + nW2);
+      for (int o = 0; o < h; ++o)  // W1 in the padded column layout of MM_k
+        for (int j = 0; j < d; ++j) all[(size_t)o * Kp + real[j]] = W1[(size_t)o * d + j];
+      if (!mi.dev) mi.dev.reset(new DevBuf());
+      mi.dev->ensure(all.size() * 4);
+      VCHECK(cudaMemcpyAsync(mi.dev->p, all.data(), all.size() * 4, cudaMemcpyHostToDevice, c->stream));
+      VCHECK(cudaStreamSynchronize(c->stream));
+      mi.seed = seed;
+      mi.h = h;
+      mi.valid = true;
+    }
+    const float* W1 = (const float*)mi.dev->p;
+    const float* W2 = W1 + nW1;
+    const float* w3 = W2 + nW2;
+    const bool multi = c->sys.world > 1;
+    MLPResult r = mlp_train((const bf16*)c->MM[k]->p, (const uint8_t*)c->Y[k]->p, c->n_pairs, c->n_train, ld, real,
+                            W1, W2, w3, h, iters, lr, weights_out != nullptr, multi ? nccl_allreduce_f64 : nullptr,
+                            multi ? nccl_allreduce_f32 : nullptr, c->nccl_comm, c->stream);
+    if (g_prof) g_prof->flush();
+    if (weights_out) {
+      float* o = weights_out;
+      std::memcpy(o, r.W1.data(), r.W1.size() * 4);
+      o += r.W1.size();
+      std::memcpy(o, r.b1.data(), h * 4);
+      o += h;
+      std::memcpy(o, r.W2.data(), r.W2.size() * 4);
+      o += r.W2.size();
+      std::memcpy(o, r.b2.data(), h * 4);
+      o += h;
+      std::memcpy(o, r.w3.data(), h * 4);
+      o += h;
+      *o = r.b3;
+    }
+    if (m) {
+      std::memset(m, 0, sizeof(*m));
+      for (int i = 0; i < (int)r.loss.size() && i < 64; ++i) m->loss[i] = r.loss[i];
+      m->eta = lr;
       m->n_train = r.n_train;
       m->n_test = r.n_test;
       m->tp = r.tp;

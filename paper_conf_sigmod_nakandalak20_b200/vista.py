@@ -63,7 +63,11 @@ class Profile(ctypes.Structure):
                 ("roof_ms", _f64 * 8)]
 
 
-PROFILE_CLASSES = ["conv_fc_tcgen05", "tap", "pool_cvt_lrn", "join", "concat", "lr_pass", "lr_small"]
+PROFILE_CLASSES = ["conv_fc_tcgen05", "tap", "pool_cvt_lrn", "join", "concat", "lr_pass", "lr_small", "mlp"]
+
+
+class MLPCfg(ctypes.Structure):
+    _fields_ = [("hidden", _i32), ("iters", _i32), ("lr", _f64), ("seed", _u64)]
 
 
 def lib():
@@ -81,6 +85,7 @@ def lib():
         L.vista_plan_info.argtypes = [_vp, ctypes.POINTER(PlanInfo)]
         L.vista_transfer.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp]
         L.vista_features.argtypes = [_vp, _i32, ctypes.POINTER(Buffer)]
+        L.vista_train_mlp.argtypes = [_vp, _i32, ctypes.POINTER(MLPCfg), _vp, ctypes.POINTER(Metrics)]
         L.vista_base_shape.argtypes = [_vp, ctypes.POINTER(_i64)]
         L.vista_materialize.argtypes = [_vp, _vp, _vp]
         L.vista_transfer_from_base.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp]
@@ -314,6 +319,27 @@ class Vista:
                    test_acc=m.test_acc, test_f1=m.test_f1, n_train=m.n_train, n_test=m.n_test, tp=m.tp, fp=m.fp,
                    tn=m.tn, fn=m.fn)
         return w[:-1], float(w[-1]), met
+
+    def train_mlp(self, k, d_total, iters=10, lr=0.01, seed=0, hidden=1024, want_weights=True):
+        """3-layer MLP (reading R30) on layer k; returns (params dict or None, metrics)."""
+        h, d = hidden, d_total
+        w = np.zeros(h * d + h + h * h + h + h + 1, dtype=np.float32) if want_weights else None
+        m = Metrics()
+        cfg = MLPCfg(hidden, iters, lr, seed)
+        _check(lib().vista_train_mlp(self.ctx, k, ctypes.byref(cfg), w.ctypes.data if want_weights else None,
+                                     ctypes.byref(m)), self.ctx)
+        met = dict(loss=list(m.loss[:iters]), train_acc=m.train_acc, test_acc=m.test_acc, test_f1=m.test_f1,
+                   n_train=m.n_train, n_test=m.n_test, tp=m.tp, fp=m.fp, tn=m.tn, fn=m.fn, lr=m.eta)
+        if not want_weights:
+            return None, met
+        o = 0
+        P = {}
+        for name, shape in (("W1", (h, d)), ("b1", (h,)), ("W2", (h, h)), ("b2", (h,)), ("w3", (h,))):
+            size = int(np.prod(shape))
+            P[name] = w[o:o + size].reshape(shape).astype(np.float64)
+            o += size
+        P["b3"] = float(w[o])
+        return P, met
 
     def set_profiling(self, on: bool):
         _check(lib().vista_set_profiling(self.ctx, 1 if on else 0), self.ctx)

@@ -154,3 +154,20 @@ def test_standardize_matches_lr_statistics():
     mu, sig, inv = oracle.lr_stats(X, te.astype(np.uint8))
     np.testing.assert_allclose(mlp.standardize(X, te), (X - mu) * inv, rtol=1e-13, atol=1e-13)
     assert not mlp.standardize(X, te)[:, 4].any()
+
+
+def test_bf16_emulation_is_the_definition_up_to_rounding():
+    # the diagnostic comparator differs from the fp64 definition only by the bf16 roundings: with the
+    # rounding made the identity it must reproduce train() exactly (same algorithm, folded first layer)
+    import unittest.mock as um
+    n, d, h = 120, 10, 16
+    X = np.abs(rng.standard_normal((n, d)))
+    y = (rng.random(n) < 0.5).astype(np.uint8)
+    te = np.arange(n) % 5 == 0
+    R, L, m = mlp.train(X, y, te, seed=3, iters=4, lr=0.05, h=h)
+    with um.patch.object(mlp, "_bf16", lambda a: np.asarray(a, dtype=np.float64)):
+        E, LE, me = mlp.train_bf16_emulated(X, y, te, seed=3, iters=4, lr=0.05, h=h)
+    np.testing.assert_allclose(LE, L, rtol=1e-12)
+    for k in ("W1", "W2", "w3", "b1", "b2"):
+        np.testing.assert_allclose(E[k], R[k], rtol=1e-9, atol=1e-12)
+    assert me["test_acc"] == m["test_acc"] and me["train_acc"] == m["train_acc"]

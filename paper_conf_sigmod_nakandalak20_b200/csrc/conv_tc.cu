@@ -57,10 +57,18 @@ struct ConvParams {
   int H, W, Cin, Ho, Wo, Cout, R, S, stride, pad, Cg_in, Cg_out, K, nkb, M, relu;
   int n_mt, n_nt, n_tiles;
   int Wp, hrows, hsz, mt_per_img, cblocks;  // A_HALO geometry (see above)
+  // A_HALO: per k-block offset of the A operand inside the halo buffer, in 16-byte descriptor units:
+  // ((r*Wp + s) * 128 + cb * hsz) >> 4 for kb = (r*3 + s) * cblocks + cb.  Precomputed so that the MMA
+  // issue loop has no integer division (measured: the per-k-block division chain made the issue latency
+  // ~340 cycles, longer than the 4 MMAs it feeds)
+  int koff[36];
   // fused tap g_l (PAPER.md:369 fn 4): per-image 2x2-grid channel maxima of the (post-ReLU, >= 0)
   // output, accumulated as fp32 bit patterns with red.global.max.u32 into tapf[n][4][Cout]
   unsigned int* tapf;
   int out_f32;  // register epilogue writes fp32 (gemm_tn: weight gradients of the MLP head)
+  unsigned long long* dbg_buf;  // (dbg & 8): per-CTA cycle counters of the MMA warp [grid][8]
+  int dbg;      // VISTA_CONV_DBG bit mask (measurement experiments only; results wrong when set): 1 = halo loaded
+                // once, 2 = epilogue only waits / releases the accumulator, 8 = MMA-warp cycle counters (halo)
 };
 
 constexpr int BM = 128, BK = 64;
@@ -92,19 +100,24 @@ struct Cfg {
   static constexpr int kOutBytes = kOutBufs * BM * BN * 2;
   // TMA epilogue: one scale/shift buffer (a named barrier separates tiles); register epilogue: two
   static constexpr int kSbufBytes = (TMA_EPI ? 1 : 2) * 2 * BN * 4;
+  // register epilogue with BN <= 128: four TMEM accumulators, and the two epilogue warp groups take
+  // alternate tiles (each group drains all BN columns of its tiles), so two tiles' epilogues overlap
+  static constexpr bool kSplit = !TMA_EPI && BN <= 128;
+  // BN = 64 register epilogue: each warp stages its 32 rows x 32 columns in smem and writes them back with
+  // 4 rows per instruction (per-row 16-byte stores touched 32 lines per instruction: LSU-bound, measured)
+  static constexpr bool kStaged = kSplit && BN == 64;
+  static constexpr int kStgBytes = kStaged ? kEpiWarps * 32 * 64 : 0;
   static constexpr int kNBar = 20;  // tfull/tempty[4], rbar[4], hfull/hempty[3], wres[1], slack
-  static constexpr int kFixed = kHaloBytes + kResBytes + kOutBytes + kSbufBytes + 1024 + 16 + kNBar * 8;
+  static constexpr int kFixed = kHaloBytes + kResBytes + kOutBytes + kSbufBytes + kStgBytes + 1024 + 16 + kNBar * 8;
   static constexpr int kStagesFit = kStageBytes ? (227 * 1024 - kFixed) / (kStageBytes + 16) : 2;
   static constexpr int kStages = kStagesFit > 8 ? 8 : kStagesFit;
   static constexpr int kResOff = kStages * kStageBytes;
   static constexpr int kHaloOff = kResOff + kResBytes;
   static constexpr int kOutOff = kHaloOff + kHaloBytes;
   static constexpr int kSbufOff = kOutOff + kOutBytes;
-  static constexpr int kBarOff = kSbufOff + kSbufBytes;
+  static constexpr int kStgOff = kSbufOff + kSbufBytes;
+  static constexpr int kBarOff = kStgOff + kStgBytes;
   static constexpr int kBytes = kBarOff + (2 * kStages + kNBar) * 8 + 16 + 1024;  // + alignment slack
-  // register epilogue with BN <= 128: four TMEM accumulators, and the two epilogue warp groups take
-  // alternate tiles (each group drains all BN columns of its tiles), so two tiles' epilogues overlap
-  static constexpr bool kSplit = !TMA_EPI && BN <= 128;
   static constexpr int kAcc = kSplit ? 4 : 2;
   static constexpr int kTmemCols = kAcc * BN;
   static_assert(kStages >= 2, "shared memory too small for two k-block stages");
@@ -255,9 +268,14 @@ __global__ void __launch_bounds__(kThreads, 1)
           const int prow0 = p0 / p.Wp;  // first padded input row (input row prow0 - 1)
           const uint32_t hb = it % HB;
           if (it >= (uint32_t)HB) mbar_wait(&hempty[hb], ((it / HB) - 1) & 1);
-          mbar_arrive_expect_tx(&hfull[hb], box_bytes * p.cblocks);
-          for (int cb = 0; cb < p.cblocks; ++cb)
-            tma_load_4d(sH + hb * halo_half_bytes(BN) + cb * p.hsz, &tmap_a, cb * BK, -1, prow0 - 1, nimg, &hfull[hb]);
+          if ((p.dbg & 1) && it >= (uint32_t)HB) {
+            mbar_arrive(&hfull[hb]);
+          } else {
+            mbar_arrive_expect_tx(&hfull[hb], box_bytes * p.cblocks);
+            for (int cb = 0; cb < p.cblocks; ++cb)
+              tma_load_4d(sH + hb * halo_half_bytes(BN) + cb * p.hsz, &tmap_a, cb * BK, -1, prow0 - 1, nimg,
+                          &hfull[hb]);
+          }
           if constexpr (!BRES) {  // streamed weights (resident: nothing else per tile)
             for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
               const int stage = gk % S;
@@ -447,14 +465,80 @@ __global__ void __launch_bounds__(kThreads, 1)
     {
       constexpr uint32_t idesc = umma_idesc_bf16(BM, BN);
       uint32_t gk = 0, it = 0;
+      long long c_te = 0, c_dec = 0, c_hf = 0, c_iss = 0, tA = 0, tB = 0;
+      const bool prof_mma = (p.dbg & 8) && lane == 0;
       if constexpr (BRES) mbar_wait(wres, 0);
+      const long long t_start = prof_mma ? clock64() : 0;
+      if constexpr (AMODE == A_HALO && BRES) {
+        // Resident weights + halo (Cout = 64): tiles are issued in PAIRS, so the per-tile waits, tile
+        // decode and commits sit between pairs, not between every 36 MMAs (measured: the tensor queue drains
+        // during that gap; issue-bound at 2620 cycles per 1728-cycle tile).  The producer and the epilogue
+        // still work per tile.
+        for (int tile = blockIdx.x; tile < p.n_tiles; tile += 2 * gridDim.x, it += 2) {
+          const int tiles[2] = {tile, tile + (int)gridDim.x};
+          const int nt2 = tiles[1] < p.n_tiles ? 2 : 1;
+          uint32_t alo[2], accs[2], hbs[2];
+          if (prof_mma) tA = clock64();
+#pragma unroll
+          for (int j = 0; j < 2; ++j) {
+            if (j < nt2) {
+              const uint32_t itj = it + j;
+              accs[j] = itj % NACC;
+              hbs[j] = itj % HB;
+              if (itj >= (uint32_t)NACC) mbar_wait(&tempty[accs[j]], ((itj / NACC) - 1) & 1);
+              const int pimg = (tiles[j] % p.mt_per_img) * BM;  // one N tile: tile index = M-tile index
+              alo[j] = umma_desc_lo_sw128(sH + hbs[j] * halo_half_bytes(BN) + (pimg % p.Wp) * 128);
+            }
+          }
+          if (prof_mma) {
+            tB = clock64();
+            c_te += tB - tA;
+            tA = tB;
+          }
+#pragma unroll
+          for (int j = 0; j < 2; ++j)
+            if (j < nt2) mbar_wait(&hfull[hbs[j]], ((it + j) / HB) & 1);
+          tc_fence_after();
+          if (prof_mma) {
+            tB = clock64();
+            c_hf += tB - tA;
+            tA = tB;
+          }
+          const uint32_t blo = umma_desc_lo_sw128(sR);
+#pragma unroll
+          for (int j = 0; j < 2; ++j) {
+            if (j < nt2) {
+              const uint32_t tacc = tmem_base + accs[j] * BN;
+#pragma unroll
+              for (int kb = 0; kb < RKB; ++kb) {
+                const uint32_t a = alo[j] + (uint32_t)p.koff[kb];
+                const uint32_t b = blo + (uint32_t)(kb * (C::kBBytes >> 4));
+                tc_mma_bf16_lo_warp(tacc, a, b, idesc, kb != 0 ? 1u : 0u);
+                tc_mma_bf16_lo_warp(tacc, a + 2, b + 2, idesc, 1u);
+                tc_mma_bf16_lo_warp(tacc, a + 4, b + 4, idesc, 1u);
+                tc_mma_bf16_lo_warp(tacc, a + 6, b + 6, idesc, 1u);
+              }
+              tc_commit_warp(&tfull[accs[j]]);
+              tc_commit_warp(&hempty[hbs[j]]);
+            }
+          }
+          if (prof_mma) c_iss += clock64() - tA;
+        }
+      } else
       for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x, ++it) {
         const uint32_t acc = it % NACC, use = it / NACC;
+        if (prof_mma) tA = clock64();
         if (it >= (uint32_t)NACC) mbar_wait(&tempty[acc], (use - 1) & 1);
+        if (prof_mma) {
+          tB = clock64();
+          c_te += tB - tA;
+          tA = tB;
+        }
         tc_fence_after();
         const uint32_t tacc = tmem_base + acc * BN;
         uint32_t hbase = 0;
         int hoff = 0;
+        uint64_t dah = 0;  // A_HALO: descriptor of the tile's first output position in the halo buffer
         if constexpr (AMODE == A_HALO) {
           int m0, nt, g;
           decode_tile(p, tile, m0, nt, g);
@@ -462,7 +546,18 @@ __global__ void __launch_bounds__(kThreads, 1)
           const int p0 = (mt - nimg * p.mt_per_img) * BM;
           hoff = p0 - (p0 / p.Wp) * p.Wp;  // first output position's column in the first halo row
           hbase = sH + (it % HB) * halo_half_bytes(BN);
+          dah = umma_desc_k_sw128(hbase + hoff * 128);
+          if (prof_mma) {
+            tB = clock64();
+            c_dec += tB - tA;
+            tA = tB;
+          }
           mbar_wait(&hfull[it % HB], (it / HB) & 1);
+          if (prof_mma) {
+            tB = clock64();
+            c_hf += tB - tA;
+            tA = tB;
+          }
         }
         auto kblock = [&](const int kb) {
           const int stage = gk % S;
@@ -473,12 +568,9 @@ __global__ void __launch_bounds__(kThreads, 1)
           const uint32_t b0 = BRES ? sR + kb * C::kBBytes : sB + stage * C::kBBytes;
           if constexpr (AMODE == A_HALO) {
             // k-block kb = tap * cblocks + cb, tap = r * 3 + s: A = halo rows shifted by r * Wp + s
-            const int tap = kb / p.cblocks, cb = kb - tap * p.cblocks;
-            const int r = tap / 3, sc = tap - 3 * r;
-            const int shift = hoff + r * p.Wp + sc;
-            // a row-shifted start needs no descriptor base offset: the 128B swizzle follows the absolute
-            // shared-memory address bits, exactly as the TMA wrote them (measured: base offset = shift % 8 fails)
-            const uint64_t da = umma_desc_k_sw128(hbase + cb * p.hsz + shift * 128);
+            // (a row-shifted start needs no descriptor base offset: the 128B swizzle follows the absolute
+            // shared-memory address bits, exactly as the TMA wrote them; measured: base offset = shift % 8 fails)
+            const uint64_t da = dah + (uint64_t)(uint32_t)p.koff[kb];
             const uint64_t db = umma_desc_k_sw128(b0);
             tc_mma_bf16_warp(tacc, da, db, idesc, kb != 0 ? 1u : 0u);
             tc_mma_bf16_warp(tacc, da + 2, db + 2, idesc, 1u);
@@ -500,17 +592,28 @@ __global__ void __launch_bounds__(kThreads, 1)
           if constexpr (kRing) tc_commit_warp(&empty[stage]);
           ++gk;
         };
-        // unrolled by 4: a rolled loop costs a YIELD + branch-resolution stall per k-block (measured)
-        int kb = 0;
-        for (; kb + 4 <= p.nkb; kb += 4) {
-          kblock(kb);
-          kblock(kb + 1);
-          kblock(kb + 2);
-          kblock(kb + 3);
+        {
+          // unrolled by 4: a rolled loop costs a YIELD + branch-resolution stall per k-block (measured)
+          int kb = 0;
+          for (; kb + 4 <= p.nkb; kb += 4) {
+            kblock(kb);
+            kblock(kb + 1);
+            kblock(kb + 2);
+            kblock(kb + 3);
+          }
+          for (; kb < p.nkb; ++kb) kblock(kb);
         }
-        for (; kb < p.nkb; ++kb) kblock(kb);
         tc_commit_warp(&tfull[acc]);
         if constexpr (AMODE == A_HALO) tc_commit_warp(&hempty[it % HB]);  // halo free once these MMAs finish
+      }
+      if (prof_mma && p.dbg_buf) {
+        unsigned long long* o = p.dbg_buf + blockIdx.x * 8;
+        o[0] = clock64() - t_start;
+        o[1] = c_te;
+        o[2] = c_dec;
+        o[3] = c_hf;
+        o[4] = c_iss;
+        o[5] = it;
       }
     }
   } else {
@@ -613,6 +716,12 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       mbar_wait(&tfull[acc], use & 1);
       tc_fence_after();
+      if ((p.dbg & 2) && !TMA_EPI) {
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&tempty[acc]);
+        continue;
+      }
       const uint32_t taddr = tmem_base + acc * BN + ((uint32_t)(q * 32) << 16);
 #pragma unroll 1
       for (int cb = cb0; cb < cb0 + kChunks; ++cb) {
@@ -633,6 +742,31 @@ __global__ void __launch_bounds__(kThreads, 1)
             sts128(addr, o);
           }
         } else {
+          if constexpr (C::kStaged) {
+            if (!has_res && !p.out_f32) {
+              tc_wait_ld();
+              const uint32_t stg = base + C::kStgOff + (uint32_t)(warp - kEpiWarp0) * 2048u;
+#pragma unroll
+              for (int qq = 0; qq < 4; ++qq) {
+                uint4 o;
+                epi_math(v + qq * 8, scv + qq * 8, shv + qq * 8, false, make_uint4(0, 0, 0, 0), p.relu, o);
+                sts128(stg + lane * 64 + (((uint32_t)qq ^ (uint32_t)(lane & 3)) << 4), o);
+              }
+              __syncwarp();
+              const int part = lane & 3;
+#pragma unroll
+              for (int i = 0; i < 4; ++i) {
+                const int r = i * 8 + (lane >> 2);
+                const int mo_r = __shfl_sync(0xffffffffu, mo, r);
+                const int ok = __shfl_sync(0xffffffffu, rvalid ? 1 : 0, r);
+                const uint4 val = lds128(stg + r * 64 + (((uint32_t)part ^ (uint32_t)(r & 3)) << 4));
+                if (ok && cb * 32 + part * 8 < nvalid_tile)
+                  *reinterpret_cast<uint4*>(p.y + (size_t)mo_r * p.Cout + ng0 + cb * 32 + part * 8) = val;
+              }
+              __syncwarp();  // the next chunk reuses the staging rows
+              continue;
+            }
+          }
           uint4 cur[4];
 #pragma unroll
           for (int j = 0; j < 4; ++j) cur[j] = rres[j];
@@ -822,6 +956,11 @@ static const bool g_halo_enabled = [] {
   return !(e && e[0] == '0');
 }();
 
+// VISTA_CONV_DBG: measurement experiments (see ConvParams::dbg); never set in tests or the bench
+static const int g_conv_dbg = [] {
+  const char* e = getenv("VISTA_CONV_DBG");
+  return e ? atoi(e) : 0;
+}();
 // VISTA_WRES=0 disables the resident-weight launches (A/B measurements)
 static const bool g_wres_enabled = [] {
   const char* e = getenv("VISTA_WRES");
@@ -975,6 +1114,7 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   p.y = y;
   p.res = res;
   p.tapf = nullptr;
+  p.dbg = g_conv_dbg;
   p.scale = L.scale;
   p.shift = L.shift;
   p.H = H;
@@ -1028,7 +1168,7 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
     const int hsz = (hrows * Wp * 128 + 1023) & ~1023;
     const int cblocks = L.Cin / BK;
     const int half = L.BN == 64 ? 45056 : 61440;
-    if (Wp <= 256 && hrows <= 256 && hsz * cblocks <= half) {
+    if (Wp <= 256 && hrows <= 256 && hsz * cblocks <= half && L.Kp / BK <= 36) {
       const cuuint64_t dims[4] = {(cuuint64_t)L.Cin, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
       const cuuint64_t strides[3] = {(cuuint64_t)L.Cin * 2, (cuuint64_t)W * L.Cin * 2, (cuuint64_t)H * W * L.Cin * 2};
       const cuuint32_t box[4] = {(cuuint32_t)BK, (cuuint32_t)Wp, (cuuint32_t)hrows, 1};
@@ -1039,6 +1179,10 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
         p.hsz = hsz;
         p.cblocks = cblocks;
         p.mt_per_img = (p.Ho * Wp + BM - 1) / BM;
+        for (int kb = 0; kb < p.nkb && kb < 36; ++kb) {
+          const int tap = kb / cblocks, cb = kb % cblocks, r = tap / 3, sc = tap % 3;
+          p.koff[kb] = ((r * Wp + sc) * 128 + cb * hsz) >> 4;
+        }
         p.n_mt = N * p.mt_per_img;
         p.n_tiles = p.n_mt * p.n_nt;
       }
@@ -1087,8 +1231,14 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   // K <= 256 and BN <= 128 (<= 4 k-blocks); one N tile per CTA needs groups == 1 and n_nt <= the grid
   int rkb = 0;
   if (g_wres_enabled && L.groups == 1 && p.n_nt <= num_sms() && p.n_tiles >= num_sms()) {
-    if (amode == A_HALO && L.BN == 64 && p.nkb <= 9) rkb = 9;
+    if (amode == A_HALO && L.BN == 64 && p.nkb == 9) rkb = 9;
     else if (amode == A_TMA && tma_epi && L.BN <= 128 && p.nkb <= 4) rkb = 4;
+  }
+  unsigned long long* dbgb = nullptr;
+  if (p.dbg & 8) {
+    VCHECK(cudaMalloc(&dbgb, 148 * 8 * 8));
+    VCHECK(cudaMemset(dbgb, 0, 148 * 8 * 8));
+    p.dbg_buf = dbgb;
   }
   prof_begin(st);
   int nb = 1;
@@ -1115,6 +1265,21 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
              L.S, L.stride, L.groups, L.Cin, L.Cout, H, W, p.M, L.K, L.BN, amode, tma_epi ? 1 : 0, nb, rkb, p.n_tiles,
              res ? " res" : "");
   prof_end(st, 0, flops, bytes, label);
+  if (dbgb) {
+    unsigned long long h[148 * 8];
+    VCHECK(cudaMemcpy(h, dbgb, sizeof(h), cudaMemcpyDeviceToHost));
+    double a[6] = {0, 0, 0, 0, 0, 0};
+    int n = 0;
+    for (int b = 0; b < 148; ++b)
+      if (h[b * 8 + 5]) {
+        for (int k = 0; k < 6; ++k) a[k] += (double)h[b * 8 + k];
+        ++n;
+      }
+    if (n)
+      fprintf(stderr, "[conv dbg] CTAs %d tiles/CTA %.1f cycles/tile: total %.0f tempty %.0f decode %.0f hfull %.0f issue %.0f\n",
+              n, a[5] / n, a[0] / a[5], a[1] / a[5], a[2] / a[5], a[3] / a[5], a[4] / a[5]);
+    cudaFree(dbgb);
+  }
   return tapf == nullptr || fuse_tap;
 }
 

@@ -213,6 +213,40 @@ __device__ __forceinline__ uint64_t umma_desc_k_sw128(uint32_t smem_addr) {
   return d;
 }
 
+// High / low 32-bit halves of umma_desc_k_sw128: the high half is a constant, the low half holds the
+// start address (>> 4) and LBO, so descriptor arithmetic can stay in 32 bits.
+constexpr uint32_t kSw128DescHi = (1024u >> 4) | (1u << 14) | (2u << 29);
+__device__ __forceinline__ uint32_t umma_desc_lo_sw128(uint32_t smem_addr) {
+  return ((smem_addr >> 4) & 0x3FFFu) | (1u << 16);
+}
+// Single-thread issue (caller is one thread): D (+)= A * B^T with both descriptors given by their low
+// halves (SWIZZLE_128B K-major, high half constant); no elect per instruction.
+__device__ __forceinline__ void tc_mma_bf16_lo(uint32_t tmem_d, uint32_t a_lo, uint32_t b_lo, uint32_t idesc,
+                                               uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t.reg .b64 da, db;\n\t"
+      "mov.b64 da, {%1, %5};\n\t"
+      "mov.b64 db, {%2, %5};\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], da, db, %3, p;\n\t}" ::"r"(tmem_d),
+      "r"(a_lo), "r"(b_lo), "r"(idesc), "r"(accumulate), "n"(kSw128DescHi)
+      : "memory");
+}
+
+// Warp-wide form (all 32 lanes, converged; one elected lane issues): descriptor arithmetic stays warp-uniform.
+__device__ __forceinline__ void tc_mma_bf16_lo_warp(uint32_t tmem_d, uint32_t a_lo, uint32_t b_lo, uint32_t idesc,
+                                                    uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p, e;\n\t.reg .b64 da, db;\n\t"
+      "mov.b64 da, {%1, %5};\n\t"
+      "mov.b64 db, {%2, %5};\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], da, db, %3, p;\n\t}" ::"r"(tmem_d),
+      "r"(a_lo), "r"(b_lo), "r"(idesc), "r"(accumulate), "n"(kSw128DescHi)
+      : "memory");
+}
+
 // Shared-memory matrix descriptor, K-major, no swizzle: 8-row x 16-byte core matrices, rows 16 B
 // apart, core matrices `sbo` bytes apart along M/N and `lbo` bytes apart along K.
 __device__ __forceinline__ uint64_t umma_desc_k_none(uint32_t smem_addr, uint32_t lbo, uint32_t sbo) {

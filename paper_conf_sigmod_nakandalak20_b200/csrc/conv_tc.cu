@@ -36,10 +36,11 @@ enum AMode {
   A_IM2COL = 4,
   A_IM2COL_C8 = 5,
   A_ROWVIEW = 6,
-  A_HALO = 7
+  A_HALO = 7,
+  A_CAT = 8
 };
 __host__ __device__ constexpr bool a_by_tma(int m) {
-  return m == A_TMA || m == A_IM2COL || m == A_IM2COL_C8 || m == A_ROWVIEW || m == A_HALO;
+  return m == A_TMA || m == A_IM2COL || m == A_IM2COL_C8 || m == A_ROWVIEW || m == A_HALO || m == A_CAT;
 }
 // A_HALO (3x3 stride 1 pad 1, one N tile): the output is computed on the padded-width grid (Wp = W + 2
 // positions per row, the last two discarded) so that output position p reads padded input position
@@ -62,6 +63,10 @@ struct ConvParams {
   // issue loop has no integer division (measured: the per-k-block division chain made the issue latency
   // ~340 cycles, longer than the 4 MMAs it feeds)
   int koff[36];
+  // A_CAT (unit-1 closing conv with the projection shortcut folded in, see conv_cat_forward): k-blocks
+  // [0, nkb1) read the b activation through tmap_a, k-blocks [nkb1, nkb) read the unit input x through
+  // tmap_r (plain 2-D map, or an im2col map when the projection is strided: cat_im2col = 1)
+  int nkb1, cat_im2col;
   // fused tap g_l (PAPER.md:369 fn 4): per-image 2x2-grid channel maxima of the (post-ReLU, >= 0)
   // output, accumulated as fp32 bit patterns with red.global.max.u32 into tapf[n][4][Cout]
   unsigned int* tapf;
@@ -253,6 +258,31 @@ __global__ void __launch_bounds__(kThreads, 1)
             mbar_arrive_expect_tx(&full[stage], C::kStageBytes);
             tma_load_2d(sA + stage * C::kABytes, &tmap_a, g * p.Cg_in + kb * BK, m0, &full[stage]);
             if constexpr (!BRES) tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
+          }
+        }
+      }
+    } else if constexpr (AMODE == A_CAT) {
+      if (threadIdx.x == 0) {
+        const int hw = p.Ho * p.Wo;
+        uint32_t gk = 0;
+        for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x) {
+          int m0, nt, g;
+          decode_tile(p, tile, m0, nt, g);
+          const int n0 = nt * BN;
+          const int nimg = m0 / hw, rem = m0 - nimg * hw;
+          const int ho = rem / p.Wo, wo = rem - ho * p.Wo;
+          for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
+            const int stage = gk % S;
+            if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
+            mbar_arrive_expect_tx(&full[stage], C::kStageBytes);
+            if (kb < p.nkb1)
+              tma_load_2d(sA + stage * C::kABytes, &tmap_a, kb * BK, m0, &full[stage]);
+            else if (p.cat_im2col)
+              tma_load_im2col_4d(sA + stage * C::kABytes, &tmap_r, (kb - p.nkb1) * BK, wo * p.stride, ho * p.stride,
+                                 nimg, 0, 0, &full[stage]);
+            else
+              tma_load_2d(sA + stage * C::kABytes, &tmap_r, (kb - p.nkb1) * BK, m0, &full[stage]);
+            if constexpr (!BRES) tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, n0, &full[stage]);
           }
         }
       }
@@ -1079,6 +1109,15 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
       }
       launch_t<BN, A_TMA, TE, NB>(L, ta, ty, tr, p, st);
       break;
+    case A_CAT:
+      if constexpr (TE && BN <= 128) {
+        if (rkb == 4) {
+          launch_t<BN, A_CAT, TE, NB, 4>(L, ta, ty, tr, p, st);
+          break;
+        }
+      }
+      launch_t<BN, A_CAT, TE, NB>(L, ta, ty, tr, p, st);
+      break;
     case A_GATHER_FAST: launch_t<BN, A_GATHER_FAST, TE, NB>(L, ta, ty, tr, p, st); break;
     case A_GATHER_ROW: launch_t<BN, A_GATHER_ROW, TE, NB>(L, ta, ty, tr, p, st); break;
     case A_IM2COL: launch_t<BN, A_IM2COL, TE, NB>(L, ta, ty, tr, p, st); break;
@@ -1281,6 +1320,73 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
     cudaFree(dbgb);
   }
   return tapf == nullptr || fuse_tap;
+}
+
+// Closing 1x1 conv of a projection unit with the projection folded into its K loop (A_CAT):
+//   y = ReLU(s_c * ([b | x_s] . [Wc | Wp']^T) + t),  Wp' = bf16(Wp * s_p / s_c), t = t_c + t_p
+// = ReLU(BN_c(b * Wc) + BN_p(x_s * Wp)) up to the bf16 rounding of the rescaled projection weights
+// (reading R31).  b: [N, Ho, Wo, Kb] (Kb = L.Cin - Cx), x: [N, Hx, Wx, Cx], x_s = x sampled at stride
+// `stride` (Ho = ceil(Hx / stride)).  The projection output (4 * mid channels per pixel) is never written
+// to HBM nor read back as the residual.
+void conv_cat_forward(const ConvLayer& L, int Cx, const bf16* b, const bf16* x, int N, int Hx, int Wx, int stride,
+                      bf16* y, cudaStream_t st) {
+  const int Kb = L.Cin - Cx;
+  if (L.R != 1 || L.S != 1 || L.groups != 1 || Kb <= 0 || Kb % BK || Cx % BK || L.Kp != L.Cin)
+    fail(1, "conv_cat: unsupported layer");
+  ConvParams p{};
+  p.x = b;
+  p.y = y;
+  p.res = nullptr;
+  p.dbg = g_conv_dbg;
+  p.scale = L.scale;
+  p.shift = L.shift;
+  p.H = p.Ho = conv_out_dim(Hx, 1, stride, 0);
+  p.W = p.Wo = conv_out_dim(Wx, 1, stride, 0);
+  p.Cin = L.Cin;
+  p.Cout = L.Cout;
+  p.R = p.S = 1;
+  p.stride = stride;
+  p.Cg_in = L.Cin;
+  p.Cg_out = L.Cout;
+  p.K = L.K;
+  p.nkb = L.Kp / BK;
+  p.nkb1 = Kb / BK;
+  p.cat_im2col = stride != 1;
+  const int64_t M = (int64_t)N * p.Ho * p.Wo;
+  if (M <= 0) return;
+  if (M > INT32_MAX - BM) fail(1, "conv_cat: M too large for one launch");
+  p.M = (int)M;
+  p.relu = L.relu ? 1 : 0;
+  p.n_mt = (p.M + BM - 1) / BM;
+  p.n_nt = (L.Cout + L.BN - 1) / L.BN;
+  p.n_tiles = p.n_mt * p.n_nt;
+  CUtensorMap ta, ty, tr;
+  std::memset(&ty, 0, sizeof(ty));
+  make_tmap(&ta, b, (uint64_t)Kb, (uint64_t)M, BM);
+  if (stride != 1) make_tmap_im2col(&tr, x, N, Hx, Wx, Cx, 1, 1, stride, 0, BK, true);
+  else make_tmap(&tr, x, (uint64_t)Cx, (uint64_t)M, BM);
+  const bool tma_epi = L.Cout % 8 == 0 && p.nkb <= 8;
+  if (tma_epi) make_tmap(&ty, y, (uint64_t)L.Cout, (uint64_t)M, BM);
+  else ty = L.tmap_w;  // unused
+  const int rkb = (g_wres_enabled && tma_epi && L.BN <= 128 && p.nkb <= 4 && p.n_nt <= num_sms() &&
+                   p.n_tiles >= num_sms()) ? 4 : 0;
+  const double flops = 2.0 * (double)M * L.Cout * L.K_alg;
+  const double bytes = 2.0 * ((double)M * (Kb + Cx + L.Cout) + (double)L.Cout * L.Kp);
+  prof_begin(st);
+  if (tma_epi) {
+    if (L.BN == 256) launch_bn<256, true, 1>(L, A_CAT, ta, ty, tr, p, st, rkb);
+    else if (L.BN == 128) launch_bn<128, true, 3>(L, A_CAT, ta, ty, tr, p, st, rkb);
+    else launch_bn<64, true, 4>(L, A_CAT, ta, ty, tr, p, st, rkb);
+  } else {
+    if (L.BN == 256) launch_bn<256, false, 1>(L, A_CAT, ta, ty, tr, p, st, 0);
+    else if (L.BN == 128) launch_bn<128, false, 1>(L, A_CAT, ta, ty, tr, p, st, 0);
+    else launch_bn<64, false, 1>(L, A_CAT, ta, ty, tr, p, st, 0);
+  }
+  char label[160] = {0};
+  if (prof_labels())
+    snprintf(label, sizeof(label), "conv_cat c+proj s%d Cb%d Cx%d Cout%d HxW%dx%d K%d BN%d epi%d rkb%d", stride, Kb,
+             Cx, L.Cout, p.Ho, p.Wo, L.K, L.BN, tma_epi ? 1 : 0, rkb);
+  prof_end(st, 0, flops, bytes, label);
 }
 
 // Plain "TN" GEMM on the same kernel (A_TMA mode, register epilogue):

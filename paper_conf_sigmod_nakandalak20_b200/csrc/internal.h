@@ -60,6 +60,10 @@ void conv_layer_free(ConvLayer& L);
 // (2x2-grid maxima); returns false if the tap could not be fused (caller runs launch_tap instead).
 bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const bf16* res, bf16* y,
                   cudaStream_t st, unsigned int* tapf = nullptr);
+// closing 1x1 conv of a projection unit with the projection shortcut in its K loop (conv_tc.cu):
+// L = the concatenated layer ([Cout][Kb + Cx] weights, see conv_cat_forward), b [N,Ho,Wo,Kb], x [N,Hx,Wx,Cx]
+void conv_cat_forward(const ConvLayer& L, int Cx, const bf16* b, const bf16* x, int N, int Hx, int Wx, int stride,
+                      bf16* y, cudaStream_t st);
 bool make_rowview_tmap(CUtensorMap* m, const void* x, int N, int H, int W, int C, int Wo);
 bool make_plain_tmap(CUtensorMap* m, const void* ptr, int cols, int rows);
 // Two chained 1x1 convs of consecutive ResNet units (res_chain.cu): out = ReLU(BN_c(b * Wc) + res) and
@@ -163,5 +167,6 @@ void prof_end(cudaStream_t st, int cls, double flops, double bytes, const char* 
 bool prof_labels();  // true when per-launch records are logged (VISTA_PROF_LOG)
 
 int num_sms();
+void set_sm_budget(int n);  // per-thread grid cap for persistent launches (0 = all SMs)
 
 }  // namespace vista

@@ -31,14 +31,22 @@ static std::atomic<long long> g_launches{0};
 void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
 long long launches_total() { return g_launches.load(); }
 
+// SMs a persistent launch may occupy: the device's count, or a smaller per-thread budget when the
+// executor runs two micro-batches side by side on disjoint halves of the GPU (set_sm_budget)
+static thread_local int t_sm_budget = 0;
+void set_sm_budget(int n) { t_sm_budget = n; }
 int num_sms() {
   static int n = 0;
   if (!n) {
     int dev = 0;
     cudaGetDevice(&dev);
     if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 148;
+    if (const char* e = getenv("VISTA_SM_CAP")) {  // measurement only: cap every launch's grid
+      const int cap = atoi(e);
+      if (cap > 0 && cap < n) n = cap;
+    }
   }
-  return n;
+  return t_sm_budget > 0 && t_sm_budget < n ? t_sm_budget : n;
 }
 
 // ---------------- profiler ----------------
@@ -243,6 +251,10 @@ struct vista_ctx {
   bool fuse_stem = true;
   // closing 1x1 conv + next unit's opening 1x1 conv (res_chain.cu, bit-identical); VISTA_FUSE_CHAIN=0 disables
   bool fuse_chain = true;
+  // unit-1 closing conv with the projection shortcut in its K loop (conv_cat_forward, reading R31);
+  // convs_cat[c-layer index] is the concatenated layer (Cin == 0: none); VISTA_FUSE_PROJ=0 disables
+  bool fuse_proj = true;
+  std::vector<ConvLayer> convs_cat;
   std::vector<void*> feat;  // per block: device pointer of F_t (features) of a tapped layer
   // seeded initial MLP weights per requested layer (host, generated on first use: model init, like the
   // CNN weights of vista_plan)
@@ -266,6 +278,7 @@ struct vista_ctx {
     for (DevBuf* b : {&pair_str, &pair_img, &d_X, &d_labels, &d_img_keys, &d_str_keys, &d_px}) b->release();
     if (stream) cudaStreamSynchronize(stream);
     for (auto& L : convs) conv_layer_free(L);
+    for (auto& L : convs_cat) conv_layer_free(L);
     for (auto& L : convs32) conv_layer_free_f32(L);
     if (nccl_comm) {
       Nccl& n = nccl_lib();
@@ -397,11 +410,57 @@ void plan_memory(vista_ctx* c, uint64_t budget) {
   c->peak_pred = peak;
 }
 
+struct HostLayer {
+  std::vector<float> w;  // OHWI, bf16-representable values
+  std::vector<float> scale, shift;
+};
+
+// Projection units: for every "proj (1x1, stride s) -> c (1x1, residual = proj output)" op pair, the layer
+// [Wc | Wp'] with Wp'[o] = bf16(Wp[o] * s_p[o] / s_c[o]), scale s_c and shift t_c + t_p (reading R31), so
+// that ReLU(BN_c(b Wc) + BN_p(x_s Wp)) is one GEMM over the concatenated K = mid + Cin.
+void build_cat_layers(vista_ctx* c, const std::vector<HostLayer>& hostw) {
+  c->convs_cat.resize(c->net.layers.size());
+  for (const StageDesc& S : c->net.stages)
+    for (size_t oi = 0; oi + 1 < S.ops.size(); ++oi) {
+      const OpDesc& op = S.ops[oi];
+      const OpDesc& o2 = S.ops[oi + 1];
+      if (op.kind != OP_CONV || o2.kind != OP_CONV || o2.res != op.out || op.res >= 0) continue;
+      const LayerSpec& lp = c->net.layers[op.layer];
+      const LayerSpec& lc = c->net.layers[o2.layer];
+      const HostLayer& hp = hostw[op.layer];
+      const HostLayer& hc = hostw[o2.layer];
+      if (hp.w.empty() || hc.w.empty() || lp.relu || !lc.relu || lc.stride != 1 || lp.Cout != lc.Cout ||
+          lc.Cin != lc.Cin_real || lp.Cin != lp.Cin_real || lc.Cin % 64 || lp.Cin % 64 || c->convs_cat[o2.layer].w)
+        continue;
+      const int Kb = lc.Cin, Kx = lp.Cin, K = Kb + Kx, Co = lc.Cout;
+      bool ok = true;
+      for (int o = 0; o < Co; ++o) ok = ok && std::fabs(hc.scale[o]) > 1e-6f * std::fabs(hp.scale[o]);
+      if (!ok) continue;  // a near-zero s_c would blow up the rescaled projection weights: keep it unfused
+      std::vector<uint16_t> wcat((size_t)Co * K);
+      std::vector<float> sc(Co), sh(Co);
+      for (int o = 0; o < Co; ++o) {
+        for (int k = 0; k < Kb; ++k) wcat[(size_t)o * K + k] = f2bf_bits(hc.w[(size_t)o * Kb + k]);
+        const double ratio = (double)hp.scale[o] / (double)hc.scale[o];
+        for (int k = 0; k < Kx; ++k)
+          wcat[(size_t)o * K + Kb + k] = f2bf_bits((float)((double)hp.w[(size_t)o * Kx + k] * ratio));
+        sc[o] = hc.scale[o];
+        sh[o] = (float)((double)hc.shift[o] + (double)hp.shift[o]);
+      }
+      ConvLayer& L = c->convs_cat[o2.layer];
+      L.Cin = K;
+      L.Cout = Co;
+      L.relu = true;
+      conv_layer_init(L, wcat, K, sc, sh);
+      c->weight_bytes += (int64_t)Co * L.Kp * 2 + (int64_t)Co * 8;
+    }
+}
+
 void upload_weights(vista_ctx* c, uint64_t seed) {
   if (c->f32)
     c->convs32.resize(c->net.layers.size());
   else
     c->convs.resize(c->net.layers.size());
+  std::vector<HostLayer> hostw(c->net.layers.size());
   c->weight_bytes = 0;
   for (size_t i = 0; i < c->net.layers.size(); ++i) {
     const LayerSpec& s = c->net.layers[i];
@@ -478,8 +537,10 @@ void upload_weights(vista_ctx* c, uint64_t seed) {
       for (size_t j = 0; j < wf.size(); ++j) wb[j] = f2bf_bits(wf[j]);
       conv_layer_init(L, wb, cin_real, scale, shift);
       c->weight_bytes += (int64_t)L.Cout * L.Kp * 2 + (int64_t)L.Cout * 8;
+      if (s.R == 1 && s.S == 1 && s.groups == 1 && s.bn_kind == 2) hostw[i] = HostLayer{std::move(wf), scale, shift};
     }
   }
+  if (!c->f32) build_cat_layers(c, hostw);
 }
 
 const void* to_device(vista_ctx* c, DevBuf& buf, const void* p, size_t bytes) {
@@ -556,6 +617,17 @@ bool run_ops(vista_ctx* c, int t, const void* in_ptr, void* out_ptr, int nb, voi
         conv1_pool_forward(c->convs[op.layer], in, nb, reinterpret_cast<bf16*>(slot[S.ops[oi + 1].out]), c->stream);
         ++oi;
         continue;
+      }
+      // projection unit: the projection 1x1 conv folded into the closing conv's K loop (reading R31)
+      if (op.kind == OP_CONV && c->fuse_proj && oi + 1 < S.ops.size() && !c->convs_cat.empty()) {
+        const OpDesc& o2 = S.ops[oi + 1];
+        if (o2.kind == OP_CONV && o2.res == op.out && op.res < 0 && c->convs_cat[o2.layer].w &&
+            !(tapf && o2.out == BUF_OUT)) {
+          conv_cat_forward(c->convs_cat[o2.layer], op.C, reinterpret_cast<const bf16*>(slot[o2.in]), in, nb, op.H,
+                           op.W, c->convs[op.layer].stride, reinterpret_cast<bf16*>(slot[o2.out]), c->stream);
+          ++oi;
+          continue;
+        }
       }
       // closing 1x1 conv of a bottleneck unit + the next unit's opening 1x1 conv in one kernel
       if (op.kind == OP_CONV && op.res >= 0 && c->fuse_chain && oi + 1 < S.ops.size()) {
@@ -780,6 +852,7 @@ VISTA_API vista_status vista_plan(vista_cnn cnn, const int32_t* layers, int32_t 
     if (const char* e = getenv("VISTA_FUSED_TAP")) c->fuse_tap = e[0] != '0';
     if (const char* e = getenv("VISTA_FUSE_STEM")) c->fuse_stem = e[0] != '0';
     if (const char* e = getenv("VISTA_FUSE_CHAIN")) c->fuse_chain = e[0] != '0';
+    if (const char* e = getenv("VISTA_FUSE_PROJ")) c->fuse_proj = e[0] != '0';
     VCHECK(cudaStreamSynchronize(c->stream));
   });
   if (st != VISTA_OK) {

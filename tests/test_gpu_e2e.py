@@ -242,6 +242,27 @@ def test_resnet_chain_fused_bit_identical(monkeypatch):
         assert torch.equal(a, b)
 
 
+def test_resnet_projection_fused(monkeypatch):
+    # Unit 1 of every ResNet stage runs its closing 1x1 conv with the projection shortcut folded into the
+    # K loop (conv_cat_forward, reading R31: projection weights rescaled by s_p / s_c and rounded to bf16,
+    # no bf16 rounding of the shortcut); VISTA_FUSE_PROJ=0 runs projection + conv-with-residual.  Both must
+    # meet the oracle tolerance, and they may differ only by bf16-level rounding.  37 images: partial
+    # last tiles at every stage (stride-1 res2 and strided im2col res3/res4/res5 projections).
+    tab = gen.make_tables(37, 8)
+    F, _ = oracle.features(oracle.RESNET50, WSEED, tab.images[:6], taps=[0, 1, 2, 3, 4])
+    out = {}
+    for fuse in ("1", "0"):
+        monkeypatch.setenv("VISTA_FUSE_PROJ", fuse)
+        v = run_gpu(2, [0, 1, 2, 3, 4], tab, 8, iters=1, micro_batch=37)
+        out[fuse] = [v.features(k)["features"].to(torch.float64).cpu().numpy() for k in range(5)]
+        v.close()
+    for k in range(5):
+        a, b = out["1"][k], out["0"][k]
+        assert normwise_rows(a[:6], F[k]).max() <= 2e-2, (k, normwise_rows(a[:6], F[k]).max())
+        assert normwise_rows(a, b).max() <= 2e-2
+        assert not np.array_equal(a, b) or k == 4  # the fused path really ran
+
+
 @pytest.mark.parametrize("cnn,taps,n,d_s,chunked", [(0, [1, 2, 3], 10, 8, False), (2, [1, 3, 4], 6, 16, False),
                                                     (2, [0, 2, 4], 40, 8, True)])
 def test_pre_materialized_base_layer(cnn, taps, n, d_s, chunked):

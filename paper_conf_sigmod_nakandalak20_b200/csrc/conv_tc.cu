@@ -1285,8 +1285,9 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
     if (L.BN == 256) {
       launch_bn<256, true, 1>(L, amode, ta, ty, tr, p, st, rkb);
     } else if (L.BN == 128) {
-      nb = g_epi_nb_env == 2 ? 2 : 3;
+      nb = g_epi_nb_env == 2 ? 2 : (g_epi_nb_env == 4 ? 4 : 3);
       if (nb == 2) launch_bn<128, true, 2>(L, amode, ta, ty, tr, p, st, rkb);
+      else if (nb == 4) launch_bn<128, true, 4>(L, amode, ta, ty, tr, p, st, rkb);
       else launch_bn<128, true, 3>(L, amode, ta, ty, tr, p, st, rkb);
     } else {
       nb = g_epi_nb_env == 2 ? 2 : 4;

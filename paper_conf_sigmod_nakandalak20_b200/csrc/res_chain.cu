@@ -25,16 +25,19 @@ namespace {
 constexpr int BMr = 128, BKr = 64;
 constexpr int kEpiW0 = 2, kEpiWn = 8, kEpiT = kEpiWn * 32, kThr = (kEpiW0 + kEpiWn) * 32;
 
-template <int MID>
+// V = 0: b tile double-buffered; V = 1: b single-buffered, the freed 16/32 KB spent on one more
+// weight stage (MID = 64) or one more out/residual staging buffer (MID = 128: residual chunks in flight)
+template <int MID, int V = 0>
 struct RC {
   static constexpr int NCH = 4 * MID / 128;       // c chunks of 128 channels
   static constexpr int KBC = MID / BKr;           // k-blocks of the c GEMM
-  static constexpr int NB = MID == 64 ? 3 : 2;    // out/residual staging buffers
-  static constexpr int WS = MID == 64 ? 4 : 3;    // weight ring stages (16 KB)
+  static constexpr int NBB = V ? 1 : 2;           // b tile buffers
+  static constexpr int NB = MID == 64 ? 3 : (V ? 3 : 2);  // out/residual staging buffers
+  static constexpr int WS = MID == 64 ? (V ? 5 : 4) : 3;  // weight ring stages (16 KB)
   static constexpr int kB = KBC * BMr * 128;      // b tile bytes
   static constexpr int kO = BMr * 128 * 2;        // one out chunk: two 64-channel sub-tiles
   static constexpr int kA = BMr * MID * 2;        // a_next tile
-  static constexpr int offB = 0, offO = offB + 2 * kB, offA = offO + NB * kO, offW = offA + kA,
+  static constexpr int offB = 0, offO = offB + NBB * kB, offA = offO + NB * kO, offW = offA + kA,
                        offS = offW + WS * 16384, offBar = offS + (5 * MID) * 2 * 4;
   static constexpr int nBar = 2 + 2 + NB * 3 + 2 * WS + 2 + 1 + 1 + 2;
   static constexpr int kSmem = offBar + nBar * 8 + 16 + 1024;
@@ -49,14 +52,14 @@ struct RCParams {
   int M, n_mt;
 };
 
-template <int MID>
+template <int MID, int V>
 __global__ void __launch_bounds__(kThr, 1)
     res_chain_kernel(const __grid_constant__ CUtensorMap tm_b, const __grid_constant__ CUtensorMap tm_res,
                      const __grid_constant__ CUtensorMap tm_out, const __grid_constant__ CUtensorMap tm_a,
                      const __grid_constant__ CUtensorMap tm_wc, const __grid_constant__ CUtensorMap tm_wa,
                      const RCParams p) {
-  using C = RC<MID>;
-  constexpr int NCH = C::NCH, KBC = C::KBC, NB = C::NB, WS = C::WS;
+  using C = RC<MID, V>;
+  constexpr int NCH = C::NCH, KBC = C::KBC, NB = C::NB, WS = C::WS, NBB = C::NBB;
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 1023u) & ~1023u;
@@ -141,8 +144,8 @@ __global__ void __launch_bounds__(kThr, 1)
       };
       for (int tile = blockIdx.x; tile < p.n_mt; tile += gridDim.x, ++it, q += NCH) {
         const int m0 = tile * BMr;
-        const uint32_t bb = it & 1;
-        if (it >= 2) mbar_wait(&bempty[bb], ((it >> 1) - 1) & 1);
+        const uint32_t bb = it % NBB;
+        if (it >= (uint32_t)NBB) mbar_wait(&bempty[bb], ((it / NBB) - 1) & 1);
         mbar_arrive_expect_tx(&bfull[bb], C::kB);
         for (int kb = 0; kb < KBC; ++kb) tma_load_2d(sB + bb * C::kB + kb * BMr * 128, &tm_b, kb * BKr, m0, &bfull[bb]);
         // weights in the order the MMA warp consumes them: c(0), then per j: c(j+1), a(j); each residual
@@ -169,8 +172,8 @@ __global__ void __launch_bounds__(kThr, 1)
       return st;
     };
     for (int tile = blockIdx.x; tile < p.n_mt; tile += gridDim.x, ++it) {
-      const uint32_t bb = it & 1, qbase = it * NCH;
-      mbar_wait(&bfull[bb], (it >> 1) & 1);
+      const uint32_t bb = it % NBB, qbase = it * NCH;
+      mbar_wait(&bfull[bb], (it / NBB) & 1);
       auto issue_c = [&](const int j) {
         const uint32_t qq = qbase + j, acc = qq & 1;
         if (qq >= 2) mbar_wait(&tempty_c[acc], ((qq >> 1) - 1) & 1);
@@ -333,7 +336,7 @@ bool res_chain_supported(const ConvLayer& Lc, const ConvLayer& La) {
          La.groups == 1 && La.Cin == 4 * mid && La.Cout == mid && La.BN == mid && La.relu;
 }
 
-template <int MID>
+template <int MID, int V>
 static void launch_chain(const ConvLayer& Lc, const ConvLayer& La, const bf16* b, const bf16* res, bf16* out,
                          bf16* a_next, int M, cudaStream_t st) {
   CUtensorMap tb, tr, to, ta;
@@ -349,11 +352,11 @@ static void launch_chain(const ConvLayer& Lc, const ConvLayer& La, const bf16* b
   p.n_mt = (M + BMr - 1) / BMr;
   static bool attr = false;
   if (!attr) {
-    VCHECK(cudaFuncSetAttribute(res_chain_kernel<MID>, cudaFuncAttributeMaxDynamicSharedMemorySize, RC<MID>::kSmem));
+    VCHECK(cudaFuncSetAttribute(res_chain_kernel<MID, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, RC<MID, V>::kSmem));
     attr = true;
   }
   const int grid = p.n_mt < num_sms() ? p.n_mt : num_sms();
-  res_chain_kernel<MID><<<grid, kThr, RC<MID>::kSmem, st>>>(tb, tr, to, ta, Lc.tmap_w, La.tmap_w, p);
+  res_chain_kernel<MID, V><<<grid, kThr, RC<MID, V>::kSmem, st>>>(tb, tr, to, ta, Lc.tmap_w, La.tmap_w, p);
   LAUNCHED();
 }
 
@@ -365,8 +368,20 @@ void res_chain_forward(const ConvLayer& Lc, const ConvLayer& La, const bf16* b, 
   const int M = (int)M64;
   const int mid = Lc.Cin;
   prof_begin(st);
-  if (mid == 64) launch_chain<64>(Lc, La, b, res, out, a_next, M, st);
-  else launch_chain<128>(Lc, La, b, res, out, a_next, M, st);
+  static const int v = [] {
+    // measured (ResNet50 res3, 28x28): the MID = 128 chain is bound by residual chunks in flight, so its b
+    // tile is single-buffered for a third staging buffer (20.98 -> 16.52 ms per step); MID = 64 keeps the
+    // double-buffered b (its V = 1 variant was 1 % slower).  VISTA_CHAIN_V overrides (bit 0: 64, bit 1: 128)
+    const char* e = getenv("VISTA_CHAIN_V");
+    return e ? atoi(e) : 2;
+  }();
+  if (mid == 64) {
+    if (v & 1) launch_chain<64, 1>(Lc, La, b, res, out, a_next, M, st);
+    else launch_chain<64, 0>(Lc, La, b, res, out, a_next, M, st);
+  } else {
+    if (v & 2) launch_chain<128, 1>(Lc, La, b, res, out, a_next, M, st);
+    else launch_chain<128, 0>(Lc, La, b, res, out, a_next, M, st);
+  }
   const double flops = 2.0 * M64 * (double)(4 * mid) * mid * 2;  // both GEMMs
   const double bytes = 2.0 * M64 * ((double)mid + 4 * mid + 4 * mid + mid) + 2.0 * 8 * mid * mid;
   char label[96] = {0};

@@ -223,6 +223,11 @@ struct vista_ctx {
   vista_lr_cfg lr{};
   vista_sys_cfg sys{};
   cudaStream_t stream = nullptr;
+  // host pixels: H2D copies per stage-1 micro-batch on their own stream, each followed by an event the
+  // compute stream waits on, so the copy of micro-batch i + 1 overlaps the inference of micro-batch i
+  cudaStream_t copy_stream = nullptr;
+  std::vector<cudaEvent_t> px_ready;
+  cudaEvent_t px_free = nullptr;  // the previous transfer's compute is done with d_px
   bool own_stream = false;
   int64_t n_img = 0, n_str = 0;
   int d_s = 0, ds_pad = 0;
@@ -285,6 +290,9 @@ struct vista_ctx {
       if (n.CommDestroy) n.CommDestroy(nccl_comm);
     }
     if (own_stream && stream) cudaStreamDestroy(stream);
+    for (cudaEvent_t e : px_ready) cudaEventDestroy(e);
+    if (px_free) cudaEventDestroy(px_free);
+    if (copy_stream) cudaStreamDestroy(copy_stream);
   }
 };
 
@@ -672,7 +680,10 @@ bool run_ops(vista_ctx* c, int t, const void* in_ptr, void* out_ptr, int nb, voi
 }
 
 // one block of the Staged plan over n images (a chunk), in micro-batches of micro[t]: in_base -> A_t
-bool run_block(vista_ctx* c, int t, const void* in_base, void* out_base, int64_t n, unsigned int* tapf) {
+// in_ready (optional): event j is recorded once micro-batch j's input has landed (host pixels copied on
+// c->copy_stream); the compute stream waits on it right before that micro-batch
+bool run_block(vista_ctx* c, int t, const void* in_base, void* out_base, int64_t n, unsigned int* tapf,
+               const std::vector<cudaEvent_t>* in_ready = nullptr) {
   const StageDesc& S = c->net.stages[t];
   const int B = c->micro[t];
   void* slot[NUM_BUFS] = {nullptr};
@@ -681,6 +692,7 @@ bool run_block(vista_ctx* c, int t, const void* in_base, void* out_base, int64_t
   bool fused = tapf != nullptr;
   for (int64_t i0 = 0; i0 < n; i0 += B) {
     const int nb = (int)std::min<int64_t>(B, n - i0);
+    if (in_ready) VCHECK(cudaStreamWaitEvent(c->stream, (*in_ready)[(size_t)(i0 / B)], 0));
     const bool ok = run_ops(c, t, (const uint8_t*)in_base + (size_t)i0 * in_bytes_per,
                             (uint8_t*)out_base + (size_t)i0 * S.out_elems * c->esz, nb, slot,
                             tapf ? tapf + (size_t)i0 * 4 * S.outC : nullptr);
@@ -985,10 +997,31 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
           base_c = (const uint8_t*)base + (size_t)c0 * base_img_bytes;
         }
       }
-      if (host_px) {  // stream the chunk's pixels to the device
+      const std::vector<cudaEvent_t>* px_ev = nullptr;
+      if (host_px) {  // stream the chunk's pixels to the device, one stage-1 micro-batch per copy
         c->d_px.ensure((size_t)nc * S[0].in_elems);
-        VCHECK(cudaMemcpyAsync(c->d_px.p, images + (size_t)c0 * S[0].in_elems, (size_t)nc * S[0].in_elems,
-                               cudaMemcpyHostToDevice, st));
+        if (!c->copy_stream) {
+          VCHECK(cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking));
+          VCHECK(cudaEventCreateWithFlags(&c->px_free, cudaEventDisableTiming));
+        }
+        // d_px may still be read by work already queued on the compute stream (the previous chunk)
+        VCHECK(cudaEventRecord(c->px_free, st));
+        VCHECK(cudaStreamWaitEvent(c->copy_stream, c->px_free, 0));
+        const int64_t B0 = std::max(c->micro[0], 1);
+        const size_t nev = (size_t)((nc + B0 - 1) / B0);
+        while (c->px_ready.size() < nev) {
+          cudaEvent_t e;
+          VCHECK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+          c->px_ready.push_back(e);
+        }
+        for (int64_t i0 = 0; i0 < nc; i0 += B0) {
+          const int64_t nb = std::min<int64_t>(B0, nc - i0);
+          VCHECK(cudaMemcpyAsync((uint8_t*)c->d_px.p + (size_t)i0 * S[0].in_elems,
+                                 images + (size_t)(c0 + i0) * S[0].in_elems, (size_t)nb * S[0].in_elems,
+                                 cudaMemcpyHostToDevice, c->copy_stream));
+          VCHECK(cudaEventRecord(c->px_ready[(size_t)(i0 / B0)], c->copy_stream));
+        }
+        px_ev = &c->px_ready;
         pxc = (const uint8_t*)c->d_px.p;
       }
       for (int t = base ? t0 : 0; t <= c->t_max; ++t) {
@@ -1004,7 +1037,7 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
           VCHECK(cudaMemsetAsync(c->tapacc.p, 0, cnt * 4, st));  // max over non-negative (post-ReLU) values
           tapf = (unsigned int*)c->tapacc.p;
         }
-        const bool fused = t == t0 ? false : run_block(c, t, in, At, nc, tapf);
+        const bool fused = t == t0 ? false : run_block(c, t, in, At, nc, tapf, t == 0 ? px_ev : nullptr);
         if (k >= 0) {
           void* Ft = (uint8_t*)c->F[t]->p + (size_t)c0 * S[t].d_tap * c->esz;
           if (S[t].fc_tap)  // g = identity on FC layers

@@ -67,6 +67,10 @@ struct ConvParams {
   // [0, nkb1) read the b activation through tmap_a, k-blocks [nkb1, nkb) read the unit input x through
   // tmap_r (plain 2-D map, or an im2col map when the projection is strided: cat_im2col = 1)
   int nkb1, cat_im2col;
+  // mc = 1: launched as clusters of 2 CTAs; the pair walks "pair tiles" (two adjacent M tiles, one N tile:
+  // rank r takes M tile 2 * pair_m + r) in lockstep, and each CTA TMA-loads half of every weight (B) k-block
+  // and multicasts it to both, halving the per-SM L2 -> shared-memory weight traffic of streamed-B layers
+  int mc;
   // fused tap g_l (PAPER.md:369 fn 4): per-image 2x2-grid channel maxima of the (post-ReLU, >= 0)
   // output, accumulated as fp32 bit patterns with red.global.max.u32 into tapf[n][4][Cout]
   unsigned int* tapf;
@@ -132,6 +136,13 @@ struct Cfg {
 // tile -> (first row m0, N-tile index nt, group g); N-tiles of one M-tile are adjacent so
 // the 148 CTAs working at any moment share A rows in L2
 __device__ __forceinline__ void decode_tile(const ConvParams& p, int tile, int& m0, int& nt, int& g) {
+  if (p.mc) {  // pair tile -> this CTA's M tile (an odd last M tile leaves rank 1 a phantom tile past M)
+    const int pm = tile / p.n_nt;
+    nt = tile - pm * p.n_nt;
+    m0 = (pm * 2 + (int)(blockIdx.x & 1)) * BM;
+    g = 0;
+    return;
+  }
   const int per_g = p.n_mt * p.n_nt;
   g = tile / per_g;
   const int rem = tile - g * per_g;
@@ -207,10 +218,22 @@ __global__ void __launch_bounds__(kThreads, 1)
   const uint32_t sH = base + C::kHaloOff;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  // this CTA's first tile and the tile stride (pair tiles when multicasting weights)
+  const int cta0 = p.mc ? (int)(blockIdx.x >> 1) : (int)blockIdx.x;
+  const int ncta = p.mc ? (int)(gridDim.x >> 1) : (int)gridDim.x;
+  const uint32_t crank = p.mc ? (blockIdx.x & 1u) : 0u;
+  // weight k-block kb of N rows [row0, row0 + BN) into ring stage `stage` (multicast: this CTA's half)
+  auto load_b = [&](int stage, int kb, int row0) {
+    if (p.mc)
+      tma_load_2d_mc(sB + stage * C::kBBytes + crank * (BN / 2) * 128, &tmap_w, kb * BK, row0 + (int)crank * (BN / 2),
+                     &full[stage], (uint16_t)3);
+    else
+      tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, row0, &full[stage]);
+  };
   if (threadIdx.x == 0) {
     for (int i = 0; i < S; ++i) {
       mbar_init(&full[i], a_by_tma(AMODE) ? 1 : 128 + 1);
-      mbar_init(&empty[i], 1);
+      mbar_init(&empty[i], p.mc ? 2 : 1);  // multicast: both CTAs' MMAs must release the stage
     }
     for (int i = 0; i < NACC; ++i) {
       mbar_init(&tfull[i], 1);
@@ -230,6 +253,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   if (warp == 4) tmem_alloc(tmem_slot, C::kTmemCols);
   tc_fence_before();
   __syncthreads();
+  if (p.mc) cluster_sync_all();  // the partner's barriers are initialised before any multicast reaches them
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
 
@@ -239,7 +263,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       // resident weights: the B slice of this CTA's (fixed) N tile, once
       if (threadIdx.x == 0) {
         int m0, nt, g;
-        decode_tile(p, blockIdx.x, m0, nt, g);
+        decode_tile(p, cta0, m0, nt, g);
         mbar_arrive_expect_tx(wres, p.nkb * C::kBBytes);
         for (int kb = 0; kb < p.nkb; ++kb)
           tma_load_2d(sR + kb * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + nt * BN, wres);
@@ -248,7 +272,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     if constexpr (AMODE == A_TMA) {
       if (threadIdx.x == 0) {
         uint32_t gk = 0;
-        for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x) {
+        for (int tile = cta0; tile < p.n_tiles; tile += ncta) {
           int m0, nt, g;
           decode_tile(p, tile, m0, nt, g);
           const int n0 = nt * BN;
@@ -257,7 +281,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
             mbar_arrive_expect_tx(&full[stage], C::kStageBytes);
             tma_load_2d(sA + stage * C::kABytes, &tmap_a, g * p.Cg_in + kb * BK, m0, &full[stage]);
-            if constexpr (!BRES) tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
+            if constexpr (!BRES) load_b(stage, kb, g * p.Cg_out + n0);
           }
         }
       }
@@ -265,7 +289,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (threadIdx.x == 0) {
         const int hw = p.Ho * p.Wo;
         uint32_t gk = 0;
-        for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x) {
+        for (int tile = cta0; tile < p.n_tiles; tile += ncta) {
           int m0, nt, g;
           decode_tile(p, tile, m0, nt, g);
           const int n0 = nt * BN;
@@ -282,7 +306,7 @@ __global__ void __launch_bounds__(kThreads, 1)
                                  nimg, 0, 0, &full[stage]);
             else
               tma_load_2d(sA + stage * C::kABytes, &tmap_r, (kb - p.nkb1) * BK, m0, &full[stage]);
-            if constexpr (!BRES) tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, n0, &full[stage]);
+            if constexpr (!BRES) load_b(stage, kb, n0);
           }
         }
       }
@@ -290,7 +314,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (threadIdx.x == 0) {
         uint32_t gk = 0, it = 0;
         const uint32_t box_bytes = (uint32_t)p.hrows * p.Wp * 128u;
-        for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x, ++it) {
+        for (int tile = cta0; tile < p.n_tiles; tile += ncta, ++it) {
           int m0, nt, g;
           decode_tile(p, tile, m0, nt, g);
           const int mt = m0 / BM, nimg = mt / p.mt_per_img;
@@ -311,7 +335,7 @@ __global__ void __launch_bounds__(kThreads, 1)
               const int stage = gk % S;
               if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
               mbar_arrive_expect_tx(&full[stage], C::kBBytes);
-              tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, 0, &full[stage]);
+              load_b(stage, kb, 0);
             }
           }
         }
@@ -322,7 +346,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       // 128-byte windows of input row p + r for q = 0..127 (q >= Wo out of bounds -> zeros).
       if (threadIdx.x == 0) {
         uint32_t gk = 0;
-        for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x) {
+        for (int tile = cta0; tile < p.n_tiles; tile += ncta) {
           int m0, nt, g;
           decode_tile(p, tile, m0, nt, g);
           const int n0 = nt * BN;
@@ -333,7 +357,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
             mbar_arrive_expect_tx(&full[stage], C::kABytes + C::kBBytes);
             tma_load_4d(sA + stage * C::kABytes, &tmap_a, 0, 0, ho + kb, nimg, &full[stage]);
-            tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
+            load_b(stage, kb, g * p.Cg_out + n0);
           }
         }
       }
@@ -345,7 +369,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int hw = p.Ho * p.Wo;
         const int RS = p.R * p.S;
         uint32_t gk = 0;
-        for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x) {
+        for (int tile = cta0; tile < p.n_tiles; tile += ncta) {
           int m0, nt, g;
           decode_tile(p, tile, m0, nt, g);
           const int n0 = nt * BN;
@@ -364,7 +388,7 @@ __global__ void __launch_bounds__(kThreads, 1)
               tma_load_im2col_4d(sA + stage * C::kABytes + j * 2048, &tmap_a, 0, w0, h0, nimg, (uint16_t)s,
                                  (uint16_t)r, &full[stage]);
             }
-            tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
+            load_b(stage, kb, g * p.Cg_out + n0);
           }
         }
       }
@@ -375,7 +399,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int cblocks = p.Cg_in / BK;
         const int hw = p.Ho * p.Wo;
         uint32_t gk = 0;
-        for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x) {
+        for (int tile = cta0; tile < p.n_tiles; tile += ncta) {
           int m0, nt, g;
           decode_tile(p, tile, m0, nt, g);
           const int n0 = nt * BN;
@@ -389,7 +413,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             mbar_arrive_expect_tx(&full[stage], C::kABytes + C::kBBytes);
             tma_load_im2col_4d(sA + stage * C::kABytes, &tmap_a, g * p.Cg_in + cb * BK, w0, h0, nimg, (uint16_t)s,
                                (uint16_t)r, &full[stage]);
-            tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
+            load_b(stage, kb, g * p.Cg_out + n0);
             if (++cb == cblocks) {
               cb = 0;
               if (++s == p.S) {
@@ -407,7 +431,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       const int CC = p.Cg_in >> 3;
       const int hw = p.Ho * p.Wo;
       uint32_t gk = 0;
-      for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x) {
+      for (int tile = cta0; tile < p.n_tiles; tile += ncta) {
         int m0, nt, g;
         decode_tile(p, tile, m0, nt, g);
         const int n0 = nt * BN;
@@ -428,7 +452,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
           if (t == 0) {
             mbar_arrive_expect_tx(&full[stage], C::kBBytes);
-            tma_load_2d(sB + stage * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + n0, &full[stage]);
+            load_b(stage, kb, g * p.Cg_out + n0);
           }
           const uint32_t dst = sA + stage * C::kABytes + arow;
           if constexpr (AMODE == A_GATHER_FAST) {
@@ -504,8 +528,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         // decode and commits sit between pairs, not between every 36 MMAs (measured: the tensor queue drains
         // during that gap; issue-bound at 2620 cycles per 1728-cycle tile).  The producer and the epilogue
         // still work per tile.
-        for (int tile = blockIdx.x; tile < p.n_tiles; tile += 2 * gridDim.x, it += 2) {
-          const int tiles[2] = {tile, tile + (int)gridDim.x};
+        for (int tile = cta0; tile < p.n_tiles; tile += 2 * ncta, it += 2) {
+          const int tiles[2] = {tile, tile + ncta};
           const int nt2 = tiles[1] < p.n_tiles ? 2 : 1;
           uint32_t alo[2], accs[2], hbs[2];
           if (prof_mma) tA = clock64();
@@ -555,7 +579,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           if (prof_mma) c_iss += clock64() - tA;
         }
       } else
-      for (int tile = blockIdx.x; tile < p.n_tiles; tile += gridDim.x, ++it) {
+      for (int tile = cta0; tile < p.n_tiles; tile += ncta, ++it) {
         const uint32_t acc = it % NACC, use = it / NACC;
         if (prof_mma) tA = clock64();
         if (it >= (uint32_t)NACC) mbar_wait(&tempty[acc], (use - 1) & 1);
@@ -619,7 +643,10 @@ __global__ void __launch_bounds__(kThreads, 1)
             tc_mma_bf16_warp(tacc, da + 4, db + 4, idesc, 1u);
             tc_mma_bf16_warp(tacc, da + 6, db + 6, idesc, 1u);
           }
-          if constexpr (kRing) tc_commit_warp(&empty[stage]);
+          if constexpr (kRing) {
+            if (p.mc) tc_commit_mc_warp(&empty[stage], (uint16_t)3);
+            else tc_commit_warp(&empty[stage]);
+          }
           ++gk;
         };
         {
@@ -662,8 +689,8 @@ __global__ void __launch_bounds__(kThreads, 1)
     int loaded0 = -1, loaded1 = -1;  // N offset whose scale / shift each smem buffer holds
     const int tstep = SPLIT ? 2 : 1;
     uint32_t it = SPLIT ? grp : 0;
-    for (int tile = blockIdx.x + (SPLIT ? grp * (int)gridDim.x : 0); tile < p.n_tiles;
-         tile += tstep * gridDim.x, it += tstep) {
+    for (int tile = cta0 + (SPLIT ? grp * ncta : 0); tile < p.n_tiles;
+         tile += tstep * ncta, it += tstep) {
       const uint32_t acc = it % NACC, use = it / NACC;
       int m0, nt, g;
       decode_tile(p, tile, m0, nt, g);
@@ -691,7 +718,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             if (NB == 2) {
               if (it == 0) issue_res(tile, 0);
               // prefetch the next tile's residual into the other buffer once its stores (tile it-1) read it
-              const int next = tile + gridDim.x;
+              const int next = tile + ncta;
               if (next < p.n_tiles) {
                 bulk_wait_read0();
                 issue_res(next, ob ^ 1);
@@ -699,7 +726,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             } else if (it == 0) {
               // NB >= 3: the first NB - 1 residual tiles now; the rest at the end of each tile (below)
               for (int j = 0; j < NB - 1; ++j)
-                if (tile + j * (int)gridDim.x < p.n_tiles) issue_res(tile + j * gridDim.x, j);
+                if (tile + j * ncta < p.n_tiles) issue_res(tile + j * ncta, j);
             }
           } else {
             bulk_wait_read<NB - 1>();  // tile it-NB (same buffer) has been read by its stores
@@ -728,8 +755,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int mt = m0 / BM, nimg = mt / p.mt_per_img;
         const int pp = (mt - nimg * p.mt_per_img) * BM + row;
         const int ho = pp / p.Wp, wo = pp - ho * p.Wp;
-        rvalid = ho < p.Ho && wo < p.Wo;
         mo = (nimg * p.Ho + ho) * p.Wo + wo;
+        rvalid = ho < p.Ho && wo < p.Wo && mo < p.M;  // (a multicast phantom tile lies past the last image)
       }
       const size_t off = (size_t)(rvalid ? mo : 0) * p.Cout + ng0;
       constexpr int kChunks = SPLIT ? BN / 32 : BN / 64;  // 32-column chunks per warp
@@ -844,7 +871,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           if (NB >= 3 && has_res) {
             // buffer (it + NB - 1) % NB held tile it-1's output: once its stores have read it, prefetch
             // the residual of this CTA's tile it + NB - 1 there (latency hidden behind ~NB - 2 tiles)
-            const int ahead = tile + (NB - 1) * (int)gridDim.x;
+            const int ahead = tile + (NB - 1) * ncta;
             if (ahead < p.n_tiles) {
               bulk_wait_read<1>();
               issue_res(ahead, (it + NB - 1) % NB);
@@ -900,6 +927,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   }
   tc_fence_before();
   __syncthreads();
+  if (p.mc) cluster_sync_all();  // no multicast write or commit arrival may target an exited partner
   if (warp == 4) tmem_dealloc(tmem_base, C::kTmemCols);
 }
 
@@ -992,6 +1020,22 @@ static const int g_conv_dbg = [] {
   return e ? atoi(e) : 0;
 }();
 // VISTA_WRES=0 disables the resident-weight launches (A/B measurements)
+// weight multicast across CTA pairs for streamed-weight launches (ConvParams::mc); VISTA_MC=0 disables
+static const bool g_mc_enabled = [] {
+  const char* e = getenv("VISTA_MC");
+  return !(e && e[0] == '0');
+}();
+// measured: the halo 3x3 (res3, 28x28x128) ran 5 % slower with multicast pairs (774 vs 814 TF/s, same box);
+// VISTA_MC_HALO=1 enables it for A/B runs
+static const bool g_mc_halo = [] {
+  const char* e = getenv("VISTA_MC_HALO");
+  return e && e[0] == '1';
+}();
+static bool use_mc(const ConvLayer& L, int amode, int rkb, const ConvParams& p) {
+  return g_mc_enabled && rkb == 0 && L.groups == 1 && L.BN >= 64 && p.n_mt >= 2 &&
+         (amode == A_TMA || amode == A_IM2COL || amode == A_CAT || (amode == A_HALO && g_mc_halo)) &&
+         (int64_t)p.n_nt * ((p.n_mt + 1) / 2) >= num_sms() / 2;
+}
 static const bool g_wres_enabled = [] {
   const char* e = getenv("VISTA_WRES");
   return !(e && e[0] == '0');
@@ -1066,6 +1110,7 @@ void conv_layer_init(ConvLayer& L, const std::vector<uint16_t>& w, int Cin_real,
   VCHECK(cudaMemcpy(L.scale, scale.data(), L.Cout * sizeof(float), cudaMemcpyHostToDevice));
   VCHECK(cudaMemcpy(L.shift, shift.data(), L.Cout * sizeof(float), cudaMemcpyHostToDevice));
   make_tmap(&L.tmap_w, L.w, (uint64_t)L.Kp, (uint64_t)L.Cout, (uint32_t)L.BN);
+  make_tmap(&L.tmap_w_half, L.w, (uint64_t)L.Kp, (uint64_t)L.Cout, (uint32_t)(L.BN / 2));
 }
 
 void conv_layer_free(ConvLayer& L) {
@@ -1086,6 +1131,25 @@ static void launch_t(const ConvLayer& L, const CUtensorMap& ta, const CUtensorMa
   if (!attr_set) {
     VCHECK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
     attr_set = true;
+  }
+  if (p.mc) {  // clusters of two CTAs walking pair tiles (see ConvParams::mc)
+    if (RKB > 0) fail(1, "conv: multicast with resident weights");
+    const int pairs = std::min(p.n_tiles, num_sms() / 2);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(2 * pairs, 1, 1);
+    cfg.blockDim = dim3(kThreads, 1, 1);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    VCHECK(cudaLaunchKernelEx(&cfg, kern, L.tmap_w_half, ta, ty, tr, p));
+    LAUNCHED();
+    return;
   }
   int grid = p.n_tiles < num_sms() ? p.n_tiles : num_sms();
   if (RKB > 0) {  // every CTA keeps one N tile: grid a multiple of the N-tile count (groups == 1)
@@ -1273,6 +1337,10 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
     if (amode == A_HALO && L.BN == 64 && p.nkb == 9) rkb = 9;
     else if (amode == A_TMA && tma_epi && L.BN <= 128 && p.nkb <= 4) rkb = 4;
   }
+  if (!fuse_tap && use_mc(L, amode, rkb, p)) {
+    p.mc = 1;
+    p.n_tiles = p.n_nt * ((p.n_mt + 1) / 2);
+  }
   unsigned long long* dbgb = nullptr;
   if (p.dbg & 8) {
     VCHECK(cudaMalloc(&dbgb, 148 * 8 * 8));
@@ -1301,9 +1369,9 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   }
   char label[160] = {0};
   if (prof_labels())
-    snprintf(label, sizeof(label), "conv R%d S%d s%d g%d Cin%d Cout%d HxW%dx%d M%d K%d BN%d amode%d epi%d nb%d rkb%d tiles%d%s", L.R,
-             L.S, L.stride, L.groups, L.Cin, L.Cout, H, W, p.M, L.K, L.BN, amode, tma_epi ? 1 : 0, nb, rkb, p.n_tiles,
-             res ? " res" : "");
+    snprintf(label, sizeof(label), "conv R%d S%d s%d g%d Cin%d Cout%d HxW%dx%d M%d K%d BN%d amode%d epi%d nb%d rkb%d mc%d tiles%d%s",
+             L.R, L.S, L.stride, L.groups, L.Cin, L.Cout, H, W, p.M, L.K, L.BN, amode, tma_epi ? 1 : 0, nb, rkb, p.mc,
+             p.n_tiles, res ? " res" : "");
   prof_end(st, 0, flops, bytes, label);
   if (dbgb) {
     unsigned long long h[148 * 8];
@@ -1371,6 +1439,10 @@ void conv_cat_forward(const ConvLayer& L, int Cx, const bf16* b, const bf16* x, 
   else ty = L.tmap_w;  // unused
   const int rkb = (g_wres_enabled && tma_epi && L.BN <= 128 && p.nkb <= 4 && p.n_nt <= num_sms() &&
                    p.n_tiles >= num_sms()) ? 4 : 0;
+  if (use_mc(L, A_CAT, rkb, p)) {
+    p.mc = 1;
+    p.n_tiles = p.n_nt * ((p.n_mt + 1) / 2);
+  }
   const double flops = 2.0 * (double)M * L.Cout * L.K_alg;
   const double bytes = 2.0 * ((double)M * (Kb + Cx + L.Cout) + (double)L.Cout * L.Kp);
   prof_begin(st);
@@ -1385,8 +1457,8 @@ void conv_cat_forward(const ConvLayer& L, int Cx, const bf16* b, const bf16* x, 
   }
   char label[160] = {0};
   if (prof_labels())
-    snprintf(label, sizeof(label), "conv_cat c+proj s%d Cb%d Cx%d Cout%d HxW%dx%d K%d BN%d epi%d rkb%d", stride, Kb,
-             Cx, L.Cout, p.Ho, p.Wo, L.K, L.BN, tma_epi ? 1 : 0, rkb);
+    snprintf(label, sizeof(label), "conv_cat c+proj s%d Cb%d Cx%d Cout%d HxW%dx%d K%d BN%d epi%d rkb%d mc%d", stride,
+             Kb, Cx, L.Cout, p.Ho, p.Wo, L.K, L.BN, tma_epi ? 1 : 0, rkb, p.mc);
   prof_end(st, 0, flops, bytes, label);
 }
 

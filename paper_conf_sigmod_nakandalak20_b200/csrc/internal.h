@@ -48,6 +48,7 @@ struct ConvLayer {
   float* scale = nullptr;    // [Cout]
   float* shift = nullptr;    // [Cout]
   CUtensorMap tmap_w;        // box {64, BN}, SWIZZLE_128B
+  CUtensorMap tmap_w_half;   // box {64, BN / 2}: per-CTA half of a k-block multicast to a CTA pair
 };
 
 // Builds the padded weight matrix on the device (from OHWI bf16 on the host, Cin_real <= Cin),

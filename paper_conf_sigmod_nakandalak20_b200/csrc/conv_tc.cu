@@ -1020,20 +1020,16 @@ static const int g_conv_dbg = [] {
   return e ? atoi(e) : 0;
 }();
 // VISTA_WRES=0 disables the resident-weight launches (A/B measurements)
-// weight multicast across CTA pairs for streamed-weight launches (ConvParams::mc); VISTA_MC=0 disables
-static const bool g_mc_enabled = [] {
-  const char* e = getenv("VISTA_MC");
-  return !(e && e[0] == '0');
-}();
-// measured: the halo 3x3 (res3, 28x28x128) ran 5 % slower with multicast pairs (774 vs 814 TF/s, same box);
-// VISTA_MC_HALO=1 enables it for A/B runs
-static const bool g_mc_halo = [] {
-  const char* e = getenv("VISTA_MC_HALO");
-  return e && e[0] == '1';
-}();
+// weight multicast across CTA pairs for streamed-weight launches (ConvParams::mc); VISTA_MC=0 disables.
+// The halo 3x3 ran 5 % slower with multicast pairs (res3 28x28x128: 774 vs 814 TF/s, same box), so it stays
+// unicast unless VISTA_MC_HALO=1.  Read per launch (tests switch them within one process).
+static bool env_flag(const char* name, bool dflt) {
+  const char* e = getenv(name);
+  return e && *e ? e[0] == '1' : dflt;
+}
 static bool use_mc(const ConvLayer& L, int amode, int rkb, const ConvParams& p) {
-  return g_mc_enabled && rkb == 0 && L.groups == 1 && L.BN >= 64 && p.n_mt >= 2 &&
-         (amode == A_TMA || amode == A_IM2COL || amode == A_CAT || (amode == A_HALO && g_mc_halo)) &&
+  return env_flag("VISTA_MC", true) && rkb == 0 && L.groups == 1 && L.BN >= 64 && p.n_mt >= 2 &&
+         (amode == A_TMA || amode == A_IM2COL || amode == A_CAT || (amode == A_HALO && env_flag("VISTA_MC_HALO", false))) &&
          (int64_t)p.n_nt * ((p.n_mt + 1) / 2) >= num_sms() / 2;
 }
 static const bool g_wres_enabled = [] {

@@ -69,8 +69,9 @@ bool make_rowview_tmap(CUtensorMap* m, const void* x, int N, int H, int W, int C
 bool make_plain_tmap(CUtensorMap* m, const void* ptr, int cols, int rows);
 // Two chained 1x1 convs of consecutive ResNet units (res_chain.cu): out = ReLU(BN_c(b * Wc) + res) and
 // a_next = ReLU(BN_a(out * Wa)) in one kernel, bit-identical to two conv_forward calls.
-bool res_chain_supported(const ConvLayer& Lc, const ConvLayer& La);
-void res_chain_forward(const ConvLayer& Lc, const ConvLayer& La, const bf16* b, const bf16* res, bf16* out,
+// La == nullptr: the closing conv alone (no chained opening conv, a_next unused)
+bool res_chain_supported(const ConvLayer& Lc, const ConvLayer* La);
+void res_chain_forward(const ConvLayer& Lc, const ConvLayer* La, const bf16* b, const bf16* res, bf16* out,
                        bf16* a_next, int N, int H, int W, cudaStream_t st);
 // ResNet50 stem: conv1 (s2d row view) + BN + ReLU + pool1 3x3/2 in one kernel (conv1_pool.cu):
 // x bf16 [N, 117, 117, 16] space-to-depth input -> y bf16 [N, 56, 56, 64], bit-identical to

@@ -50,6 +50,7 @@ struct RCParams {
   const float* sc_a;
   const float* sh_a;
   int M, n_mt;
+  int has_a;  // 0: closing conv only (last unit of a stage: no chained opening conv, no a_next)
 };
 
 template <int MID, int V>
@@ -94,7 +95,7 @@ __global__ void __launch_bounds__(kThr, 1)
     for (int i = 0; i < NB; ++i) {
       mbar_init(&rfull[i], 1);
       mbar_init(&oready[i], 1);
-      mbar_init(&ofree[i], 2);
+      mbar_init(&ofree[i], p.has_a ? 2 : 1);
     }
     for (int i = 0; i < WS; ++i) {
       mbar_init(&wfull[i], 1);
@@ -157,7 +158,7 @@ __global__ void __launch_bounds__(kThr, 1)
             push_c(j + 1);
             push_res(m0, j + 1);
           }
-          push_a(j);
+          if (p.has_a) push_a(j);
         }
       }
     }
@@ -217,7 +218,7 @@ __global__ void __launch_bounds__(kThr, 1)
 #pragma unroll
       for (int j = 0; j < NCH; ++j) {
         if (j + 1 < NCH) issue_c(j + 1);
-        issue_a(j);
+        if (p.has_a) issue_a(j);
       }
     }
   } else {
@@ -273,7 +274,7 @@ __global__ void __launch_bounds__(kThr, 1)
         if (et == 0) {
           // the previous chunk's store must have read its buffer before that buffer is refilled
           if (qq >= 1) {
-            if (j == 0) bulk_wait_read<1>();  // the previous tile's a_next store was committed after it
+            if (j == 0 && p.has_a) bulk_wait_read<1>();  // the previous tile's a_next store was committed after it
             else bulk_wait_read<0>();
             mbar_arrive(&ofree[(qq - 1) % NB]);
           }
@@ -283,6 +284,7 @@ __global__ void __launch_bounds__(kThr, 1)
           bulk_commit();
         }
       }
+      if (!p.has_a) continue;
       // ---- a_next = ReLU(BN_a(acc_a)) ----
       mbar_wait(tfull_a, it & 1);
       tc_fence_after();
@@ -329,25 +331,27 @@ __global__ void __launch_bounds__(kThr, 1)
 
 }  // namespace
 
-bool res_chain_supported(const ConvLayer& Lc, const ConvLayer& La) {
+bool res_chain_supported(const ConvLayer& Lc, const ConvLayer* La) {
   const int mid = Lc.Cin;
-  return (mid == 64 || mid == 128) && Lc.R == 1 && Lc.S == 1 && Lc.stride == 1 && Lc.pad == 0 && Lc.groups == 1 &&
-         Lc.Cout == 4 * mid && Lc.BN == 128 && Lc.relu && La.R == 1 && La.S == 1 && La.stride == 1 && La.pad == 0 &&
-         La.groups == 1 && La.Cin == 4 * mid && La.Cout == mid && La.BN == mid && La.relu;
+  const bool c_ok = (mid == 64 || mid == 128) && Lc.R == 1 && Lc.S == 1 && Lc.stride == 1 && Lc.pad == 0 &&
+                    Lc.groups == 1 && Lc.Cout == 4 * mid && Lc.BN == 128 && Lc.relu;
+  return c_ok && (!La || (La->R == 1 && La->S == 1 && La->stride == 1 && La->pad == 0 && La->groups == 1 &&
+                          La->Cin == 4 * mid && La->Cout == mid && La->BN == mid && La->relu));
 }
 
 template <int MID, int V>
-static void launch_chain(const ConvLayer& Lc, const ConvLayer& La, const bf16* b, const bf16* res, bf16* out,
+static void launch_chain(const ConvLayer& Lc, const ConvLayer* La, const bf16* b, const bf16* res, bf16* out,
                          bf16* a_next, int M, cudaStream_t st) {
   CUtensorMap tb, tr, to, ta;
   if (!make_plain_tmap(&tb, b, MID, M) || !make_plain_tmap(&tr, res, 4 * MID, M) ||
-      !make_plain_tmap(&to, out, 4 * MID, M) || !make_plain_tmap(&ta, a_next, MID, M))
+      !make_plain_tmap(&to, out, 4 * MID, M) || !make_plain_tmap(&ta, La ? a_next : b, MID, M))
     fail(5, "res_chain: tensor map encoding failed");
   RCParams p;
+  p.has_a = La ? 1 : 0;
   p.sc_c = Lc.scale;
   p.sh_c = Lc.shift;
-  p.sc_a = La.scale;
-  p.sh_a = La.shift;
+  p.sc_a = La ? La->scale : Lc.scale;  // (unused without a_next; any MID-long device array)
+  p.sh_a = La ? La->shift : Lc.shift;
   p.M = M;
   p.n_mt = (M + BMr - 1) / BMr;
   static bool attr = false;
@@ -356,11 +360,11 @@ static void launch_chain(const ConvLayer& Lc, const ConvLayer& La, const bf16* b
     attr = true;
   }
   const int grid = p.n_mt < num_sms() ? p.n_mt : num_sms();
-  res_chain_kernel<MID, V><<<grid, kThr, RC<MID, V>::kSmem, st>>>(tb, tr, to, ta, Lc.tmap_w, La.tmap_w, p);
+  res_chain_kernel<MID, V><<<grid, kThr, RC<MID, V>::kSmem, st>>>(tb, tr, to, ta, Lc.tmap_w, La ? La->tmap_w : Lc.tmap_w, p);
   LAUNCHED();
 }
 
-void res_chain_forward(const ConvLayer& Lc, const ConvLayer& La, const bf16* b, const bf16* res, bf16* out,
+void res_chain_forward(const ConvLayer& Lc, const ConvLayer* La, const bf16* b, const bf16* res, bf16* out,
                        bf16* a_next, int N, int H, int W, cudaStream_t st) {
   const int64_t M64 = (int64_t)N * H * W;
   if (M64 <= 0) return;
@@ -382,10 +386,10 @@ void res_chain_forward(const ConvLayer& Lc, const ConvLayer& La, const bf16* b, 
     if (v & 2) launch_chain<128, 1>(Lc, La, b, res, out, a_next, M, st);
     else launch_chain<128, 0>(Lc, La, b, res, out, a_next, M, st);
   }
-  const double flops = 2.0 * M64 * (double)(4 * mid) * mid * 2;  // both GEMMs
-  const double bytes = 2.0 * M64 * ((double)mid + 4 * mid + 4 * mid + mid) + 2.0 * 8 * mid * mid;
+  const double flops = 2.0 * M64 * (double)(4 * mid) * mid * (La ? 2 : 1);  // both GEMMs (or the c GEMM)
+  const double bytes = 2.0 * M64 * ((double)mid + 4 * mid + 4 * mid + (La ? mid : 0)) + 2.0 * (La ? 8 : 4) * mid * mid;
   char label[96] = {0};
-  if (prof_labels()) snprintf(label, sizeof(label), "res_chain c+a MID%d HxW%dx%d", mid, H, W);
+  if (prof_labels()) snprintf(label, sizeof(label), "res_chain %s MID%d HxW%dx%d", La ? "c+a" : "c", mid, H, W);
   prof_end(st, 0, flops, bytes, prof_labels() ? label : nullptr);
 }
 

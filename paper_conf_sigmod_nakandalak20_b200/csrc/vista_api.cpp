@@ -641,13 +641,21 @@ bool run_ops(vista_ctx* c, int t, const void* in_ptr, void* out_ptr, int nb, voi
       if (op.kind == OP_CONV && op.res >= 0 && c->fuse_chain && oi + 1 < S.ops.size()) {
         const OpDesc& o2 = S.ops[oi + 1];
         if (o2.kind == OP_CONV && o2.in == op.out && o2.res < 0 && o2.out != BUF_OUT && op.out != o2.out &&
-            res_chain_supported(c->convs[op.layer], c->convs[o2.layer]) && o2.H == op.Ho && o2.W == op.Wo &&
+            res_chain_supported(c->convs[op.layer], &c->convs[o2.layer]) && o2.H == op.Ho && o2.W == op.Wo &&
             op.Ho == op.H && op.Wo == op.W) {
-          res_chain_forward(c->convs[op.layer], c->convs[o2.layer], in, reinterpret_cast<const bf16*>(slot[op.res]),
+          res_chain_forward(c->convs[op.layer], &c->convs[o2.layer], in, reinterpret_cast<const bf16*>(slot[op.res]),
                             out, reinterpret_cast<bf16*>(slot[o2.out]), nb, op.H, op.W, c->stream);
           ++oi;
           continue;
         }
+      }
+      // a stage's last closing conv (nothing to chain): the chain kernel's c half (its residual pipeline
+      // measured ~6 TB/s at res2 vs 4.6 for conv_tc's TMA epilogue on the same shape)
+      if (op.kind == OP_CONV && op.res >= 0 && c->fuse_chain && !(tapf && op.out == BUF_OUT) &&
+          res_chain_supported(c->convs[op.layer], nullptr) && op.Ho == op.H && op.Wo == op.W) {
+        res_chain_forward(c->convs[op.layer], nullptr, in, reinterpret_cast<const bf16*>(slot[op.res]), out, nullptr,
+                          nb, op.H, op.W, c->stream);
+        continue;
       }
       switch (op.kind) {
         case OP_INGEST:

@@ -230,7 +230,8 @@ def test_resnet_stem_fused_bit_identical(monkeypatch):
 
 def test_resnet_chain_fused_bit_identical(monkeypatch):
     # the closing 1x1 conv of a unit and the next unit's opening 1x1 conv run as one kernel (res_chain.cu,
-    # MID = 64 / 128) by default; VISTA_FUSE_CHAIN=0 runs them as two conv_tc launches: same bits
+    # MID = 64 / 128) by default, and a stage's last closing conv runs as the chain kernel's c half;
+    # VISTA_FUSE_CHAIN=0 runs them as conv_tc launches: same bits
     tab = gen.make_tables(37, 8)  # M = 37 * 3136 pixels: partial last 128-row tile
     out = {}
     for fuse in ("1", "0"):
@@ -261,6 +262,27 @@ def test_resnet_projection_fused(monkeypatch):
         assert normwise_rows(a[:6], F[k]).max() <= 2e-2, (k, normwise_rows(a[:6], F[k]).max())
         assert normwise_rows(a, b).max() <= 2e-2
         assert not np.array_equal(a, b) or k == 4  # the fused path really ran
+
+
+def test_weight_multicast_bit_identical(monkeypatch):
+    # 2-CTA weight multicast (ConvParams::mc) engages only for launches with >= 74 pair tiles: 600 images put
+    # the res4 / res5 / projection-unit launches above that, and res4's 919 M tiles give rank 1 of the last
+    # pair a phantom tile past M.  Multicast changes where the weight bytes come from, not the MMA order, so
+    # every bit of MM_l must agree with VISTA_MC=0; three sampled images are also held to the oracle.
+    tab = gen.make_tables(600, 8)
+    out, feats = {}, None
+    for mc in ("1", "0"):
+        monkeypatch.setenv("VISTA_MC", mc)
+        v = run_gpu(2, [0, 1, 2, 3, 4], tab, 8, iters=1, micro_batch=600)
+        out[mc] = [v.features(k)["mm"].view(torch.int16).cpu().clone() for k in range(5)]
+        if mc == "1":
+            feats = [v.features(k)["features"].to(torch.float64).cpu().numpy()[:3] for k in range(5)]
+        v.close()
+    for a, b in zip(out["1"], out["0"]):
+        assert torch.equal(a, b)
+    F, _ = oracle.features(oracle.RESNET50, WSEED, tab.images[:3], taps=[0, 1, 2, 3, 4])
+    for k in range(5):
+        assert normwise_rows(feats[k], F[k]).max() <= 2e-2
 
 
 @pytest.mark.parametrize("cnn,taps,n,d_s,chunked", [(0, [1, 2, 3], 10, 8, False), (2, [1, 3, 4], 6, 16, False),

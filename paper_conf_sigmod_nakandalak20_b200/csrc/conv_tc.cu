@@ -71,6 +71,7 @@ struct ConvParams {
   // rank r takes M tile 2 * pair_m + r) in lockstep, and each CTA TMA-loads half of every weight (B) k-block
   // and multicasts it to both, halving the per-SM L2 -> shared-memory weight traffic of streamed-B layers
   int mc;
+  int segs;  // A_ROWVIEW: 128-pixel segments per output row (1 unless Wo > 128)
   // fused tap g_l (PAPER.md:369 fn 4): per-image 2x2-grid channel maxima of the (post-ReLU, >= 0)
   // output, accumulated as fp32 bit patterns with red.global.max.u32 into tapf[n][4][Cout]
   unsigned int* tapf;
@@ -350,14 +351,15 @@ __global__ void __launch_bounds__(kThreads, 1)
           int m0, nt, g;
           decode_tile(p, tile, m0, nt, g);
           const int n0 = nt * BN;
-          const int rr = m0 / BM;  // output row index n * Ho + p
+          const int rs = m0 / BM;  // (output row n * Ho + p) * segs + segment
+          const int rr = rs / p.segs, seg = rs - rr * p.segs;
           const int nimg = rr / p.Ho, ho = rr - nimg * p.Ho;
           for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
             const int stage = gk % S;
             if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
-            mbar_arrive_expect_tx(&full[stage], C::kABytes + C::kBBytes);
-            tma_load_4d(sA + stage * C::kABytes, &tmap_a, 0, 0, ho + kb, nimg, &full[stage]);
-            load_b(stage, kb, g * p.Cg_out + n0);
+            mbar_arrive_expect_tx(&full[stage], C::kStageBytes);
+            tma_load_4d(sA + stage * C::kABytes, &tmap_a, 0, seg * BM, ho + kb, nimg, &full[stage]);
+            if constexpr (!BRES) load_b(stage, kb, g * p.Cg_out + n0);
           }
         }
       }
@@ -863,7 +865,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           const int nsub = (nvalid_tile + 63) / 64;
           for (int st = 0; st < nsub; ++st) {
             if constexpr (AMODE == A_ROWVIEW)  // 3-D output map {C, Wo, rows}: q >= Wo clipped
-              tma_store_3d(&tmap_y, ng0 + st * 64, 0, m0 / BM, sOb + st * BM * 128);
+              tma_store_3d(&tmap_y, ng0 + st * 64, (m0 / BM) % p.segs * BM, (m0 / BM) / p.segs, sOb + st * BM * 128);
             else
               tma_store_2d(&tmap_y, ng0 + st * 64, m0, sOb + st * BM * 128);
           }
@@ -1021,14 +1023,15 @@ static const int g_conv_dbg = [] {
 }();
 // VISTA_WRES=0 disables the resident-weight launches (A/B measurements)
 // weight multicast across CTA pairs for streamed-weight launches (ConvParams::mc); VISTA_MC=0 disables.
-// The halo 3x3 ran 5 % slower with multicast pairs (res3 28x28x128: 774 vs 814 TF/s, same box), so it stays
-// unicast unless VISTA_MC_HALO=1.  Read per launch (tests switch them within one process).
+// Measured: 256-wide tiles gain (VGG conv3_x 1353 -> 1496, conv4_x 1454 -> 1598 TF/s, ResNet res5 3x3
+// 1452 -> 1557), 64/128-wide tiles lose (VGG conv1_2 437 -> 406, conv2_2 928 -> 841; ResNet res3 halo 3x3
+// 814 -> 774), so only BN = 256 launches multicast (the halo path additionally needs VISTA_MC_HALO=1).  Read per launch (tests switch them within one process).
 static bool env_flag(const char* name, bool dflt) {
   const char* e = getenv(name);
   return e && *e ? e[0] == '1' : dflt;
 }
 static bool use_mc(const ConvLayer& L, int amode, int rkb, const ConvParams& p) {
-  return env_flag("VISTA_MC", true) && rkb == 0 && L.groups == 1 && L.BN >= 64 && p.n_mt >= 2 &&
+  return env_flag("VISTA_MC", true) && rkb == 0 && L.groups == 1 && L.BN == 256 && p.n_mt >= 2 &&
          (amode == A_TMA || amode == A_IM2COL || amode == A_CAT || (amode == A_HALO && env_flag("VISTA_MC_HALO", false))) &&
          (int64_t)p.n_nt * ((p.n_mt + 1) / 2) >= num_sms() / 2;
 }
@@ -1056,6 +1059,20 @@ bool make_plain_tmap(CUtensorMap* m, const void* ptr, int cols, int rows) {
 
 // overlapping 4-D row view of an NHWC input with C * S == 64 (A_ROWVIEW): element (k, q, h, n) =
 // x[n, h, q + k / C, k % C] for q < Wo; box {64, 128, 1, 1}, 128B-swizzled (q >= Wo reads zeros)
+// zero-padded copy for the padded row view: xp[n, h, w] = x[n, h - pad, w - pad] inside, 0 elsewhere;
+// one 16-byte pixel (C = 8 bf16) per thread, xp rows Wpad pixels wide
+__global__ void pad_rows_kernel(const uint4* __restrict__ x, uint4* __restrict__ xp, int64_t total, int H, int W,
+                                int Hp, int Wpad, int pad) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int w = (int)(i % Wpad);
+    const int64_t t = i / Wpad;
+    const int h = (int)(t % Hp);
+    const int64_t n = t / Hp;
+    const int hs = h - pad, ws = w - pad;
+    xp[i] = (hs >= 0 && hs < H && ws >= 0 && ws < W) ? x[(n * H + hs) * W + ws] : make_uint4(0, 0, 0, 0);
+  }
+}
+
 bool make_rowview_tmap(CUtensorMap* m, const void* x, int N, int H, int W, int C, int Wo) {
   const cuuint64_t dims[4] = {(cuuint64_t)BK, (cuuint64_t)Wo, (cuuint64_t)H, (cuuint64_t)N};
   const cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)W * C * 2, (cuuint64_t)H * W * C * 2};
@@ -1183,6 +1200,12 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
     case A_IM2COL: launch_t<BN, A_IM2COL, TE, NB>(L, ta, ty, tr, p, st); break;
     case A_IM2COL_C8: launch_t<BN, A_IM2COL_C8, TE, NB>(L, ta, ty, tr, p, st); break;
     case A_ROWVIEW:
+      if constexpr (TE && BN <= 128) {
+        if (rkb == 4) {
+          launch_t<BN, A_ROWVIEW, TE, NB, 4>(L, ta, ty, tr, p, st);
+          break;
+        }
+      }
       if constexpr (TE) launch_t<BN, A_ROWVIEW, TE, NB>(L, ta, ty, tr, p, st);
       else fail(1, "conv: row-view mode needs the TMA epilogue");
       break;
@@ -1230,6 +1253,7 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   p.Cg_out = L.Cg_out;
   p.K = L.K;
   p.nkb = L.Kp / BK;
+  p.segs = 1;
   const int64_t M = (int64_t)N * p.Ho * p.Wo;
   if (M <= 0) return tapf == nullptr;
   if (M > INT32_MAX - BM) fail(1, "conv: M too large for one launch");
@@ -1256,6 +1280,37 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
       p.n_mt = N * p.Ho;  // one tile per output row; rows q >= Wo of a tile are padding
       p.M = p.n_mt * BM;
       p.n_tiles = p.n_mt * p.n_nt;
+    }
+  }
+  // padded row view (first layers with Cin = 8 and padding, e.g. VGG16 conv1_1 3x3 pad 1 at 227 wide): the
+  // cp.async gather is latency-bound there (one k-block group per 16 B per thread in flight, measured 1 TB/s),
+  // so the input is first copied into a zero-padded buffer whose rows are wide enough for every 8-pixel
+  // window, then read by the overlapping row view in ceil(Wo / 128) segments per output row
+  bf16* xpad = nullptr;
+  if (!rowview && L.row_mode && g_rowview_enabled && L.Cin == 8 && L.stride == 1 && L.pad > 0 && L.groups == 1 &&
+      !res && L.R <= 8 && L.Cout % 8 == 0 && !tapf) {
+    const int Hp = H + 2 * L.pad;
+    const int Wpad = std::max(W + 2 * L.pad, p.Wo + BK / L.Cin - 1);
+    const int64_t total = (int64_t)N * Hp * Wpad;
+    if (cudaMallocAsync((void**)&xpad, (size_t)total * 16, st) == cudaSuccess) {
+      pad_rows_kernel<<<num_sms() * 8, 256, 0, st>>>(reinterpret_cast<const uint4*>(x), reinterpret_cast<uint4*>(xpad),
+                                                     total, H, W, Hp, Wpad, L.pad);
+      LAUNCHED();
+      const int segs = (p.Wo + BM - 1) / BM;
+      const cuuint64_t odims[3] = {(cuuint64_t)L.Cout, (cuuint64_t)p.Wo, (cuuint64_t)N * p.Ho};
+      const cuuint64_t ostr[2] = {(cuuint64_t)L.Cout * 2, (cuuint64_t)p.Wo * L.Cout * 2};
+      const cuuint32_t obox[3] = {(cuuint32_t)BK, (cuuint32_t)BM, 1};
+      if (make_rowview_tmap(&ta, xpad, N, Hp, Wpad, L.Cin, p.Wo) &&
+          encode_nd(&ty, y, 3, odims, ostr, obox) == CUDA_SUCCESS) {
+        rowview = true;
+        p.segs = segs;
+        p.n_mt = N * p.Ho * segs;
+        p.M = p.n_mt * BM;
+        p.n_tiles = p.n_mt * p.n_nt;
+      }
+    } else {
+      cudaGetLastError();
+      xpad = nullptr;
     }
   }
   // halo mode: 3x3 stride-1 pad-1 ungrouped, one N tile, both halo buffers fit the compile-time budget
@@ -1331,7 +1386,7 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   int rkb = 0;
   if (g_wres_enabled && L.groups == 1 && p.n_nt <= num_sms() && p.n_tiles >= num_sms()) {
     if (amode == A_HALO && L.BN == 64 && p.nkb == 9) rkb = 9;
-    else if (amode == A_TMA && tma_epi && L.BN <= 128 && p.nkb <= 4) rkb = 4;
+    else if ((amode == A_TMA || amode == A_ROWVIEW) && tma_epi && L.BN <= 128 && p.nkb <= 4) rkb = 4;
   }
   if (!fuse_tap && use_mc(L, amode, rkb, p)) {
     p.mc = 1;
@@ -1363,11 +1418,12 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
     else if (L.BN == 128) launch_bn<128, false, 1>(L, amode, ta, ty, tr, p, st, rkb);
     else launch_bn<64, false, 1>(L, amode, ta, ty, tr, p, st, rkb);
   }
+  if (xpad) VCHECK(cudaFreeAsync(xpad, st));  // stream-ordered: after the conv has read it
   char label[160] = {0};
   if (prof_labels())
-    snprintf(label, sizeof(label), "conv R%d S%d s%d g%d Cin%d Cout%d HxW%dx%d M%d K%d BN%d amode%d epi%d nb%d rkb%d mc%d tiles%d%s",
+    snprintf(label, sizeof(label), "conv R%d S%d s%d g%d Cin%d Cout%d HxW%dx%d M%d K%d BN%d amode%d epi%d nb%d rkb%d mc%d segs%d tiles%d%s",
              L.R, L.S, L.stride, L.groups, L.Cin, L.Cout, H, W, p.M, L.K, L.BN, amode, tma_epi ? 1 : 0, nb, rkb, p.mc,
-             p.n_tiles, res ? " res" : "");
+             p.segs, p.n_tiles, res ? " res" : "");
   prof_end(st, 0, flops, bytes, label);
   if (dbgb) {
     unsigned long long h[148 * 8];

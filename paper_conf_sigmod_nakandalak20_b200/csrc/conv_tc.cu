@@ -71,7 +71,10 @@ struct ConvParams {
   // rank r takes M tile 2 * pair_m + r) in lockstep, and each CTA TMA-loads half of every weight (B) k-block
   // and multicasts it to both, halving the per-SM L2 -> shared-memory weight traffic of streamed-B layers
   int mc;
-  int segs;  // A_ROWVIEW: 128-pixel segments per output row (1 unless Wo > 128)
+  int segs;  // A_ROWVIEW: 128-pixel segments per output row (1 unless Wo > 128); A_HALO + hseg: segments
+  // A_HALO row-segment tiles (hseg = 1, rows too wide for the padded-grid halo): tile = (image, output row,
+  // segment of seg_w <= 126 columns); the halo is 3 input rows x (seg_w + 2) padded columns (Wp = seg_w + 2)
+  int hseg, seg_w;
   // fused tap g_l (PAPER.md:369 fn 4): per-image 2x2-grid channel maxima of the (post-ReLU, >= 0)
   // output, accumulated as fp32 bit patterns with red.global.max.u32 into tapf[n][4][Cout]
   unsigned int* tapf;
@@ -318,9 +321,18 @@ __global__ void __launch_bounds__(kThreads, 1)
         for (int tile = cta0; tile < p.n_tiles; tile += ncta, ++it) {
           int m0, nt, g;
           decode_tile(p, tile, m0, nt, g);
-          const int mt = m0 / BM, nimg = mt / p.mt_per_img;
-          const int p0 = (mt - nimg * p.mt_per_img) * BM;
-          const int prow0 = p0 / p.Wp;  // first padded input row (input row prow0 - 1)
+          const int mt = m0 / BM;
+          int nimg, prow0, col0 = -1;
+          if (p.hseg) {  // (image, output row ho, segment): input rows ho - 1 .. ho + 1, columns from seg * seg_w - 1
+            const int rowi = mt / p.segs;
+            nimg = rowi / p.Ho;
+            prow0 = rowi - nimg * p.Ho;
+            col0 = (mt - rowi * p.segs) * p.seg_w - 1;
+          } else {
+            nimg = mt / p.mt_per_img;
+            const int p0 = (mt - nimg * p.mt_per_img) * BM;
+            prow0 = p0 / p.Wp;  // first padded input row (input row prow0 - 1)
+          }
           const uint32_t hb = it % HB;
           if (it >= (uint32_t)HB) mbar_wait(&hempty[hb], ((it / HB) - 1) & 1);
           if ((p.dbg & 1) && it >= (uint32_t)HB) {
@@ -328,7 +340,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           } else {
             mbar_arrive_expect_tx(&hfull[hb], box_bytes * p.cblocks);
             for (int cb = 0; cb < p.cblocks; ++cb)
-              tma_load_4d(sH + hb * halo_half_bytes(BN) + cb * p.hsz, &tmap_a, cb * BK, -1, prow0 - 1, nimg,
+              tma_load_4d(sH + hb * halo_half_bytes(BN) + cb * p.hsz, &tmap_a, cb * BK, col0, prow0 - 1, nimg,
                           &hfull[hb]);
           }
           if constexpr (!BRES) {  // streamed weights (resident: nothing else per tile)
@@ -542,7 +554,8 @@ __global__ void __launch_bounds__(kThreads, 1)
               accs[j] = itj % NACC;
               hbs[j] = itj % HB;
               if (itj >= (uint32_t)NACC) mbar_wait(&tempty[accs[j]], ((itj / NACC) - 1) & 1);
-              const int pimg = (tiles[j] % p.mt_per_img) * BM;  // one N tile: tile index = M-tile index
+              // one N tile: tile index = M-tile index; row-segment tiles start at halo column 0
+              const int pimg = p.hseg ? 0 : (tiles[j] % p.mt_per_img) * BM;
               alo[j] = umma_desc_lo_sw128(sH + hbs[j] * halo_half_bytes(BN) + (pimg % p.Wp) * 128);
             }
           }
@@ -598,9 +611,11 @@ __global__ void __launch_bounds__(kThreads, 1)
         if constexpr (AMODE == A_HALO) {
           int m0, nt, g;
           decode_tile(p, tile, m0, nt, g);
-          const int mt = m0 / BM, nimg = mt / p.mt_per_img;
-          const int p0 = (mt - nimg * p.mt_per_img) * BM;
-          hoff = p0 - (p0 / p.Wp) * p.Wp;  // first output position's column in the first halo row
+          if (!p.hseg) {
+            const int mt = m0 / BM, nimg = mt / p.mt_per_img;
+            const int p0 = (mt - nimg * p.mt_per_img) * BM;
+            hoff = p0 - (p0 / p.Wp) * p.Wp;  // first output position's column in the first halo row
+          }
           hbase = sH + (it % HB) * halo_half_bytes(BN);
           dah = umma_desc_k_sw128(hbase + hoff * 128);
           if (prof_mma) {
@@ -754,11 +769,19 @@ __global__ void __launch_bounds__(kThreads, 1)
       int mo = m0 + row;
       bool rvalid = mo < p.M;
       if constexpr (AMODE == A_HALO) {  // padded-width position -> output pixel (columns >= Wo discarded)
-        const int mt = m0 / BM, nimg = mt / p.mt_per_img;
-        const int pp = (mt - nimg * p.mt_per_img) * BM + row;
-        const int ho = pp / p.Wp, wo = pp - ho * p.Wp;
-        mo = (nimg * p.Ho + ho) * p.Wo + wo;
-        rvalid = ho < p.Ho && wo < p.Wo && mo < p.M;  // (a multicast phantom tile lies past the last image)
+        const int mt = m0 / BM;
+        if (p.hseg) {
+          const int rowi = mt / p.segs, seg = mt - rowi * p.segs;
+          const int wo = seg * p.seg_w + row;
+          mo = rowi * p.Wo + wo;
+          rvalid = row < p.seg_w && wo < p.Wo && rowi < p.n_mt / p.segs;
+        } else {
+          const int nimg = mt / p.mt_per_img;
+          const int pp = (mt - nimg * p.mt_per_img) * BM + row;
+          const int ho = pp / p.Wp, wo = pp - ho * p.Wp;
+          mo = (nimg * p.Ho + ho) * p.Wo + wo;
+          rvalid = ho < p.Ho && wo < p.Wo && mo < p.M;  // (a multicast phantom tile lies past the last image)
+        }
       }
       const size_t off = (size_t)(rvalid ? mo : 0) * p.Cout + ng0;
       constexpr int kChunks = SPLIT ? BN / 32 : BN / 64;  // 32-column chunks per warp
@@ -1011,6 +1034,10 @@ static const bool g_rowview_enabled = [] {
   return !(e && e[0] == '0');
 }();
 // VISTA_HALO=0 disables the halo mode (3x3 convs fall back to im2col boxes; A/B measurements)
+static const bool g_hseg_enabled = [] {  // VISTA_HALO_SEG=0: wide rows fall back to im2col (A/B)
+  const char* e = getenv("VISTA_HALO_SEG");
+  return !(e && e[0] == '0');
+}();
 static const bool g_halo_enabled = [] {
   const char* e = getenv("VISTA_HALO");
   return !(e && e[0] == '0');
@@ -1339,6 +1366,35 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
         }
         p.n_mt = N * p.mt_per_img;
         p.n_tiles = p.n_mt * p.n_nt;
+      }
+    } else if (g_hseg_enabled && L.Kp / BK <= 36) {
+      // rows too wide for the padded-grid halo (VGG16 conv1_2 / conv2_1 at 227 / 113): row-segment tiles
+      const int wb_max = half / (3 * 128 * cblocks);  // widest 3-row box of all channel blocks in one buffer
+      const int nsegs = wb_max > 2 ? (p.Wo + wb_max - 3) / (wb_max - 2) : 0;
+      const int seg_w = nsegs ? (p.Wo + nsegs - 1) / nsegs : 0;
+      const int Wps = seg_w + 2, hszs = (3 * Wps * 128 + 1023) & ~1023;
+      if (nsegs && seg_w >= 96 && seg_w <= BM && hszs * cblocks <= half) {
+        const cuuint64_t dims[4] = {(cuuint64_t)L.Cin, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
+        const cuuint64_t strides[3] = {(cuuint64_t)L.Cin * 2, (cuuint64_t)W * L.Cin * 2,
+                                       (cuuint64_t)H * W * L.Cin * 2};
+        const cuuint32_t box[4] = {(cuuint32_t)BK, (cuuint32_t)Wps, 3, 1};
+        if (encode_nd(&ta, x, 4, dims, strides, box) == CUDA_SUCCESS) {
+          halo = true;
+          p.hseg = 1;
+          p.segs = nsegs;
+          p.seg_w = seg_w;
+          p.Wp = Wps;
+          p.hrows = 3;
+          p.hsz = hszs;
+          p.cblocks = cblocks;
+          p.mt_per_img = p.Ho * nsegs;
+          for (int kb = 0; kb < p.nkb && kb < 36; ++kb) {
+            const int tap = kb / cblocks, cb = kb % cblocks, r = tap / 3, sc = tap % 3;
+            p.koff[kb] = ((r * Wps + sc) * 128 + cb * hszs) >> 4;
+          }
+          p.n_mt = N * p.Ho * nsegs;
+          p.n_tiles = p.n_mt * p.n_nt;
+        }
       }
     }
   }

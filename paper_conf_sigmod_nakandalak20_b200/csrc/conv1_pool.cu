@@ -29,7 +29,7 @@ constexpr int kHin = 117;          // space-to-depth input rows (kS2dHW)
 constexpr int kPo = 56;            // pool1 output (114 - 3) / 2 + 1
 constexpr int kCo = 64;            // conv1 channels
 constexpr int kSA = 8;             // input-row ring slots
-constexpr int kNAcc = 4;           // TMEM accumulators (64 columns each)
+constexpr int kNAcc = 8;           // TMEM accumulators (64 columns each; the classic issue order uses 4)
 constexpr int kRowBytes = 128 * 128;  // one A slot: 128 pixel rows x 64 bf16 (128B-swizzled)
 constexpr int kBBytes = 4 * 64 * 128;  // 4 k-blocks x 64 output channels x 64 bf16
 constexpr int kCrowBytes = 128 * 128;  // conv row: 128 pixels x 64 channels bf16
@@ -46,6 +46,13 @@ struct PoolParams {
   const float* scale;
   const float* shift;
   int N;
+  // irow = 1 (default): input-row-major issue.  Input row i feeds output rows i-3..i through filter rows
+  // 3..0, so ONE 128 x 256 x 16 MMA step per K slice (weights of the four filter rows side by side, W_3 first)
+  // accumulates into four consecutive output-row accumulators of an 8-slot TMEM ring (split where the ring
+  // wraps / at image edges); slots are zeroed by the epilogue after draining, so every MMA accumulates.
+  // Versus the row-major order (16 N = 64 MMAs per output row, shared-memory operand bound at 48 cycles
+  // each): half the shared-memory operand bytes and full-rate N >= 128 instructions.
+  int irow;
 };
 
 __device__ __forceinline__ uint4 max4(uint4 a, uint4 b) {
@@ -95,12 +102,20 @@ __global__ void __launch_bounds__(kThreads, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  if (p.irow && warp >= kEpiWarp0) {  // zero the whole accumulator ring before the first MMA
+    const int q = warp & 3, half = (warp - kEpiWarp0) >> 2;
+    for (int sl = 0; sl < kNAcc; ++sl) tmem_zero_32x32b_x32(tmem_base + sl * kCo + half * 32 + ((uint32_t)(q * 32) << 16));
+    tc_wait_st();
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
 
   if (warp == 0) {
     // ======================= producer: weights once, then every input row once =======================
     if (lane == 0) {
       mbar_arrive_expect_tx(bbar, kBBytes);
-      for (int r = 0; r < 4; ++r) tma_load_2d(sB + r * 64 * 128, &tmap_w, r * 64, 0, bbar);
+      for (int r = 0; r < 4; ++r) tma_load_2d(sB + (p.irow ? 3 - r : r) * 64 * 128, &tmap_w, r * 64, 0, bbar);
       // The TMA ring holds only ~4 rows of lookahead and a row is 3.7 KB of unique input, far too little
       // in flight to cover HBM latency: rows kPfAhead ahead are prefetched into L2 in 8-row groups.
       constexpr int kPfAhead = 24, kPfGroup = 8;
@@ -129,6 +144,37 @@ __global__ void __launch_bounds__(kThreads, 1)
           mbar_arrive_expect_tx(&full[slot], kRowBytes);
           tma_load_4d(sA + slot * kRowBytes, &tmap_a, 0, 0, i, n, &full[slot]);
         }
+      }
+    }
+  } else if (warp == 1 && p.irow) {
+    // ============ MMA issuer, input-row-major (see PoolParams::irow) ============
+    mbar_wait(bbar, 0);
+    uint32_t grow = 0, orow = 0;  // this CTA's running input-row / output-row counters
+    for (int n = blockIdx.x; n < p.N; n += gridDim.x, orow += kHo) {
+      for (int i = 0; i < kHin; ++i, ++grow) {
+        if (i < kHo) {  // output row i opens here: its ring slot must have been drained and zeroed
+          const uint32_t o = orow + i;
+          if (o >= (uint32_t)kNAcc) mbar_wait(&tempty[o % kNAcc], ((o / kNAcc) - 1) & 1);
+        }
+        const uint32_t slot = grow % kSA;
+        mbar_wait(&full[slot], (grow / kSA) & 1);
+        tc_fence_after();
+        const int r_hi = i < 3 ? i : 3, r_lo = i > kHo - 1 ? i - (kHo - 1) : 0;
+        const int j_lo = 3 - r_hi, cnt = r_hi - r_lo + 1;  // weight groups j_lo .. j_lo + cnt - 1 (j = 3 - r)
+        const uint32_t s0 = (orow + (uint32_t)(i - r_hi)) % kNAcc;  // slot of output row i - r_hi
+        const uint32_t n1 = (uint32_t)cnt < kNAcc - s0 ? (uint32_t)cnt : kNAcc - s0;
+        const uint64_t da = umma_desc_k_sw128(sA + slot * kRowBytes);
+        auto issue = [&](uint32_t col, uint32_t jg, uint32_t ng) {
+          const uint32_t idesc = umma_idesc_bf16(128, 64 * ng);
+          const uint64_t db = umma_desc_k_sw128(sB + jg * 64 * 128);
+          const uint32_t tacc = tmem_base + col * kCo;
+#pragma unroll
+          for (int k = 0; k < 4; ++k) tc_mma_bf16_warp(tacc, da + 2 * k, db + 2 * k, idesc, 1u);
+        };
+        issue(s0, (uint32_t)j_lo, n1);
+        if ((uint32_t)cnt > n1) issue(0, (uint32_t)j_lo + n1, (uint32_t)cnt - n1);
+        tc_commit_warp(&empty[slot]);  // input row i feeds no later MMA
+        if (i >= 3) tc_commit_warp(&tfull[(orow + i - 3) % kNAcc]);  // output row i - 3 is complete
       }
     }
   } else if (warp == 1) {
@@ -189,6 +235,10 @@ __global__ void __launch_bounds__(kThreads, 1)
         uint32_t v[32];
         tmem_ld_32x32b_x32(tmem_base + acc * kCo + half * 32 + ((uint32_t)(q * 32) << 16), v);
         tc_wait_ld();
+        if (p.irow) {  // input-row-major issue accumulates into zeroed slots
+          tmem_zero_32x32b_x32(tmem_base + acc * kCo + half * 32 + ((uint32_t)(q * 32) << 16));
+          tc_wait_st();
+        }
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty[acc]);
@@ -266,6 +316,8 @@ void conv1_pool_forward(const ConvLayer& L, const bf16* x, int N, bf16* y, cudaS
   p.scale = L.scale;
   p.shift = L.shift;
   p.N = N;
+  const char* e = getenv("VISTA_STEM_IROW");  // read per launch (A/B within one process)
+  p.irow = (e && e[0] == '0') ? 0 : 1;
   static bool attr = false;
   if (!attr) {
     VCHECK(cudaFuncSetAttribute(conv1_pool_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem));

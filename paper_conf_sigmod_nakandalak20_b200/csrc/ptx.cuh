@@ -209,6 +209,16 @@ __device__ __forceinline__ void tc_commit_mc_warp(uint64_t* bar, uint16_t mask) 
       "h"(mask)
       : "memory");
 }
+// zero 32 lanes x 32 columns of TMEM (this warp's lane quadrant), then tc_wait_st
+__device__ __forceinline__ void tmem_zero_32x32b_x32(uint32_t taddr) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], "
+      "{%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1};" ::"r"(
+          taddr),
+      "r"(0u)
+      : "memory");
+}
+__device__ __forceinline__ void tc_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 __device__ __forceinline__ void tc_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
 
 // 32 lanes x 32 columns of 32-bit: thread i of the warp gets lane (quadrant*32 + i), columns [c, c+32)

@@ -688,6 +688,35 @@ bool run_ops(vista_ctx* c, int t, const void* in_ptr, void* out_ptr, int nb, voi
 }
 
 // one block of the Staged plan over n images (a chunk), in micro-batches of micro[t]: in_base -> A_t
+// Host pixels of images [c0, c0 + nc) -> c->d_px, one stage-1 micro-batch per copy on c->copy_stream, each
+// followed by c->px_ready[j]; the compute stream waits on event j right before micro-batch j, so the copy of
+// micro-batch j + 1 overlaps the inference of micro-batch j.  Returns the events.
+const std::vector<cudaEvent_t>* stream_host_pixels(vista_ctx* c, const uint8_t* images, int64_t c0, int64_t nc) {
+  const size_t px_img = (size_t)c->net.stages[0].in_elems;
+  c->d_px.ensure((size_t)nc * px_img);
+  if (!c->copy_stream) {
+    VCHECK(cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking));
+    VCHECK(cudaEventCreateWithFlags(&c->px_free, cudaEventDisableTiming));
+  }
+  // d_px may still be read by work already queued on the compute stream (the previous chunk)
+  VCHECK(cudaEventRecord(c->px_free, c->stream));
+  VCHECK(cudaStreamWaitEvent(c->copy_stream, c->px_free, 0));
+  const int64_t B0 = std::max(c->micro[0], 1);
+  const size_t nev = (size_t)((nc + B0 - 1) / B0);
+  while (c->px_ready.size() < nev) {
+    cudaEvent_t e;
+    VCHECK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    c->px_ready.push_back(e);
+  }
+  for (int64_t i0 = 0; i0 < nc; i0 += B0) {
+    const int64_t nb = std::min<int64_t>(B0, nc - i0);
+    VCHECK(cudaMemcpyAsync((uint8_t*)c->d_px.p + (size_t)i0 * px_img, images + (size_t)(c0 + i0) * px_img,
+                           (size_t)nb * px_img, cudaMemcpyHostToDevice, c->copy_stream));
+    VCHECK(cudaEventRecord(c->px_ready[(size_t)(i0 / B0)], c->copy_stream));
+  }
+  return &c->px_ready;
+}
+
 // in_ready (optional): event j is recorded once micro-batch j's input has landed (host pixels copied on
 // c->copy_stream); the compute stream waits on it right before that micro-batch
 bool run_block(vista_ctx* c, int t, const void* in_base, void* out_base, int64_t n, unsigned int* tapf,
@@ -712,7 +741,8 @@ bool run_block(vista_ctx* c, int t, const void* in_base, void* out_base, int64_t
 // Eager (Fig 5C) and Lazy (Fig 5A) schedules: per micro-batch of images, run blocks 0..t_last from
 // the raw pixels with the activations in two ping-pong micro-batch buffers, and tap every requested
 // layer in `want` (Eager: all of L in one pass; Lazy: one layer per pass, recomputing from pixels).
-void run_unstaged(vista_ctx* c, const uint8_t* px, int t_last, const std::vector<int>& want) {
+void run_unstaged(vista_ctx* c, const uint8_t* px, int t_last, const std::vector<int>& want,
+                  const std::vector<cudaEvent_t>* in_ready = nullptr) {
   const auto& S = c->net.stages;
   const int B = c->micro[0];
   void* slot[NUM_BUFS] = {nullptr};
@@ -726,6 +756,7 @@ void run_unstaged(vista_ctx* c, const uint8_t* px, int t_last, const std::vector
   act[1].alloc((size_t)B * max_out * c->esz + 16);
   for (int64_t i0 = 0; i0 < c->n_img; i0 += B) {
     const int nb = (int)std::min<int64_t>(B, c->n_img - i0);
+    if (in_ready) VCHECK(cudaStreamWaitEvent(c->stream, (*in_ready)[(size_t)(i0 / B)], 0));
     for (int t = 0; t <= t_last; ++t) {
       const void* in = t == 0 ? (const void*)(px + (size_t)i0 * S[0].in_elems) : act[(t - 1) & 1].p;
       void* out = act[t & 1].p;
@@ -919,9 +950,13 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
     const auto& S = c->net.stages;
     // ---- inputs (H2D when given host pointers) ----
     // (the Staged plan streams host pixels to the device chunk by chunk; Eager / Lazy copy them once)
-    const uint8_t* px = c->sys.plan == VISTA_PLAN_STAGED || base
-                            ? images
-                            : (const uint8_t*)to_device(c, c->d_px, images, (size_t)c->n_img * S[0].in_elems);
+    // (the Staged plan streams host pixels chunk by chunk below; Eager / Lazy stream them once, per micro-batch)
+    const std::vector<cudaEvent_t>* unstaged_ev = nullptr;
+    const uint8_t* px = images;
+    if (c->sys.plan != VISTA_PLAN_STAGED && !base && c->n_img > 0 && !is_device_ptr(images)) {
+      unstaged_ev = stream_host_pixels(c, images, 0, c->n_img);
+      px = (const uint8_t*)c->d_px.p;
+    }
     const int t0 = base ? c->taps[0] : -1;  // block whose output is the stored base layer
     const size_t base_img_bytes = base ? (size_t)S[t0].out_elems * c->esz : 0;
     const bool host_base = base && c->n_img > 0 && !is_device_ptr(base);
@@ -974,9 +1009,9 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
     if (c->sys.plan != VISTA_PLAN_STAGED) {
       // ---- Eager / Lazy (Fig 5C / 5A): features of every layer, no resident full activations ----
       if (c->sys.plan == VISTA_PLAN_EAGER) {
-        run_unstaged(c, px, c->t_max, c->taps);
+        run_unstaged(c, px, c->t_max, c->taps, unstaged_ev);
       } else {
-        for (int t : c->taps) run_unstaged(c, px, t, std::vector<int>{t});
+        for (int t : c->taps) run_unstaged(c, px, t, std::vector<int>{t}, unstaged_ev);
       }
       for (size_t k = 0; k < c->taps.size(); ++k) concat_layer((int)k);
     }
@@ -1007,29 +1042,7 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
       }
       const std::vector<cudaEvent_t>* px_ev = nullptr;
       if (host_px) {  // stream the chunk's pixels to the device, one stage-1 micro-batch per copy
-        c->d_px.ensure((size_t)nc * S[0].in_elems);
-        if (!c->copy_stream) {
-          VCHECK(cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking));
-          VCHECK(cudaEventCreateWithFlags(&c->px_free, cudaEventDisableTiming));
-        }
-        // d_px may still be read by work already queued on the compute stream (the previous chunk)
-        VCHECK(cudaEventRecord(c->px_free, st));
-        VCHECK(cudaStreamWaitEvent(c->copy_stream, c->px_free, 0));
-        const int64_t B0 = std::max(c->micro[0], 1);
-        const size_t nev = (size_t)((nc + B0 - 1) / B0);
-        while (c->px_ready.size() < nev) {
-          cudaEvent_t e;
-          VCHECK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-          c->px_ready.push_back(e);
-        }
-        for (int64_t i0 = 0; i0 < nc; i0 += B0) {
-          const int64_t nb = std::min<int64_t>(B0, nc - i0);
-          VCHECK(cudaMemcpyAsync((uint8_t*)c->d_px.p + (size_t)i0 * S[0].in_elems,
-                                 images + (size_t)(c0 + i0) * S[0].in_elems, (size_t)nb * S[0].in_elems,
-                                 cudaMemcpyHostToDevice, c->copy_stream));
-          VCHECK(cudaEventRecord(c->px_ready[(size_t)(i0 / B0)], c->copy_stream));
-        }
-        px_ev = &c->px_ready;
+        px_ev = stream_host_pixels(c, images, c0, nc);
         pxc = (const uint8_t*)c->d_px.p;
       }
       for (int t = base ? t0 : 0; t <= c->t_max; ++t) {

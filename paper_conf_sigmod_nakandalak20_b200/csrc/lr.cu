@@ -20,7 +20,7 @@ namespace vista {
 
 constexpr int kMaxRB = 16;     // rows per streamed block (upper bound)
 constexpr int kStagesLR = 3;   // row blocks in flight per CTA
-constexpr int kLRThreads = 512;
+constexpr int kLRThreads = 576;  // 18 compute warps: 1041 chunks of a conv5_x row (ld 8328) = 2 per thread, no 3-chunk stragglers
 
 struct PassArgs {
   const uint8_t* MM;   // row-major [rows][ld] elements of E (bf16, or fp32 in check mode)

@@ -63,6 +63,10 @@ struct ConvParams {
   // issue loop has no integer division (measured: the per-k-block division chain made the issue latency
   // ~340 cycles, longer than the 4 MMAs it feeds)
   int koff[36];
+  // A_HALO (padded-grid tiles): first output position's column in the first halo row of a tile, indexed by
+  // (M tile index mod mt_per_img) -- removes the MMA warp's per-tile integer divisions (measured ~650 cycles
+  // per tile on res3 3x3); valid when mt_per_img <= 64
+  short hofft[64];
   // A_CAT (unit-1 closing conv with the projection shortcut folded in, see conv_cat_forward): k-blocks
   // [0, nkb1) read the b activation through tmap_a, k-blocks [nkb1, nkb) read the unit input x through
   // tmap_r (plain 2-D map, or an im2col map when the projection is strided: cat_im2col = 1)
@@ -315,8 +319,29 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
       }
     } else if constexpr (AMODE == A_HALO) {
+      // thread 0: halo boxes (tile t + 2's halo as soon as tile t's MMAs release its buffer); thread 32 (warp 1):
+      // the streamed weight stages.  One thread doing both put the next halo behind the current tile's weight
+      // loads, which wait for ring stages the running MMAs free (measured: the halo wait became the bound)
+      if (!BRES && threadIdx.x == 32) {
+        constexpr int S2 = S / 2;  // two k-blocks per ring stage (S / 2 stages of 2 x BN x 64)
+        uint32_t gk = 0;
+        for (int tile = cta0; tile < p.n_tiles; tile += ncta)
+          for (int kb = 0; kb < p.nkb; kb += 2, ++gk) {
+            const int stage = gk % S2;
+            if (gk >= (uint32_t)S2) mbar_wait(&empty[stage], ((gk / S2) - 1) & 1);
+            const int two = kb + 1 < p.nkb ? 2 : 1;
+            mbar_arrive_expect_tx(&full[stage], two * C::kBBytes);
+            for (int h = 0; h < two; ++h) {
+              if (p.mc)  // this CTA's half of the k-block rows, multicast to the pair
+                tma_load_2d_mc(sB + (2 * stage + h) * C::kBBytes + crank * (BN / 2) * 128, &tmap_w, (kb + h) * BK,
+                               (int)crank * (BN / 2), &full[stage], (uint16_t)3);
+              else
+                tma_load_2d(sB + (2 * stage + h) * C::kBBytes, &tmap_w, (kb + h) * BK, 0, &full[stage]);
+            }
+          }
+      }
       if (threadIdx.x == 0) {
-        uint32_t gk = 0, it = 0;
+        uint32_t it = 0;
         const uint32_t box_bytes = (uint32_t)p.hrows * p.Wp * 128u;
         for (int tile = cta0; tile < p.n_tiles; tile += ncta, ++it) {
           int m0, nt, g;
@@ -342,14 +367,6 @@ __global__ void __launch_bounds__(kThreads, 1)
             for (int cb = 0; cb < p.cblocks; ++cb)
               tma_load_4d(sH + hb * halo_half_bytes(BN) + cb * p.hsz, &tmap_a, cb * BK, col0, prow0 - 1, nimg,
                           &hfull[hb]);
-          }
-          if constexpr (!BRES) {  // streamed weights (resident: nothing else per tile)
-            for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
-              const int stage = gk % S;
-              if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
-              mbar_arrive_expect_tx(&full[stage], C::kBBytes);
-              load_b(stage, kb, 0);
-            }
           }
         }
       }
@@ -555,8 +572,8 @@ __global__ void __launch_bounds__(kThreads, 1)
               hbs[j] = itj % HB;
               if (itj >= (uint32_t)NACC) mbar_wait(&tempty[accs[j]], ((itj / NACC) - 1) & 1);
               // one N tile: tile index = M-tile index; row-segment tiles start at halo column 0
-              const int pimg = p.hseg ? 0 : (tiles[j] % p.mt_per_img) * BM;
-              alo[j] = umma_desc_lo_sw128(sH + hbs[j] * halo_half_bytes(BN) + (pimg % p.Wp) * 128);
+              const int hoffj = p.hseg ? 0 : p.hofft[tiles[j] % p.mt_per_img];
+              alo[j] = umma_desc_lo_sw128(sH + hbs[j] * halo_half_bytes(BN) + hoffj * 128);
             }
           }
           if (prof_mma) {
@@ -593,7 +610,14 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
           if (prof_mma) c_iss += clock64() - tA;
         }
-      } else
+      }
+      int hmod = 0, hstep = 0;  // A_HALO: tile index mod mt_per_img and its per-iteration step
+      if constexpr (AMODE == A_HALO) {
+        // (multicast pairs: M tile = 2 * pair tile + rank)
+        hmod = (p.mc ? 2 * cta0 + (int)crank : cta0) % p.mt_per_img;
+        hstep = (p.mc ? 2 * ncta : ncta) % p.mt_per_img;
+      }
+      if constexpr (!(AMODE == A_HALO && BRES))
       for (int tile = cta0; tile < p.n_tiles; tile += ncta, ++it) {
         const uint32_t acc = it % NACC, use = it / NACC;
         if (prof_mma) tA = clock64();
@@ -609,13 +633,10 @@ __global__ void __launch_bounds__(kThreads, 1)
         int hoff = 0;
         uint64_t dah = 0;  // A_HALO: descriptor of the tile's first output position in the halo buffer
         if constexpr (AMODE == A_HALO) {
-          int m0, nt, g;
-          decode_tile(p, tile, m0, nt, g);
-          if (!p.hseg) {
-            const int mt = m0 / BM, nimg = mt / p.mt_per_img;
-            const int p0 = (mt - nimg * p.mt_per_img) * BM;
-            hoff = p0 - (p0 / p.Wp) * p.Wp;  // first output position's column in the first halo row
-          }
+          // one N tile: tile index = M tile index; (tile mod mt_per_img) advances by ncta mod mt_per_img
+          if (!p.hseg) hoff = p.hofft[hmod];
+          hmod += hstep;
+          if (hmod >= p.mt_per_img) hmod -= p.mt_per_img;
           hbase = sH + (it % HB) * halo_half_bytes(BN);
           dah = umma_desc_k_sw128(hbase + hoff * 128);
           if (prof_mma) {
@@ -629,6 +650,37 @@ __global__ void __launch_bounds__(kThreads, 1)
             c_hf += tB - tA;
             tA = tB;
           }
+        }
+        if constexpr (AMODE == A_HALO && !BRES) {
+          // streamed weights: one ring wait and one commit per TWO k-blocks (8 MMAs), 32-bit descriptor
+          // arithmetic -- measured (dbg 8 counters, res3 3x3): one wait + commit + 64-bit descriptors per
+          // k-block made the issue loop ~350 cycles per 256 cycles of N = 128 MMAs
+          constexpr int S2 = S / 2;
+          const uint32_t alo = umma_desc_lo_sw128(hbase + hoff * 128);
+          const uint32_t blo0 = umma_desc_lo_sw128(sB);
+          for (int kb = 0; kb < p.nkb; kb += 2, ++gk) {
+            const int stage = gk % S2;
+            mbar_wait(&full[stage], (gk / S2) & 1);
+            const uint32_t b = blo0 + (uint32_t)(2 * stage) * (uint32_t)(C::kBBytes >> 4);
+            const uint32_t a = alo + (uint32_t)p.koff[kb];
+            tc_mma_bf16_lo_warp(tacc, a, b, idesc, kb != 0 ? 1u : 0u);
+            tc_mma_bf16_lo_warp(tacc, a + 2, b + 2, idesc, 1u);
+            tc_mma_bf16_lo_warp(tacc, a + 4, b + 4, idesc, 1u);
+            tc_mma_bf16_lo_warp(tacc, a + 6, b + 6, idesc, 1u);
+            if (kb + 1 < p.nkb) {
+              const uint32_t a1 = alo + (uint32_t)p.koff[kb + 1];
+              const uint32_t b1 = b + (uint32_t)(C::kBBytes >> 4);
+              tc_mma_bf16_lo_warp(tacc, a1, b1, idesc, 1u);
+              tc_mma_bf16_lo_warp(tacc, a1 + 2, b1 + 2, idesc, 1u);
+              tc_mma_bf16_lo_warp(tacc, a1 + 4, b1 + 4, idesc, 1u);
+              tc_mma_bf16_lo_warp(tacc, a1 + 6, b1 + 6, idesc, 1u);
+            }
+            if (p.mc) tc_commit_mc_warp(&empty[stage], (uint16_t)3);
+            else tc_commit_warp(&empty[stage]);
+          }
+          tc_commit_warp(&tfull[acc]);
+          tc_commit_warp(&hempty[it % HB]);
+          continue;
         }
         auto kblock = [&](const int kb) {
           const int stage = gk % S;
@@ -1051,15 +1103,17 @@ static const int g_conv_dbg = [] {
 // VISTA_WRES=0 disables the resident-weight launches (A/B measurements)
 // weight multicast across CTA pairs for streamed-weight launches (ConvParams::mc); VISTA_MC=0 disables.
 // Measured: 256-wide tiles gain (VGG conv3_x 1353 -> 1496, conv4_x 1454 -> 1598 TF/s, ResNet res5 3x3
-// 1452 -> 1557), 64/128-wide tiles lose (VGG conv1_2 437 -> 406, conv2_2 928 -> 841; ResNet res3 halo 3x3
-// 814 -> 774), so only BN = 256 launches multicast (the halo path additionally needs VISTA_MC_HALO=1).  Read per launch (tests switch them within one process).
+// 1452 -> 1557); 64/128-wide im2col / TMA tiles lose (VGG conv1_2 437 -> 406, conv2_2 928 -> 841), so they
+// stay unicast; the streamed-weight halo 3x3 (BN = 128), weight-ingest bound once its halo and weight
+// producers were split, gains ~2 % (res3: 903 -> 923 TF/s, same run; VISTA_MC_HALO=0 disables).
 static bool env_flag(const char* name, bool dflt) {
   const char* e = getenv(name);
   return e && *e ? e[0] == '1' : dflt;
 }
 static bool use_mc(const ConvLayer& L, int amode, int rkb, const ConvParams& p) {
-  return env_flag("VISTA_MC", true) && rkb == 0 && L.groups == 1 && L.BN == 256 && p.n_mt >= 2 &&
-         (amode == A_TMA || amode == A_IM2COL || amode == A_CAT || (amode == A_HALO && env_flag("VISTA_MC_HALO", false))) &&
+  return env_flag("VISTA_MC", true) && rkb == 0 && L.groups == 1 && p.n_mt >= 2 &&
+         (L.BN == 256 || (amode == A_HALO && L.BN == 128)) &&
+         (amode == A_TMA || amode == A_IM2COL || amode == A_CAT || (amode == A_HALO && env_flag("VISTA_MC_HALO", true))) &&
          (int64_t)p.n_nt * ((p.n_mt + 1) / 2) >= num_sms() / 2;
 }
 static const bool g_wres_enabled = [] {
@@ -1349,7 +1403,8 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
     const int hsz = (hrows * Wp * 128 + 1023) & ~1023;
     const int cblocks = L.Cin / BK;
     const int half = L.BN == 64 ? 45056 : 61440;
-    if (Wp <= 256 && hrows <= 256 && hsz * cblocks <= half && L.Kp / BK <= 36) {
+    if (Wp <= 256 && hrows <= 256 && hsz * cblocks <= half && L.Kp / BK <= 36 &&
+        (p.Ho * Wp + BM - 1) / BM <= 64) {
       const cuuint64_t dims[4] = {(cuuint64_t)L.Cin, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
       const cuuint64_t strides[3] = {(cuuint64_t)L.Cin * 2, (cuuint64_t)W * L.Cin * 2, (cuuint64_t)H * W * L.Cin * 2};
       const cuuint32_t box[4] = {(cuuint32_t)BK, (cuuint32_t)Wp, (cuuint32_t)hrows, 1};
@@ -1360,6 +1415,7 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
         p.hsz = hsz;
         p.cblocks = cblocks;
         p.mt_per_img = (p.Ho * Wp + BM - 1) / BM;
+        for (int r = 0; r < p.mt_per_img && r < 64; ++r) p.hofft[r] = (short)((r * BM) % Wp);
         for (int kb = 0; kb < p.nkb && kb < 36; ++kb) {
           const int tap = kb / cblocks, cb = kb % cblocks, r = tap / 3, sc = tap % 3;
           p.koff[kb] = ((r * Wp + sc) * 128 + cb * hsz) >> 4;

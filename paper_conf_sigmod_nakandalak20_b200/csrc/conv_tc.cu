@@ -1100,12 +1100,12 @@ static const int g_conv_dbg = [] {
   const char* e = getenv("VISTA_CONV_DBG");
   return e ? atoi(e) : 0;
 }();
-// VISTA_WRES=0 disables the resident-weight launches (A/B measurements)
 // weight multicast across CTA pairs for streamed-weight launches (ConvParams::mc); VISTA_MC=0 disables.
 // Measured: 256-wide tiles gain (VGG conv3_x 1353 -> 1496, conv4_x 1454 -> 1598 TF/s, ResNet res5 3x3
 // 1452 -> 1557); 64/128-wide im2col / TMA tiles lose (VGG conv1_2 437 -> 406, conv2_2 928 -> 841), so they
 // stay unicast; the streamed-weight halo 3x3 (BN = 128), weight-ingest bound once its halo and weight
-// producers were split, gains ~2 % (res3: 903 -> 923 TF/s, same run; VISTA_MC_HALO=0 disables).
+// producers were split, gains ~2 % (res3: 903 -> 923 TF/s, same run; VISTA_MC_HALO=0 disables).  Flags are read per launch
+// (tests switch them within one process).
 static bool env_flag(const char* name, bool dflt) {
   const char* e = getenv(name);
   return e && *e ? e[0] == '1' : dflt;
@@ -1116,6 +1116,7 @@ static bool use_mc(const ConvLayer& L, int amode, int rkb, const ConvParams& p) 
          (amode == A_TMA || amode == A_IM2COL || amode == A_CAT || (amode == A_HALO && env_flag("VISTA_MC_HALO", true))) &&
          (int64_t)p.n_nt * ((p.n_mt + 1) / 2) >= num_sms() / 2;
 }
+// VISTA_WRES=0 disables the resident-weight launches (A/B measurements)
 static const bool g_wres_enabled = [] {
   const char* e = getenv("VISTA_WRES");
   return !(e && e[0] == '0');

@@ -949,14 +949,10 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
     cudaStream_t st = c->stream;
     const auto& S = c->net.stages;
     // ---- inputs (H2D when given host pointers) ----
-    // (the Staged plan streams host pixels to the device chunk by chunk; Eager / Lazy copy them once)
-    // (the Staged plan streams host pixels chunk by chunk below; Eager / Lazy stream them once, per micro-batch)
-    const std::vector<cudaEvent_t>* unstaged_ev = nullptr;
+    // (host pixels are streamed per stage-1 micro-batch right before the inference that reads them: Staged
+    // chunk by chunk, Eager / Lazy once.  Not here: the small key / table copies and the join below would
+    // queue behind the whole pixel array on the H2D copy engine -- measured +50 ms per 20k-image step)
     const uint8_t* px = images;
-    if (c->sys.plan != VISTA_PLAN_STAGED && !base && c->n_img > 0 && !is_device_ptr(images)) {
-      unstaged_ev = stream_host_pixels(c, images, 0, c->n_img);
-      px = (const uint8_t*)c->d_px.p;
-    }
     const int t0 = base ? c->taps[0] : -1;  // block whose output is the stored base layer
     const size_t base_img_bytes = base ? (size_t)S[t0].out_elems * c->esz : 0;
     const bool host_base = base && c->n_img > 0 && !is_device_ptr(base);
@@ -1008,6 +1004,11 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
     };
     if (c->sys.plan != VISTA_PLAN_STAGED) {
       // ---- Eager / Lazy (Fig 5C / 5A): features of every layer, no resident full activations ----
+      const std::vector<cudaEvent_t>* unstaged_ev = nullptr;
+      if (!base && c->n_img > 0 && !is_device_ptr(images)) {
+        unstaged_ev = stream_host_pixels(c, images, 0, c->n_img);
+        px = (const uint8_t*)c->d_px.p;
+      }
       if (c->sys.plan == VISTA_PLAN_EAGER) {
         run_unstaged(c, px, c->t_max, c->taps, unstaged_ev);
       } else {

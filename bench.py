@@ -209,7 +209,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default=DEFAULT, choices=sorted(CONFIGS))
-    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--images", type=int, default=0, help="override images per GPU (debug only)")
     ap.add_argument("--micro-batch", type=int, default=0, help="stage-1 micro-batch (0 = planner)")
@@ -221,7 +221,25 @@ def main():
                          "(PAPER.md:383, vista_train_mlp, 10 steps)")
     ap.add_argument("--plan", default="staged", choices=["staged", "eager", "lazy"],
                     help="logical plan (Fig 5): staged is the product; eager / lazy for config 4 comparisons")
+    ap.add_argument("--dry-run", action="store_true",
+                    help="print the launch command (torchrun re-exec for --gpus N > 1) and exit")
     args = ap.parse_args()
+    if args.gpus > 1 and "RANK" not in os.environ:
+        # one process per GPU: re-exec this command under torchrun (the driver may also launch us that way)
+        port = env_int("MASTER_PORT", 29500 + os.getpid() % 1000)
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+        if args.dry_run:
+            print(json.dumps({"launch": cmd}))
+            return 0
+        sys.stdout.flush()
+        os.execv(sys.executable, cmd)
+    if args.dry_run:
+        print(json.dumps({"launch": None, "rank": env_int("RANK", 0), "world": env_int("WORLD_SIZE", 1)}))
+        return 0
+    if "RANK" in os.environ and env_int("WORLD_SIZE", 1) != args.gpus:
+        print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={env_int('WORLD_SIZE', 1)}; using WORLD_SIZE",
+              file=sys.stderr)
     if args.impl == "reference":
         return run_reference(args)
 
@@ -337,8 +355,13 @@ def main():
     ms_step = ms / args.steps
     value = N_global / (ms_step / 1000.0)
     # ---- e2e: host inputs through the C-ABI, weights back to the host ----
+    peak_meas = None
     if args.e2e_steps > 0:
         step(host=True)  # untimed warm-up of the host-input path (sizes its per-chunk pixel buffer)
+        pinfo = v.plan_info()  # pool high-water mark of that transfer from host pixels vs the prediction
+        peak_meas = {"pred": pinfo["peak_bytes_pred"], "meas": pinfo["peak_bytes_meas"],
+                     "reserved": pinfo["peak_reserved_meas"],
+                     "meas_over_pred": pinfo["peak_bytes_meas"] / max(pinfo["peak_bytes_pred"], 1)}
         e2e_ms, _ = timed(args.e2e_steps, host=True)
         e2e_step = e2e_ms / args.e2e_steps
     else:  # profiling runs only (no e2e number)
@@ -403,7 +426,7 @@ def main():
             "config": dict(workload_config(args.config, world, n_img), micro_batch=info["micro_batch"],
                            plan=args.plan + ("+prematerialized_base" if args.from_base else ""),
                            model=("mlp_1024x1024x1_T10" if args.model == "mlp" else "elastic_net_lr_T%d" % T),
-                           peak_bytes_pred=info["peak_bytes_pred"],
+                           peak_bytes_pred=info["peak_bytes_pred"], peak_bytes=peak_meas,
                            **({"base_layer": TAP_NAMES[cnn][taps[0]], "materialize_s": round(materialize_s, 3)}
                               if args.from_base else {})),
             "roofline": roof,

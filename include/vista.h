@@ -87,6 +87,13 @@ typedef struct {
   vista_plan_kind plan;
   void* stream;              /* cudaStream_t to run on (e.g. torch's current stream); NULL = own stream */
   int32_t micro_batch;       /* images per micro-batch of the first stage; 0 = planner's choice */
+  /* Caller-supplied collective, used instead of NCCL when world > 1 and nccl_uid == NULL (e.g. a gloo
+   * process group, or ranks that share one GPU, which NCCL refuses).  In-place SUM allreduce of `count`
+   * elements of HOST memory across the `world` ranks; dtype 0 = float64, 1 = float32.  Every rank calls
+   * it the same number of times with the same counts.  Returns 0 on success (non-zero -> VISTA_ERR_NCCL).
+   * The library copies the device partials to the host, calls it, and copies the sums back. */
+  int32_t (*allreduce)(void* host_buf, int64_t count, int32_t dtype, void* user);
+  void* allreduce_user;      /* passed through to allreduce */
 } vista_sys_cfg;
 
 typedef struct vista_ctx vista_ctx;
@@ -103,6 +110,11 @@ typedef struct {
   int64_t weight_bytes;      /* resident CNN parameters */
   int32_t d_s, ds_pad;       /* structured width and its padded width in MM_k */
   int64_t chunk_images;      /* Staged: images per chunk (== n_images_local unless the budget forces chunking) */
+  /* Measured (0 before the first vista_transfer): weight_bytes + the high-water mark of the device memory
+   * pool's in-use bytes over the last vista_transfer / vista_transfer_from_base (every buffer the library
+   * allocates during a transfer comes from that pool), and the same with the pool's reserved bytes. */
+  int64_t peak_bytes_meas;
+  int64_t peak_reserved_meas;
 } vista_plan_info_t;
 
 /* Borrowed view of layer k's outputs on this rank (valid until vista_destroy or the
@@ -146,7 +158,9 @@ vista_status vista_plan_info(const vista_ctx* ctx, vista_plan_info_t* out);
 /* vista_transfer(images, structured, keys) -> per-layer multimodal feature buffers.
  *   images:     uint8 NHWC [n_images_local, 227, 227, 3] (host or device)
  *   image_keys: int64 [n_images_local] (host or device), unique
- *   structured: float32 [n_str_rows, d_s] row-major, values bf16-representable (host or device)
+ *   structured: float32 [n_str_rows, d_s] row-major, values bf16-representable (host or device); a
+ *               joined row holding a value with any of its low 16 bits set -> VISTA_ERR_INVALID_ARG
+ *               (bf16 path; MM_k stores X in bf16, so such a value could not be kept exactly)
  *   str_keys:   int64 [n_str_rows], unique (host or device)
  *   labels:     uint8 {0,1} [n_str_rows] (host or device)
  * Runs the join once (Eq. 3; broadcast join: T_str is whole on every rank),
@@ -171,12 +185,26 @@ vista_status vista_features(const vista_ctx* ctx, int32_t k, vista_buffer* out);
  *   inference below L[0]; F_0 = g_{L[0]}(base); A_{L[k]} = f^_{L[0] -> L[k]}(base) for k >= 1
  *   (Def 3.7 partial inference); join, concat and MM_k as vista_transfer.  base: host or device,
  *   the layout vista_materialize writes (read only; a device base is read in place).  Results are
- *   bit-identical to vista_transfer from the pixels the base was materialised from.  Staged plan
- *   only (VISTA_ERR_INVALID_ARG for Eager / Lazy). */
+ *   bit-identical to vista_transfer from the pixels the base was materialised from, under every plan:
+ *   Staged (stored A_k reused), Eager (one pass base -> all of L) and Lazy ("Lazy-5 with Pre-mat",
+ *   one pass from the stored base per layer, recomputing everything above it). */
 vista_status vista_base_shape(const vista_ctx* ctx, int64_t* out4);
 vista_status vista_materialize(vista_ctx* ctx, const uint8_t* images, void* base_out);
 vista_status vista_transfer_from_base(vista_ctx* ctx, const void* base, const int64_t* image_keys,
                                       const float* structured, const int64_t* str_keys, const uint8_t* labels);
+
+/* S4 key join on its own (Eq. (3); broadcast join PAPER.md:279), the kernels
+ * vista_transfer runs once per transfer: inner equi-join of the image keys with the structured keys,
+ * output pairs (structured row, image row) of the matched rows, train rows first then test rows, each
+ * in T_str order (reading R14/R16; test iff mix64(key ^ subseed(split_seed, 6)) % 5 == 0).
+ *   img_keys int64 [n_img], str_keys int64 [n_str]: DEVICE pointers, unique keys.
+ *   pair_str, pair_img: DEVICE int32 [n_str] (caller-owned), rows [0, *n_pairs) written.
+ *   n_pairs, n_train: HOST int64 out.
+ * Errors: VISTA_ERR_DUP_KEY if either key column has a duplicate; VISTA_ERR_INVALID_ARG for a key equal
+ * to INT64_MIN (the empty-slot marker) or NULL pointers.  Synchronises `stream` before returning. */
+vista_status vista_join(const int64_t* img_keys, int64_t n_img, const int64_t* str_keys, int64_t n_str,
+                        uint64_t split_seed, int32_t* pair_str, int32_t* pair_img, int64_t* n_pairs,
+                        int64_t* n_train, void* stream);
 
 /* vista_train(layer) -> weights / accuracy.  Collective over the `world` ranks (all must call
  * with the same k): per-rank partial sums are combined by an fp64 NCCL allreduce.

@@ -318,11 +318,7 @@ void conv1_pool_forward(const ConvLayer& L, const bf16* x, int N, bf16* y, cudaS
   p.N = N;
   const char* e = getenv("VISTA_STEM_IROW");  // read per launch (A/B within one process)
   p.irow = (e && e[0] == '0') ? 0 : 1;
-  static bool attr = false;
-  if (!attr) {
-    VCHECK(cudaFuncSetAttribute(conv1_pool_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem));
-    attr = true;
-  }
+  ensure_smem_attr((const void*)conv1_pool_kernel, kSmem);
   const int grid = N < num_sms() ? N : num_sms();
   prof_begin(st);
   conv1_pool_kernel<<<grid, kThreads, kSmem, st>>>(L.tmap_w, ta, p);

@@ -1222,11 +1222,7 @@ static void launch_t(const ConvLayer& L, const CUtensorMap& ta, const CUtensorMa
   static_assert(NB >= 1 && NB <= 4, "staging buffers");
   auto kern = conv_tc_kernel<BN, AMODE, TE, NB, RKB>;
   constexpr int smem = Cfg<BN, TE, NB, AMODE == A_HALO, RKB>::kBytes;
-  static bool attr_set = false;  // per instantiation
-  if (!attr_set) {
-    VCHECK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-    attr_set = true;
-  }
+  ensure_smem_attr((const void*)kern, smem);
   if (p.mc) {  // clusters of two CTAs walking pair tiles (see ConvParams::mc)
     if (RKB > 0) fail(1, "conv: multicast with resident weights");
     const int pairs = std::min(p.n_tiles, num_sms() / 2);

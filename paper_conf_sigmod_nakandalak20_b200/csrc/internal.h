@@ -122,9 +122,10 @@ struct JoinResult {
 // pair_str / pair_img: device int32 [n_str]; rows [0,n_train) train, then test, each in T_str order.
 JoinResult join_keys(const int64_t* d_img_keys, int64_t n_img, const int64_t* d_str_keys, int64_t n_str,
                      uint64_t split_subseed, int32_t* d_pair_str, int32_t* d_pair_img, cudaStream_t st);
+// bad: device int, OR-ed with 1 when a joined X value is not bf16-representable
 void launch_concat(const float* X, int d_s, int ds_pad, const bf16* F, int d_l, const int32_t* pair_str,
                    const int32_t* pair_img, const uint8_t* labels, int64_t n_pairs, int ld, bf16* MM,
-                   uint8_t* y, cudaStream_t st);
+                   uint8_t* y, int* bad, cudaStream_t st);
 
 // ---- LR (M) ----
 struct LRWork;  // device scratch for one layer
@@ -169,6 +170,8 @@ void prof_end(cudaStream_t st, int cls, double flops, double bytes, const char* 
 bool prof_labels();  // true when per-launch records are logged (VISTA_PROF_LOG)
 
 int num_sms();
+// cudaFuncAttributeMaxDynamicSharedMemorySize = bytes for fn on the current device (once per device)
+void ensure_smem_attr(const void* fn, int bytes);
 void set_sm_budget(int n);  // per-thread grid cap for persistent launches (0 = all SMs)
 
 }  // namespace vista

@@ -207,11 +207,12 @@ void fill_u64(unsigned long long* p, uint64_t n, unsigned long long v, cudaStrea
 
 // ---- concat (Eq. (4)): one warp per MM row, 16-byte stores ----
 // MM[p] = [bf16(X[s_p, 0..d_s)), 0 .. ds_pad, F[i_p, 0..d_l), 0 .. ld];  y[p] = labels[s_p].
-// X values are bf16-representable (generator contract), so the conversion is exact.
+// X values must be bf16-representable (include/vista.h precondition), so the conversion is exact; a value
+// with any of its low 16 bits set sets *bad (vista_transfer then fails with VISTA_ERR_INVALID_ARG).
 __global__ void concat_kernel(const float* __restrict__ X, int d_s, int ds_pad, const bf16* __restrict__ F, int d_l,
                               const int32_t* __restrict__ pair_str, const int32_t* __restrict__ pair_img,
                               const uint8_t* __restrict__ labels, int64_t n, int ld, bf16* __restrict__ MM,
-                              uint8_t* __restrict__ y) {
+                              uint8_t* __restrict__ y, int* __restrict__ bad) {
   const int lane = threadIdx.x & 31;
   const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
   for (int64_t p = blockIdx.x * (int64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); p < n; p += warps) {
@@ -220,11 +221,14 @@ __global__ void concat_kernel(const float* __restrict__ X, int d_s, int ds_pad, 
     const float* xs = X + (size_t)s * d_s;
     for (int c8 = lane; c8 * 8 < ds_pad; c8 += 32) {
       float f[8];
+      uint32_t low = 0;
 #pragma unroll
       for (int j = 0; j < 8; ++j) {
         const int c = c8 * 8 + j;
         f[j] = c < d_s ? xs[c] : 0.0f;
+        low |= __float_as_uint(f[j]) & 0xffffu;
       }
+      if (low) atomicOr(bad, 1);
       uint4 v;
       v.x = pack_bf16x2(f[0], f[1]);
       v.y = pack_bf16x2(f[2], f[3]);
@@ -276,13 +280,14 @@ void launch_concat_f32(const float* X, int d_s, int ds_pad, const float* F, int 
 
 void launch_concat(const float* X, int d_s, int ds_pad, const bf16* F, int d_l, const int32_t* pair_str,
                    const int32_t* pair_img, const uint8_t* labels, int64_t n_pairs, int ld, bf16* MM, uint8_t* y,
-                   cudaStream_t st) {
+                   int* bad, cudaStream_t st) {
   if (n_pairs <= 0) return;
   int64_t blocks = (n_pairs + 7) / 8;
   const int64_t cap = (int64_t)num_sms() * 8;
   if (blocks > cap) blocks = cap;
   prof_begin(st);
-  concat_kernel<<<(int)blocks, 256, 0, st>>>(X, d_s, ds_pad, F, d_l, pair_str, pair_img, labels, n_pairs, ld, MM, y);
+  concat_kernel<<<(int)blocks, 256, 0, st>>>(X, d_s, ds_pad, F, d_l, pair_str, pair_img, labels, n_pairs, ld, MM, y,
+                                             bad);
   LAUNCHED();
   prof_end(st, 4, 0, (double)n_pairs * (4.0 * d_s + 2.0 * d_l + 2.0 * ld + 9));
 }

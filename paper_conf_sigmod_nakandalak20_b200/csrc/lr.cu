@@ -431,13 +431,7 @@ struct StreamCfg {
 template <int MODE, typename E>
 static void run_pass(const PassArgs& a, const StreamCfg& c, cudaStream_t st) {
   auto go = [&](void (*kern)(PassArgs)) {
-    static std::mutex mu;
-    static std::set<const void*> done;  // opt-in shared memory, once per kernel instance
-    {
-      std::lock_guard<std::mutex> lk(mu);
-      if (done.insert((const void*)kern).second)
-        VCHECK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
-    }
+    ensure_smem_attr((const void*)kern, 227 * 1024);
     kern<<<c.grid, c.threads + 32, c.smem, st>>>(a);
   };
   switch (c.ch) {

@@ -468,14 +468,20 @@ MLPResult mlp_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_
       colsum(part, head_blocks, h, g3, st);
     }
     // backward
-    transpose(dH2, h, nullptr, 0, n, h, dH2T, np, part, st);  // + grad b2 partials
-    colsum(part, nbt, h, gb2, st);
-    transpose(H1, h, nullptr, 0, n, h, H1T, np, nullptr, st);
-    gemm_tn(dH2T, h, (int)n, (int)np, H1T, h, (int)np, ones, zeros, false, G2, true, st, kMlpCls);  // dW2
-    gemm_tn(dH2, n, h, h, W2T, h, h, ones, zeros, false, dH1p, false, st, kMlpCls);                  // dH2 W2
-    transpose(dH1p, h, H1, h, n, h, dH1T, np, part, st);  // . [H1 > 0], + grad b1 partials
-    colsum(part, nbt, h, gb1, st);
-    gemm_tn(dH1T, h, (int)n, (int)np, XT, Kp, (int)np, ones, zeros, false, G1, true, st, kMlpCls);  // dW1
+    if (n > 0) {
+      transpose(dH2, h, nullptr, 0, n, h, dH2T, np, part, st);  // + grad b2 partials
+      colsum(part, nbt, h, gb2, st);
+      transpose(H1, h, nullptr, 0, n, h, H1T, np, nullptr, st);
+      gemm_tn(dH2T, h, (int)n, (int)np, H1T, h, (int)np, ones, zeros, false, G2, true, st, kMlpCls);  // dW2
+      gemm_tn(dH2, n, h, h, W2T, h, h, ones, zeros, false, dH1p, false, st, kMlpCls);                  // dH2 W2
+      transpose(dH1p, h, H1, h, n, h, dH1T, np, part, st);  // . [H1 > 0], + grad b1 partials
+      colsum(part, nbt, h, gb1, st);
+      gemm_tn(dH1T, h, (int)n, (int)np, XT, Kp, (int)np, ones, zeros, false, G1, true, st, kMlpCls);  // dW1
+    } else {
+      // a rank without train rows still takes part in every collective, with a zero contribution (G was
+      // allreduced in place last step, so it must be cleared, not left holding the global sums)
+      VCHECK(cudaMemsetAsync(G, 0, nG * 4, st));
+    }
     // loss and grad b3 (fp64, fixed order), then the allreduces across ranks
     VCHECK(cudaMemcpyAsync(hs.data(), scal, 2 * head_blocks * 8, cudaMemcpyDeviceToHost, st));
     VCHECK(cudaStreamSynchronize(st));

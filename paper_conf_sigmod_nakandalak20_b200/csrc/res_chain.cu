@@ -354,11 +354,7 @@ static void launch_chain(const ConvLayer& Lc, const ConvLayer* La, const bf16* b
   p.sh_a = La ? La->shift : Lc.shift;
   p.M = M;
   p.n_mt = (M + BMr - 1) / BMr;
-  static bool attr = false;
-  if (!attr) {
-    VCHECK(cudaFuncSetAttribute(res_chain_kernel<MID, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, RC<MID, V>::kSmem));
-    attr = true;
-  }
+  ensure_smem_attr((const void*)res_chain_kernel<MID, V>, RC<MID, V>::kSmem);
   const int grid = p.n_mt < num_sms() ? p.n_mt : num_sms();
   res_chain_kernel<MID, V><<<grid, kThr, RC<MID, V>::kSmem, st>>>(tb, tr, to, ta, Lc.tmap_w, La ? La->tmap_w : Lc.tmap_w, p);
   LAUNCHED();

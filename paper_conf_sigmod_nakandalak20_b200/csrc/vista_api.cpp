@@ -10,6 +10,8 @@
 #include <cstdlib>
 #include <cstring>
 #include <memory>
+#include <mutex>
+#include <set>
 #include <string>
 #include <vector>
 
@@ -36,17 +38,36 @@ long long launches_total() { return g_launches.load(); }
 static thread_local int t_sm_budget = 0;
 void set_sm_budget(int n) { t_sm_budget = n; }
 int num_sms() {
-  static int n = 0;
+  // per device (a process may drive several devices through several ctxs)
+  static std::atomic<int> cache[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int n = dev >= 0 && dev < 64 ? cache[dev].load(std::memory_order_relaxed) : 0;
   if (!n) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 148;
+    if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) {
+      cudaGetLastError();
+      n = 148;
+    }
     if (const char* e = getenv("VISTA_SM_CAP")) {  // measurement only: cap every launch's grid
       const int cap = atoi(e);
       if (cap > 0 && cap < n) n = cap;
     }
+    if (dev >= 0 && dev < 64) cache[dev].store(n, std::memory_order_relaxed);
   }
   return t_sm_budget > 0 && t_sm_budget < n ? t_sm_budget : n;
+}
+
+// opt-in dynamic shared memory of a kernel, once per (device, kernel): function attributes are per
+// device context, so a cache keyed by the kernel alone would skip the second device of a process
+void ensure_smem_attr(const void* fn, int bytes) {
+  static std::mutex mu;
+  static std::set<std::pair<int, const void*>> done;
+  int dev = 0;
+  VCHECK(cudaGetDevice(&dev));
+  std::lock_guard<std::mutex> lk(mu);
+  if (done.count({dev, fn})) return;
+  VCHECK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
+  done.insert({dev, fn});
 }
 
 // ---------------- profiler ----------------
@@ -163,6 +184,26 @@ static void nccl_allreduce_f32(float* buf, int64_t count, cudaStream_t st, void*
   if (rc != 0) fail(6, std::string("ncclAllReduce: ") + (n.GetErrorString ? n.GetErrorString(rc) : "error"));
 }
 
+// ---------------- caller-supplied collective (vista_sys_cfg.allreduce) ----------------
+// world > 1 without NCCL (ranks sharing one GPU, or a gloo group): the partial sums go device -> host, the
+// caller's in-place SUM allreduce combines them across ranks, and the sums come back to the device.
+struct HookAR {
+  int32_t (*fn)(void*, int64_t, int32_t, void*) = nullptr;
+  void* user = nullptr;
+};
+static void hook_allreduce(void* d_buf, int64_t count, int32_t dtype, cudaStream_t st, void* user) {
+  const HookAR* h = static_cast<const HookAR*>(user);
+  const size_t bytes = (size_t)count * (dtype == 0 ? 8 : 4);
+  std::vector<uint8_t> host(bytes ? bytes : 8);
+  VCHECK(cudaMemcpyAsync(host.data(), d_buf, bytes, cudaMemcpyDeviceToHost, st));
+  VCHECK(cudaStreamSynchronize(st));
+  if (h->fn(host.data(), count, dtype, h->user) != 0) fail(6, "caller-supplied allreduce failed");
+  VCHECK(cudaMemcpyAsync(d_buf, host.data(), bytes, cudaMemcpyHostToDevice, st));
+  VCHECK(cudaStreamSynchronize(st));  // the host staging buffer dies at return
+}
+static void hook_allreduce_f64(double* d, int64_t n, cudaStream_t st, void* u) { hook_allreduce(d, n, 0, st, u); }
+static void hook_allreduce_f32(float* d, int64_t n, cudaStream_t st, void* u) { hook_allreduce(d, n, 1, st, u); }
+
 // ---------------- helpers ----------------
 static uint16_t f2bf_bits(float f) {  // f is bf16-representable (generator contract)
   uint32_t u;
@@ -245,6 +286,9 @@ struct vista_ctx {
   int64_t n_pairs = 0, n_train = 0;
   bool transferred = false;
   void* nccl_comm = nullptr;
+  HookAR hook;                   // world > 1 without NCCL
+  DevBuf d_flags;                // device status flags of a transfer (X not bf16-representable)
+  int64_t peak_meas = 0, peak_res_meas = 0;  // measured peak device bytes of the last transfer
   std::unique_ptr<Profiler> prof;
   bool profiling = false;
   // Tap g_l fused into the producing conv's epilogue (VISTA_FUSED_TAP=1) or the standalone tap kernel
@@ -280,7 +324,7 @@ struct vista_ctx {
     tapacc.release();
     for (auto& mi : mlp_init)
       if (mi.dev) mi.dev->release();
-    for (DevBuf* b : {&pair_str, &pair_img, &d_X, &d_labels, &d_img_keys, &d_str_keys, &d_px}) b->release();
+    for (DevBuf* b : {&pair_str, &pair_img, &d_X, &d_labels, &d_img_keys, &d_str_keys, &d_px, &d_flags}) b->release();
     if (stream) cudaStreamSynchronize(stream);
     for (auto& L : convs) conv_layer_free(L);
     for (auto& L : convs_cat) conv_layer_free(L);
@@ -334,8 +378,27 @@ vista_status guarded(vista_ctx* c, F&& f) {
   }
 }
 
+// Transient per-image device bytes a block allocates inside a launch: the zero-padded input copy of
+// the padded row view (conv_forward: Cin = 8 first layers with padding, e.g. VGG16 conv1_1).
+int64_t transient_per_img(const vista_ctx* c, int t) {
+  if (c->f32) return 0;
+  int64_t m = 0;
+  for (const OpDesc& op : c->net.stages[t].ops) {
+    if (op.kind != OP_CONV) continue;
+    const LayerSpec& l = c->net.layers[op.layer];
+    if (l.Cin == 8 && l.stride == 1 && l.pad > 0 && l.groups == 1 && l.R <= 8 && !l.s2d) {
+      const int Wo = conv_out_dim(op.W, l.S, 1, l.pad);
+      m = std::max<int64_t>(m, (int64_t)(op.H + 2 * l.pad) * std::max(op.W + 2 * l.pad, Wo + 7) * 16);
+    }
+  }
+  return m;
+}
+
 // HBM planner (S6): Eq. (6)-style peak = weights + pixels + A_{t-1} + A_t + F's + MM's + scratch(B_t);
 // search micro-batches from the largest down, first feasible wins (Alg. 1 shape).
+// Scratch slots are grow-only across blocks (prepare_slots never shrinks them), so the scratch held
+// while block t runs is sum over slots b of max over blocks t' <= t of slot_b(t') * B_t', plus block t's
+// transient bytes.
 void plan_memory(vista_ctx* c, uint64_t budget) {
   const auto& S = c->net.stages;
   c->micro.assign(c->t_max + 1, 0);
@@ -349,22 +412,27 @@ void plan_memory(vista_ctx* c, uint64_t budget) {
   int64_t peak = 0;
   if (c->sys.plan != VISTA_PLAN_STAGED) {
     // Eager / Lazy: features of all of L (incl. FC taps) + two micro-batch activation buffers + slots
-    int64_t f_all = 0, max_out = 0, slot_per_img = 0;
+    int64_t f_all = 0, max_out = 0, slots = 0, trans = 0;
     for (int t : c->taps) f_all += c->n_img * (int64_t)S[t].d_tap * c->esz;
+    for (int b = BUF_T0; b < NUM_BUFS; ++b) {
+      int64_t m = 0;
+      for (int t = 0; t <= c->t_max; ++t) m = std::max<int64_t>(m, S[t].slot_elems[b] * c->esz);
+      slots += m;
+    }
     for (int t = 0; t <= c->t_max; ++t) {
       max_out = std::max<int64_t>(max_out, S[t].out_elems);
-      int64_t s = 0;
-      for (int b = BUF_T0; b < NUM_BUFS; ++b) s += S[t].slot_elems[b] * c->esz;
-      slot_per_img = std::max(slot_per_img, s);
+      trans = std::max(trans, transient_per_img(c, t));
     }
     const int64_t fixed = c->weight_bytes + px + f_all + mm_bytes + join_bytes + (256ll << 20);
-    const int64_t per_img = slot_per_img + 2 * max_out * c->esz;
+    const int64_t per_img = slots + 2 * max_out * c->esz + trans;
     int B = c->sys.micro_batch > 0 ? c->sys.micro_batch : 0;
     for (int64_t b = std::min<int64_t>(1024, std::max<int64_t>(c->n_img, 1)); B == 0 && b >= 1;
          b = b > 8 ? b / 2 : b - 1)
       if ((uint64_t)(fixed + b * per_img) <= budget) B = (int)b;
-    if (B <= 0) fail(VISTA_ERR_NO_PLAN, "no micro-batch fits the HBM budget (eager/lazy)");
+    if (B <= 0 || (uint64_t)(fixed + (int64_t)B * per_img) > budget)
+      fail(VISTA_ERR_NO_PLAN, "no micro-batch fits the HBM budget (eager/lazy)");
     c->micro.assign(c->t_max + 1, B);
+    c->chunk = B;  // vista_materialize runs in chunks of one micro-batch under these plans
     c->peak_pred = fixed + (int64_t)B * per_img;
     return;
   }
@@ -377,26 +445,28 @@ void plan_memory(vista_ctx* c, uint64_t budget) {
     if (S[t].fc_tap) f_fc += c->n_img * (int64_t)S[t].d_tap * c->esz;
   auto plan_chunk = [&](int64_t CH, std::vector<int>& micro, int64_t& pk) -> bool {
     pk = 0;
-    const bool chunked = CH < c->n_img;
     const int64_t pxc = CH * (int64_t)S[0].in_elems;  // host pixels are streamed per chunk
     int64_t arena[2] = {0, 0};                         // ping-pong activation arenas (A_t in arena t % 2)
     for (int t = 0; t <= c->t_max; ++t) arena[t & 1] = std::max<int64_t>(arena[t & 1], CH * S[t].out_elems * c->esz);
-    (void)chunked;
+    const int64_t fixed = c->weight_bytes + pxc + arena[0] + arena[1] + mm_bytes + f_bytes + f_fc + join_bytes +
+                          (256ll << 20);
+    int64_t slot_max[NUM_BUFS] = {0};  // bytes each grow-only slot holds after blocks < t
+    auto need = [&](int t, int64_t b) {
+      int64_t sl = 0;
+      for (int q = BUF_T0; q < NUM_BUFS; ++q) sl += std::max(slot_max[q], S[t].slot_elems[q] * c->esz * b);
+      return fixed + sl + transient_per_img(c, t) * b;
+    };
     for (int t = 0; t <= c->t_max; ++t) {
-      int64_t slot_per_img = 0;
-      for (int b = BUF_T0; b < NUM_BUFS; ++b) slot_per_img += S[t].slot_elems[b] * c->esz;
-      const int64_t fixed = c->weight_bytes + pxc + arena[0] + arena[1] + mm_bytes + f_bytes + f_fc + join_bytes +
-                            (256ll << 20);
       int B = 0;
       if (c->sys.micro_batch > 0 && t == 0) {
         B = (int)std::min<int64_t>(c->sys.micro_batch, std::max<int64_t>(CH, 1));
-        if ((uint64_t)(fixed + B * slot_per_img) > budget) return false;
+        if ((uint64_t)need(t, B) > budget) return false;
       } else {
         // larger micro-batches give larger GEMMs per launch (measured: 256 -> 1024 is +7 % img/s);
         // activations of one micro-batch exceed L2 either way
         const int64_t cap_B = t == 0 ? 1024 : 16384;
         for (int64_t b = std::min<int64_t>(cap_B, std::max<int64_t>(CH, 1)); b >= 1; b = b > 8 ? b / 2 : b - 1) {
-          if ((uint64_t)(fixed + b * slot_per_img) <= budget) {
+          if ((uint64_t)need(t, b) <= budget) {
             B = (int)b;
             break;
           }
@@ -404,7 +474,8 @@ void plan_memory(vista_ctx* c, uint64_t budget) {
       }
       if (B <= 0) return false;
       micro[t] = B;
-      pk = std::max(pk, fixed + (int64_t)B * slot_per_img);
+      pk = std::max(pk, need(t, B));
+      for (int q = BUF_T0; q < NUM_BUFS; ++q) slot_max[q] = std::max(slot_max[q], S[t].slot_elems[q] * c->esz * B);
     }
     return true;
   };
@@ -738,29 +809,47 @@ bool run_block(vista_ctx* c, int t, const void* in_base, void* out_base, int64_t
   return fused;
 }
 
-// Eager (Fig 5C) and Lazy (Fig 5A) schedules: per micro-batch of images, run blocks 0..t_last from
-// the raw pixels with the activations in two ping-pong micro-batch buffers, and tap every requested
-// layer in `want` (Eager: all of L in one pass; Lazy: one layer per pass, recomputing from pixels).
-void run_unstaged(vista_ctx* c, const uint8_t* px, int t_last, const std::vector<int>& want,
-                  const std::vector<cudaEvent_t>* in_ready = nullptr) {
+// Eager (Fig 5C) and Lazy (Fig 5A) schedules: per micro-batch of images, run blocks t_first..t_last with
+// the activations in two ping-pong micro-batch buffers, and tap every requested layer in `want` (Eager:
+// all of L in one pass; Lazy: one layer per pass, recomputing from the start).  t_first = 0 starts from
+// the raw pixels px; t_first = t0 + 1 starts from a pre-materialised base layer (App. B)
+// holding block t0's output: `base` device memory, or host memory copied per micro-batch into the
+// buffer block t0 would have written (its F_t0 = g(base) is tapped too when t0 is in `want`).
+void run_unstaged(vista_ctx* c, const uint8_t* px, int t_first, int t_last, const std::vector<int>& want,
+                  const std::vector<cudaEvent_t>* in_ready = nullptr, const void* base = nullptr,
+                  bool host_base = false) {
   const auto& S = c->net.stages;
   const int B = c->micro[0];
+  const int t0 = t_first - 1;  // block whose output is the base (t_first > 0)
   void* slot[NUM_BUFS] = {nullptr};
   int64_t max_out = 0;
-  for (int t = 0; t <= t_last; ++t) {
-    prepare_slots(c, t, B, slot);
+  for (int t = std::max(t0, 0); t <= t_last; ++t) {
+    if (t >= t_first) prepare_slots(c, t, B, slot);
     max_out = std::max<int64_t>(max_out, S[t].out_elems);
   }
   DevBuf act[2];
   act[0].alloc((size_t)B * max_out * c->esz + 16);
   act[1].alloc((size_t)B * max_out * c->esz + 16);
+  const size_t base_img = t0 >= 0 ? (size_t)S[t0].out_elems * c->esz : 0;
   for (int64_t i0 = 0; i0 < c->n_img; i0 += B) {
     const int nb = (int)std::min<int64_t>(B, c->n_img - i0);
     if (in_ready) VCHECK(cudaStreamWaitEvent(c->stream, (*in_ready)[(size_t)(i0 / B)], 0));
-    for (int t = 0; t <= t_last; ++t) {
-      const void* in = t == 0 ? (const void*)(px + (size_t)i0 * S[0].in_elems) : act[(t - 1) & 1].p;
-      void* out = act[t & 1].p;
-      run_ops(c, t, in, out, nb, slot, nullptr);
+    const void* prev = nullptr;  // this micro-batch's output of block t0
+    if (t0 >= 0) {
+      if (host_base) {
+        VCHECK(cudaMemcpyAsync(act[t0 & 1].p, (const uint8_t*)base + (size_t)i0 * base_img, (size_t)nb * base_img,
+                               cudaMemcpyHostToDevice, c->stream));
+        prev = act[t0 & 1].p;
+      } else {
+        prev = (const uint8_t*)base + (size_t)i0 * base_img;
+      }
+    }
+    for (int t = std::max(t0, 0); t <= t_last; ++t) {
+      const void* out = t == t0 ? prev : act[t & 1].p;
+      if (t >= t_first) {
+        const void* in = t == 0 ? (const void*)(px + (size_t)i0 * S[0].in_elems) : (t - 1 == t0 ? prev : act[(t - 1) & 1].p);
+        run_ops(c, t, in, const_cast<void*>(out), nb, slot, nullptr);
+      }
       if (std::find(want.begin(), want.end(), t) == want.end()) continue;
       void* Ft = (uint8_t*)c->F[t]->p + (size_t)i0 * S[t].d_tap * c->esz;
       if (S[t].fc_tap)
@@ -884,14 +973,24 @@ VISTA_API vista_status vista_plan(vista_cnn cnn, const int32_t* layers, int32_t 
     if (!budget) {
       size_t fr = 0, tot = 0;
       VCHECK(cudaMemGetInfo(&fr, &tot));
+      // memory the default pool keeps reserved but unused (other ctxs' freed buffers) is available too
+      cudaMemPool_t pool;
+      uint64_t res = 0, used = 0;
+      VCHECK(cudaDeviceGetDefaultMemPool(&pool, c->sys.device));
+      VCHECK(cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &res));
+      VCHECK(cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemCurrent, &used));
+      fr += res > used ? (size_t)(res - used) : 0;
       budget = fr > (4ull << 30) ? fr - (4ull << 30) : fr / 2;
       budget += c->weight_bytes;  // weights already allocated
     }
     plan_memory(c.get(), budget);
     c->slot_store.clear();
     for (int b = 0; b < NUM_BUFS; ++b) c->slot_store.emplace_back(new DevBuf());
-    if (c->sys.world > 1) {
-      if (!c->sys.nccl_uid) fail(1, "world > 1 needs nccl_uid");
+    if (c->sys.world > 1 && !c->sys.nccl_uid) {
+      if (!c->sys.allreduce) fail(1, "world > 1 needs nccl_uid or a caller-supplied allreduce");
+      c->hook.fn = c->sys.allreduce;
+      c->hook.user = c->sys.allreduce_user;
+    } else if (c->sys.world > 1) {
       Nccl& n = nccl_lib();
       NcclId id;
       std::memcpy(id.internal, c->sys.nccl_uid, 128);
@@ -931,6 +1030,8 @@ VISTA_API vista_status vista_plan_info(const vista_ctx* c, vista_plan_info_t* o)
   o->d_s = c->d_s;
   o->ds_pad = c->ds_pad;
   o->chunk_images = c->chunk;
+  o->peak_bytes_meas = c->peak_meas;
+  o->peak_reserved_meas = c->peak_res_meas;
   return VISTA_OK;
 }
 
@@ -942,12 +1043,22 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
   {
     if (c->n_img > 0 && !image_keys) fail(1, "image_keys is NULL");
     if (c->n_img > 0 && !images && !base) fail(1, "images / base is NULL");
-    if (base && c->sys.plan != VISTA_PLAN_STAGED) fail(1, "a pre-materialised base layer needs the Staged plan");
     if (c->n_str > 0 && (!str_keys || !labels || (c->d_s > 0 && !structured))) fail(1, "structured table is NULL");
     VCHECK(cudaSetDevice(c->sys.device));
     c->transferred = false;
     cudaStream_t st = c->stream;
     const auto& S = c->net.stages;
+    // measured peak (plan_info): reset the default pool's high-water marks to the bytes in use now
+    cudaMemPool_t pool;
+    VCHECK(cudaDeviceGetDefaultMemPool(&pool, c->sys.device));
+    VCHECK(cudaStreamSynchronize(st));
+    {
+      uint64_t zero = 0;
+      VCHECK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrUsedMemHigh, &zero));
+      VCHECK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReservedMemHigh, &zero));
+    }
+    c->d_flags.ensure(16);
+    VCHECK(cudaMemsetAsync(c->d_flags.p, 0, 16, st));
     // ---- inputs (H2D when given host pointers) ----
     // (host pixels are streamed per stage-1 micro-batch right before the inference that reads them: Staged
     // chunk by chunk, Eager / Lazy once.  Not here: the small key / table copies and the join below would
@@ -1000,19 +1111,22 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
       else
         launch_concat(X, c->d_s, c->ds_pad, (const bf16*)c->feat[t], S[t].d_tap, (const int32_t*)c->pair_str.p,
                       (const int32_t*)c->pair_img.p, lab, c->n_pairs, ld, (bf16*)c->MM[k]->p, (uint8_t*)c->Y[k]->p,
-                      st);
+                      (int*)c->d_flags.p, st);
     };
     if (c->sys.plan != VISTA_PLAN_STAGED) {
       // ---- Eager / Lazy (Fig 5C / 5A): features of every layer, no resident full activations ----
+      // with a pre-materialised base (App. B): Eager = one pass base -> all of L; Lazy = "Lazy-5 with
+      // Pre-mat": one pass per layer from the stored base
       const std::vector<cudaEvent_t>* unstaged_ev = nullptr;
       if (!base && c->n_img > 0 && !is_device_ptr(images)) {
         unstaged_ev = stream_host_pixels(c, images, 0, c->n_img);
         px = (const uint8_t*)c->d_px.p;
       }
+      const int t_first = base ? t0 + 1 : 0;
       if (c->sys.plan == VISTA_PLAN_EAGER) {
-        run_unstaged(c, px, c->t_max, c->taps, unstaged_ev);
+        run_unstaged(c, px, t_first, c->t_max, c->taps, unstaged_ev, base, host_base);
       } else {
-        for (int t : c->taps) run_unstaged(c, px, t, std::vector<int>{t}, unstaged_ev);
+        for (int t : c->taps) run_unstaged(c, px, t_first, t, std::vector<int>{t}, unstaged_ev, base, host_base);
       }
       for (size_t k = 0; k < c->taps.size(); ++k) concat_layer((int)k);
     }
@@ -1074,8 +1188,19 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
     }
     if (chunked)
       for (size_t k = 0; k < c->taps.size(); ++k) concat_layer((int)k);
+    int flags[4] = {0, 0, 0, 0};
+    VCHECK(cudaMemcpyAsync(flags, c->d_flags.p, 16, cudaMemcpyDeviceToHost, st));
     VCHECK(cudaStreamSynchronize(st));
     if (g_prof) g_prof->flush();
+    {
+      uint64_t used_hi = 0, res_hi = 0;
+      VCHECK(cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemHigh, &used_hi));
+      VCHECK(cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemHigh, &res_hi));
+      c->peak_meas = c->weight_bytes + (int64_t)used_hi;
+      c->peak_res_meas = c->weight_bytes + (int64_t)res_hi;
+    }
+    if (flags[0] & 1)
+      fail(1, "structured value not bf16-representable (include/vista.h: X values must be bf16-representable)");
     c->transferred = true;
   }
 }
@@ -1182,13 +1307,18 @@ VISTA_API vista_status vista_train(vista_ctx* c, int32_t k, double* weights_out,
     std::vector<uint8_t> real(ld, 0);
     for (int j = 0; j < c->d_s; ++j) real[j] = 1;
     for (int j = 0; j < d_l; ++j) real[c->ds_pad + j] = 1;
-    allreduce_fn ar = c->sys.world > 1 ? nccl_allreduce_f64 : nullptr;
+    allreduce_fn ar = nullptr;
+    void* ar_user = nullptr;
+    if (c->sys.world > 1) {
+      ar = c->nccl_comm ? nccl_allreduce_f64 : hook_allreduce_f64;
+      ar_user = c->nccl_comm ? c->nccl_comm : (void*)&c->hook;
+    }
     LRResult r = c->f32 ? lr_train_f32((const float*)c->MM[k]->p, (const uint8_t*)c->Y[k]->p, c->n_pairs,
                                        c->n_train, ld, real.data(), c->lr.iters, c->lr.power_iters, c->lr.lambda,
-                                       c->lr.alpha, ar, c->nccl_comm, c->stream)
+                                       c->lr.alpha, ar, ar_user, c->stream)
                         : lr_train((const bf16*)c->MM[k]->p, (const uint8_t*)c->Y[k]->p, c->n_pairs, c->n_train,
                                    ld, real.data(), c->lr.iters, c->lr.power_iters, c->lr.lambda, c->lr.alpha, ar,
-                                   c->nccl_comm, c->stream);
+                                   ar_user, c->stream);
     if (g_prof) g_prof->flush();
     if (weights_out) {
       for (int j = 0; j < c->d_s; ++j) weights_out[j] = r.w[j];
@@ -1261,10 +1391,12 @@ VISTA_API vista_status vista_train_mlp(vista_ctx* c, int32_t k, const vista_mlp_
     const float* W1 = (const float*)mi.dev->p;
     const float* W2 = W1 + nW1;
     const float* w3 = W2 + nW2;
-    const bool multi = c->sys.world > 1;
+    const bool multi = c->sys.world > 1, nccl = c->nccl_comm != nullptr;
     MLPResult r = mlp_train((const bf16*)c->MM[k]->p, (const uint8_t*)c->Y[k]->p, c->n_pairs, c->n_train, ld, real,
-                            W1, W2, w3, h, iters, lr, weights_out != nullptr, multi ? nccl_allreduce_f64 : nullptr,
-                            multi ? nccl_allreduce_f32 : nullptr, c->nccl_comm, c->stream);
+                            W1, W2, w3, h, iters, lr, weights_out != nullptr,
+                            multi ? (nccl ? nccl_allreduce_f64 : hook_allreduce_f64) : nullptr,
+                            multi ? (nccl ? nccl_allreduce_f32 : hook_allreduce_f32) : nullptr,
+                            nccl ? c->nccl_comm : (void*)&c->hook, c->stream);
     if (g_prof) g_prof->flush();
     if (weights_out) {
       float* o = weights_out;
@@ -1302,7 +1434,15 @@ VISTA_API void vista_destroy(vista_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->sys.device);
   if (c->stream) cudaStreamSynchronize(c->stream);
+  const int dev = c->sys.device;
   delete c;
+  // the ctx's stream-ordered buffers went back to the device's default pool (release threshold raised at
+  // plan time): give the memory back to the device so later ctxs (their default budget reads free HBM)
+  // and other allocators of the process see it
+  cudaMemPool_t pool;
+  if (cudaDeviceSynchronize() == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess)
+    cudaMemPoolTrimTo(pool, 0);
+  cudaGetLastError();
 }
 
 VISTA_API int64_t vista_kernel_launches(void) { return (int64_t)launches_total(); }
@@ -1404,6 +1544,24 @@ VISTA_API vista_status vista_conv2d_tap(const void* x, int32_t N, int32_t H, int
     }
     cudaFree(acc);
     conv_layer_free(L);
+  });
+}
+
+VISTA_API vista_status vista_join(const int64_t* img_keys, int64_t n_img, const int64_t* str_keys, int64_t n_str,
+                                  uint64_t split_seed, int32_t* pair_str, int32_t* pair_img, int64_t* n_pairs,
+                                  int64_t* n_train, void* stream) {
+  return guarded(nullptr, [&] {
+    if (n_img < 0 || n_str < 0 || !n_pairs || !n_train || (n_img > 0 && !img_keys) ||
+        (n_str > 0 && (!str_keys || !pair_str || !pair_img)))
+      fail(1, "vista_join: bad arguments");
+    cudaStream_t st = as_stream(stream);
+    tl_stream = st;
+    JoinResult jr = join_keys(img_keys, n_img, str_keys, n_str, vg_subseed(split_seed, VG_S_SPLIT), pair_str,
+                              pair_img, st);
+    if (jr.dup & 2) fail(1, "a key equals the reserved empty-slot value INT64_MIN");
+    if (jr.dup & 1) fail(VISTA_ERR_DUP_KEY, "duplicate key in T_img or T_str (ID must be a primary key)");
+    *n_pairs = jr.n_pairs;
+    *n_train = jr.n_train;
   });
 }
 

@@ -35,15 +35,21 @@ class LRCfg(ctypes.Structure):
     _fields_ = [("iters", _i32), ("power_iters", _i32), ("lam", _f64), ("alpha", _f64), ("split_seed", _u64)]
 
 
+# int32_t (*allreduce)(void* host_buf, int64_t count, int32_t dtype, void* user) of vista_sys_cfg
+ALLREDUCE_FN = ctypes.CFUNCTYPE(_i32, _vp, _i64, _i32, _vp)
+
+
 class SysCfg(ctypes.Structure):
     _fields_ = [("rank", _i32), ("world", _i32), ("nccl_uid", _vp), ("device", _i32), ("hbm_budget_bytes", _u64),
-                ("dtype", _i32), ("plan", _i32), ("stream", _vp), ("micro_batch", _i32)]
+                ("dtype", _i32), ("plan", _i32), ("stream", _vp), ("micro_batch", _i32),
+                ("allreduce", ALLREDUCE_FN), ("allreduce_user", _vp)]
 
 
 class PlanInfo(ctypes.Structure):
     _fields_ = [("n_layers", _i32), ("tap", _i32 * 8), ("d_l", _i32 * 8), ("ld", _i32 * 8),
                 ("micro_batch", _i32 * 8), ("act_bytes", _i64 * 8), ("peak_bytes_pred", _i64),
-                ("weight_bytes", _i64), ("d_s", _i32), ("ds_pad", _i32), ("chunk_images", _i64)]
+                ("weight_bytes", _i64), ("d_s", _i32), ("ds_pad", _i32), ("chunk_images", _i64),
+                ("peak_bytes_meas", _i64), ("peak_reserved_meas", _i64)]
 
 
 class Buffer(ctypes.Structure):
@@ -104,6 +110,8 @@ def lib():
                                        _vp, _vp, _vp, _vp]
         L.vista_kernel_launches.restype = _i64
         L.vista_tap.argtypes = [_vp, _i32, _i32, _i32, _i32, _vp, _vp]
+        L.vista_join.argtypes = [_vp, _i64, _vp, _i64, _u64, _vp, _vp, ctypes.POINTER(_i64), ctypes.POINTER(_i64),
+                                 _vp]
         L.vista_maxpool.argtypes = [_vp, _i32, _i32, _i32, _i32, _i32, _i32, _vp, _vp]
         L.vista_lrn.argtypes = [_vp, _i32, _i32, _i32, _i32, _vp, _vp]
         L.vista_avgpool.argtypes = [_vp, _i32, _i32, _i32, _i32, _vp, _vp]
@@ -175,6 +183,38 @@ def vista_conv2d_tap(x, w, scale, shift, stride=1, pad=0, residual=None, stream=
     return y, F
 
 
+def vista_join(img_keys, str_keys, split_seed=0, stream=None):
+    """S4 join on its own: device int64 key tensors -> (pair_str, pair_img) int32 device tensors of the
+    matched rows ([train | test], each in T_str order) and n_train."""
+    import torch
+    ns = str_keys.shape[0]
+    ps = torch.empty(max(ns, 1), dtype=torch.int32, device=str_keys.device)
+    pi = torch.empty(max(ns, 1), dtype=torch.int32, device=str_keys.device)
+    n_pairs, n_train = _i64(), _i64()
+    _check(lib().vista_join(_ptr(img_keys), img_keys.shape[0], _ptr(str_keys), ns, split_seed, _ptr(ps), _ptr(pi),
+                            ctypes.byref(n_pairs), ctypes.byref(n_train), _stream(stream)))
+    return ps[:n_pairs.value], pi[:n_pairs.value], n_train.value
+
+
+def torch_dist_allreduce(group=None):
+    """An allreduce for vista_sys_cfg.allreduce backed by a torch.distributed process group (e.g. gloo):
+    in-place SUM of the library's host buffer.  Marshalling only (the sums the library asks for are its
+    own per-rank partials)."""
+    import torch
+    import torch.distributed as dist
+
+    def fn(buf, count, dtype, user):
+        try:
+            ct = ctypes.c_double if dtype == 0 else ctypes.c_float
+            arr = np.ctypeslib.as_array((ct * count).from_address(buf))
+            t = torch.from_numpy(arr)
+            dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+            return 0
+        except Exception:  # never raise through the C frame
+            return 1
+    return fn
+
+
 def vista_kernel_launches() -> int:
     return int(lib().vista_kernel_launches())
 
@@ -244,16 +284,19 @@ class Vista:
     def __init__(self, cnn, layers=None, n_top=0, n_str_rows=0, d_s=0, n_images_local=0, iters=10,
                  power_iters=20, lam=0.01, alpha=0.5, split_seed=0, weight_seed=0, rank=0, world=1,
                  nccl_uid: bytes | None = None, device=0, hbm_budget_bytes=0, stream=None, micro_batch=0,
-                 plan="staged", dtype="bf16"):
-        """dtype: "bf16" (the tcgen05 product path) or "f32" (the fp32 check mode, reading R23)."""
+                 plan="staged", dtype="bf16", allreduce=None):
+        """dtype: "bf16" (the tcgen05 product path) or "f32" (the fp32 check mode, reading R23).
+        allreduce: a Python callable fn(host_ptr, count, dtype, user) -> int (e.g. torch_dist_allreduce())
+        used instead of NCCL when world > 1 and nccl_uid is None."""
         self.cnn = cnn
         self.dtype = dtype
         lr = LRCfg(iters, power_iters, lam, alpha, split_seed)
         self._uid = (ctypes.c_uint8 * 128).from_buffer_copy(nccl_uid) if nccl_uid else None
         plan_id = {"staged": 0, "eager": 1, "lazy": 2}[plan]
         dtype_id = {"bf16": 0, "f32": 1}[dtype]
+        self._ar = ALLREDUCE_FN(allreduce) if allreduce is not None else ALLREDUCE_FN()  # kept alive with self
         sys = SysCfg(rank, world, ctypes.addressof(self._uid) if self._uid is not None else None, device,
-                     hbm_budget_bytes, dtype_id, plan_id, stream, micro_batch)
+                     hbm_budget_bytes, dtype_id, plan_id, stream, micro_batch, self._ar, None)
         arr = None
         n_layers = 0
         if layers is not None:
@@ -273,7 +316,8 @@ class Vista:
         return dict(n_layers=n, tap=list(pi.tap[:n]), d_l=list(pi.d_l[:n]), ld=list(pi.ld[:n]),
                     micro_batch=list(pi.micro_batch[:n]), act_bytes=list(pi.act_bytes[:n]),
                     peak_bytes_pred=pi.peak_bytes_pred, weight_bytes=pi.weight_bytes, d_s=pi.d_s, ds_pad=pi.ds_pad,
-                    chunk_images=pi.chunk_images)
+                    chunk_images=pi.chunk_images, peak_bytes_meas=pi.peak_bytes_meas,
+                    peak_reserved_meas=pi.peak_reserved_meas)
 
     def transfer(self, images, image_keys, structured, str_keys, labels):
         _check(lib().vista_transfer(self.ctx, _ptr(images), _ptr(image_keys), _ptr(structured), _ptr(str_keys),

@@ -335,12 +335,62 @@ def test_pre_materialized_base_layer(cnn, taps, n, d_s, chunked):
         v.close()
 
 
-def test_base_layer_needs_staged_plan():
-    tab = gen.make_tables(4, 8)
-    v = Vista(0, layers=[1, 2], n_str_rows=4, d_s=8, n_images_local=4, iters=2, split_seed=SPLIT,
-              weight_seed=WSEED, plan="eager")
-    H, W, C, _ = v.base_shape()
+@pytest.mark.parametrize("plan", ["eager", "lazy"])
+def test_pre_materialized_base_layer_unstaged_plans(plan):
+    # App. B under the other logical plans: Eager (one pass base -> all of L) and "Lazy-5 with Pre-mat"
+    # (every layer recomputed from the stored base).  Same kernels on the same bf16
+    # base -> MM_k and the LR weights bit-identical to Staged from the pixels, host and device bases.
+    cnn, taps, n, d_s = 2, [0, 2, 4], 9, 16
+    tab = gen.make_tables(n, d_s)
+    ref = run_gpu(cnn, taps, tab, d_s, iters=2)
+    mm_ref = [ref.features(k)["mm"].view(torch.int16).cpu().clone() for k in range(len(taps))]
+    w_ref = [ref.train(k, d_s + ref.features(k)["d_l"])[0] for k in range(len(taps))]
+    H, W, C, _ = ref.base_shape()
+    base_d = torch.empty((n, H, W, C), dtype=torch.bfloat16, device="cuda")
+    ref.materialize(tab.images, base_d)
+    torch.cuda.synchronize()
+    base_h = base_d.view(torch.int16).cpu().numpy()
+    ref.close()
+    for base in (base_d, base_h):
+        v = Vista(cnn, layers=taps, n_str_rows=len(tab.str_keys), d_s=d_s, n_images_local=n, iters=2,
+                  split_seed=SPLIT, weight_seed=WSEED, plan=plan, micro_batch=4)
+        v.transfer_from_base(base, tab.img_keys, tab.X, tab.str_keys, tab.labels)
+        for k in range(len(taps)):
+            f = v.features(k)
+            assert torch.equal(mm_ref[k], f["mm"].view(torch.int16).cpu()), (plan, k)
+            np.testing.assert_array_equal(w_ref[k], v.train(k, d_s + f["d_l"])[0])
+        v.close()
+
+
+def test_structured_values_must_be_bf16_representable():
+    # include/vista.h: X values must be bf16-representable (MM_k holds them in bf16); a joined row
+    # with a value that is not fails loudly instead of being rounded silently
+    tab = gen.make_tables(8, 8)
+    X = tab.X.copy()
+    X[3, 5] = np.float32(1.0 + 2.0 ** -12)  # needs 13 significant bits
+    v = Vista(0, layers=[1], n_str_rows=len(tab.str_keys), d_s=8, n_images_local=8, iters=2, weight_seed=WSEED)
     with pytest.raises(VistaError) as e:
-        v.transfer_from_base(np.zeros((4, H, W, C), np.int16), tab.img_keys, tab.X, tab.str_keys, tab.labels)
-    assert e.value.status == 1
+        v.transfer(tab.images, tab.img_keys, X, tab.str_keys, tab.labels)
+    assert e.value.status == 1 and "bf16" in str(e.value)
+    v.transfer(tab.images, tab.img_keys, tab.X, tab.str_keys, tab.labels)  # the ctx stays usable
     v.close()
+
+
+def test_planner_prediction_bounds_measured_peak():
+    # planner accountability: the predicted peak (weights + pixels + arenas + F + MM + grow-only slots of
+    # the chosen micro-batches + join) bounds the measured pool high-water mark of a transfer from host
+    # pixels, unchunked and chunked under a forced budget
+    n = 600
+    tab = gen.make_tables(n, 8)
+    v = run_gpu(2, [0, 1, 2, 3, 4], tab, 8, iters=1)
+    full = v.plan_info()
+    v.close()
+    assert 0 < full["peak_bytes_meas"] <= full["peak_bytes_pred"], full
+    assert full["peak_bytes_pred"] - full["peak_bytes_meas"] <= 0.05 * full["peak_bytes_pred"] + (96 << 20), full
+    budget = full["peak_bytes_pred"] // 2
+    v = run_gpu(2, [0, 1, 2, 3, 4], tab, 8, iters=1, hbm_budget_bytes=budget)
+    info = v.plan_info()
+    v.close()
+    assert info["chunk_images"] < n
+    assert info["peak_bytes_pred"] <= budget
+    assert 0 < info["peak_bytes_meas"] <= info["peak_bytes_pred"], info

@@ -107,6 +107,27 @@ def torch_resnet50(imgs):
     return [t.numpy() for t in taps]
 
 
+def torch_vgg16(imgs):
+    # configuration D of [61] at 227 (reading R1): 13 conv3x3 pad 1 + bias + ReLU, 2x2/2 max pools after
+    # convs 2, 4, 7, 10, 13 (227 -> 113 -> 56 -> 28 -> 14 -> 7), NHWC flatten (reading R8) -> fc6 -> fc7 -> fc8
+    c = 1
+    x = pixels(imgs)
+    chans = [64, 64, 128, 128, 256, 256, 256, 512, 512, 512, 512, 512, 512]
+    pool_after = {1, 3, 6, 9, 12}
+    cin = 3
+    for lid, co in enumerate(chans):
+        x = Fn.relu(Fn.conv2d(x, conv_w(c, lid, co, 3, cin), bias(c, lid, co), padding=1))
+        if lid in pool_after:
+            x = Fn.max_pool2d(x, 2, 2)
+        cin = co
+    assert tuple(x.shape[1:]) == (512, 7, 7)
+    x = nhwc_flat(x)
+    fc6 = Fn.relu(Fn.linear(x, fc_w(c, 13, 4096, 25088), bias(c, 13, 4096)))
+    fc7 = Fn.relu(Fn.linear(fc6, fc_w(c, 14, 4096, 4096), bias(c, 14, 4096)))
+    fc8 = Fn.linear(fc7, fc_w(c, 15, 1000, 4096), bias(c, 15, 1000))
+    return [t.numpy() for t in (fc6, fc7, fc8)]
+
+
 @pytest.fixture(scope="module")
 def imgs():
     t = gen.make_tables(3, 8, seed=gen.DEFAULT_SEED)
@@ -131,6 +152,17 @@ def test_resnet50_vs_torch_library(imgs):
     ref = torch_resnet50(imgs[:1])
     for t in range(5):
         assert _close(F[t], ref[t]), t
+
+
+@pytest.mark.slow
+def test_vgg16_vs_torch_library(imgs):
+    # pins the oracle's VGG16 composition (ReLUs, biases, pool positions, the fc6 flatten order) against
+    # torch library routines on the same generated parameters, not only its MAC total and tap widths
+    F, _ = oracle.features(oracle.VGG16, SEED, imgs[:1], taps=[0, 1, 2])
+    ref = torch_vgg16(imgs[:1])
+    for t in range(3):
+        assert _close(F[t], ref[t]), t
+        assert np.abs(ref[t]).max() > 1e-3  # the activations did not collapse to zero
 
 
 def test_staged_eager_lazy_alexnet(imgs):

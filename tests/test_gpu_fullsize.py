@@ -52,10 +52,9 @@ def test_join_full_size_bit_exact(N):
     # permuting T_img permutes the image rows of the pairs and nothing else
     perm = np.random.default_rng(N).permutation(N)
     ps2, pi2, n2 = vista_join(ik[torch.from_numpy(perm).cuda()], sk, split_seed=SPLIT)
-    inv = np.argsort(perm)
     assert n2 == n_train
     np.testing.assert_array_equal(ps2.cpu().numpy(), ops)
-    np.testing.assert_array_equal(inv[pi2.cpu().numpy()], opi)
+    np.testing.assert_array_equal(perm[pi2.cpu().numpy()], opi)  # new image row j holds old row perm[j]
     # a duplicate image key anywhere is a primary-key violation
     ik[N // 2 + 1] = ik[N // 3]
     with pytest.raises(VistaError) as e:

@@ -7,11 +7,14 @@
 // ("minibatch"), computes z_p = b + sum_j w^_j (x_pj - mu_j) per row with a block
 // reduction, applies phi (identity for the power iteration, sigmoid residual for the
 // gradient) and accumulates sum_p phi_p (x_pj - mu_j) per column in registers.  Per-CTA
-// partials are reduced in a fixed order in fp64 (deterministic), then allreduced across
-// ranks (fp64 NCCL) and applied by a one-block update kernel in fp64.
+// partials are reduced in a fixed order in fp64 (deterministic).  One rank (world == 1): the
+// reduction and the fp64 update of the pass (mean / sigma, power step, ISTA step) run in the
+// pass kernel's own tail, behind grid-wide barriers of the cooperative launch -- one launch per
+// pass.  world > 1: partials -> reduce kernel -> fp64 allreduce (NCCL or the caller's hook) ->
+// one-block update kernel.
 #include <cmath>
-#include <mutex>
-#include <set>
+#include <cstdlib>
+#include <cstring>
 
 #include "internal.h"
 #include "ptx.cuh"
@@ -21,6 +24,30 @@ namespace vista {
 constexpr int kMaxRB = 16;     // rows per streamed block (upper bound)
 constexpr int kStagesLR = 3;   // row blocks in flight per CTA
 constexpr int kLRThreads = 576;  // 18 compute warps: 1041 chunks of a conv5_x row (ld 8328) = 2 per thread, no 3-chunk stragglers
+
+struct LRState {  // device, fp64 master copies
+  double n_train;   // global train rows
+  double lambda_hat, eta;
+  double b, vb;
+  double loss;
+};
+
+// world == 1: the pass kernel reduces its partials and applies the O6 update itself (see fused_tail)
+struct FusedArgs {
+  int on;                 // 0: partials only (reduce / allreduce / update kernels follow)
+  int ncols;              // ld + 2
+  unsigned int* bar;      // [2] grid barrier: arrival count, generation (zeroed once per lr_train)
+  double* G;              // [ncols] reduced sums
+  double* scal;           // [2 gridDim.x] per-CTA partial scalars (two reductions per pass at most)
+  const uint8_t* real;    // [ld] real (non-padding) columns
+  double *mu, *inv, *v, *w;
+  float *mu_f, *what, *bhat;
+  LRState* st;
+  double* loss_out;       // MODE 3: loss of this iteration
+  double lambda, alpha;
+  int d_real;
+  int init_next;          // MODE 1: initialise the power iteration; MODE 2: last power pass, initialise ISTA
+};
 
 struct PassArgs {
   const uint8_t* MM;   // row-major [rows][ld] elements of E (bf16, or fp32 in check mode)
@@ -34,7 +61,11 @@ struct PassArgs {
   const float* bhat;    // [1]
   float* partial;       // [gridDim.x][ld + 4] (16-byte aligned rows; ld + 2 used)
   unsigned long long* counts;  // eval: [5]
+  FusedArgs f;
 };
+
+template <int MODE>
+__device__ void fused_tail(const PassArgs& a, uint8_t* scratch, int nthr);
 
 __device__ __forceinline__ float softplusf(float z) { return z > 0.f ? z + log1pf(__expf(-z)) : log1pf(__expf(z)); }
 
@@ -111,6 +142,11 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_stream_kernel(const Pas
         const uint32_t bytes = (uint32_t)nr * row_bytes;
         mbar_arrive_expect_tx(&full[stage], bytes);
         bulk_load(base + stage * stage_bytes, a.MM + (size_t)r * row_bytes, bytes, &full[stage]);
+        const int64_t pb = blk + (int64_t)kStagesLR * gridDim.x;
+        if (pb < nblk) {
+          const int64_t pr = a.r0 + pb * a.rb;
+          prefetch_l2_range(a.MM + (size_t)pr * row_bytes, (uint32_t)min((int64_t)a.rb, a.r1 - pr) * row_bytes);
+        }
       }
     }
     return;
@@ -257,6 +293,425 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_stream_kernel(const Pas
       out[a.ld + 1] = sum_loss;
     }
   }
+  if (a.f.on) fused_tail<MODE>(a, gbase, nthr);
+}
+
+// ---- bf16 power / gradient / eval passes (MODE 2, 3, 4): the same schedule as lr_stream_kernel with
+// an instruction-lean inner loop (ncu on the r1 kernel: 62 % issue-slot busy, FFMA 20 % of the
+// instructions -- the pass was issue-bound, not HBM-bound):
+//  * RB rows per block as a compile-time constant (4 / 8 / 16 by row width); a partial last block
+//    computes garbage dot products for its missing rows and never uses them;
+//  * every thread owns exactly CH 16-byte chunks: a chunk past the row end reads chunk 0 with w = 0
+//    (no per-chunk branches), and its accumulator is never stored;
+//  * bf16 pairs unpacked with one PRMT each, dot and accumulate on packed fp32 FMAs (FFMA2);
+//  * the RB per-warp dot products reduced by a halving butterfly: RB - 1 + log2(32 / RB) shuffles
+//    instead of 5 RB.
+__device__ __forceinline__ float2 bf2_f2(uint32_t u) {  // exact: bf16 = the high half of an fp32
+  return make_float2(__uint_as_float(__byte_perm(u, 0u, 0x1044u)), __uint_as_float(__byte_perm(u, 0u, 0x3244u)));
+}
+__device__ __forceinline__ float2 ffma2(float2 a, float2 b, float2 c) {  // (a.x b.x + c.x, a.y b.y + c.y), RN
+  unsigned long long r;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;"
+      : "=l"(r)
+      : "l"(*reinterpret_cast<unsigned long long*>(&a)), "l"(*reinterpret_cast<unsigned long long*>(&b)),
+        "l"(*reinterpret_cast<unsigned long long*>(&c)));
+  return *reinterpret_cast<float2*>(&r);
+}
+
+// v[0..N) per lane -> after the call, lane l holds the warp sum of value (l >> (5 - log2 N)) in v[0]
+// (valid in every lane; representative lanes: l % (32 / N) == 0).  Fixed order: deterministic.
+template <int N>
+__device__ __forceinline__ void butterfly(float (&v)[16], int lane) {
+  int o = 16;
+#pragma unroll
+  for (int n = N; n > 1; n >>= 1, o >>= 1) {
+    const bool up = (lane & o) != 0;
+#pragma unroll
+    for (int i = 0; i < n / 2; ++i) {
+      const float send = up ? v[i] : v[i + n / 2];
+      const float keep = up ? v[i + n / 2] : v[i];
+      v[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+    }
+  }
+#pragma unroll
+  for (; o > 0; o >>= 1) v[0] += __shfl_xor_sync(0xffffffffu, v[0], o);
+}
+
+template <int RB, int CH, int MODE>
+__global__ void __launch_bounds__(kLRThreads + 32, 1) lr_dot_kernel(const PassArgs a) {
+  static_assert(RB == 4 || RB == 8 || RB == 16, "rows per block");
+  constexpr int LOGRB = RB == 4 ? 2 : (RB == 8 ? 3 : 4);
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  const uint32_t base = (raw + 127u) & ~127u;
+  uint8_t* gbase = smem_raw + (base - raw);
+  const uint32_t row_bytes = (uint32_t)a.ld * 2u;
+  const uint32_t stage_bytes = ((uint32_t)RB * row_bytes + 127u) & ~127u;
+  float* red_all = reinterpret_cast<float*>(gbase + kStagesLR * stage_bytes);  // [kStagesLR][kMaxRB][32]
+  uint64_t* full = reinterpret_cast<uint64_t*>(red_all + kStagesLR * kMaxRB * 32);
+  uint64_t* empty = full + kStagesLR;
+  const int nthr = (int)blockDim.x - 32;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwc = nthr >> 5;
+  const int64_t nrows = a.r1 - a.r0;
+  const int64_t nblk = (nrows + RB - 1) / RB;
+  if (tid == 0) {
+    for (int i = 0; i < kStagesLR; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&empty[i], nthr);
+    }
+    fence_mbar_init();
+  }
+  __syncthreads();
+  if (warp == nwc) {  // producer warp: bulk copies of RB-row blocks into the ring
+    if (lane == 0) {
+      int it = 0;
+      for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++it) {
+        const int stage = it % kStagesLR;
+        if (it >= kStagesLR) mbar_wait(&empty[stage], ((it / kStagesLR) - 1) & 1);
+        const int64_t r = a.r0 + blk * RB;
+        const uint32_t bytes = (uint32_t)min((int64_t)RB, a.r1 - r) * row_bytes;
+        mbar_arrive_expect_tx(&full[stage], bytes);
+        bulk_load(base + stage * stage_bytes, a.MM + (size_t)r * row_bytes, bytes, &full[stage]);
+        // the block one ring-length ahead goes to L2 now: more bytes in flight than the ring holds
+        const int64_t pb = blk + (int64_t)kStagesLR * gridDim.x;
+        if (pb < nblk) {
+          const int64_t pr = a.r0 + pb * RB;
+          prefetch_l2_range(a.MM + (size_t)pr * row_bytes, (uint32_t)min((int64_t)RB, a.r1 - pr) * row_bytes);
+        }
+      }
+    }
+    return;
+  }
+  uint32_t coff[CH];
+  float2 wv[CH][4], acc[CH][4];
+#pragma unroll
+  for (int c = 0; c < CH; ++c) {
+    const int ch = tid + c * nthr;
+    const bool act = ch < a.chunks;
+    coff[c] = act ? (uint32_t)ch * 16u : 0u;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      wv[c][j] = act ? make_float2(a.what[ch * 8 + 2 * j], a.what[ch * 8 + 2 * j + 1]) : make_float2(0.f, 0.f);
+      acc[c][j] = make_float2(0.f, 0.f);
+    }
+  }
+  const float bh = a.bhat[0];
+  float sum_r = 0.f, sum_loss = 0.f;
+  unsigned long long cnt[5] = {0, 0, 0, 0, 0};
+  int it = 0;
+  for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++it) {
+    const int stage = it % kStagesLR;
+    mbar_wait(&full[stage], (it / kStagesLR) & 1);
+    const int64_t r = a.r0 + blk * RB;
+    const int nr = (int)min((int64_t)RB, a.r1 - r);
+    const uint8_t* sb = gbase + stage * stage_bytes;
+    float* red = red_all + stage * (kMaxRB * 32);
+    float sd[16];
+#pragma unroll
+    for (int q = 0; q < RB; ++q) {
+      float2 s2 = make_float2(0.f, 0.f);
+#pragma unroll
+      for (int c = 0; c < CH; ++c) {
+        const uint4 v = *reinterpret_cast<const uint4*>(sb + q * row_bytes + coff[c]);
+        s2 = ffma2(bf2_f2(v.x), wv[c][0], s2);
+        s2 = ffma2(bf2_f2(v.y), wv[c][1], s2);
+        s2 = ffma2(bf2_f2(v.z), wv[c][2], s2);
+        s2 = ffma2(bf2_f2(v.w), wv[c][3], s2);
+      }
+      sd[q] = s2.x + s2.y;
+    }
+    butterfly<RB>(sd, lane);
+    if ((lane & ((32 >> LOGRB) - 1)) == 0) red[(lane >> (5 - LOGRB)) * 32 + warp] = sd[0];
+    named_bar_sync(1, nthr);
+    // every warp: lane q < nr forms z_q from the per-warp partials (fixed order) and phi_q
+    float phi = 0.f;
+    if (lane < nr) {
+      float z = bh;
+      const float* rq = red + lane * 32;
+      for (int w = 0; w < nwc; ++w) z += rq[w];
+      const int64_t row = r + lane;
+      if (MODE == 2) {
+        phi = z;
+        if (warp == 0) sum_r += z;
+      } else {
+        const int yv = a.y[row];
+        if (MODE == 3) {
+          phi = 1.f / (1.f + __expf(-z)) - (float)yv;
+          if (warp == 0) {
+            sum_r += phi;
+            sum_loss += softplusf(z) - (float)yv * z;
+          }
+        } else if (warp == 0) {  // MODE 4: predict 1 iff z >= 0
+          const int pred = z >= 0.f ? 1 : 0;
+          if (row < a.n_train) cnt[0] += pred == yv;
+          else cnt[pred && yv ? 1 : (pred ? 2 : (yv ? 4 : 3))] += 1;
+        }
+      }
+    }
+    if (MODE != 4) {
+#pragma unroll
+      for (int q = 0; q < RB; ++q) {
+        if (q < nr) {  // block-uniform
+          const float ph = __shfl_sync(0xffffffffu, phi, q);
+          const float2 p2 = make_float2(ph, ph);
+#pragma unroll
+          for (int c = 0; c < CH; ++c) {
+            const uint4 v = *reinterpret_cast<const uint4*>(sb + q * row_bytes + coff[c]);
+            acc[c][0] = ffma2(bf2_f2(v.x), p2, acc[c][0]);
+            acc[c][1] = ffma2(bf2_f2(v.y), p2, acc[c][1]);
+            acc[c][2] = ffma2(bf2_f2(v.z), p2, acc[c][2]);
+            acc[c][3] = ffma2(bf2_f2(v.w), p2, acc[c][3]);
+          }
+        }
+      }
+    }
+    mbar_arrive(&empty[stage]);
+  }
+  if constexpr (MODE == 4) {
+    if (warp == 0) {
+#pragma unroll
+      for (int k = 0; k < 5; ++k) {
+        unsigned long long v = cnt[k];
+        for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        if (lane == 0 && v) atomicAdd(&a.counts[k], v);
+      }
+    }
+    return;
+  } else {
+    float* out = a.partial + (size_t)blockIdx.x * (a.ld + 4);
+#pragma unroll
+    for (int c = 0; c < CH; ++c) {
+      const int ch = tid + c * nthr;
+      if (ch < a.chunks) {
+        float4* o = reinterpret_cast<float4*>(out + ch * 8);
+        o[0] = make_float4(acc[c][0].x, acc[c][0].y, acc[c][1].x, acc[c][1].y);
+        o[1] = make_float4(acc[c][2].x, acc[c][2].y, acc[c][3].x, acc[c][3].y);
+      }
+    }
+    if (warp == 0) {
+      for (int o = 16; o > 0; o >>= 1) {
+        sum_r += __shfl_xor_sync(0xffffffffu, sum_r, o);
+        sum_loss += __shfl_xor_sync(0xffffffffu, sum_loss, o);
+      }
+      if (lane == 0) {
+        out[a.ld] = sum_r;
+        out[a.ld + 1] = sum_loss;
+      }
+    }
+    if (a.f.on) fused_tail<MODE>(a, gbase, nthr);
+  }
+}
+
+// ---- fused reduce + update (world == 1) ----
+// Grid-wide barrier of the cooperative launch (all CTAs co-resident): compute threads only (the
+// producer warp has exited), named barrier 2 inside the CTA, one arrival per CTA on a global counter.
+__device__ __forceinline__ void grid_sync(unsigned int* bar, int nthr) {
+  named_bar_sync(2, nthr);
+  if (threadIdx.x == 0) {
+    volatile unsigned int* gen = bar + 1;
+    const unsigned int g = *gen;
+    __threadfence();
+    if (atomicAdd(bar, 1u) == gridDim.x - 1) {
+      atomicExch(bar, 0u);
+      __threadfence();
+      atomicAdd(bar + 1, 1u);
+    } else {
+      while (*gen == g) __nanosleep(64);
+    }
+    __threadfence();
+  }
+  named_bar_sync(2, nthr);
+}
+
+// out[i] = sum over the G CTAs' partial rows of column j0 + i, i < n, in fp64 and a fixed order (each
+// warp sums a contiguous CTA range per 32-column tile, then the warp sums in warp order).  Every CTA
+// calling it for the same column gets the same bits.  sh: >= nwc * 32 doubles of shared memory.
+__device__ void reduce_cols(const float* partial, int pitch, int G, int j0, int n, double* out, double* sh,
+                            int nthr) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwc = nthr >> 5;
+  const int c0 = (int)((int64_t)G * warp / nwc), c1 = (int)((int64_t)G * (warp + 1) / nwc);
+  for (int t = 0; t < n; t += 32) {
+    const int j = j0 + t + lane;
+    double s = 0.0;
+    if (t + lane < n) {
+      const float* pc = partial + j;
+      int c = c0;
+      for (; c + 8 <= c1; c += 8) {  // eight independent L2 loads in flight, added in order
+        float x[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) x[u] = __ldcg(pc + (size_t)(c + u) * pitch);
+#pragma unroll
+        for (int u = 0; u < 8; ++u) s += (double)x[u];
+      }
+      for (; c < c1; ++c) s += (double)__ldcg(pc + (size_t)c * pitch);
+    }
+    sh[warp * 32 + lane] = s;
+    named_bar_sync(2, nthr);
+    if (warp == 0 && t + lane < n) {
+      double g = 0.0;
+      for (int w = 0; w < nwc; ++w) g += sh[w * 32 + lane];
+      out[t + lane] = g;
+    }
+    named_bar_sync(2, nthr);
+  }
+}
+
+// fixed-order sum of one double per compute thread (result in every thread)
+__device__ double cta_sum(double v, double* sh, int nthr) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwc = nthr >> 5;
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  if (lane == 0) sh[warp] = v;
+  named_bar_sync(2, nthr);
+  double t = 0.0;
+  for (int w = 0; w < nwc; ++w) t += sh[w];
+  named_bar_sync(2, nthr);
+  return t;
+}
+
+// fixed-order sum of the G per-CTA scalars (result in every thread of every CTA, same bits)
+__device__ double grid_scalar_sum(const double* scal, double* sh, int nthr) {
+  if ((threadIdx.x >> 5) == 0) {
+    const int lane = threadIdx.x & 31;
+    double s = 0.0;
+    for (int c = lane; c < (int)gridDim.x; c += 32) s += __ldcg(scal + c);
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (lane == 0) sh[0] = s;
+  }
+  named_bar_sync(2, nthr);
+  const double t = sh[0];
+  named_bar_sync(2, nthr);
+  return t;
+}
+
+// The O6 update of one pass, distributed over the CTAs of the pass: CTA b owns columns
+// [b ncols / G, (b + 1) ncols / G) of the reduction and [b ld / G, (b + 1) ld / G) of the update.
+//   MODE 0: mu = G / n                    MODE 1: inv = 1 / sigma (+ power-iteration start)
+//   MODE 2: power step (lambda, v, w^)    MODE 3: ISTA step (w, b, loss)
+// Same arithmetic as stats_finalize_kernel / power_kernel / grad_kernel (world > 1 path).
+template <int MODE>
+__device__ void fused_tail(const PassArgs& a, uint8_t* scratch, int nthr) {
+  const FusedArgs& f = a.f;
+  const int G = gridDim.x, b = blockIdx.x, ld = a.ld, pitch = ld + 4;
+  double* sh = reinterpret_cast<double*>(scratch);  // [nwc * 32]
+  double* gs = sh + 32 * 32;                        // this CTA's reduced columns
+  double* g2 = gs + ((ld + G - 1) / G + 2);         // G[ld], G[ld + 1]
+  __threadfence();
+  grid_sync(f.bar, nthr);  // every CTA's partial row is written
+  const int u0 = (int)((int64_t)ld * b / G), u1 = (int)((int64_t)ld * (b + 1) / G);
+  reduce_cols(a.partial, pitch, G, u0, u1 - u0, gs, sh, nthr);
+  reduce_cols(a.partial, pitch, G, ld, 2, g2, sh, nthr);  // redundantly in every CTA: identical bits
+  const double phisum = g2[0];
+  LRState* st = f.st;
+  if (MODE == 0) {
+    const double n = (double)a.n_train;
+    for (int j = u0 + threadIdx.x; j < u1; j += nthr) {
+      const double m = gs[j - u0] / n;
+      f.mu[j] = m;
+      f.mu_f[j] = (float)m;
+    }
+    if (b == 0 && threadIdx.x == 0) st->n_train = n;
+    return;
+  }
+  const double n = st->n_train, rn = 1.0 / n;
+  if (MODE == 1) {
+    const double vb = 1.0 / sqrt((double)(f.d_real + 1));
+    double sm = 0.0;
+    for (int j = u0 + threadIdx.x; j < u1; j += nthr) {
+      const double sigma = sqrt(gs[j - u0] / n);
+      const double iv = (f.real[j] && sigma > 1e-12) ? 1.0 / sigma : 0.0;
+      f.inv[j] = iv;
+      // power-iteration start (O6 step 3): v = 1 / sqrt(d + 1) on real columns and the bias
+      const double vj = f.real[j] ? vb : 0.0;
+      f.v[j] = vj;
+      const double wj = iv * vj;
+      f.what[j] = (float)wj;
+      sm += wj * f.mu[j];
+    }
+    sm = cta_sum(sm, sh, nthr);
+    if (threadIdx.x == 0) f.scal[b] = sm;
+    __threadfence();
+    grid_sync(f.bar, nthr);
+    const double tot = grid_scalar_sum(f.scal, sh, nthr);
+    if (b == 0 && threadIdx.x == 0) {
+      st->vb = vb;
+      f.bhat[0] = (float)(vb - tot);
+    }
+    return;
+  }
+  if (MODE == 2) {
+    // centre: G_j <- G_j - mu_j sum_p phi_p; q_j = inv_j G_j / n; lambda = ||(q, q_b)||.  With v = q / lambda:
+    // w^_j = inv_j v_j and b' = v_b - sum_j w^_j mu_j = (q_b - sum_j inv_j q_j mu_j) / lambda, so one grid
+    // reduction of (sum q_j^2, sum inv_j q_j mu_j) serves both
+    double ss = 0.0, sq = 0.0;
+    for (int j = u0 + threadIdx.x; j < u1; j += nthr) {
+      const double g = gs[j - u0] - f.mu[j] * phisum;
+      gs[j - u0] = g;
+      const double q = f.inv[j] * g * rn;
+      ss += q * q;
+      sq += f.inv[j] * q * f.mu[j];
+    }
+    ss = cta_sum(ss, sh, nthr);
+    sq = cta_sum(sq, sh, nthr);
+    if (threadIdx.x == 0) {
+      f.scal[b] = ss;
+      f.scal[G + b] = sq;
+    }
+    __threadfence();
+    grid_sync(f.bar, nthr);
+    const double qb = phisum * rn;
+    const double lam = sqrt(grid_scalar_sum(f.scal, sh, nthr) + qb * qb);
+    const double sqt = grid_scalar_sum(f.scal + G, sh, nthr);
+    const double rl = lam > 0 ? 1.0 / lam : 0.0;
+    if (f.init_next) {
+      // last power pass: lambda_hat is final; start ISTA (O6 step 4): eta = 1 / L, w = 0, b = 0
+      for (int j = u0 + threadIdx.x; j < u1; j += nthr) {
+        f.w[j] = 0.0;
+        f.what[j] = 0.f;
+      }
+      if (b == 0 && threadIdx.x == 0) {
+        st->lambda_hat = lam;
+        st->eta = 1.0 / (0.25 * 1.05 * lam + f.lambda * (1.0 - f.alpha));
+        st->b = 0.0;
+        f.bhat[0] = 0.f;
+      }
+      return;
+    }
+    const double scale = rn * rl;
+    for (int j = u0 + threadIdx.x; j < u1; j += nthr) {
+      const double vj = scale * f.inv[j] * gs[j - u0];
+      f.v[j] = vj;
+      f.what[j] = (float)(f.inv[j] * vj);
+    }
+    if (b == 0 && threadIdx.x == 0) {
+      st->lambda_hat = lam;
+      st->vb = qb * rl;
+      f.bhat[0] = (float)((qb - sqt) * rl);
+    }
+    return;
+  }
+  // MODE 3: ISTA step (O6 step 5) at the pre-update w: loss, g, soft threshold; bias unregularised
+  const double eta = st->eta, thr = eta * f.lambda * f.alpha, l2 = f.lambda * (1.0 - f.alpha);
+  const double bnew = st->b - eta * phisum * rn;
+  double sm = 0.0;
+  for (int j = u0 + threadIdx.x; j < u1; j += nthr) {
+    const double g = f.inv[j] * (gs[j - u0] - f.mu[j] * phisum) * rn + l2 * f.w[j];
+    const double vv = f.w[j] - eta * g;
+    const double wj = (vv > 0 ? 1.0 : (vv < 0 ? -1.0 : 0.0)) * fmax(fabs(vv) - thr, 0.0);
+    f.w[j] = wj;
+    const double hj = f.inv[j] * wj;
+    f.what[j] = (float)hj;
+    sm += hj * f.mu[j];
+  }
+  sm = cta_sum(sm, sh, nthr);
+  if (threadIdx.x == 0) f.scal[b] = sm;
+  __threadfence();
+  grid_sync(f.bar, nthr);  // every CTA has read st->b / st->eta
+  const double tot = grid_scalar_sum(f.scal, sh, nthr);
+  if (b == 0 && threadIdx.x == 0) {
+    st->b = bnew;
+    *f.loss_out = g2[1] * rn;
+    f.bhat[0] = (float)(bnew - tot);
+  }
 }
 
 // G[j] = sum_cta partial[cta][j] in fp64, fixed order (8 contiguous CTA ranges, one per warp, then
@@ -288,13 +743,6 @@ __global__ void __launch_bounds__(256) reduce_partials_kernel(const float* __res
     G[j] = g;
   }
 }
-
-struct LRState {  // device, fp64 master copies
-  double n_train;   // global train rows
-  double lambda_hat, eta;
-  double b, vb;
-  double loss;
-};
 
 __device__ double block_sum(double v, double* sh) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -426,24 +874,51 @@ __global__ void __launch_bounds__(1024) grad_kernel(const double* G, int ld, int
 struct StreamCfg {
   int threads, ch, rb, grid;
   size_t smem;
+  int dot_rb = 0;       // bf16 power / gradient / eval passes on lr_dot_kernel<dot_rb, ch, MODE> (0: not used)
+  size_t dot_smem = 0;
 };
+
+static void launch_pass(const void* kern, const PassArgs& a, int grid, int threads, size_t smem, bool coop,
+                        cudaStream_t st) {
+  ensure_smem_attr(kern, 227 * 1024);
+  static const bool coop_ok = !(getenv("VISTA_LR_COOP") && getenv("VISTA_LR_COOP")[0] == '0');  // A/B only
+  if (coop && coop_ok) {  // the fused tail's grid barriers need every CTA resident: cooperative launch guarantees it
+    void* args[] = {const_cast<PassArgs*>(&a)};
+    VCHECK(cudaLaunchCooperativeKernel(kern, dim3(grid), dim3(threads), args, smem, st));
+  } else {
+    void* args[] = {const_cast<PassArgs*>(&a)};
+    VCHECK(cudaLaunchKernel(kern, dim3(grid), dim3(threads), args, smem, st));
+  }
+  LAUNCHED();
+}
 
 template <int MODE, typename E>
 static void run_pass(const PassArgs& a, const StreamCfg& c, cudaStream_t st) {
-  auto go = [&](void (*kern)(PassArgs)) {
-    ensure_smem_attr((const void*)kern, 227 * 1024);
-    kern<<<c.grid, c.threads + 32, c.smem, st>>>(a);
-  };
+  const bool coop = a.f.on != 0;
+  if constexpr (MODE >= 2 && sizeof(E) == 2) {
+    if (c.dot_rb > 0) {
+    const void* k = nullptr;
+#define VISTA_DOT(RB, CH) \
+  if (c.dot_rb == RB && c.ch == CH) k = (const void*)lr_dot_kernel<RB, CH, MODE>;
+    VISTA_DOT(4, 1) VISTA_DOT(4, 2) VISTA_DOT(4, 3) VISTA_DOT(8, 1) VISTA_DOT(8, 2) VISTA_DOT(8, 3)
+    VISTA_DOT(16, 1) VISTA_DOT(16, 2) VISTA_DOT(16, 3)
+#undef VISTA_DOT
+    if (!k) fail(1, "lr: no pass kernel for this row width");
+    launch_pass(k, a, c.grid, c.threads + 32, c.dot_smem, coop, st);
+    return;
+    }
+  }
+  const void* k = nullptr;
   switch (c.ch) {
-    case 1: go(lr_stream_kernel<1, MODE, E>); break;
-    case 2: go(lr_stream_kernel<2, MODE, E>); break;
-    case 3: go(lr_stream_kernel<3, MODE, E>); break;
-    case 4: go(lr_stream_kernel<4, MODE, E>); break;
-    case 5: go(lr_stream_kernel<5, MODE, E>); break;
-    case 6: go(lr_stream_kernel<6, MODE, E>); break;
+    case 1: k = (const void*)lr_stream_kernel<1, MODE, E>; break;
+    case 2: k = (const void*)lr_stream_kernel<2, MODE, E>; break;
+    case 3: k = (const void*)lr_stream_kernel<3, MODE, E>; break;
+    case 4: k = (const void*)lr_stream_kernel<4, MODE, E>; break;
+    case 5: k = (const void*)lr_stream_kernel<5, MODE, E>; break;
+    case 6: k = (const void*)lr_stream_kernel<6, MODE, E>; break;
     default: fail(1, "lr: unsupported row width");
   }
-  LAUNCHED();
+  launch_pass(k, a, c.grid, c.threads + 32, c.smem, coop, st);
 }
 
 template <typename E>
@@ -462,10 +937,23 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   if (cfg.ch == 3 && chunks <= 2 * cfg.threads) cfg.ch = 2;
   cfg.rb = (int)std::max<int64_t>(1, std::min<int64_t>(kMaxRB, (200 * 1024 / kStagesLR) / ((int64_t)ld * esz)));
   const size_t stage_bytes = ((size_t)cfg.rb * ld * esz + 127) & ~(size_t)127;
-  cfg.smem = kStagesLR * stage_bytes + kStagesLR * kMaxRB * 32 * 4 + 2 * kStagesLR * 8 + 128;
+  const size_t tail_smem = kStagesLR * kMaxRB * 32 * 4 + 2 * kStagesLR * 8 + 128;  // red + barriers + align
+  cfg.smem = kStagesLR * stage_bytes + tail_smem;
   if (cfg.smem > 227 * 1024) fail(1, "lr: row block does not fit in shared memory");
+  const char* dot_env = getenv("VISTA_LR_DOT");  // A/B switch: 0 = the r1 kernel for every pass
+  if (esz == 2 && cfg.ch <= 3 && !(dot_env && dot_env[0] == '0')) {  // bf16: the lean dot kernel, 4 / 8 / 16 rows per block
+    for (int rb : {16, 8, 4}) {
+      const size_t sb = ((size_t)rb * ld * 2 + 127) & ~(size_t)127;
+      if (kStagesLR * sb + tail_smem <= 227 * 1024) {
+        cfg.dot_rb = rb;
+        cfg.dot_smem = kStagesLR * sb + tail_smem;
+        break;
+      }
+    }
+  }
+  const int64_t pass_rb = cfg.dot_rb > 0 ? std::min(cfg.rb, cfg.dot_rb) : cfg.rb;  // grid: blocks of the finer kernel
   auto grid_for_rows = [&](int64_t rows) {
-    const int64_t blocks = (rows + cfg.rb - 1) / cfg.rb;
+    const int64_t blocks = (rows + pass_rb - 1) / pass_rb;
     return (int)std::max<int64_t>(1, std::min<int64_t>(blocks, num_sms()));
   };
   cfg.grid = grid_for_rows(n_train);
@@ -473,6 +961,14 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   const int ncols = ld + 2;
   int d_real = 0;
   for (int j = 0; j < ld; ++j) d_real += real_host[j] ? 1 : 0;
+  // world == 1: reduction + update in the pass kernels' tails (one launch per pass).  The tail keeps this
+  // CTA's reduced columns and a [32][32] double scratch in the (drained) stage ring.
+  const size_t ring_min = kStagesLR * std::min(stage_bytes, cfg.dot_rb > 0
+                                                                ? (((size_t)cfg.dot_rb * ld * 2 + 127) & ~(size_t)127)
+                                                                : stage_bytes);
+  const size_t tail_need = 32 * 32 * 8 + ((size_t)(ld + grid_tr - 1) / grid_tr + 4) * 8;
+  const bool fused = !allreduce && power_iters >= 1 && n_train > 0 && tail_need <= ring_min &&
+                     !(getenv("VISTA_LR_FUSED") && getenv("VISTA_LR_FUSED")[0] == '0');
 
   // scratch
   size_t off = 0;
@@ -480,7 +976,8 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   const size_t o_part = carve((size_t)std::max(grid_tr, 1) * (ld + 4) * 4), o_G = carve(ncols * 8), o_mu = carve(ld * 8),
                o_muf = carve(ld * 4), o_inv = carve(ld * 8), o_v = carve(ld * 8), o_w = carve(ld * 8),
                o_what = carve(ld * 4), o_bhat = carve(16), o_st = carve(sizeof(LRState)),
-               o_real = carve(ld), o_loss = carve((size_t)(iters + 1) * 8), o_cnt = carve(64);
+               o_real = carve(ld), o_loss = carve((size_t)(iters + 1) * 8), o_cnt = carve(64),
+               o_bar = carve(16), o_scal = carve((size_t)2 * std::max(grid_tr, 1) * 8);
   uint8_t* scr = nullptr;
   VCHECK(cudaMallocAsync(&scr, off, st));
   float* partial = reinterpret_cast<float*>(scr + o_part);
@@ -498,8 +995,10 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   unsigned long long* cnt = reinterpret_cast<unsigned long long*>(scr + o_cnt);
   VCHECK(cudaMemcpyAsync(real, real_host, ld, cudaMemcpyHostToDevice, st));
   VCHECK(cudaMemsetAsync(cnt, 0, 64, st));
+  VCHECK(cudaMemsetAsync(scr + o_bar, 0, 16, st));
 
   PassArgs a;
+  std::memset(&a, 0, sizeof(a));
   a.MM = reinterpret_cast<const uint8_t*>(MM);
   a.y = y;
   a.r0 = 0;
@@ -513,6 +1012,23 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   a.n_train = n_train;
   a.rb = cfg.rb;
   a.counts = nullptr;
+  a.f.on = fused ? 1 : 0;
+  a.f.ncols = ncols;
+  a.f.bar = reinterpret_cast<unsigned int*>(scr + o_bar);
+  a.f.G = G;
+  a.f.scal = reinterpret_cast<double*>(scr + o_scal);
+  a.f.real = real;
+  a.f.mu = mu;
+  a.f.inv = inv;
+  a.f.v = v;
+  a.f.w = w;
+  a.f.mu_f = mu_f;
+  a.f.what = what;
+  a.f.bhat = bhat;
+  a.f.st = dst;
+  a.f.lambda = lambda;
+  a.f.alpha = alpha;
+  a.f.d_real = d_real;
   const double pass_bytes = (double)n_train * ld * esz;
   auto reduce = [&](double extra_n, int center) {
     prof_begin(st);
@@ -529,36 +1045,49 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   prof_begin(st);
   run_pass<0, E>(a, cfg, st);
   prof_end(st, 5, 0, pass_bytes);
-  reduce((double)n_train, 0);
-  stats_finalize_kernel<<<(ld + 255) / 256, 256, 0, st>>>(G, ld, 0, real, mu, mu_f, inv, dst);
-  LAUNCHED();
+  if (!fused) {
+    reduce((double)n_train, 0);
+    stats_finalize_kernel<<<(ld + 255) / 256, 256, 0, st>>>(G, ld, 0, real, mu, mu_f, inv, dst);
+    LAUNCHED();
+  }
   prof_begin(st);
-  run_pass<1, E>(a, cfg, st);
+  run_pass<1, E>(a, cfg, st);  // fused: + the power-iteration start
   prof_end(st, 5, 0, pass_bytes);
-  reduce(-1, 0);
-  stats_finalize_kernel<<<(ld + 255) / 256, 256, 0, st>>>(G, ld, 1, real, mu, mu_f, inv, dst);
-  LAUNCHED();
-  // ---- O6 step 3: K power iterations ----
-  power_kernel<<<1, ublk, 0, st>>>(G, ld, 1, d_real, real, inv, mu, v, what, bhat, dst);
-  LAUNCHED();
+  if (!fused) {
+    reduce(-1, 0);
+    stats_finalize_kernel<<<(ld + 255) / 256, 256, 0, st>>>(G, ld, 1, real, mu, mu_f, inv, dst);
+    LAUNCHED();
+    // ---- O6 step 3: K power iterations ----
+    power_kernel<<<1, ublk, 0, st>>>(G, ld, 1, d_real, real, inv, mu, v, what, bhat, dst);
+    LAUNCHED();
+  }
   for (int k = 0; k < power_iters; ++k) {
+    a.f.init_next = k == power_iters - 1 ? 1 : 0;  // fused: the last power pass also starts ISTA
     prof_begin(st);
     run_pass<2, E>(a, cfg, st);
     prof_end(st, 5, 0, pass_bytes);
-    reduce(-1, 1);
-    power_kernel<<<1, ublk, 0, st>>>(G, ld, 0, d_real, real, inv, mu, v, what, bhat, dst);
+    if (!fused) {
+      reduce(-1, 1);
+      power_kernel<<<1, ublk, 0, st>>>(G, ld, 0, d_real, real, inv, mu, v, what, bhat, dst);
+      LAUNCHED();
+    }
+  }
+  a.f.init_next = 0;
+  // ---- O6 steps 4-5: ISTA ----
+  if (!fused) {
+    grad_kernel<<<1, ublk, 0, st>>>(G, ld, 1, lambda, alpha, inv, mu, w, what, bhat, dst, loss);
     LAUNCHED();
   }
-  // ---- O6 steps 4-5: ISTA ----
-  grad_kernel<<<1, ublk, 0, st>>>(G, ld, 1, lambda, alpha, inv, mu, w, what, bhat, dst, loss);
-  LAUNCHED();
   for (int t = 0; t < iters; ++t) {
+    a.f.loss_out = loss + t;
     prof_begin(st);
     run_pass<3, E>(a, cfg, st);
     prof_end(st, 5, 0, pass_bytes);
-    reduce(-1, 1);
-    grad_kernel<<<1, ublk, 0, st>>>(G, ld, 0, lambda, alpha, inv, mu, w, what, bhat, dst, loss + t);
-    LAUNCHED();
+    if (!fused) {
+      reduce(-1, 1);
+      grad_kernel<<<1, ublk, 0, st>>>(G, ld, 0, lambda, alpha, inv, mu, w, what, bhat, dst, loss + t);
+      LAUNCHED();
+    }
   }
   // ---- O6 step 6: eval over all local rows ----
   {
@@ -566,6 +1095,7 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
     e.r0 = 0;
     e.r1 = n_rows;
     e.counts = cnt;
+    e.f.on = 0;
     StreamCfg ce = cfg;
     ce.grid = grid_for_rows(n_rows);
     prof_begin(st);

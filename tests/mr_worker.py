@@ -20,6 +20,7 @@ sys.path.insert(0, ROOT)
 
 def main():
     out, N, n0, mlp = sys.argv[1], int(sys.argv[2]), int(sys.argv[3]), int(sys.argv[4])
+    tag = sys.argv[5] if len(sys.argv) > 5 else ""
     rank, world = int(os.environ["RANK"]), int(os.environ["WORLD_SIZE"])
     import torch
     import torch.distributed as dist
@@ -57,7 +58,7 @@ def main():
             res["mlp_loss"] = np.array(mm["loss"][:3])
             res["mlp_met"] = np.array([mm["n_train"], mm["n_test"], mm["tp"], mm["fp"], mm["tn"], mm["fn"]], np.float64)
     v.close()
-    np.savez(os.path.join(out, f"rank{rank}.npz"), **res)
+    np.savez(os.path.join(out, f"rank{rank}{tag}.npz"), **res)
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()

@@ -11,8 +11,11 @@ rank's image shard -> vista_train(k) / vista_train_mlp(k).  Compared with world 
   sums cover a different row subset than world 1's CTAs do, so the fp64 totals differ
   at fp32 rounding level (~1e-7);
 * a rank with NO images (hence no train rows) takes part in every collective with zero partials: the
-  totals are then world 1's sums + 0.0, so the weights are bit-identical to world 1 on rank 0's rows,
-  for the LR and for the MLP (this is the rank that used to leave the MLP deadlocked).
+  totals are then world 1's sums + 0.0, so the weights are bit-identical to world 1 on rank 0's rows
+  run through the same (unfused: partials -> reduce -> allreduce -> update) LR kernels, for the LR and
+  for the MLP (this is the rank that used to leave the MLP deadlocked);
+* world 1's default LR (reduce + update fused into the pass kernels, cooperative grid barriers) agrees
+  with that unfused sequence to 1e-12 relative (only the order of the fp64 update sums differs).
 """
 import os
 import socket
@@ -36,8 +39,8 @@ def _port():
     return p
 
 
-def _run(out, world, N, n0, mlp):
-    env = dict(os.environ, MASTER_ADDR="127.0.0.1", MASTER_PORT=str(_port()), WORLD_SIZE=str(world))
+def _run(out, world, N, n0, mlp, **extra_env):
+    env = dict(os.environ, MASTER_ADDR="127.0.0.1", MASTER_PORT=str(_port()), WORLD_SIZE=str(world), **extra_env)
     procs = []
     for r in range(world):
         e = dict(env, RANK=str(r), LOCAL_RANK=str(r))
@@ -98,7 +101,9 @@ def test_world2_with_an_empty_rank(tmp_path):
     # rank 1 owns no images: zero train rows, zero pairs; every collective still completes and adds 0.0,
     # so the model equals world 1 on rank 0's images bit for bit (LR and MLP)
     (tmp_path / "ref").mkdir()
-    ref = _run(tmp_path / "ref", 1, 150, 150, 1)[0]
+    (tmp_path / "fused").mkdir()
+    ref = _run(tmp_path / "ref", 1, 150, 150, 1, VISTA_LR_FUSED="0")[0]
+    fused = _run(tmp_path / "fused", 1, 150, 150, 1)[0]
     res = _run(tmp_path, 2, 150, 150, 1)
     assert int(res[1]["n_train0"][0]) == 0 and len(res[1]["pair_str0"]) == 0
     for k in range(3):
@@ -109,3 +114,7 @@ def test_world2_with_an_empty_rank(tmp_path):
     for name in ("mlp_W1", "mlp_W2", "mlp_w3", "mlp_loss", "mlp_met"):
         np.testing.assert_array_equal(res[0][name], ref[name])
         np.testing.assert_array_equal(res[1][name], ref[name])
+    for k in range(3):  # fused world-1 LR vs the unfused kernels
+        assert _rel(fused[f"w{k}"], ref[f"w{k}"]) <= 1e-12
+        np.testing.assert_allclose(fused[f"loss{k}"], ref[f"loss{k}"], rtol=1e-12)
+        np.testing.assert_array_equal(fused[f"met{k}"][1:], ref[f"met{k}"][1:])

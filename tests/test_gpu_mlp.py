@@ -2,26 +2,32 @@
 vista_train_mlp against the fp64 oracle (oracle/mlp.py) on identical inputs: the GPU's own MM_k
 rows (bf16, upcast) and the same seeded bf16 initial weights.
 
-Tolerances (R30).  The GPU rounds H1, H2, dH2, dH2 W2 and the weight operands to bf16
-(2^-9 relative) around fp32-accumulated tcgen05 GEMMs.  The MLP's full-batch gradient at init is a
-small residual of large per-row terms, so those roundings move the weight UPDATE W_T - W_0 by several
-percent (reproduced in numpy by oracle.mlp.train_bf16_emulated).  Two comparisons:
-  kernels    vs the bf16-emulated algorithm: loss curve <= 1e-3 relative, updates <= 5e-2 normwise
-  precision  vs the fp64 definition:         loss curve <= 3e-2 relative, updates <= 0.15 normwise,
-             test accuracy within max(0.5 points, 3 test rows) (vs the emulation: one row)
+Pass/fail is against the fp64 DEFINITION (oracle.mlp.train), with tolerances derived a priori from
+the oracle's own quantities by the bf16 error budget of tests/mlp_budget.py (R30): the B200
+path stores activations, back-propagated activations and weight operands in bf16, and the budget
+predicts, per parameter group, how far that storage can move the weight update (4 standard deviations
+of a first-order probabilistic rounding model that includes ReLU-mask flips), the loss curve, and how
+many test predictions can flip.  The budget itself is checked against real bf16 rounding on the CPU
+(tests/test_oracle_mlp.py::test_bf16_budget_covers_bf16_rounding).
+
+Implementation check (separate, diagnostic of kernel bugs vs precision): the bf16-emulated algorithm
+(oracle.mlp.train_bf16_emulated, the same rounding points) must agree to fp32-vs-fp64 accumulation.
 """
 import numpy as np
 import pytest
 import torch
 
 import gen
+import mlp_budget
 from oracle import mlp
 from paper_conf_sigmod_nakandalak20_b200 import Vista, VistaError
 
 pytestmark = pytest.mark.gpu
 WSEED, SPLIT, MSEED = 11, 5, 21
-TOL_LOSS_EMU, TOL_UPD_EMU = 1e-3, 5e-2   # measured on B200: <= 1.7e-4 and <= 2.3e-2
-TOL_LOSS_DEF, TOL_UPD_DEF = 3e-2, 0.15    # measured on B200: <= 1.4e-2 and <= 8.5e-2
+# implementation check vs the emulation (same rounding points; fp32 vs fp64 accumulation and the order
+# of the fp32 GEMM sums differ): 2^-9-level relative on the loss, a few % on the update (which is a
+# small residual of large per-row terms: see mlp_budget)
+TOL_LOSS_EMU, TOL_UPD_EMU = 1e-3, 5e-2
 
 
 def gpu_rows(v, k):
@@ -61,17 +67,19 @@ def test_mlp_vs_oracle_identical_inputs(cnn, taps, k, n, d_s, iters):
     print("mlp parity", cnn, k, "vs bf16-emulation", e_emu, l_emu, "vs fp64", e_def, l_def,
           met["test_acc"], emet["test_acc"], rmet["test_acc"])
     assert met["n_train"] == rmet["n_train"] and met["n_test"] == rmet["n_test"]
-    # kernels: the GPU equals the bf16-emulated algorithm up to fp32-vs-fp64 accumulation
+    # parity vs the fp64 definition, within the a-priori bf16 budget
+    B = mlp_budget.budget(X, y, te, seed=MSEED, iters=iters, lr=0.01)
+    print("budget", B["upd"], B["loss"], B["flips"])
+    for name, e in e_def.items():
+        assert e <= B["upd"][name], (name, e, B["upd"][name])
+    assert np.all(np.abs(np.array(met["loss"][:iters]) - losses) <= B["loss"]), (met["loss"][:iters], losses, B["loss"])
+    n_te = max(rmet["n_test"], 1)
+    assert abs(met["test_acc"] - rmet["test_acc"]) <= 100.0 * B["flips"] / n_te + 1e-9
+    # implementation check vs the bf16-emulated algorithm
     assert l_emu <= TOL_LOSS_EMU, l_emu
     for name, e in e_emu.items():
         assert e <= TOL_UPD_EMU, (name, e)
-    # precision: the fp64 definition, within the measured bf16 drift
-    assert l_def <= TOL_LOSS_DEF, l_def
-    for name, e in e_def.items():
-        assert e <= TOL_UPD_DEF, (name, e)
-    one_row = 100.0 / max(rmet["n_test"], 1)
-    assert abs(met["test_acc"] - emet["test_acc"]) <= max(0.5, one_row) + 1e-9
-    assert abs(met["test_acc"] - rmet["test_acc"]) <= max(0.5, 3 * one_row) + 1e-9
+    assert abs(met["test_acc"] - emet["test_acc"]) <= max(0.5, 100.0 / n_te) + 1e-9
 
 
 def test_mlp_before_transfer_is_a_state_error():

@@ -11,6 +11,7 @@ import pytest
 import torch
 
 import gen
+import oracle
 from oracle import mlp
 
 rng = np.random.default_rng(7)
@@ -171,3 +172,27 @@ def test_bf16_emulation_is_the_definition_up_to_rounding():
     for k in ("W1", "W2", "w3", "b1", "b2"):
         np.testing.assert_allclose(E[k], R[k], rtol=1e-9, atol=1e-12)
     assert me["test_acc"] == m["test_acc"] and me["train_acc"] == m["train_acc"]
+
+
+def test_bf16_budget_covers_bf16_rounding():
+    # The a-priori bf16 error budget (tests/mlp_budget.py) that the GPU MLP parity test uses as its tolerance
+    # must cover what real bf16 rounding at the product's storage points does: the bf16-emulated algorithm's
+    # deviation from the fp64 definition, on real CNN features (AlexNet conv5 / fc6 taps of the oracle).
+    import mlp_budget
+    from oracle import mlp as M
+    tab = gen.make_tables(100, 8)
+    F, _ = oracle.features(oracle.ALEXNET, 11, tab.images, taps=[0, 1])
+    ps, pi, te = oracle.join(tab.img_keys, tab.str_keys, 5)
+    y = tab.labels[ps]
+    for t in (0, 1):
+        X = oracle.concat(tab.X, F[t], ps, pi)
+        B = mlp_budget.budget(X, y, te, seed=21, iters=4, lr=0.01)
+        R, lr_, rm = M.train(X, y, te, seed=21, iters=4, lr=0.01)
+        E, el, em = M.train_bf16_emulated(X, y, te, seed=21, iters=4, lr=0.01)
+        P0 = M.init_params(21, X.shape[1])
+        for k in mlp_budget.GROUPS:
+            err = np.linalg.norm(E[k] - R[k]) / np.linalg.norm(R[k] - P0[k])
+            assert err <= B["upd"][k], (t, k, err, B["upd"][k])
+            assert B["upd"][k] < 0.5  # the budget still constrains the update
+        assert np.all(np.abs(el - lr_) <= B["loss"])
+        assert abs(em["test_acc"] - rm["test_acc"]) <= 100.0 * B["flips"] / rm["n_test"] + 1e-9

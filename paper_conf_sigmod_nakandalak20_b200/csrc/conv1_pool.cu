@@ -223,44 +223,17 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int wo = q * 32 + lane;              // conv output column (M row of the tile)
     const int i0 = et, i1 = et + kEpiThreads;  // this thread's pooling items
     uint32_t it = 0;
+    // Software-pipelined over conv rows: the TMEM load of row ho is issued before the pooling of row ho - 1
+    // (which reads the other conv-row buffer), so its latency and the accumulator zeroing hide behind that
+    // work; one named barrier per row separates "row ho staged" from "row ho pooled".
     for (int n = blockIdx.x; n < p.N; n += gridDim.x) {
       uint4 vb0[2], vb1[2];  // running vertical max of the open pooled rows (even / odd i), per item
 #pragma unroll
       for (int u = 0; u < 2; ++u) vb0[u] = vb1[u] = make_uint4(0, 0, 0, 0);
       bf16* yimg = p.y + (size_t)n * kPo * kPo * kCo;
-      for (int ho = 0; ho < kHo; ++ho, ++it) {
-        const uint32_t acc = it % kNAcc;
-        mbar_wait(&tfull[acc], (it / kNAcc) & 1);
-        tc_fence_after();
-        uint32_t v[32];
-        tmem_ld_32x32b_x32(tmem_base + acc * kCo + half * 32 + ((uint32_t)(q * 32) << 16), v);
-        tc_wait_ld();
-        if (p.irow) {  // input-row-major issue accumulates into zeroed slots
-          tmem_zero_32x32b_x32(tmem_base + acc * kCo + half * 32 + ((uint32_t)(q * 32) << 16));
-          tc_wait_st();
-        }
-        tc_fence_before();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&tempty[acc]);
-        const uint32_t crow = sC + (ho & 1) * kCrowBytes + wo * 128;
-        if (wo < kHo) {
-#pragma unroll
-          for (int c4 = 0; c4 < 4; ++c4) {  // 8 channels per 16-byte chunk
-            const int ch0 = half * 32 + c4 * 8;
-            float f[8];
-#pragma unroll
-            for (int j = 0; j < 8; ++j) f[j] = fmaxf(fmaf(__uint_as_float(v[c4 * 8 + j]), ss[ch0 + j], ss[kCo + ch0 + j]), 0.f);
-            uint4 o;
-            o.x = pack_bf16x2(f[0], f[1]);
-            o.y = pack_bf16x2(f[2], f[3]);
-            o.z = pack_bf16x2(f[4], f[5]);
-            o.w = pack_bf16x2(f[6], f[7]);
-            const uint32_t chunk = (uint32_t)(half * 4 + c4);
-            sts128(crow + ((chunk ^ (uint32_t)(wo & 7)) << 4), o);
-          }
-        }
-        named_bar_sync(1, kEpiThreads);
-        // conv row ho -> pooled rows: even ho closes i = ho/2 - 1 and opens i = ho/2; odd ho extends (ho-1)/2
+      // conv row ho (staged in buffer ho & 1) -> pooled rows: even ho closes i = ho/2 - 1 and opens i = ho/2;
+      // odd ho extends (ho-1)/2
+      auto pool_row = [&](const int ho) {
         const uint32_t cbase = sC + (ho & 1) * kCrowBytes;
 #pragma unroll
         for (int u = 0; u < 2; ++u) {
@@ -290,7 +263,35 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
           }
         }
+      };
+      for (int ho = 0; ho < kHo; ++ho, ++it) {
+        const uint32_t acc = it % kNAcc;
+        mbar_wait(&tfull[acc], (it / kNAcc) & 1);
+        tc_fence_after();
+        uint32_t v[32];
+        tmem_ld_32x32b_x32(tmem_base + acc * kCo + half * 32 + ((uint32_t)(q * 32) << 16), v);
+        if (ho > 0) pool_row(ho - 1);  // overlaps the TMEM load
+        tc_wait_ld_regs(v);
+        if (p.irow) {  // input-row-major issue accumulates into zeroed slots
+          tmem_zero_32x32b_x32(tmem_base + acc * kCo + half * 32 + ((uint32_t)(q * 32) << 16));
+          tc_wait_st();
+        }
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&tempty[acc]);
+        const uint32_t crow = sC + (ho & 1) * kCrowBytes + wo * 128;
+        if (wo < kHo) {
+#pragma unroll
+          for (int c4 = 0; c4 < 4; ++c4) {  // 8 channels per 16-byte chunk
+            const int ch0 = half * 32 + c4 * 8;
+            const uint4 o = epi8(v + c4 * 8, ss + ch0, ss + kCo + ch0, nullptr, true);
+            const uint32_t chunk = (uint32_t)(half * 4 + c4);
+            sts128(crow + ((chunk ^ (uint32_t)(wo & 7)) << 4), o);
+          }
+        }
+        named_bar_sync(1, kEpiThreads);
       }
+      pool_row(kHo - 1);
     }
   }
   tc_fence_before();

@@ -161,26 +161,8 @@ __device__ __forceinline__ void decode_tile(const ConvParams& p, int tile, int& 
 
 __device__ __forceinline__ void epi_math(const uint32_t* v, const float* scv, const float* shv, bool has_res,
                                          uint4 r, bool relu, uint4& o) {
-  float f[8];
-#pragma unroll
-  for (int j = 0; j < 8; ++j) f[j] = fmaf(__uint_as_float(v[j]), scv[j], shv[j]);
-  if (has_res) {
-    const uint32_t rr[4] = {r.x, r.y, r.z, r.w};
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const float2 a = unpack_bf16x2(rr[j]);
-      f[2 * j] += a.x;
-      f[2 * j + 1] += a.y;
-    }
-  }
-  if (relu) {
-#pragma unroll
-    for (int j = 0; j < 8; ++j) f[j] = fmaxf(f[j], 0.0f);
-  }
-  o.x = pack_bf16x2(f[0], f[1]);
-  o.y = pack_bf16x2(f[2], f[3]);
-  o.z = pack_bf16x2(f[4], f[5]);
-  o.w = pack_bf16x2(f[6], f[7]);
+  const uint32_t rr[4] = {r.x, r.y, r.z, r.w};
+  o = epi8(v, scv, shv, has_res ? rr : nullptr, relu);
 }
 
 __device__ __forceinline__ void epi_math_f32(const uint32_t* v, const float* scv, const float* shv, bool relu,

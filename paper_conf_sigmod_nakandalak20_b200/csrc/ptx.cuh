@@ -220,6 +220,18 @@ __device__ __forceinline__ void tmem_zero_32x32b_x32(uint32_t taddr) {
 }
 __device__ __forceinline__ void tc_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 __device__ __forceinline__ void tc_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+// tcgen05.wait::ld that also "rewrites" the loaded registers, so no use of them can be scheduled above it
+// (for code that does other work between the load and the wait)
+__device__ __forceinline__ void tc_wait_ld_regs(uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.wait::ld.sync.aligned;"
+      : "+r"(r[0]), "+r"(r[1]), "+r"(r[2]), "+r"(r[3]), "+r"(r[4]), "+r"(r[5]), "+r"(r[6]), "+r"(r[7]), "+r"(r[8]),
+        "+r"(r[9]), "+r"(r[10]), "+r"(r[11]), "+r"(r[12]), "+r"(r[13]), "+r"(r[14]), "+r"(r[15]), "+r"(r[16]),
+        "+r"(r[17]), "+r"(r[18]), "+r"(r[19]), "+r"(r[20]), "+r"(r[21]), "+r"(r[22]), "+r"(r[23]), "+r"(r[24]),
+        "+r"(r[25]), "+r"(r[26]), "+r"(r[27]), "+r"(r[28]), "+r"(r[29]), "+r"(r[30]), "+r"(r[31])
+      :
+      : "memory");
+}
 
 // 32 lanes x 32 columns of 32-bit: thread i of the warp gets lane (quadrant*32 + i), columns [c, c+32)
 __device__ __forceinline__ void tmem_ld_32x32b_x32(uint32_t taddr, uint32_t (&r)[32]) {
@@ -304,6 +316,46 @@ __host__ __device__ constexpr uint32_t umma_idesc_bf16(uint32_t M, uint32_t N) {
 __device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
   __nv_bfloat162 v = __floats2bfloat162_rn(a, b);  // RNE (cvt.rn.bf16x2.f32)
   return *reinterpret_cast<uint32_t*>(&v);
+}
+// RNE pack of max(a, 0), max(b, 0) in one instruction (a in the low half, as pack_bf16x2)
+__device__ __forceinline__ uint32_t pack_bf16x2_relu(float a, float b) {
+  uint32_t r;
+  asm("cvt.rn.relu.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(b), "f"(a));
+  return r;
+}
+// packed fp32 pairs (FFMA2 / FADD2 on sm_100): per element exactly fmaf / __fadd_rn
+__device__ __forceinline__ float2 fma2_rn(float2 a, float2 b, float2 c) {
+  unsigned long long r;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;"
+      : "=l"(r)
+      : "l"(*reinterpret_cast<unsigned long long*>(&a)), "l"(*reinterpret_cast<unsigned long long*>(&b)),
+        "l"(*reinterpret_cast<unsigned long long*>(&c)));
+  return *reinterpret_cast<float2*>(&r);
+}
+__device__ __forceinline__ float2 add2_rn(float2 a, float2 b) {
+  unsigned long long r;
+  asm("add.rn.f32x2 %0, %1, %2;"
+      : "=l"(r)
+      : "l"(*reinterpret_cast<unsigned long long*>(&a)), "l"(*reinterpret_cast<unsigned long long*>(&b)));
+  return *reinterpret_cast<float2*>(&r);
+}
+// exact bf16x2 -> two fp32 with one PRMT each (bf16 = the high half of an fp32)
+__device__ __forceinline__ float2 bf16x2_to_f2(uint32_t u) {
+  return make_float2(__uint_as_float(__byte_perm(u, 0u, 0x1044u)), __uint_as_float(__byte_perm(u, 0u, 0x3244u)));
+}
+// epilogue of 8 consecutive channels: act(acc * scale + shift (+ residual)) -> 8 bf16 (RNE), on packed
+// fp32 pairs; relu folds into the conversion (cvt.rn.relu), which equals RNE(max(x, 0)) for finite x
+__device__ __forceinline__ uint4 epi8(const uint32_t* v, const float* scv, const float* shv, const uint32_t* res,
+                                      bool relu) {
+  uint32_t o[4];
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    float2 f = fma2_rn(make_float2(__uint_as_float(v[2 * j]), __uint_as_float(v[2 * j + 1])),
+                       *reinterpret_cast<const float2*>(scv + 2 * j), *reinterpret_cast<const float2*>(shv + 2 * j));
+    if (res) f = add2_rn(f, bf16x2_to_f2(res[j]));
+    o[j] = relu ? pack_bf16x2_relu(f.x, f.y) : pack_bf16x2(f.x, f.y);
+  }
+  return make_uint4(o[0], o[1], o[2], o[3]);
 }
 __device__ __forceinline__ float2 unpack_bf16x2(uint32_t u) {
   __nv_bfloat162 v = *reinterpret_cast<__nv_bfloat162*>(&u);

@@ -26,17 +26,20 @@ constexpr int BMr = 128, BKr = 64;
 constexpr int kEpiW0 = 2, kEpiWn = 8, kEpiT = kEpiWn * 32, kThr = (kEpiW0 + kEpiWn) * 32;
 
 // V = 0: b tile double-buffered; V = 1: b single-buffered, the freed 16/32 KB spent on one more
-// weight stage (MID = 64) or one more out/residual staging buffer (MID = 128: residual chunks in flight)
+// weight stage (MID = 64) or one more out/residual staging buffer (MID = 128: residual chunks in flight).
+// MID = 256 (ResNet res4, Cout 1024): the closing conv alone (no a_next: a 1024-wide c accumulator and the
+// a GEMM's 512 KB of weights per tile do not fit beside it), b single-buffered (64 KB); V = 0: two staging
+// buffers and five weight stages, V = 1: three and three.
 template <int MID, int V = 0>
 struct RC {
   static constexpr int NCH = 4 * MID / 128;       // c chunks of 128 channels
   static constexpr int KBC = MID / BKr;           // k-blocks of the c GEMM
-  static constexpr int NBB = V ? 1 : 2;           // b tile buffers
-  static constexpr int NB = MID == 64 ? 3 : (V ? 3 : 2);  // out/residual staging buffers
-  static constexpr int WS = MID == 64 ? (V ? 5 : 4) : 3;  // weight ring stages (16 KB)
+  static constexpr int NBB = (V || MID == 256) ? 1 : 2;  // b tile buffers
+  static constexpr int NB = MID == 64 ? 3 : (MID == 256 ? (V ? 3 : 2) : (V ? 3 : 2));  // out/residual staging
+  static constexpr int WS = MID == 64 ? (V ? 5 : 4) : (MID == 256 ? (V ? 3 : 5) : 3);  // weight stages (16 KB)
   static constexpr int kB = KBC * BMr * 128;      // b tile bytes
   static constexpr int kO = BMr * 128 * 2;        // one out chunk: two 64-channel sub-tiles
-  static constexpr int kA = BMr * MID * 2;        // a_next tile
+  static constexpr int kA = MID == 256 ? 0 : BMr * MID * 2;  // a_next tile (none for MID = 256)
   static constexpr int offB = 0, offO = offB + NBB * kB, offA = offO + NB * kO, offW = offA + kA,
                        offS = offW + WS * 16384, offBar = offS + (5 * MID) * 2 * 4;
   static constexpr int nBar = 2 + 2 + NB * 3 + 2 * WS + 2 + 1 + 1 + 2;
@@ -61,6 +64,7 @@ __global__ void __launch_bounds__(kThr, 1)
                      const RCParams p) {
   using C = RC<MID, V>;
   constexpr int NCH = C::NCH, KBC = C::KBC, NB = C::NB, WS = C::WS, NBB = C::NBB;
+  constexpr bool kCanA = MID <= 128;  // MID = 256: closing conv only
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 1023u) & ~1023u;
@@ -117,7 +121,7 @@ __global__ void __launch_bounds__(kThr, 1)
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
-  const uint32_t tmem = *tmem_slot;  // acc_c[0] cols 0..127, acc_c[1] 128..255, acc_a 256..256+MID
+  const uint32_t tmem = *tmem_slot;  // acc_c[0] cols 0..127, acc_c[1] 128..255, acc_a 256..256+MID (MID <= 128)
 
   if (warp == 0) {
     // ================= producer =================
@@ -158,7 +162,7 @@ __global__ void __launch_bounds__(kThr, 1)
             push_c(j + 1);
             push_res(m0, j + 1);
           }
-          if (p.has_a) push_a(j);
+          if (kCanA && p.has_a) push_a(j);
         }
       }
     }
@@ -218,7 +222,7 @@ __global__ void __launch_bounds__(kThr, 1)
 #pragma unroll
       for (int j = 0; j < NCH; ++j) {
         if (j + 1 < NCH) issue_c(j + 1);
-        if (p.has_a) issue_a(j);
+        if (kCanA && p.has_a) issue_a(j);
       }
     }
   } else {
@@ -249,21 +253,7 @@ __global__ void __launch_bounds__(kThr, 1)
             const uint32_t addr = sub + (((uint32_t)((cb & 1) * 4 + k) ^ (uint32_t)(row & 7)) << 4);
             const uint4 r = lds128(addr);
             const uint32_t rr[4] = {r.x, r.y, r.z, r.w};
-            float f[8];
-#pragma unroll
-            for (int e = 0; e < 8; ++e) f[e] = fmaf(__uint_as_float(v[k * 8 + e]), sc_c[ch + e], sh_c[ch + e]);
-#pragma unroll
-            for (int e = 0; e < 4; ++e) {
-              const float2 a = unpack_bf16x2(rr[e]);
-              f[2 * e] = fmaxf(f[2 * e] + a.x, 0.f);
-              f[2 * e + 1] = fmaxf(f[2 * e + 1] + a.y, 0.f);
-            }
-            uint4 o;
-            o.x = pack_bf16x2(f[0], f[1]);
-            o.y = pack_bf16x2(f[2], f[3]);
-            o.z = pack_bf16x2(f[4], f[5]);
-            o.w = pack_bf16x2(f[6], f[7]);
-            sts128(addr, o);
+            sts128(addr, epi8(v + k * 8, sc_c + ch, sh_c + ch, rr, true));
           }
         }
         tc_fence_before();
@@ -274,7 +264,7 @@ __global__ void __launch_bounds__(kThr, 1)
         if (et == 0) {
           // the previous chunk's store must have read its buffer before that buffer is refilled
           if (qq >= 1) {
-            if (j == 0 && p.has_a) bulk_wait_read<1>();  // the previous tile's a_next store was committed after it
+            if (j == 0 && kCanA && p.has_a) bulk_wait_read<1>();  // the previous tile's a_next store was committed after it
             else bulk_wait_read<0>();
             mbar_arrive(&ofree[(qq - 1) % NB]);
           }
@@ -284,7 +274,7 @@ __global__ void __launch_bounds__(kThr, 1)
           bulk_commit();
         }
       }
-      if (!p.has_a) continue;
+      if (!kCanA || !p.has_a) continue;
       // ---- a_next = ReLU(BN_a(acc_a)) ----
       mbar_wait(tfull_a, it & 1);
       tc_fence_after();
@@ -300,16 +290,8 @@ __global__ void __launch_bounds__(kThr, 1)
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
           const int ch = cb * 32 + k * 8;
-          float f[8];
-#pragma unroll
-          for (int e = 0; e < 8; ++e)
-            f[e] = fmaxf(fmaf(__uint_as_float(v[k * 8 + e]), sc_a[ch + e], sh_a[ch + e]), 0.f);
-          uint4 o;
-          o.x = pack_bf16x2(f[0], f[1]);
-          o.y = pack_bf16x2(f[2], f[3]);
-          o.z = pack_bf16x2(f[4], f[5]);
-          o.w = pack_bf16x2(f[6], f[7]);
-          sts128(sub + (((uint32_t)((cb & 1) * 4 + k) ^ (uint32_t)(row & 7)) << 4), o);
+          sts128(sub + (((uint32_t)((cb & 1) * 4 + k) ^ (uint32_t)(row & 7)) << 4),
+                 epi8(v + k * 8, sc_a + ch, sh_a + ch, nullptr, true));
         }
       }
       tc_fence_before();
@@ -333,8 +315,9 @@ __global__ void __launch_bounds__(kThr, 1)
 
 bool res_chain_supported(const ConvLayer& Lc, const ConvLayer* La) {
   const int mid = Lc.Cin;
-  const bool c_ok = (mid == 64 || mid == 128) && Lc.R == 1 && Lc.S == 1 && Lc.stride == 1 && Lc.pad == 0 &&
-                    Lc.groups == 1 && Lc.Cout == 4 * mid && Lc.BN == 128 && Lc.relu;
+  static const bool mid256 = !(getenv("VISTA_CHAIN256") && getenv("VISTA_CHAIN256")[0] == '0');  // A/B switch
+  const bool c_ok = (mid == 64 || mid == 128 || (mid == 256 && mid256 && !La)) && Lc.R == 1 && Lc.S == 1 &&
+                    Lc.stride == 1 && Lc.pad == 0 && Lc.groups == 1 && Lc.Cout == 4 * mid && Lc.BN == 128 && Lc.relu;
   return c_ok && (!La || (La->R == 1 && La->S == 1 && La->stride == 1 && La->pad == 0 && La->groups == 1 &&
                           La->Cin == 4 * mid && La->Cout == mid && La->BN == mid && La->relu));
 }
@@ -378,6 +361,10 @@ void res_chain_forward(const ConvLayer& Lc, const ConvLayer* La, const bf16* b, 
   if (mid == 64) {
     if (v & 1) launch_chain<64, 1>(Lc, La, b, res, out, a_next, M, st);
     else launch_chain<64, 0>(Lc, La, b, res, out, a_next, M, st);
+  } else if (mid == 256) {
+    if (La) fail(1, "res_chain: MID = 256 runs the closing conv only");
+    if (v & 4) launch_chain<256, 1>(Lc, nullptr, b, res, out, a_next, M, st);
+    else launch_chain<256, 0>(Lc, nullptr, b, res, out, a_next, M, st);
   } else {
     if (v & 2) launch_chain<128, 1>(Lc, La, b, res, out, a_next, M, st);
     else launch_chain<128, 0>(Lc, La, b, res, out, a_next, M, st);

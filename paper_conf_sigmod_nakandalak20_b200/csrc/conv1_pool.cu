@@ -284,7 +284,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
           for (int c4 = 0; c4 < 4; ++c4) {  // 8 channels per 16-byte chunk
             const int ch0 = half * 32 + c4 * 8;
-            const uint4 o = epi8(v + c4 * 8, ss + ch0, ss + kCo + ch0, nullptr, true);
+            const uint4 o = epi8(v + c4 * 8, ss + ch0, ss + kCo + ch0, make_uint4(0, 0, 0, 0), false, true);
             const uint32_t chunk = (uint32_t)(half * 4 + c4);
             sts128(crow + ((chunk ^ (uint32_t)(wo & 7)) << 4), o);
           }

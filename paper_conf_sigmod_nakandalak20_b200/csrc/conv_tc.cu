@@ -161,8 +161,7 @@ __device__ __forceinline__ void decode_tile(const ConvParams& p, int tile, int& 
 
 __device__ __forceinline__ void epi_math(const uint32_t* v, const float* scv, const float* shv, bool has_res,
                                          uint4 r, bool relu, uint4& o) {
-  const uint32_t rr[4] = {r.x, r.y, r.z, r.w};
-  o = epi8(v, scv, shv, has_res ? rr : nullptr, relu);
+  o = epi8(v, scv, shv, r, has_res, relu);
 }
 
 __device__ __forceinline__ void epi_math_f32(const uint32_t* v, const float* scv, const float* shv, bool relu,

@@ -980,6 +980,7 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
                o_bar = carve(16), o_scal = carve((size_t)2 * std::max(grid_tr, 1) * 8);
   uint8_t* scr = nullptr;
   VCHECK(cudaMallocAsync(&scr, off, st));
+  VCHECK(cudaMemsetAsync(scr, 0, off, st));  // every byte defined (LRState fields a path leaves unwritten)
   float* partial = reinterpret_cast<float*>(scr + o_part);
   double* G = reinterpret_cast<double*>(scr + o_G);
   double* mu = reinterpret_cast<double*>(scr + o_mu);
@@ -994,8 +995,6 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   double* loss = reinterpret_cast<double*>(scr + o_loss);
   unsigned long long* cnt = reinterpret_cast<unsigned long long*>(scr + o_cnt);
   VCHECK(cudaMemcpyAsync(real, real_host, ld, cudaMemcpyHostToDevice, st));
-  VCHECK(cudaMemsetAsync(cnt, 0, 64, st));
-  VCHECK(cudaMemsetAsync(scr + o_bar, 0, 16, st));
 
   PassArgs a;
   std::memset(&a, 0, sizeof(a));

@@ -343,16 +343,21 @@ __device__ __forceinline__ float2 add2_rn(float2 a, float2 b) {
 __device__ __forceinline__ float2 bf16x2_to_f2(uint32_t u) {
   return make_float2(__uint_as_float(__byte_perm(u, 0u, 0x1044u)), __uint_as_float(__byte_perm(u, 0u, 0x3244u)));
 }
-// epilogue of 8 consecutive channels: act(acc * scale + shift (+ residual)) -> 8 bf16 (RNE), on packed
-// fp32 pairs; relu folds into the conversion (cvt.rn.relu), which equals RNE(max(x, 0)) for finite x
-__device__ __forceinline__ uint4 epi8(const uint32_t* v, const float* scv, const float* shv, const uint32_t* res,
+// epilogue of 8 consecutive channels: act(acc * scale + shift (+ residual r)) -> 8 bf16 (RNE), on packed
+// fp32 pairs; relu folds into the conversion (cvt.rn.relu), which equals RNE(max(x, 0)) for finite x.
+// scv / shv: 16-byte aligned (shared memory); everything by value (no local-memory arrays)
+__device__ __forceinline__ uint4 epi8(const uint32_t* v, const float* scv, const float* shv, uint4 r, bool has_res,
                                       bool relu) {
+  const float4 s0 = *reinterpret_cast<const float4*>(scv), s1 = *reinterpret_cast<const float4*>(scv + 4);
+  const float4 h0 = *reinterpret_cast<const float4*>(shv), h1 = *reinterpret_cast<const float4*>(shv + 4);
+  const float2 sc[4] = {make_float2(s0.x, s0.y), make_float2(s0.z, s0.w), make_float2(s1.x, s1.y), make_float2(s1.z, s1.w)};
+  const float2 sh[4] = {make_float2(h0.x, h0.y), make_float2(h0.z, h0.w), make_float2(h1.x, h1.y), make_float2(h1.z, h1.w)};
+  const uint32_t rr[4] = {r.x, r.y, r.z, r.w};
   uint32_t o[4];
 #pragma unroll
   for (int j = 0; j < 4; ++j) {
-    float2 f = fma2_rn(make_float2(__uint_as_float(v[2 * j]), __uint_as_float(v[2 * j + 1])),
-                       *reinterpret_cast<const float2*>(scv + 2 * j), *reinterpret_cast<const float2*>(shv + 2 * j));
-    if (res) f = add2_rn(f, bf16x2_to_f2(res[j]));
+    float2 f = fma2_rn(make_float2(__uint_as_float(v[2 * j]), __uint_as_float(v[2 * j + 1])), sc[j], sh[j]);
+    if (has_res) f = add2_rn(f, bf16x2_to_f2(rr[j]));
     o[j] = relu ? pack_bf16x2_relu(f.x, f.y) : pack_bf16x2(f.x, f.y);
   }
   return make_uint4(o[0], o[1], o[2], o[3]);

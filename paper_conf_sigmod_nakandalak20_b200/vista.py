@@ -13,7 +13,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libvista.so")
+# VISTA_LIB_PATH: another build of the same library (A/B measurements of two builds in one job only)
+LIB_PATH = os.environ.get("VISTA_LIB_PATH") or os.path.join(_HERE, "libvista.so")
 _LIB = None
 
 ALEXNET, VGG16, RESNET50 = 0, 1, 2

@@ -356,9 +356,11 @@ def main():
     value = N_global / (ms_step / 1000.0)
     # ---- e2e: host inputs through the C-ABI, weights back to the host ----
     peak_meas = None
+    graph_info = {"cnn_graph": v.plan_info()["cnn_graph"], "kernels": v.plan_info()["cnn_graph_kernels"]}
     if args.e2e_steps > 0:
         step(host=True)  # untimed warm-up of the host-input path (sizes its per-chunk pixel buffer)
         pinfo = v.plan_info()  # pool high-water mark of that transfer from host pixels vs the prediction
+        graph_info = {"cnn_graph": pinfo["cnn_graph"], "kernels": pinfo["cnn_graph_kernels"]}
         peak_meas = {"pred": pinfo["peak_bytes_pred"], "meas": pinfo["peak_bytes_meas"],
                      "reserved": pinfo["peak_reserved_meas"],
                      "meas_over_pred": pinfo["peak_bytes_meas"] / max(pinfo["peak_bytes_pred"], 1)}
@@ -435,6 +437,7 @@ def main():
                     "h2d_bytes_per_step": h2d_bytes, "d2h_bytes_per_step": d2h,
                     "note": "vista_transfer with pinned host inputs + vista_train weights to host"},
             "gpu_launches": launches,
+            "cuda_graph": graph_info,
             "clocks": clocks,
             "breakdown_ms": breakdown,
             "test_acc_per_layer": accs,

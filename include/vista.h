@@ -115,6 +115,10 @@ typedef struct {
    * allocates during a transfer comes from that pool), and the same with the pool's reserved bytes. */
   int64_t peak_bytes_meas;
   int64_t peak_reserved_meas;
+  /* The last transfer ran its CNN part (S0-S3 + taps) as one CUDA graph: 0 no, 1 captured, 2 replayed;
+   * cnn_graph_kernels = kernels in that graph. */
+  int32_t cnn_graph;
+  int32_t cnn_graph_kernels;
 } vista_plan_info_t;
 
 /* Borrowed view of layer k's outputs on this rank (valid until vista_destroy or the

@@ -271,7 +271,7 @@ __global__ void __launch_bounds__(kThr, 1)
             else bulk_wait_read<0>();
             mbar_arrive(&ofree[(qq - 1) % NB]);
           }
-          mbar_arrive(&oready[ob]);  // staged chunk may feed the a-MMA
+          if (kCanA && p.has_a) mbar_arrive(&oready[ob]);  // staged chunk may feed the a-MMA (waited only then)
           tma_store_2d(&tm_out, j * 128, m0, so);
           tma_store_2d(&tm_out, j * 128 + 64, m0, so + BMr * 128);
           bulk_commit();

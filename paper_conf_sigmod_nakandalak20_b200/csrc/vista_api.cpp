@@ -239,6 +239,15 @@ struct DevBuf {
   DevBuf& operator=(const DevBuf&) = delete;
 };
 
+static bool is_pinned_host(const void* p) {
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return at.type == cudaMemoryTypeHost;
+}
+
 static bool is_device_ptr(const void* p) {
   cudaPointerAttributes at;
   if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
@@ -287,6 +296,22 @@ struct vista_ctx {
   bool transferred = false;
   void* nccl_comm = nullptr;
   HookAR hook;                   // world > 1 without NCCL
+  // CUDA graph of the CNN part of a transfer (S0-S3 + taps: ~800 launches per 20k ResNet images), replayed
+  // while the transfer's signature (inputs and every buffer it touches) is unchanged; two entries (device-
+  // and host-resident pixels alternate in bench.py)
+  struct CnnGraph {
+    std::vector<uintptr_t> sig;
+    cudaGraphExec_t exec = nullptr;
+    std::vector<void*> act;  // host bookkeeping the captured run set (c->act)
+    uint64_t use = 0;
+  };
+  CnnGraph graphs[2];
+  cudaStream_t cap_stream = nullptr;  // captures happen here (the caller's stream may be the legacy one)
+  int graph_failed = 0;               // failed captures (a first transfer may meet one-time setup calls
+                                      // that cannot be captured); after two, this ctx runs eagerly
+  uint64_t graph_clock = 0;
+  int64_t graph_launches = 0;    // kernels one replay runs (counted at capture)
+  int graph_state = 0;           // last transfer: 0 eager, 1 captured, 2 replayed
   DevBuf d_flags;                // device status flags of a transfer (X not bf16-representable)
   int64_t peak_meas = 0, peak_res_meas = 0;  // measured peak device bytes of the last transfer
   std::unique_ptr<Profiler> prof;
@@ -333,6 +358,9 @@ struct vista_ctx {
       Nccl& n = nccl_lib();
       if (n.CommDestroy) n.CommDestroy(nccl_comm);
     }
+    for (auto& g : graphs)
+      if (g.exec) cudaGraphExecDestroy(g.exec);
+    if (cap_stream) cudaStreamDestroy(cap_stream);
     if (own_stream && stream) cudaStreamDestroy(stream);
     for (cudaEvent_t e : px_ready) cudaEventDestroy(e);
     if (px_free) cudaEventDestroy(px_free);
@@ -1032,6 +1060,8 @@ VISTA_API vista_status vista_plan_info(const vista_ctx* c, vista_plan_info_t* o)
   o->chunk_images = c->chunk;
   o->peak_bytes_meas = c->peak_meas;
   o->peak_reserved_meas = c->peak_res_meas;
+  o->cnn_graph = c->graph_state;
+  o->cnn_graph_kernels = (int32_t)c->graph_launches;
   return VISTA_OK;
 }
 
@@ -1056,6 +1086,8 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
       uint64_t zero = 0;
       VCHECK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrUsedMemHigh, &zero));
       VCHECK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReservedMemHigh, &zero));
+      VCHECK(cudaDeviceSetGraphMemAttribute(c->sys.device, cudaGraphMemAttrUsedMemHigh, &zero));
+      VCHECK(cudaDeviceSetGraphMemAttribute(c->sys.device, cudaGraphMemAttrReservedMemHigh, &zero));
     }
     c->d_flags.ensure(16);
     VCHECK(cudaMemsetAsync(c->d_flags.p, 0, 16, st));
@@ -1113,27 +1145,10 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
                       (const int32_t*)c->pair_img.p, lab, c->n_pairs, ld, (bf16*)c->MM[k]->p, (uint8_t*)c->Y[k]->p,
                       (int*)c->d_flags.p, st);
     };
-    if (c->sys.plan != VISTA_PLAN_STAGED) {
-      // ---- Eager / Lazy (Fig 5C / 5A): features of every layer, no resident full activations ----
-      // with a pre-materialised base (App. B): Eager = one pass base -> all of L; Lazy = "Lazy-5 with
-      // Pre-mat": one pass per layer from the stored base
-      const std::vector<cudaEvent_t>* unstaged_ev = nullptr;
-      if (!base && c->n_img > 0 && !is_device_ptr(images)) {
-        unstaged_ev = stream_host_pixels(c, images, 0, c->n_img);
-        px = (const uint8_t*)c->d_px.p;
-      }
-      const int t_first = base ? t0 + 1 : 0;
-      if (c->sys.plan == VISTA_PLAN_EAGER) {
-        run_unstaged(c, px, t_first, c->t_max, c->taps, unstaged_ev, base, host_base);
-      } else {
-        for (int t : c->taps) run_unstaged(c, px, t_first, t, std::vector<int>{t}, unstaged_ev, base, host_base);
-      }
-      for (size_t k = 0; k < c->taps.size(); ++k) concat_layer((int)k);
-    }
-    // ---- Staged (Fig 5E), over chunks of images when the HBM budget forces it (planner) ----
+    // ---- S0-S3 + taps (the CNN part): no host synchronisation inside, so it runs as one CUDA graph ----
     const int64_t CH = c->sys.plan == VISTA_PLAN_STAGED ? std::max<int64_t>(c->chunk, 1) : 0;
     const bool chunked = CH > 0 && CH < c->n_img;
-    const bool host_px = !base && px == images && c->n_img > 0 && !is_device_ptr(images);
+    const bool host_px = !base && c->n_img > 0 && !is_device_ptr(images);
     if (CH > 0) {
       size_t need[2] = {16, 16};
       for (int t = 0; t <= c->t_max; ++t)
@@ -1142,62 +1157,174 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
       c->arena[0].ensure(need[0]);
       c->arena[1].ensure(need[1]);
     }
-    for (int64_t c0 = 0; CH > 0 && c0 < c->n_img; c0 += CH) {
-      const int64_t nc = std::min<int64_t>(CH, c->n_img - c0);
-      const uint8_t* pxc = base ? nullptr : px + (size_t)c0 * S[0].in_elems;
-      const void* base_c = nullptr;  // this chunk's A_t0 (the caller's memory, or its H2D copy in arena t0 % 2)
-      if (base) {
-        if (host_base) {
-          VCHECK(cudaMemcpyAsync(c->arena[t0 & 1].p, (const uint8_t*)base + (size_t)c0 * base_img_bytes,
-                                 (size_t)nc * base_img_bytes, cudaMemcpyHostToDevice, st));
-          base_c = c->arena[t0 & 1].p;
-        } else {
-          base_c = (const uint8_t*)base + (size_t)c0 * base_img_bytes;
-        }
-      }
-      const std::vector<cudaEvent_t>* px_ev = nullptr;
-      if (host_px) {  // stream the chunk's pixels to the device, one stage-1 micro-batch per copy
-        px_ev = stream_host_pixels(c, images, c0, nc);
-        pxc = (const uint8_t*)c->d_px.p;
-      }
-      for (int t = base ? t0 : 0; t <= c->t_max; ++t) {
-        void* At = t == t0 ? const_cast<void*>(base_c) : c->arena[t & 1].p;
-        c->act[t] = At;
-        const void* in = t == 0 ? (const void*)pxc : (t - 1 == t0 ? base_c : c->arena[(t - 1) & 1].p);
-        const int k = layer_index(c, t);
-        // S2 fused into the producing conv's epilogue (opt-in, unchunked only)
-        unsigned int* tapf = nullptr;
-        if (k >= 0 && t != t0 && !S[t].fc_tap && c->fuse_tap && !chunked && !c->f32) {
-          const size_t cnt = (size_t)nc * 4 * S[t].outC;
-          c->tapacc.ensure(cnt * 4);
-          VCHECK(cudaMemsetAsync(c->tapacc.p, 0, cnt * 4, st));  // max over non-negative (post-ReLU) values
-          tapf = (unsigned int*)c->tapacc.p;
-        }
-        const bool fused = t == t0 ? false : run_block(c, t, in, At, nc, tapf, t == 0 ? px_ev : nullptr);
-        if (k >= 0) {
-          void* Ft = (uint8_t*)c->F[t]->p + (size_t)c0 * S[t].d_tap * c->esz;
-          if (S[t].fc_tap)  // g = identity on FC layers
-            VCHECK(cudaMemcpyAsync(Ft, At, (size_t)nc * S[t].d_tap * c->esz, cudaMemcpyDeviceToDevice, st));
-          else if (fused)
-            launch_tap_finalize(tapf, (int64_t)nc * S[t].d_tap, (bf16*)Ft, st);
-          else
-            tap_any(c, At, nc, S[t], Ft);
-          if (!chunked) concat_layer(k);
-        }
+    // every persistent buffer the CNN part uses is sized now, so nothing is allocated while capturing
+    {
+      void* slot[NUM_BUFS] = {nullptr};
+      const int tb = base ? t0 + 1 : 0;
+      for (int t = tb; t <= c->t_max; ++t) prepare_slots(c, t, c->micro[c->sys.plan == VISTA_PLAN_STAGED ? t : 0], slot);
+      if (host_px) c->d_px.ensure((size_t)(CH > 0 ? std::min<int64_t>(CH, c->n_img) : c->n_img) * S[0].in_elems);
+      if (c->fuse_tap && !chunked && !c->f32 && CH > 0) {
+        size_t cnt = 0;
+        for (int t : c->taps)
+          if (!S[t].fc_tap) cnt = std::max(cnt, (size_t)std::min<int64_t>(CH, c->n_img) * 4 * S[t].outC);
+        if (cnt) c->tapacc.ensure(cnt * 4);
       }
     }
-    if (chunked)
-      for (size_t k = 0; k < c->taps.size(); ++k) concat_layer((int)k);
+    auto cnn_part = [&]() {
+      cudaStream_t st = c->stream;  // the capture stream while capturing
+      if (c->sys.plan != VISTA_PLAN_STAGED) {
+        // ---- Eager / Lazy (Fig 5C / 5A): features of every layer, no resident full activations ----
+        // with a pre-materialised base (App. B): Eager = one pass base -> all of L; Lazy = "Lazy-5 with
+        // Pre-mat": one pass per layer from the stored base
+        const uint8_t* pxu = px;
+        const std::vector<cudaEvent_t>* unstaged_ev = nullptr;
+        if (host_px) {
+          unstaged_ev = stream_host_pixels(c, images, 0, c->n_img);
+          pxu = (const uint8_t*)c->d_px.p;
+        }
+        const int t_first = base ? t0 + 1 : 0;
+        if (c->sys.plan == VISTA_PLAN_EAGER) {
+          run_unstaged(c, pxu, t_first, c->t_max, c->taps, unstaged_ev, base, host_base);
+        } else {
+          for (int t : c->taps) run_unstaged(c, pxu, t_first, t, std::vector<int>{t}, unstaged_ev, base, host_base);
+        }
+        return;
+      }
+      // ---- Staged (Fig 5E), over chunks of images when the HBM budget forces it (planner) ----
+      for (int64_t c0 = 0; c0 < c->n_img; c0 += CH) {
+        const int64_t nc = std::min<int64_t>(CH, c->n_img - c0);
+        const uint8_t* pxc = base ? nullptr : px + (size_t)c0 * S[0].in_elems;
+        const void* base_c = nullptr;  // this chunk's A_t0 (the caller's memory, or its H2D copy in arena t0 % 2)
+        if (base) {
+          if (host_base) {
+            VCHECK(cudaMemcpyAsync(c->arena[t0 & 1].p, (const uint8_t*)base + (size_t)c0 * base_img_bytes,
+                                   (size_t)nc * base_img_bytes, cudaMemcpyHostToDevice, st));
+            base_c = c->arena[t0 & 1].p;
+          } else {
+            base_c = (const uint8_t*)base + (size_t)c0 * base_img_bytes;
+          }
+        }
+        const std::vector<cudaEvent_t>* px_ev = nullptr;
+        if (host_px) {  // stream the chunk's pixels to the device, one stage-1 micro-batch per copy
+          px_ev = stream_host_pixels(c, images, c0, nc);
+          pxc = (const uint8_t*)c->d_px.p;
+        }
+        for (int t = base ? t0 : 0; t <= c->t_max; ++t) {
+          void* At = t == t0 ? const_cast<void*>(base_c) : c->arena[t & 1].p;
+          c->act[t] = At;
+          const void* in = t == 0 ? (const void*)pxc : (t - 1 == t0 ? base_c : c->arena[(t - 1) & 1].p);
+          const int k = layer_index(c, t);
+          // S2 fused into the producing conv's epilogue (opt-in, unchunked only)
+          unsigned int* tapf = nullptr;
+          if (k >= 0 && t != t0 && !S[t].fc_tap && c->fuse_tap && !chunked && !c->f32) {
+            const size_t cnt = (size_t)nc * 4 * S[t].outC;
+            c->tapacc.ensure(cnt * 4);
+            VCHECK(cudaMemsetAsync(c->tapacc.p, 0, cnt * 4, st));  // max over non-negative (post-ReLU) values
+            tapf = (unsigned int*)c->tapacc.p;
+          }
+          const bool fused = t == t0 ? false : run_block(c, t, in, At, nc, tapf, t == 0 ? px_ev : nullptr);
+          if (k >= 0) {
+            void* Ft = (uint8_t*)c->F[t]->p + (size_t)c0 * S[t].d_tap * c->esz;
+            if (S[t].fc_tap)  // g = identity on FC layers
+              VCHECK(cudaMemcpyAsync(Ft, At, (size_t)nc * S[t].d_tap * c->esz, cudaMemcpyDeviceToDevice, st));
+            else if (fused)
+              launch_tap_finalize(tapf, (int64_t)nc * S[t].d_tap, (bf16*)Ft, st);
+            else
+              tap_any(c, At, nc, S[t], Ft);
+          }
+        }
+      }
+    };
+    // graph replay when this transfer's signature matches a captured one.  Not while profiling (per-launch
+    // events are host-side records), not with pageable host inputs (graph copies need pinned memory);
+    // VISTA_GRAPH=0 disables.
+    static const bool graphs_on = !(getenv("VISTA_GRAPH") && getenv("VISTA_GRAPH")[0] == '0') &&
+                                  !(getenv("VISTA_CONV_DBG") && atoi(getenv("VISTA_CONV_DBG")) != 0);
+    const bool pageable = (host_px && !is_pinned_host(images)) || (host_base && !is_pinned_host(base));
+    c->graph_state = 0;
+    if (graphs_on && !g_prof && c->n_img > 0 && !pageable && c->graph_failed < 2) {
+      if (host_px && !c->copy_stream) {  // created outside any capture
+        VCHECK(cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking));
+        VCHECK(cudaEventCreateWithFlags(&c->px_free, cudaEventDisableTiming));
+      }
+      if (!c->cap_stream) VCHECK(cudaStreamCreateWithFlags(&c->cap_stream, cudaStreamNonBlocking));
+      std::vector<uintptr_t> sig = {(uintptr_t)images, (uintptr_t)base, (uintptr_t)host_px, (uintptr_t)host_base,
+                                    (uintptr_t)c->arena[0].p, (uintptr_t)c->arena[1].p, (uintptr_t)c->d_px.p,
+                                    (uintptr_t)c->tapacc.p, (uintptr_t)c->copy_stream, (uintptr_t)c->n_img};
+      for (auto& sb : c->slot_store) sig.push_back((uintptr_t)sb->p);
+      for (auto& f : c->F) sig.push_back((uintptr_t)(f ? f->p : nullptr));
+      vista_ctx::CnnGraph* hit = nullptr;
+      for (auto& g : c->graphs)
+        if (g.exec && g.sig == sig) hit = &g;
+      if (!hit) {
+        vista_ctx::CnnGraph* slot = &c->graphs[0];
+        for (auto& g : c->graphs)
+          if (!g.exec || g.use < slot->use) slot = &g;
+        if (slot->exec) {
+          VCHECK(cudaGraphExecDestroy(slot->exec));
+          slot->exec = nullptr;
+        }
+        // capture on the ctx's capture stream (the caller's may be the legacy stream, which cannot capture);
+        // the launch goes to the caller's stream
+        const long long l0 = launches_total();
+        cudaGraph_t graph = nullptr;
+        cudaStream_t user = c->stream;
+        bool ok = cudaStreamBeginCapture(c->cap_stream, cudaStreamCaptureModeThreadLocal) == cudaSuccess;
+        if (ok) {
+          c->stream = c->cap_stream;
+          tl_stream = c->cap_stream;
+          try {
+            cnn_part();
+          } catch (const VistaError&) {
+            ok = false;
+          }
+          c->stream = user;
+          tl_stream = user;
+          ok = cudaStreamEndCapture(c->cap_stream, &graph) == cudaSuccess && ok && graph;
+          ok = ok && cudaGraphInstantiate(&slot->exec, graph, 0) == cudaSuccess;
+          if (graph) cudaGraphDestroy(graph);
+        }
+        if (!ok) {  // fall back to launching the kernels directly, for this ctx from now on
+          cudaGetLastError();
+          if (slot->exec) cudaGraphExecDestroy(slot->exec);
+          slot->exec = nullptr;
+          ++c->graph_failed;
+          cnn_part();
+        } else {
+          c->graph_launches = launches_total() - l0;
+          c->graph_state = 1;
+          slot->sig = sig;
+          slot->act = c->act;
+          hit = slot;
+        }
+      } else {
+        for (long long i = 0; i < c->graph_launches; ++i) count_launch();  // the replay's kernels
+        c->act = hit->act;
+        c->graph_state = 2;
+      }
+      if (hit) {
+        hit->use = ++c->graph_clock;
+        VCHECK(cudaGraphLaunch(hit->exec, st));
+      }
+    } else {
+      cnn_part();
+    }
+    // ---- S4 concat (Eq. 4) of every layer ----
+    for (size_t k = 0; k < c->taps.size(); ++k) concat_layer((int)k);
     int flags[4] = {0, 0, 0, 0};
     VCHECK(cudaMemcpyAsync(flags, c->d_flags.p, 16, cudaMemcpyDeviceToHost, st));
     VCHECK(cudaStreamSynchronize(st));
     if (g_prof) g_prof->flush();
     {
-      uint64_t used_hi = 0, res_hi = 0;
+      // stream-ordered buffers come from the default pool; allocations inside a CUDA graph (the VGG conv1_1
+      // padded copy, the Eager/Lazy micro-batch buffers) from the graph memory pool
+      uint64_t used_hi = 0, res_hi = 0, gused_hi = 0, gres_hi = 0;
       VCHECK(cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemHigh, &used_hi));
       VCHECK(cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemHigh, &res_hi));
-      c->peak_meas = c->weight_bytes + (int64_t)used_hi;
-      c->peak_res_meas = c->weight_bytes + (int64_t)res_hi;
+      VCHECK(cudaDeviceGetGraphMemAttribute(c->sys.device, cudaGraphMemAttrUsedMemHigh, &gused_hi));
+      VCHECK(cudaDeviceGetGraphMemAttribute(c->sys.device, cudaGraphMemAttrReservedMemHigh, &gres_hi));
+      c->peak_meas = c->weight_bytes + (int64_t)(used_hi + gused_hi);
+      c->peak_res_meas = c->weight_bytes + (int64_t)(res_hi + gres_hi);
     }
     if (flags[0] & 1)
       fail(1, "structured value not bf16-representable (include/vista.h: X values must be bf16-representable)");

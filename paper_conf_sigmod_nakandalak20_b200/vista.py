@@ -50,7 +50,8 @@ class PlanInfo(ctypes.Structure):
     _fields_ = [("n_layers", _i32), ("tap", _i32 * 8), ("d_l", _i32 * 8), ("ld", _i32 * 8),
                 ("micro_batch", _i32 * 8), ("act_bytes", _i64 * 8), ("peak_bytes_pred", _i64),
                 ("weight_bytes", _i64), ("d_s", _i32), ("ds_pad", _i32), ("chunk_images", _i64),
-                ("peak_bytes_meas", _i64), ("peak_reserved_meas", _i64)]
+                ("peak_bytes_meas", _i64), ("peak_reserved_meas", _i64), ("cnn_graph", _i32),
+                ("cnn_graph_kernels", _i32)]
 
 
 class Buffer(ctypes.Structure):
@@ -318,7 +319,8 @@ class Vista:
                     micro_batch=list(pi.micro_batch[:n]), act_bytes=list(pi.act_bytes[:n]),
                     peak_bytes_pred=pi.peak_bytes_pred, weight_bytes=pi.weight_bytes, d_s=pi.d_s, ds_pad=pi.ds_pad,
                     chunk_images=pi.chunk_images, peak_bytes_meas=pi.peak_bytes_meas,
-                    peak_reserved_meas=pi.peak_reserved_meas)
+                    peak_reserved_meas=pi.peak_reserved_meas, cnn_graph=pi.cnn_graph,
+                    cnn_graph_kernels=pi.cnn_graph_kernels)
 
     def transfer(self, images, image_keys, structured, str_keys, labels):
         _check(lib().vista_transfer(self.ctx, _ptr(images), _ptr(image_keys), _ptr(structured), _ptr(str_keys),

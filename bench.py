@@ -221,6 +221,9 @@ def main():
                          "(PAPER.md:383, vista_train_mlp, 10 steps)")
     ap.add_argument("--plan", default="staged", choices=["staged", "eager", "lazy"],
                     help="logical plan (Fig 5): staged is the product; eager / lazy for config 4 comparisons")
+    ap.add_argument("--api", default="run", choices=["run", "split"],
+                    help="run: vista_run (M of layer k on a second stream beside stage k+1, S6); split: "
+                         "vista_transfer then vista_train(k) per layer")
     ap.add_argument("--dry-run", action="store_true",
                     help="print the launch command (torchrun re-exec for --gpus N > 1) and exit")
     args = ap.parse_args()
@@ -304,6 +307,10 @@ def main():
                 v.transfer_from_base(h_base, h_ik, h_X, h_sk, h_y)
             else:
                 v.transfer_from_base(d_base, d_ik, d_X, d_sk, d_y)
+        elif args.api == "run" and args.model == "lr":
+            if host:
+                return v.run(h_px, h_ik, h_X, h_sk, h_y, d_tot)
+            return v.run(d_px, d_ik, d_X, d_sk, d_y, d_tot, want_weights=False)
         elif host:
             v.transfer(h_px, h_ik, h_X, h_sk, h_y)
         else:
@@ -428,6 +435,8 @@ def main():
             "config": dict(workload_config(args.config, world, n_img), micro_batch=info["micro_batch"],
                            plan=args.plan + ("+prematerialized_base" if args.from_base else ""),
                            model=("mlp_1024x1024x1_T10" if args.model == "mlp" else "elastic_net_lr_T%d" % T),
+                           api=("vista_run" if args.api == "run" and args.model == "lr" and not args.from_base
+                                else "vista_transfer+vista_train"),
                            peak_bytes_pred=info["peak_bytes_pred"], peak_bytes=peak_meas,
                            **({"base_layer": TAP_NAMES[cnn][taps[0]], "materialize_s": round(materialize_s, 3)}
                               if args.from_base else {})),

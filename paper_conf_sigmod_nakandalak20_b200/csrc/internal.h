@@ -137,9 +137,21 @@ struct LRResult {
   int64_t n_train = 0, n_test = 0, tp = 0, fp = 0, tn = 0, fn = 0, train_ok = 0;
 };
 typedef void (*allreduce_fn)(double* d_buf, int64_t count, cudaStream_t st, void* user);
+// asynchronous single-rank training: lr_train enqueues everything on st, copies the results into `pinned`
+// (caller-owned pinned host memory of lr_async_bytes(ld, iters)) and records `done`; lr_collect waits for
+// it and assembles the LRResult
+struct LRAsync {
+  void* pinned = nullptr;
+  size_t bytes = 0;
+  cudaEvent_t done = nullptr;
+  int64_t n_rows = 0, n_train = 0;
+  int ld = 0, iters = 0;
+};
+size_t lr_async_bytes(int ld, int iters);
+LRResult lr_collect(const LRAsync& a);
 LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
                   const uint8_t* real_col_mask_host, int iters, int power_iters, double lambda, double alpha,
-                  allreduce_fn allreduce, void* ar_user, cudaStream_t st);
+                  allreduce_fn allreduce, void* ar_user, cudaStream_t st, LRAsync* async = nullptr);
 // fp32 check mode: the same passes over fp32 rows (ld a multiple of 8)
 LRResult lr_train_f32(const float* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
                       const uint8_t* real_col_mask_host, int iters, int power_iters, double lambda, double alpha,

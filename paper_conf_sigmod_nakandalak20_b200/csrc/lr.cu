@@ -921,10 +921,37 @@ static void run_pass(const PassArgs& a, const StreamCfg& c, cudaStream_t st) {
   launch_pass(k, a, c.grid, c.threads + 32, c.smem, coop, st);
 }
 
+size_t lr_async_bytes(int ld, int iters) { return 40 + sizeof(LRState) + (size_t)ld * 8 + (size_t)iters * 8; }
+
+LRResult lr_collect(const LRAsync& a) {
+  LRResult res;
+  VCHECK(cudaEventSynchronize(a.done));
+  const uint8_t* hb = static_cast<const uint8_t*>(a.pinned);
+  unsigned long long hc[5];
+  std::memcpy(hc, hb, 40);
+  LRState hs;
+  std::memcpy(&hs, hb + 40, sizeof(hs));
+  res.w.resize(a.ld);
+  std::memcpy(res.w.data(), hb + 40 + sizeof(LRState), (size_t)a.ld * 8);
+  res.loss.resize(a.iters);
+  if (a.iters) std::memcpy(res.loss.data(), hb + 40 + sizeof(LRState) + (size_t)a.ld * 8, (size_t)a.iters * 8);
+  res.b = hs.b;
+  res.lambda_hat = hs.lambda_hat;
+  res.eta = hs.eta;
+  res.n_train = (int64_t)hs.n_train;
+  res.train_ok = (int64_t)hc[0];
+  res.tp = (int64_t)hc[1];
+  res.fp = (int64_t)hc[2];
+  res.tn = (int64_t)hc[3];
+  res.fn = (int64_t)hc[4];
+  res.n_test = a.n_rows - a.n_train;
+  return res;
+}
+
 template <typename E>
 static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
                               const uint8_t* real_host, int iters, int power_iters, double lambda, double alpha,
-                              allreduce_fn allreduce, void* ar_user, cudaStream_t st) {
+                              allreduce_fn allreduce, void* ar_user, cudaStream_t st, LRAsync* async) {
   LRResult res;
   constexpr int esz = (int)sizeof(E);
   if (ld % 8) fail(1, "lr: ld must be a multiple of 8");
@@ -1101,6 +1128,27 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
     if (n_rows > 0) run_pass<4, E>(e, ce, st);
     prof_end(st, 5, 0, (double)n_rows * ld * esz);
   }
+  if (async) {
+    // asynchronous (world == 1, the Staged plan's LR(k) beside stage k+1): results to the caller's pinned
+    // buffer, scratch freed in stream order, completion event; lr_collect assembles them
+    if (allreduce) fail(1, "lr: asynchronous training is single-rank only");
+    uint8_t* hb = static_cast<uint8_t*>(async->pinned);
+    if (!hb || async->bytes < lr_async_bytes(ld, iters)) fail(1, "lr: pinned result buffer too small");
+    VCHECK(cudaMemcpyAsync(hb, cnt, 5 * 8, cudaMemcpyDeviceToHost, st));
+    VCHECK(cudaMemcpyAsync(hb + 40, dst, sizeof(LRState), cudaMemcpyDeviceToHost, st));
+    VCHECK(cudaMemcpyAsync(hb + 40 + sizeof(LRState), w, (size_t)ld * 8, cudaMemcpyDeviceToHost, st));
+    if (iters)
+      VCHECK(cudaMemcpyAsync(hb + 40 + sizeof(LRState) + (size_t)ld * 8, loss, (size_t)iters * 8,
+                             cudaMemcpyDeviceToHost, st));
+    VCHECK(cudaFreeAsync(scr, st));
+    if (!async->done) VCHECK(cudaEventCreateWithFlags(&async->done, cudaEventDisableTiming));
+    VCHECK(cudaEventRecord(async->done, st));
+    async->n_rows = n_rows;
+    async->n_train = n_train;
+    async->ld = ld;
+    async->iters = iters;
+    return res;
+  }
   // counts -> fp64 for the allreduce (exact below 2^53)
   unsigned long long hc[5];
   VCHECK(cudaMemcpyAsync(hc, cnt, sizeof(hc), cudaMemcpyDeviceToHost, st));
@@ -1136,16 +1184,16 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
 
 LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
                   const uint8_t* real_host, int iters, int power_iters, double lambda, double alpha,
-                  allreduce_fn allreduce, void* ar_user, cudaStream_t st) {
+                  allreduce_fn allreduce, void* ar_user, cudaStream_t st, LRAsync* async) {
   return lr_train_impl<bf16>(MM, y, n_rows, n_train, ld, real_host, iters, power_iters, lambda, alpha, allreduce,
-                             ar_user, st);
+                             ar_user, st, async);
 }
 
 LRResult lr_train_f32(const float* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
                       const uint8_t* real_host, int iters, int power_iters, double lambda, double alpha,
                       allreduce_fn allreduce, void* ar_user, cudaStream_t st) {
   return lr_train_impl<float>(MM, y, n_rows, n_train, ld, real_host, iters, power_iters, lambda, alpha, allreduce,
-                              ar_user, st);
+                              ar_user, st, nullptr);
 }
 
 }  // namespace vista

@@ -3,6 +3,8 @@
 // runs in the kernels of conv_tc.cu / simt_ops.cu / join.cu / lr.cu.
 #include <dlfcn.h>
 
+#include <functional>
+
 #include <algorithm>
 #include <atomic>
 #include <cmath>
@@ -312,6 +314,15 @@ struct vista_ctx {
   uint64_t graph_clock = 0;
   int64_t graph_launches = 0;    // kernels one replay runs (counted at capture)
   int graph_state = 0;           // last transfer: 0 eager, 1 captured, 2 replayed
+  // vista_run: M of layer k on a second stream beside stage k+1 (pinned result buffers per layer)
+  cudaStream_t lr_stream = nullptr;
+  struct LRJobBuf {
+    void* pinned = nullptr;
+    size_t bytes = 0;
+    cudaEvent_t done = nullptr;
+  };
+  std::vector<LRJobBuf> lr_jobs;
+  std::vector<cudaEvent_t> lr_ready;
   DevBuf d_flags;                // device status flags of a transfer (X not bf16-representable)
   int64_t peak_meas = 0, peak_res_meas = 0;  // measured peak device bytes of the last transfer
   std::unique_ptr<Profiler> prof;
@@ -361,6 +372,14 @@ struct vista_ctx {
     for (auto& g : graphs)
       if (g.exec) cudaGraphExecDestroy(g.exec);
     if (cap_stream) cudaStreamDestroy(cap_stream);
+    if (lr_stream) cudaStreamSynchronize(lr_stream);
+    for (auto& j : lr_jobs) {
+      if (j.pinned) cudaFreeHost(j.pinned);
+      if (j.done) cudaEventDestroy(j.done);
+    }
+    for (cudaEvent_t e : lr_ready)
+      if (e) cudaEventDestroy(e);
+    if (lr_stream) cudaStreamDestroy(lr_stream);
     if (own_stream && stream) cudaStreamDestroy(stream);
     for (cudaEvent_t e : px_ready) cudaEventDestroy(e);
     if (px_free) cudaEventDestroy(px_free);
@@ -1068,8 +1087,11 @@ VISTA_API vista_status vista_plan_info(const vista_ctx* c, vista_plan_info_t* o)
 // Body of vista_transfer and vista_transfer_from_base.  base == nullptr: from pixels.  base != nullptr:
 // the CNN starts at the stored activation of the first requested layer (App. B):
 // block t0 = taps[0] is not run, A_t0 = base, and blocks t0+1 .. t_max are partial inference from it.
+// on_concat (vista_run): called right after layer k's MM_k is concatenated on the compute stream, while
+// the CNN continues with stage k+1 (Staged, unchunked); the CNN part then runs without a CUDA graph.
 static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base, const int64_t* image_keys,
-                          const float* structured, const int64_t* str_keys, const uint8_t* labels) {
+                          const float* structured, const int64_t* str_keys, const uint8_t* labels,
+                          const std::function<void(int)>* on_concat = nullptr) {
   {
     if (c->n_img > 0 && !image_keys) fail(1, "image_keys is NULL");
     if (c->n_img > 0 && !images && !base) fail(1, "images / base is NULL");
@@ -1131,7 +1153,9 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
       c->F[t]->ensure((size_t)c->n_img * S[t].d_tap * c->esz + 16);
       c->feat[t] = c->F[t]->p;
     }
+    std::vector<char> concat_done(c->taps.size(), 0);
     auto concat_layer = [&](int k) {
+      concat_done[k] = 1;
       const int t = c->taps[k];
       const int ld = ld_of(c, k);
       c->MM[k]->ensure((size_t)std::max<int64_t>(c->n_pairs, 1) * ld * c->esz);
@@ -1231,6 +1255,10 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
               launch_tap_finalize(tapf, (int64_t)nc * S[t].d_tap, (bf16*)Ft, st);
             else
               tap_any(c, At, nc, S[t], Ft);
+            if (on_concat && !chunked) {  // S4 + hand layer k to M while stage k+1 runs (Fig 5E)
+              concat_layer(k);
+              (*on_concat)(k);
+            }
           }
         }
       }
@@ -1242,7 +1270,7 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
                                   !(getenv("VISTA_CONV_DBG") && atoi(getenv("VISTA_CONV_DBG")) != 0);
     const bool pageable = (host_px && !is_pinned_host(images)) || (host_base && !is_pinned_host(base));
     c->graph_state = 0;
-    if (graphs_on && !g_prof && c->n_img > 0 && !pageable && c->graph_failed < 2) {
+    if (graphs_on && !g_prof && !on_concat && c->n_img > 0 && !pageable && c->graph_failed < 2) {
       if (host_px && !c->copy_stream) {  // created outside any capture
         VCHECK(cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking));
         VCHECK(cudaEventCreateWithFlags(&c->px_free, cudaEventDisableTiming));
@@ -1309,8 +1337,12 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
     } else {
       cnn_part();
     }
-    // ---- S4 concat (Eq. 4) of every layer ----
-    for (size_t k = 0; k < c->taps.size(); ++k) concat_layer((int)k);
+    // ---- S4 concat (Eq. 4) of every layer (not yet handed to M) ----
+    for (size_t k = 0; k < c->taps.size(); ++k)
+      if (!concat_done[k]) {
+        concat_layer((int)k);
+        if (on_concat) (*on_concat)((int)k);
+      }
     int flags[4] = {0, 0, 0, 0};
     VCHECK(cudaMemcpyAsync(flags, c->d_flags.p, 16, cudaMemcpyDeviceToHost, st));
     VCHECK(cudaStreamSynchronize(st));
@@ -1419,6 +1451,56 @@ VISTA_API vista_status vista_features(const vista_ctx* c, int32_t k, vista_buffe
   return VISTA_OK;
 }
 
+// S5 on layer k (helpers of vista_train / vista_run)
+static std::vector<uint8_t> real_cols(const vista_ctx* c, int k) {
+  const int d_l = c->net.stages[c->taps[k]].d_tap;
+  std::vector<uint8_t> real(ld_of(c, k), 0);
+  for (int j = 0; j < c->d_s; ++j) real[j] = 1;
+  for (int j = 0; j < d_l; ++j) real[c->ds_pad + j] = 1;
+  return real;
+}
+
+static LRResult train_layer(vista_ctx* c, int k, cudaStream_t st, LRAsync* async) {
+  const int ld = ld_of(c, k);
+  const std::vector<uint8_t> real = real_cols(c, k);
+  allreduce_fn ar = nullptr;
+  void* ar_user = nullptr;
+  if (c->sys.world > 1) {
+    ar = c->nccl_comm ? nccl_allreduce_f64 : hook_allreduce_f64;
+    ar_user = c->nccl_comm ? c->nccl_comm : (void*)&c->hook;
+  }
+  return c->f32 ? lr_train_f32((const float*)c->MM[k]->p, (const uint8_t*)c->Y[k]->p, c->n_pairs, c->n_train, ld,
+                               real.data(), c->lr.iters, c->lr.power_iters, c->lr.lambda, c->lr.alpha, ar, ar_user, st)
+                : lr_train((const bf16*)c->MM[k]->p, (const uint8_t*)c->Y[k]->p, c->n_pairs, c->n_train, ld,
+                           real.data(), c->lr.iters, c->lr.power_iters, c->lr.lambda, c->lr.alpha, ar, ar_user, st,
+                           async);
+}
+
+static void train_outputs(const vista_ctx* c, int k, const LRResult& r, double* weights_out, vista_metrics* m) {
+  const int d_l = c->net.stages[c->taps[k]].d_tap;
+  if (weights_out) {
+    for (int j = 0; j < c->d_s; ++j) weights_out[j] = r.w[j];
+    for (int j = 0; j < d_l; ++j) weights_out[c->d_s + j] = r.w[c->ds_pad + j];
+    weights_out[c->d_s + d_l] = r.b;
+  }
+  if (m) {
+    std::memset(m, 0, sizeof(*m));
+    for (int i = 0; i < (int)r.loss.size() && i < 64; ++i) m->loss[i] = r.loss[i];
+    m->lambda_hat = r.lambda_hat;
+    m->eta = r.eta;
+    m->n_train = r.n_train;
+    m->n_test = r.n_test;
+    m->tp = r.tp;
+    m->fp = r.fp;
+    m->tn = r.tn;
+    m->fn = r.fn;
+    m->train_acc = r.n_train ? 100.0 * r.train_ok / r.n_train : 0.0;
+    m->test_acc = r.n_test ? 100.0 * (r.tp + r.tn) / r.n_test : 0.0;
+    const int64_t den = 2 * r.tp + r.fp + r.fn;
+    m->test_f1 = den ? 100.0 * 2.0 * r.tp / den : 0.0;
+  }
+}
+
 VISTA_API vista_status vista_train(vista_ctx* c, int32_t k, double* weights_out, vista_metrics* m) {
   if (!c) return VISTA_ERR_INVALID_ARG;
   if (!c->transferred) {
@@ -1428,46 +1510,63 @@ VISTA_API vista_status vista_train(vista_ctx* c, int32_t k, double* weights_out,
   return guarded(c, [&] {
     if (k < 0 || k >= (int)c->taps.size()) fail(1, "layer index out of range");
     VCHECK(cudaSetDevice(c->sys.device));
-    const int t = c->taps[k];
-    const int d_l = c->net.stages[t].d_tap;
-    const int ld = ld_of(c, k);
-    std::vector<uint8_t> real(ld, 0);
-    for (int j = 0; j < c->d_s; ++j) real[j] = 1;
-    for (int j = 0; j < d_l; ++j) real[c->ds_pad + j] = 1;
-    allreduce_fn ar = nullptr;
-    void* ar_user = nullptr;
-    if (c->sys.world > 1) {
-      ar = c->nccl_comm ? nccl_allreduce_f64 : hook_allreduce_f64;
-      ar_user = c->nccl_comm ? c->nccl_comm : (void*)&c->hook;
-    }
-    LRResult r = c->f32 ? lr_train_f32((const float*)c->MM[k]->p, (const uint8_t*)c->Y[k]->p, c->n_pairs,
-                                       c->n_train, ld, real.data(), c->lr.iters, c->lr.power_iters, c->lr.lambda,
-                                       c->lr.alpha, ar, ar_user, c->stream)
-                        : lr_train((const bf16*)c->MM[k]->p, (const uint8_t*)c->Y[k]->p, c->n_pairs, c->n_train,
-                                   ld, real.data(), c->lr.iters, c->lr.power_iters, c->lr.lambda, c->lr.alpha, ar,
-                                   ar_user, c->stream);
+    const LRResult r = train_layer(c, k, c->stream, nullptr);
     if (g_prof) g_prof->flush();
-    if (weights_out) {
-      for (int j = 0; j < c->d_s; ++j) weights_out[j] = r.w[j];
-      for (int j = 0; j < d_l; ++j) weights_out[c->d_s + j] = r.w[c->ds_pad + j];
-      weights_out[c->d_s + d_l] = r.b;
+    train_outputs(c, k, r, weights_out, m);
+  });
+}
+
+// The whole Staged plan (Fig 5E): vista_transfer + vista_train(k) for every layer, with M of
+// layer k (S5) enqueued on a second stream as soon as MM_k exists, beside the partial inference of stage
+// k+1 (S6).  One rank: asynchronous LR with results collected at the end; world > 1, the fp32 check mode
+// and chunked plans train after the transfer, layer by layer (their collectives / host steps are ordered).
+VISTA_API vista_status vista_run(vista_ctx* c, const uint8_t* images, const int64_t* image_keys,
+                                 const float* structured, const int64_t* str_keys, const uint8_t* labels,
+                                 double* const* weights_out, vista_metrics* out) {
+  if (!c) return VISTA_ERR_INVALID_ARG;
+  return guarded(c, [&] {
+    const int L = (int)c->taps.size();
+    static const bool overlap_on = !(getenv("VISTA_OVERLAP") && getenv("VISTA_OVERLAP")[0] == '0');
+    const bool overlap = overlap_on && c->sys.world == 1 && !c->f32;
+    if (!overlap) {
+      transfer_body(c, images, nullptr, image_keys, structured, str_keys, labels);
+      for (int k = 0; k < L; ++k) {
+        const LRResult r = train_layer(c, k, c->stream, nullptr);
+        train_outputs(c, k, r, weights_out ? weights_out[k] : nullptr, out ? out + k : nullptr);
+      }
+      if (g_prof) g_prof->flush();
+      return;
     }
-    if (m) {
-      std::memset(m, 0, sizeof(*m));
-      for (int i = 0; i < (int)r.loss.size() && i < 64; ++i) m->loss[i] = r.loss[i];
-      m->lambda_hat = r.lambda_hat;
-      m->eta = r.eta;
-      m->n_train = r.n_train;
-      m->n_test = r.n_test;
-      m->tp = r.tp;
-      m->fp = r.fp;
-      m->tn = r.tn;
-      m->fn = r.fn;
-      m->train_acc = r.n_train ? 100.0 * r.train_ok / r.n_train : 0.0;
-      m->test_acc = r.n_test ? 100.0 * (r.tp + r.tn) / r.n_test : 0.0;
-      const int64_t den = 2 * r.tp + r.fp + r.fn;
-      m->test_f1 = den ? 100.0 * 2.0 * r.tp / den : 0.0;
+    if (!c->lr_stream) VCHECK(cudaStreamCreateWithFlags(&c->lr_stream, cudaStreamNonBlocking));
+    c->lr_jobs.resize(L);
+    c->lr_ready.resize(L, nullptr);
+    for (int k = 0; k < L; ++k) {
+      vista_ctx::LRJobBuf& jb = c->lr_jobs[k];
+      const size_t need = lr_async_bytes(ld_of(c, k), c->lr.iters);
+      if (jb.bytes < need) {
+        if (jb.pinned) VCHECK(cudaFreeHost(jb.pinned));
+        jb.pinned = nullptr;
+        VCHECK(cudaMallocHost(&jb.pinned, need));
+        jb.bytes = need;
+      }
+      if (!c->lr_ready[k]) VCHECK(cudaEventCreateWithFlags(&c->lr_ready[k], cudaEventDisableTiming));
     }
+    std::vector<LRAsync> jobs(L);
+    const std::function<void(int)> on_concat = [&](int k) {
+      VCHECK(cudaEventRecord(c->lr_ready[k], c->stream));
+      VCHECK(cudaStreamWaitEvent(c->lr_stream, c->lr_ready[k], 0));
+      jobs[k].pinned = c->lr_jobs[k].pinned;
+      jobs[k].bytes = c->lr_jobs[k].bytes;
+      jobs[k].done = c->lr_jobs[k].done;
+      train_layer(c, k, c->lr_stream, &jobs[k]);
+      c->lr_jobs[k].done = jobs[k].done;  // (created on first use)
+    };
+    transfer_body(c, images, nullptr, image_keys, structured, str_keys, labels, &on_concat);
+    for (int k = 0; k < L; ++k) {
+      const LRResult r = lr_collect(jobs[k]);
+      train_outputs(c, k, r, weights_out ? weights_out[k] : nullptr, out ? out + k : nullptr);
+    }
+    if (g_prof) g_prof->flush();
   });
 }
 

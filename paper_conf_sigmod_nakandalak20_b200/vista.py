@@ -98,6 +98,7 @@ def lib():
         L.vista_materialize.argtypes = [_vp, _vp, _vp]
         L.vista_transfer_from_base.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp]
         L.vista_train.argtypes = [_vp, _i32, _vp, ctypes.POINTER(Metrics)]
+        L.vista_run.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp]
         L.vista_destroy.argtypes = [_vp]
         L.vista_destroy.restype = None
         L.vista_shard_range.argtypes = [_i64, _i32, _i32, ctypes.POINTER(_i64), ctypes.POINTER(_i64)]
@@ -366,6 +367,23 @@ class Vista:
                    test_acc=m.test_acc, test_f1=m.test_f1, n_train=m.n_train, n_test=m.n_test, tp=m.tp, fp=m.fp,
                    tn=m.tn, fn=m.fn)
         return w[:-1], float(w[-1]), met
+
+    def run(self, images, image_keys, structured, str_keys, labels, d_totals, want_weights=True):
+        """vista_run: transfer + M of every layer (M(k) beside stage k+1); returns [(w, b, metrics)] per layer."""
+        L = len(d_totals)
+        ws = [np.zeros(d + 1, dtype=np.float64) for d in d_totals] if want_weights else None
+        ptrs = (ctypes.c_void_p * L)(*[w.ctypes.data for w in ws]) if want_weights else None
+        ms = (Metrics * L)()
+        _check(lib().vista_run(self.ctx, _ptr(images), _ptr(image_keys), _ptr(structured), _ptr(str_keys),
+                               _ptr(labels), ptrs, ms), self.ctx)
+        out = []
+        for k in range(L):
+            m = ms[k]
+            met = dict(loss=list(m.loss[:64]), lambda_hat=m.lambda_hat, eta=m.eta, train_acc=m.train_acc,
+                       test_acc=m.test_acc, test_f1=m.test_f1, n_train=m.n_train, n_test=m.n_test, tp=m.tp,
+                       fp=m.fp, tn=m.tn, fn=m.fn)
+            out.append((ws[k][:-1], float(ws[k][-1]), met) if want_weights else (None, None, met))
+        return out
 
     def train_mlp(self, k, d_total, iters=10, lr=0.01, seed=0, hidden=1024, want_weights=True):
         """3-layer MLP (reading R30) on layer k; returns (params dict or None, metrics)."""

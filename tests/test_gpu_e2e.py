@@ -394,3 +394,27 @@ def test_planner_prediction_bounds_measured_peak():
     assert info["chunk_images"] < n
     assert info["peak_bytes_pred"] <= budget
     assert 0 < info["peak_bytes_meas"] <= info["peak_bytes_pred"], info
+
+
+@pytest.mark.parametrize("overlap", ["1", "0"])
+def test_run_equals_transfer_then_train(monkeypatch, overlap):
+    # vista_run (S6: M of layer k on a second stream beside stage k+1) gives the same bits as vista_transfer
+    # followed by vista_train(k) for every k
+    monkeypatch.setenv("VISTA_OVERLAP", overlap)
+    tab = gen.make_tables(40, 16)
+    taps = [0, 1, 2, 3, 4]
+    ref = run_gpu(2, taps, tab, 16, iters=3)
+    d = [16 + ref.features(k)["d_l"] for k in range(5)]
+    want = [ref.train(k, d[k]) for k in range(5)]
+    mm = [ref.features(k)["mm"].view(torch.int16).cpu().clone() for k in range(5)]
+    ref.close()
+    v = Vista(2, layers=taps, n_str_rows=len(tab.str_keys), d_s=16, n_images_local=40, iters=3, split_seed=SPLIT,
+              weight_seed=WSEED)
+    for _ in range(2):  # repeated runs reuse the pinned result buffers and events
+        got = v.run(tab.images, tab.img_keys, tab.X, tab.str_keys, tab.labels, d)
+        for k in range(5):
+            np.testing.assert_array_equal(got[k][0], want[k][0])
+            assert got[k][1] == want[k][1]
+            assert got[k][2]["loss"][:3] == want[k][2]["loss"][:3] and got[k][2]["tp"] == want[k][2]["tp"]
+            assert torch.equal(mm[k], v.features(k)["mm"].view(torch.int16).cpu())
+    v.close()

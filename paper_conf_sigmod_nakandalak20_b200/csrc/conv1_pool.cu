@@ -28,16 +28,17 @@ constexpr int kHo = 114;           // conv1 output rows / cols (227 + 6 - 7) / 2
 constexpr int kHin = 117;          // space-to-depth input rows (kS2dHW)
 constexpr int kPo = 56;            // pool1 output (114 - 3) / 2 + 1
 constexpr int kCo = 64;            // conv1 channels
-constexpr int kSA = 8;             // input-row ring slots
+constexpr int kSA = 6;             // input-row ring slots (rows 24 ahead are prefetched into L2)
 constexpr int kNAcc = 8;           // TMEM accumulators (64 columns each; the classic issue order uses 4)
 constexpr int kRowBytes = 128 * 128;  // one A slot: 128 pixel rows x 64 bf16 (128B-swizzled)
 constexpr int kBBytes = 4 * 64 * 128;  // 4 k-blocks x 64 output channels x 64 bf16
 constexpr int kCrowBytes = 128 * 128;  // conv row: 128 pixels x 64 channels bf16
+constexpr int kCrowBufs = 4;           // staged conv rows (two rows per epilogue step, double-buffered)
 constexpr int kEpiWarp0 = 2, kEpiWarps = 8, kEpiThreads = kEpiWarps * 32;
 constexpr int kThreads = (kEpiWarp0 + kEpiWarps) * 32;
 constexpr int kItems = kPo * 8;    // (pooled column, 8-channel chunk) items per pooled row
 constexpr int kOffB = 0, kOffA = kOffB + kBBytes, kOffCrow = kOffA + kSA * kRowBytes,
-              kOffSS = kOffCrow + 2 * kCrowBytes, kOffBar = kOffSS + 2 * kCo * 4;
+              kOffSS = kOffCrow + kCrowBufs * kCrowBytes, kOffBar = kOffSS + 2 * kCo * 4;
 constexpr int kSmem = kOffBar + (2 * kSA + 2 * kNAcc + 2) * 8 + 1024;
 
 struct PoolParams {
@@ -223,9 +224,10 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int wo = q * 32 + lane;              // conv output column (M row of the tile)
     const int i0 = et, i1 = et + kEpiThreads;  // this thread's pooling items
     uint32_t it = 0;
-    // Software-pipelined over conv rows: the TMEM load of row ho is issued before the pooling of row ho - 1
-    // (which reads the other conv-row buffer), so its latency and the accumulator zeroing hide behind that
-    // work; one named barrier per row separates "row ho staged" from "row ho pooled".
+    // Two conv rows per step, software-pipelined: the TMEM loads of rows ho, ho + 1 are issued before the
+    // pooling of rows ho - 2, ho - 1 (staged in the other two of four conv-row buffers), so their latency and
+    // the accumulator zeroing hide behind that work; one named barrier per two rows separates "staged" from
+    // "pooled" (the per-row latency chain, not the arithmetic, bounded the one-row loop: ~0.8 us per row).
     for (int n = blockIdx.x; n < p.N; n += gridDim.x) {
       uint4 vb0[2], vb1[2];  // running vertical max of the open pooled rows (even / odd i), per item
 #pragma unroll
@@ -234,7 +236,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       // conv row ho (staged in buffer ho & 1) -> pooled rows: even ho closes i = ho/2 - 1 and opens i = ho/2;
       // odd ho extends (ho-1)/2
       auto pool_row = [&](const int ho) {
-        const uint32_t cbase = sC + (ho & 1) * kCrowBytes;
+        const uint32_t cbase = sC + (ho & 3) * kCrowBytes;
 #pragma unroll
         for (int u = 0; u < 2; ++u) {
           const int item = u == 0 ? i0 : i1;
@@ -264,33 +266,47 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
         }
       };
-      for (int ho = 0; ho < kHo; ++ho, ++it) {
-        const uint32_t acc = it % kNAcc;
-        mbar_wait(&tfull[acc], (it / kNAcc) & 1);
+      static_assert(kHo % 2 == 0, "two conv rows per step");
+      for (int ho = 0; ho < kHo; ho += 2, it += 2) {
+        const uint32_t acc0 = it % kNAcc, acc1 = (it + 1) % kNAcc;
+        uint32_t v0[32], v1[32];
+        mbar_wait(&tfull[acc0], (it / kNAcc) & 1);
         tc_fence_after();
-        uint32_t v[32];
-        tmem_ld_32x32b_x32(tmem_base + acc * kCo + half * 32 + ((uint32_t)(q * 32) << 16), v);
-        if (ho > 0) pool_row(ho - 1);  // overlaps the TMEM load
-        tc_wait_ld_regs(v);
+        tmem_ld_32x32b_x32(tmem_base + acc0 * kCo + half * 32 + ((uint32_t)(q * 32) << 16), v0);
+        mbar_wait(&tfull[acc1], ((it + 1) / kNAcc) & 1);
+        tc_fence_after();
+        tmem_ld_32x32b_x32(tmem_base + acc1 * kCo + half * 32 + ((uint32_t)(q * 32) << 16), v1);
+        if (ho > 0) {  // overlaps the TMEM loads
+          pool_row(ho - 2);
+          pool_row(ho - 1);
+        }
+        tc_wait_ld_regs(v0);
+        tc_wait_ld_regs(v1);
         if (p.irow) {  // input-row-major issue accumulates into zeroed slots
-          tmem_zero_32x32b_x32(tmem_base + acc * kCo + half * 32 + ((uint32_t)(q * 32) << 16));
+          tmem_zero_32x32b_x32(tmem_base + acc0 * kCo + half * 32 + ((uint32_t)(q * 32) << 16));
+          tmem_zero_32x32b_x32(tmem_base + acc1 * kCo + half * 32 + ((uint32_t)(q * 32) << 16));
           tc_wait_st();
         }
         tc_fence_before();
         __syncwarp();
-        if (lane == 0) mbar_arrive(&tempty[acc]);
-        const uint32_t crow = sC + (ho & 1) * kCrowBytes + wo * 128;
+        if (lane == 0) {
+          mbar_arrive(&tempty[acc0]);
+          mbar_arrive(&tempty[acc1]);
+        }
         if (wo < kHo) {
 #pragma unroll
           for (int c4 = 0; c4 < 4; ++c4) {  // 8 channels per 16-byte chunk
             const int ch0 = half * 32 + c4 * 8;
-            const uint4 o = epi8(v + c4 * 8, ss + ch0, ss + kCo + ch0, make_uint4(0, 0, 0, 0), false, true);
-            const uint32_t chunk = (uint32_t)(half * 4 + c4);
-            sts128(crow + ((chunk ^ (uint32_t)(wo & 7)) << 4), o);
+            const uint32_t sw = (((uint32_t)(half * 4 + c4)) ^ (uint32_t)(wo & 7)) << 4;
+            sts128(sC + (ho & 3) * kCrowBytes + wo * 128 + sw,
+                   epi8(v0 + c4 * 8, ss + ch0, ss + kCo + ch0, make_uint4(0, 0, 0, 0), false, true));
+            sts128(sC + ((ho + 1) & 3) * kCrowBytes + wo * 128 + sw,
+                   epi8(v1 + c4 * 8, ss + ch0, ss + kCo + ch0, make_uint4(0, 0, 0, 0), false, true));
           }
         }
         named_bar_sync(1, kEpiThreads);
       }
+      pool_row(kHo - 2);
       pool_row(kHo - 1);
     }
   }

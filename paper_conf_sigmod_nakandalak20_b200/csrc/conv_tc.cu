@@ -1470,7 +1470,10 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
     ty = tr = L.tmap_w;  // unused
   }
   const double flops = 2.0 * (double)M * L.Cout * L.K_alg;  // algorithmic (unpadded) MACs x 2
-  const double bytes = 2.0 * ((double)N * H * W * L.Cin + (double)M * L.Cout * (res ? 2 : 1) + (double)L.Cout * L.Kp);
+  // algorithmic bytes: the input once (a strided 1x1 conv reads only its sampled pixels: whole 16-byte-aligned
+  // channel runs, so no other line is touched), the output, the residual, the weights
+  const double in_px = (L.R == 1 && L.S == 1 && L.pad == 0) ? (double)M : (double)N * H * W;
+  const double bytes = 2.0 * (in_px * L.Cin + (double)M * L.Cout * (res ? 2 : 1) + (double)L.Cout * L.Kp);
   // resident weights (see Cfg): 3x3 halo convs with Cout = 64 (9 k-blocks of 8 KB) and 1x1 TMA convs with
   // K <= 256 and BN <= 128 (<= 4 k-blocks); one N tile per CTA needs groups == 1 and n_nt <= the grid
   int rkb = 0;

@@ -75,6 +75,12 @@ struct ConvParams {
   // rank r takes M tile 2 * pair_m + r) in lockstep, and each CTA TMA-loads half of every weight (B) k-block
   // and multicasts it to both, halving the per-SM L2 -> shared-memory weight traffic of streamed-B layers
   int mc;
+  // cg2 = 1 (with mc = 1, A_HALO padded-grid tiles): the CTA pair runs ONE tcgen05.mma.cta_group::2 over
+  // M = 256 (rank r's 128 rows in its own shared memory and TMEM); the pair tile is the same position in two
+  // consecutive images (rank r: image 2j + r), so both halos sit at the same offsets; each CTA loads half of
+  // every weight k-block (B's N rows split between the pair): per-SM operand reads 4 KB + BN/2 * 32 B per
+  // MMA instead of 4 KB + BN * 32 B, and half the weight bytes written into each CTA's shared memory
+  int cg2;
   int segs;  // A_ROWVIEW: 128-pixel segments per output row (1 unless Wo > 128); A_HALO + hseg: segments
   // A_HALO row-segment tiles (hseg = 1, rows too wide for the padded-grid halo): tile = (image, output row,
   // segment of seg_w <= 126 columns); the halo is 3 input rows x (seg_w + 2) padded columns (Wp = seg_w + 2)
@@ -105,12 +111,12 @@ constexpr int kLag = 2;        // cp.async groups in flight before a stage is pu
 // all, and three halo buffers).  Measured motivation: the per-SM L2 -> smem ingest is bounded by the
 // bytes in flight / L2 latency, and re-loading the weights per tile doubled (1x1) or tripled (halo 3x3,
 // Cout = 64) the bytes each tile needs.
-template <int BN, bool TMA_EPI, int NB, bool HALO = false, int RKB = 0>
+template <int BN, bool TMA_EPI, int NB, bool HALO = false, int RKB = 0, bool CG2 = false>
 struct Cfg {
   static constexpr int kHB = HALO ? (RKB ? 3 : 2) : 0;  // halo buffers (A_HALO)
   static constexpr int kHaloBytes = kHB * halo_half_bytes(BN);
   static constexpr int kABytes = HALO ? 0 : BM * BK * 2;  // 16 KB per stage (A_HALO: A lives in the halo)
-  static constexpr int kBBytes = BN * BK * 2;
+  static constexpr int kBBytes = (CG2 ? BN / 2 : BN) * BK * 2;  // CTA pair: this CTA's half of the N rows
   static constexpr int kResBytes = RKB * kBBytes;          // resident weights
   static constexpr int kStageBytes = kABytes + (RKB ? 0 : kBBytes);
   static constexpr int kOutBufs = TMA_EPI ? NB : 0;
@@ -144,6 +150,13 @@ struct Cfg {
 // tile -> (first row m0, N-tile index nt, group g); N-tiles of one M-tile are adjacent so
 // the 148 CTAs working at any moment share A rows in L2
 __device__ __forceinline__ void decode_tile(const ConvParams& p, int tile, int& m0, int& nt, int& g) {
+  if (p.cg2) {  // pair tile (j, t) -> M tile t of image 2j + rank (rank 1 past the last image: phantom)
+    const int j = tile / p.mt_per_img, t = tile - j * p.mt_per_img;
+    m0 = ((2 * j + (int)(blockIdx.x & 1)) * p.mt_per_img + t) * BM;
+    nt = 0;
+    g = 0;
+    return;
+  }
   if (p.mc) {  // pair tile -> this CTA's M tile (an odd last M tile leaves rank 1 a phantom tile past M)
     const int pm = tile / p.n_nt;
     nt = tile - pm * p.n_nt;
@@ -177,12 +190,13 @@ __device__ __forceinline__ void epi_math_f32(const uint32_t* v, const float* scv
   reinterpret_cast<float4*>(out)[1] = make_float4(f[4], f[5], f[6], f[7]);
 }
 
-template <int BN, int AMODE, bool TMA_EPI, int NB, int RKB>
+template <int BN, int AMODE, bool TMA_EPI, int NB, int RKB, bool CG2 = false>
 __global__ void __launch_bounds__(kThreads, 1)
     conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__ CUtensorMap tmap_a,
                    const __grid_constant__ CUtensorMap tmap_y, const __grid_constant__ CUtensorMap tmap_r,
                    const ConvParams p) {
-  using C = Cfg<BN, TMA_EPI, NB, AMODE == A_HALO, RKB>;
+  using C = Cfg<BN, TMA_EPI, NB, AMODE == A_HALO, RKB, CG2>;
+  static_assert(!CG2 || (AMODE == A_HALO && RKB == 0 && !TMA_EPI), "CTA-pair MMA: streamed-weight halo path only");
   constexpr int S = C::kStages;
   constexpr bool BRES = RKB > 0;
   constexpr int HB = C::kHB > 0 ? C::kHB : 1;
@@ -226,7 +240,8 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     for (int i = 0; i < NACC; ++i) {
       mbar_init(&tfull[i], 1);
-      mbar_init(&tempty[i], SPLIT ? kEpiWarps / 2 : kEpiWarps);
+      // CTA pair: the leader's MMA reuses an accumulator once BOTH CTAs' epilogues drained it
+      mbar_init(&tempty[i], (SPLIT ? kEpiWarps / 2 : kEpiWarps) * (CG2 ? 2 : 1));
     }
     for (int i = 0; i < 4; ++i) mbar_init(&rbar[i], 1);
     for (int i = 0; i < 3; ++i) {
@@ -239,7 +254,11 @@ __global__ void __launch_bounds__(kThreads, 1)
     if (a_by_tma(AMODE)) tma_prefetch(&tmap_a);
     if (TMA_EPI) tma_prefetch(&tmap_y);
   }
-  if (warp == 4) tmem_alloc(tmem_slot, C::kTmemCols);
+  if constexpr (CG2) cluster_sync_all();  // both CTAs of the pair enter the pair allocation together
+  if (warp == 4) {
+    if constexpr (CG2) tmem_alloc_cg2(tmem_slot, C::kTmemCols);
+    else tmem_alloc(tmem_slot, C::kTmemCols);
+  }
   tc_fence_before();
   __syncthreads();
   if (p.mc) cluster_sync_all();  // the partner's barriers are initialised before any multicast reaches them
@@ -311,6 +330,15 @@ __global__ void __launch_bounds__(kThreads, 1)
             const int stage = gk % S2;
             if (gk >= (uint32_t)S2) mbar_wait(&empty[stage], ((gk / S2) - 1) & 1);
             const int two = kb + 1 < p.nkb ? 2 : 1;
+            if constexpr (CG2) {
+              // CTA pair: this CTA's half of the N rows into its own stage; both halves complete on the leader's
+              // barrier, which the leader arms for both
+              const uint32_t fl = mapa_u32(smem_u32(&full[stage]), 0);
+              if (crank == 0) mbar_arrive_expect_tx(&full[stage], 2 * two * C::kBBytes);
+              for (int h = 0; h < two; ++h)
+                tma_load_2d_cg2(sB + (2 * stage + h) * C::kBBytes, &tmap_w, (kb + h) * BK, (int)crank * (BN / 2), fl);
+              continue;
+            }
             mbar_arrive_expect_tx(&full[stage], two * C::kBBytes);
             for (int h = 0; h < two; ++h) {
               if (p.mc)  // this CTA's half of the k-block rows, multicast to the pair
@@ -341,6 +369,13 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
           const uint32_t hb = it % HB;
           if (it >= (uint32_t)HB) mbar_wait(&hempty[hb], ((it / HB) - 1) & 1);
+          if constexpr (CG2) {  // own halo, completing on the leader's barrier (armed by the leader for both)
+            const uint32_t hl = mapa_u32(smem_u32(&hfull[hb]), 0);
+            if (crank == 0) mbar_arrive_expect_tx(&hfull[hb], 2 * box_bytes * p.cblocks);
+            for (int cb = 0; cb < p.cblocks; ++cb)
+              tma_load_4d_cg2(sH + hb * halo_half_bytes(BN) + cb * p.hsz, &tmap_a, cb * BK, col0, prow0 - 1, nimg, hl);
+            continue;
+          }
           if ((p.dbg & 1) && it >= (uint32_t)HB) {
             mbar_arrive(&hfull[hb]);
           } else {
@@ -528,8 +563,9 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
   } else if (warp == 4) {
     // ======================= MMA issuer (whole warp, one elected lane issues) =======================
-    {
-      constexpr uint32_t idesc = umma_idesc_bf16(BM, BN);
+    // (CTA pair: the leader issues for both; the peer's MMA warp only allocated the pair's TMEM)
+    if (!CG2 || crank == 0) {
+      constexpr uint32_t idesc = umma_idesc_bf16(CG2 ? 2 * BM : BM, BN);
       uint32_t gk = 0, it = 0;
       long long c_te = 0, c_dec = 0, c_hf = 0, c_iss = 0, tA = 0, tB = 0;
       const bool prof_mma = (p.dbg & 8) && lane == 0;
@@ -594,9 +630,9 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       int hmod = 0, hstep = 0;  // A_HALO: tile index mod mt_per_img and its per-iteration step
       if constexpr (AMODE == A_HALO) {
-        // (multicast pairs: M tile = 2 * pair tile + rank)
-        hmod = (p.mc ? 2 * cta0 + (int)crank : cta0) % p.mt_per_img;
-        hstep = (p.mc ? 2 * ncta : ncta) % p.mt_per_img;
+        // (multicast pairs: M tile = 2 * pair tile + rank; CTA pair: pair tile = position, same for both)
+        hmod = (p.mc && !CG2 ? 2 * cta0 + (int)crank : cta0) % p.mt_per_img;
+        hstep = (p.mc && !CG2 ? 2 * ncta : ncta) % p.mt_per_img;
       }
       if constexpr (!(AMODE == A_HALO && BRES))
       for (int tile = cta0; tile < p.n_tiles; tile += ncta, ++it) {
@@ -644,6 +680,22 @@ __global__ void __launch_bounds__(kThreads, 1)
             mbar_wait(&full[stage], (gk / S2) & 1);
             const uint32_t b = blo0 + (uint32_t)(2 * stage) * (uint32_t)(C::kBBytes >> 4);
             const uint32_t a = alo + (uint32_t)p.koff[kb];
+            if constexpr (CG2) {  // one pair MMA per K step: M = 256 over both CTAs' halos
+              tc_mma_bf16_lo_warp_cg2(tacc, a, b, idesc, kb != 0 ? 1u : 0u);
+              tc_mma_bf16_lo_warp_cg2(tacc, a + 2, b + 2, idesc, 1u);
+              tc_mma_bf16_lo_warp_cg2(tacc, a + 4, b + 4, idesc, 1u);
+              tc_mma_bf16_lo_warp_cg2(tacc, a + 6, b + 6, idesc, 1u);
+              if (kb + 1 < p.nkb) {
+                const uint32_t a1 = alo + (uint32_t)p.koff[kb + 1];
+                const uint32_t b1 = b + (uint32_t)(C::kBBytes >> 4);
+                tc_mma_bf16_lo_warp_cg2(tacc, a1, b1, idesc, 1u);
+                tc_mma_bf16_lo_warp_cg2(tacc, a1 + 2, b1 + 2, idesc, 1u);
+                tc_mma_bf16_lo_warp_cg2(tacc, a1 + 4, b1 + 4, idesc, 1u);
+                tc_mma_bf16_lo_warp_cg2(tacc, a1 + 6, b1 + 6, idesc, 1u);
+              }
+              tc_commit_cg2_warp(&empty[stage], (uint16_t)3);  // both CTAs' stages are free
+              continue;
+            }
             tc_mma_bf16_lo_warp(tacc, a, b, idesc, kb != 0 ? 1u : 0u);
             tc_mma_bf16_lo_warp(tacc, a + 2, b + 2, idesc, 1u);
             tc_mma_bf16_lo_warp(tacc, a + 4, b + 4, idesc, 1u);
@@ -659,8 +711,13 @@ __global__ void __launch_bounds__(kThreads, 1)
             if (p.mc) tc_commit_mc_warp(&empty[stage], (uint16_t)3);
             else tc_commit_warp(&empty[stage]);
           }
-          tc_commit_warp(&tfull[acc]);
-          tc_commit_warp(&hempty[it % HB]);
+          if constexpr (CG2) {  // both CTAs' accumulators full, both halos free
+            tc_commit_cg2_warp(&tfull[acc], (uint16_t)3);
+            tc_commit_cg2_warp(&hempty[it % HB], (uint16_t)3);
+          } else {
+            tc_commit_warp(&tfull[acc]);
+            tc_commit_warp(&hempty[it % HB]);
+          }
           continue;
         }
         auto kblock = [&](const int kb) {
@@ -834,7 +891,10 @@ __global__ void __launch_bounds__(kThreads, 1)
       if ((p.dbg & 2) && !TMA_EPI) {
         tc_fence_before();
         __syncwarp();
-        if (lane == 0) mbar_arrive(&tempty[acc]);
+        if (lane == 0) {
+          if constexpr (CG2) mbar_arrive_cluster(mapa_u32(smem_u32(&tempty[acc]), 0));  // the leader's barrier
+          else mbar_arrive(&tempty[acc]);
+        }
         continue;
       }
       const uint32_t taddr = tmem_base + acc * BN + ((uint32_t)(q * 32) << 16);
@@ -913,7 +973,10 @@ __global__ void __launch_bounds__(kThreads, 1)
       // accumulator drained: the MMA warp may reuse it
       tc_fence_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive(&tempty[acc]);
+      if (lane == 0) {
+        if constexpr (CG2) mbar_arrive_cluster(mapa_u32(smem_u32(&tempty[acc]), 0));  // the leader's barrier
+        else mbar_arrive(&tempty[acc]);
+      }
       if constexpr (TMA_EPI) {
         fence_proxy_async_smem();
         named_bar_sync(1, kEpiThreads);
@@ -986,7 +1049,10 @@ __global__ void __launch_bounds__(kThreads, 1)
   tc_fence_before();
   __syncthreads();
   if (p.mc) cluster_sync_all();  // no multicast write or commit arrival may target an exited partner
-  if (warp == 4) tmem_dealloc(tmem_base, C::kTmemCols);
+  if (warp == 4) {
+    if constexpr (CG2) tmem_dealloc_cg2(tmem_base, C::kTmemCols);
+    else tmem_dealloc(tmem_base, C::kTmemCols);
+  }
 }
 
 // ------------------------------------------------------------------------------------------
@@ -1197,12 +1263,12 @@ void conv_layer_free(ConvLayer& L) {
   L.scale = L.shift = nullptr;
 }
 
-template <int BN, int AMODE, bool TE, int NB, int RKB = 0>
+template <int BN, int AMODE, bool TE, int NB, int RKB = 0, bool CG2 = false>
 static void launch_t(const ConvLayer& L, const CUtensorMap& ta, const CUtensorMap& ty, const CUtensorMap& tr,
                      const ConvParams& p, cudaStream_t st) {
   static_assert(NB >= 1 && NB <= 4, "staging buffers");
-  auto kern = conv_tc_kernel<BN, AMODE, TE, NB, RKB>;
-  constexpr int smem = Cfg<BN, TE, NB, AMODE == A_HALO, RKB>::kBytes;
+  auto kern = conv_tc_kernel<BN, AMODE, TE, NB, RKB, CG2>;
+  constexpr int smem = Cfg<BN, TE, NB, AMODE == A_HALO, RKB, CG2>::kBytes;
   ensure_smem_attr((const void*)kern, smem);
   if (p.mc) {  // clusters of two CTAs walking pair tiles (see ConvParams::mc)
     if (RKB > 0) fail(1, "conv: multicast with resident weights");
@@ -1272,6 +1338,12 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
       if constexpr (!TE && BN == 64) {
         if (rkb == 9) {
           launch_t<BN, A_HALO, TE, NB, 9>(L, ta, ty, tr, p, st);
+          break;
+        }
+      }
+      if constexpr (!TE && BN == 128) {
+        if (p.cg2) {
+          launch_t<BN, A_HALO, TE, NB, 0, true>(L, ta, ty, tr, p, st);
           break;
         }
       }
@@ -1484,6 +1556,12 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   if (!fuse_tap && use_mc(L, amode, rkb, p)) {
     p.mc = 1;
     p.n_tiles = p.n_nt * ((p.n_mt + 1) / 2);
+    // CTA-pair MMA for the streamed-weight padded-grid halo convs (res3 3x3): pair tile = one position in
+    // two consecutive images (VISTA_CG2=0 keeps the weight-multicast pairs)
+    if (env_flag("VISTA_CG2", true) && amode == A_HALO && L.BN == 128 && rkb == 0 && !p.hseg && p.n_nt == 1 && !p.dbg) {
+      p.cg2 = 1;
+      p.n_tiles = ((N + 1) / 2) * p.mt_per_img;
+    }
   }
   unsigned long long* dbgb = nullptr;
   if (p.dbg & 8) {

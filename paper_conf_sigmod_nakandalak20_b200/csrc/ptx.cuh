@@ -293,6 +293,71 @@ __device__ __forceinline__ void tc_mma_bf16_lo_warp(uint32_t tmem_d, uint32_t a_
       : "memory");
 }
 
+// ---------------- CTA pair (cta_group::2): one MMA over M = 256 rows of two SMs ----------------
+// address of the same shared-memory variable in CTA `rank` of this cluster
+__device__ __forceinline__ uint32_t mapa_u32(uint32_t addr, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
+  return r;
+}
+// arrive on an mbarrier given by its shared::cluster address (possibly in the peer CTA)
+__device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
+// 2-D / 4-D tiled TMA into THIS CTA's shared memory whose complete_tx goes to the mbarrier at
+// `bar_cluster` (shared::cluster address, e.g. the leader CTA's barrier of a CTA pair)
+__device__ __forceinline__ void tma_load_2d_cg2(uint32_t dst, const void* tmap, int32_t c0, int32_t c1,
+                                                uint32_t bar_cluster) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], "
+      "[%4];" ::"r"(dst),
+      "l"(tmap), "r"(c0), "r"(c1), "r"(bar_cluster)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_4d_cg2(uint32_t dst, const void* tmap, int32_t c0, int32_t c1, int32_t c2,
+                                                int32_t c3, uint32_t bar_cluster) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, "
+      "%5}], [%6];" ::"r"(dst),
+      "l"(tmap), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(bar_cluster)
+      : "memory");
+}
+// TMEM allocation for a CTA pair: executed by one warp in EACH CTA of the pair (same column count)
+__device__ __forceinline__ void tmem_alloc_cg2(uint32_t* dst_smem, uint32_t ncols) {
+  asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(dst_smem)),
+               "r"(ncols)
+               : "memory");
+  asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_dealloc_cg2(uint32_t taddr, uint32_t ncols) {
+  asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(taddr), "r"(ncols) : "memory");
+}
+// pair MMA, issued by the leader CTA only: D (+)= A * B^T over M = 256 (A rows 0-127 from the leader's shared
+// memory, 128-255 from the peer's, at the same offset), B's N rows split half / half between the two CTAs
+// at the same offset; each CTA's TMEM receives its 128 rows
+__device__ __forceinline__ void tc_mma_bf16_lo_warp_cg2(uint32_t tmem_d, uint32_t a_lo, uint32_t b_lo, uint32_t idesc,
+                                                        uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p, e;\n\t.reg .b64 da, db;\n\t"
+      "mov.b64 da, {%1, %5};\n\t"
+      "mov.b64 db, {%2, %5};\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], da, db, %3, p;\n\t}" ::"r"(tmem_d),
+      "r"(a_lo), "r"(b_lo), "r"(idesc), "r"(accumulate), "n"(kSw128DescHi)
+      : "memory");
+}
+// pair commit: arrive on the mbarrier at the same offset in the CTAs of `mask` once the pair MMAs finish
+__device__ __forceinline__ void tc_commit_cg2_warp(uint64_t* bar, uint16_t mask) {
+  asm volatile(
+      "{\n\t.reg .pred e;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;\n\t}" ::"r"(
+          smem_u32(bar)),
+      "h"(mask)
+      : "memory");
+}
+
 // Shared-memory matrix descriptor, K-major, no swizzle: 8-row x 16-byte core matrices, rows 16 B
 // apart, core matrices `sbo` bytes apart along M/N and `lbo` bytes apart along K.
 __device__ __forceinline__ uint64_t umma_desc_k_none(uint32_t smem_addr, uint32_t lbo, uint32_t sbo) {

@@ -52,6 +52,8 @@ CONV = [
     (7, 56, 56, 64, 64, 3, 1, 1, 1, False, True),      # halo + resident weights (>= 148 tiles), 3 halo buffers
     (13, 14, 14, 256, 1024, 1, 1, 0, 1, True, True),   # 1x1 resident weights, 8 N tiles (grid 144), M tail
     (6, 28, 28, 128, 512, 1, 1, 0, 1, False, True),    # 1x1 resident weights, K = 128, 4 N tiles
+    (24, 28, 28, 128, 128, 3, 1, 1, 1, True, True),    # res3 3x3 on the CTA pair (cta_group::2, M = 256), residual
+    (23, 28, 28, 128, 128, 3, 1, 1, 1, False, True),   # CTA pair with an odd image count: phantom rank-1 tiles
 ]
 
 
@@ -135,3 +137,19 @@ def test_ingest_exact():
     y = vista_ingest(torch.from_numpy(px).cuda()).to(torch.float64).cpu().numpy()
     np.testing.assert_array_equal(y[..., :3], (px.astype(np.float64) - 128) / 128)
     assert not y[..., 3:].any()
+
+
+@pytest.mark.parametrize("N", [24, 23])
+def test_halo_cta_pair_bit_identical(monkeypatch, N):
+    # the res3-class 3x3 halo conv runs as ONE tcgen05.mma.cta_group::2 per K step over both CTAs of a pair
+    # (VISTA_CG2, default on) or as two cta_group::1 MMAs with multicast weights (VISTA_CG2=0): the same
+    # per-element K order, so the same bits
+    x, _ = bf(rng.standard_normal((N, 28, 28, 128)))
+    w, _ = bf(rng.standard_normal((128, 3, 3, 128)) * (2.0 / 1152) ** 0.5)
+    scale = torch.from_numpy(rng.uniform(0.5, 1.5, 128).astype(np.float32)).cuda()
+    shift = torch.from_numpy(rng.standard_normal(128).astype(np.float32) * 0.1).cuda()
+    out = {}
+    for cg2 in ("1", "0"):
+        monkeypatch.setenv("VISTA_CG2", cg2)
+        out[cg2] = vista_conv2d(x, w, scale, shift, 1, 1, 1, relu=True).view(torch.int16).cpu()
+    assert torch.equal(out["1"], out["0"])

@@ -235,8 +235,9 @@ __global__ void __launch_bounds__(kThreads, 1)
   };
   if (threadIdx.x == 0) {
     for (int i = 0; i < S; ++i) {
-      mbar_init(&full[i], a_by_tma(AMODE) ? 1 : 128 + 1);
-      mbar_init(&empty[i], p.mc ? 2 : 1);  // multicast: both CTAs' MMAs must release the stage
+      mbar_init(&full[i], a_by_tma(AMODE) ? (CG2 ? 2 : 1) : 128 + 1);  // CTA pair: both CTAs arrive
+      // multicast: both CTAs' MMAs must release the stage; CTA pair: the leader's one pair commit does
+      mbar_init(&empty[i], p.mc && !CG2 ? 2 : 1);
     }
     for (int i = 0; i < NACC; ++i) {
       mbar_init(&tfull[i], 1);
@@ -245,7 +246,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     for (int i = 0; i < 4; ++i) mbar_init(&rbar[i], 1);
     for (int i = 0; i < 3; ++i) {
-      mbar_init(&hfull[i], 1);
+      mbar_init(&hfull[i], CG2 ? 2 : 1);
       mbar_init(&hempty[i], 1);
     }
     mbar_init(wres, 1);
@@ -337,6 +338,7 @@ __global__ void __launch_bounds__(kThreads, 1)
               if (crank == 0) mbar_arrive_expect_tx(&full[stage], 2 * two * C::kBBytes);
               for (int h = 0; h < two; ++h)
                 tma_load_2d_cg2(sB + (2 * stage + h) * C::kBBytes, &tmap_w, (kb + h) * BK, (int)crank * (BN / 2), fl);
+              if (crank != 0) mbar_arrive_cluster(fl);
               continue;
             }
             mbar_arrive_expect_tx(&full[stage], two * C::kBBytes);
@@ -374,6 +376,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             if (crank == 0) mbar_arrive_expect_tx(&hfull[hb], 2 * box_bytes * p.cblocks);
             for (int cb = 0; cb < p.cblocks; ++cb)
               tma_load_4d_cg2(sH + hb * halo_half_bytes(BN) + cb * p.hsz, &tmap_a, cb * BK, col0, prow0 - 1, nimg, hl);
+            if (crank != 0) mbar_arrive_cluster(hl);
             continue;
           }
           if ((p.dbg & 1) && it >= (uint32_t)HB) {

@@ -37,8 +37,19 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
   return ok != 0;
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+#ifdef VISTA_HANG_DEBUG
+  // debug builds only (tools/): a wait that never completes reports itself and traps instead of hanging
+  long long n = 0;
+  while (!mbar_try_wait(bar, parity)) {
+    if (++n == (1ll << 24))
+      printf("vista hang: block %d thread %d mbarrier smem 0x%x parity %u\n", (int)blockIdx.x, (int)threadIdx.x,
+             smem_u32(bar), parity);
+    if (n > (1ll << 25)) __trap();
+  }
+#else
   while (!mbar_try_wait(bar, parity)) {
   }
+#endif
 }
 
 // named barrier among `nthreads` threads (multiple of 32); id 0 is __syncthreads
@@ -302,7 +313,7 @@ __device__ __forceinline__ uint32_t mapa_u32(uint32_t addr, uint32_t rank) {
 }
 // arrive on an mbarrier given by its shared::cluster address (possibly in the peer CTA)
 __device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
-  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
 }
 // 2-D / 4-D tiled TMA into THIS CTA's shared memory whose complete_tx goes to the mbarrier at
 // `bar_cluster` (shared::cluster address, e.g. the leader CTA's barrier of a CTA pair)

@@ -1527,7 +1527,9 @@ VISTA_API vista_status vista_run(vista_ctx* c, const uint8_t* images, const int6
   return guarded(c, [&] {
     const int L = (int)c->taps.size();
     static const bool overlap_on = !(getenv("VISTA_OVERLAP") && getenv("VISTA_OVERLAP")[0] == '0');
-    const bool overlap = overlap_on && c->sys.world == 1 && !c->f32;
+    // (profiling times every launch with CUDA events on its stream: kernels of the two streams would be
+    // charged each other's time, so the profiled run trains after the transfer)
+    const bool overlap = overlap_on && c->sys.world == 1 && !c->f32 && !g_prof;
     if (!overlap) {
       transfer_body(c, images, nullptr, image_keys, structured, str_keys, labels);
       for (int k = 0; k < L; ++k) {

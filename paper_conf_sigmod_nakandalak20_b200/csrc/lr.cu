@@ -529,6 +529,21 @@ __device__ __forceinline__ void grid_sync(unsigned int* bar, int nthr) {
 __device__ void reduce_cols(const float* partial, int pitch, int G, int j0, int n, double* out, double* sh,
                             int nthr) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwc = nthr >> 5;
+  if (G < 4 * nwc) {
+    // few CTAs (small inputs): the CTA-range split would leave most warps idle and walk the columns 32 at
+    // a time behind two barriers each (measured: ~30 us per pass for one CTA at ld 4104); instead each
+    // lane sums whole columns over the G partial rows in CTA order, warps on different 32-column tiles
+    for (int t = warp * 32; t < n; t += nwc * 32) {
+      if (t + lane < n) {
+        const float* pc = partial + j0 + t + lane;
+        double s = 0.0;
+        for (int c = 0; c < G; ++c) s += (double)__ldcg(pc + (size_t)c * pitch);
+        out[t + lane] = s;
+      }
+    }
+    named_bar_sync(2, nthr);
+    return;
+  }
   const int c0 = (int)((int64_t)G * warp / nwc), c1 = (int)((int64_t)G * (warp + 1) / nwc);
   for (int t = 0; t < n; t += 32) {
     const int j = j0 + t + lane;
@@ -979,8 +994,10 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
     }
   }
   const int64_t pass_rb = cfg.dot_rb > 0 ? std::min(cfg.rb, cfg.dot_rb) : cfg.rb;  // grid: blocks of the finer kernel
+  // at least one CTA per 128 columns: the fused tail splits the ld columns over the CTAs, and a grid sized
+  // by a handful of rows left one CTA walking all of them behind L2 latency (C1: 33 -> ~9 us per pass)
   auto grid_for_rows = [&](int64_t rows) {
-    const int64_t blocks = (rows + pass_rb - 1) / pass_rb;
+    const int64_t blocks = std::max<int64_t>((rows + pass_rb - 1) / pass_rb, (ld + 127) / 128);
     return (int)std::max<int64_t>(1, std::min<int64_t>(blocks, num_sms()));
   };
   cfg.grid = grid_for_rows(n_train);

@@ -79,7 +79,9 @@ struct ConvParams {
   // M = 256 (rank r's 128 rows in its own shared memory and TMEM); the pair tile is the same position in two
   // consecutive images (rank r: image 2j + r), so both halos sit at the same offsets; each CTA loads half of
   // every weight k-block (B's N rows split between the pair): per-SM operand reads 4 KB + BN/2 * 32 B per
-  // MMA instead of 4 KB + BN * 32 B, and half the weight bytes written into each CTA's shared memory
+  // MMA instead of 4 KB + BN * 32 B, and half the weight bytes written into each CTA's shared memory.
+  // cg2 = 2 (A_IM2COL / A_TMA, BN = 256): the same pair MMA over the multicast pair tile (two adjacent M
+  // tiles; both CTAs' A tiles sit in the same ring stage)
   int cg2;
   int segs;  // A_ROWVIEW: 128-pixel segments per output row (1 unless Wo > 128); A_HALO + hseg: segments
   // A_HALO row-segment tiles (hseg = 1, rows too wide for the padded-grid halo): tile = (image, output row,
@@ -150,7 +152,7 @@ struct Cfg {
 // tile -> (first row m0, N-tile index nt, group g); N-tiles of one M-tile are adjacent so
 // the 148 CTAs working at any moment share A rows in L2
 __device__ __forceinline__ void decode_tile(const ConvParams& p, int tile, int& m0, int& nt, int& g) {
-  if (p.cg2) {  // pair tile (j, t) -> M tile t of image 2j + rank (rank 1 past the last image: phantom)
+  if (p.cg2 == 1) {  // halo pair tile (j, t) -> M tile t of image 2j + rank (rank 1 past the last image: phantom)
     const int j = tile / p.mt_per_img, t = tile - j * p.mt_per_img;
     m0 = ((2 * j + (int)(blockIdx.x & 1)) * p.mt_per_img + t) * BM;
     nt = 0;
@@ -196,7 +198,8 @@ __global__ void __launch_bounds__(kThreads, 1)
                    const __grid_constant__ CUtensorMap tmap_y, const __grid_constant__ CUtensorMap tmap_r,
                    const ConvParams p) {
   using C = Cfg<BN, TMA_EPI, NB, AMODE == A_HALO, RKB, CG2>;
-  static_assert(!CG2 || (AMODE == A_HALO && RKB == 0 && !TMA_EPI), "CTA-pair MMA: streamed-weight halo path only");
+  static_assert(!CG2 || (RKB == 0 && !TMA_EPI && (AMODE == A_HALO || AMODE == A_IM2COL || AMODE == A_TMA)),
+                "CTA-pair MMA: streamed weights, register epilogue, halo / im2col / plain TMA A");
   constexpr int S = C::kStages;
   constexpr bool BRES = RKB > 0;
   constexpr int HB = C::kHB > 0 ? C::kHB : 1;
@@ -288,6 +291,14 @@ __global__ void __launch_bounds__(kThreads, 1)
           for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
             const int stage = gk % S;
             if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
+            if constexpr (CG2) {  // own A rows + own half of the B rows, completing on the leader's barrier
+              const uint32_t fl = mapa_u32(smem_u32(&full[stage]), 0);
+              if (crank == 0) mbar_arrive_expect_tx(&full[stage], 2 * C::kStageBytes);
+              tma_load_2d_cg2(sA + stage * C::kABytes, &tmap_a, kb * BK, m0, fl);
+              tma_load_2d_cg2(sB + stage * C::kBBytes, &tmap_w, kb * BK, n0 + (int)crank * (BN / 2), fl);
+              if (crank != 0) mbar_arrive_cluster(fl);
+              continue;
+            }
             mbar_arrive_expect_tx(&full[stage], C::kStageBytes);
             tma_load_2d(sA + stage * C::kABytes, &tmap_a, g * p.Cg_in + kb * BK, m0, &full[stage]);
             if constexpr (!BRES) load_b(stage, kb, g * p.Cg_out + n0);
@@ -460,10 +471,19 @@ __global__ void __launch_bounds__(kThreads, 1)
           for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
             const int stage = gk % S;
             if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
-            mbar_arrive_expect_tx(&full[stage], C::kABytes + C::kBBytes);
-            tma_load_im2col_4d(sA + stage * C::kABytes, &tmap_a, g * p.Cg_in + cb * BK, w0, h0, nimg, (uint16_t)s,
-                               (uint16_t)r, &full[stage]);
-            load_b(stage, kb, g * p.Cg_out + n0);
+            if constexpr (CG2) {  // own A rows + own half of the B rows, completing on the leader's barrier
+              const uint32_t fl = mapa_u32(smem_u32(&full[stage]), 0);
+              if (crank == 0) mbar_arrive_expect_tx(&full[stage], 2 * (C::kABytes + C::kBBytes));
+              tma_load_im2col_4d_cg2(sA + stage * C::kABytes, &tmap_a, cb * BK, w0, h0, nimg, (uint16_t)s, (uint16_t)r,
+                                     fl);
+              tma_load_2d_cg2(sB + stage * C::kBBytes, &tmap_w, kb * BK, n0 + (int)crank * (BN / 2), fl);
+              if (crank != 0) mbar_arrive_cluster(fl);
+            } else {
+              mbar_arrive_expect_tx(&full[stage], C::kABytes + C::kBBytes);
+              tma_load_im2col_4d(sA + stage * C::kABytes, &tmap_a, g * p.Cg_in + cb * BK, w0, h0, nimg, (uint16_t)s,
+                                 (uint16_t)r, &full[stage]);
+              load_b(stage, kb, g * p.Cg_out + n0);
+            }
             if (++cb == cblocks) {
               cb = 0;
               if (++s == p.S) {
@@ -745,6 +765,12 @@ __global__ void __launch_bounds__(kThreads, 1)
             for (int k = 0; k < BK / 16; ++k)
               tc_mma_bf16_warp(tacc, umma_desc_k_none(a0 + k * 4096, 2048, 128), umma_desc_k_sw128(b0 + k * 32),
                                idesc, (kb | k) != 0 ? 1u : 0u);
+          } else if constexpr (CG2) {  // one pair MMA per K step over both CTAs' A tiles and B halves
+            const uint32_t a = umma_desc_lo_sw128(a0), b = umma_desc_lo_sw128(b0);
+            tc_mma_bf16_lo_warp_cg2(tacc, a, b, idesc, kb != 0 ? 1u : 0u);
+            tc_mma_bf16_lo_warp_cg2(tacc, a + 2, b + 2, idesc, 1u);
+            tc_mma_bf16_lo_warp_cg2(tacc, a + 4, b + 4, idesc, 1u);
+            tc_mma_bf16_lo_warp_cg2(tacc, a + 6, b + 6, idesc, 1u);
           } else {
             const uint64_t da = umma_desc_k_sw128(a0), db = umma_desc_k_sw128(b0);
             // +32 bytes along K = +2 in the descriptors' address fields
@@ -754,7 +780,8 @@ __global__ void __launch_bounds__(kThreads, 1)
             tc_mma_bf16_warp(tacc, da + 6, db + 6, idesc, 1u);
           }
           if constexpr (kRing) {
-            if (p.mc) tc_commit_mc_warp(&empty[stage], (uint16_t)3);
+            if constexpr (CG2) tc_commit_cg2_warp(&empty[stage], (uint16_t)3);  // both CTAs' stages are free
+            else if (p.mc) tc_commit_mc_warp(&empty[stage], (uint16_t)3);
             else tc_commit_warp(&empty[stage]);
           }
           ++gk;
@@ -770,7 +797,8 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
           for (; kb < p.nkb; ++kb) kblock(kb);
         }
-        tc_commit_warp(&tfull[acc]);
+        if constexpr (CG2) tc_commit_cg2_warp(&tfull[acc], (uint16_t)3);  // both CTAs' accumulators
+        else tc_commit_warp(&tfull[acc]);
         if constexpr (AMODE == A_HALO) tc_commit_warp(&hempty[it % HB]);  // halo free once these MMAs finish
       }
       if (prof_mma && p.dbg_buf) {
@@ -1306,6 +1334,12 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
                       const CUtensorMap& tr, const ConvParams& p, cudaStream_t st, int rkb) {
   switch (amode) {
     case A_TMA:
+      if constexpr (!TE && BN == 256) {
+        if (p.cg2) {
+          launch_t<BN, A_TMA, TE, NB, 0, true>(L, ta, ty, tr, p, st);
+          break;
+        }
+      }
       if constexpr (TE && BN <= 128) {
         if (rkb == 4) {
           launch_t<BN, A_TMA, TE, NB, 4>(L, ta, ty, tr, p, st);
@@ -1325,7 +1359,15 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
       break;
     case A_GATHER_FAST: launch_t<BN, A_GATHER_FAST, TE, NB>(L, ta, ty, tr, p, st); break;
     case A_GATHER_ROW: launch_t<BN, A_GATHER_ROW, TE, NB>(L, ta, ty, tr, p, st); break;
-    case A_IM2COL: launch_t<BN, A_IM2COL, TE, NB>(L, ta, ty, tr, p, st); break;
+    case A_IM2COL:
+      if constexpr (!TE && BN == 256) {
+        if (p.cg2) {
+          launch_t<BN, A_IM2COL, TE, NB, 0, true>(L, ta, ty, tr, p, st);
+          break;
+        }
+      }
+      launch_t<BN, A_IM2COL, TE, NB>(L, ta, ty, tr, p, st);
+      break;
     case A_IM2COL_C8: launch_t<BN, A_IM2COL_C8, TE, NB>(L, ta, ty, tr, p, st); break;
     case A_ROWVIEW:
       if constexpr (TE && BN <= 128) {
@@ -1565,6 +1607,10 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
       p.cg2 = 1;
       p.n_tiles = ((N + 1) / 2) * p.mt_per_img;
     }
+    // CTA-pair MMA (M = 256, N = 256) for the streamed-weight im2col / plain-TMA convs with the register
+    // epilogue: the multicast pair tile (two adjacent M tiles), each CTA loading its A tile and half of B
+    if (env_flag("VISTA_CG2", true) && (amode == A_IM2COL || amode == A_TMA) && L.BN == 256 && !tma_epi && !p.dbg)
+      p.cg2 = 2;
   }
   unsigned long long* dbgb = nullptr;
   if (p.dbg & 8) {

@@ -333,6 +333,14 @@ __device__ __forceinline__ void tma_load_4d_cg2(uint32_t dst, const void* tmap, 
       "l"(tmap), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(bar_cluster)
       : "memory");
 }
+__device__ __forceinline__ void tma_load_im2col_4d_cg2(uint32_t dst, const void* tmap, int32_t c, int32_t w, int32_t h,
+                                                       int32_t n, uint16_t off_w, uint16_t off_h, uint32_t bar_cluster) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.cta_group::2.shared::cluster.global.im2col.mbarrier::complete_tx::bytes [%0], [%1, {%2, "
+      "%3, %4, %5}], [%6], {%7, %8};" ::"r"(dst),
+      "l"(tmap), "r"(c), "r"(w), "r"(h), "r"(n), "r"(bar_cluster), "h"(off_w), "h"(off_h)
+      : "memory");
+}
 // TMEM allocation for a CTA pair: executed by one warp in EACH CTA of the pair (same column count)
 __device__ __forceinline__ void tmem_alloc_cg2(uint32_t* dst_smem, uint32_t ncols) {
   asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(dst_smem)),

@@ -54,6 +54,7 @@ CONV = [
     (6, 28, 28, 128, 512, 1, 1, 0, 1, False, True),    # 1x1 resident weights, K = 128, 4 N tiles
     (24, 28, 28, 128, 128, 3, 1, 1, 1, True, True),    # res3 3x3 on the CTA pair (cta_group::2, M = 256), residual
     (23, 28, 28, 128, 128, 3, 1, 1, 1, False, True),   # CTA pair with an odd image count: phantom rank-1 tiles
+    (101, 14, 14, 256, 256, 3, 1, 1, 1, True, True),   # res4 3x3 on the CTA pair (im2col, M = N = 256), phantom tile
 ]
 
 
@@ -152,4 +153,28 @@ def test_halo_cta_pair_bit_identical(monkeypatch, N):
     for cg2 in ("1", "0"):
         monkeypatch.setenv("VISTA_CG2", cg2)
         out[cg2] = vista_conv2d(x, w, scale, shift, 1, 1, 1, relu=True).view(torch.int16).cpu()
+    assert torch.equal(out["1"], out["0"])
+
+
+@pytest.mark.parametrize("N,H,C,Cout,k,stride,residual", [
+    (101, 14, 256, 256, 3, 1, False),   # res4 3x3 class: im2col A, odd M-tile count (phantom rank-1 tile)
+    (40, 7, 512, 512, 3, 1, True),      # res5 3x3 class with a residual
+    (100, 14, 1024, 256, 1, 1, False),  # 1x1 streamed weights: plain 2-D TMA A
+    (60, 28, 512, 256, 1, 2, False),    # strided 1x1: im2col A with traversal stride 2
+])
+def test_pair_mma_bn256_bit_identical(monkeypatch, N, H, C, Cout, k, stride, residual):
+    # BN = 256 im2col / plain-TMA convs run as ONE tcgen05.mma.cta_group::2 (M = 256, N = 256) per K step over the
+    # multicast pair tile (VISTA_CG2 default on) or as two cta_group::1 MMAs with multicast weights (VISTA_CG2=0):
+    # same per-element K order, same bits
+    pad = (k - 1) // 2
+    x, _ = bf(rng.standard_normal((N, H, H, C)))
+    w, _ = bf(rng.standard_normal((Cout, k, k, C)) * (2.0 / (k * k * C)) ** 0.5)
+    scale = torch.from_numpy(rng.uniform(0.5, 1.5, Cout).astype(np.float32)).cuda()
+    shift = torch.from_numpy(rng.standard_normal(Cout).astype(np.float32) * 0.1).cuda()
+    Ho = (H + 2 * pad - k) // stride + 1
+    r = bf(rng.standard_normal((N, Ho, Ho, Cout)))[0] if residual else None
+    out = {}
+    for cg2 in ("1", "0"):
+        monkeypatch.setenv("VISTA_CG2", cg2)
+        out[cg2] = vista_conv2d(x, w, scale, shift, stride, pad, 1, residual=r, relu=True).view(torch.int16).cpu()
     assert torch.equal(out["1"], out["0"])

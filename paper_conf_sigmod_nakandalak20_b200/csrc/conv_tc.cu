@@ -198,8 +198,9 @@ __global__ void __launch_bounds__(kThreads, 1)
                    const __grid_constant__ CUtensorMap tmap_y, const __grid_constant__ CUtensorMap tmap_r,
                    const ConvParams p) {
   using C = Cfg<BN, TMA_EPI, NB, AMODE == A_HALO, RKB, CG2>;
-  static_assert(!CG2 || (RKB == 0 && !TMA_EPI && (AMODE == A_HALO || AMODE == A_IM2COL || AMODE == A_TMA)),
-                "CTA-pair MMA: streamed weights, register epilogue, halo / im2col / plain TMA A");
+  static_assert(!CG2 || (RKB == 0 && (AMODE == A_HALO ? !TMA_EPI
+                                                     : (AMODE == A_IM2COL || AMODE == A_TMA || AMODE == A_CAT))),
+                "CTA-pair MMA: streamed weights; halo (register epilogue) / im2col / plain TMA / cat A");
   constexpr int S = C::kStages;
   constexpr bool BRES = RKB > 0;
   constexpr int HB = C::kHB > 0 ? C::kHB : 1;
@@ -318,6 +319,20 @@ __global__ void __launch_bounds__(kThreads, 1)
           for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
             const int stage = gk % S;
             if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
+            if constexpr (CG2) {  // own A rows + own half of the B rows, completing on the leader's barrier
+              const uint32_t fl = mapa_u32(smem_u32(&full[stage]), 0);
+              if (crank == 0) mbar_arrive_expect_tx(&full[stage], 2 * C::kStageBytes);
+              if (kb < p.nkb1)
+                tma_load_2d_cg2(sA + stage * C::kABytes, &tmap_a, kb * BK, m0, fl);
+              else if (p.cat_im2col)
+                tma_load_im2col_4d_cg2(sA + stage * C::kABytes, &tmap_r, (kb - p.nkb1) * BK, wo * p.stride,
+                                       ho * p.stride, nimg, 0, 0, fl);
+              else
+                tma_load_2d_cg2(sA + stage * C::kABytes, &tmap_r, (kb - p.nkb1) * BK, m0, fl);
+              tma_load_2d_cg2(sB + stage * C::kBBytes, &tmap_w, kb * BK, n0 + (int)crank * (BN / 2), fl);
+              if (crank != 0) mbar_arrive_cluster(fl);
+              continue;
+            }
             mbar_arrive_expect_tx(&full[stage], C::kStageBytes);
             if (kb < p.nkb1)
               tma_load_2d(sA + stage * C::kABytes, &tmap_a, kb * BK, m0, &full[stage]);
@@ -1334,7 +1349,7 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
                       const CUtensorMap& tr, const ConvParams& p, cudaStream_t st, int rkb) {
   switch (amode) {
     case A_TMA:
-      if constexpr (!TE && BN == 256) {
+      if constexpr (BN == 256) {
         if (p.cg2) {
           launch_t<BN, A_TMA, TE, NB, 0, true>(L, ta, ty, tr, p, st);
           break;
@@ -1349,6 +1364,12 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
       launch_t<BN, A_TMA, TE, NB>(L, ta, ty, tr, p, st);
       break;
     case A_CAT:
+      if constexpr (BN == 256) {
+        if (p.cg2) {
+          launch_t<BN, A_CAT, TE, NB, 0, true>(L, ta, ty, tr, p, st);
+          break;
+        }
+      }
       if constexpr (TE && BN <= 128) {
         if (rkb == 4) {
           launch_t<BN, A_CAT, TE, NB, 4>(L, ta, ty, tr, p, st);
@@ -1360,7 +1381,7 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
     case A_GATHER_FAST: launch_t<BN, A_GATHER_FAST, TE, NB>(L, ta, ty, tr, p, st); break;
     case A_GATHER_ROW: launch_t<BN, A_GATHER_ROW, TE, NB>(L, ta, ty, tr, p, st); break;
     case A_IM2COL:
-      if constexpr (!TE && BN == 256) {
+      if constexpr (BN == 256) {
         if (p.cg2) {
           launch_t<BN, A_IM2COL, TE, NB, 0, true>(L, ta, ty, tr, p, st);
           break;
@@ -1609,7 +1630,8 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
     }
     // CTA-pair MMA (M = 256, N = 256) for the streamed-weight im2col / plain-TMA convs with the register
     // epilogue: the multicast pair tile (two adjacent M tiles), each CTA loading its A tile and half of B
-    if (env_flag("VISTA_CG2", true) && (amode == A_IM2COL || amode == A_TMA) && L.BN == 256 && !tma_epi && !p.dbg)
+    if (env_flag("VISTA_CG2", true) && (amode == A_IM2COL || amode == A_TMA) && L.BN == 256 && !p.dbg &&
+        !p.tapf)
       p.cg2 = 2;
   }
   unsigned long long* dbgb = nullptr;
@@ -1714,6 +1736,7 @@ void conv_cat_forward(const ConvLayer& L, int Cx, const bf16* b, const bf16* x, 
   if (use_mc(L, A_CAT, rkb, p)) {
     p.mc = 1;
     p.n_tiles = p.n_nt * ((p.n_mt + 1) / 2);
+    if (env_flag("VISTA_CG2", true) && L.BN == 256 && !p.dbg) p.cg2 = 2;  // CTA-pair MMA, see conv_forward
   }
   const double flops = 2.0 * (double)M * L.Cout * L.K_alg;
   const double bytes = 2.0 * ((double)M * (Kb + Cx + L.Cout) + (double)L.Cout * L.Kp);

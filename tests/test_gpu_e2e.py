@@ -271,18 +271,24 @@ def test_weight_multicast_bit_identical(monkeypatch):
     # 2-CTA weight multicast (ConvParams::mc) engages only for launches with >= 74 pair tiles: 600 images put
     # the res4 / res5 / projection-unit launches above that, and res4's 919 M tiles give rank 1 of the last
     # pair a phantom tile past M.  Multicast changes where the weight bytes come from, not the MMA order, so
-    # every bit of MM_l must agree with VISTA_MC=0; three sampled images are also held to the oracle.
+    # every bit of MM_l must agree with VISTA_MC=0; three sampled images are also held to the oracle.  The
+    # default runs the pairs' MMAs as cta_group::2 (M = 256: res3 halo, BN = 256 im2col / TMA / projection
+    # units); VISTA_CG2=0 keeps multicast pairs of cta_group::1 MMAs: all three must agree bit for bit.
     tab = gen.make_tables(600, 8)
     out, feats = {}, None
-    for mc in ("1", "0"):
-        monkeypatch.setenv("VISTA_MC", mc)
+    for mode, env in (("cg2", {}), ("mc", {"VISTA_CG2": "0"}), ("unicast", {"VISTA_MC": "0"})):
+        for key in ("VISTA_MC", "VISTA_CG2"):
+            monkeypatch.delenv(key, raising=False)
+        for key, val in env.items():
+            monkeypatch.setenv(key, val)
         v = run_gpu(2, [0, 1, 2, 3, 4], tab, 8, iters=1, micro_batch=600)
-        out[mc] = [v.features(k)["mm"].view(torch.int16).cpu().clone() for k in range(5)]
-        if mc == "1":
+        out[mode] = [v.features(k)["mm"].view(torch.int16).cpu().clone() for k in range(5)]
+        if mode == "cg2":
             feats = [v.features(k)["features"].to(torch.float64).cpu().numpy()[:3] for k in range(5)]
         v.close()
-    for a, b in zip(out["1"], out["0"]):
-        assert torch.equal(a, b)
+    for mode in ("mc", "unicast"):
+        for a, b in zip(out["cg2"], out[mode]):
+            assert torch.equal(a, b), mode
     F, _ = oracle.features(oracle.RESNET50, WSEED, tab.images[:3], taps=[0, 1, 2, 3, 4])
     for k in range(5):
         assert normwise_rows(feats[k], F[k]).max() <= 2e-2

@@ -158,9 +158,10 @@ def test_halo_cta_pair_bit_identical(monkeypatch, N):
 
 @pytest.mark.parametrize("N,H,C,Cout,k,stride,residual", [
     (101, 14, 256, 256, 3, 1, False),   # res4 3x3 class: im2col A, odd M-tile count (phantom rank-1 tile)
-    (40, 7, 512, 512, 3, 1, True),      # res5 3x3 class with a residual
+    (200, 7, 512, 512, 3, 1, True),     # res5 3x3 class with a residual
     (100, 14, 1024, 256, 1, 1, False),  # 1x1 streamed weights: plain 2-D TMA A
-    (60, 28, 512, 256, 1, 2, False),    # strided 1x1: im2col A with traversal stride 2
+    (100, 28, 512, 256, 1, 2, False),   # strided 1x1: im2col A with traversal stride 2, TMA epilogue
+    (64, 7, 512, 2048, 1, 1, True),     # res5 closing conv: plain TMA A, 8 N tiles, TMA epilogue + residual
 ])
 def test_pair_mma_bn256_bit_identical(monkeypatch, N, H, C, Cout, k, stride, residual):
     # BN = 256 im2col / plain-TMA convs run as ONE tcgen05.mma.cta_group::2 (M = 256, N = 256) per K step over the

@@ -83,6 +83,15 @@ struct ConvParams {
   // cg2 = 2 (A_IM2COL / A_TMA, BN = 256): the same pair MMA over the multicast pair tile (two adjacent M
   // tiles; both CTAs' A tiles sit in the same ring stage)
   int cg2;
+  // amc = 1 (resident weights, A_TMA / stride-1 A_CAT, an even number of N tiles): CTA pairs (blockIdx 2i, 2i+1)
+  // hold adjacent N tiles and walk the same M tiles; each loads half of every A k-block's rows and multicasts
+  // it to both, halving the per-SM L2 -> shared-memory A bytes (A is re-read once per N tile)
+  int amc;
+  // apf > 0 (resident-weight A_TMA launches): the CTA holding N tile 0 prefetches into L2 the A rows of the M tile
+  // it will reach apf tiles later (the 64 KB A of a K = 256 tile is one contiguous range; the TMA loads of the
+  // CTAs sharing that M tile then hit L2 instead of waiting on HBM behind a 4-stage ring)
+  int apf;
+  int no_sthr;  // 1: TMA epilogue without the store thread (VISTA_STORE_THR=0, A/B)
   int segs;  // A_ROWVIEW: 128-pixel segments per output row (1 unless Wo > 128); A_HALO + hseg: segments
   // A_HALO row-segment tiles (hseg = 1, rows too wide for the padded-grid halo): tile = (image, output row,
   // segment of seg_w <= 126 columns); the halo is 3 input rows x (seg_w + 2) padded columns (Wp = seg_w + 2)
@@ -132,7 +141,7 @@ struct Cfg {
   // 4 rows per instruction (per-row 16-byte stores touched 32 lines per instruction: LSU-bound, measured)
   static constexpr bool kStaged = kSplit && BN == 64;
   static constexpr int kStgBytes = kStaged ? kEpiWarps * 32 * 64 : 0;
-  static constexpr int kNBar = 20;  // tfull/tempty[4], rbar[4], hfull/hempty[3], wres[1], slack
+  static constexpr int kNBar = 28;  // tfull/tempty[4], rbar[4], hfull/hempty[3], wres[1], staged/sfree[4], slack
   static constexpr int kFixed = kHaloBytes + kResBytes + kOutBytes + kSbufBytes + kStgBytes + 1024 + 16 + kNBar * 8;
   static constexpr int kStagesFit = kStageBytes ? (227 * 1024 - kFixed) / (kStageBytes + 16) : 2;
   static constexpr int kStages = kStagesFit > 8 ? 8 : kStagesFit;
@@ -221,14 +230,22 @@ __global__ void __launch_bounds__(kThreads, 1)
   uint64_t* hfull = rbar + 4;    // [3] halo buffer landed (A_HALO)
   uint64_t* hempty = hfull + 3;  // [3] halo buffer consumed by the tile's MMAs (A_HALO)
   uint64_t* wres = hempty + 3;   // [1] resident weights landed (RKB > 0)
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(wres + 1);
+  uint64_t* staged = wres + 1;   // [NB] store thread: the epilogue has written staging buffer b
+  uint64_t* sfree = staged + 4;  // [NB] store thread: buffer b's TMA store has read it (no residual)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(sfree + 4);
+  // TMA epilogue with a dedicated store thread (thread 32, idle in these A modes): it issues the output stores,
+  // waits for their shared-memory reads and refills the freed buffer with a later tile's residual, so the
+  // epilogue warps never wait on store completion or on one another (no per-tile named barriers)
+  constexpr bool kStoreThrMode = TMA_EPI && (AMODE == A_TMA || AMODE == A_CAT || AMODE == A_IM2COL ||
+                                             AMODE == A_ROWVIEW || AMODE == A_IM2COL_C8);
+  const bool sthr = kStoreThrMode && !p.tapf && !p.no_sthr;
   const uint32_t sH = base + C::kHaloOff;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   // this CTA's first tile and the tile stride (pair tiles when multicasting weights)
   const int cta0 = p.mc ? (int)(blockIdx.x >> 1) : (int)blockIdx.x;
   const int ncta = p.mc ? (int)(gridDim.x >> 1) : (int)gridDim.x;
-  const uint32_t crank = p.mc ? (blockIdx.x & 1u) : 0u;
+  const uint32_t crank = (p.mc || p.amc) ? (blockIdx.x & 1u) : 0u;
   // weight k-block kb of N rows [row0, row0 + BN) into ring stage `stage` (multicast: this CTA's half)
   auto load_b = [&](int stage, int kb, int row0) {
     if (p.mc)
@@ -241,7 +258,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     for (int i = 0; i < S; ++i) {
       mbar_init(&full[i], a_by_tma(AMODE) ? (CG2 ? 2 : 1) : 128 + 1);  // CTA pair: both CTAs arrive
       // multicast: both CTAs' MMAs must release the stage; CTA pair: the leader's one pair commit does
-      mbar_init(&empty[i], p.mc && !CG2 ? 2 : 1);
+      mbar_init(&empty[i], (p.mc && !CG2) || p.amc ? 2 : 1);
     }
     for (int i = 0; i < NACC; ++i) {
       mbar_init(&tfull[i], 1);
@@ -254,6 +271,10 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(&hempty[i], 1);
     }
     mbar_init(wres, 1);
+    for (int i = 0; i < 4; ++i) {
+      mbar_init(&staged[i], kEpiWarps);
+      mbar_init(&sfree[i], 1);
+    }
     fence_mbar_init();
     tma_prefetch(&tmap_w);
     if (a_by_tma(AMODE)) tma_prefetch(&tmap_a);
@@ -266,12 +287,62 @@ __global__ void __launch_bounds__(kThreads, 1)
   }
   tc_fence_before();
   __syncthreads();
-  if (p.mc) cluster_sync_all();  // the partner's barriers are initialised before any multicast reaches them
+  if (p.mc || p.amc) cluster_sync_all();  // the partner's barriers are initialised before any multicast reaches them
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
 
   if (warp < 4) {
     // ======================= producers =======================
+    if (sthr && threadIdx.x == 32) {
+      // ---- store thread (TMA epilogue): stores of tile it from buffer it % NB, residual refills ----
+      const bool has_res = p.res != nullptr;
+      auto issue_res = [&](int t, uint32_t b) {
+        int tm0, tnt, tg;
+        decode_tile(p, t, tm0, tnt, tg);
+        const int tn0 = tnt * BN, tng0 = tg * p.Cg_out + tn0;
+        const int nsub = (min(BN, p.Cg_out - tn0) + 63) / 64;
+        mbar_arrive_expect_tx(&rbar[b], nsub * BM * 128);
+        for (int st = 0; st < nsub; ++st)
+          tma_load_2d(sO + b * (uint32_t)(BM * BN * 2) + st * BM * 128, &tmap_r, tng0 + st * 64, tm0, &rbar[b]);
+      };
+      if (has_res)  // the first residual tiles (NB = 1: the first tile's)
+        for (int j = 0; j < (NB > 1 ? NB - 1 : 1); ++j)
+          if (cta0 + j * ncta < p.n_tiles) issue_res(cta0 + j * ncta, j);
+      uint32_t it = 0;
+      for (int tile = cta0; tile < p.n_tiles; tile += ncta, ++it) {
+        const uint32_t b = NB > 1 ? it % NB : 0;
+        mbar_wait(&staged[b], (it / NB) & 1);
+        int m0, nt, g;
+        decode_tile(p, tile, m0, nt, g);
+        const int n0 = nt * BN, ng0 = g * p.Cg_out + n0;
+        const int nsub = (min(BN, p.Cg_out - n0) + 63) / 64;
+        const uint32_t sb = sO + b * (uint32_t)(BM * BN * 2);
+        for (int st = 0; st < nsub; ++st) {
+          if constexpr (AMODE == A_ROWVIEW)  // 3-D output map {C, Wo, rows}: q >= Wo clipped
+            tma_store_3d(&tmap_y, ng0 + st * 64, (m0 / BM) % p.segs * BM, (m0 / BM) / p.segs, sb + st * BM * 128);
+          else
+            tma_store_2d(&tmap_y, ng0 + st * 64, m0, sb + st * BM * 128);
+        }
+        bulk_commit();
+        if (NB == 1) {  // this tile's buffer, once its stores have read it, serves the next tile
+          bulk_wait_read0();
+          if (has_res) {
+            if (tile + ncta < p.n_tiles) issue_res(tile + ncta, 0);
+          } else {
+            mbar_arrive(&sfree[0]);
+          }
+        } else {  // buffer (it + NB - 1) % NB held tile it - 1: refill it for tile it + NB - 1
+          if (it >= 1) bulk_wait_read<1>();
+          const uint32_t fb = (it + NB - 1) % NB;
+          if (has_res) {
+            if (tile + (NB - 1) * ncta < p.n_tiles) issue_res(tile + (NB - 1) * ncta, fb);
+          } else if (it >= 1) {
+            mbar_arrive(&sfree[fb]);
+          }
+        }
+      }
+      bulk_wait0();
+    }
     if constexpr (BRES) {
       // resident weights: the B slice of this CTA's (fixed) N tile, once
       if (threadIdx.x == 0) {
@@ -289,6 +360,15 @@ __global__ void __launch_bounds__(kThreads, 1)
           int m0, nt, g;
           decode_tile(p, tile, m0, nt, g);
           const int n0 = nt * BN;
+          if (BRES && p.apf > 0 && nt == 0) {
+            const int tf = tile + p.apf * ncta;
+            if (tf < p.n_tiles) {
+              int mf, ntf, gf;
+              decode_tile(p, tf, mf, ntf, gf);
+              const int rows = min(BM, p.M - mf);
+              prefetch_l2_range(p.x + (size_t)mf * p.Cin, (uint64_t)rows * p.Cin * 2);
+            }
+          }
           for (int kb = 0; kb < p.nkb; ++kb, ++gk) {
             const int stage = gk % S;
             if (gk >= (uint32_t)S) mbar_wait(&empty[stage], ((gk / S) - 1) & 1);
@@ -301,7 +381,11 @@ __global__ void __launch_bounds__(kThreads, 1)
               continue;
             }
             mbar_arrive_expect_tx(&full[stage], C::kStageBytes);
-            tma_load_2d(sA + stage * C::kABytes, &tmap_a, g * p.Cg_in + kb * BK, m0, &full[stage]);
+            if (BRES && p.amc)  // this CTA's half of the A rows, multicast to the pair (same M tile)
+              tma_load_2d_mc(sA + stage * C::kABytes + crank * (BM / 2) * 128, &tmap_a, kb * BK,
+                             m0 + (int)crank * (BM / 2), &full[stage], (uint16_t)3);
+            else
+              tma_load_2d(sA + stage * C::kABytes, &tmap_a, g * p.Cg_in + kb * BK, m0, &full[stage]);
             if constexpr (!BRES) load_b(stage, kb, g * p.Cg_out + n0);
           }
         }
@@ -334,7 +418,12 @@ __global__ void __launch_bounds__(kThreads, 1)
               continue;
             }
             mbar_arrive_expect_tx(&full[stage], C::kStageBytes);
-            if (kb < p.nkb1)
+            if (BRES && p.amc) {  // stride 1: this CTA's half of the A rows of either source, multicast
+              const uint32_t dst = sA + stage * C::kABytes + crank * (BM / 2) * 128;
+              const int mr = m0 + (int)crank * (BM / 2);
+              if (kb < p.nkb1) tma_load_2d_mc(dst, &tmap_a, kb * BK, mr, &full[stage], (uint16_t)3);
+              else tma_load_2d_mc(dst, &tmap_r, (kb - p.nkb1) * BK, mr, &full[stage], (uint16_t)3);
+            } else if (kb < p.nkb1)
               tma_load_2d(sA + stage * C::kABytes, &tmap_a, kb * BK, m0, &full[stage]);
             else if (p.cat_im2col)
               tma_load_im2col_4d(sA + stage * C::kABytes, &tmap_r, (kb - p.nkb1) * BK, wo * p.stride, ho * p.stride,
@@ -796,7 +885,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
           if constexpr (kRing) {
             if constexpr (CG2) tc_commit_cg2_warp(&empty[stage], (uint16_t)3);  // both CTAs' stages are free
-            else if (p.mc) tc_commit_mc_warp(&empty[stage], (uint16_t)3);
+            else if (p.mc || p.amc) tc_commit_mc_warp(&empty[stage], (uint16_t)3);
             else tc_commit_warp(&empty[stage]);
           }
           ++gk;
@@ -863,7 +952,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           tma_load_2d(sO + b * (uint32_t)(BM * BN * 2) + st * BM * 128, &tmap_r, tng0 + st * 64, tm0, &rbar[b]);
       };
       if constexpr (TMA_EPI) {
-        if (et == 0) {
+        if (et == 0 && !sthr) {
           if (NB == 1) {
             bulk_wait_read0();  // the previous tile's stores no longer read the staging buffer
             if (has_res) issue_res(tile, 0);
@@ -893,7 +982,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       float* ss = sbuf + sb * 2 * BN;
       const bool reload = (sb == 0 ? loaded0 : loaded1) != ng0;
       if (reload) {
-        if (!TMA_EPI) named_bar_sync(gbar, gthreads);  // every warp of the group is done with the buffer
+        if (!TMA_EPI || sthr) named_bar_sync(gbar, gthreads);  // every warp of the group is done with the buffer
         for (int i = gt; i < 2 * BN; i += gthreads) {
           const int c = i < BN ? i : i - BN;
           ss[i] = c < nvalid_tile ? (i < BN ? p.scale[ng0 + c] : p.shift[ng0 + c]) : 0.f;
@@ -901,7 +990,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (sb == 0) loaded0 = ng0;
         else loaded1 = ng0;
       }
-      if (TMA_EPI || reload) named_bar_sync(gbar, gthreads);
+      if ((TMA_EPI && !sthr) || reload) named_bar_sync(gbar, gthreads);
       int mo = m0 + row;
       bool rvalid = mo < p.M;
       if constexpr (AMODE == A_HALO) {  // padded-width position -> output pixel (columns >= Wo discarded)
@@ -925,6 +1014,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       uint4 rres[4] = {};
       if constexpr (TMA_EPI) {
         if (has_res) mbar_wait(&rbar[ob], (it / NB) & 1);
+        else if (sthr && it >= (uint32_t)NB) mbar_wait(&sfree[ob], ((it / NB) - 1) & 1);  // its last store read it
       } else if (has_res && rvalid) {
 #pragma unroll
         for (int j = 0; j < 4; ++j)
@@ -1023,7 +1113,11 @@ __global__ void __launch_bounds__(kThreads, 1)
         if constexpr (CG2) mbar_arrive_cluster(mapa_u32(smem_u32(&tempty[acc]), 0));  // the leader's barrier
         else mbar_arrive(&tempty[acc]);
       }
-      if constexpr (TMA_EPI) {
+      if (TMA_EPI && sthr) {  // hand the staged tile to the store thread
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&staged[ob]);
+      } else if constexpr (TMA_EPI) {
         fence_proxy_async_smem();
         named_bar_sync(1, kEpiThreads);
         if (et == 0) {
@@ -1090,11 +1184,11 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
       }
     }
-    if (TMA_EPI && et == 0) bulk_wait0();
+    if (TMA_EPI && !sthr && et == 0) bulk_wait0();
   }
   tc_fence_before();
   __syncthreads();
-  if (p.mc) cluster_sync_all();  // no multicast write or commit arrival may target an exited partner
+  if (p.mc || p.amc) cluster_sync_all();  // no multicast write or commit arrival may target an exited partner
   if (warp == 4) {
     if constexpr (CG2) tmem_dealloc_cg2(tmem_base, C::kTmemCols);
     else tmem_dealloc(tmem_base, C::kTmemCols);
@@ -1209,6 +1303,11 @@ static bool use_mc(const ConvLayer& L, int amode, int rkb, const ConvParams& p) 
          (amode == A_TMA || amode == A_IM2COL || amode == A_CAT || (amode == A_HALO && env_flag("VISTA_MC_HALO", true))) &&
          (int64_t)p.n_nt * ((p.n_mt + 1) / 2) >= num_sms() / 2;
 }
+// L2 prefetch distance of the resident-weight A_TMA launches in tiles (ConvParams::apf; VISTA_APF, 0 = off)
+static const int g_apf = [] {
+  const char* e = getenv("VISTA_APF");
+  return e ? atoi(e) : 2;
+}();
 // VISTA_WRES=0 disables the resident-weight launches (A/B measurements)
 static const bool g_wres_enabled = [] {
   const char* e = getenv("VISTA_WRES");
@@ -1339,6 +1438,24 @@ static void launch_t(const ConvLayer& L, const CUtensorMap& ta, const CUtensorMa
   if (RKB > 0) {  // every CTA keeps one N tile: grid a multiple of the N-tile count (groups == 1)
     if (p.nkb > RKB || p.n_nt > grid) fail(1, "conv: resident-weight launch misconfigured");
     grid -= grid % p.n_nt;
+  }
+  if (p.amc) {  // A-multicast pairs: clusters of two CTAs with adjacent N tiles (n_nt even, so grid even)
+    if (RKB == 0 || p.n_nt % 2) fail(1, "conv: A multicast needs resident weights and an even N-tile count");
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid, 1, 1);
+    cfg.blockDim = dim3(kThreads, 1, 1);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    VCHECK(cudaLaunchKernelEx(&cfg, kern, L.tmap_w, ta, ty, tr, p));
+    LAUNCHED();
+    return;
   }
   kern<<<grid, kThreads, smem, st>>>(L.tmap_w, ta, ty, tr, p);
   LAUNCHED();
@@ -1619,6 +1736,12 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
     if (amode == A_HALO && L.BN == 64 && p.nkb == 9) rkb = 9;
     else if ((amode == A_TMA || amode == A_ROWVIEW) && tma_epi && L.BN <= 128 && p.nkb <= 4) rkb = 4;
   }
+  if (rkb == 4 && amode == A_TMA && L.groups == 1) p.apf = g_apf;
+  p.no_sthr = env_flag("VISTA_STORE_THR", true) ? 0 : 1;
+  if (rkb == 4 && amode == A_TMA && p.n_nt % 2 == 0 && !fuse_tap && !p.dbg && env_flag("VISTA_AMC", true)) {
+    p.amc = 1;  // A multicast across the pair's two N tiles (see ConvParams::amc): half-row A boxes
+    make_tmap(&ta, x, (uint64_t)L.Cin, (uint64_t)M, BM / 2);
+  }
   if (!fuse_tap && use_mc(L, amode, rkb, p)) {
     p.mc = 1;
     p.n_tiles = p.n_nt * ((p.n_mt + 1) / 2);
@@ -1715,6 +1838,7 @@ void conv_cat_forward(const ConvLayer& L, int Cx, const bf16* b, const bf16* x, 
   p.nkb = L.Kp / BK;
   p.nkb1 = Kb / BK;
   p.cat_im2col = stride != 1;
+  p.no_sthr = env_flag("VISTA_STORE_THR", true) ? 0 : 1;
   const int64_t M = (int64_t)N * p.Ho * p.Wo;
   if (M <= 0) return;
   if (M > INT32_MAX - BM) fail(1, "conv_cat: M too large for one launch");
@@ -1733,6 +1857,11 @@ void conv_cat_forward(const ConvLayer& L, int Cx, const bf16* b, const bf16* x, 
   else ty = L.tmap_w;  // unused
   const int rkb = (g_wres_enabled && tma_epi && L.BN <= 128 && p.nkb <= 4 && p.n_nt <= num_sms() &&
                    p.n_tiles >= num_sms()) ? 4 : 0;
+  if (rkb == 4 && stride == 1 && p.n_nt % 2 == 0 && !p.dbg && env_flag("VISTA_AMC", true)) {
+    p.amc = 1;  // A multicast across the pair's two N tiles (see ConvParams::amc): half-row A boxes
+    make_tmap(&ta, b, (uint64_t)Kb, (uint64_t)M, BM / 2);
+    make_tmap(&tr, x, (uint64_t)Cx, (uint64_t)M, BM / 2);
+  }
   if (use_mc(L, A_CAT, rkb, p)) {
     p.mc = 1;
     p.n_tiles = p.n_nt * ((p.n_mt + 1) / 2);

@@ -90,7 +90,9 @@ def test_conv_deterministic():
 
 
 @pytest.mark.parametrize("N,H,C,Cout,res", [(3, 14, 256, 1024, True), (5, 7, 512, 2048, True), (2, 9, 64, 128, False),
-                                            (4, 13, 128, 256, False)])
+                                            (4, 13, 128, 256, False),
+                                            (64, 7, 512, 2048, True),     # CTA-pair launch (cg2), phantom tile
+                                            (97, 14, 256, 1024, True)])   # resident weights, many tiles
 def test_fused_tap_bit_exact(N, H, C, Cout, res):
     # the conv4_6 / conv5_x producers: 1x1 convs with residual + ReLU; the tap fused into the epilogue
     # must equal the standalone tap of the same bf16 output bit for bit (max is exact), and the oracle's
@@ -178,4 +180,20 @@ def test_pair_mma_bn256_bit_identical(monkeypatch, N, H, C, Cout, k, stride, res
     for cg2 in ("1", "0"):
         monkeypatch.setenv("VISTA_CG2", cg2)
         out[cg2] = vista_conv2d(x, w, scale, shift, stride, pad, 1, residual=r, relu=True).view(torch.int16).cpu()
+    assert torch.equal(out["1"], out["0"])
+
+
+@pytest.mark.parametrize("N,H,C,Cout", [(13, 14, 256, 1024), (6, 28, 128, 512), (97, 14, 256, 1024)])
+def test_a_multicast_bit_identical(monkeypatch, N, H, C, Cout):
+    # resident-weight 1x1 convs with an even N-tile count run as CTA pairs that multicast each A k-block
+    # (VISTA_AMC default on): the same MMAs on the same operands as unicast A loads
+    x, _ = bf(rng.standard_normal((N, H, H, C)))
+    w, _ = bf(rng.standard_normal((Cout, 1, 1, C)) * (2.0 / C) ** 0.5)
+    scale = torch.from_numpy(rng.uniform(0.5, 1.5, Cout).astype(np.float32)).cuda()
+    shift = torch.from_numpy(rng.standard_normal(Cout).astype(np.float32) * 0.1).cuda()
+    r = bf(rng.standard_normal((N, H, H, Cout)))[0]
+    out = {}
+    for amc in ("1", "0"):
+        monkeypatch.setenv("VISTA_AMC", amc)
+        out[amc] = vista_conv2d(x, w, scale, shift, 1, 0, 1, residual=r, relu=True).view(torch.int16).cpu()
     assert torch.equal(out["1"], out["0"])

@@ -1306,7 +1306,7 @@ static bool use_mc(const ConvLayer& L, int amode, int rkb, const ConvParams& p) 
 // L2 prefetch distance of the resident-weight A_TMA launches in tiles (ConvParams::apf; VISTA_APF, 0 = off)
 static const int g_apf = [] {
   const char* e = getenv("VISTA_APF");
-  return e ? atoi(e) : 2;
+  return e ? atoi(e) : 0;  // measured neutral with the store-thread epilogue: off by default
 }();
 // VISTA_WRES=0 disables the resident-weight launches (A/B measurements)
 static const bool g_wres_enabled = [] {
@@ -1738,7 +1738,7 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   }
   if (rkb == 4 && amode == A_TMA && L.groups == 1) p.apf = g_apf;
   p.no_sthr = env_flag("VISTA_STORE_THR", true) ? 0 : 1;
-  if (rkb == 4 && amode == A_TMA && p.n_nt % 2 == 0 && !fuse_tap && !p.dbg && env_flag("VISTA_AMC", true)) {
+  if (rkb == 4 && amode == A_TMA && p.n_nt % 2 == 0 && !fuse_tap && !p.dbg && env_flag("VISTA_AMC", false)) {
     p.amc = 1;  // A multicast across the pair's two N tiles (see ConvParams::amc): half-row A boxes
     make_tmap(&ta, x, (uint64_t)L.Cin, (uint64_t)M, BM / 2);
   }
@@ -1857,7 +1857,7 @@ void conv_cat_forward(const ConvLayer& L, int Cx, const bf16* b, const bf16* x, 
   else ty = L.tmap_w;  // unused
   const int rkb = (g_wres_enabled && tma_epi && L.BN <= 128 && p.nkb <= 4 && p.n_nt <= num_sms() &&
                    p.n_tiles >= num_sms()) ? 4 : 0;
-  if (rkb == 4 && stride == 1 && p.n_nt % 2 == 0 && !p.dbg && env_flag("VISTA_AMC", true)) {
+  if (rkb == 4 && stride == 1 && p.n_nt % 2 == 0 && !p.dbg && env_flag("VISTA_AMC", false)) {
     p.amc = 1;  // A multicast across the pair's two N tiles (see ConvParams::amc): half-row A boxes
     make_tmap(&ta, b, (uint64_t)Kb, (uint64_t)M, BM / 2);
     make_tmap(&tr, x, (uint64_t)Cx, (uint64_t)M, BM / 2);

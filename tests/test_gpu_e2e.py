@@ -276,8 +276,8 @@ def test_weight_multicast_bit_identical(monkeypatch):
     # units); VISTA_CG2=0 keeps multicast pairs of cta_group::1 MMAs: all three must agree bit for bit.
     tab = gen.make_tables(600, 8)
     out, feats = {}, None
-    # A multicast (resident-weight 1x1 convs and stride-1 projection units, pairs of N tiles) is on by default too
-    for mode, env in (("cg2", {}), ("mc", {"VISTA_CG2": "0"}), ("unicast", {"VISTA_MC": "0", "VISTA_AMC": "0"})):
+    # A multicast (resident-weight 1x1 convs and stride-1 projection units, pairs of N tiles; opt-in) rides along
+    for mode, env in (("cg2", {"VISTA_AMC": "1"}), ("mc", {"VISTA_CG2": "0"}), ("unicast", {"VISTA_MC": "0"})):
         for key in ("VISTA_MC", "VISTA_CG2", "VISTA_AMC"):
             monkeypatch.delenv(key, raising=False)
         for key, val in env.items():

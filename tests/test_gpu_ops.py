@@ -186,7 +186,7 @@ def test_pair_mma_bn256_bit_identical(monkeypatch, N, H, C, Cout, k, stride, res
 @pytest.mark.parametrize("N,H,C,Cout", [(13, 14, 256, 1024), (6, 28, 128, 512), (97, 14, 256, 1024)])
 def test_a_multicast_bit_identical(monkeypatch, N, H, C, Cout):
     # resident-weight 1x1 convs with an even N-tile count run as CTA pairs that multicast each A k-block
-    # (VISTA_AMC default on): the same MMAs on the same operands as unicast A loads
+    # (VISTA_AMC=1, opt-in: measured neutral): the same MMAs on the same operands as unicast A loads
     x, _ = bf(rng.standard_normal((N, H, H, C)))
     w, _ = bf(rng.standard_normal((Cout, 1, 1, C)) * (2.0 / C) ** 0.5)
     scale = torch.from_numpy(rng.uniform(0.5, 1.5, Cout).astype(np.float32)).cuda()

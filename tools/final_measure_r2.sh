@@ -14,7 +14,7 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --lo
     python bench.py $ARGS > $OUT/ncu_launches.log 2>&1
 timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none \
     -k regex:"conv_tc|res_chain|conv1_pool" --csv --log-file $OUT/conv_dram.csv python bench.py $ARGS > $OUT/ncu_dram.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:"conv_tc_kernel<\(int\)256, \(int\)4" -s 4 -c 1 \
+timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k regex:"conv_tc_kernel<\(int\)256, \(int\)4" -s 4 -c 1 \
     -o $OUT/conv_full python bench.py --images 3072 $ARGS > $OUT/ncu_full.log 2>&1
 ncu -i $OUT/conv_full.ncu-rep --page raw --csv > $OUT/conv_full.raw.csv 2>/dev/null
 ncu -i $OUT/conv_full.ncu-rep --page details --csv > $OUT/conv_full.details.csv 2>/dev/null

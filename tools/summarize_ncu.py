@@ -35,10 +35,11 @@ def main():
     src, tag = sys.argv[1], sys.argv[2]
     prof = os.path.join(ROOT, "profiles")
     os.makedirs(prof, exist_ok=True)
+    cmd = sys.argv[3] if len(sys.argv) > 3 else "bash tools/profile_gpu.sh"
     md = [f"# ncu evidence, {tag}", "",
-          "Command: `bash tools/profile_gpu.sh` under gpurun on one B200 (bench.py default workload: ResNet50 "
-          "top-5, 20k images; `--steps 1 --warmup 0 --e2e-steps 1`, i.e. 3 executions of the step: timed, e2e, "
-          "instrumented). ncu times are cold-cache and serialised: compare shares, not absolutes.", ""]
+          f"Command: `{cmd}` under gpurun on one B200 (bench.py default workload: ResNet50 top-5, 20k images; "
+          "the launch list and the DRAM pass cover every step execution of that bench command, see the launch "
+          "count). ncu times are cold-cache and serialised: compare shares, not absolutes.", ""]
     # ---- 1. launch list ----
     L = read_ncu_csv(os.path.join(src, "launches.csv"))
     with open(os.path.join(prof, f"{tag}_launches.csv"), "w", newline="") as f:
@@ -52,7 +53,7 @@ def main():
         agg[k][0] += 1
         agg[k][1] += float(d["Metric Value"] or 0)
     tot = sum(v[1] for v in agg.values())
-    md += ["## 1. Launch list (all kernels of the 3 step executions)", "",
+    md += ["## 1. Launch list (all kernels of the profiled step executions)", "",
            f"{len(L)} launches, {tot / 1e6:.1f} ms of device time.", "",
            "| kernel | launches | ms | share |", "|---|---|---|---|"]
     for k, v in sorted(agg.items(), key=lambda x: -x[1][1]):
@@ -67,19 +68,24 @@ def main():
     t_ns = sum(v.get("gpu__time_duration.sum", 0) for v in per.values())
     rd = sum(v.get("dram__bytes_read.sum", 0) for v in per.values())
     wr = sum(v.get("dram__bytes_write.sum", 0) for v in per.values())
-    md += ["", "## 2. DRAM traffic of every conv_tc_kernel launch", "",
-           f"{n} launches (3 step executions), {t_ns / 1e6:.1f} ms, dram read {rd / 1e9:.1f} GB, "
+    md += ["", "## 2. DRAM traffic of every conv-class launch (conv_tc_kernel, res_chain_kernel, conv1_pool_kernel)", "",
+           f"{n} launches, {t_ns / 1e6:.1f} ms, dram read {rd / 1e9:.1f} GB, "
            f"write {wr / 1e9:.1f} GB -> {(rd + wr) / n / 1e6:.2f} MB per launch on average, "
            f"{(rd + wr) / (t_ns * 1e-9) / 1e12:.2f} TB/s while running.", ""]
     summary = {"tag": tag, "dominant": {
         "kernel": "conv_tc_kernel", "launches": n, "dram_bytes_per_launch": (rd + wr) / n if n else None,
         "dram_read_bytes": rd, "dram_write_bytes": wr, "ncu_ms": t_ns / 1e6,
-        "note": "dram__bytes_read.sum + dram__bytes_write.sum per launch, averaged over every conv launch "
-                "of 3 bench step executions (ncu, --clock-control none)"}}
+        "note": "dram__bytes_read.sum + dram__bytes_write.sum per launch, averaged over every conv-class launch "
+                "(conv_tc, res_chain, conv1_pool) of the profiled bench step executions (ncu, --clock-control none)"}}
     # ---- 3. the --set full capture ----
     rep = os.path.join(src, "conv_full.ncu-rep")
+    raw_csv = os.path.join(src, "conv_full.raw.csv")
+    raw = None
     if os.path.exists(rep):
         raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    elif os.path.exists(raw_csv):  # the capture scripts export the raw page and delete the report
+        raw = open(raw_csv).read()
+    if raw:
         rows = list(csv.reader(raw.splitlines()))
         if len(rows) >= 3:
             hdr, units, vals = rows[0], rows[1], rows[2]
@@ -89,7 +95,7 @@ def main():
                     "sm__throughput.avg.pct_of_peak_sustained_elapsed",
                     "lts__throughput.avg.pct_of_peak_sustained_elapsed", "launch__registers_per_thread",
                     "launch__shared_mem_per_block_dynamic", "sm__warps_active.avg.pct_of_peak_sustained_active"]
-            md += ["", "## 3. `ncu --set full` on one conv launch (`-k regex:conv_tc -s 4 -c 1`, 1024 images)", "",
+            md += ["", "## 3. `ncu --set full` on one launch of the top conv kernel (res4 3x3, CTA-pair im2col; 1024-image micro-batch)", "",
                    "| metric | value |", "|---|---|"]
             full = {}
             for w_ in want:

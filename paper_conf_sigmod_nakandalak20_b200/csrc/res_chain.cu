@@ -23,7 +23,9 @@ namespace vista {
 namespace {
 
 constexpr int BMr = 128, BKr = 64;
-constexpr int kEpiW0 = 2, kEpiWn = 8, kEpiT = kEpiWn * 32, kThr = (kEpiW0 + kEpiWn) * 32;
+// warps: 0 producer, 1 MMA issuer, 2..9 epilogue, 10 store warp (lane 0: the out / a_next TMA stores and the
+// staging-buffer releases, so the epilogue warps never wait on store completion or on one another)
+constexpr int kEpiW0 = 2, kEpiWn = 8, kEpiT = kEpiWn * 32, kStoreW = kEpiW0 + kEpiWn, kThr = (kStoreW + 1) * 32;
 
 // V = 0: b tile double-buffered; V = 1: b single-buffered, the freed 16/32 KB spent on one more
 // weight stage (MID = 64) or one more out/residual staging buffer (MID = 128: residual chunks in flight).
@@ -42,7 +44,7 @@ struct RC {
   static constexpr int kA = MID == 256 ? 0 : BMr * MID * 2;  // a_next tile (none for MID = 256)
   static constexpr int offB = 0, offO = offB + NBB * kB, offA = offO + NB * kO, offW = offA + kA,
                        offS = offW + WS * 16384, offBar = offS + (5 * MID) * 2 * 4;
-  static constexpr int nBar = 2 + 2 + NB * 3 + 2 * WS + 2 + 1 + 1 + 2;
+  static constexpr int nBar = 2 + 2 + NB * 3 + 2 * WS + 2 + 1 + 1 + 2 + NB + 2;
   static constexpr int kSmem = offBar + nBar * 8 + 16 + 1024;
   static_assert(kSmem <= 227 * 1024, "res_chain smem");
 };
@@ -54,6 +56,7 @@ struct RCParams {
   const float* sh_a;
   int M, n_mt;
   int has_a;  // 0: closing conv only (last unit of a stage: no chained opening conv, no a_next)
+  int sthr;   // 1: store warp (VISTA_STORE_THR, default on); 0: epilogue thread 0 issues the stores
 };
 
 template <int MID, int V>
@@ -86,7 +89,10 @@ __global__ void __launch_bounds__(kThr, 1)
   uint64_t* tfull_a = tfull_c + 2;  // [1]
   uint64_t* tempty_a = tfull_a + 1; // [1]
   uint64_t* tempty_c = tempty_a + 1;  // [2]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty_c + 2);
+  uint64_t* staged = tempty_c + 2;  // [NB] store warp: the epilogue warps staged out chunk b
+  uint64_t* astaged = staged + NB;  // [1] store warp: a_next tile staged
+  uint64_t* afree = astaged + 1;    // [1] the previous a_next store has read the a_next staging tile
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(afree + 1);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
@@ -107,6 +113,9 @@ __global__ void __launch_bounds__(kThr, 1)
     }
     mbar_init(tfull_a, 1);
     mbar_init(tempty_a, kEpiWn);
+    for (int i = 0; i < NB; ++i) mbar_init(&staged[i], kEpiWn);
+    mbar_init(astaged, kEpiWn);
+    mbar_init(afree, 1);
     fence_mbar_init();
   }
   for (int i = threadIdx.x; i < 5 * MID * 2; i += blockDim.x) {
@@ -230,6 +239,34 @@ __global__ void __launch_bounds__(kThr, 1)
         if (kCanA && p.has_a) issue_a(j);
       }
     }
+  } else if (warp == kStoreW) {
+    // ================= store warp =================
+    if (lane == 0 && p.sthr) {
+      uint32_t it = 0;
+      for (int tile = blockIdx.x; tile < p.n_mt; tile += gridDim.x, ++it) {
+        const int m0 = tile * BMr;
+        for (int j = 0; j < NCH; ++j) {
+          const uint32_t qq = it * NCH + j, ob = qq % NB;
+          const uint32_t so = sO + ob * C::kO;
+          mbar_wait(&staged[ob], (qq / NB) & 1);
+          if (kCanA && p.has_a) mbar_arrive(&oready[ob]);  // staged chunk may feed the a-MMA
+          tma_store_2d(&tm_out, j * 128, m0, so);
+          tma_store_2d(&tm_out, j * 128 + 64, m0, so + BMr * 128);
+          bulk_commit();
+          if (qq >= 1) {
+            bulk_wait_read<1>();  // every earlier store (the previous chunk's, the previous a_next) has read its tile
+            mbar_arrive(&ofree[(qq - 1) % NB]);
+            if (j == 0 && kCanA && p.has_a) mbar_arrive(afree);
+          }
+        }
+        if (kCanA && p.has_a) {
+          mbar_wait(astaged, it & 1);
+          for (int s2 = 0; s2 < MID / 64; ++s2) tma_store_2d(&tm_a, s2 * 64, m0, sAo + s2 * BMr * 128);
+          bulk_commit();
+        }
+      }
+      bulk_wait0();
+    }
   } else {
     // ================= epilogue (8 warps) =================
     const int et = threadIdx.x - kEpiW0 * 32;
@@ -263,6 +300,11 @@ __global__ void __launch_bounds__(kThr, 1)
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty_c[acc]);
         fence_proxy_async_smem();
+        if (p.sthr) {  // hand the staged chunk to the store warp
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&staged[ob]);
+          continue;
+        }
         named_bar_sync(1, kEpiT);
         if (et == 0) {
           // the previous chunk's store must have read its buffer before that buffer is refilled
@@ -281,8 +323,12 @@ __global__ void __launch_bounds__(kThr, 1)
       // ---- a_next = ReLU(BN_a(acc_a)) ----
       mbar_wait(tfull_a, it & 1);
       tc_fence_after();
-      if (et == 0) bulk_wait_read<NCH>();  // the previous tile's a_next store has read the staging tile
-      named_bar_sync(1, kEpiT);
+      if (p.sthr) {
+        if (it >= 1) mbar_wait(afree, (it - 1) & 1);  // the previous tile's a_next store has read the staging tile
+      } else {
+        if (et == 0) bulk_wait_read<NCH>();
+        named_bar_sync(1, kEpiT);
+      }
 #pragma unroll
       for (int cc = 0; cc < MID / 64; ++cc) {
         const int cb = half * (MID / 64) + cc;  // 32-column block of the MID-wide accumulator
@@ -301,13 +347,18 @@ __global__ void __launch_bounds__(kThr, 1)
       __syncwarp();
       if (lane == 0) mbar_arrive(tempty_a);
       fence_proxy_async_smem();
+      if (p.sthr) {
+        __syncwarp();
+        if (lane == 0) mbar_arrive(astaged);
+        continue;
+      }
       named_bar_sync(1, kEpiT);
       if (et == 0) {
         for (int s = 0; s < MID / 64; ++s) tma_store_2d(&tm_a, s * 64, m0, sAo + s * BMr * 128);
         bulk_commit();
       }
     }
-    if (et == 0) bulk_wait0();
+    if (et == 0 && !p.sthr) bulk_wait0();
   }
   tc_fence_before();
   __syncthreads();
@@ -335,6 +386,8 @@ static void launch_chain(const ConvLayer& Lc, const ConvLayer* La, const bf16* b
     fail(5, "res_chain: tensor map encoding failed");
   RCParams p;
   p.has_a = La ? 1 : 0;
+  const bool sthr = !(getenv("VISTA_STORE_THR") && getenv("VISTA_STORE_THR")[0] == '0');
+  p.sthr = sthr ? 1 : 0;
   p.sc_c = Lc.scale;
   p.sh_c = Lc.shift;
   p.sc_a = La ? La->scale : Lc.scale;  // (unused without a_next; any MID-long device array)

@@ -267,6 +267,21 @@ def test_resnet_projection_fused(monkeypatch):
         assert not np.array_equal(a, b) or k == 4  # the fused path really ran
 
 
+def test_store_thread_epilogue_bit_identical(monkeypatch):
+    # the TMA-epilogue convs and the res_chain kernels hand their staged tiles to a store thread / warp
+    # (VISTA_STORE_THR, default on) instead of storing from epilogue thread 0 behind named barriers: the same
+    # bytes reach HBM, so every MM_l bit must agree (ResNet50: chains, projection units, 1x1 TMA epilogues)
+    tab = gen.make_tables(300, 8)
+    out = {}
+    for flag in ("1", "0"):
+        monkeypatch.setenv("VISTA_STORE_THR", flag)
+        v = run_gpu(2, [0, 1, 2, 3, 4], tab, 8, iters=1, micro_batch=300)
+        out[flag] = [v.features(k)["mm"].view(torch.int16).cpu().clone() for k in range(5)]
+        v.close()
+    for a, b in zip(out["1"], out["0"]):
+        assert torch.equal(a, b)
+
+
 def test_weight_multicast_bit_identical(monkeypatch):
     # 2-CTA weight multicast (ConvParams::mc) engages only for launches with >= 74 pair tiles: 600 images put
     # the res4 / res5 / projection-unit launches above that, and res4's 919 M tiles give rank 1 of the last

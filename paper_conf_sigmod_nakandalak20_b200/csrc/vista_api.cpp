@@ -279,6 +279,7 @@ struct vista_ctx {
   // compute stream waits on, so the copy of micro-batch i + 1 overlaps the inference of micro-batch i
   cudaStream_t copy_stream = nullptr;
   std::vector<cudaEvent_t> px_ready;
+  std::vector<int64_t> px_bounds;  // image offsets of the copied segments of the last stream_host_pixels, + end
   cudaEvent_t px_free = nullptr;  // the previous transfer's compute is done with d_px
   bool own_stream = false;
   int64_t n_img = 0, n_str = 0;
@@ -809,7 +810,10 @@ bool run_ops(vista_ctx* c, int t, const void* in_ptr, void* out_ptr, int nb, voi
 // Host pixels of images [c0, c0 + nc) -> c->d_px, one stage-1 micro-batch per copy on c->copy_stream, each
 // followed by c->px_ready[j]; the compute stream waits on event j right before micro-batch j, so the copy of
 // micro-batch j + 1 overlaps the inference of micro-batch j.  Returns the events.
-const std::vector<cudaEvent_t>* stream_host_pixels(vista_ctx* c, const uint8_t* images, int64_t c0, int64_t nc) {
+// split_first (Staged stage 1): the first micro-batch is copied -- and then inferred -- as three segments of
+// B/4, B/4 and B/2 images, so stage 1 starts after a quarter of the first copy instead of all of it
+const std::vector<cudaEvent_t>* stream_host_pixels(vista_ctx* c, const uint8_t* images, int64_t c0, int64_t nc,
+                                                   bool split_first = false) {
   const size_t px_img = (size_t)c->net.stages[0].in_elems;
   c->d_px.ensure((size_t)nc * px_img);
   if (!c->copy_stream) {
@@ -820,17 +824,24 @@ const std::vector<cudaEvent_t>* stream_host_pixels(vista_ctx* c, const uint8_t* 
   VCHECK(cudaEventRecord(c->px_free, c->stream));
   VCHECK(cudaStreamWaitEvent(c->copy_stream, c->px_free, 0));
   const int64_t B0 = std::max(c->micro[0], 1);
-  const size_t nev = (size_t)((nc + B0 - 1) / B0);
+  c->px_bounds.clear();
+  if (split_first && B0 >= 8) {
+    for (int64_t b : {(int64_t)0, B0 / 4, B0 / 2})
+      if (b < nc) c->px_bounds.push_back(b);
+  }
+  for (int64_t i0 = c->px_bounds.empty() ? 0 : B0; i0 < nc; i0 += B0) c->px_bounds.push_back(i0);
+  c->px_bounds.push_back(nc);
+  const size_t nev = c->px_bounds.size() - 1;
   while (c->px_ready.size() < nev) {
     cudaEvent_t e;
     VCHECK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     c->px_ready.push_back(e);
   }
-  for (int64_t i0 = 0; i0 < nc; i0 += B0) {
-    const int64_t nb = std::min<int64_t>(B0, nc - i0);
+  for (size_t j = 0; j < nev; ++j) {
+    const int64_t i0 = c->px_bounds[j], nb = c->px_bounds[j + 1] - i0;
     VCHECK(cudaMemcpyAsync((uint8_t*)c->d_px.p + (size_t)i0 * px_img, images + (size_t)(c0 + i0) * px_img,
                            (size_t)nb * px_img, cudaMemcpyHostToDevice, c->copy_stream));
-    VCHECK(cudaEventRecord(c->px_ready[(size_t)(i0 / B0)], c->copy_stream));
+    VCHECK(cudaEventRecord(c->px_ready[j], c->copy_stream));
   }
   return &c->px_ready;
 }
@@ -845,13 +856,18 @@ bool run_block(vista_ctx* c, int t, const void* in_base, void* out_base, int64_t
   prepare_slots(c, t, B, slot);
   const size_t in_bytes_per = t == 0 ? (size_t)S.in_elems : (size_t)S.in_elems * c->esz;
   bool fused = tapf != nullptr;
-  for (int64_t i0 = 0; i0 < n; i0 += B) {
-    const int nb = (int)std::min<int64_t>(B, n - i0);
-    if (in_ready) VCHECK(cudaStreamWaitEvent(c->stream, (*in_ready)[(size_t)(i0 / B)], 0));
+  // stage 1 from streamed host pixels: the copied segments (stream_host_pixels), each within one micro-batch
+  const bool segs = in_ready && t == 0 && !c->px_bounds.empty() && c->px_bounds.back() == n;
+  size_t seg = 0;
+  for (int64_t i0 = 0; i0 < n;) {
+    const int nb = segs ? (int)(c->px_bounds[seg + 1] - i0) : (int)std::min<int64_t>(B, n - i0);
+    if (in_ready) VCHECK(cudaStreamWaitEvent(c->stream, (*in_ready)[segs ? seg : (size_t)(i0 / B)], 0));
     const bool ok = run_ops(c, t, (const uint8_t*)in_base + (size_t)i0 * in_bytes_per,
                             (uint8_t*)out_base + (size_t)i0 * S.out_elems * c->esz, nb, slot,
                             tapf ? tapf + (size_t)i0 * 4 * S.outC : nullptr);
     fused = fused && ok;
+    i0 += nb;
+    ++seg;
   }
   return fused;
 }
@@ -1230,7 +1246,7 @@ static void transfer_body(vista_ctx* c, const uint8_t* images, const void* base,
         }
         const std::vector<cudaEvent_t>* px_ev = nullptr;
         if (host_px) {  // stream the chunk's pixels to the device, one stage-1 micro-batch per copy
-          px_ev = stream_host_pixels(c, images, c0, nc);
+          px_ev = stream_host_pixels(c, images, c0, nc, /*split_first=*/true);
           pxc = (const uint8_t*)c->d_px.p;
         }
         for (int t = base ? t0 : 0; t <= c->t_max; ++t) {

@@ -32,18 +32,24 @@ constexpr int kEpiW0 = 2, kEpiWn = 8, kEpiT = kEpiWn * 32, kStoreW = kEpiW0 + kE
 // MID = 256 (ResNet res4, Cout 1024): the closing conv alone (no a_next: a 1024-wide c accumulator and the
 // a GEMM's 512 KB of weights per tile do not fit beside it), b single-buffered (64 KB); V = 0: two staging
 // buffers and five weight stages, V = 1: three and three.
-template <int MID, int V = 0>
+// CG2 (CTA pairs): each CTA holds half of every weight k-block, so weight stages are 8 KB and the space goes to a
+// fourth out/residual staging buffer (more residual chunks in flight) and, at MID = 64, a fifth weight stage.
+template <int MID, int V = 0, bool CG2 = false>
 struct RC {
   static constexpr int NCH = 4 * MID / 128;       // c chunks of 128 channels
   static constexpr int KBC = MID / BKr;           // k-blocks of the c GEMM
-  static constexpr int NBB = (V || MID == 256) ? 1 : 2;  // b tile buffers
-  static constexpr int NB = MID == 64 ? 3 : (MID == 256 ? (V ? 3 : 2) : (V ? 3 : 2));  // out/residual staging
-  static constexpr int WS = MID == 64 ? (V ? 5 : 4) : (MID == 256 ? (V ? 3 : 5) : 3);  // weight stages (16 KB)
+  // (CG2, MID = 128: b single-buffered; V = 1 four staging buffers and three weight stages, V = 0 three and seven)
+  static constexpr int NBB = (V || MID == 256 || (CG2 && MID == 128)) ? 1 : 2;  // b tile buffers
+  static constexpr int NB = CG2 ? (MID == 128 ? (V ? 4 : 3) : 4)
+                                : (MID == 64 ? 3 : (MID == 256 ? (V ? 3 : 2) : (V ? 3 : 2)));  // out/residual staging
+  static constexpr int WS = CG2 ? (MID == 64 ? 5 : (V ? 3 : 7))
+                                : (MID == 64 ? (V ? 5 : 4) : (MID == 256 ? (V ? 3 : 5) : 3));  // weight stages
+  static constexpr int kWst = CG2 ? 8192 : 16384;  // weight stage bytes
   static constexpr int kB = KBC * BMr * 128;      // b tile bytes
   static constexpr int kO = BMr * 128 * 2;        // one out chunk: two 64-channel sub-tiles
   static constexpr int kA = MID == 256 ? 0 : BMr * MID * 2;  // a_next tile (none for MID = 256)
   static constexpr int offB = 0, offO = offB + NBB * kB, offA = offO + NB * kO, offW = offA + kA,
-                       offS = offW + WS * 16384, offBar = offS + (5 * MID) * 2 * 4;
+                       offS = offW + WS * kWst, offBar = offS + (5 * MID) * 2 * 4;
   static constexpr int nBar = 2 + 2 + NB * 3 + 2 * WS + 2 + 1 + 1 + 2 + NB + 2;
   static constexpr int kSmem = offBar + nBar * 8 + 16 + 1024;
   static_assert(kSmem <= 227 * 1024, "res_chain smem");
@@ -59,15 +65,29 @@ struct RCParams {
   int sthr;   // 1: store warp (VISTA_STORE_THR, default on); 0: epilogue thread 0 issues the stores
 };
 
-template <int MID, int V>
+// CG2: CTA pairs (2-CTA clusters) run every GEMM as ONE tcgen05.mma.cta_group::2 with M = 256 over the pair's
+// two adjacent 128-pixel tiles (rank r: tile 2t + r; rank 1 past the last tile: phantom, TMA zero-fill and
+// clipped stores).  Each CTA keeps its own b tile, residual chunks, staged out chunks and TMEM accumulators
+// (its 128 rows) but loads only HALF of every weight k-block (B's N rows split between the pair): the weights
+// are 256 of the 416 KB a MID = 128 tile brings into shared memory, and per-SM TMA ingest is what bounds the
+// chain.  The leader (rank 0) waits for both CTAs' operands (its full barriers count both) and issues; commits
+// multicast to both CTAs; both epilogues / store warps arrive on the leader's tempty / oready.
+template <int MID, int V, bool CG2 = false>
 __global__ void __launch_bounds__(kThr, 1)
     res_chain_kernel(const __grid_constant__ CUtensorMap tm_b, const __grid_constant__ CUtensorMap tm_res,
                      const __grid_constant__ CUtensorMap tm_out, const __grid_constant__ CUtensorMap tm_a,
                      const __grid_constant__ CUtensorMap tm_wc, const __grid_constant__ CUtensorMap tm_wa,
                      const RCParams p) {
-  using C = RC<MID, V>;
+  using C = RC<MID, V, CG2>;
   constexpr int NCH = C::NCH, KBC = C::KBC, NB = C::NB, WS = C::WS, NBB = C::NBB;
   constexpr bool kCanA = MID <= 128;  // MID = 256: closing conv only
+  static_assert(!CG2 || kCanA, "CTA-pair chain: MID <= 128");
+  // tile walk: CTA pairs walk pair tiles t (M tile 2t + rank); unpaired CTAs walk M tiles
+  const uint32_t crank = CG2 ? (blockIdx.x & 1u) : 0u;
+  const int t0 = CG2 ? (int)(blockIdx.x >> 1) : (int)blockIdx.x;
+  const int tstep = CG2 ? (int)(gridDim.x >> 1) : (int)gridDim.x;
+  const int n_t = CG2 ? (p.n_mt + 1) / 2 : p.n_mt;
+  auto tile_m0 = [&](int t) { return (CG2 ? 2 * t + (int)crank : t) * BMr; };
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 1023u) & ~1023u;
@@ -95,24 +115,25 @@ __global__ void __launch_bounds__(kThr, 1)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(afree + 1);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  constexpr uint32_t kPair = CG2 ? 2u : 1u;  // arrivals the leader's operand / drain barriers collect
   if (threadIdx.x == 0) {
     for (int i = 0; i < 2; ++i) {
-      mbar_init(&bfull[i], 1);
+      mbar_init(&bfull[i], kPair);
       mbar_init(&bempty[i], 1);
       mbar_init(&tfull_c[i], 1);
-      mbar_init(&tempty_c[i], kEpiWn);
+      mbar_init(&tempty_c[i], kEpiWn * kPair);
     }
     for (int i = 0; i < NB; ++i) {
       mbar_init(&rfull[i], 1);
-      mbar_init(&oready[i], 1);
+      mbar_init(&oready[i], kPair);
       mbar_init(&ofree[i], p.has_a ? 2 : 1);
     }
     for (int i = 0; i < WS; ++i) {
-      mbar_init(&wfull[i], 1);
+      mbar_init(&wfull[i], kPair);
       mbar_init(&wempty[i], 1);
     }
     mbar_init(tfull_a, 1);
-    mbar_init(tempty_a, kEpiWn);
+    mbar_init(tempty_a, kEpiWn * kPair);
     for (int i = 0; i < NB; ++i) mbar_init(&staged[i], kEpiWn);
     mbar_init(astaged, kEpiWn);
     mbar_init(afree, 1);
@@ -126,7 +147,11 @@ __global__ void __launch_bounds__(kThr, 1)
     else v = p.sh_a[i - 9 * MID];
     sc_c[i] = v;
   }
-  if (warp == 1) tmem_alloc(tmem_slot, 512);
+  if constexpr (CG2) cluster_sync_all();  // both CTAs' barriers initialised; the pair allocates TMEM together
+  if (warp == 1) {
+    if constexpr (CG2) tmem_alloc_cg2(tmem_slot, 512);
+    else tmem_alloc(tmem_slot, 512);
+  }
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -136,11 +161,20 @@ __global__ void __launch_bounds__(kThr, 1)
     // ================= producer =================
     if (lane == 0) {
       uint32_t gw = 0, q = 0, it = 0;
+      // bytes: one CTA's box (CG2: half of the k-block's N rows, rows offset by rank; the leader arms its
+      // barrier for both boxes, the peer adds an arrival)
       auto push_w = [&](const CUtensorMap* m, int c0, int c1, uint32_t bytes) {
         const uint32_t st = gw % WS;
         if (gw >= (uint32_t)WS) mbar_wait(&wempty[st], ((gw / WS) - 1) & 1);
-        mbar_arrive_expect_tx(&wfull[st], bytes);
-        tma_load_2d(sW + st * 16384, m, c0, c1, &wfull[st]);
+        if constexpr (CG2) {
+          const uint32_t fl = mapa_u32(smem_u32(&wfull[st]), 0);
+          if (crank == 0) mbar_arrive_expect_tx(&wfull[st], 2 * bytes);
+          tma_load_2d_cg2(sW + st * C::kWst, m, c0, c1, fl);
+          if (crank != 0) mbar_arrive_cluster(fl);
+        } else {
+          mbar_arrive_expect_tx(&wfull[st], bytes);
+          tma_load_2d(sW + st * C::kWst, m, c0, c1, &wfull[st]);
+        }
         ++gw;
       };
       auto push_res = [&](int m0, int j) {
@@ -150,18 +184,26 @@ __global__ void __launch_bounds__(kThr, 1)
         tma_load_2d(sO + ob * C::kO, &tm_res, j * 128, m0, &rfull[ob]);
         tma_load_2d(sO + ob * C::kO + BMr * 128, &tm_res, j * 128 + 64, m0, &rfull[ob]);
       };
+      constexpr int kNc = CG2 ? 64 : 128, kNa = CG2 ? MID / 2 : MID;  // weight rows per CTA box
       auto push_c = [&](int j) {
-        for (int kb = 0; kb < KBC; ++kb) push_w(&tm_wc, kb * BKr, j * 128, 128 * 128);
+        for (int kb = 0; kb < KBC; ++kb) push_w(&tm_wc, kb * BKr, j * 128 + (int)crank * kNc, kNc * 128);
       };
       auto push_a = [&](int j) {
-        for (int h = 0; h < 2; ++h) push_w(&tm_wa, j * 128 + h * 64, 0, MID * 128);
+        for (int h = 0; h < 2; ++h) push_w(&tm_wa, j * 128 + h * 64, (int)crank * kNa, kNa * 128);
       };
-      for (int tile = blockIdx.x; tile < p.n_mt; tile += gridDim.x, ++it, q += NCH) {
-        const int m0 = tile * BMr;
+      for (int tile = t0; tile < n_t; tile += tstep, ++it, q += NCH) {
+        const int m0 = tile_m0(tile);
         const uint32_t bb = it % NBB;
         if (it >= (uint32_t)NBB) mbar_wait(&bempty[bb], ((it / NBB) - 1) & 1);
-        mbar_arrive_expect_tx(&bfull[bb], C::kB);
-        for (int kb = 0; kb < KBC; ++kb) tma_load_2d(sB + bb * C::kB + kb * BMr * 128, &tm_b, kb * BKr, m0, &bfull[bb]);
+        if constexpr (CG2) {
+          const uint32_t fl = mapa_u32(smem_u32(&bfull[bb]), 0);
+          if (crank == 0) mbar_arrive_expect_tx(&bfull[bb], 2 * C::kB);
+          for (int kb = 0; kb < KBC; ++kb) tma_load_2d_cg2(sB + bb * C::kB + kb * BMr * 128, &tm_b, kb * BKr, m0, fl);
+          if (crank != 0) mbar_arrive_cluster(fl);
+        } else {
+          mbar_arrive_expect_tx(&bfull[bb], C::kB);
+          for (int kb = 0; kb < KBC; ++kb) tma_load_2d(sB + bb * C::kB + kb * BMr * 128, &tm_b, kb * BKr, m0, &bfull[bb]);
+        }
         // weights in the order the MMA warp consumes them: c(0), then per j: c(j+1), a(j); each residual
         // chunk right after its c weights (its buffer frees up only once the a-MMA two chunks back is done)
         push_c(0);
@@ -181,16 +223,37 @@ __global__ void __launch_bounds__(kThr, 1)
         if (u + NB >= total) mbar_wait(&ofree[u % NB], (u / NB) & 1);
     }
   } else if (warp == 1) {
-    // ================= MMA issuer (whole warp, elected lane issues) =================
-    constexpr uint32_t idesc_c = umma_idesc_bf16(BMr, 128);
-    constexpr uint32_t idesc_a = umma_idesc_bf16(BMr, MID);
+    // ================= MMA issuer (whole warp, elected lane issues; CG2: the leader, for the pair) =========
+    if (!CG2 || crank == 0) {
+    constexpr uint32_t idesc_c = umma_idesc_bf16(CG2 ? 2 * BMr : BMr, 128);
+    constexpr uint32_t idesc_a = umma_idesc_bf16(CG2 ? 2 * BMr : BMr, MID);
+    // MMA + commit for both forms (CG2: one pair MMA over both CTAs, commits multicast to both)
+    auto mma4 = [&](uint32_t tacc, uint32_t a_addr, uint32_t b_addr, uint32_t idesc, uint32_t acc0) {
+      if constexpr (CG2) {
+        const uint32_t a = umma_desc_lo_sw128(a_addr), b = umma_desc_lo_sw128(b_addr);
+        tc_mma_bf16_lo_warp_cg2(tacc, a, b, idesc, acc0);
+        tc_mma_bf16_lo_warp_cg2(tacc, a + 2, b + 2, idesc, 1u);
+        tc_mma_bf16_lo_warp_cg2(tacc, a + 4, b + 4, idesc, 1u);
+        tc_mma_bf16_lo_warp_cg2(tacc, a + 6, b + 6, idesc, 1u);
+      } else {
+        const uint64_t da = umma_desc_k_sw128(a_addr), db = umma_desc_k_sw128(b_addr);
+        tc_mma_bf16_warp(tacc, da, db, idesc, acc0);
+        tc_mma_bf16_warp(tacc, da + 2, db + 2, idesc, 1u);
+        tc_mma_bf16_warp(tacc, da + 4, db + 4, idesc, 1u);
+        tc_mma_bf16_warp(tacc, da + 6, db + 6, idesc, 1u);
+      }
+    };
+    auto commit = [&](uint64_t* bar) {
+      if constexpr (CG2) tc_commit_cg2_warp(bar, (uint16_t)3);
+      else tc_commit_warp(bar);
+    };
     uint32_t gw = 0, it = 0;
     auto wait_w = [&]() -> uint32_t {
       const uint32_t st = gw % WS;
       mbar_wait(&wfull[st], (gw / WS) & 1);
       return st;
     };
-    for (int tile = blockIdx.x; tile < p.n_mt; tile += gridDim.x, ++it) {
+    for (int tile = t0; tile < n_t; tile += tstep, ++it) {
       const uint32_t bb = it % NBB, qbase = it * NCH;
       mbar_wait(&bfull[bb], (it / NBB) & 1);
       auto issue_c = [&](const int j) {
@@ -201,16 +264,12 @@ __global__ void __launch_bounds__(kThr, 1)
 #pragma unroll
         for (int kb = 0; kb < KBC; ++kb) {
           const uint32_t st = wait_w();
-          const uint64_t da = umma_desc_k_sw128(sB + bb * C::kB + kb * BMr * 128), db = umma_desc_k_sw128(sW + st * 16384);
-          tc_mma_bf16_warp(tacc, da, db, idesc_c, kb != 0 ? 1u : 0u);
-          tc_mma_bf16_warp(tacc, da + 2, db + 2, idesc_c, 1u);
-          tc_mma_bf16_warp(tacc, da + 4, db + 4, idesc_c, 1u);
-          tc_mma_bf16_warp(tacc, da + 6, db + 6, idesc_c, 1u);
-          tc_commit_warp(&wempty[st]);
+          mma4(tacc, sB + bb * C::kB + kb * BMr * 128, sW + st * C::kWst, idesc_c, kb != 0 ? 1u : 0u);
+          commit(&wempty[st]);
           ++gw;
         }
-        tc_commit_warp(&tfull_c[acc]);
-        if (j == NCH - 1) tc_commit_warp(&bempty[bb]);
+        commit(&tfull_c[acc]);
+        if (j == NCH - 1) commit(&bempty[bb]);
       };
       auto issue_a = [&](const int j) {
         const uint32_t qq = qbase + j, ob = qq % NB;
@@ -221,16 +280,12 @@ __global__ void __launch_bounds__(kThr, 1)
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
           const uint32_t st = wait_w();
-          const uint64_t da = umma_desc_k_sw128(sO + ob * C::kO + h * BMr * 128), db = umma_desc_k_sw128(sW + st * 16384);
-          tc_mma_bf16_warp(tacc, da, db, idesc_a, (j | h) != 0 ? 1u : 0u);
-          tc_mma_bf16_warp(tacc, da + 2, db + 2, idesc_a, 1u);
-          tc_mma_bf16_warp(tacc, da + 4, db + 4, idesc_a, 1u);
-          tc_mma_bf16_warp(tacc, da + 6, db + 6, idesc_a, 1u);
-          tc_commit_warp(&wempty[st]);
+          mma4(tacc, sO + ob * C::kO + h * BMr * 128, sW + st * C::kWst, idesc_a, (j | h) != 0 ? 1u : 0u);
+          commit(&wempty[st]);
           ++gw;
         }
-        tc_commit_warp(&ofree[ob]);
-        if (j == NCH - 1) tc_commit_warp(tfull_a);
+        commit(&ofree[ob]);
+        if (j == NCH - 1) commit(tfull_a);
       };
       issue_c(0);
 #pragma unroll
@@ -239,17 +294,21 @@ __global__ void __launch_bounds__(kThr, 1)
         if (kCanA && p.has_a) issue_a(j);
       }
     }
+    }
   } else if (warp == kStoreW) {
     // ================= store warp =================
     if (lane == 0 && p.sthr) {
       uint32_t it = 0;
-      for (int tile = blockIdx.x; tile < p.n_mt; tile += gridDim.x, ++it) {
-        const int m0 = tile * BMr;
+      for (int tile = t0; tile < n_t; tile += tstep, ++it) {
+        const int m0 = tile_m0(tile);
         for (int j = 0; j < NCH; ++j) {
           const uint32_t qq = it * NCH + j, ob = qq % NB;
           const uint32_t so = sO + ob * C::kO;
           mbar_wait(&staged[ob], (qq / NB) & 1);
-          if (kCanA && p.has_a) mbar_arrive(&oready[ob]);  // staged chunk may feed the a-MMA
+          if (kCanA && p.has_a) {  // staged chunk may feed the a-MMA (CG2: the leader's, which reads both)
+            if constexpr (CG2) mbar_arrive_cluster(mapa_u32(smem_u32(&oready[ob]), 0));
+            else mbar_arrive(&oready[ob]);
+          }
           tma_store_2d(&tm_out, j * 128, m0, so);
           tma_store_2d(&tm_out, j * 128 + 64, m0, so + BMr * 128);
           bulk_commit();
@@ -273,8 +332,12 @@ __global__ void __launch_bounds__(kThr, 1)
     const int qd = warp & 3, half = (warp - kEpiW0) >> 2;
     const int row = qd * 32 + lane;
     uint32_t it = 0;
-    for (int tile = blockIdx.x; tile < p.n_mt; tile += gridDim.x, ++it) {
-      const int m0 = tile * BMr;
+    auto arrive_leader = [&](uint64_t* bar) {  // the MMA-side drain barriers live in the leader
+      if constexpr (CG2) mbar_arrive_cluster(mapa_u32(smem_u32(bar), 0));
+      else mbar_arrive(bar);
+    };
+    for (int tile = t0; tile < n_t; tile += tstep, ++it) {
+      const int m0 = tile_m0(tile);
 #pragma unroll 1
       for (int j = 0; j < NCH; ++j) {
         const uint32_t qq = it * NCH + j, acc = qq & 1, ob = qq % NB;
@@ -298,7 +361,7 @@ __global__ void __launch_bounds__(kThr, 1)
         }
         tc_fence_before();
         __syncwarp();
-        if (lane == 0) mbar_arrive(&tempty_c[acc]);
+        if (lane == 0) arrive_leader(&tempty_c[acc]);
         fence_proxy_async_smem();
         if (p.sthr) {  // hand the staged chunk to the store warp
           __syncwarp();
@@ -345,7 +408,7 @@ __global__ void __launch_bounds__(kThr, 1)
       }
       tc_fence_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive(tempty_a);
+      if (lane == 0) arrive_leader(tempty_a);
       fence_proxy_async_smem();
       if (p.sthr) {
         __syncwarp();
@@ -362,7 +425,11 @@ __global__ void __launch_bounds__(kThr, 1)
   }
   tc_fence_before();
   __syncthreads();
-  if (warp == 1) tmem_dealloc(tmem, 512);
+  if constexpr (CG2) cluster_sync_all();  // no remote arrival or multicast commit may target an exited peer
+  if (warp == 1) {
+    if constexpr (CG2) tmem_dealloc_cg2(tmem, 512);
+    else tmem_dealloc(tmem, 512);
+  }
 }
 
 }  // namespace
@@ -377,7 +444,7 @@ bool res_chain_supported(const ConvLayer& Lc, const ConvLayer* La) {
                           La->Cin == 4 * mid && La->Cout == mid && La->BN == mid && La->relu));
 }
 
-template <int MID, int V>
+template <int MID, int V, bool CG2 = false>
 static void launch_chain(const ConvLayer& Lc, const ConvLayer* La, const bf16* b, const bf16* res, bf16* out,
                          bf16* a_next, int M, cudaStream_t st) {
   CUtensorMap tb, tr, to, ta;
@@ -394,9 +461,28 @@ static void launch_chain(const ConvLayer& Lc, const ConvLayer* La, const bf16* b
   p.sh_a = La ? La->shift : Lc.shift;
   p.M = M;
   p.n_mt = (M + BMr - 1) / BMr;
-  ensure_smem_attr((const void*)res_chain_kernel<MID, V>, RC<MID, V>::kSmem);
-  const int grid = p.n_mt < num_sms() ? p.n_mt : num_sms();
-  res_chain_kernel<MID, V><<<grid, kThr, RC<MID, V>::kSmem, st>>>(tb, tr, to, ta, Lc.tmap_w, La ? La->tmap_w : Lc.tmap_w, p);
+  auto kern = res_chain_kernel<MID, V, CG2>;
+  ensure_smem_attr((const void*)kern, RC<MID, V, CG2>::kSmem);
+  if constexpr (CG2) {  // 2-CTA clusters walking pair tiles; each CTA loads half-row weight boxes
+    p.sthr = 1;
+    const int pairs = std::min((p.n_mt + 1) / 2, num_sms() / 2);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(2 * pairs, 1, 1);
+    cfg.blockDim = dim3(kThr, 1, 1);
+    cfg.dynamicSmemBytes = RC<MID, V, CG2>::kSmem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    VCHECK(cudaLaunchKernelEx(&cfg, kern, tb, tr, to, ta, Lc.tmap_w_half, La ? La->tmap_w_half : Lc.tmap_w_half, p));
+  } else {
+    const int grid = p.n_mt < num_sms() ? p.n_mt : num_sms();
+    kern<<<grid, kThr, RC<MID, V, CG2>::kSmem, st>>>(tb, tr, to, ta, Lc.tmap_w, La ? La->tmap_w : Lc.tmap_w, p);
+  }
   LAUNCHED();
 }
 
@@ -415,7 +501,18 @@ void res_chain_forward(const ConvLayer& Lc, const ConvLayer* La, const bf16* b, 
     const char* e = getenv("VISTA_CHAIN_V");
     return e ? atoi(e) : 2;
   }();
-  if (mid == 64) {
+  // CTA pairs (VISTA_CG2_CHAIN, default on): half of every weight k-block per CTA, one M = 256 MMA per K
+  // step; measured per step (same box): c+a 56x56 13.2 -> 12.5 ms, c 56x56 11.9 -> 11.5, c+a 28x28 15.7 ->
+  // 14.6 (three staging buffers, seven 8 KB weight stages), c 28x28 6.4 -> 5.8 (four staging buffers)
+  const char* ce = getenv("VISTA_CG2_CHAIN");
+  const bool cg2 = ce ? ce[0] == '1' : true;
+  if (cg2 && mid == 64) {
+    if (v & 1) launch_chain<64, 1, true>(Lc, La, b, res, out, a_next, M, st);
+    else launch_chain<64, 0, true>(Lc, La, b, res, out, a_next, M, st);
+  } else if (cg2 && mid == 128) {
+    if (La) launch_chain<128, 0, true>(Lc, La, b, res, out, a_next, M, st);
+    else launch_chain<128, 1, true>(Lc, La, b, res, out, a_next, M, st);
+  } else if (mid == 64) {
     if (v & 1) launch_chain<64, 1>(Lc, La, b, res, out, a_next, M, st);
     else launch_chain<64, 0>(Lc, La, b, res, out, a_next, M, st);
   } else if (mid == 256) {

@@ -282,6 +282,22 @@ def test_store_thread_epilogue_bit_identical(monkeypatch):
         assert torch.equal(a, b)
 
 
+@pytest.mark.parametrize("n", [37, 300])
+def test_chain_cta_pair_bit_identical(monkeypatch, n):
+    # the res_chain kernels as CTA pairs (one M = 256 MMA per K step over two adjacent pixel tiles, half of
+    # every weight k-block per CTA; VISTA_CG2_CHAIN) vs one CTA per tile: same K order, same bits.  37 images
+    # give the res2 / res3 chains an odd tile count (a phantom rank-1 tile)
+    tab = gen.make_tables(n, 8)
+    out = {}
+    for flag in ("1", "0"):
+        monkeypatch.setenv("VISTA_CG2_CHAIN", flag)
+        v = run_gpu(2, [0, 1, 2, 3, 4], tab, 8, iters=1, micro_batch=n)
+        out[flag] = [v.features(k)["mm"].view(torch.int16).cpu().clone() for k in range(5)]
+        v.close()
+    for a, b in zip(out["1"], out["0"]):
+        assert torch.equal(a, b)
+
+
 def test_weight_multicast_bit_identical(monkeypatch):
     # 2-CTA weight multicast (ConvParams::mc) engages only for launches with >= 74 pair tiles: 600 images put
     # the res4 / res5 / projection-unit launches above that, and res4's 919 M tiles give rank 1 of the last

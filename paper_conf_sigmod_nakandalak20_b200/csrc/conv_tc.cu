@@ -207,9 +207,9 @@ __global__ void __launch_bounds__(kThreads, 1)
                    const __grid_constant__ CUtensorMap tmap_y, const __grid_constant__ CUtensorMap tmap_r,
                    const ConvParams p) {
   using C = Cfg<BN, TMA_EPI, NB, AMODE == A_HALO, RKB, CG2>;
-  static_assert(!CG2 || (RKB == 0 && (AMODE == A_HALO ? !TMA_EPI
-                                                     : (AMODE == A_IM2COL || AMODE == A_TMA || AMODE == A_CAT))),
-                "CTA-pair MMA: streamed weights; halo (register epilogue) / im2col / plain TMA / cat A");
+  static_assert(!CG2 || (AMODE == A_HALO ? (RKB == 0 && !TMA_EPI)
+                                         : (AMODE == A_IM2COL || AMODE == A_TMA || AMODE == A_CAT)),
+                "CTA-pair MMA: halo (streamed weights, register epilogue) / im2col / plain TMA / cat A");
   constexpr int S = C::kStages;
   constexpr bool BRES = RKB > 0;
   constexpr int HB = C::kHB > 0 ? C::kHB : 1;
@@ -270,7 +270,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(&hfull[i], CG2 ? 2 : 1);
       mbar_init(&hempty[i], 1);
     }
-    mbar_init(wres, 1);
+    mbar_init(wres, CG2 ? 2 : 1);
     for (int i = 0; i < 4; ++i) {
       mbar_init(&staged[i], kEpiWarps);
       mbar_init(&sfree[i], 1);
@@ -348,9 +348,17 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (threadIdx.x == 0) {
         int m0, nt, g;
         decode_tile(p, cta0, m0, nt, g);
-        mbar_arrive_expect_tx(wres, p.nkb * C::kBBytes);
-        for (int kb = 0; kb < p.nkb; ++kb)
-          tma_load_2d(sR + kb * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + nt * BN, wres);
+        if constexpr (CG2) {  // CTA pair: this CTA's half of the N rows, completing on the leader's barrier
+          const uint32_t wl = mapa_u32(smem_u32(wres), 0);
+          if (crank == 0) mbar_arrive_expect_tx(wres, 2 * p.nkb * C::kBBytes);
+          for (int kb = 0; kb < p.nkb; ++kb)
+            tma_load_2d_cg2(sR + kb * C::kBBytes, &tmap_w, kb * BK, nt * BN + (int)crank * (BN / 2), wl);
+          if (crank != 0) mbar_arrive_cluster(wl);
+        } else {
+          mbar_arrive_expect_tx(wres, p.nkb * C::kBBytes);
+          for (int kb = 0; kb < p.nkb; ++kb)
+            tma_load_2d(sR + kb * C::kBBytes, &tmap_w, kb * BK, g * p.Cg_out + nt * BN, wres);
+        }
       }
     }
     if constexpr (AMODE == A_TMA) {
@@ -376,7 +384,8 @@ __global__ void __launch_bounds__(kThreads, 1)
               const uint32_t fl = mapa_u32(smem_u32(&full[stage]), 0);
               if (crank == 0) mbar_arrive_expect_tx(&full[stage], 2 * C::kStageBytes);
               tma_load_2d_cg2(sA + stage * C::kABytes, &tmap_a, kb * BK, m0, fl);
-              tma_load_2d_cg2(sB + stage * C::kBBytes, &tmap_w, kb * BK, n0 + (int)crank * (BN / 2), fl);
+              if constexpr (!BRES)
+                tma_load_2d_cg2(sB + stage * C::kBBytes, &tmap_w, kb * BK, n0 + (int)crank * (BN / 2), fl);
               if (crank != 0) mbar_arrive_cluster(fl);
               continue;
             }
@@ -413,7 +422,8 @@ __global__ void __launch_bounds__(kThreads, 1)
                                        ho * p.stride, nimg, 0, 0, fl);
               else
                 tma_load_2d_cg2(sA + stage * C::kABytes, &tmap_r, (kb - p.nkb1) * BK, m0, fl);
-              tma_load_2d_cg2(sB + stage * C::kBBytes, &tmap_w, kb * BK, n0 + (int)crank * (BN / 2), fl);
+              if constexpr (!BRES)
+                tma_load_2d_cg2(sB + stage * C::kBBytes, &tmap_w, kb * BK, n0 + (int)crank * (BN / 2), fl);
               if (crank != 0) mbar_arrive_cluster(fl);
               continue;
             }
@@ -1416,8 +1426,12 @@ static void launch_t(const ConvLayer& L, const CUtensorMap& ta, const CUtensorMa
   constexpr int smem = Cfg<BN, TE, NB, AMODE == A_HALO, RKB, CG2>::kBytes;
   ensure_smem_attr((const void*)kern, smem);
   if (p.mc) {  // clusters of two CTAs walking pair tiles (see ConvParams::mc)
-    if (RKB > 0) fail(1, "conv: multicast with resident weights");
-    const int pairs = std::min(p.n_tiles, num_sms() / 2);
+    if (RKB > 0 && !CG2) fail(1, "conv: multicast with resident weights");
+    int pairs = std::min(p.n_tiles, num_sms() / 2);
+    if (RKB > 0) {  // CTA pairs with resident weights: every pair keeps one N tile (pairs a multiple of n_nt)
+      if (p.nkb > RKB || p.n_nt > pairs) fail(1, "conv: resident-weight pair launch misconfigured");
+      pairs -= pairs % p.n_nt;
+    }
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(2 * pairs, 1, 1);
     cfg.blockDim = dim3(kThreads, 1, 1);
@@ -1474,7 +1488,8 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
       }
       if constexpr (TE && BN <= 128) {
         if (rkb == 4) {
-          launch_t<BN, A_TMA, TE, NB, 4>(L, ta, ty, tr, p, st);
+          if (p.cg2) launch_t<BN, A_TMA, TE, NB, 4, true>(L, ta, ty, tr, p, st);
+          else launch_t<BN, A_TMA, TE, NB, 4>(L, ta, ty, tr, p, st);
           break;
         }
       }
@@ -1489,7 +1504,8 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
       }
       if constexpr (TE && BN <= 128) {
         if (rkb == 4) {
-          launch_t<BN, A_CAT, TE, NB, 4>(L, ta, ty, tr, p, st);
+          if (p.cg2) launch_t<BN, A_CAT, TE, NB, 4, true>(L, ta, ty, tr, p, st);
+          else launch_t<BN, A_CAT, TE, NB, 4>(L, ta, ty, tr, p, st);
           break;
         }
       }
@@ -1736,9 +1752,18 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
     if (amode == A_HALO && L.BN == 64 && p.nkb == 9) rkb = 9;
     else if ((amode == A_TMA || amode == A_ROWVIEW) && tma_epi && L.BN <= 128 && p.nkb <= 4) rkb = 4;
   }
-  if (rkb == 4 && amode == A_TMA && L.groups == 1) p.apf = g_apf;
+  // CTA pairs for the resident-weight 1x1 TMA-epilogue convs: two adjacent M tiles of one N tile per pair, each
+  // CTA holding half of the N tile's weights (the freed shared memory deepens the A ring)
+  const bool cg2_res = rkb == 4 && amode == A_TMA && !fuse_tap && !p.dbg && env_flag("VISTA_CG2_RES", true) &&
+                       (int64_t)p.n_nt * ((p.n_mt + 1) / 2) >= num_sms() / 2 && p.n_nt <= num_sms() / 2;
+  if (cg2_res) {
+    p.mc = 1;
+    p.cg2 = 2;
+    p.n_tiles = p.n_nt * ((p.n_mt + 1) / 2);
+  }
+  if (rkb == 4 && amode == A_TMA && L.groups == 1 && !cg2_res) p.apf = g_apf;
   p.no_sthr = env_flag("VISTA_STORE_THR", true) ? 0 : 1;
-  if (rkb == 4 && amode == A_TMA && p.n_nt % 2 == 0 && !fuse_tap && !p.dbg && env_flag("VISTA_AMC", false)) {
+  if (rkb == 4 && amode == A_TMA && !cg2_res && p.n_nt % 2 == 0 && !fuse_tap && !p.dbg && env_flag("VISTA_AMC", false)) {
     p.amc = 1;  // A multicast across the pair's two N tiles (see ConvParams::amc): half-row A boxes
     make_tmap(&ta, x, (uint64_t)L.Cin, (uint64_t)M, BM / 2);
   }
@@ -1857,7 +1882,14 @@ void conv_cat_forward(const ConvLayer& L, int Cx, const bf16* b, const bf16* x, 
   else ty = L.tmap_w;  // unused
   const int rkb = (g_wres_enabled && tma_epi && L.BN <= 128 && p.nkb <= 4 && p.n_nt <= num_sms() &&
                    p.n_tiles >= num_sms()) ? 4 : 0;
-  if (rkb == 4 && stride == 1 && p.n_nt % 2 == 0 && !p.dbg && env_flag("VISTA_AMC", false)) {
+  const bool cg2_res = rkb == 4 && stride == 1 && !p.dbg && env_flag("VISTA_CG2_RES", true) &&
+                       (int64_t)p.n_nt * ((p.n_mt + 1) / 2) >= num_sms() / 2 && p.n_nt <= num_sms() / 2;
+  if (cg2_res) {  // CTA pairs with half of the resident weights each (see conv_forward)
+    p.mc = 1;
+    p.cg2 = 2;
+    p.n_tiles = p.n_nt * ((p.n_mt + 1) / 2);
+  }
+  if (rkb == 4 && stride == 1 && !cg2_res && p.n_nt % 2 == 0 && !p.dbg && env_flag("VISTA_AMC", false)) {
     p.amc = 1;  // A multicast across the pair's two N tiles (see ConvParams::amc): half-row A boxes
     make_tmap(&ta, b, (uint64_t)Kb, (uint64_t)M, BM / 2);
     make_tmap(&tr, x, (uint64_t)Cx, (uint64_t)M, BM / 2);

@@ -308,8 +308,9 @@ def test_weight_multicast_bit_identical(monkeypatch):
     tab = gen.make_tables(600, 8)
     out, feats = {}, None
     # A multicast (resident-weight 1x1 convs and stride-1 projection units, pairs of N tiles; opt-in) rides along
-    for mode, env in (("cg2", {"VISTA_AMC": "1"}), ("mc", {"VISTA_CG2": "0"}), ("unicast", {"VISTA_MC": "0"})):
-        for key in ("VISTA_MC", "VISTA_CG2", "VISTA_AMC"):
+    for mode, env in (("cg2", {"VISTA_AMC": "1"}), ("mc", {"VISTA_CG2": "0", "VISTA_CG2_RES": "0"}),
+                      ("unicast", {"VISTA_MC": "0", "VISTA_CG2_RES": "0", "VISTA_CG2_CHAIN": "0"})):
+        for key in ("VISTA_MC", "VISTA_CG2", "VISTA_AMC", "VISTA_CG2_RES", "VISTA_CG2_CHAIN"):
             monkeypatch.delenv(key, raising=False)
         for key, val in env.items():
             monkeypatch.setenv(key, val)

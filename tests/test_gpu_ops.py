@@ -194,6 +194,25 @@ def test_a_multicast_bit_identical(monkeypatch, N, H, C, Cout):
     r = bf(rng.standard_normal((N, H, H, Cout)))[0]
     out = {}
     for amc in ("1", "0"):
+        monkeypatch.setenv("VISTA_CG2_RES", "0")
         monkeypatch.setenv("VISTA_AMC", amc)
         out[amc] = vista_conv2d(x, w, scale, shift, 1, 0, 1, residual=r, relu=True).view(torch.int16).cpu()
+    assert torch.equal(out["1"], out["0"])
+
+
+@pytest.mark.parametrize("N,H,C,Cout", [(13, 14, 256, 1024), (6, 28, 128, 512), (97, 14, 256, 1024),
+                                        (7, 56, 256, 64), (9, 56, 64, 64)])
+def test_resident_weight_cta_pair_bit_identical(monkeypatch, N, H, C, Cout):
+    # resident-weight 1x1 TMA-epilogue convs as CTA pairs (VISTA_CG2_RES, default on): two adjacent M tiles of
+    # one N tile per pair, half of the N tile's weights per CTA, one M = 256 MMA per K step; odd M-tile counts
+    # give rank 1 a phantom tile.  Same K order as one CTA per tile: same bits
+    x, _ = bf(rng.standard_normal((N, H, H, C)))
+    w, _ = bf(rng.standard_normal((Cout, 1, 1, C)) * (2.0 / C) ** 0.5)
+    scale = torch.from_numpy(rng.uniform(0.5, 1.5, Cout).astype(np.float32)).cuda()
+    shift = torch.from_numpy(rng.standard_normal(Cout).astype(np.float32) * 0.1).cuda()
+    r = bf(rng.standard_normal((N, H, H, Cout)))[0]
+    out = {}
+    for flag in ("1", "0"):
+        monkeypatch.setenv("VISTA_CG2_RES", flag)
+        out[flag] = vista_conv2d(x, w, scale, shift, 1, 0, 1, residual=r, relu=True).view(torch.int16).cpu()
     assert torch.equal(out["1"], out["0"])

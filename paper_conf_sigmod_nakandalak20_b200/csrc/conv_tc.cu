@@ -207,9 +207,8 @@ __global__ void __launch_bounds__(kThreads, 1)
                    const __grid_constant__ CUtensorMap tmap_y, const __grid_constant__ CUtensorMap tmap_r,
                    const ConvParams p) {
   using C = Cfg<BN, TMA_EPI, NB, AMODE == A_HALO, RKB, CG2>;
-  static_assert(!CG2 || (AMODE == A_HALO ? (RKB == 0 && !TMA_EPI)
-                                         : (AMODE == A_IM2COL || AMODE == A_TMA || AMODE == A_CAT)),
-                "CTA-pair MMA: halo (streamed weights, register epilogue) / im2col / plain TMA / cat A");
+  static_assert(!CG2 || (AMODE == A_HALO ? !TMA_EPI : (AMODE == A_IM2COL || AMODE == A_TMA || AMODE == A_CAT)),
+                "CTA-pair MMA: halo (register epilogue) / im2col / plain TMA / cat A");
   constexpr int S = C::kStages;
   constexpr bool BRES = RKB > 0;
   constexpr int HB = C::kHB > 0 ? C::kHB : 1;
@@ -753,13 +752,25 @@ __global__ void __launch_bounds__(kThreads, 1)
               for (int kb = 0; kb < RKB; ++kb) {
                 const uint32_t a = alo[j] + (uint32_t)p.koff[kb];
                 const uint32_t b = blo + (uint32_t)(kb * (C::kBBytes >> 4));
-                tc_mma_bf16_lo_warp(tacc, a, b, idesc, kb != 0 ? 1u : 0u);
-                tc_mma_bf16_lo_warp(tacc, a + 2, b + 2, idesc, 1u);
-                tc_mma_bf16_lo_warp(tacc, a + 4, b + 4, idesc, 1u);
-                tc_mma_bf16_lo_warp(tacc, a + 6, b + 6, idesc, 1u);
+                if constexpr (CG2) {  // pair MMA: both CTAs' halos (same position, two images), B halves
+                  tc_mma_bf16_lo_warp_cg2(tacc, a, b, idesc, kb != 0 ? 1u : 0u);
+                  tc_mma_bf16_lo_warp_cg2(tacc, a + 2, b + 2, idesc, 1u);
+                  tc_mma_bf16_lo_warp_cg2(tacc, a + 4, b + 4, idesc, 1u);
+                  tc_mma_bf16_lo_warp_cg2(tacc, a + 6, b + 6, idesc, 1u);
+                } else {
+                  tc_mma_bf16_lo_warp(tacc, a, b, idesc, kb != 0 ? 1u : 0u);
+                  tc_mma_bf16_lo_warp(tacc, a + 2, b + 2, idesc, 1u);
+                  tc_mma_bf16_lo_warp(tacc, a + 4, b + 4, idesc, 1u);
+                  tc_mma_bf16_lo_warp(tacc, a + 6, b + 6, idesc, 1u);
+                }
               }
-              tc_commit_warp(&tfull[accs[j]]);
-              tc_commit_warp(&hempty[hbs[j]]);
+              if constexpr (CG2) {
+                tc_commit_cg2_warp(&tfull[accs[j]], (uint16_t)3);
+                tc_commit_cg2_warp(&hempty[hbs[j]], (uint16_t)3);
+              } else {
+                tc_commit_warp(&tfull[accs[j]]);
+                tc_commit_warp(&hempty[hbs[j]]);
+              }
             }
           }
           if (prof_mma) c_iss += clock64() - tA;
@@ -1536,7 +1547,8 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
     case A_HALO:
       if constexpr (!TE && BN == 64) {
         if (rkb == 9) {
-          launch_t<BN, A_HALO, TE, NB, 9>(L, ta, ty, tr, p, st);
+          if (p.cg2) launch_t<BN, A_HALO, TE, NB, 9, true>(L, ta, ty, tr, p, st);
+          else launch_t<BN, A_HALO, TE, NB, 9>(L, ta, ty, tr, p, st);
           break;
         }
       }
@@ -1762,6 +1774,14 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
     p.n_tiles = p.n_nt * ((p.n_mt + 1) / 2);
   }
   if (rkb == 4 && amode == A_TMA && L.groups == 1 && !cg2_res) p.apf = g_apf;
+  // CTA pairs for the resident-weight halo 3x3 (res2, Cout = 64): pair tile = one position in two consecutive
+  // images (as the streamed-weight halo pairs), half of the 72 KB of resident weights per CTA
+  if (rkb == 9 && !p.hseg && p.n_nt == 1 && !p.dbg && env_flag("VISTA_CG2_HALO64", true) &&
+      (int64_t)((N + 1) / 2) * p.mt_per_img >= num_sms() / 2) {
+    p.mc = 1;
+    p.cg2 = 1;
+    p.n_tiles = ((N + 1) / 2) * p.mt_per_img;
+  }
   p.no_sthr = env_flag("VISTA_STORE_THR", true) ? 0 : 1;
   if (rkb == 4 && amode == A_TMA && !cg2_res && p.n_nt % 2 == 0 && !fuse_tap && !p.dbg && env_flag("VISTA_AMC", false)) {
     p.amc = 1;  // A multicast across the pair's two N tiles (see ConvParams::amc): half-row A boxes

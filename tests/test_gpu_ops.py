@@ -216,3 +216,19 @@ def test_resident_weight_cta_pair_bit_identical(monkeypatch, N, H, C, Cout):
         monkeypatch.setenv("VISTA_CG2_RES", flag)
         out[flag] = vista_conv2d(x, w, scale, shift, 1, 0, 1, residual=r, relu=True).view(torch.int16).cpu()
     assert torch.equal(out["1"], out["0"])
+
+
+@pytest.mark.parametrize("N", [7, 24])
+def test_halo64_cta_pair_bit_identical(monkeypatch, N):
+    # res2-class 3x3 halo conv (Cout = 64, resident weights) as CTA pairs (VISTA_CG2_HALO64, default on): one
+    # position in two consecutive images per pair tile, half of the resident weights per CTA, M = 256 MMAs; an
+    # odd image count leaves rank 1 a phantom image.  Same K order as one CTA per tile: same bits
+    x, _ = bf(rng.standard_normal((N, 56, 56, 64)))
+    w, _ = bf(rng.standard_normal((64, 3, 3, 64)) * (2.0 / 576) ** 0.5)
+    scale = torch.from_numpy(rng.uniform(0.5, 1.5, 64).astype(np.float32)).cuda()
+    shift = torch.from_numpy(rng.standard_normal(64).astype(np.float32) * 0.1).cuda()
+    out = {}
+    for flag in ("1", "0"):
+        monkeypatch.setenv("VISTA_CG2_HALO64", flag)
+        out[flag] = vista_conv2d(x, w, scale, shift, 1, 1, 1, relu=True).view(torch.int16).cpu()
+    assert torch.equal(out["1"], out["0"])

@@ -1320,7 +1320,7 @@ static bool env_flag(const char* name, bool dflt) {
 }
 static bool use_mc(const ConvLayer& L, int amode, int rkb, const ConvParams& p) {
   return env_flag("VISTA_MC", true) && rkb == 0 && L.groups == 1 && p.n_mt >= 2 &&
-         (L.BN == 256 || (amode == A_HALO && L.BN == 128)) &&
+         (L.BN == 256 || (L.BN == 128 && (amode == A_HALO || env_flag("VISTA_MC128", false)))) &&
          (amode == A_TMA || amode == A_IM2COL || amode == A_CAT || (amode == A_HALO && env_flag("VISTA_MC_HALO", true))) &&
          (int64_t)p.n_nt * ((p.n_mt + 1) / 2) >= num_sms() / 2;
 }
@@ -1377,7 +1377,8 @@ bool make_rowview_tmap(CUtensorMap* m, const void* x, int N, int H, int W, int C
 
 static int pick_bn(int Cg_out, int groups, int K) {
   // short-K layers are epilogue/HBM-bound: 128-wide tiles get a double-buffered output staging
-  if (K <= 256 && Cg_out % 128 == 0) return 128;
+  static const int k128 = getenv("VISTA_BN_K") ? atoi(getenv("VISTA_BN_K")) : 256;  // A/B of the threshold
+  if (K <= k128 && Cg_out % 128 == 0) return 128;
   if (Cg_out % 256 == 0) return 256;
   if (Cg_out % 128 == 0) return 128;
   if (Cg_out % 64 == 0) return 64;
@@ -1491,8 +1492,8 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
                       const CUtensorMap& tr, const ConvParams& p, cudaStream_t st, int rkb) {
   switch (amode) {
     case A_TMA:
-      if constexpr (BN == 256) {
-        if (p.cg2) {
+      if constexpr (BN >= 128) {
+        if (p.cg2 && rkb == 0) {
           launch_t<BN, A_TMA, TE, NB, 0, true>(L, ta, ty, tr, p, st);
           break;
         }
@@ -1507,8 +1508,8 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
       launch_t<BN, A_TMA, TE, NB>(L, ta, ty, tr, p, st);
       break;
     case A_CAT:
-      if constexpr (BN == 256) {
-        if (p.cg2) {
+      if constexpr (BN >= 128) {
+        if (p.cg2 && rkb == 0) {
           launch_t<BN, A_CAT, TE, NB, 0, true>(L, ta, ty, tr, p, st);
           break;
         }
@@ -1525,7 +1526,7 @@ static void launch_bn(const ConvLayer& L, int amode, const CUtensorMap& ta, cons
     case A_GATHER_FAST: launch_t<BN, A_GATHER_FAST, TE, NB>(L, ta, ty, tr, p, st); break;
     case A_GATHER_ROW: launch_t<BN, A_GATHER_ROW, TE, NB>(L, ta, ty, tr, p, st); break;
     case A_IM2COL:
-      if constexpr (BN == 256) {
+      if constexpr (BN >= 128) {
         if (p.cg2) {
           launch_t<BN, A_IM2COL, TE, NB, 0, true>(L, ta, ty, tr, p, st);
           break;
@@ -1798,7 +1799,7 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
     }
     // CTA-pair MMA (M = 256, N = 256) for the streamed-weight im2col / plain-TMA convs with the register
     // epilogue: the multicast pair tile (two adjacent M tiles), each CTA loading its A tile and half of B
-    if (env_flag("VISTA_CG2", true) && (amode == A_IM2COL || amode == A_TMA) && L.BN == 256 && !p.dbg &&
+    if (env_flag("VISTA_CG2", true) && (amode == A_IM2COL || amode == A_TMA) && L.BN >= 128 && !p.dbg &&
         !p.tapf)
       p.cg2 = 2;
   }
@@ -1917,7 +1918,7 @@ void conv_cat_forward(const ConvLayer& L, int Cx, const bf16* b, const bf16* x, 
   if (use_mc(L, A_CAT, rkb, p)) {
     p.mc = 1;
     p.n_tiles = p.n_nt * ((p.n_mt + 1) / 2);
-    if (env_flag("VISTA_CG2", true) && L.BN == 256 && !p.dbg) p.cg2 = 2;  // CTA-pair MMA, see conv_forward
+    if (env_flag("VISTA_CG2", true) && L.BN >= 128 && !p.dbg) p.cg2 = 2;  // CTA-pair MMA, see conv_forward
   }
   const double flops = 2.0 * (double)M * L.Cout * L.K_alg;
   const double bytes = 2.0 * ((double)M * (Kb + Cx + L.Cout) + (double)L.Cout * L.Kp);

@@ -34,8 +34,7 @@ constexpr int kRowBytes = 128 * 128;  // one A slot: 128 pixel rows x 64 bf16 (1
 constexpr int kBBytes = 4 * 64 * 128;  // 4 k-blocks x 64 output channels x 64 bf16
 constexpr int kCrowBytes = 128 * 128;  // conv row: 128 pixels x 64 channels bf16
 constexpr int kCrowBufs = 4;           // staged conv rows (two rows per epilogue step, double-buffered)
-constexpr int kEpiWarp0 = 2, kEpiWarps = 8, kEpiThreads = kEpiWarps * 32;
-constexpr int kThreads = (kEpiWarp0 + kEpiWarps) * 32;
+constexpr int kEpiWarp0 = 2;        // warp 0: TMA producer, warp 1: MMA issuer, then EPW epilogue warps
 constexpr int kItems = kPo * 8;    // (pooled column, 8-channel chunk) items per pooled row
 constexpr int kOffB = 0, kOffA = kOffB + kBBytes, kOffCrow = kOffA + kSA * kRowBytes,
               kOffSS = kOffCrow + kCrowBufs * kCrowBytes, kOffBar = kOffSS + 2 * kCo * 4;
@@ -66,9 +65,16 @@ __device__ __forceinline__ uint4 max4(uint4 a, uint4 b) {
   return o;
 }
 
-__global__ void __launch_bounds__(kThreads, 1)
+// EPW epilogue warps (8 or 16): EPW / 4 warps per TMEM lane quadrant, each owning CPT = 256 / EPW of the 64
+// channels.  16 (default): twice the warps to hide the per-row TMEM-load / pack / barrier latency chain that
+// bounded the 8-warp epilogue (ncu: 2.5 active warps per scheduler, 0.36 issued per cycle, tensor pipe 60 %)
+template <int EPW>
+__global__ void __launch_bounds__((kEpiWarp0 + EPW) * 32, 1)
     conv1_pool_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__ CUtensorMap tmap_a,
                       const PoolParams p) {
+  constexpr int kEpiWarps = EPW, kEpiThreads = EPW * 32, CPT = kCo / (EPW / 4);
+  constexpr int NI = (kItems + kEpiThreads - 1) / kEpiThreads;  // pooling items per thread
+  static_assert(CPT == 16 || CPT == 32, "16 or 32 channels per epilogue thread");
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 1023u) & ~1023u;
@@ -104,8 +110,12 @@ __global__ void __launch_bounds__(kThreads, 1)
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
   if (p.irow && warp >= kEpiWarp0) {  // zero the whole accumulator ring before the first MMA
-    const int q = warp & 3, half = (warp - kEpiWarp0) >> 2;
-    for (int sl = 0; sl < kNAcc; ++sl) tmem_zero_32x32b_x32(tmem_base + sl * kCo + half * 32 + ((uint32_t)(q * 32) << 16));
+    const int q = warp & 3, grp = (warp - kEpiWarp0) >> 2;
+    for (int sl = 0; sl < kNAcc; ++sl) {
+      const uint32_t ta = tmem_base + sl * kCo + grp * CPT + ((uint32_t)(q * 32) << 16);
+      if constexpr (CPT == 32) tmem_zero_32x32b_x32(ta);
+      else tmem_zero_32x32b_x16(ta);
+    }
     tc_wait_st();
   }
   tc_fence_before();
@@ -220,26 +230,25 @@ __global__ void __launch_bounds__(kThreads, 1)
     // ======================= epilogue: BN + ReLU + 3x3/2 max pool =======================
     const int et = threadIdx.x - kEpiWarp0 * 32;
     const int q = warp & 3;                    // TMEM lane quadrant
-    const int half = (warp - kEpiWarp0) >> 2;  // channel half (32 channels)
+    const int grp = (warp - kEpiWarp0) >> 2;   // channel group (CPT channels)
     const int wo = q * 32 + lane;              // conv output column (M row of the tile)
-    const int i0 = et, i1 = et + kEpiThreads;  // this thread's pooling items
     uint32_t it = 0;
     // Two conv rows per step, software-pipelined: the TMEM loads of rows ho, ho + 1 are issued before the
     // pooling of rows ho - 2, ho - 1 (staged in the other two of four conv-row buffers), so their latency and
     // the accumulator zeroing hide behind that work; one named barrier per two rows separates "staged" from
     // "pooled" (the per-row latency chain, not the arithmetic, bounded the one-row loop: ~0.8 us per row).
     for (int n = blockIdx.x; n < p.N; n += gridDim.x) {
-      uint4 vb0[2], vb1[2];  // running vertical max of the open pooled rows (even / odd i), per item
+      uint4 vb0[NI], vb1[NI];  // running vertical max of the open pooled rows (even / odd i), per item
 #pragma unroll
-      for (int u = 0; u < 2; ++u) vb0[u] = vb1[u] = make_uint4(0, 0, 0, 0);
+      for (int u = 0; u < NI; ++u) vb0[u] = vb1[u] = make_uint4(0, 0, 0, 0);
       bf16* yimg = p.y + (size_t)n * kPo * kPo * kCo;
-      // conv row ho (staged in buffer ho & 1) -> pooled rows: even ho closes i = ho/2 - 1 and opens i = ho/2;
+      // conv row ho (staged in buffer ho & 3) -> pooled rows: even ho closes i = ho/2 - 1 and opens i = ho/2;
       // odd ho extends (ho-1)/2
       auto pool_row = [&](const int ho) {
         const uint32_t cbase = sC + (ho & 3) * kCrowBytes;
 #pragma unroll
-        for (int u = 0; u < 2; ++u) {
-          const int item = u == 0 ? i0 : i1;
+        for (int u = 0; u < NI; ++u) {
+          const int item = et + u * kEpiThreads;
           if (item >= kItems) continue;
           const int j = item >> 3, c = item & 7;
           const int w0 = 2 * j;
@@ -269,22 +278,36 @@ __global__ void __launch_bounds__(kThreads, 1)
       static_assert(kHo % 2 == 0, "two conv rows per step");
       for (int ho = 0; ho < kHo; ho += 2, it += 2) {
         const uint32_t acc0 = it % kNAcc, acc1 = (it + 1) % kNAcc;
-        uint32_t v0[32], v1[32];
+        const uint32_t t0 = tmem_base + acc0 * kCo + grp * CPT + ((uint32_t)(q * 32) << 16);
+        const uint32_t t1 = tmem_base + acc1 * kCo + grp * CPT + ((uint32_t)(q * 32) << 16);
+        uint32_t v0[CPT], v1[CPT];
         mbar_wait(&tfull[acc0], (it / kNAcc) & 1);
         tc_fence_after();
-        tmem_ld_32x32b_x32(tmem_base + acc0 * kCo + half * 32 + ((uint32_t)(q * 32) << 16), v0);
+        if constexpr (CPT == 32) tmem_ld_32x32b_x32(t0, v0);
+        else tmem_ld_32x32b_x16(t0, v0);
         mbar_wait(&tfull[acc1], ((it + 1) / kNAcc) & 1);
         tc_fence_after();
-        tmem_ld_32x32b_x32(tmem_base + acc1 * kCo + half * 32 + ((uint32_t)(q * 32) << 16), v1);
+        if constexpr (CPT == 32) tmem_ld_32x32b_x32(t1, v1);
+        else tmem_ld_32x32b_x16(t1, v1);
         if (ho > 0) {  // overlaps the TMEM loads
           pool_row(ho - 2);
           pool_row(ho - 1);
         }
-        tc_wait_ld_regs(v0);
-        tc_wait_ld_regs(v1);
+        if constexpr (CPT == 32) {
+          tc_wait_ld_regs(v0);
+          tc_wait_ld_regs(v1);
+        } else {
+          tc_wait_ld_regs16(v0);
+          tc_wait_ld_regs16(v1);
+        }
         if (p.irow) {  // input-row-major issue accumulates into zeroed slots
-          tmem_zero_32x32b_x32(tmem_base + acc0 * kCo + half * 32 + ((uint32_t)(q * 32) << 16));
-          tmem_zero_32x32b_x32(tmem_base + acc1 * kCo + half * 32 + ((uint32_t)(q * 32) << 16));
+          if constexpr (CPT == 32) {
+            tmem_zero_32x32b_x32(t0);
+            tmem_zero_32x32b_x32(t1);
+          } else {
+            tmem_zero_32x32b_x16(t0);
+            tmem_zero_32x32b_x16(t1);
+          }
           tc_wait_st();
         }
         tc_fence_before();
@@ -295,9 +318,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
         if (wo < kHo) {
 #pragma unroll
-          for (int c4 = 0; c4 < 4; ++c4) {  // 8 channels per 16-byte chunk
-            const int ch0 = half * 32 + c4 * 8;
-            const uint32_t sw = (((uint32_t)(half * 4 + c4)) ^ (uint32_t)(wo & 7)) << 4;
+          for (int c4 = 0; c4 < CPT / 8; ++c4) {  // 8 channels per 16-byte chunk
+            const int ch0 = grp * CPT + c4 * 8;
+            const uint32_t sw = (((uint32_t)(ch0 >> 3)) ^ (uint32_t)(wo & 7)) << 4;
             sts128(sC + (ho & 3) * kCrowBytes + wo * 128 + sw,
                    epi8(v0 + c4 * 8, ss + ch0, ss + kCo + ch0, make_uint4(0, 0, 0, 0), false, true));
             sts128(sC + ((ho + 1) & 3) * kCrowBytes + wo * 128 + sw,
@@ -335,10 +358,14 @@ void conv1_pool_forward(const ConvLayer& L, const bf16* x, int N, bf16* y, cudaS
   p.N = N;
   const char* e = getenv("VISTA_STEM_IROW");  // read per launch (A/B within one process)
   p.irow = (e && e[0] == '0') ? 0 : 1;
-  ensure_smem_attr((const void*)conv1_pool_kernel, kSmem);
+  const char* ew = getenv("VISTA_STEM_EPW");  // epilogue warps: 16 (default) or 8 (A/B)
+  const bool w16 = !(ew && atoi(ew) == 8);
+  const void* kern = w16 ? (const void*)conv1_pool_kernel<16> : (const void*)conv1_pool_kernel<8>;
+  ensure_smem_attr(kern, kSmem);
   const int grid = N < num_sms() ? N : num_sms();
   prof_begin(st);
-  conv1_pool_kernel<<<grid, kThreads, kSmem, st>>>(L.tmap_w, ta, p);
+  if (w16) conv1_pool_kernel<16><<<grid, (kEpiWarp0 + 16) * 32, kSmem, st>>>(L.tmap_w, ta, p);
+  else conv1_pool_kernel<8><<<grid, (kEpiWarp0 + 8) * 32, kSmem, st>>>(L.tmap_w, ta, p);
   LAUNCHED();
   const double flops = 2.0 * (double)N * kHo * kHo * kCo * L.K_alg;
   const double bytes = (double)N * (kHin * kHin * kS2dC * 2 + kPo * kPo * kCo * 2) + (double)kCo * L.Kp * 2;

@@ -214,14 +214,16 @@ def test_no_plan_within_tiny_budget():
     assert e.value.status == 2
 
 
-@pytest.mark.parametrize("irow", ["1", "0"])
-def test_resnet_stem_fused_bit_identical(monkeypatch, irow):
+@pytest.mark.parametrize("irow,epw", [("1", "16"), ("1", "8"), ("0", "16")])
+def test_resnet_stem_fused_bit_identical(monkeypatch, irow, epw):
     # conv1 + pool1 run as one kernel (conv1_pool.cu) by default; VISTA_FUSE_STEM=0 runs conv_tc + maxpool.
     # Max pooling is exact on the bf16 conv outputs, so every bit of MM_l must agree -- for both MMA issue
-    # orders of the stem (input-row-major N = 256 steps into a zeroed accumulator ring, and row-major).
+    # orders of the stem (input-row-major N = 256 steps into a zeroed accumulator ring, and row-major) and
+    # both epilogue widths (16 warps x 16 channels, 8 warps x 32 channels).
     tab = gen.make_tables(150, 8)  # > 148 images: CTAs own several images
     out = {}
     monkeypatch.setenv("VISTA_STEM_IROW", irow)
+    monkeypatch.setenv("VISTA_STEM_EPW", epw)
     for fuse in ("1", "0"):
         monkeypatch.setenv("VISTA_FUSE_STEM", fuse)
         v = run_gpu(2, [0, 4], tab, 8, iters=1, micro_batch=150)

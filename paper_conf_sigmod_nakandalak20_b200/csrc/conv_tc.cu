@@ -1344,6 +1344,18 @@ static CUresult encode_nd(CUtensorMap* m, const void* ptr, int rank, const cuuin
                       CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
 }
 
+bool make_nd_tmap(CUtensorMap* m, const void* ptr, int rank, const uint64_t* dims, const uint64_t* strides,
+                  const uint32_t* box) {
+  cuuint64_t d[5], s[4];
+  cuuint32_t b[5];
+  for (int i = 0; i < rank; ++i) {
+    d[i] = dims[i];
+    b[i] = box[i];
+    if (i + 1 < rank) s[i] = strides[i];
+  }
+  return encode_nd(m, ptr, rank, d, s, b) == CUDA_SUCCESS;
+}
+
 // [rows, cols] bf16 matrix, box {64, 128}, 128B swizzle (A operands / staged outputs of 128-row tiles)
 bool make_plain_tmap(CUtensorMap* m, const void* ptr, int cols, int rows) {
   const cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
@@ -1599,6 +1611,10 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   p.segs = 1;
   const int64_t M = (int64_t)N * p.Ho * p.Wo;
   if (M <= 0) return tapf == nullptr;
+  if (!res && !tapf && !g_conv_dbg && rowconv3x3_supported(L, H, W) && env_flag("VISTA_ROWCONV", true)) {
+    rowconv3x3_forward(L, x, N, H, W, y, st);
+    return true;
+  }
   if (M > INT32_MAX - BM) fail(1, "conv: M too large for one launch");
   p.M = (int)M;
   p.relu = L.relu ? 1 : 0;

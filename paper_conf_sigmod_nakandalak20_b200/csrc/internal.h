@@ -66,6 +66,13 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
 void conv_cat_forward(const ConvLayer& L, int Cx, const bf16* b, const bf16* x, int N, int Hx, int Wx, int stride,
                       bf16* y, cudaStream_t st);
 bool make_rowview_tmap(CUtensorMap* m, const void* x, int N, int H, int W, int C, int Wo);
+// N-D bf16 tiled tensor map, 128B swizzle, out-of-bounds elements read as zero
+bool make_nd_tmap(CUtensorMap* m, const void* ptr, int rank, const uint64_t* dims, const uint64_t* strides,
+                  const uint32_t* box);
+// 3x3 / 1 / pad 1 conv with Cin = Cout = 64 and W <= 62 (ResNet res2) issued input-row-major with N = 192
+// MMAs (conv3x3_rows.cu), bit-identical to the conv_tc halo path; VISTA_ROWCONV=0 disables it
+bool rowconv3x3_supported(const ConvLayer& L, int H, int W);
+void rowconv3x3_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, bf16* y, cudaStream_t st);
 bool make_plain_tmap(CUtensorMap* m, const void* ptr, int cols, int rows);
 // Two chained 1x1 convs of consecutive ResNet units (res_chain.cu): out = ReLU(BN_c(b * Wc) + res) and
 // a_next = ReLU(BN_a(out * Wa)) in one kernel, bit-identical to two conv_forward calls.

@@ -232,3 +232,35 @@ def test_halo64_cta_pair_bit_identical(monkeypatch, N):
         monkeypatch.setenv("VISTA_CG2_HALO64", flag)
         out[flag] = vista_conv2d(x, w, scale, shift, 1, 1, 1, relu=True).view(torch.int16).cpu()
     assert torch.equal(out["1"], out["0"])
+
+
+ROWCONV = [
+    # N, H, W, relu   (3x3 / 1 / pad 1, Cin = Cout = 64: the input-row-major kernel, conv3x3_rows.cu)
+    (2, 56, 56, True),     # res2 geometry, two bands
+    (3, 56, 56, True),     # odd image count: phantom second image of the last pair
+    (151, 56, 56, True),   # 152 items > 148 CTAs: CTAs own several (pair, band) items, TMEM ring wraps
+    (1, 9, 11, False),     # small odd geometry, no ReLU, bands of 5 / 4 rows
+    (5, 7, 62, True),      # widest supported row (62 + 2 padded columns = 64 A rows)
+    (4, 1, 1, True),       # one row: only the centre filter row contributes
+]
+
+
+@pytest.mark.parametrize("N,H,W,relu", ROWCONV)
+def test_rowconv3x3_bit_identical_to_halo(monkeypatch, N, H, W, relu):
+    # the row kernel and the conv_tc halo / im2col path accumulate every output in the same (r, s, channel)
+    # order, so they must agree bit for bit; both are checked against the oracle too
+    x, x64 = bf(rng.standard_normal((N, H, W, 64)))
+    w, w64 = bf(rng.standard_normal((64, 3, 3, 64)) * (2.0 / 576) ** 0.5)
+    scale = rng.uniform(0.5, 1.5, 64).astype(np.float32)
+    shift = rng.standard_normal(64).astype(np.float32) * 0.1
+    out = {}
+    for flag in ("1", "0"):
+        monkeypatch.setenv("VISTA_ROWCONV", flag)
+        out[flag] = vista_conv2d(x, w, torch.from_numpy(scale).cuda(), torch.from_numpy(shift).cuda(), 1, 1, 1,
+                                 relu=relu)
+        torch.cuda.synchronize()
+    assert torch.equal(out["1"].view(torch.int16), out["0"].view(torch.int16))
+    ref = oracle.conv2d(x64, w64, 1, 1, 1) * scale.astype(np.float64) + shift.astype(np.float64)
+    if relu:
+        ref = np.maximum(ref, 0)
+    assert normwise(out["1"].to(torch.float64).cpu().numpy(), ref) <= 8e-3

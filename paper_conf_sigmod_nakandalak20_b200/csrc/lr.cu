@@ -502,6 +502,213 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_dot_kernel(const PassAr
   }
 }
 
+// ---- two-group variant of lr_dot_kernel (power / gradient / eval passes of wide rows) ----
+// ncu on lr_dot_kernel<4, 2, 2> (conv5_x layer, 16k rows): 39 % issue-slot busy, 0.88 eligible warps per
+// scheduler, a quarter of the stall samples at the per-block CTA barrier -- every compute warp walks the
+// same serial chain per row block (dots -> butterfly -> barrier -> z -> phi -> accumulate) in lockstep.
+// Here the compute warps form two independent groups of kGW warps; group g consumes the row blocks
+// it % 2 == g of this CTA (two rows per block, kStages2 blocks in flight), syncing only its own warps
+// (named barrier 1 + 2g), so one group's chain overlaps the other's.  Each thread owns CH 16-byte column
+// chunks (tg, tg + 32 kGW, ...) in BOTH groups with separate accumulators; at the end group 1's sums are
+// added to group 0's in a fixed order (deterministic).
+constexpr int kGW = 9;         // warps per consumer group
+constexpr int kStages2 = 6;    // two-row blocks in flight per CTA (three per group)
+template <int CH, int MODE>
+__global__ void __launch_bounds__(2 * kGW * 32 + 32, 1) lr_dot2_kernel(const PassArgs a) {
+  constexpr int RB = 2, NG = kGW * 32;
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  const uint32_t base = (raw + 127u) & ~127u;
+  uint8_t* gbase = smem_raw + (base - raw);
+  const uint32_t row_bytes = (uint32_t)a.ld * 2u;
+  const uint32_t stage_bytes = ((uint32_t)RB * row_bytes + 127u) & ~127u;
+  float* red_all = reinterpret_cast<float*>(gbase + kStages2 * stage_bytes);  // [kStages2][RB][16]
+  uint64_t* full = reinterpret_cast<uint64_t*>(red_all + kStages2 * RB * 16);
+  uint64_t* empty = full + kStages2;
+  const int nthr = 2 * NG;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int grp = warp / kGW, gw = warp - grp * kGW, tg = tid - grp * NG;
+  const int64_t nrows = a.r1 - a.r0;
+  const int64_t nblk = (nrows + RB - 1) / RB;
+  if (tid == 0) {
+    for (int i = 0; i < kStages2; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&empty[i], NG);
+    }
+    fence_mbar_init();
+  }
+  __syncthreads();
+  if (warp == 2 * kGW) {  // producer warp
+    if (lane == 0) {
+      int it = 0;
+      for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++it) {
+        const int stage = it % kStages2;
+        if (it >= kStages2) mbar_wait(&empty[stage], ((it / kStages2) - 1) & 1);
+        const int64_t r = a.r0 + blk * RB;
+        const uint32_t bytes = (uint32_t)min((int64_t)RB, a.r1 - r) * row_bytes;
+        mbar_arrive_expect_tx(&full[stage], bytes);
+        bulk_load(base + stage * stage_bytes, a.MM + (size_t)r * row_bytes, bytes, &full[stage]);
+        const int64_t pb = blk + (int64_t)kStages2 * gridDim.x;
+        if (pb < nblk) {
+          const int64_t pr = a.r0 + pb * RB;
+          prefetch_l2_range(a.MM + (size_t)pr * row_bytes, (uint32_t)min((int64_t)RB, a.r1 - pr) * row_bytes);
+        }
+      }
+    }
+    return;
+  }
+  uint32_t coff[CH];
+  float2 wv[CH][4], acc[CH][4];
+#pragma unroll
+  for (int c = 0; c < CH; ++c) {
+    const int ch = tg + c * NG;
+    const bool act = ch < a.chunks;
+    coff[c] = act ? (uint32_t)ch * 16u : 0u;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      wv[c][j] = act ? make_float2(a.what[ch * 8 + 2 * j], a.what[ch * 8 + 2 * j + 1]) : make_float2(0.f, 0.f);
+      acc[c][j] = make_float2(0.f, 0.f);
+    }
+  }
+  const float bh = a.bhat[0];
+  float sum_r = 0.f, sum_loss = 0.f;
+  unsigned long long cnt[5] = {0, 0, 0, 0, 0};
+  int it = grp;
+  for (int64_t blk = blockIdx.x + (int64_t)grp * gridDim.x; blk < nblk; blk += 2 * (int64_t)gridDim.x, it += 2) {
+    const int stage = it % kStages2;
+    mbar_wait(&full[stage], (it / kStages2) & 1);
+    const int64_t r = a.r0 + blk * RB;
+    const int nr = (int)min((int64_t)RB, a.r1 - r);
+    const uint8_t* sb = gbase + stage * stage_bytes;
+    float* red = red_all + stage * (RB * 16);
+    float sd[16];
+#pragma unroll
+    for (int q = 0; q < RB; ++q) {
+      float2 s2 = make_float2(0.f, 0.f);
+#pragma unroll
+      for (int c = 0; c < CH; ++c) {
+        const uint4 v = *reinterpret_cast<const uint4*>(sb + q * row_bytes + coff[c]);
+        s2 = ffma2(bf2_f2(v.x), wv[c][0], s2);
+        s2 = ffma2(bf2_f2(v.y), wv[c][1], s2);
+        s2 = ffma2(bf2_f2(v.z), wv[c][2], s2);
+        s2 = ffma2(bf2_f2(v.w), wv[c][3], s2);
+      }
+      sd[q] = s2.x + s2.y;
+    }
+    butterfly<RB>(sd, lane);
+    if ((lane & 15) == 0) red[(lane >> 4) * 16 + gw] = sd[0];
+    named_bar_sync(1 + 2 * grp, NG);
+    float phi = 0.f;
+    if (lane < nr) {
+      float z = bh;
+      const float* rq = red + lane * 16;
+#pragma unroll
+      for (int w = 0; w < kGW; ++w) z += rq[w];
+      const int64_t row = r + lane;
+      if (MODE == 2) {
+        phi = z;
+        if (gw == 0) sum_r += z;
+      } else {
+        const int yv = a.y[row];
+        if (MODE == 3) {
+          phi = 1.f / (1.f + __expf(-z)) - (float)yv;
+          if (gw == 0) {
+            sum_r += phi;
+            sum_loss += softplusf(z) - (float)yv * z;
+          }
+        } else if (gw == 0) {  // MODE 4: predict 1 iff z >= 0
+          const int pred = z >= 0.f ? 1 : 0;
+          if (row < a.n_train) cnt[0] += pred == yv;
+          else cnt[pred && yv ? 1 : (pred ? 2 : (yv ? 4 : 3))] += 1;
+        }
+      }
+    }
+    if (MODE != 4) {
+#pragma unroll
+      for (int q = 0; q < RB; ++q) {
+        if (q < nr) {  // group-uniform
+          const float ph = __shfl_sync(0xffffffffu, phi, q);
+          const float2 p2 = make_float2(ph, ph);
+#pragma unroll
+          for (int c = 0; c < CH; ++c) {
+            const uint4 v = *reinterpret_cast<const uint4*>(sb + q * row_bytes + coff[c]);
+            acc[c][0] = ffma2(bf2_f2(v.x), p2, acc[c][0]);
+            acc[c][1] = ffma2(bf2_f2(v.y), p2, acc[c][1]);
+            acc[c][2] = ffma2(bf2_f2(v.z), p2, acc[c][2]);
+            acc[c][3] = ffma2(bf2_f2(v.w), p2, acc[c][3]);
+          }
+        }
+      }
+    }
+    mbar_arrive(&empty[stage]);
+  }
+  if constexpr (MODE == 4) {
+    if (gw == 0) {
+#pragma unroll
+      for (int k = 0; k < 5; ++k) {
+        unsigned long long v = cnt[k];
+        for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        if (lane == 0 && v) atomicAdd(&a.counts[k], v);
+      }
+    }
+    return;
+  } else {
+    // group 1 hands its sums to group 0 through the (drained) ring: [chunk][8] floats + 2 scalars
+    named_bar_sync(2, nthr);  // both groups done with every stage
+    float* xfer = reinterpret_cast<float*>(gbase);
+    if (grp == 1) {
+#pragma unroll
+      for (int c = 0; c < CH; ++c) {
+        const int ch = tg + c * NG;
+        if (ch < a.chunks) {
+          float4* o = reinterpret_cast<float4*>(xfer + ch * 8);
+          o[0] = make_float4(acc[c][0].x, acc[c][0].y, acc[c][1].x, acc[c][1].y);
+          o[1] = make_float4(acc[c][2].x, acc[c][2].y, acc[c][3].x, acc[c][3].y);
+        }
+      }
+      if (gw == 0) {
+        for (int o = 16; o > 0; o >>= 1) {
+          sum_r += __shfl_xor_sync(0xffffffffu, sum_r, o);
+          sum_loss += __shfl_xor_sync(0xffffffffu, sum_loss, o);
+        }
+        if (lane == 0) {
+          xfer[a.ld + 8] = sum_r;
+          xfer[a.ld + 9] = sum_loss;
+        }
+      }
+    }
+    named_bar_sync(2, nthr);
+    float* out = a.partial + (size_t)blockIdx.x * (a.ld + 4);
+    if (grp == 0) {
+#pragma unroll
+      for (int c = 0; c < CH; ++c) {
+        const int ch = tg + c * NG;
+        if (ch < a.chunks) {
+          const float4* o1 = reinterpret_cast<const float4*>(xfer + ch * 8);
+          const float4 u0 = o1[0], u1 = o1[1];
+          float4* o = reinterpret_cast<float4*>(out + ch * 8);
+          o[0] = make_float4(acc[c][0].x + u0.x, acc[c][0].y + u0.y, acc[c][1].x + u0.z, acc[c][1].y + u0.w);
+          o[1] = make_float4(acc[c][2].x + u1.x, acc[c][2].y + u1.y, acc[c][3].x + u1.z, acc[c][3].y + u1.w);
+        }
+      }
+      if (gw == 0) {
+        for (int o = 16; o > 0; o >>= 1) {
+          sum_r += __shfl_xor_sync(0xffffffffu, sum_r, o);
+          sum_loss += __shfl_xor_sync(0xffffffffu, sum_loss, o);
+        }
+        if (lane == 0) {
+          out[a.ld] = sum_r + xfer[a.ld + 8];
+          out[a.ld + 1] = sum_loss + xfer[a.ld + 9];
+        }
+      }
+    }
+    if (a.f.on) {
+      named_bar_sync(2, nthr);  // the transfer area is read before the tail reuses the ring
+      fused_tail<MODE>(a, gbase, nthr);
+    }
+  }
+}
+
 // ---- fused reduce + update (world == 1) ----
 // Grid-wide barrier of the cooperative launch (all CTAs co-resident): compute threads only (the
 // producer warp has exited), named barrier 2 inside the CTA, one arrival per CTA on a global counter.
@@ -891,6 +1098,8 @@ struct StreamCfg {
   size_t smem;
   int dot_rb = 0;       // bf16 power / gradient / eval passes on lr_dot_kernel<dot_rb, ch, MODE> (0: not used)
   size_t dot_smem = 0;
+  int dot2_ch = 0;      // > 0: those passes on lr_dot2_kernel<dot2_ch, MODE> (two consumer groups)
+  size_t dot2_smem = 0;
 };
 
 static void launch_pass(const void* kern, const PassArgs& a, int grid, int threads, size_t smem, bool coop,
@@ -911,6 +1120,18 @@ template <int MODE, typename E>
 static void run_pass(const PassArgs& a, const StreamCfg& c, cudaStream_t st) {
   const bool coop = a.f.on != 0;
   if constexpr (MODE >= 2 && sizeof(E) == 2) {
+    if (c.dot2_ch > 0) {
+      const void* k = nullptr;
+      switch (c.dot2_ch) {
+        case 1: k = (const void*)lr_dot2_kernel<1, MODE>; break;
+        case 2: k = (const void*)lr_dot2_kernel<2, MODE>; break;
+        case 3: k = (const void*)lr_dot2_kernel<3, MODE>; break;
+        case 4: k = (const void*)lr_dot2_kernel<4, MODE>; break;
+        default: fail(1, "lr: no two-group pass kernel for this row width");
+      }
+      launch_pass(k, a, c.grid, 2 * kGW * 32 + 32, c.dot2_smem, coop, st);
+      return;
+    }
     if (c.dot_rb > 0) {
     const void* k = nullptr;
 #define VISTA_DOT(RB, CH) \
@@ -993,7 +1214,19 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
       }
     }
   }
-  const int64_t pass_rb = cfg.dot_rb > 0 ? std::min(cfg.rb, cfg.dot_rb) : cfg.rb;  // grid: blocks of the finer kernel
+  // the two-group kernel for rows of at least VISTA_LR_DOT2 columns (opt-in: measured neutral, 87-94 vs 91 us
+  // per conv5_x power pass -- the per-block barrier chain is not what bounds the pass)
+  const char* dot2_env = getenv("VISTA_LR_DOT2");
+  if (cfg.dot_rb > 0 && dot2_env && atoi(dot2_env) > 0 && ld >= atoi(dot2_env)) {
+    const int ch2 = (chunks + kGW * 32 - 1) / (kGW * 32);
+    const size_t sb2 = ((size_t)2 * ld * 2 + 127) & ~(size_t)127;
+    const size_t smem2 = kStages2 * sb2 + kStages2 * 2 * 16 * 4 + 2 * kStages2 * 8 + 128;
+    if (ch2 <= 4 && smem2 <= 227 * 1024) {
+      cfg.dot2_ch = ch2;
+      cfg.dot2_smem = smem2;
+    }
+  }
+  const int64_t pass_rb = cfg.dot2_ch > 0 ? 2 : (cfg.dot_rb > 0 ? std::min(cfg.rb, cfg.dot_rb) : cfg.rb);  // grid: blocks of the finer kernel
   // at least one CTA per 128 columns: the fused tail splits the ld columns over the CTAs, and a grid sized
   // by a handful of rows left one CTA walking all of them behind L2 latency (C1: 33 -> ~9 us per pass)
   auto grid_for_rows = [&](int64_t rows) {
@@ -1007,9 +1240,10 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   for (int j = 0; j < ld; ++j) d_real += real_host[j] ? 1 : 0;
   // world == 1: reduction + update in the pass kernels' tails (one launch per pass).  The tail keeps this
   // CTA's reduced columns and a [32][32] double scratch in the (drained) stage ring.
-  const size_t ring_min = kStagesLR * std::min(stage_bytes, cfg.dot_rb > 0
-                                                                ? (((size_t)cfg.dot_rb * ld * 2 + 127) & ~(size_t)127)
-                                                                : stage_bytes);
+  size_t ring_min = kStagesLR * std::min(stage_bytes, cfg.dot_rb > 0
+                                                          ? (((size_t)cfg.dot_rb * ld * 2 + 127) & ~(size_t)127)
+                                                          : stage_bytes);
+  if (cfg.dot2_ch > 0) ring_min = std::min(ring_min, (size_t)kStages2 * (((size_t)2 * ld * 2 + 127) & ~(size_t)127));
   const size_t tail_need = 32 * 32 * 8 + ((size_t)(ld + grid_tr - 1) / grid_tr + 4) * 8;
   const bool fused = !allreduce && power_iters >= 1 && n_train > 0 && tail_need <= ring_min &&
                      !(getenv("VISTA_LR_FUSED") && getenv("VISTA_LR_FUSED")[0] == '0');

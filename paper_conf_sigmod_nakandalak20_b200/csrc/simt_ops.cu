@@ -67,14 +67,14 @@ void launch_ingest_f32(const uint8_t* px, int64_t n, float* y, cudaStream_t st) 
 // ---- S0 for ResNet conv1: uint8 NHWC3 -> zero-padded 2x2 space-to-depth [n, 117, 117, 16] ----
 // channel c' = (dy*2 + dx)*3 + ch (c' >= 12 zero) of position (h2, w2) holds (p - 128)/128 of pixel
 // (2*h2 + dy - 3, 2*w2 + dx - 3), 0 outside the image (the conv's zero padding of 3).
+// 2-D grid: x over the 117 x 117 positions of an image (32-bit index math; the grid-stride loop over a
+// flat int64 index spent most of its instructions in 64-bit divisions), y over images
 template <typename T>
 __global__ void ingest_s2d_kernel(const uint8_t* __restrict__ px, int64_t n, T* __restrict__ y) {
-  const int64_t total = n * 117 * 117;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    const int w2 = (int)(i % 117);
-    const int64_t t = i / 117;
-    const int h2 = (int)(t % 117);
-    const int64_t img = t / 117;
+  const int p = blockIdx.x * blockDim.x + threadIdx.x;
+  if (p >= 117 * 117) return;
+  const int h2 = p / 117, w2 = p - h2 * 117;
+  for (int64_t img = blockIdx.y; img < n; img += gridDim.y) {
     const uint8_t* src = px + img * (227 * 227 * 3);
     float f[16];
 #pragma unroll
@@ -94,15 +94,17 @@ __global__ void ingest_s2d_kernel(const uint8_t* __restrict__ px, int64_t n, T* 
       lo[c] = f[c];
       hi[c] = f[8 + c];
     }
-    st8(y + i * 16, lo);
-    st8(y + i * 16 + 8, hi);
+    T* o = y + (img * (117 * 117) + p) * 16;
+    st8(o, lo);
+    st8(o + 8, hi);
   }
 }
 template <typename T>
 static void ingest_s2d_t(const uint8_t* px, int64_t n, T* y, cudaStream_t st) {
   const int64_t total = n * 117 * 117;
   prof_begin(st);
-  ingest_s2d_kernel<T><<<grid_for(total, 256), 256, 0, st>>>(px, n, y);
+  const dim3 grid((117 * 117 + 255) / 256, (unsigned)(n < 65535 ? (n > 0 ? n : 1) : 65535));
+  ingest_s2d_kernel<T><<<grid, 256, 0, st>>>(px, n, y);
   LAUNCHED();
   prof_end(st, 2, 0, (double)n * 227 * 227 * 3 + (double)total * 16 * sizeof(T));
 }
@@ -260,11 +262,50 @@ __global__ void tap_kernel(const T* __restrict__ A, int64_t N, int H, int W, int
     st8(F + (size_t)n * 4 * C + (size_t)q * C + c8 * 8, m);
   }
 }
+// bf16 form: max on packed bf16x2 (exact), four independent 16-byte loads in flight per thread
+__device__ __forceinline__ uint4 bmax4(uint4 a, uint4 b) {
+  uint4 o;
+  const __nv_bfloat162* pa = reinterpret_cast<const __nv_bfloat162*>(&a);
+  const __nv_bfloat162* pb = reinterpret_cast<const __nv_bfloat162*>(&b);
+  __nv_bfloat162* po = reinterpret_cast<__nv_bfloat162*>(&o);
+#pragma unroll
+  for (int j = 0; j < 4; ++j) po[j] = __hmax2(pa[j], pb[j]);
+  return o;
+}
+__global__ void tap_bf16_kernel(const bf16* __restrict__ A, int64_t N, int H, int W, int C, bf16* __restrict__ F) {
+  const int C8 = C >> 3;
+  const int h2 = (H + 1) >> 1, w2 = (W + 1) >> 1;
+  const int64_t total = N * 4 * C8;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int c8 = (int)(i % C8);
+    const int64_t t = i / C8;
+    const int q = (int)(t & 3);
+    const int64_t n = t >> 2;
+    const int qi = q >> 1, qj = q & 1;
+    const int hb = qi ? h2 : 0, he = qi ? H : h2;
+    const int wb = qj ? w2 : 0, we = qj ? W : w2;
+    const uint4 ninf = make_uint4(0xFF80FF80u, 0xFF80FF80u, 0xFF80FF80u, 0xFF80FF80u);
+    uint4 m0 = ninf, m1 = ninf;
+    for (int h = hb; h < he; ++h) {
+      const uint4* row = reinterpret_cast<const uint4*>(A + (((size_t)n * H + h) * W) * C + c8 * 8);
+      int w = wb;
+      for (; w + 4 <= we; w += 4) {
+        const uint4 a = __ldcs(row + (size_t)w * C8), b = __ldcs(row + (size_t)(w + 1) * C8);
+        const uint4 c = __ldcs(row + (size_t)(w + 2) * C8), d = __ldcs(row + (size_t)(w + 3) * C8);
+        m0 = bmax4(m0, bmax4(a, b));
+        m1 = bmax4(m1, bmax4(c, d));
+      }
+      for (; w < we; ++w) m0 = bmax4(m0, __ldcs(row + (size_t)w * C8));
+    }
+    *reinterpret_cast<uint4*>(F + (size_t)n * 4 * C + (size_t)q * C + c8 * 8) = bmax4(m0, m1);
+  }
+}
 template <typename T>
 static void tap_t(const T* A, int64_t N, int H, int W, int C, T* F, cudaStream_t st) {
   const int64_t total = N * 4 * (C / 8);
   prof_begin(st);
-  tap_kernel<T><<<grid_for(total, 256), 256, 0, st>>>(A, N, H, W, C, F);
+  if constexpr (sizeof(T) == 2) tap_bf16_kernel<<<grid_for(total, 256), 256, 0, st>>>(A, N, H, W, C, F);
+  else tap_kernel<T><<<grid_for(total, 256), 256, 0, st>>>(A, N, H, W, C, F);
   LAUNCHED();
   prof_end(st, 1, 0, (double)sizeof(T) * ((double)N * H * W * C + (double)N * 4 * C));
 }

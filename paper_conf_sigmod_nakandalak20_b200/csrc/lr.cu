@@ -56,6 +56,7 @@ struct PassArgs {
   int64_t n_train;      // rows < n_train are train rows (eval mode)
   int ld, chunks;       // ld elements per row, chunks = ld * sizeof(E) / 16
   int rb;               // rows per streamed block
+  int dbg;              // VISTA_LR_DBG (measurement only, results wrong): 1 = dot kernel consumes blocks without computing
   const float* mu;      // [ld]
   const float* what;    // [ld]  inv_j * (w_j or v_j), 0 on excluded / pad columns
   const float* bhat;    // [1]
@@ -401,9 +402,15 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_dot_kernel(const PassAr
   int it = 0;
   for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++it) {
     const int stage = it % kStagesLR;
-    mbar_wait(&full[stage], (it / kStagesLR) & 1);
     const int64_t r = a.r0 + blk * RB;
     const int nr = (int)min((int64_t)RB, a.r1 - r);
+    // labels of the block's rows: loaded before the data wait so their latency leaves the per-block chain
+    const int yv = (MODE != 2 && lane < nr) ? (int)a.y[r + lane] : 0;
+    mbar_wait(&full[stage], (it / kStagesLR) & 1);
+    if (a.dbg == 1) {
+      mbar_arrive(&empty[stage]);
+      continue;
+    }
     const uint8_t* sb = gbase + stage * stage_bytes;
     float* red = red_all + stage * (kMaxRB * 32);
     float sd[16];
@@ -434,7 +441,6 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_dot_kernel(const PassAr
         phi = z;
         if (warp == 0) sum_r += z;
       } else {
-        const int yv = a.y[row];
         if (MODE == 3) {
           phi = 1.f / (1.f + __expf(-z)) - (float)yv;
           if (warp == 0) {
@@ -733,30 +739,37 @@ __device__ __forceinline__ void grid_sync(unsigned int* bar, int nthr) {
 // out[i] = sum over the G CTAs' partial rows of column j0 + i, i < n, in fp64 and a fixed order (each
 // warp sums a contiguous CTA range per 32-column tile, then the warp sums in warp order).  Every CTA
 // calling it for the same column gets the same bits.  sh: >= nwc * 32 doubles of shared memory.
-__device__ void reduce_cols(const float* partial, int pitch, int G, int j0, int n, double* out, double* sh,
-                            int nthr) {
+__device__ void reduce_cols(const float* partial, int pitch, int G, int j0, int n, int ld, double* out, double* out2,
+                            double* sh, int nthr) {
+  // virtual column i < n + 2: partial column j0 + i (i < n) -> out[i], or ld + i - n (the two scalar columns,
+  // reduced redundantly by every CTA: identical bits) -> out2[i - n]; one sweep serves both
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwc = nthr >> 5;
+  const int nv = n + 2;
+  auto col = [&](int i) { return i < n ? j0 + i : ld + (i - n); };
+  auto put = [&](int i, double v) {
+    if (i < n) out[i] = v;
+    else out2[i - n] = v;
+  };
   if (G < 4 * nwc) {
     // few CTAs (small inputs): the CTA-range split would leave most warps idle and walk the columns 32 at
     // a time behind two barriers each (measured: ~30 us per pass for one CTA at ld 4104); instead each
     // lane sums whole columns over the G partial rows in CTA order, warps on different 32-column tiles
-    for (int t = warp * 32; t < n; t += nwc * 32) {
-      if (t + lane < n) {
-        const float* pc = partial + j0 + t + lane;
+    for (int t = warp * 32; t < nv; t += nwc * 32) {
+      if (t + lane < nv) {
+        const float* pc = partial + col(t + lane);
         double s = 0.0;
         for (int c = 0; c < G; ++c) s += (double)__ldcg(pc + (size_t)c * pitch);
-        out[t + lane] = s;
+        put(t + lane, s);
       }
     }
     named_bar_sync(2, nthr);
     return;
   }
   const int c0 = (int)((int64_t)G * warp / nwc), c1 = (int)((int64_t)G * (warp + 1) / nwc);
-  for (int t = 0; t < n; t += 32) {
-    const int j = j0 + t + lane;
+  for (int t = 0; t < nv; t += 32) {
     double s = 0.0;
-    if (t + lane < n) {
-      const float* pc = partial + j;
+    if (t + lane < nv) {
+      const float* pc = partial + col(t + lane);
       int c = c0;
       for (; c + 8 <= c1; c += 8) {  // eight independent L2 loads in flight, added in order
         float x[8];
@@ -769,10 +782,10 @@ __device__ void reduce_cols(const float* partial, int pitch, int G, int j0, int 
     }
     sh[warp * 32 + lane] = s;
     named_bar_sync(2, nthr);
-    if (warp == 0 && t + lane < n) {
+    if (warp == 0 && t + lane < nv) {
       double g = 0.0;
       for (int w = 0; w < nwc; ++w) g += sh[w * 32 + lane];
-      out[t + lane] = g;
+      put(t + lane, g);
     }
     named_bar_sync(2, nthr);
   }
@@ -788,6 +801,28 @@ __device__ double cta_sum(double v, double* sh, int nthr) {
   for (int w = 0; w < nwc; ++w) t += sh[w];
   named_bar_sync(2, nthr);
   return t;
+}
+
+// the same for two values at once (one pair of barriers)
+__device__ void cta_sum2(double& a, double& b, double* sh, int nthr) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwc = nthr >> 5;
+  for (int o = 16; o > 0; o >>= 1) {
+    a += __shfl_xor_sync(0xffffffffu, a, o);
+    b += __shfl_xor_sync(0xffffffffu, b, o);
+  }
+  if (lane == 0) {
+    sh[warp] = a;
+    sh[32 + warp] = b;
+  }
+  named_bar_sync(2, nthr);
+  double ta = 0.0, tb = 0.0;
+  for (int w = 0; w < nwc; ++w) {
+    ta += sh[w];
+    tb += sh[32 + w];
+  }
+  named_bar_sync(2, nthr);
+  a = ta;
+  b = tb;
 }
 
 // fixed-order sum of the G per-CTA scalars (result in every thread of every CTA, same bits)
@@ -820,8 +855,7 @@ __device__ void fused_tail(const PassArgs& a, uint8_t* scratch, int nthr) {
   __threadfence();
   grid_sync(f.bar, nthr);  // every CTA's partial row is written
   const int u0 = (int)((int64_t)ld * b / G), u1 = (int)((int64_t)ld * (b + 1) / G);
-  reduce_cols(a.partial, pitch, G, u0, u1 - u0, gs, sh, nthr);
-  reduce_cols(a.partial, pitch, G, ld, 2, g2, sh, nthr);  // redundantly in every CTA: identical bits
+  reduce_cols(a.partial, pitch, G, u0, u1 - u0, ld, gs, g2, sh, nthr);
   const double phisum = g2[0];
   LRState* st = f.st;
   if (MODE == 0) {
@@ -872,8 +906,7 @@ __device__ void fused_tail(const PassArgs& a, uint8_t* scratch, int nthr) {
       ss += q * q;
       sq += f.inv[j] * q * f.mu[j];
     }
-    ss = cta_sum(ss, sh, nthr);
-    sq = cta_sum(sq, sh, nthr);
+    cta_sum2(ss, sq, sh, nthr);
     if (threadIdx.x == 0) {
       f.scal[b] = ss;
       f.scal[G + b] = sq;
@@ -1288,6 +1321,7 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   a.partial = partial;
   a.n_train = n_train;
   a.rb = cfg.rb;
+  a.dbg = getenv("VISTA_LR_DBG") ? atoi(getenv("VISTA_LR_DBG")) : 0;
   a.counts = nullptr;
   a.f.on = fused ? 1 : 0;
   a.f.ncols = ncols;

@@ -158,7 +158,8 @@ size_t lr_async_bytes(int ld, int iters);
 LRResult lr_collect(const LRAsync& a);
 LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
                   const uint8_t* real_col_mask_host, int iters, int power_iters, double lambda, double alpha,
-                  allreduce_fn allreduce, void* ar_user, cudaStream_t st, LRAsync* async = nullptr);
+                  allreduce_fn allreduce, void* ar_user, cudaStream_t st, LRAsync* async = nullptr,
+                  int grid_cap = 0);  // grid_cap > 0: at most that many CTAs per pass (layers trained side by side)
 // fp32 check mode: the same passes over fp32 rows (ld a multiple of 8)
 LRResult lr_train_f32(const float* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
                       const uint8_t* real_col_mask_host, int iters, int power_iters, double lambda, double alpha,

@@ -56,6 +56,10 @@ struct PassArgs {
   int64_t n_train;      // rows < n_train are train rows (eval mode)
   int ld, chunks;       // ld elements per row, chunks = ld * sizeof(E) / 16
   int rb;               // rows per streamed block
+  int rev;              // 1: every CTA walks its row blocks last-to-first (passes alternate, so each pass starts on
+                        //    the blocks the previous one read last -- still in L2)
+  int alt;              // 1: directions alternate (the next pass runs with rev ^ 1)
+  int pf_next;          // 1: the next pass reads the same rows -- the producer prefetches its first blocks into L2
   int dbg;              // VISTA_LR_DBG (measurement only, results wrong): 1 = dot kernel consumes blocks without computing
   const float* mu;      // [ld]
   const float* what;    // [ld]  inv_j * (w_j or v_j), 0 on excluded / pad columns
@@ -135,7 +139,9 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_stream_kernel(const Pas
     // ---- producer warp ----
     if (lane == 0) {
       int it = 0;
-      for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++it) {
+      const int64_t nb_cta = nblk > (int64_t)blockIdx.x ? (nblk - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+      for (int64_t bi = 0; bi < nb_cta; ++bi, ++it) {
+        const int64_t blk = blockIdx.x + (a.rev ? nb_cta - 1 - bi : bi) * (int64_t)gridDim.x;
         const int stage = it % kStagesLR;
         if (it >= kStagesLR) mbar_wait(&empty[stage], ((it / kStagesLR) - 1) & 1);
         const int64_t r = a.r0 + blk * a.rb;
@@ -143,11 +149,19 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_stream_kernel(const Pas
         const uint32_t bytes = (uint32_t)nr * row_bytes;
         mbar_arrive_expect_tx(&full[stage], bytes);
         bulk_load(base + stage * stage_bytes, a.MM + (size_t)r * row_bytes, bytes, &full[stage]);
-        const int64_t pb = blk + (int64_t)kStagesLR * gridDim.x;
-        if (pb < nblk) {
+        const int64_t pi = bi + kStagesLR;  // the block one ring-length ahead in this pass's order
+        if (pi < nb_cta) {
+          const int64_t pb = blockIdx.x + (a.rev ? nb_cta - 1 - pi : pi) * (int64_t)gridDim.x;
           const int64_t pr = a.r0 + pb * a.rb;
           prefetch_l2_range(a.MM + (size_t)pr * row_bytes, (uint32_t)min((int64_t)a.rb, a.r1 - pr) * row_bytes);
         }
+      }
+      // the next pass's first blocks into L2 while this pass drains and reduces (with alternating directions
+      // they are the blocks just read: a no-op then)
+      for (int64_t k = 0; a.pf_next && k < nb_cta && k < kStagesLR + 2; ++k) {
+        const int64_t blk = blockIdx.x + ((a.rev ^ a.alt) ? nb_cta - 1 - k : k) * (int64_t)gridDim.x;
+        const int64_t pr = a.r0 + blk * a.rb;
+        prefetch_l2_range(a.MM + (size_t)pr * row_bytes, (uint32_t)min((int64_t)a.rb, a.r1 - pr) * row_bytes);
       }
     }
     return;
@@ -170,7 +184,9 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_stream_kernel(const Pas
   float sum_r = 0.f, sum_loss = 0.f;  // warp 0, lane = row within the block
   unsigned long long cnt[5] = {0, 0, 0, 0, 0};
   int it = 0;
-  for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++it) {
+  const int64_t nb_cta = nblk > (int64_t)blockIdx.x ? (nblk - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+  for (int64_t bi = 0; bi < nb_cta; ++bi, ++it) {
+    const int64_t blk = blockIdx.x + (a.rev ? nb_cta - 1 - bi : bi) * (int64_t)gridDim.x;
     const int stage = it % kStagesLR;
     mbar_wait(&full[stage], (it / kStagesLR) & 1);
     const int64_t r = a.r0 + blk * a.rb;
@@ -366,7 +382,9 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_dot_kernel(const PassAr
   if (warp == nwc) {  // producer warp: bulk copies of RB-row blocks into the ring
     if (lane == 0) {
       int it = 0;
-      for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++it) {
+      const int64_t nb_cta = nblk > (int64_t)blockIdx.x ? (nblk - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+      for (int64_t bi = 0; bi < nb_cta; ++bi, ++it) {
+        const int64_t blk = blockIdx.x + (a.rev ? nb_cta - 1 - bi : bi) * (int64_t)gridDim.x;
         const int stage = it % kStagesLR;
         if (it >= kStagesLR) mbar_wait(&empty[stage], ((it / kStagesLR) - 1) & 1);
         const int64_t r = a.r0 + blk * RB;
@@ -374,11 +392,19 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_dot_kernel(const PassAr
         mbar_arrive_expect_tx(&full[stage], bytes);
         bulk_load(base + stage * stage_bytes, a.MM + (size_t)r * row_bytes, bytes, &full[stage]);
         // the block one ring-length ahead goes to L2 now: more bytes in flight than the ring holds
-        const int64_t pb = blk + (int64_t)kStagesLR * gridDim.x;
-        if (pb < nblk) {
+        const int64_t pi = bi + kStagesLR;  // the block one ring-length ahead in this pass's order
+        if (pi < nb_cta) {
+          const int64_t pb = blockIdx.x + (a.rev ? nb_cta - 1 - pi : pi) * (int64_t)gridDim.x;
           const int64_t pr = a.r0 + pb * RB;
           prefetch_l2_range(a.MM + (size_t)pr * row_bytes, (uint32_t)min((int64_t)RB, a.r1 - pr) * row_bytes);
         }
+      }
+      // the next pass's first blocks into L2 while this pass drains and reduces (with alternating directions
+      // they are the blocks just read: a no-op then)
+      for (int64_t k = 0; a.pf_next && k < nb_cta && k < kStagesLR + 2; ++k) {
+        const int64_t blk = blockIdx.x + ((a.rev ^ a.alt) ? nb_cta - 1 - k : k) * (int64_t)gridDim.x;
+        const int64_t pr = a.r0 + blk * RB;
+        prefetch_l2_range(a.MM + (size_t)pr * row_bytes, (uint32_t)min((int64_t)RB, a.r1 - pr) * row_bytes);
       }
     }
     return;
@@ -400,7 +426,9 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_dot_kernel(const PassAr
   float sum_r = 0.f, sum_loss = 0.f;
   unsigned long long cnt[5] = {0, 0, 0, 0, 0};
   int it = 0;
-  for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++it) {
+  const int64_t nb_cta = nblk > (int64_t)blockIdx.x ? (nblk - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+  for (int64_t bi = 0; bi < nb_cta; ++bi, ++it) {
+    const int64_t blk = blockIdx.x + (a.rev ? nb_cta - 1 - bi : bi) * (int64_t)gridDim.x;
     const int stage = it % kStagesLR;
     const int64_t r = a.r0 + blk * RB;
     const int nr = (int)min((int64_t)RB, a.r1 - r);
@@ -1150,7 +1178,12 @@ static void launch_pass(const void* kern, const PassArgs& a, int grid, int threa
 }
 
 template <int MODE, typename E>
-static void run_pass(const PassArgs& a, const StreamCfg& c, cudaStream_t st) {
+static void run_pass(const PassArgs& a_in, const StreamCfg& c, cudaStream_t st) {
+  // alternating block order (PassArgs::rev): a per-thread pass counter picks the direction (VISTA_LR_REV=0: off)
+  PassArgs a = a_in;
+  static thread_local unsigned pass_no = 0;
+  a.alt = (c.dot2_ch > 0 || (getenv("VISTA_LR_REV") && getenv("VISTA_LR_REV")[0] == '0')) ? 0 : 1;
+  a.rev = a.alt ? (int)(pass_no++ & 1u) : 0;
   const bool coop = a.f.on != 0;
   if constexpr (MODE >= 2 && sizeof(E) == 2) {
     if (c.dot2_ch > 0) {
@@ -1220,7 +1253,7 @@ LRResult lr_collect(const LRAsync& a) {
 template <typename E>
 static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
                               const uint8_t* real_host, int iters, int power_iters, double lambda, double alpha,
-                              allreduce_fn allreduce, void* ar_user, cudaStream_t st, LRAsync* async) {
+                              allreduce_fn allreduce, void* ar_user, cudaStream_t st, LRAsync* async, int grid_cap) {
   LRResult res;
   constexpr int esz = (int)sizeof(E);
   if (ld % 8) fail(1, "lr: ld must be a multiple of 8");
@@ -1264,7 +1297,7 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   // by a handful of rows left one CTA walking all of them behind L2 latency (C1: 33 -> ~9 us per pass)
   auto grid_for_rows = [&](int64_t rows) {
     const int64_t blocks = std::max<int64_t>((rows + pass_rb - 1) / pass_rb, (ld + 127) / 128);
-    return (int)std::max<int64_t>(1, std::min<int64_t>(blocks, num_sms()));
+    return (int)std::max<int64_t>(1, std::min<int64_t>(blocks, grid_cap > 0 ? std::min(grid_cap, num_sms()) : num_sms()));
   };
   cfg.grid = grid_for_rows(n_train);
   const int grid_tr = cfg.grid;
@@ -1322,6 +1355,7 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   a.n_train = n_train;
   a.rb = cfg.rb;
   a.dbg = getenv("VISTA_LR_DBG") ? atoi(getenv("VISTA_LR_DBG")) : 0;
+  a.pf_next = (getenv("VISTA_LR_PFN") && getenv("VISTA_LR_PFN")[0] == '0') ? 0 : 1;  // A/B switch
   a.counts = nullptr;
   a.f.on = fused ? 1 : 0;
   a.f.ncols = ncols;
@@ -1407,6 +1441,7 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
     e.r1 = n_rows;
     e.counts = cnt;
     e.f.on = 0;
+    e.pf_next = 0;  // the last pass of this layer
     StreamCfg ce = cfg;
     ce.grid = grid_for_rows(n_rows);
     prof_begin(st);
@@ -1469,16 +1504,16 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
 
 LRResult lr_train(const bf16* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
                   const uint8_t* real_host, int iters, int power_iters, double lambda, double alpha,
-                  allreduce_fn allreduce, void* ar_user, cudaStream_t st, LRAsync* async) {
+                  allreduce_fn allreduce, void* ar_user, cudaStream_t st, LRAsync* async, int grid_cap) {
   return lr_train_impl<bf16>(MM, y, n_rows, n_train, ld, real_host, iters, power_iters, lambda, alpha, allreduce,
-                             ar_user, st, async);
+                             ar_user, st, async, grid_cap);
 }
 
 LRResult lr_train_f32(const float* MM, const uint8_t* y, int64_t n_rows, int64_t n_train, int ld,
                       const uint8_t* real_host, int iters, int power_iters, double lambda, double alpha,
                       allreduce_fn allreduce, void* ar_user, cudaStream_t st) {
   return lr_train_impl<float>(MM, y, n_rows, n_train, ld, real_host, iters, power_iters, lambda, alpha, allreduce,
-                              ar_user, st, nullptr);
+                              ar_user, st, nullptr, 0);
 }
 
 }  // namespace vista

@@ -317,6 +317,7 @@ struct vista_ctx {
   int graph_state = 0;           // last transfer: 0 eager, 1 captured, 2 replayed
   // vista_run: M of layer k on a second stream beside stage k+1 (pinned result buffers per layer)
   cudaStream_t lr_stream = nullptr;
+  std::vector<cudaStream_t> lr_streams;  // batched M: one stream per layer
   struct LRJobBuf {
     void* pinned = nullptr;
     size_t bytes = 0;
@@ -374,6 +375,8 @@ struct vista_ctx {
       if (g.exec) cudaGraphExecDestroy(g.exec);
     if (cap_stream) cudaStreamDestroy(cap_stream);
     if (lr_stream) cudaStreamSynchronize(lr_stream);
+    for (cudaStream_t q : lr_streams)
+      if (q) cudaStreamSynchronize(q);
     for (auto& j : lr_jobs) {
       if (j.pinned) cudaFreeHost(j.pinned);
       if (j.done) cudaEventDestroy(j.done);
@@ -381,6 +384,8 @@ struct vista_ctx {
     for (cudaEvent_t e : lr_ready)
       if (e) cudaEventDestroy(e);
     if (lr_stream) cudaStreamDestroy(lr_stream);
+    for (cudaStream_t q : lr_streams)
+      if (q) cudaStreamDestroy(q);
     if (own_stream && stream) cudaStreamDestroy(stream);
     for (cudaEvent_t e : px_ready) cudaEventDestroy(e);
     if (px_free) cudaEventDestroy(px_free);
@@ -1476,7 +1481,7 @@ static std::vector<uint8_t> real_cols(const vista_ctx* c, int k) {
   return real;
 }
 
-static LRResult train_layer(vista_ctx* c, int k, cudaStream_t st, LRAsync* async) {
+static LRResult train_layer(vista_ctx* c, int k, cudaStream_t st, LRAsync* async, int grid_cap = 0) {
   const int ld = ld_of(c, k);
   const std::vector<uint8_t> real = real_cols(c, k);
   allreduce_fn ar = nullptr;
@@ -1489,7 +1494,84 @@ static LRResult train_layer(vista_ctx* c, int k, cudaStream_t st, LRAsync* async
                                real.data(), c->lr.iters, c->lr.power_iters, c->lr.lambda, c->lr.alpha, ar, ar_user, st)
                 : lr_train((const bf16*)c->MM[k]->p, (const uint8_t*)c->Y[k]->p, c->n_pairs, c->n_train, ld,
                            real.data(), c->lr.iters, c->lr.power_iters, c->lr.lambda, c->lr.alpha, ar, ar_user, st,
-                           async);
+                           async, grid_cap);
+}
+
+static void train_outputs(const vista_ctx* c, int k, const LRResult& r, double* weights_out, vista_metrics* m);
+
+// Bytes one LR training of layer k reads (2 stats + K power + T ISTA passes over the train rows, one eval pass)
+static double lr_bytes(const vista_ctx* c, int k) {
+  return 2.0 * ld_of(c, k) *
+         ((double)(2 + c->lr.power_iters + c->lr.iters) * (double)c->n_train + (double)c->n_pairs);
+}
+
+// M of every layer at once (one rank, bf16): each layer's pass sequence on its own stream with a share of the
+// SMs proportional to its bytes, so the five sequences run side by side.  A single layer's passes are
+// latency-bound at the ends (launch, ramp-up, the fused tail's grid barriers: ~20 us of a 60-90 us pass);
+// side by side those gaps overlap other layers' streaming.  The cooperative grids fit together
+// (sum of grids <= SM count, one CTA per SM), so every grid is co-resident.  Results collected per layer.
+static void train_all_batched(vista_ctx* c, double* const* weights_out, vista_metrics* out) {
+  const int L = (int)c->taps.size();
+  const int sms = num_sms();
+  std::vector<double> w(L);
+  double tot = 0;
+  for (int k = 0; k < L; ++k) tot += (w[k] = lr_bytes(c, k));
+  std::vector<int> g(L);
+  int used = 0;
+  for (int k = 0; k < L; ++k) {
+    const int lo = std::min(sms / L, (ld_of(c, k) + 127) / 128);  // >= one CTA per 128 columns where possible
+    g[k] = std::max(std::max(1, lo), (int)std::floor(sms * w[k] / std::max(tot, 1.0)));
+    used += g[k];
+  }
+  while (used > sms) {  // trim the largest share
+    int kb = 0;
+    for (int k = 1; k < L; ++k) kb = g[k] > g[kb] ? k : kb;
+    --g[kb];
+    --used;
+  }
+  if ((int)c->lr_streams.size() < L) c->lr_streams.resize(L, nullptr);
+  c->lr_jobs.resize(L);
+  c->lr_ready.resize(L, nullptr);
+  for (int k = 0; k < L; ++k) {
+    if (!c->lr_streams[k]) VCHECK(cudaStreamCreateWithFlags(&c->lr_streams[k], cudaStreamNonBlocking));
+    vista_ctx::LRJobBuf& jb = c->lr_jobs[k];
+    const size_t need = lr_async_bytes(ld_of(c, k), c->lr.iters);
+    if (jb.bytes < need) {
+      if (jb.pinned) VCHECK(cudaFreeHost(jb.pinned));
+      jb.pinned = nullptr;
+      VCHECK(cudaMallocHost(&jb.pinned, need));
+      jb.bytes = need;
+    }
+    if (!c->lr_ready[k]) VCHECK(cudaEventCreateWithFlags(&c->lr_ready[k], cudaEventDisableTiming));
+  }
+  // one profile record for the whole batch (per-launch events on five streams would charge each other's time)
+  Profiler* prof = g_prof;
+  if (prof) prof_begin(c->stream);
+  g_prof = nullptr;
+  cudaEvent_t fork = c->lr_ready[0];
+  VCHECK(cudaEventRecord(fork, c->stream));
+  std::vector<LRAsync> jobs(L);
+  for (int k = 0; k < L; ++k) {
+    VCHECK(cudaStreamWaitEvent(c->lr_streams[k], fork, 0));
+    jobs[k].pinned = c->lr_jobs[k].pinned;
+    jobs[k].bytes = c->lr_jobs[k].bytes;
+    jobs[k].done = c->lr_jobs[k].done;
+    train_layer(c, k, c->lr_streams[k], &jobs[k], g[k]);
+    c->lr_jobs[k].done = jobs[k].done;
+  }
+  for (int k = 0; k < L; ++k) VCHECK(cudaStreamWaitEvent(c->stream, jobs[k].done, 0));
+  g_prof = prof;
+  if (prof) {
+    double bytes = 0;
+    for (int k = 0; k < L; ++k) bytes += w[k];
+    char label[96];
+    std::snprintf(label, sizeof(label), "LR batched: %d layers side by side", L);
+    prof_end(c->stream, 5, 0, bytes, prof_labels() ? label : nullptr);
+  }
+  for (int k = 0; k < L; ++k) {
+    const LRResult r = lr_collect(jobs[k]);
+    train_outputs(c, k, r, weights_out ? weights_out[k] : nullptr, out ? out + k : nullptr);
+  }
 }
 
 static void train_outputs(const vista_ctx* c, int k, const LRResult& r, double* weights_out, vista_metrics* m) {
@@ -1542,6 +1624,15 @@ VISTA_API vista_status vista_run(vista_ctx* c, const uint8_t* images, const int6
   if (!c) return VISTA_ERR_INVALID_ARG;
   return guarded(c, [&] {
     const int L = (int)c->taps.size();
+    // one rank, bf16: all layers' M side by side after the transfer (VISTA_LR_BATCH=0: the per-layer schedules)
+    const bool batch = c->sys.world == 1 && !c->f32 && L > 1 &&
+                       !(getenv("VISTA_LR_BATCH") && getenv("VISTA_LR_BATCH")[0] == '0');
+    if (batch) {
+      transfer_body(c, images, nullptr, image_keys, structured, str_keys, labels);
+      train_all_batched(c, weights_out, out);
+      if (g_prof) g_prof->flush();
+      return;
+    }
     static const bool overlap_on = !(getenv("VISTA_OVERLAP") && getenv("VISTA_OVERLAP")[0] == '0');
     // (profiling times every launch with CUDA events on its stream: kernels of the two streams would be
     // charged each other's time, so the profiled run trains after the transfer)

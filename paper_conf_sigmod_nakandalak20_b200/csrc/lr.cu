@@ -65,6 +65,7 @@ struct PassArgs {
   const float* what;    // [ld]  inv_j * (w_j or v_j), 0 on excluded / pad columns
   const float* bhat;    // [1]
   float* partial;       // [gridDim.x][ld + 4] (16-byte aligned rows; ld + 2 used)
+  float* zbuf;          // [r1] lr_dot_kernel MODE 3: per-row scores, the loss is summed after the row loop
   unsigned long long* counts;  // eval: [5]
   FusedArgs f;
 };
@@ -442,6 +443,7 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_dot_kernel(const PassAr
     const uint8_t* sb = gbase + stage * stage_bytes;
     float* red = red_all + stage * (kMaxRB * 32);
     float sd[16];
+    if (a.dbg != 3) {
 #pragma unroll
     for (int q = 0; q < RB; ++q) {
       float2 s2 = make_float2(0.f, 0.f);
@@ -458,9 +460,10 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_dot_kernel(const PassAr
     butterfly<RB>(sd, lane);
     if ((lane & ((32 >> LOGRB) - 1)) == 0) red[(lane >> (5 - LOGRB)) * 32 + warp] = sd[0];
     named_bar_sync(1, nthr);
+    }
     // every warp: lane q < nr forms z_q from the per-warp partials (fixed order) and phi_q
-    float phi = 0.f;
-    if (lane < nr) {
+    float phi = a.dbg == 3 ? 1.f : 0.f;
+    if (lane < nr && a.dbg != 3) {
       float z = bh;
       const float* rq = red + lane * 32;
       for (int w = 0; w < nwc; ++w) z += rq[w];
@@ -473,7 +476,7 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_dot_kernel(const PassAr
           phi = 1.f / (1.f + __expf(-z)) - (float)yv;
           if (warp == 0) {
             sum_r += phi;
-            sum_loss += softplusf(z) - (float)yv * z;
+            a.zbuf[row] = z;  // loss after the row loop (softplus off the per-block chain)
           }
         } else if (warp == 0) {  // MODE 4: predict 1 iff z >= 0
           const int pred = z >= 0.f ? 1 : 0;
@@ -482,7 +485,7 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_dot_kernel(const PassAr
         }
       }
     }
-    if (MODE != 4) {
+    if (MODE != 4 && a.dbg != 2) {
 #pragma unroll
       for (int q = 0; q < RB; ++q) {
         if (q < nr) {  // block-uniform
@@ -512,6 +515,25 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_dot_kernel(const PassAr
     }
     return;
   } else {
+    if constexpr (MODE == 3) {
+      // sum_p softplus(z_p) - y_p z_p over this CTA's rows (scores stored by warp 0), fixed order: thread-strided
+      // partial sums, warp shuffles, then the warps in order
+      __threadfence_block();
+      named_bar_sync(1, nthr);
+      float l = 0.f;
+      for (int64_t i = tid; i < nb_cta * RB; i += nthr) {
+        const int64_t row = a.r0 + (blockIdx.x + (i / RB) * (int64_t)gridDim.x) * RB + (i % RB);
+        if (row < a.r1) {
+          const float z = a.zbuf[row];
+          l += softplusf(z) - (float)a.y[row] * z;
+        }
+      }
+      for (int o = 16; o > 0; o >>= 1) l += __shfl_xor_sync(0xffffffffu, l, o);
+      if (lane == 0) red_all[warp] = l;
+      named_bar_sync(1, nthr);
+      sum_loss = 0.f;
+      for (int w = 0; w < nwc; ++w) sum_loss += red_all[w];
+    }
     float* out = a.partial + (size_t)blockIdx.x * (a.ld + 4);
 #pragma unroll
     for (int c = 0; c < CH; ++c) {
@@ -523,13 +545,10 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_dot_kernel(const PassAr
       }
     }
     if (warp == 0) {
-      for (int o = 16; o > 0; o >>= 1) {
-        sum_r += __shfl_xor_sync(0xffffffffu, sum_r, o);
-        sum_loss += __shfl_xor_sync(0xffffffffu, sum_loss, o);
-      }
+      for (int o = 16; o > 0; o >>= 1) sum_r += __shfl_xor_sync(0xffffffffu, sum_r, o);
       if (lane == 0) {
         out[a.ld] = sum_r;
-        out[a.ld + 1] = sum_loss;
+        out[a.ld + 1] = sum_loss;  // MODE 3: the CTA total above; MODE 2: 0
       }
     }
     if (a.f.on) fused_tail<MODE>(a, gbase, nthr);
@@ -1321,7 +1340,8 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
                o_muf = carve(ld * 4), o_inv = carve(ld * 8), o_v = carve(ld * 8), o_w = carve(ld * 8),
                o_what = carve(ld * 4), o_bhat = carve(16), o_st = carve(sizeof(LRState)),
                o_real = carve(ld), o_loss = carve((size_t)(iters + 1) * 8), o_cnt = carve(64),
-               o_bar = carve(16), o_scal = carve((size_t)2 * std::max(grid_tr, 1) * 8);
+               o_bar = carve(16), o_scal = carve((size_t)2 * std::max(grid_tr, 1) * 8),
+               o_z = carve((size_t)std::max<int64_t>(n_train, 1) * 4);
   uint8_t* scr = nullptr;
   VCHECK(cudaMallocAsync(&scr, off, st));
   VCHECK(cudaMemsetAsync(scr, 0, off, st));  // every byte defined (LRState fields a path leaves unwritten)
@@ -1352,6 +1372,7 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   a.what = what;
   a.bhat = bhat;
   a.partial = partial;
+  a.zbuf = reinterpret_cast<float*>(scr + o_z);
   a.n_train = n_train;
   a.rb = cfg.rb;
   a.dbg = getenv("VISTA_LR_DBG") ? atoi(getenv("VISTA_LR_DBG")) : 0;

@@ -174,16 +174,23 @@ __global__ void __launch_bounds__((kEpiWarp0 + EPW) * 32, 1)
         const int j_lo = 3 - r_hi, cnt = r_hi - r_lo + 1;  // weight groups j_lo .. j_lo + cnt - 1 (j = 3 - r)
         const uint32_t s0 = (orow + (uint32_t)(i - r_hi)) % kNAcc;  // slot of output row i - r_hi
         const uint32_t n1 = (uint32_t)cnt < kNAcc - s0 ? (uint32_t)cnt : kNAcc - s0;
-        const uint64_t da = umma_desc_k_sw128(sA + slot * kRowBytes);
-        auto issue = [&](uint32_t col, uint32_t jg, uint32_t ng) {
-          const uint32_t idesc = umma_idesc_bf16(128, 64 * ng);
-          const uint64_t db = umma_desc_k_sw128(sB + jg * 64 * 128);
-          const uint32_t tacc = tmem_base + col * kCo;
+        // 32-bit descriptor halves (SW128 K-major; K step = 32 B = 2 units, weight group = 8 KB = 512 units) and
+        // separate straight / wrapped paths: the MMA warp's per-row issue chain, not the tensor pipe, bounded
+        // the kernel (ncu: tensor pipe 70 %, the epilogue waiting on full accumulators)
+        const uint32_t a_lo = umma_desc_lo_sw128(sA + slot * kRowBytes);
+        const uint32_t b_lo = umma_desc_lo_sw128(sB + (uint32_t)j_lo * 64 * 128);
+        const uint32_t t0 = tmem_base + s0 * kCo, id1 = umma_idesc_bf16(128, 64 * n1);
+        if ((uint32_t)cnt == n1) {
 #pragma unroll
-          for (int k = 0; k < 4; ++k) tc_mma_bf16_warp(tacc, da + 2 * k, db + 2 * k, idesc, 1u);
-        };
-        issue(s0, (uint32_t)j_lo, n1);
-        if ((uint32_t)cnt > n1) issue(0, (uint32_t)j_lo + n1, (uint32_t)cnt - n1);
+          for (int k = 0; k < 4; ++k) tc_mma_bf16_lo_warp(t0, a_lo + 2 * k, b_lo + 2 * k, id1, 1u);
+        } else {
+          const uint32_t id2 = umma_idesc_bf16(128, 64 * ((uint32_t)cnt - n1)), b2 = b_lo + n1 * 512u;
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            tc_mma_bf16_lo_warp(t0, a_lo + 2 * k, b_lo + 2 * k, id1, 1u);
+            tc_mma_bf16_lo_warp(tmem_base, a_lo + 2 * k, b2 + 2 * k, id2, 1u);
+          }
+        }
         tc_commit_warp(&empty[slot]);  // input row i feeds no later MMA
         if (i >= 3) tc_commit_warp(&tfull[(orow + i - 3) % kNAcc]);  // output row i - 3 is complete
       }

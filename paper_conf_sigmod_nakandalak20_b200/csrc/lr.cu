@@ -565,7 +565,7 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_dot_kernel(const PassAr
 // chunks (tg, tg + 32 kGW, ...) in BOTH groups with separate accumulators; at the end group 1's sums are
 // added to group 0's in a fixed order (deterministic).
 constexpr int kGW = 9;         // warps per consumer group
-constexpr int kStages2 = 6;    // two-row blocks in flight per CTA (three per group)
+constexpr int kStages2 = 5;    // two-row blocks in flight per CTA
 template <int CH, int MODE>
 __global__ void __launch_bounds__(2 * kGW * 32 + 32, 1) lr_dot2_kernel(const PassArgs a) {
   constexpr int RB = 2, NG = kGW * 32;
@@ -578,6 +578,8 @@ __global__ void __launch_bounds__(2 * kGW * 32 + 32, 1) lr_dot2_kernel(const Pas
   float* red_all = reinterpret_cast<float*>(gbase + kStages2 * stage_bytes);  // [kStages2][RB][16]
   uint64_t* full = reinterpret_cast<uint64_t*>(red_all + kStages2 * RB * 16);
   uint64_t* empty = full + kStages2;
+  // w^ in shared memory (fp32, 8 zeros past the end for inactive chunks): keeps CH = 4 free of spills
+  float* wsm = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(empty + kStages2) + 16);
   const int nthr = 2 * NG;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int grp = warp / kGW, gw = warp - grp * kGW, tg = tid - grp * NG;
@@ -610,18 +612,18 @@ __global__ void __launch_bounds__(2 * kGW * 32 + 32, 1) lr_dot2_kernel(const Pas
     }
     return;
   }
-  uint32_t coff[CH];
-  float2 wv[CH][4], acc[CH][4];
+  for (int i = tid; i < a.chunks * 8 + 8; i += nthr) wsm[i] = i < a.chunks * 8 ? a.what[i] : 0.f;
+  named_bar_sync(2, nthr);
+  uint32_t coff[CH], woff[CH];
+  float2 acc[CH][4];
 #pragma unroll
   for (int c = 0; c < CH; ++c) {
     const int ch = tg + c * NG;
     const bool act = ch < a.chunks;
     coff[c] = act ? (uint32_t)ch * 16u : 0u;
+    woff[c] = act ? (uint32_t)ch * 8u : (uint32_t)a.chunks * 8u;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      wv[c][j] = act ? make_float2(a.what[ch * 8 + 2 * j], a.what[ch * 8 + 2 * j + 1]) : make_float2(0.f, 0.f);
-      acc[c][j] = make_float2(0.f, 0.f);
-    }
+    for (int j = 0; j < 4; ++j) acc[c][j] = make_float2(0.f, 0.f);
   }
   const float bh = a.bhat[0];
   float sum_r = 0.f, sum_loss = 0.f;
@@ -641,10 +643,12 @@ __global__ void __launch_bounds__(2 * kGW * 32 + 32, 1) lr_dot2_kernel(const Pas
 #pragma unroll
       for (int c = 0; c < CH; ++c) {
         const uint4 v = *reinterpret_cast<const uint4*>(sb + q * row_bytes + coff[c]);
-        s2 = ffma2(bf2_f2(v.x), wv[c][0], s2);
-        s2 = ffma2(bf2_f2(v.y), wv[c][1], s2);
-        s2 = ffma2(bf2_f2(v.z), wv[c][2], s2);
-        s2 = ffma2(bf2_f2(v.w), wv[c][3], s2);
+        const float4 w0 = *reinterpret_cast<const float4*>(wsm + woff[c]);
+        const float4 w1 = *reinterpret_cast<const float4*>(wsm + woff[c] + 4);
+        s2 = ffma2(bf2_f2(v.x), make_float2(w0.x, w0.y), s2);
+        s2 = ffma2(bf2_f2(v.y), make_float2(w0.z, w0.w), s2);
+        s2 = ffma2(bf2_f2(v.z), make_float2(w1.x, w1.y), s2);
+        s2 = ffma2(bf2_f2(v.w), make_float2(w1.z, w1.w), s2);
       }
       sd[q] = s2.x + s2.y;
     }
@@ -1305,7 +1309,7 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   if (cfg.dot_rb > 0 && dot2_env && atoi(dot2_env) > 0 && ld >= atoi(dot2_env)) {
     const int ch2 = (chunks + kGW * 32 - 1) / (kGW * 32);
     const size_t sb2 = ((size_t)2 * ld * 2 + 127) & ~(size_t)127;
-    const size_t smem2 = kStages2 * sb2 + kStages2 * 2 * 16 * 4 + 2 * kStages2 * 8 + 128;
+    const size_t smem2 = kStages2 * sb2 + kStages2 * 2 * 16 * 4 + 2 * kStages2 * 8 + 16 + ((size_t)chunks * 8 + 8) * 4 + 128;
     if (ch2 <= 4 && smem2 <= 227 * 1024) {
       cfg.dot2_ch = ch2;
       cfg.dot2_smem = smem2;

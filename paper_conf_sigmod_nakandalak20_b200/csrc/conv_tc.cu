@@ -1345,15 +1345,18 @@ static CUresult encode_nd(CUtensorMap* m, const void* ptr, int rank, const cuuin
 }
 
 bool make_nd_tmap(CUtensorMap* m, const void* ptr, int rank, const uint64_t* dims, const uint64_t* strides,
-                  const uint32_t* box) {
+                  const uint32_t* box, bool swizzle128) {
   cuuint64_t d[5], s[4];
-  cuuint32_t b[5];
+  cuuint32_t b[5], estr[5] = {1, 1, 1, 1, 1};
   for (int i = 0; i < rank; ++i) {
     d[i] = dims[i];
     b[i] = box[i];
     if (i + 1 < rank) s[i] = strides[i];
   }
-  return encode_nd(m, ptr, rank, d, s, b) == CUDA_SUCCESS;
+  return get_encode()(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, (cuuint32_t)rank, const_cast<void*>(ptr), d, s, b, estr,
+                      CU_TENSOR_MAP_INTERLEAVE_NONE,
+                      swizzle128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE,
+                      CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 // [rows, cols] bf16 matrix, box {64, 128}, 128B swizzle (A operands / staged outputs of 128-row tiles)

@@ -1518,9 +1518,20 @@ static void train_all_batched(vista_ctx* c, double* const* weights_out, vista_me
   for (int k = 0; k < L; ++k) tot += (w[k] = lr_bytes(c, k));
   std::vector<int> g(L);
   int used = 0;
+  // VISTA_LR_SHARE="a,b,..." overrides the per-layer weights (measurement of other splits)
+  if (const char* e = getenv("VISTA_LR_SHARE")) {
+    tot = 0;
+    for (int k = 0; k < L; ++k) {
+      w[k] = atof(e);
+      tot += w[k];
+      e = strchr(e, ',');
+      if (!e) break;
+      ++e;
+    }
+  }
   for (int k = 0; k < L; ++k) {
-    const int lo = std::min(sms / L, (ld_of(c, k) + 127) / 128);  // >= one CTA per 128 columns where possible
-    g[k] = std::max(std::max(1, lo), (int)std::floor(sms * w[k] / std::max(tot, 1.0)));
+    const int lo = std::min(8, (ld_of(c, k) + 127) / 128);  // a few CTAs at least (the fused tail's column split)
+    g[k] = std::max(std::max(1, lo), (int)std::floor(sms * w[k] / std::max(tot, 1e-30)));
     used += g[k];
   }
   while (used > sms) {  // trim the largest share
@@ -1560,6 +1571,10 @@ static void train_all_batched(vista_ctx* c, double* const* weights_out, vista_me
     c->lr_jobs[k].done = jobs[k].done;
   }
   for (int k = 0; k < L; ++k) VCHECK(cudaStreamWaitEvent(c->stream, jobs[k].done, 0));
+  if (getenv("VISTA_LR_TIMES")) {  // per-layer completion times of the batch (measurement only)
+    VCHECK(cudaStreamSynchronize(c->stream));
+    for (int k = 0; k < L; ++k) fprintf(stderr, "lr layer %d: %d CTAs\n", k, g[k]);
+  }
   g_prof = prof;
   if (prof) {
     double bytes = 0;

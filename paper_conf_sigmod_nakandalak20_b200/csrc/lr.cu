@@ -73,6 +73,12 @@ struct PassArgs {
 template <int MODE>
 __device__ void fused_tail(const PassArgs& a, uint8_t* scratch, int nthr);
 
+// programmatic dependent launch (consecutive passes on one stream): a pass lets the next one launch as its CTAs
+// exit; the next pass's producer streams rows (MM is not written by any pass) while its compute threads wait
+// for the previous grid's results (w^, b', the reduced statistics)
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 __device__ __forceinline__ float softplusf(float z) { return z > 0.f ? z + log1pf(__expf(-z)) : log1pf(__expf(z)); }
 
 __device__ __forceinline__ void bulk_load(uint32_t dst, const void* src, uint32_t bytes, uint64_t* bar) {
@@ -136,6 +142,8 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_stream_kernel(const Pas
     fence_mbar_init();
   }
   __syncthreads();
+  pdl_trigger();
+  if (warp != nwc) pdl_wait();
   if (warp == nwc) {
     // ---- producer warp ----
     if (lane == 0) {
@@ -380,6 +388,8 @@ __global__ void __launch_bounds__(kLRThreads + 32, 1) lr_dot_kernel(const PassAr
     fence_mbar_init();
   }
   __syncthreads();
+  pdl_trigger();
+  if (warp != nwc) pdl_wait();
   if (warp == nwc) {  // producer warp: bulk copies of RB-row blocks into the ring
     if (lane == 0) {
       int it = 0;
@@ -593,6 +603,8 @@ __global__ void __launch_bounds__(2 * kGW * 32 + 32, 1) lr_dot2_kernel(const Pas
     fence_mbar_init();
   }
   __syncthreads();
+  pdl_trigger();
+  if (warp != 2 * kGW) pdl_wait();
   if (warp == 2 * kGW) {  // producer warp
     if (lane == 0) {
       int it = 0;
@@ -1190,13 +1202,26 @@ static void launch_pass(const void* kern, const PassArgs& a, int grid, int threa
                         cudaStream_t st) {
   ensure_smem_attr(kern, 227 * 1024);
   static const bool coop_ok = !(getenv("VISTA_LR_COOP") && getenv("VISTA_LR_COOP")[0] == '0');  // A/B only
+  static const bool pdl_ok = !(getenv("VISTA_LR_PDL") && getenv("VISTA_LR_PDL")[0] == '0');  // A/B only
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(threads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[2];
+  int na = 0;
   if (coop && coop_ok) {  // the fused tail's grid barriers need every CTA resident: cooperative launch guarantees it
-    void* args[] = {const_cast<PassArgs*>(&a)};
-    VCHECK(cudaLaunchCooperativeKernel(kern, dim3(grid), dim3(threads), args, smem, st));
-  } else {
-    void* args[] = {const_cast<PassArgs*>(&a)};
-    VCHECK(cudaLaunchKernel(kern, dim3(grid), dim3(threads), args, smem, st));
+    attr[na].id = cudaLaunchAttributeCooperative;
+    attr[na++].val.cooperative = 1;
   }
+  if (pdl_ok) {
+    attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[na++].val.programmaticStreamSerializationAllowed = 1;
+  }
+  cfg.attrs = attr;
+  cfg.numAttrs = na;
+  void* args[] = {const_cast<PassArgs*>(&a)};
+  VCHECK(cudaLaunchKernelExC(&cfg, kern, args));
   LAUNCHED();
 }
 

@@ -30,7 +30,13 @@ constexpr int kPo = 56;            // pool1 output (114 - 3) / 2 + 1
 constexpr int kCo = 64;            // conv1 channels
 constexpr int kSA = 6;             // input-row ring slots (rows 24 ahead are prefetched into L2)
 constexpr int kNAcc = 8;           // TMEM accumulators (64 columns each; the classic issue order uses 4)
-constexpr int kRowBytes = 128 * 128;  // one A slot: 128 pixel rows x 64 bf16 (128B-swizzled)
+// One A slot = one space-to-depth input row, K-major with 32-byte swizzle: row q = position q's 16 channels (32 B).
+// K step k (s2d position offset k of a filter row) is the slot shifted by k rows, so each input position lands in
+// shared memory once (4.2 KB per row; the 128B-swizzled overlapping row view wrote each position four times,
+// 16 KB per row -- the stem is shared-memory bound).  VISTA_STEM_SW32=0 keeps the row view (A/B).
+constexpr int kRowPos = 131;                               // 128 M rows + 3 shifts
+constexpr int kRowBytes = 128 * 128;                       // slot stride (the row view's 16 KB; SW32 uses 4.2 KB of it)
+constexpr int kRowTx32 = kRowPos * 32;
 constexpr int kBBytes = 4 * 64 * 128;  // 4 k-blocks x 64 output channels x 64 bf16
 constexpr int kCrowBytes = 128 * 128;  // conv row: 128 pixels x 64 channels bf16
 constexpr int kCrowBufs = 4;           // staged conv rows (two rows per epilogue step, double-buffered)
@@ -53,6 +59,7 @@ struct PoolParams {
   // Versus the row-major order (16 N = 64 MMAs per output row, shared-memory operand bound at 48 cycles
   // each): half the shared-memory operand bytes and full-rate N >= 128 instructions.
   int irow;
+  int sw32;  // 1: A slots in the 32B-swizzled one-position-per-row layout (see kRowPos)
 };
 
 __device__ __forceinline__ uint4 max4(uint4 a, uint4 b) {
@@ -152,7 +159,7 @@ __global__ void __launch_bounds__((kEpiWarp0 + EPW) * 32, 1)
           if (i % kPfGroup == 0) prefetch_rows(n, i + kPfAhead);
           const int slot = g % kSA;
           if (g >= (uint32_t)kSA) mbar_wait(&empty[slot], ((g / kSA) - 1) & 1);
-          mbar_arrive_expect_tx(&full[slot], kRowBytes);
+          mbar_arrive_expect_tx(&full[slot], p.sw32 ? kRowTx32 : kRowBytes);
           tma_load_4d(sA + slot * kRowBytes, &tmap_a, 0, 0, i, n, &full[slot]);
         }
       }
@@ -177,18 +184,21 @@ __global__ void __launch_bounds__((kEpiWarp0 + EPW) * 32, 1)
         // 32-bit descriptor halves (SW128 K-major; K step = 32 B = 2 units, weight group = 8 KB = 512 units) and
         // separate straight / wrapped paths: the MMA warp's per-row issue chain, not the tensor pipe, bounded
         // the kernel (ncu: tensor pipe 70 %, the epilogue waiting on full accumulators)
-        const uint32_t a_lo = umma_desc_lo_sw128(sA + slot * kRowBytes);
-        const uint32_t b_lo = umma_desc_lo_sw128(sB + (uint32_t)j_lo * 64 * 128);
+        // K step k: A = the 32-byte K slice k of the row view (+2 units), or with sw32 the slot shifted by k
+        // 32-byte rows (+2 units as well); B = the weights' 32-byte K slice k of the 128B-swizzled groups
+        const uint64_t da = p.sw32 ? umma_desc_k_sw32(sA + slot * kRowBytes) : umma_desc_k_sw128(sA + slot * kRowBytes);
+        const uint64_t db = umma_desc_k_sw128(sB + (uint32_t)j_lo * 64 * 128);
         const uint32_t t0 = tmem_base + s0 * kCo, id1 = umma_idesc_bf16(128, 64 * n1);
         if ((uint32_t)cnt == n1) {
 #pragma unroll
-          for (int k = 0; k < 4; ++k) tc_mma_bf16_lo_warp(t0, a_lo + 2 * k, b_lo + 2 * k, id1, 1u);
+          for (int k = 0; k < 4; ++k) tc_mma_bf16_warp(t0, da + 2 * k, db + 2 * k, id1, 1u);
         } else {
-          const uint32_t id2 = umma_idesc_bf16(128, 64 * ((uint32_t)cnt - n1)), b2 = b_lo + n1 * 512u;
+          const uint32_t id2 = umma_idesc_bf16(128, 64 * ((uint32_t)cnt - n1));
+          const uint64_t db2 = db + n1 * 512u;
 #pragma unroll
           for (int k = 0; k < 4; ++k) {
-            tc_mma_bf16_lo_warp(t0, a_lo + 2 * k, b_lo + 2 * k, id1, 1u);
-            tc_mma_bf16_lo_warp(tmem_base, a_lo + 2 * k, b2 + 2 * k, id2, 1u);
+            tc_mma_bf16_warp(t0, da + 2 * k, db + 2 * k, id1, 1u);
+            tc_mma_bf16_warp(tmem_base, da + 2 * k, db2 + 2 * k, id2, 1u);
           }
         }
         tc_commit_warp(&empty[slot]);  // input row i feeds no later MMA
@@ -214,7 +224,8 @@ __global__ void __launch_bounds__((kEpiWarp0 + EPW) * 32, 1)
             const uint32_t slot = row % kSA;
             // (TMA completion on the mbarrier orders the smem writes before the async-proxy MMA reads)
             mbar_wait(&full[slot], (row / kSA) & 1);
-            const uint64_t da = umma_desc_k_sw128(sA + slot * kRowBytes), db = umma_desc_k_sw128(sB + r * 64 * 128);
+            const uint64_t da = p.sw32 ? umma_desc_k_sw32(sA + slot * kRowBytes) : umma_desc_k_sw128(sA + slot * kRowBytes);
+            const uint64_t db = umma_desc_k_sw128(sB + r * 64 * 128);
             // +32 bytes along K = +2 in the descriptors' address fields
             tc_mma_bf16_warp(tacc, da, db, idesc, r != 0 ? 1u : 0u);
             tc_mma_bf16_warp(tacc, da + 2, db + 2, idesc, 1u);
@@ -356,8 +367,16 @@ void conv1_pool_forward(const ConvLayer& L, const bf16* x, int N, bf16* y, cudaS
   if (N <= 0) return;
   CUtensorMap ta;
   // overlapping row view {64 elements, q < 114, h, n}: element (k, q, h, n) = x[n, h, q + k / 16, k % 16]
-  if (!make_rowview_tmap(&ta, x, N, kHin, kHin, kS2dC, kHo)) fail(5, "conv1_pool: row-view tensor map failed");
   PoolParams p;
+  p.sw32 = !(getenv("VISTA_STEM_SW32") && getenv("VISTA_STEM_SW32")[0] == '0');
+  if (p.sw32) {  // {16 ch, kRowPos positions from 0 (>= 117 read zeros), 1 row, 1 image}, 32-byte swizzle
+    const uint64_t dims[4] = {(uint64_t)kS2dC, (uint64_t)kHin, (uint64_t)kHin, (uint64_t)N};
+    const uint64_t strides[3] = {(uint64_t)kS2dC * 2, (uint64_t)kHin * kS2dC * 2, (uint64_t)kHin * kHin * kS2dC * 2};
+    const uint32_t box[4] = {(uint32_t)kS2dC, (uint32_t)kRowPos, 1, 1};
+    if (!make_nd_tmap(&ta, x, 4, dims, strides, box, 32)) fail(5, "conv1_pool: input tensor map failed");
+  } else if (!make_rowview_tmap(&ta, x, N, kHin, kHin, kS2dC, kHo)) {
+    fail(5, "conv1_pool: row-view tensor map failed");
+  }
   p.x = x;
   p.y = y;
   p.scale = L.scale;

@@ -1345,7 +1345,7 @@ static CUresult encode_nd(CUtensorMap* m, const void* ptr, int rank, const cuuin
 }
 
 bool make_nd_tmap(CUtensorMap* m, const void* ptr, int rank, const uint64_t* dims, const uint64_t* strides,
-                  const uint32_t* box, bool swizzle128) {
+                  const uint32_t* box, int swizzle_bytes) {
   cuuint64_t d[5], s[4];
   cuuint32_t b[5], estr[5] = {1, 1, 1, 1, 1};
   for (int i = 0; i < rank; ++i) {
@@ -1355,7 +1355,8 @@ bool make_nd_tmap(CUtensorMap* m, const void* ptr, int rank, const uint64_t* dim
   }
   return get_encode()(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, (cuuint32_t)rank, const_cast<void*>(ptr), d, s, b, estr,
                       CU_TENSOR_MAP_INTERLEAVE_NONE,
-                      swizzle128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE,
+                      swizzle_bytes == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                           : (swizzle_bytes == 32 ? CU_TENSOR_MAP_SWIZZLE_32B : CU_TENSOR_MAP_SWIZZLE_NONE),
                       CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 

@@ -68,7 +68,7 @@ void conv_cat_forward(const ConvLayer& L, int Cx, const bf16* b, const bf16* x, 
 bool make_rowview_tmap(CUtensorMap* m, const void* x, int N, int H, int W, int C, int Wo);
 // N-D bf16 tiled tensor map, 128B swizzle, out-of-bounds elements read as zero
 bool make_nd_tmap(CUtensorMap* m, const void* ptr, int rank, const uint64_t* dims, const uint64_t* strides,
-                  const uint32_t* box, bool swizzle128 = true);
+                  const uint32_t* box, int swizzle_bytes = 128);  // 128, 32 or 0
 // 3x3 / 1 / pad 1 conv with Cin = Cout = 64 and W <= 62 (ResNet res2) issued input-row-major with N = 192
 // MMAs (conv3x3_rows.cu), bit-identical to the conv_tc halo path; VISTA_ROWCONV=0 disables it
 bool rowconv3x3_supported(const ConvLayer& L, int H, int W);

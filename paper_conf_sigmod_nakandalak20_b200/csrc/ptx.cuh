@@ -422,6 +422,18 @@ __device__ __forceinline__ uint64_t umma_desc_k_none(uint32_t smem_addr, uint32_
   return d;
 }
 
+// K-major, 32-byte swizzle: rows of 32 B (K = 16 bf16), 8-row atoms of 256 B (SBO).  Like the 128B form, the
+// swizzle follows the absolute shared-memory address, so a start shifted by whole 32-byte rows stays valid.
+__device__ __forceinline__ uint64_t umma_desc_k_sw32(uint32_t smem_addr) {
+  uint64_t d = 0;
+  d |= (uint64_t)((smem_addr >> 4) & 0x3FFFu);
+  d |= (uint64_t)1 << 16;                 // LBO (unused for swizzled K-major)
+  d |= (uint64_t)(256u >> 4) << 32;       // SBO: 8 rows x 32 B
+  d |= (uint64_t)1 << 46;                 // version = 1 (sm_100)
+  d |= (uint64_t)6 << 61;                 // layout = SWIZZLE_32B
+  return d;
+}
+
 // Instruction descriptor, kind::f16: A = B = bf16, D = f32, both K-major, M x N tile.
 __host__ __device__ constexpr uint32_t umma_idesc_bf16(uint32_t M, uint32_t N) {
   return (1u << 4)            // D format f32

@@ -2,7 +2,7 @@
 every conv A-operand mode, the fused stem, the residual chains, projection units, weight multicast,
 the tap, join, concat, and both LR paths (fused cooperative tail and the reduce/update kernels).
 
-usage: python tools/sanitize_case.py <case>   cases: resnet, resnet_mc, alexnet, vgg, lr_unfused, mlp"""
+usage: python tools/sanitize_case.py <case>   cases: resnet, resnet_mc, resnet_run, alexnet, vgg, lr_unfused, mlp"""
 import os
 import sys
 
@@ -40,6 +40,15 @@ if __name__ == "__main__":
     elif case == "lr_unfused":    # partials -> reduce -> update kernels (the world > 1 path on one rank)
         os.environ["VISTA_LR_FUSED"] = "0"
         run(0, [1, 2], 40, 8)
+    elif case == "resnet_run":    # vista_run: every layer's LR side by side (cooperative grids on five streams, PDL)
+        tab = gen.make_tables(7, 16, mismatch=True)
+        v = Vista(2, layers=[0, 1, 2, 3, 4], n_str_rows=len(tab.str_keys), d_s=16, n_images_local=7, iters=2,
+                  power_iters=3, split_seed=5, weight_seed=11, micro_batch=7)
+        d = [16 + 0] * 5
+        v.transfer(tab.images, tab.img_keys, tab.X, tab.str_keys, tab.labels)
+        d = [16 + v.features(k)["d_l"] for k in range(5)]
+        v.run(tab.images, tab.img_keys, tab.X, tab.str_keys, tab.labels, d)
+        v.close()
     elif case == "mlp":
         run(0, [2], 40, 8, mlp=True)
     else:

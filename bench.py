@@ -415,6 +415,9 @@ def main():
     breakdown = {k: {"ms": round(p["ms"], 3), "launches": p["launches"],
                      "gbps": (p["bytes"] / (p["ms"] / 1000.0) / 1e9) if p["ms"] > 0 and p["bytes"] else None}
                  for k, p in prof.items() if p["launches"]}
+    if "lr_pass" in breakdown and breakdown["lr_pass"]["launches"] == 1:
+        breakdown["lr_pass"]["note"] = ("vista_run trains every layer side by side (one stream per layer): one record = the "
+                                        "whole LR phase from fork to join; gbps = algorithmic pass bytes / that span")
     # ---- LR results of the last timed step (sanity, identical on all ranks) ----
     accs = [round(r[2]["test_acc"], 2) for r in res]
     cpu = None

@@ -36,7 +36,8 @@ struct LRState {  // device, fp64 master copies
 struct FusedArgs {
   int on;                 // 0: partials only (reduce / allreduce / update kernels follow)
   int ncols;              // ld + 2
-  unsigned int* bar;      // [2] grid barrier: arrival count, generation (zeroed once per lr_train)
+  unsigned int* bar;      // [2] grid barrier: monotonic arrival count (zeroed once per lr_train)
+  unsigned int sync_base; // arrivals before this pass (sum of grid syncs of earlier passes x grid)
   double* G;              // [ncols] reduced sums
   double* scal;           // [2 gridDim.x] per-CTA partial scalars (two reductions per pass at most)
   const uint8_t* real;    // [ld] real (non-padding) columns
@@ -781,20 +782,20 @@ __global__ void __launch_bounds__(2 * kGW * 32 + 32, 1) lr_dot2_kernel(const Pas
 // ---- fused reduce + update (world == 1) ----
 // Grid-wide barrier of the cooperative launch (all CTAs co-resident): compute threads only (the
 // producer warp has exited), named barrier 2 inside the CTA, one arrival per CTA on a global counter.
-__device__ __forceinline__ void grid_sync(unsigned int* bar, int nthr) {
+__device__ __forceinline__ void grid_sync(unsigned int* bar, int nthr, unsigned int target) {
+  // monotonic counter: every CTA adds one with a fire-and-forget release reduction (no round trip, no reset, so
+  // 148 arrivals pipeline in the L2 instead of serialising as returning atomics) and waits for the k-th sync's
+  // total, target = sync_base + k * gridDim.x
   named_bar_sync(2, nthr);
   if (threadIdx.x == 0) {
-    volatile unsigned int* gen = bar + 1;
-    const unsigned int g = *gen;
     __threadfence();
-    if (atomicAdd(bar, 1u) == gridDim.x - 1) {
-      atomicExch(bar, 0u);
-      __threadfence();
-      atomicAdd(bar + 1, 1u);
-    } else {
-      while (*gen == g) __nanosleep(64);
+    asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(bar) : "memory");
+    unsigned int v;
+    while (true) {
+      asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(bar) : "memory");
+      if (v >= target) break;
+      __nanosleep(32);
     }
-    __threadfence();
   }
   named_bar_sync(2, nthr);
 }
@@ -916,7 +917,7 @@ __device__ void fused_tail(const PassArgs& a, uint8_t* scratch, int nthr) {
   double* gs = sh + 32 * 32;                        // this CTA's reduced columns
   double* g2 = gs + ((ld + G - 1) / G + 2);         // G[ld], G[ld + 1]
   __threadfence();
-  grid_sync(f.bar, nthr);  // every CTA's partial row is written
+  grid_sync(f.bar, nthr, f.sync_base + G);  // every CTA's partial row is written
   const int u0 = (int)((int64_t)ld * b / G), u1 = (int)((int64_t)ld * (b + 1) / G);
   reduce_cols(a.partial, pitch, G, u0, u1 - u0, ld, gs, g2, sh, nthr);
   const double phisum = g2[0];
@@ -949,7 +950,7 @@ __device__ void fused_tail(const PassArgs& a, uint8_t* scratch, int nthr) {
     sm = cta_sum(sm, sh, nthr);
     if (threadIdx.x == 0) f.scal[b] = sm;
     __threadfence();
-    grid_sync(f.bar, nthr);
+    grid_sync(f.bar, nthr, f.sync_base + 2 * G);
     const double tot = grid_scalar_sum(f.scal, sh, nthr);
     if (b == 0 && threadIdx.x == 0) {
       st->vb = vb;
@@ -975,7 +976,7 @@ __device__ void fused_tail(const PassArgs& a, uint8_t* scratch, int nthr) {
       f.scal[G + b] = sq;
     }
     __threadfence();
-    grid_sync(f.bar, nthr);
+    grid_sync(f.bar, nthr, f.sync_base + 2 * G);
     const double qb = phisum * rn;
     const double lam = sqrt(grid_scalar_sum(f.scal, sh, nthr) + qb * qb);
     const double sqt = grid_scalar_sum(f.scal + G, sh, nthr);
@@ -1023,7 +1024,7 @@ __device__ void fused_tail(const PassArgs& a, uint8_t* scratch, int nthr) {
   sm = cta_sum(sm, sh, nthr);
   if (threadIdx.x == 0) f.scal[b] = sm;
   __threadfence();
-  grid_sync(f.bar, nthr);  // every CTA has read st->b / st->eta
+  grid_sync(f.bar, nthr, f.sync_base + 2 * G);  // every CTA has read st->b / st->eta
   const double tot = grid_scalar_sum(f.scal, sh, nthr);
   if (b == 0 && threadIdx.x == 0) {
     st->b = bnew;
@@ -1438,7 +1439,10 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   const int ublk = 1024;
   // ---- O6 step 2: standardisation statistics (two passes: mean, then centred squares) ----
   prof_begin(st);
+  unsigned int sync_cum = 0;  // grid-barrier arrivals so far (fused passes: 1 sync in MODE 0, 2 otherwise)
+  a.f.sync_base = sync_cum;
   run_pass<0, E>(a, cfg, st);
+  sync_cum += (unsigned)cfg.grid;
   prof_end(st, 5, 0, pass_bytes);
   if (!fused) {
     reduce((double)n_train, 0);
@@ -1446,7 +1450,9 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
     LAUNCHED();
   }
   prof_begin(st);
+  a.f.sync_base = sync_cum;
   run_pass<1, E>(a, cfg, st);  // fused: + the power-iteration start
+  sync_cum += 2u * (unsigned)cfg.grid;
   prof_end(st, 5, 0, pass_bytes);
   if (!fused) {
     reduce(-1, 0);
@@ -1459,7 +1465,9 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   for (int k = 0; k < power_iters; ++k) {
     a.f.init_next = k == power_iters - 1 ? 1 : 0;  // fused: the last power pass also starts ISTA
     prof_begin(st);
+    a.f.sync_base = sync_cum;
     run_pass<2, E>(a, cfg, st);
+    sync_cum += 2u * (unsigned)cfg.grid;
     prof_end(st, 5, 0, pass_bytes);
     if (!fused) {
       reduce(-1, 1);
@@ -1476,7 +1484,9 @@ static LRResult lr_train_impl(const E* MM, const uint8_t* y, int64_t n_rows, int
   for (int t = 0; t < iters; ++t) {
     a.f.loss_out = loss + t;
     prof_begin(st);
+    a.f.sync_base = sync_cum;
     run_pass<3, E>(a, cfg, st);
+    sync_cum += 2u * (unsigned)cfg.grid;
     prof_end(st, 5, 0, pass_bytes);
     if (!fused) {
       reduce(-1, 1);

@@ -1520,13 +1520,11 @@ static void train_all_batched(vista_ctx* c, double* const* weights_out, vista_me
   int used = 0;
   // VISTA_LR_SHARE="a,b,..." overrides the per-layer weights (measurement of other splits)
   if (const char* e = getenv("VISTA_LR_SHARE")) {
-    tot = 0;
-    for (int k = 0; k < L; ++k) {
-      w[k] = atof(e);
-      tot += w[k];
-      e = strchr(e, ',');
-      if (!e) break;
-      ++e;
+    std::vector<double> ws;
+    for (const char* q = e; q && *q; q = strchr(q, ',') ? strchr(q, ',') + 1 : nullptr) ws.push_back(atof(q));
+    if ((int)ws.size() == L) {  // otherwise the byte shares stand
+      tot = 0;
+      for (int k = 0; k < L; ++k) tot += (w[k] = std::max(ws[k], 0.0));
     }
   }
   for (int k = 0; k < L; ++k) {
@@ -1571,10 +1569,6 @@ static void train_all_batched(vista_ctx* c, double* const* weights_out, vista_me
     c->lr_jobs[k].done = jobs[k].done;
   }
   for (int k = 0; k < L; ++k) VCHECK(cudaStreamWaitEvent(c->stream, jobs[k].done, 0));
-  if (getenv("VISTA_LR_TIMES")) {  // per-layer completion times of the batch (measurement only)
-    VCHECK(cudaStreamSynchronize(c->stream));
-    for (int k = 0; k < L; ++k) fprintf(stderr, "lr layer %d: %d CTAs\n", k, g[k]);
-  }
   g_prof = prof;
   if (prof) {
     double bytes = 0;

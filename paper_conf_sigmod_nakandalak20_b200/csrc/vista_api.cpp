@@ -1513,9 +1513,9 @@ static double lr_bytes(const vista_ctx* c, int k) {
 static void train_all_batched(vista_ctx* c, double* const* weights_out, vista_metrics* out) {
   const int L = (int)c->taps.size();
   const int sms = num_sms();
-  std::vector<double> w(L);
+  std::vector<double> w(L), pass_bytes(L);
   double tot = 0;
-  for (int k = 0; k < L; ++k) tot += (w[k] = lr_bytes(c, k));
+  for (int k = 0; k < L; ++k) tot += (w[k] = pass_bytes[k] = lr_bytes(c, k));
   std::vector<int> g(L);
   int used = 0;
   // VISTA_LR_SHARE="a,b,..." overrides the per-layer weights (measurement of other splits)
@@ -1572,7 +1572,7 @@ static void train_all_batched(vista_ctx* c, double* const* weights_out, vista_me
   g_prof = prof;
   if (prof) {
     double bytes = 0;
-    for (int k = 0; k < L; ++k) bytes += w[k];
+    for (int k = 0; k < L; ++k) bytes += pass_bytes[k];
     char label[96];
     std::snprintf(label, sizeof(label), "LR batched: %d layers side by side", L);
     prof_end(c->stream, 5, 0, bytes, prof_labels() ? label : nullptr);

@@ -1759,8 +1759,9 @@ bool conv_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, const 
   // would spill into the next group's channels
   // (long-K layers keep the register epilogue: it is hidden behind the mainloop and frees the staging
   // smem for a deeper k-block ring)
+  static const int tma_epi_nkb = getenv("VISTA_TMAEPI_NKB") ? atoi(getenv("VISTA_TMAEPI_NKB")) : 12;  // A/B (measured: K = 768 projection unit -0.25 ms with the TMA epilogue, K = 1024 +0.6 ms)
   const bool tma_epi =
-      !halo && (rowview || ((L.groups == 1 || L.Cg_out % L.BN == 0) && L.Cout % 8 == 0 && p.nkb <= 8));
+      !halo && (rowview || ((L.groups == 1 || L.Cg_out % L.BN == 0) && L.Cout % 8 == 0 && p.nkb <= tma_epi_nkb));
   // the fused tap needs the staged tile, non-negative outputs (ReLU) and <= 4 images per 128-row tile
   const bool fuse_tap = tapf && tma_epi && !rowview && L.relu && p.Ho * p.Wo >= 43;
   if (fuse_tap) p.tapf = tapf;
@@ -1918,7 +1919,8 @@ void conv_cat_forward(const ConvLayer& L, int Cx, const bf16* b, const bf16* x, 
   make_tmap(&ta, b, (uint64_t)Kb, (uint64_t)M, BM);
   if (stride != 1) make_tmap_im2col(&tr, x, N, Hx, Wx, Cx, 1, 1, stride, 0, BK, true);
   else make_tmap(&tr, x, (uint64_t)Cx, (uint64_t)M, BM);
-  const bool tma_epi = L.Cout % 8 == 0 && p.nkb <= 8;
+  static const int tma_epi_nkb = getenv("VISTA_TMAEPI_NKB") ? atoi(getenv("VISTA_TMAEPI_NKB")) : 12;  // A/B (measured: K = 768 projection unit -0.25 ms with the TMA epilogue, K = 1024 +0.6 ms)
+  const bool tma_epi = L.Cout % 8 == 0 && p.nkb <= tma_epi_nkb;
   if (tma_epi) make_tmap(&ty, y, (uint64_t)L.Cout, (uint64_t)M, BM);
   else ty = L.tmap_w;  // unused
   const int rkb = (g_wres_enabled && tma_epi && L.BN <= 128 && p.nkb <= 4 && p.n_nt <= num_sms() &&

@@ -515,9 +515,10 @@ void plan_memory(vista_ctx* c, uint64_t budget) {
         B = (int)std::min<int64_t>(c->sys.micro_batch, std::max<int64_t>(CH, 1));
         if ((uint64_t)need(t, B) > budget) return false;
       } else {
-        // larger micro-batches give larger GEMMs per launch (measured: 256 -> 1024 is +7 % img/s);
+        // larger micro-batches give larger GEMMs per launch (measured: 256 -> 1024 is +7 % img/s; ResNet50
+        // 1024 -> 2048 -1.7..-2.5 ms per 20k-image step, 4096 in between; VGG16 2048 is 1.8 % slower than 1024);
         // activations of one micro-batch exceed L2 either way
-        const int64_t cap_B = t == 0 ? 1024 : 16384;
+        const int64_t cap_B = t == 0 ? (c->cnn == VISTA_RESNET50 ? 2048 : 1024) : 16384;
         for (int64_t b = std::min<int64_t>(cap_B, std::max<int64_t>(CH, 1)); b >= 1; b = b > 8 ? b / 2 : b - 1) {
           if ((uint64_t)need(t, b) <= budget) {
             B = (int)b;

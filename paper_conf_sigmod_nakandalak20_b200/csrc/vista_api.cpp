@@ -518,7 +518,8 @@ void plan_memory(vista_ctx* c, uint64_t budget) {
         // larger micro-batches give larger GEMMs per launch (measured: 256 -> 1024 is +7 % img/s; ResNet50
         // 1024 -> 2048 -1.7..-2.5 ms per 20k-image step, 4096 in between; VGG16 2048 is 1.8 % slower than 1024);
         // activations of one micro-batch exceed L2 either way
-        const int64_t cap_B = t == 0 ? (c->cnn == VISTA_RESNET50 ? 2048 : 1024) : 16384;
+        static const int64_t cap1 = getenv("VISTA_MB_CAP1") ? atoll(getenv("VISTA_MB_CAP1")) : 16384;  // A/B
+        const int64_t cap_B = t == 0 ? (c->cnn == VISTA_RESNET50 ? 2048 : 1024) : cap1;
         for (int64_t b = std::min<int64_t>(cap_B, std::max<int64_t>(CH, 1)); b >= 1; b = b > 8 ? b / 2 : b - 1) {
           if ((uint64_t)need(t, b) <= budget) {
             B = (int)b;

@@ -389,10 +389,16 @@ def main():
         hbm_peak, hbm_src = 7700.0, "fallback B200_PROFILING.md nominal 7.7 TB/s"
     v.set_profiling(True)
     v.set_roofline(tensor_peak, hbm_peak)
-    v.profile(reset=True)
-    step()
-    prof = v.profile(reset=True)
+    # three instrumented steps, the one with the median conv-class time reported (one step's per-class sums move by
+    # ~2 % with the power-capped clock)
+    profs = []
+    for _ in range(1 if os.environ.get("VISTA_PROF_LOG") else 3):  # (a per-launch log holds exactly one step)
+        v.profile(reset=True)
+        step()
+        profs.append(v.profile(reset=True))
     v.set_profiling(False)
+    profs.sort(key=lambda q: q["conv_fc_tcgen05"]["ms"])
+    prof = profs[len(profs) // 2]
     conv = prof["conv_fc_tcgen05"]
     achieved = conv["flops"] / (conv["ms"] / 1000.0) / 1e12 if conv["ms"] > 0 else None
     total_prof_ms = sum(p["ms"] for p in prof.values())
@@ -447,7 +453,9 @@ def main():
             "cpu_baseline": cpu,
             "e2e": {"value": N_global / (e2e_step / 1000.0), "unit": "images/s", "ms_per_step": e2e_step,
                     "h2d_bytes_per_step": h2d_bytes, "d2h_bytes_per_step": d2h,
-                    "note": "vista_transfer with pinned host inputs + vista_train weights to host"},
+                    "note": ("vista_run with pinned host inputs (H2D per stage-1 micro-batch inside the step), every "
+                             "layer's trained weights and metrics read back" if args.api == "run" else
+                             "vista_transfer with pinned host inputs + vista_train weights to host")},
             "gpu_launches": launches,
             "cuda_graph": graph_info,
             "clocks": clocks,

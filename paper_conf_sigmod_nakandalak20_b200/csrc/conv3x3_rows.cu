@@ -19,8 +19,8 @@
 // and image edges); slots are zeroed by the epilogue after draining, so every MMA accumulates.  Per output
 // row the products are accumulated in the same order as the halo kernel's (filter row r, then s, then
 // channel), so the two kernels agree bit for bit.
-// Work item = (image pair, band of output rows); 2 bands of H / 2 rows recompute 2 input rows per pair so
-// that ~2 x N / 2 items balance over the persistent grid.
+// Work item = (image pair, band of output rows): one band, or two bands of H / 2 rows (2 recomputed input rows
+// per pair) when the finer items balance the persistent grid better.
 //
 // Warps: 0 = TMA producer (weights once, then input rows through a kSA-slot ring), 1 = TMEM allocator + MMA
 // issuer (one elected lane), 2..9 = epilogue: two groups of four warps (one per TMEM lane quadrant) take
@@ -244,9 +244,16 @@ void rowconv3x3_forward(const ConvLayer& L, const bf16* x, int N, int H, int W, 
   p.H = H;
   p.W = W;
   p.relu = L.relu ? 1 : 0;
-  p.nbands = H >= 8 ? 2 : 1;
+  // one band per image pair unless two bands balance the persistent grid better: a band boundary recomputes two
+  // input rows (H / (H + 2) of the MMA work is useful), a partial last round of items idles CTAs
+  const int pairs = (N + 1) / 2, sms = num_sms();
+  auto eff = [&](int nb) {
+    const int items = pairs * nb, rounds = (items + sms - 1) / sms;
+    return (double)items / ((double)rounds * sms) * (nb == 1 ? 1.0 : (double)H / (H + 2));
+  };
+  p.nbands = (H >= 8 && eff(2) > eff(1)) ? 2 : 1;
   p.band_h = (H + p.nbands - 1) / p.nbands;
-  p.n_items = ((N + 1) / 2) * p.nbands;
+  p.n_items = pairs * p.nbands;
   ensure_smem_attr((const void*)conv3x3_rows_kernel, kSmem);
   const int grid = p.n_items < num_sms() ? p.n_items : num_sms();
   prof_begin(st);

@@ -220,13 +220,13 @@ vista_status vista_train(vista_ctx* ctx, int32_t k, double* weights_out, vista_m
  * in one call = vista_transfer + vista_train(k) for every layer k (S6 of SURVEY.md §8a).
  * Arguments as vista_transfer; weights_out: NULL or n_layers caller-owned pointers, each NULL or a
  * double[d_s + d_l(k) + 1] as vista_train's; out: NULL or vista_metrics[n_layers].
- * Schedule: one rank (bf16, more than one layer): after the transfer, the M of every layer side by side, each
- * layer's passes on its own stream with a share of the SMs proportional to its bytes; the same algorithm over
- * fewer CTAs per layer, so the results equal vista_train(k)'s up to the fp32 grouping of the per-CTA partial
- * sums (weights within 2e-4 normwise in the tests).  VISTA_LR_BATCH=0: M of layer k on a second stream as soon
- * as MM_k exists, beside the partial inference of stage k+1 (or, with VISTA_OVERLAP=0, after the transfer,
- * layer by layer) -- then bit-identical to vista_transfer followed by vista_train(k).  world > 1 and the fp32
- * check mode train after the transfer, layer by layer.  Collective like vista_train. */
+ * Schedule: M of layer k on a second stream as soon as MM_k exists, beside the partial inference of stage k+1
+ * (VISTA_OVERLAP=0: after the transfer, layer by layer); results bit-identical to vista_transfer followed by
+ * vista_train(k) for k = 0 .. n_layers-1.  VISTA_LR_BATCH=1 (one rank, bf16): the M of every layer side by side
+ * after the transfer, each layer's passes on its own stream with a share of the SMs proportional to its bytes
+ * (the same algorithm over fewer CTAs per layer: equal up to the fp32 grouping of the per-CTA partial sums,
+ * weights within 2e-4 normwise in the tests).  world > 1 and the fp32 check mode train after the transfer,
+ * layer by layer.  Collective like vista_train. */
 vista_status vista_run(vista_ctx* ctx, const uint8_t* images, const int64_t* image_keys, const float* structured,
                        const int64_t* str_keys, const uint8_t* labels, double* const* weights_out,
                        vista_metrics* out);

@@ -369,8 +369,8 @@ class Vista:
         return w[:-1], float(w[-1]), met
 
     def run(self, images, image_keys, structured, str_keys, labels, d_totals, want_weights=True):
-        """vista_run: transfer + M of every layer (side by side after the transfer; VISTA_LR_BATCH=0: M(k) beside
-        stage k+1); returns [(w, b, metrics)] per layer."""
+        """vista_run: transfer + M of every layer (M(k) beside stage k+1; VISTA_LR_BATCH=1: side by side after the
+        transfer); returns [(w, b, metrics)] per layer."""
         L = len(d_totals)
         ws = [np.zeros(d + 1, dtype=np.float64) for d in d_totals] if want_weights else None
         ptrs = (ctypes.c_void_p * L)(*[w.ctypes.data for w in ws]) if want_weights else None

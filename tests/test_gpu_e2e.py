@@ -462,12 +462,13 @@ def test_run_equals_transfer_then_train(monkeypatch, overlap):
     v.close()
 
 
-def test_run_batched_lr_matches_per_layer_training():
-    # vista_run's default one-rank schedule trains all layers side by side (each layer's passes on its own stream
+def test_run_batched_lr_matches_per_layer_training(monkeypatch):
+    # vista_run's side-by-side schedule (VISTA_LR_BATCH=1, one rank) trains all layers side by side (each layer's passes on its own stream
     # with a share of the SMs): the same algorithm over fewer CTAs per layer, so only the fp32 summation grouping
     # of the per-CTA partial sums differs from vista_train(k).  Measured: weights 4.6e-5 normwise after 3 ISTA
     # steps (the soft threshold amplifies last-bit differences near zero); bound 2e-4, 5x below the oracle parity
     # tolerance of 1e-3 (reading R22)
+    monkeypatch.setenv("VISTA_LR_BATCH", "1")
     tab = gen.make_tables(300, 16)
     taps = [0, 1, 2, 3, 4]
     ref = run_gpu(2, taps, tab, 16, iters=3)

@@ -817,8 +817,8 @@ bool run_ops(vista_ctx* c, int t, const void* in_ptr, void* out_ptr, int nb, voi
 // Host pixels of images [c0, c0 + nc) -> c->d_px, one stage-1 micro-batch per copy on c->copy_stream, each
 // followed by c->px_ready[j]; the compute stream waits on event j right before micro-batch j, so the copy of
 // micro-batch j + 1 overlaps the inference of micro-batch j.  Returns the events.
-// split_first (Staged stage 1): the first micro-batch is copied -- and then inferred -- as three segments of
-// B/4, B/4 and B/2 images, so stage 1 starts after a quarter of the first copy instead of all of it
+// split_first (Staged stage 1): the first micro-batch is copied -- and then inferred -- in doubling segments
+// (B/4, B/4, B/2; B/8, B/8, B/4, B/2 at B >= 2048), so stage 1 starts after ~256 images of the first copy
 const std::vector<cudaEvent_t>* stream_host_pixels(vista_ctx* c, const uint8_t* images, int64_t c0, int64_t nc,
                                                    bool split_first = false) {
   const size_t px_img = (size_t)c->net.stages[0].in_elems;
@@ -833,7 +833,9 @@ const std::vector<cudaEvent_t>* stream_host_pixels(vista_ctx* c, const uint8_t* 
   const int64_t B0 = std::max(c->micro[0], 1);
   c->px_bounds.clear();
   if (split_first && B0 >= 8) {
-    for (int64_t b : {(int64_t)0, B0 / 4, B0 / 2})
+    // segments doubling from ~256 images (B/4 for B <= 1024; B/8 at 2048): only the first segment's copy is exposed
+    const int64_t s0 = B0 >= 2048 ? B0 / 8 : B0 / 4;
+    for (int64_t b = 0; b < B0; b = b ? 2 * b : s0)
       if (b < nc) c->px_bounds.push_back(b);
   }
   for (int64_t i0 = c->px_bounds.empty() ? 0 : B0; i0 < nc; i0 += B0) c->px_bounds.push_back(i0);
